@@ -1,0 +1,251 @@
+/*
+ * mp.h — C ABI of mpx, a B200-native implementation of the multi-path intra-node
+ * GPU→GPU transfer of Sojoodi et al., "Accelerating Intra-Node GPU Communication:
+ * A Performance Model for Multi-Path Transfers" (SC-W '25).  P:<line> cites
+ * /root/reference/PAPER.md; C<n> cites the readings table in DESIGN.md §3.
+ *
+ * One message of n bytes from a source GPU to a destination GPU is split over
+ * several intra-node paths at once: the direct NVLink/NVSwitch path,
+ * two-hop relays staged through intermediate GPUs, and a pinned-host PCIe path.
+ * The split θ and the per-path chunk counts k come from the paper's
+ * extended-Hockney model (Eq 1-24) through Algorithm 1; the bytes are moved
+ * by hand-written sm_100a kernels (SM-driven 128-bit stores into peer / pinned-host
+ * memory, flag release/acquire handoff between pipeline stages).
+ *
+ * Conventions for every function below
+ *   - returns an int status: MP_OK (0) or a negative MP_ERR_*; never aborts, never
+ *     throws.  mp_strerror(status) names the code; mp_last_error(ctx) gives the last
+ *     message recorded on ctx (library-owned string, valid until the next call).
+ *   - pointers: "host" = CPU memory, "device" = CUDA device memory of the calling
+ *     rank's GPU.  Buffers passed in are owned by the caller; the library keeps no
+ *     reference after the call returns unless stated (stream-ordered work keeps
+ *     using a buffer until that work completes on its stream).
+ *   - units (C11): bytes, seconds, bytes/second.
+ *   - a `stream` argument is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  Work is enqueued; completion is stream-ordered.
+ *   - thread safety: a context may be used by one host thread at a time.
+ */
+#ifndef MPX_MP_H
+#define MPX_MP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MP_ABI_VERSION 1
+#define MP_MAX_PATHS 16
+
+/* Status codes. */
+enum {
+  MP_OK = 0,
+  MP_ERR_INVALID = -1,     /* bad argument (NULL, size mismatch, Σ shares != n, k out of range) */
+  MP_ERR_CUDA = -2,        /* a CUDA runtime call failed (message in mp_last_error) */
+  MP_ERR_TOPOLOGY = -3,    /* unknown rank / path not available between src and dst */
+  MP_ERR_NOMEM = -4,       /* heap, ring or host allocation failed */
+  MP_ERR_STATE = -5,       /* call not valid in this context state (e.g. model-only ctx) */
+  MP_ERR_UNSUPPORTED = -6, /* feature not built / not supported on this system */
+  MP_ERR_TIMEOUT = -7,     /* a device-side wait exceeded the timeout (sticky) */
+  MP_ERR_MISMATCH = -8     /* send/recv size or tag mismatch detected on the device (sticky) */
+};
+
+/* Path kinds, P:107-111 (§3.1). */
+enum { MP_PATH_DIRECT = 0, MP_PATH_GPU = 1, MP_PATH_HOST = 2 };
+
+/* Model modes (C3, C8, C14, C18).
+ * PAPER: Eq 13 with the printed case rule, stagger σ_j = α_j, no shared port.
+ * B200 : exact two-stage pipeline time, calibrated stagger σ, one shared port
+ *        (NVSwitch egress/ingress, or HBM in single-GPU loopback), integer-k pass 3. */
+enum { MP_MODEL_PAPER = 0, MP_MODEL_B200 = 1 };
+
+/* Init flags. */
+enum {
+  MP_INIT_MODEL_ONLY = 1,  /* no CUDA at all: model evaluator + selector only (CPU tests) */
+  MP_INIT_NO_CALIBRATE = 2 /* do not measure α/β at init (use defaults / param file / mp_set_model) */
+};
+
+typedef struct mp_ctx mp_ctx;  /* opaque, library-owned */
+
+/* One path between a (src, dst) pair.  via = relay rank for MP_PATH_GPU (in
+ * single-GPU loopback: the index of an emulated relay ring), -1 otherwise. */
+typedef struct mp_path {
+  int32_t kind;
+  int32_t via;
+} mp_path;
+
+/* Per-path model parameters — Table 1.  For a direct path only alpha,
+ * beta (and sigma, w) are used (Eq 6: α' = ε = 0, 1/β' = 0). */
+typedef struct mp_path_params {
+  double alpha;   /* α_i  first-link startup latency [s] */
+  double beta;    /* β_i  first-link bandwidth [B/s] */
+  double alpha2;  /* α'_i second-link startup latency [s] (staged) */
+  double beta2;   /* β'_i second-link bandwidth [B/s] (staged) */
+  double eps;     /* ε_i  synchronisation overhead at the staging device [s] */
+  double c;       /* multiplier of the topology constant φ_i (C4; 1 = Eq 14/15 at θ⁽⁰⁾) */
+  double sigma;   /* issue latency counted by the stagger in B200 mode (C8) [s] */
+  double w;       /* bytes of shared-port traffic per payload byte (C14) */
+} mp_path_params;
+
+/* The shared port of B200 mode (C14): T >= alpha + Σ_i w_i b_i / beta.
+ * beta <= 0 or +inf disables it. */
+typedef struct mp_port_params {
+  double alpha;
+  double beta;
+} mp_port_params;
+
+/* Selector options (readings C5, C7, C8, C18). */
+typedef struct mp_model_opts {
+  int32_t mode;        /* MP_MODEL_PAPER | MP_MODEL_B200 */
+  int32_t stagger;     /* 1: Alg 1 line 17 issue stagger; 0: off */
+  int32_t refine;      /* pass 3 (C18): 1 on, 0 off, -1 = mode default (B200 on) */
+  int32_t reserved;
+  uint64_t align;      /* A: share alignment and chunk unit, >= 1 (default 256) */
+  uint64_t c_min;      /* smallest staged share and chunk (default 65536) */
+  uint64_t k_max;      /* chunk-count cap (default 1024) */
+  uint64_t slot_bytes; /* largest chunk a staging slot holds (0 = unlimited) */
+} mp_model_opts;
+
+/* Algorithm 1 output: shares[] and configs[] per path.  Caller-allocated.
+ * bytes[] is authoritative and sums to n; theta[] is informational. */
+typedef struct mp_config {
+  int32_t npaths;
+  int32_t reserved;
+  mp_path path[MP_MAX_PATHS];
+  double theta[MP_MAX_PATHS];
+  uint64_t bytes[MP_MAX_PATHS];
+  uint32_t chunks[MP_MAX_PATHS]; /* k_i >= 1 when bytes[i] > 0, else 0; direct k = 1 */
+  double t_pred;                 /* O2 model time of this config [s] */
+  double t_level;                /* linearised common finish time of the last level solve [s] */
+} mp_config;
+
+/* Bootstrap all-gather: every rank contributes `bytes` bytes at `in`; on return
+ * `out` holds world*bytes bytes, rank-major.  Return 0 on success.  The library
+ * calls it only inside mp_init/mp_finalize (collective calls). */
+typedef int (*mp_allgather_fn)(void *user, const void *in, void *out, uint64_t bytes);
+
+typedef struct mp_init_args {
+  int32_t rank;          /* this process's rank, 0..world-1 */
+  int32_t world;         /* number of ranks (one GPU each); 1 = single-GPU loopback */
+  int32_t device;        /* local CUDA device ordinal */
+  int32_t flags;         /* MP_INIT_* */
+  int32_t n_loop_relays; /* loopback only: emulated relay rings (default 6 if < 0) */
+  int32_t host_path;     /* 1: enable the pinned-host PCIe path (default 1 if < 0) */
+  int32_t slots;         /* staging slots per ring (default 4 if <= 0) */
+  int32_t relay_ctas;    /* CTAs per staged-path stage (default 16 if <= 0, max 32) */
+  uint64_t heap_bytes;   /* symmetric receive heap per rank (default 2.25 GiB if 0) */
+  uint64_t slot_bytes;   /* bytes per staging slot (default 32 MiB if 0) */
+  double timeout_s;      /* device wait timeout (default 20 s if <= 0) */
+  mp_allgather_fn allgather; /* required when world > 1 */
+  void *allgather_user;
+  const char *param_file;    /* optional: load model parameters (Step 2) */
+} mp_init_args;
+
+/* ---------------------------------------------------------------- lifetime */
+
+/* Create a context.  Collective over all ranks when world > 1.  Discovers the
+ * topology (peer access, PCIe host path), allocates the heap, relay rings and the
+ * pinned host ring, exchanges IPC handles, and — unless MP_INIT_NO_CALIBRATE —
+ * calibrates α/β/ε of every path with the engine's own kernels (Step 1).
+ * With MP_INIT_MODEL_ONLY no CUDA call is made; world/rank still define the pairs.
+ * Errors: MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_NOMEM, MP_ERR_TOPOLOGY. */
+int mp_init(mp_ctx **ctx, const mp_init_args *args);
+
+/* Destroy a context: waits for outstanding work, stops relay kernels, unmaps and
+ * frees everything.  Collective when world > 1.  ctx may be NULL. */
+int mp_finalize(mp_ctx *ctx);
+
+const char *mp_strerror(int status);
+const char *mp_last_error(mp_ctx *ctx);
+int mp_abi_version(void);
+
+/* ---------------------------------------------------------------- model (host, fp64) */
+
+/* The default path list for (src, dst) in the order of reading A1: direct, GPU
+ * relays by ascending rank (or loopback ring index), host.  out: MP_MAX_PATHS entries. */
+int mp_paths(mp_ctx *ctx, int src, int dst, mp_path *out, int *npaths);
+
+/* Install model parameters for the ordered pair (src, dst) (tests / parity /
+ * Step 2 injection).  paths[i] and params[i] describe path i; paths[0] must be
+ * MP_PATH_DIRECT.  port may be NULL (no shared port).  Invalidates the config
+ * cache.  Errors: MP_ERR_INVALID (npaths out of range, β <= 0, staged α <= 0 with
+ * β < β', staged ε + α' <= 0, ...). */
+int mp_set_model(mp_ctx *ctx, int src, int dst, const mp_path *paths,
+                 const mp_path_params *params, int npaths, const mp_port_params *port);
+int mp_get_model(mp_ctx *ctx, int src, int dst, mp_path *paths, mp_path_params *params,
+                 int *npaths, mp_port_params *port);
+
+/* Selector options for this context (invalidates the cache). */
+int mp_set_options(mp_ctx *ctx, const mp_model_opts *opts);
+int mp_get_options(mp_ctx *ctx, mp_model_opts *opts);
+
+/* mp_predict — O2: modelled time of moving `bytes` from src to dst with
+ * config `cfg` (Eq 6 direct, Eq 13 staged, + stagger, T = max_i T_i (Eq 4); B200
+ * mode: exact pipeline and the shared port).  cfg->bytes must sum to `bytes`.
+ * *seconds receives the time.  Host-only; no CUDA. */
+int mp_predict(mp_ctx *ctx, int src, int dst, uint64_t bytes, const mp_config *cfg,
+               double *seconds);
+
+/* mp_select — Algorithm 1 without exhaustive search, reading O3: θ from
+ * Eq 11 then Eq 24 with the two-pass φ (C4) and the active set (C2), k from Eq 19
+ * (C5), shares floored to A with the leftover to the direct path (C7), optional
+ * pass 3 (C18).  path_mask bit i enables path i of mp_paths() (bit 0, the direct
+ * path, is always on; 0 = all paths).  Results are cached (C10).  Host-only. */
+int mp_select(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t path_mask,
+              mp_config *out);
+
+/* ---------------------------------------------------------------- memory */
+
+/* Allocate / free device memory from this rank's registered heap.  A buffer that
+ * receives (mp_recv) must come from here when world > 1 (peers address it by heap
+ * offset, the analogue of UCX cuda_ipc's cached IPC mappings).  256-B aligned. */
+int mp_alloc(mp_ctx *ctx, uint64_t bytes, void **dptr);
+int mp_free(mp_ctx *ctx, void *dptr);
+
+/* ---------------------------------------------------------------- transfer */
+
+/* Send `bytes` bytes at device pointer `buf` to rank dst with `tag`.  cfg = NULL
+ * selects with mp_select(all paths); otherwise cfg->bytes/chunks/path are used as
+ * given (validated: Σ bytes == n, 1 <= k <= max(1, ⌊b/A⌋), chunk <= slot_bytes,
+ * paths available).  Stream-ordered: the send kernel waits on the device for the
+ * matching mp_recv.  In single-GPU loopback (dst == rank == 0) the send is
+ * recorded and the fused transfer is launched by the matching mp_recv. */
+int mp_send(mp_ctx *ctx, const void *buf, uint64_t bytes, int dst, int tag,
+            const mp_config *cfg, void *stream);
+
+/* Receive `bytes` bytes from rank src with `tag` into device pointer `buf`
+ * (heap memory when world > 1).  Matching is FIFO per (src, dst); the tag and the
+ * size must equal the sender's or the device raises MP_ERR_MISMATCH.  Work after
+ * mp_recv on `stream` sees the whole message. */
+int mp_recv(mp_ctx *ctx, void *buf, uint64_t bytes, int src, int tag, void *stream);
+
+/* Single-process transfer src → dst on this GPU through every selected path
+ * (loopback engine; the relay rings and the host ring stand in for the
+ * intermediate GPUs and the host).  One fused kernel launch on `stream`.
+ * cfg = NULL selects.  Used by calibration, the sweep and the benchmark. */
+int mp_xfer(mp_ctx *ctx, void *dst, const void *src, uint64_t bytes, const mp_config *cfg,
+            void *stream);
+
+/* Block until all work this context enqueued has finished, then report any
+ * sticky device error (MP_ERR_TIMEOUT / MP_ERR_MISMATCH). */
+int mp_sync(mp_ctx *ctx);
+
+/* ---------------------------------------------------------------- calibration */
+
+/* Step 1: measure α, β (per link) and ε (per staging device) with the
+ * engine's own kernels on this GPU, fit (C12) and install them for (0, 0)
+ * loopback, plus the shared port.  sizes: byte counts to sweep (NULL = default),
+ * reps: repeats per size (median).  Requires world == 1. */
+int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
+
+/* Save / load the model parameters of every pair (Step 1/2). */
+int mp_save_params(mp_ctx *ctx, const char *path);
+int mp_load_params(mp_ctx *ctx, const char *path);
+
+/* Launch statistics: number of engine kernels launched by this context so far. */
+int mp_stats(mp_ctx *ctx, uint64_t *kernel_launches);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MPX_MP_H */

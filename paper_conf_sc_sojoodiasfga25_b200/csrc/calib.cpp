@@ -1,0 +1,211 @@
+// calib.cpp — Step 1 of PAPER.md §4: extract the model parameters of every
+// path once per topology, with the engine's own kernels (reading C12).
+//
+// Single-GPU loopback: the "links" are
+//   direct        src HBM  → dst HBM
+//   relay leg 1   src      → relay ring      leg 2  relay ring → dst
+//   host leg 1    src      → pinned host ring (PCIe writes)   leg 2  host ring → dst (PCIe reads)
+// Each link is timed with a direct-only fused launch between the two buffers
+// (median of `reps` CUDA-event timings per size, L2 flushed before each), and
+// T(n) = α + n/β is fitted by least squares weighted by 1/T² over the sizes.
+// ε of a staging device is half the round trip of a flag ping-pong between two CTAs
+// through that device's flag memory (the same release/acquire the pipeline uses).
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "ctx.h"
+
+using namespace mpx;
+
+namespace {
+
+int cfail(mp_ctx *c, int code, const std::string &msg) {
+  c->last_error = msg;
+  return code;
+}
+
+#define CKC(call)                                                                          \
+  do {                                                                                     \
+    cudaError_t e__ = (call);                                                              \
+    if (e__ != cudaSuccess) return cfail(c, MP_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e__)); \
+  } while (0)
+
+struct Fit {
+  double alpha, beta;
+};
+
+// Weighted least squares of T = α + n·g (g = 1/β), weights 1/T² (relative error).
+Fit fit_hockney(const std::vector<double> &n, const std::vector<double> &t) {
+  double s00 = 0, s01 = 0, s11 = 0, r0 = 0, r1 = 0;
+  for (size_t i = 0; i < n.size(); ++i) {
+    const double w = 1.0 / (t[i] * t[i]);
+    s00 += w;
+    s01 += w * n[i];
+    s11 += w * n[i] * n[i];
+    r0 += w * t[i];
+    r1 += w * n[i] * t[i];
+  }
+  const double det = s00 * s11 - s01 * s01;
+  double a = (r0 * s11 - r1 * s01) / det;
+  double g = (s00 * r1 - s01 * r0) / det;
+  if (!(g > 0)) g = t.back() / n.back();
+  if (!(a > 1e-7)) a = 1e-7;  // Eq 14 needs α > 0
+  return Fit{a, 1.0 / g};
+}
+
+double median(std::vector<double> v) {
+  std::sort(v.begin(), v.end());
+  return v[v.size() / 2];
+}
+
+struct Bench {
+  mp_ctx *c;
+  cudaStream_t s = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  void *flush = nullptr;
+  uint64_t flush_bytes = 256ull << 20;
+};
+
+// One direct-only fused launch dst ← src of n bytes; returns seconds.
+int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double *out) {
+  mp_ctx *c = b.c;
+  mp_config cfg;
+  std::memset(&cfg, 0, sizeof(cfg));
+  mp_path paths[MP_MAX_PATHS];
+  int np = 0;
+  if (int st = mp_paths(c, 0, 0, paths, &np)) return st;
+  cfg.npaths = np;
+  for (int i = 0; i < np; ++i) cfg.path[i] = paths[i];
+  cfg.bytes[0] = n;
+  cfg.chunks[0] = 1;
+  std::vector<double> ts;
+  for (int r = 0; r < reps + 1; ++r) {
+    CKC(cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s));
+    CKC(cudaEventRecord(b.e0, b.s));
+    if (int st = mp_xfer(c, dst, src, n, &cfg, b.s)) return st;
+    CKC(cudaEventRecord(b.e1, b.s));
+    CKC(cudaEventSynchronize(b.e1));
+    float ms = 0;
+    CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
+    if (r > 0) ts.push_back(ms * 1e-3);  // first launch is a warm-up
+  }
+  *out = median(ts);
+  return MP_OK;
+}
+
+int fit_link(Bench &b, void *dst, const void *src, const std::vector<uint64_t> &sizes, uint64_t cap,
+             int reps, Fit *f) {
+  std::vector<double> n, t;
+  for (uint64_t s : sizes) {
+    if (s > cap) continue;
+    double sec = 0;
+    if (int st = time_copy(b, dst, src, s, reps, &sec)) return st;
+    n.push_back(static_cast<double>(s));
+    t.push_back(sec);
+  }
+  if (n.size() < 2) return cfail(b.c, MP_ERR_INVALID, "calibration needs at least two sizes");
+  *f = fit_hockney(n, t);
+  return MP_OK;
+}
+
+int time_pingpong(Bench &b, uint64_t *flags, bool host, int iters, double *eps) {
+  mp_ctx *c = b.c;
+  if (host)
+    std::memset(flags, 0, 16);
+  else
+    CKC(cudaMemsetAsync(flags, 0, 16, b.s));
+  CKC(cudaEventRecord(b.e0, b.s));
+  int e = launch_pingpong(flags, iters, static_cast<uint64_t>(c->timeout_s * 1e9), c->d_err, b.s);
+  if (e) return cfail(c, MP_ERR_CUDA, "pingpong launch");
+  c->launches += 1;
+  CKC(cudaEventRecord(b.e1, b.s));
+  CKC(cudaEventSynchronize(b.e1));
+  float ms = 0;
+  CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
+  *eps = ms * 1e-3 / (2.0 * iters);
+  return MP_OK;
+}
+
+}  // namespace
+
+extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int reps) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (c->world != 1) return cfail(c, MP_ERR_UNSUPPORTED, "calibration runs on the loopback engine");
+  if (reps <= 0) reps = 5;
+  std::vector<uint64_t> sizes;
+  if (sizes_in && nsizes > 0)
+    sizes.assign(sizes_in, sizes_in + nsizes);
+  else
+    for (uint64_t s = 1ull << 20; s <= (256ull << 20); s <<= 1) sizes.push_back(s);
+  const uint64_t big = *std::max_element(sizes.begin(), sizes.end());
+
+  Bench b;
+  b.c = c;
+  CKC(cudaSetDevice(c->device));
+  CKC(cudaStreamCreateWithFlags(&b.s, cudaStreamNonBlocking));
+  CKC(cudaEventCreate(&b.e0));
+  CKC(cudaEventCreate(&b.e1));
+  void *src = nullptr, *dst = nullptr;
+  CKC(cudaMalloc(&b.flush, b.flush_bytes));
+  CKC(cudaMalloc(&src, big));
+  CKC(cudaMalloc(&dst, big));
+  CKC(cudaMemset(src, 0x5a, big));
+
+  int st = MP_OK;
+  Fit fd{}, f1{}, f2{}, fh1{}, fh2{};
+  double eps_dev = 0, eps_host = 0;
+  const uint64_t ring_cap = static_cast<uint64_t>(c->slots) * c->slot_bytes;
+  do {
+    if ((st = fit_link(b, dst, src, sizes, big, reps, &fd))) break;
+    if (c->n_loop_relays > 0) {
+      uint8_t *ring = c->rings[0].data;
+      if ((st = fit_link(b, ring, src, sizes, ring_cap, reps, &f1))) break;
+      if ((st = fit_link(b, dst, ring, sizes, ring_cap, reps, &f2))) break;
+      if ((st = time_pingpong(b, c->d_probe, false, 2000, &eps_dev))) break;
+    }
+    if (c->host_path) {
+      uint8_t *hr = c->rings[c->n_loop_relays].data;
+      std::vector<uint64_t> hs;
+      for (uint64_t s : sizes)
+        if (s <= std::min<uint64_t>(ring_cap, 64ull << 20)) hs.push_back(s);
+      if ((st = fit_link(b, hr, src, hs, ring_cap, std::max(3, reps / 2), &fh1))) break;
+      if ((st = fit_link(b, dst, hr, hs, ring_cap, std::max(3, reps / 2), &fh2))) break;
+      if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) break;
+    }
+  } while (false);
+
+  cudaStreamSynchronize(b.s);
+  cudaFree(src);
+  cudaFree(dst);
+  cudaFree(b.flush);
+  cudaEventDestroy(b.e0);
+  cudaEventDestroy(b.e1);
+  cudaStreamDestroy(b.s);
+  if (st) return st;
+  int32_t derr = 0;
+  CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
+  if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration probe timed out");
+
+  // Install the loopback pair (0, 0): paths in A1 order.  Shared port = HBM:
+  // a direct byte costs a read + a write (w = 2), a relay byte 4 (slot write + read
+  // on top), a host byte 2 (src read, dst write; the slot is in host DRAM).
+  mp_path paths[MP_MAX_PATHS];
+  mp_path_params prm[MP_MAX_PATHS];
+  int np = 0;
+  paths[np] = mp_path{MP_PATH_DIRECT, -1};
+  prm[np++] = mp_path_params{fd.alpha, fd.beta, 0, 0, 0, 1, 0, 2};
+  for (int r = 0; r < c->n_loop_relays; ++r) {
+    paths[np] = mp_path{MP_PATH_GPU, r};
+    prm[np++] = mp_path_params{f1.alpha, f1.beta, f2.alpha, f2.beta, std::max(eps_dev, 1e-8), 1, 0, 4};
+  }
+  if (c->host_path) {
+    paths[np] = mp_path{MP_PATH_HOST, -1};
+    prm[np++] = mp_path_params{fh1.alpha, fh1.beta, fh2.alpha, fh2.beta, std::max(eps_host, 1e-8), 1, 0, 2};
+  }
+  mp_port_params port{fd.alpha, 2.0 * fd.beta};
+  return mp_set_model(c, 0, 0, paths, prm, np, &port);
+}

@@ -1,0 +1,693 @@
+// capi.cpp — the C ABI of include/mp.h: context lifetime, model calls, heap,
+// loopback transfer launcher.  PAPER.md §4 (Steps 1-5; Alg 1).
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <limits>
+#include <new>
+#include <string>
+
+#include "ctx.h"
+
+using namespace mpx;
+
+namespace {
+
+int fail(mp_ctx *c, int code, const std::string &msg) {
+  if (c) c->last_error = msg;
+  return code;
+}
+
+int cuda_fail(mp_ctx *c, cudaError_t e, const char *what) {
+  return fail(c, MP_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(call)                                        \
+  do {                                                  \
+    cudaError_t e__ = (call);                           \
+    if (e__ != cudaSuccess) return cuda_fail(c, e__, #call); \
+  } while (0)
+
+// Default model parameters before calibration (B200-like guesses, not from the
+// paper; replaced by mp_calibrate / mp_load_params / mp_set_model).
+PathModel default_path(int kind, int via, bool loopback) {
+  PathModel p;
+  p.kind = kind;
+  p.via = via;
+  p.c = 1.0;
+  if (kind == K_DIRECT) {
+    p.alpha = 4e-6;
+    p.beta = loopback ? 3.0e12 : 7.5e11;
+    p.w = loopback ? 2.0 : 1.0;
+  } else if (kind == K_GPU) {
+    p.alpha = 4e-6;
+    p.beta = loopback ? 3.0e12 : 7.5e11;
+    p.alpha2 = 1e-6;
+    p.beta2 = loopback ? 3.0e12 : 7.5e11;
+    p.eps = 2e-6;
+    p.w = loopback ? 4.0 : 1.0;
+  } else {
+    p.alpha = 5e-6;
+    p.beta = 5.0e10;
+    p.alpha2 = 2e-6;
+    p.beta2 = 5.0e10;
+    p.eps = 3e-6;
+    p.w = loopback ? 2.0 : 0.0;
+  }
+  return p;
+}
+
+// Reading A1: direct, GPU relays by ascending rank (loopback: ring index), host.
+PairModel default_pair(const mp_ctx *c, int src, int dst) {
+  PairModel m;
+  const bool loop = (src == dst);
+  m.paths.push_back(default_path(K_DIRECT, -1, loop));
+  if (loop) {
+    for (int r = 0; r < c->n_loop_relays; ++r) m.paths.push_back(default_path(K_GPU, r, true));
+  } else {
+    for (int r = 0; r < c->world; ++r)
+      if (r != src && r != dst) m.paths.push_back(default_path(K_GPU, r, false));
+  }
+  if (c->host_path) m.paths.push_back(default_path(K_HOST, -1, loop));
+  m.port_alpha = 4e-6;
+  m.port_beta = loop ? 6.5e12 : 9.0e11;
+  return m;
+}
+
+bool pair_ok(const mp_ctx *c, int src, int dst) {
+  if (src < 0 || dst < 0 || src >= c->world || dst >= c->world) return false;
+  return true;
+}
+
+PairModel *pair_model(mp_ctx *c, int src, int dst) {
+  auto key = std::make_pair(src, dst);
+  auto it = c->models.find(key);
+  if (it == c->models.end()) it = c->models.emplace(key, default_pair(c, src, dst)).first;
+  return &it->second;
+}
+
+void fill_config(const PairModel &m, const Selection &s, mp_config *out) {
+  std::memset(out, 0, sizeof(*out));
+  out->npaths = static_cast<int32_t>(m.paths.size());
+  for (size_t i = 0; i < m.paths.size(); ++i) {
+    out->path[i].kind = m.paths[i].kind;
+    out->path[i].via = m.paths[i].via;
+    out->theta[i] = s.theta[i];
+    out->bytes[i] = s.bytes[i];
+    out->chunks[i] = s.chunks[i];
+  }
+  out->t_pred = s.t_pred;
+  out->t_level = s.t_level;
+}
+
+// Engine-side validation of a config against the pair's paths (mp_send/mp_xfer).
+int check_config(mp_ctx *c, const PairModel &m, uint64_t n, const mp_config *cfg) {
+  if (cfg->npaths != static_cast<int32_t>(m.paths.size()))
+    return fail(c, MP_ERR_INVALID, "config npaths does not match the pair's paths");
+  uint64_t sum = 0;
+  for (int i = 0; i < cfg->npaths; ++i) {
+    if (cfg->path[i].kind != m.paths[i].kind || cfg->path[i].via != m.paths[i].via)
+      return fail(c, MP_ERR_TOPOLOGY, "config path " + std::to_string(i) + " is not available");
+    const uint64_t b = cfg->bytes[i];
+    sum += b;
+    if (i == 0 || b == 0) continue;
+    const uint64_t A = c->opts.align, U = b / A, rem = b - U * A;
+    const uint64_t k = cfg->chunks[i];
+    if (k < 1 || k > std::max<uint64_t>(1, U))
+      return fail(c, MP_ERR_INVALID, "chunk count out of range on path " + std::to_string(i));
+    const uint64_t max_chunk = A * ((U + k - 1) / k) + rem;
+    if (max_chunk > c->slot_bytes)
+      return fail(c, MP_ERR_INVALID, "chunk larger than a staging slot on path " + std::to_string(i));
+  }
+  if (sum != n) return fail(c, MP_ERR_INVALID, "config bytes do not sum to the message size");
+  return MP_OK;
+}
+
+int check_err(mp_ctx *c) {
+  if (!c->d_err) return MP_OK;
+  int32_t e = 0;
+  CK(cudaMemcpy(&e, c->d_err, sizeof(e), cudaMemcpyDeviceToHost));
+  if (e == DERR_TIMEOUT) return fail(c, MP_ERR_TIMEOUT, "a device-side wait timed out");
+  if (e == DERR_MISMATCH) return fail(c, MP_ERR_MISMATCH, "send/recv mismatch detected on the device");
+  return MP_OK;
+}
+
+void free_engine(mp_ctx *c) {
+  for (auto &r : c->rings) {
+    if (r.host) {
+      if (r.data) cudaFreeHost(r.data);
+      if (r.full) cudaFreeHost(r.full);
+    } else {
+      if (r.data) cudaFree(r.data);
+      if (r.full) cudaFree(r.full);
+    }
+  }
+  c->rings.clear();
+  if (c->heap.base) cudaFree(c->heap.base);
+  c->heap = Heap();
+  if (c->d_err) cudaFree(c->d_err);
+  c->d_err = nullptr;
+  if (c->d_probe) cudaFree(c->d_probe);
+  c->d_probe = nullptr;
+  if (c->h_probe) cudaFreeHost(c->h_probe);
+  c->h_probe = nullptr;
+  for (auto &p : c->pending) cudaEventDestroy(p.ready);
+  c->pending.clear();
+}
+
+int alloc_ring(mp_ctx *c, bool host, Ring *r) {
+  const uint64_t stride = c->slot_bytes + kSlotSlack;
+  const uint64_t data_bytes = stride * static_cast<uint64_t>(c->slots);
+  const uint64_t flag_bytes = 2ull * c->slots * kFlagStride * sizeof(uint64_t);
+  r->host = host;
+  if (host) {
+    void *d = nullptr, *f = nullptr;
+    CK(cudaHostAlloc(&d, data_bytes, cudaHostAllocMapped | cudaHostAllocPortable));
+    r->data = static_cast<uint8_t *>(d);
+    CK(cudaHostAlloc(&f, flag_bytes, cudaHostAllocMapped | cudaHostAllocPortable));
+    std::memset(f, 0, flag_bytes);
+    r->full = static_cast<uint64_t *>(f);
+  } else {
+    void *d = nullptr, *f = nullptr;
+    CK(cudaMalloc(&d, data_bytes));
+    r->data = static_cast<uint8_t *>(d);
+    CK(cudaMalloc(&f, flag_bytes));
+    CK(cudaMemset(f, 0, flag_bytes));
+    r->full = static_cast<uint64_t *>(f);
+  }
+  r->freef = r->full + static_cast<uint64_t>(c->slots) * kFlagStride;
+  r->q = 0;
+  return MP_OK;
+}
+
+int init_engine(mp_ctx *c) {
+  CK(cudaSetDevice(c->device));
+  if (int e = xfer_capacity(c->device, &c->per_sm, &c->sms))
+    return cuda_fail(c, static_cast<cudaError_t>(e), "occupancy query");
+  void *p = nullptr;
+  CK(cudaMalloc(&p, sizeof(int32_t)));
+  c->d_err = static_cast<int32_t *>(p);
+  CK(cudaMemset(c->d_err, 0, sizeof(int32_t)));
+  CK(cudaMalloc(&p, 64));
+  c->d_probe = static_cast<uint64_t *>(p);
+  CK(cudaHostAlloc(&p, 64, cudaHostAllocMapped | cudaHostAllocPortable));
+  c->h_probe = static_cast<uint64_t *>(p);
+  if (c->heap.size) {
+    void *h = nullptr;
+    cudaError_t e = cudaMalloc(&h, c->heap.size);
+    if (e != cudaSuccess) return fail(c, MP_ERR_NOMEM, "heap allocation failed");
+    c->heap.reset(static_cast<uint8_t *>(h), c->heap.size);
+  }
+  if (c->world == 1) {
+    c->rings.resize(c->n_loop_relays + (c->host_path ? 1 : 0));
+    for (int r = 0; r < c->n_loop_relays; ++r)
+      if (int s = alloc_ring(c, false, &c->rings[r])) return s;
+    if (c->host_path)
+      if (int s = alloc_ring(c, true, &c->rings[c->n_loop_relays])) return s;
+  }
+  return MP_OK;
+}
+
+// Builds the fused launch of one loopback message (A7-A9) and enqueues it.
+int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_config &cfg,
+                    void *stream) {
+  XferParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  P.err = c->d_err;
+  const int cap = std::max(1, c->per_sm * c->sms);
+  uint32_t staged_ctas = 0;
+  for (int i = 1; i < cfg.npaths; ++i)
+    if (cfg.bytes[i]) staged_ctas += 2u * static_cast<uint32_t>(c->relay_ctas);
+  // direct group: up to 4 CTAs per SM, at least 256 KiB per CTA, leaving room
+  // for every staged group to be co-resident.
+  const uint64_t want = std::max<uint64_t>(1, (cfg.bytes[0] + (256u << 10) - 1) / (256u << 10));
+  const int room = std::max(1, cap - static_cast<int>(staged_ctas));
+  const uint32_t g_direct = static_cast<uint32_t>(
+      std::min<uint64_t>(want, static_cast<uint64_t>(std::min(room, 4 * c->sms))));
+  uint32_t next = 0;
+  uint64_t off = 0;
+  P.npaths = static_cast<uint32_t>(cfg.npaths);
+  for (int i = 0; i < cfg.npaths; ++i) {
+    DevPath &d = P.p[i];
+    const uint64_t b = cfg.bytes[i];
+    d.bytes = b;
+    d.src = static_cast<const uint8_t *>(src) + off;
+    d.dst = static_cast<uint8_t *>(dst) + off;
+    d.align = c->opts.align;
+    off += b;
+    if (b == 0) continue;
+    if (i == 0) {
+      d.kind = DK_DIRECT;
+      d.g_in = g_direct;
+      d.cta0_in = next;
+      next += g_direct;
+      continue;
+    }
+    const int ring_idx = cfg.path[i].kind == MP_PATH_HOST ? c->n_loop_relays : cfg.path[i].via;
+    Ring &r = c->rings[ring_idx];
+    d.kind = DK_STAGED;
+    d.k = cfg.chunks[i];
+    d.slots = static_cast<uint32_t>(c->slots);
+    d.host_ring = r.host ? 1u : 0u;
+    d.q0 = r.q;
+    d.slot_stride = c->slot_bytes + kSlotSlack;
+    d.ring = r.data;
+    d.full = r.full;
+    d.freef = r.freef;
+    d.g_out = static_cast<uint32_t>(c->relay_ctas);
+    d.g_in = static_cast<uint32_t>(c->relay_ctas);
+    d.cta0_out = next;  // consumers before producers (deadlock-free dispatch order)
+    next += d.g_out;
+    d.cta0_in = next;
+    next += d.g_in;
+    r.q += d.k;
+  }
+  P.nblocks = next;
+  const int e = launch_xfer(P, stream);
+  if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "xfer launch");
+  c->launches += 1;
+  return MP_OK;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ Heap
+
+void mpx::Heap::reset(uint8_t *b, uint64_t n) {
+  base = b;
+  size = n;
+  free_.clear();
+  used_.clear();
+  if (n) free_[0] = n;
+}
+
+void *mpx::Heap::alloc(uint64_t n) {
+  n = (std::max<uint64_t>(n, 1) + 255) & ~uint64_t(255);
+  for (auto it = free_.begin(); it != free_.end(); ++it) {
+    if (it->second < n) continue;
+    const uint64_t off = it->first, len = it->second;
+    free_.erase(it);
+    if (len > n) free_[off + n] = len - n;
+    used_[off] = n;
+    return base + off;
+  }
+  return nullptr;
+}
+
+bool mpx::Heap::release(void *p) {
+  if (!base) return false;
+  const uint64_t off = static_cast<uint64_t>(static_cast<uint8_t *>(p) - base);
+  auto it = used_.find(off);
+  if (it == used_.end()) return false;
+  uint64_t o = off, len = it->second;
+  used_.erase(it);
+  auto nx = free_.lower_bound(o);
+  if (nx != free_.end() && nx->first == o + len) {
+    len += nx->second;
+    free_.erase(nx);
+  }
+  auto pv = free_.lower_bound(o);
+  if (pv != free_.begin()) {
+    --pv;
+    if (pv->first + pv->second == o) {
+      o = pv->first;
+      len += pv->second;
+      free_.erase(pv);
+    }
+  }
+  free_[o] = len;
+  return true;
+}
+
+// ------------------------------------------------------------------ ABI
+
+extern "C" {
+
+int mp_abi_version(void) { return MP_ABI_VERSION; }
+
+const char *mp_strerror(int s) {
+  switch (s) {
+    case MP_OK: return "MP_OK";
+    case MP_ERR_INVALID: return "MP_ERR_INVALID";
+    case MP_ERR_CUDA: return "MP_ERR_CUDA";
+    case MP_ERR_TOPOLOGY: return "MP_ERR_TOPOLOGY";
+    case MP_ERR_NOMEM: return "MP_ERR_NOMEM";
+    case MP_ERR_STATE: return "MP_ERR_STATE";
+    case MP_ERR_UNSUPPORTED: return "MP_ERR_UNSUPPORTED";
+    case MP_ERR_TIMEOUT: return "MP_ERR_TIMEOUT";
+    case MP_ERR_MISMATCH: return "MP_ERR_MISMATCH";
+    default: return "MP_ERR_UNKNOWN";
+  }
+}
+
+const char *mp_last_error(mp_ctx *c) { return c ? c->last_error.c_str() : "null context"; }
+
+int mp_init(mp_ctx **out, const mp_init_args *a) {
+  if (!out || !a) return MP_ERR_INVALID;
+  *out = nullptr;
+  if (a->world < 1 || a->rank < 0 || a->rank >= a->world) return MP_ERR_INVALID;
+  mp_ctx *c = new (std::nothrow) mp_ctx();
+  if (!c) return MP_ERR_NOMEM;
+  c->rank = a->rank;
+  c->world = a->world;
+  c->device = a->device;
+  c->flags = a->flags;
+  c->model_only = (a->flags & MP_INIT_MODEL_ONLY) != 0;
+  c->n_loop_relays = a->n_loop_relays < 0 ? 6 : std::min(a->n_loop_relays, MP_MAX_PATHS - 2);
+  c->host_path = a->host_path < 0 ? true : a->host_path != 0;
+  c->slots = a->slots > 0 ? a->slots : 4;
+  c->relay_ctas = a->relay_ctas > 0 ? std::min(a->relay_ctas, kFlagStride) : 16;
+  c->slot_bytes = a->slot_bytes ? ((a->slot_bytes + 255) & ~uint64_t(255)) : (32ull << 20);
+  c->timeout_s = a->timeout_s > 0 ? a->timeout_s : 20.0;
+  c->heap.size = a->heap_bytes ? a->heap_bytes : (2304ull << 20);
+  c->opts.slot_bytes = c->slot_bytes > 2 * c->opts.align ? c->slot_bytes - 2 * c->opts.align : 0;
+  if (c->world > MP_MAX_PATHS) {
+    delete c;
+    return MP_ERR_INVALID;
+  }
+  if (!c->model_only) {
+    if (c->world > 1) {
+      delete c;
+      return MP_ERR_UNSUPPORTED;  // multi-process engine: mp_init_world
+    }
+    if (int s = init_engine(c)) {
+      std::string msg = c->last_error;
+      free_engine(c);
+      delete c;
+      std::fprintf(stderr, "mp_init: %s\n", msg.c_str());
+      return s;
+    }
+  }
+  if (a->param_file && a->param_file[0]) {
+    FILE *f = std::fopen(a->param_file, "r");
+    if (f) {
+      std::fclose(f);
+      if (int s = mp_load_params(c, a->param_file)) {
+        mp_finalize(c);
+        return s;
+      }
+    }
+  }
+  if (!c->model_only && !(a->flags & MP_INIT_NO_CALIBRATE) && c->world == 1) {
+    if (int s = mp_calibrate(c, nullptr, 0, 0)) {
+      std::fprintf(stderr, "mp_init: calibration failed: %s\n", c->last_error.c_str());
+      mp_finalize(c);
+      return s;
+    }
+  }
+  *out = c;
+  return MP_OK;
+}
+
+int mp_finalize(mp_ctx *c) {
+  if (!c) return MP_OK;
+  if (!c->model_only) {
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    free_engine(c);
+  }
+  delete c;
+  return MP_OK;
+}
+
+int mp_paths(mp_ctx *c, int src, int dst, mp_path *out, int *npaths) {
+  if (!c || !out || !npaths) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  for (size_t i = 0; i < m->paths.size(); ++i) {
+    out[i].kind = m->paths[i].kind;
+    out[i].via = m->paths[i].via;
+  }
+  *npaths = static_cast<int>(m->paths.size());
+  return MP_OK;
+}
+
+int mp_set_model(mp_ctx *c, int src, int dst, const mp_path *paths, const mp_path_params *prm,
+                 int npaths, const mp_port_params *port) {
+  if (!c || !paths || !prm) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  if (npaths < 1 || npaths > MP_MAX_PATHS) return fail(c, MP_ERR_INVALID, "npaths out of range");
+  PairModel m;
+  for (int i = 0; i < npaths; ++i) {
+    PathModel p;
+    p.kind = paths[i].kind;
+    p.via = paths[i].via;
+    p.alpha = prm[i].alpha;
+    p.beta = prm[i].beta;
+    p.alpha2 = prm[i].alpha2;
+    p.beta2 = prm[i].beta2;
+    p.eps = prm[i].eps;
+    p.c = prm[i].c;
+    p.sigma = prm[i].sigma;
+    p.w = prm[i].w;
+    m.paths.push_back(p);
+  }
+  if (port) {
+    m.port_alpha = port->alpha;
+    m.port_beta = port->beta;
+  }
+  const std::string why = validate_model(m);
+  if (!why.empty()) return fail(c, MP_ERR_INVALID, why);
+  if (!c->model_only && src == dst) {  // loopback paths must map onto existing rings
+    for (const PathModel &p : m.paths) {
+      if (p.kind == K_GPU && (p.via < 0 || p.via >= c->n_loop_relays))
+        return fail(c, MP_ERR_TOPOLOGY, "loopback relay ring does not exist");
+      if (p.kind == K_HOST && !c->host_path) return fail(c, MP_ERR_TOPOLOGY, "host path disabled");
+    }
+  }
+  c->models[std::make_pair(src, dst)] = m;
+  c->cache.clear();
+  return MP_OK;
+}
+
+int mp_get_model(mp_ctx *c, int src, int dst, mp_path *paths, mp_path_params *prm, int *npaths,
+                 mp_port_params *port) {
+  if (!c || !npaths) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  *npaths = static_cast<int>(m->paths.size());
+  for (size_t i = 0; i < m->paths.size(); ++i) {
+    const PathModel &p = m->paths[i];
+    if (paths) {
+      paths[i].kind = p.kind;
+      paths[i].via = p.via;
+    }
+    if (prm) prm[i] = mp_path_params{p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w};
+  }
+  if (port) {
+    port->alpha = m->port_alpha;
+    port->beta = m->port_beta;
+  }
+  return MP_OK;
+}
+
+int mp_set_options(mp_ctx *c, const mp_model_opts *o) {
+  if (!c || !o) return fail(c, MP_ERR_INVALID, "null argument");
+  if (o->mode != MP_MODEL_PAPER && o->mode != MP_MODEL_B200) return fail(c, MP_ERR_INVALID, "bad mode");
+  if (o->align < 1 || o->k_max < 1) return fail(c, MP_ERR_INVALID, "align and k_max must be >= 1");
+  ModelOpts m;
+  m.mode = o->mode;
+  m.stagger = o->stagger ? 1 : 0;
+  m.refine = o->refine < 0 ? -1 : (o->refine ? 1 : 0);
+  m.align = o->align;
+  m.c_min = o->c_min;
+  m.k_max = o->k_max;
+  m.slot_bytes = o->slot_bytes;
+  if (!c->model_only) {  // chunks must fit the engine's staging slots
+    const uint64_t lim = c->slot_bytes > 2 * m.align ? c->slot_bytes - 2 * m.align : 1;
+    if (m.slot_bytes == 0 || m.slot_bytes > lim) m.slot_bytes = lim;
+  }
+  c->opts = m;
+  c->cache.clear();
+  return MP_OK;
+}
+
+int mp_get_options(mp_ctx *c, mp_model_opts *o) {
+  if (!c || !o) return fail(c, MP_ERR_INVALID, "null argument");
+  std::memset(o, 0, sizeof(*o));
+  o->mode = c->opts.mode;
+  o->stagger = c->opts.stagger;
+  o->refine = c->opts.refine;
+  o->align = c->opts.align;
+  o->c_min = c->opts.c_min;
+  o->k_max = c->opts.k_max;
+  o->slot_bytes = c->opts.slot_bytes;
+  return MP_OK;
+}
+
+int mp_predict(mp_ctx *c, int src, int dst, uint64_t bytes, const mp_config *cfg, double *seconds) {
+  if (!c || !cfg || !seconds) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  if (cfg->npaths != static_cast<int32_t>(m->paths.size()))
+    return fail(c, MP_ERR_INVALID, "config npaths does not match the pair's paths");
+  uint64_t sum = 0;
+  for (int i = 0; i < cfg->npaths; ++i) {
+    sum += cfg->bytes[i];
+    if (i > 0 && cfg->bytes[i] && cfg->chunks[i] < 1)
+      return fail(c, MP_ERR_INVALID, "staged path with bytes needs chunks >= 1");
+  }
+  if (sum != bytes) return fail(c, MP_ERR_INVALID, "config bytes do not sum to the message size");
+  *seconds = predict(*m, bytes, cfg->bytes, cfg->chunks, c->opts);
+  return MP_OK;
+}
+
+int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_config *out) {
+  if (!c || !out) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  const CacheKey key{src, dst, mask, bytes};
+  auto it = c->cache.find(key);  // Alg 1 lines 4-6 (C10)
+  if (it == c->cache.end()) {
+    Selection s;
+    select(*m, bytes, mask, c->opts, &s);
+    it = c->cache.emplace(key, std::move(s)).first;  // Alg 1 line 29
+  }
+  fill_config(*m, it->second, out);
+  return MP_OK;
+}
+
+int mp_alloc(mp_ctx *c, uint64_t bytes, void **dptr) {
+  if (!c || !dptr) return fail(c, MP_ERR_INVALID, "null argument");
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  void *p = c->heap.alloc(bytes);
+  if (!p) return fail(c, MP_ERR_NOMEM, "heap exhausted");
+  *dptr = p;
+  return MP_OK;
+}
+
+int mp_free(mp_ctx *c, void *dptr) {
+  if (!c) return MP_ERR_INVALID;
+  if (!dptr) return MP_OK;
+  if (!c->heap.release(dptr)) return fail(c, MP_ERR_INVALID, "pointer not from mp_alloc");
+  return MP_OK;
+}
+
+int mp_xfer(mp_ctx *c, void *dst, const void *src, uint64_t bytes, const mp_config *cfg,
+            void *stream) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  if (c->world != 1) return fail(c, MP_ERR_STATE, "mp_xfer is the single-GPU engine");
+  if (bytes == 0) return MP_OK;
+  if (!dst || !src) return fail(c, MP_ERR_INVALID, "null buffer");
+  const PairModel *m = pair_model(c, 0, 0);
+  mp_config sel;
+  if (!cfg) {
+    if (int s = mp_select(c, 0, 0, bytes, 0, &sel)) return s;
+    cfg = &sel;
+  }
+  if (int s = check_config(c, *m, bytes, cfg)) return s;
+  return launch_loopback(c, dst, src, bytes, *cfg, stream);
+}
+
+int mp_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config *cfg,
+            void *stream) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  if (dst < 0 || dst >= c->world) return fail(c, MP_ERR_TOPOLOGY, "no such rank");
+  if (bytes && !buf) return fail(c, MP_ERR_INVALID, "null buffer");
+  if (c->world != 1) return fail(c, MP_ERR_UNSUPPORTED, "multi-rank send");
+  PendingSend ps;
+  ps.buf = buf;
+  ps.bytes = bytes;
+  ps.tag = tag;
+  ps.has_cfg = cfg != nullptr;
+  if (cfg) {
+    ps.cfg = *cfg;
+    if (int s = check_config(c, *pair_model(c, 0, 0), bytes, cfg)) return s;
+  }
+  CK(cudaEventCreateWithFlags(&ps.ready, cudaEventDisableTiming));
+  CK(cudaEventRecord(ps.ready, static_cast<cudaStream_t>(stream)));
+  c->pending.push_back(ps);
+  return MP_OK;
+}
+
+int mp_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  if (src < 0 || src >= c->world) return fail(c, MP_ERR_TOPOLOGY, "no such rank");
+  if (c->world != 1) return fail(c, MP_ERR_UNSUPPORTED, "multi-rank recv");
+  if (c->pending.empty()) return fail(c, MP_ERR_STATE, "loopback recv without a posted send");
+  PendingSend ps = c->pending.front();
+  if (ps.bytes != bytes || ps.tag != tag) {
+    return fail(c, MP_ERR_MISMATCH, "loopback send/recv size or tag mismatch");
+  }
+  c->pending.pop_front();
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaStreamWaitEvent(st, ps.ready, 0);
+  cudaEventDestroy(ps.ready);
+  if (e != cudaSuccess) return cuda_fail(c, e, "cudaStreamWaitEvent");
+  return mp_xfer(c, buf, ps.buf, bytes, ps.has_cfg ? &ps.cfg : nullptr, stream);
+}
+
+int mp_sync(mp_ctx *c) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return MP_OK;
+  CK(cudaSetDevice(c->device));
+  CK(cudaDeviceSynchronize());
+  return check_err(c);
+}
+
+int mp_stats(mp_ctx *c, uint64_t *launches) {
+  if (!c || !launches) return MP_ERR_INVALID;
+  *launches = c->launches;
+  return MP_OK;
+}
+
+int mp_save_params(mp_ctx *c, const char *path) {
+  if (!c || !path) return MP_ERR_INVALID;
+  FILE *f = std::fopen(path, "w");
+  if (!f) return fail(c, MP_ERR_INVALID, std::string("cannot write ") + path);
+  std::fprintf(f, "mpx-params 1\n");
+  for (const auto &kv : c->models) {
+    const PairModel &m = kv.second;
+    std::fprintf(f, "pair %d %d %zu %.17g %.17g\n", kv.first.first, kv.first.second, m.paths.size(),
+                 m.port_alpha, m.port_beta);
+    for (const PathModel &p : m.paths)
+      std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via,
+                   p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
+  }
+  std::fclose(f);
+  return MP_OK;
+}
+
+int mp_load_params(mp_ctx *c, const char *path) {
+  if (!c || !path) return MP_ERR_INVALID;
+  FILE *f = std::fopen(path, "r");
+  if (!f) return fail(c, MP_ERR_INVALID, std::string("cannot read ") + path);
+  char tag[32];
+  int ver = 0;
+  if (std::fscanf(f, "%31s %d", tag, &ver) != 2 || std::strcmp(tag, "mpx-params") != 0 || ver != 1) {
+    std::fclose(f);
+    return fail(c, MP_ERR_INVALID, "not an mpx parameter file");
+  }
+  int src, dst;
+  size_t np;
+  double pa, pb;
+  while (std::fscanf(f, "%31s %d %d %zu %lf %lf", tag, &src, &dst, &np, &pa, &pb) == 6) {
+    if (std::strcmp(tag, "pair") || np < 1 || np > MP_MAX_PATHS) break;
+    mp_path paths[MP_MAX_PATHS];
+    mp_path_params prm[MP_MAX_PATHS];
+    for (size_t i = 0; i < np; ++i) {
+      mp_path_params &q = prm[i];
+      if (std::fscanf(f, "%31s %d %d %lf %lf %lf %lf %lf %lf %lf %lf", tag, &paths[i].kind, &paths[i].via,
+                      &q.alpha, &q.beta, &q.alpha2, &q.beta2, &q.eps, &q.c, &q.sigma, &q.w) != 11) {
+        std::fclose(f);
+        return fail(c, MP_ERR_INVALID, "truncated parameter file");
+      }
+    }
+    mp_port_params port{pa, pb};
+    if (pair_ok(c, src, dst)) {
+      if (int s = mp_set_model(c, src, dst, paths, prm, static_cast<int>(np), &port)) {
+        std::fclose(f);
+        return s;
+      }
+    }
+  }
+  std::fclose(f);
+  return MP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,359 @@
+// model.cpp — the paper's extended-Hockney model and Algorithm 1, host fp64.
+//
+// Sojoodi et al., SC-W '25, §3-§4.  Readings C1-C18: DESIGN.md §3.
+// This is the product-side implementation behind mp_predict / mp_select; the
+// test-side restatement lives in oracle/model.py and shares nothing with it.
+#include "model.h"
+
+#include <algorithm>
+#include <cmath>
+#include <limits>
+#include <numeric>
+
+namespace mpx {
+
+namespace {
+
+constexpr double kInf = std::numeric_limits<double>::infinity();
+
+// Eq 13 case: case 1 iff β < β'; B200 mode breaks β = β' by α vs ε + α' (C3).
+inline int bottleneck(const PathModel &p, int mode) {
+  if (p.beta < p.beta2) return 1;
+  if (mode == M_B200 && p.beta == p.beta2 && p.alpha > p.eps + p.alpha2) return 1;
+  return 2;
+}
+
+// Staged path carrying x bytes in k chunks.  m = x/k (Eq 12);
+// s1 = α + m/β, s2 = ε + α' + m/β'.  PAPER: Eq 13 (case 1 k·s1 + s2, case 2
+// s1 + k·s2).  B200: s1 + s2 + (k−1)·max(s1, s2) (C3).
+inline double staged_time(const PathModel &p, double x, uint32_t k, int mode) {
+  const double m = x / static_cast<double>(k);
+  const double s1 = p.alpha + m / p.beta;
+  const double s2 = p.eps + p.alpha2 + m / p.beta2;
+  if (mode == M_B200) return s1 + s2 + static_cast<double>(k - 1) * std::max(s1, s2);
+  if (bottleneck(p, M_PAPER) == 1) return static_cast<double>(k) * s1 + s2;
+  return s1 + static_cast<double>(k) * s2;
+}
+
+// Ω, Δ of the unpipelined model; direct Ω = 1/β, Δ = α.
+inline void od_unpipelined(const PathModel &p, double *om, double *de) {
+  if (p.kind == K_DIRECT) {
+    *om = 1.0 / p.beta;
+    *de = p.alpha;
+  } else {
+    *om = 1.0 / p.beta + 1.0 / p.beta2;
+    *de = p.alpha + p.alpha2 + p.eps;
+  }
+}
+
+// φ from the first-pass share x0 (Eq 19, two-pass reading C4).
+inline double phi_of(const PathModel &p, double x0, int mode) {
+  if (bottleneck(p, mode) == 1) return p.c * std::sqrt(p.alpha * p.beta2 / x0);
+  return p.c * std::sqrt((p.eps + p.alpha2) * p.beta / x0);
+}
+
+// Ω, Δ of Eq 22.
+inline void od_eq22(const PathModel &p, double phi, int mode, double *om, double *de) {
+  if (bottleneck(p, mode) == 1) {
+    *om = 1.0 / p.beta + phi / p.beta2;
+    *de = p.eps + p.alpha2 + p.alpha / phi;
+  } else {
+    *om = phi / p.beta + 1.0 / p.beta2;
+    *de = p.alpha + (p.eps + p.alpha2) / phi;
+  }
+}
+
+// Eq 13 at a fixed integer k as an affine T = Ω x + Δ (pass 3, C18).
+inline void od_fixed_k(const PathModel &p, uint32_t k, int mode, double *om, double *de) {
+  if (p.kind == K_DIRECT) {
+    *om = 1.0 / p.beta;
+    *de = p.alpha;
+    return;
+  }
+  const double kd = static_cast<double>(k);
+  if (bottleneck(p, mode) == 1) {
+    *om = 1.0 / p.beta + 1.0 / (kd * p.beta2);
+    *de = kd * p.alpha + p.eps + p.alpha2;
+  } else {
+    *om = 1.0 / (kd * p.beta) + 1.0 / p.beta2;
+    *de = p.alpha + kd * (p.eps + p.alpha2);
+  }
+}
+
+// Eq 19.
+inline double k_eq19(const PathModel &p, double x, double phi, int mode) {
+  if (bottleneck(p, mode) == 1) return phi * x / (p.alpha * p.beta2);
+  return phi * x / ((p.eps + p.alpha2) * p.beta);
+}
+
+// Alg 1 line 17 / P:318: accumulated issue latency of earlier active paths (C8).
+void stagger_of(const PairModel &m, const std::vector<char> &act, const ModelOpts &o,
+                std::vector<double> *st) {
+  st->assign(m.paths.size(), 0.0);
+  double acc = 0.0;
+  for (size_t i = 0; i < m.paths.size(); ++i) {
+    (*st)[i] = o.stagger ? acc : 0.0;
+    if (act[i]) acc += (o.mode == M_PAPER) ? m.paths[i].alpha : m.paths[i].sigma;
+  }
+}
+
+struct Level {
+  std::vector<double> theta;
+  double t = 0.0;
+  std::vector<char> act;
+};
+
+// Eq 24 over the active set, dropping θ < 0 paths until none is left (C2).
+Level level_paper(const PairModel &m, double n, const std::vector<double> &om,
+                  const std::vector<double> &de, std::vector<char> act, const ModelOpts &o) {
+  const size_t p = m.paths.size();
+  std::vector<double> st;
+  for (;;) {
+    stagger_of(m, act, o, &st);
+    double inv_sum = 0.0, delta_sum = 0.0;  // Alg 1 line 22
+    for (size_t i = 0; i < p; ++i)
+      if (act[i]) {
+        inv_sum += 1.0 / om[i];
+        delta_sum += (de[i] + st[i]) / om[i];
+      }
+    Level L;
+    L.theta.assign(p, 0.0);
+    bool any_neg = false;
+    std::vector<char> next = act;
+    for (size_t i = 0; i < p; ++i) {
+      if (!act[i]) continue;
+      const double d = de[i] + st[i];
+      const double th = 1.0 / (om[i] * inv_sum) * (1.0 - d / n * inv_sum + delta_sum / n);
+      L.theta[i] = th;
+      if (th < 0.0) {
+        any_neg = true;
+        next[i] = 0;
+      }
+    }
+    if (!any_neg) {
+      L.t = (n + delta_sum) / inv_sum;
+      L.act = act;
+      return L;
+    }
+    act.swap(next);
+  }
+}
+
+// B200 mode (C14): bytes deliverable by time T; fractional knapsack on the shared
+// port, paths in ascending (w, index).
+double port_fill(const PairModel &m, double T, const std::vector<double> &om,
+                 const std::vector<double> &de, const std::vector<char> &act,
+                 const std::vector<size_t> &order, std::vector<double> *x) {
+  const bool port = m.has_port();
+  double room = port ? std::max(0.0, T - m.port_alpha) * m.port_beta : kInf;
+  double total = 0.0;
+  if (x) x->assign(m.paths.size(), 0.0);
+  for (size_t i : order) {
+    if (!act[i]) continue;
+    double u = std::max(0.0, (T - de[i]) / om[i]);
+    const double w = m.paths[i].w;
+    if (w > 0.0 && port) {
+      u = std::min(u, room / w);
+      room -= w * u;
+    }
+    if (x) (*x)[i] = u;
+    total += u;
+  }
+  return total;
+}
+
+Level level_port(const PairModel &m, double n, const std::vector<double> &om,
+                 const std::vector<double> &de, std::vector<char> act, const ModelOpts &o) {
+  const size_t p = m.paths.size();
+  std::vector<size_t> order(p);
+  std::iota(order.begin(), order.end(), size_t{0});
+  std::stable_sort(order.begin(), order.end(),
+                   [&](size_t a, size_t b) { return m.paths[a].w < m.paths[b].w; });
+  std::vector<double> st, ds(p), x;
+  for (;;) {
+    stagger_of(m, act, o, &st);
+    for (size_t i = 0; i < p; ++i) ds[i] = de[i] + st[i];
+    double lo = 0.0, hi = 1e-9;
+    while (port_fill(m, hi, om, ds, act, order, nullptr) < n) hi *= 2.0;
+    for (int it = 0; it < 200; ++it) {
+      const double mid = 0.5 * (lo + hi);
+      if (port_fill(m, mid, om, ds, act, order, nullptr) >= n)
+        hi = mid;
+      else
+        lo = mid;
+    }
+    port_fill(m, hi, om, ds, act, order, &x);
+    bool changed = false;
+    std::vector<char> next = act;
+    for (size_t i = 0; i < p; ++i)
+      if (act[i] && !(x[i] > 0.0)) {
+        next[i] = 0;
+        changed = true;
+      }
+    if (!changed) {
+      Level L;
+      L.theta.resize(p);
+      for (size_t i = 0; i < p; ++i) L.theta[i] = x[i] / n;
+      L.t = hi;
+      L.act = act;
+      return L;
+    }
+    act.swap(next);
+  }
+}
+
+Level solve(const PairModel &m, double n, const std::vector<double> &om,
+            const std::vector<double> &de, const std::vector<char> &act, const ModelOpts &o) {
+  return o.mode == M_B200 ? level_port(m, n, om, de, act, o) : level_paper(m, n, om, de, act, o);
+}
+
+// Alg 1 lines 23-28 (C7): floor non-direct shares to A, drop below C_min,
+// leftover to the direct path.
+void shares_of(uint64_t n, const Level &L, const ModelOpts &o, std::vector<uint64_t> *b) {
+  const size_t p = L.theta.size();
+  b->assign(p, 0);
+  uint64_t sum = 0;
+  for (size_t i = 1; i < p; ++i) {
+    if (!L.act[i] || !(L.theta[i] > 0.0)) continue;
+    const double units = std::floor(L.theta[i] * static_cast<double>(n) / static_cast<double>(o.align));
+    uint64_t v = static_cast<uint64_t>(units) * o.align;
+    if (v < o.c_min) v = 0;
+    (*b)[i] = v;
+    sum += v;
+  }
+  (*b)[0] = n - sum;
+}
+
+// C5 clamp: [⌈b/slot⌉, min(K_max, ⌊b/C_min⌋)], the slot bound winning.
+uint32_t clamp_k(uint64_t k, uint64_t b, const ModelOpts &o) {
+  const uint64_t hi = std::min<uint64_t>(o.k_max, std::max<uint64_t>(1, o.c_min ? b / o.c_min : b));
+  k = std::min(k, hi);
+  if (o.slot_bytes > 0) k = std::max<uint64_t>(k, (b + o.slot_bytes - 1) / o.slot_bytes);
+  return static_cast<uint32_t>(std::max<uint64_t>(1, k));
+}
+
+}  // namespace
+
+bool PairModel::has_port() const { return port_beta > 0.0 && std::isfinite(port_beta); }
+
+uint32_t k_from_real(double k_real) {
+  // C5: smallest k >= 1 with k(k+1) >= k_real² (1e-12 relative slack for exact ties).
+  const double target = k_real * k_real * (1.0 - 1e-12);
+  uint64_t k = 1;
+  if (!(target > 2.0)) return 1;
+  if (!(target < 1e18)) return 0xffffffffu;  // clamped to K_max by the caller
+  // start near sqrt(target) and settle exactly
+  k = static_cast<uint64_t>(std::max(1.0, std::floor(std::sqrt(target)) - 1.0));
+  while (k > 1 && static_cast<double>((k - 1) * k) >= target) --k;
+  while (static_cast<double>(k * (k + 1)) < target) ++k;
+  return static_cast<uint32_t>(std::min<uint64_t>(k, 0xffffffffu));
+}
+
+std::string validate_model(const PairModel &m) {
+  if (m.paths.empty()) return "no paths";
+  if (m.paths.size() > 16) return "more than MP_MAX_PATHS paths";
+  if (m.paths[0].kind != K_DIRECT) return "paths[0] must be the direct path";
+  for (size_t i = 0; i < m.paths.size(); ++i) {
+    const PathModel &p = m.paths[i];
+    if (p.kind < K_DIRECT || p.kind > K_HOST) return "bad path kind";
+    if (i > 0 && p.kind == K_DIRECT) return "only paths[0] may be direct";
+    if (!(p.beta > 0.0) || !std::isfinite(p.beta)) return "beta must be finite and > 0";
+    if (!(p.alpha >= 0.0) || !std::isfinite(p.alpha)) return "alpha must be finite and >= 0";
+    if (!(p.w >= 0.0) || !(p.sigma >= 0.0)) return "w and sigma must be >= 0";
+    if (p.kind != K_DIRECT) {
+      if (!(p.beta2 > 0.0) || !std::isfinite(p.beta2)) return "staged beta2 must be finite and > 0";
+      if (!(p.alpha2 >= 0.0) || !(p.eps >= 0.0)) return "staged alpha2/eps must be >= 0";
+      if (!(p.c > 0.0)) return "c must be > 0";
+      // Eq 14/19 need α > 0 in case 1 (either mode may pick case 1) and ε + α' > 0 in case 2
+      if (!(p.alpha > 0.0)) return "staged alpha must be > 0 (Eq 14)";
+      if (!(p.eps + p.alpha2 > 0.0)) return "staged eps + alpha2 must be > 0 (Eq 15)";
+    }
+  }
+  return "";
+}
+
+double predict(const PairModel &m, uint64_t n, const uint64_t *bytes, const uint32_t *chunks,
+               const ModelOpts &o) {
+  if (n == 0) return 0.0;
+  const size_t p = m.paths.size();
+  std::vector<char> act(p);
+  for (size_t i = 0; i < p; ++i) act[i] = bytes[i] > 0;
+  std::vector<double> st;
+  stagger_of(m, act, o, &st);
+  double t = 0.0;
+  for (size_t i = 0; i < p; ++i) {
+    if (!act[i]) continue;
+    const PathModel &q = m.paths[i];
+    const double b = static_cast<double>(bytes[i]);
+    const double ti = (q.kind == K_DIRECT) ? q.alpha + b / q.beta           // Eq 6
+                                           : staged_time(q, b, chunks[i], o.mode);  // Eq 13
+    t = std::max(t, ti + st[i]);                                            // Eq 4
+  }
+  if (o.mode == M_B200 && m.has_port()) {
+    double load = 0.0;
+    for (size_t i = 0; i < p; ++i) load += m.paths[i].w * static_cast<double>(bytes[i]);
+    if (load > 0.0) t = std::max(t, m.port_alpha + load / m.port_beta);
+  }
+  return t;
+}
+
+void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, Selection *out) {
+  const size_t p = m.paths.size();
+  out->bytes.assign(p, 0);
+  out->chunks.assign(p, 0);
+  out->theta.assign(p, 0.0);
+  out->t_pred = out->t_level = 0.0;
+  if (n == 0) return;
+  const double nd = static_cast<double>(n);
+  std::vector<char> act(p);
+  for (size_t i = 0; i < p; ++i) act[i] = (i == 0) || mask == 0 || ((mask >> i) & 1u);
+
+  // Pass 1: unpipelined Ω, Δ; Eq 11 / port level with the active set.
+  std::vector<double> om(p), de(p);
+  for (size_t i = 0; i < p; ++i) od_unpipelined(m.paths[i], &om[i], &de[i]);
+  Level L0 = solve(m, nd, om, de, act, o);
+
+  // Pass 2: φ from θ⁽⁰⁾, Eq 22, Eq 24.
+  std::vector<double> phi(p, 0.0);
+  for (size_t i = 0; i < p; ++i) {
+    const PathModel &q = m.paths[i];
+    if (q.kind == K_DIRECT || !L0.act[i]) {
+      od_unpipelined(q, &om[i], &de[i]);
+    } else {
+      phi[i] = phi_of(q, L0.theta[i] * nd, o.mode);
+      od_eq22(q, phi[i], o.mode, &om[i], &de[i]);
+    }
+  }
+  std::vector<char> act1 = L0.act;
+  act1[0] = 1;
+  Level L = solve(m, nd, om, de, act1, o);
+
+  shares_of(n, L, o, &out->bytes);
+  out->chunks[0] = 1;
+  for (size_t i = 1; i < p; ++i) {
+    if (!out->bytes[i]) continue;
+    const double kr = k_eq19(m.paths[i], L.theta[i] * nd, phi[i], o.mode);
+    out->chunks[i] = clamp_k(k_from_real(kr), out->bytes[i], o);
+  }
+
+  const bool refine = o.refine >= 0 ? o.refine != 0 : o.mode == M_B200;
+  if (refine) {  // pass 3 (C18)
+    std::vector<char> act3(p);
+    for (size_t i = 0; i < p; ++i) {
+      od_fixed_k(m.paths[i], std::max<uint32_t>(1, out->chunks[i]), o.mode, &om[i], &de[i]);
+      act3[i] = (i == 0) || out->bytes[i] > 0;
+    }
+    L = solve(m, nd, om, de, act3, o);
+    std::vector<uint32_t> k_prev = out->chunks;
+    shares_of(n, L, o, &out->bytes);
+    for (size_t i = 1; i < p; ++i)
+      out->chunks[i] = out->bytes[i] ? clamp_k(k_prev[i], out->bytes[i], o) : 0;
+  }
+
+  for (size_t i = 0; i < p; ++i)
+    out->theta[i] = (i == 0 || out->bytes[i] > 0) ? L.theta[i] : 0.0;
+  out->t_level = L.t;
+  out->t_pred = predict(m, n, out->bytes.data(), out->chunks.data(), o);
+}
+
+}  // namespace mpx

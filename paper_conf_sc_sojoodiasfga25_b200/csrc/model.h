@@ -1,0 +1,59 @@
+// model.h — host-side fp64 model evaluator and Algorithm 1 selector (internal).
+//
+// PAPER.md §3 (Eq 1-24) and §4 (Alg 1) under the readings of DESIGN.md §3.
+// Independent of oracle/ (which is the test-side restatement); the two share no code.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace mpx {
+
+enum { K_DIRECT = 0, K_GPU = 1, K_HOST = 2 };
+enum { M_PAPER = 0, M_B200 = 1 };
+
+struct PathModel {
+  int kind = K_DIRECT;
+  int via = -1;
+  double alpha = 0, beta = 0, alpha2 = 0, beta2 = 0, eps = 0, c = 1, sigma = 0, w = 0;
+};
+
+struct PairModel {
+  std::vector<PathModel> paths;  // paths[0] is the direct path
+  double port_alpha = 0.0;
+  double port_beta = 0.0;        // <= 0 or inf: no shared port
+  bool has_port() const;
+};
+
+struct ModelOpts {
+  int mode = M_PAPER;
+  int stagger = 1;
+  int refine = -1;
+  uint64_t align = 256;
+  uint64_t c_min = 65536;
+  uint64_t k_max = 1024;
+  uint64_t slot_bytes = 0;
+};
+
+struct Selection {
+  std::vector<uint64_t> bytes;
+  std::vector<uint32_t> chunks;
+  std::vector<double> theta;
+  double t_pred = 0.0;
+  double t_level = 0.0;
+};
+
+// Returns an empty string when the pair model is valid, else the reason.
+std::string validate_model(const PairModel &m);
+
+// O2: predicted time of a config (bytes sum to n).
+double predict(const PairModel &m, uint64_t n, const uint64_t *bytes, const uint32_t *chunks,
+               const ModelOpts &o);
+
+// O3: Algorithm 1.  mask bit i enables path i (bit 0 forced on).
+void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, Selection *out);
+
+// The C5 integer rule (exposed for tests through the selector only).
+uint32_t k_from_real(double k_real);
+
+}  // namespace mpx

@@ -1,0 +1,283 @@
+"""Thin ctypes binding of the C ABI in include/mp.h (argument marshalling only).
+
+Every step of the hot path runs in libmpx.so (host C++ model/selector, sm_100a
+kernels).  There is no Python or CPU fallback: if the library cannot be loaded the
+import raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from typing import List, Optional, Sequence
+
+from . import _build
+
+MP_MAX_PATHS = 16
+MP_PATH_DIRECT, MP_PATH_GPU, MP_PATH_HOST = 0, 1, 2
+MP_MODEL_PAPER, MP_MODEL_B200 = 0, 1
+MP_INIT_MODEL_ONLY, MP_INIT_NO_CALIBRATE = 1, 2
+
+STATUS = {0: "MP_OK", -1: "MP_ERR_INVALID", -2: "MP_ERR_CUDA", -3: "MP_ERR_TOPOLOGY",
+          -4: "MP_ERR_NOMEM", -5: "MP_ERR_STATE", -6: "MP_ERR_UNSUPPORTED",
+          -7: "MP_ERR_TIMEOUT", -8: "MP_ERR_MISMATCH"}
+
+
+class MPError(RuntimeError):
+    def __init__(self, status: int, msg: str = ""):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class mp_path(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("via", C.c_int32)]
+
+
+class mp_path_params(C.Structure):
+    _fields_ = [(n, C.c_double) for n in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")]
+
+
+class mp_port_params(C.Structure):
+    _fields_ = [("alpha", C.c_double), ("beta", C.c_double)]
+
+
+class mp_model_opts(C.Structure):
+    _fields_ = [("mode", C.c_int32), ("stagger", C.c_int32), ("refine", C.c_int32),
+                ("reserved", C.c_int32), ("align", C.c_uint64), ("c_min", C.c_uint64),
+                ("k_max", C.c_uint64), ("slot_bytes", C.c_uint64)]
+
+
+class mp_config(C.Structure):
+    _fields_ = [("npaths", C.c_int32), ("reserved", C.c_int32),
+                ("path", mp_path * MP_MAX_PATHS), ("theta", C.c_double * MP_MAX_PATHS),
+                ("bytes", C.c_uint64 * MP_MAX_PATHS), ("chunks", C.c_uint32 * MP_MAX_PATHS),
+                ("t_pred", C.c_double), ("t_level", C.c_double)]
+
+    def as_dict(self):
+        n = self.npaths
+        return dict(paths=[(self.path[i].kind, self.path[i].via) for i in range(n)],
+                    theta=[self.theta[i] for i in range(n)],
+                    bytes=[int(self.bytes[i]) for i in range(n)],
+                    chunks=[int(self.chunks[i]) for i in range(n)],
+                    t_pred=self.t_pred, t_level=self.t_level)
+
+
+ALLGATHER = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64)
+
+
+class mp_init_args(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("device", C.c_int32), ("flags", C.c_int32),
+                ("n_loop_relays", C.c_int32), ("host_path", C.c_int32), ("slots", C.c_int32),
+                ("relay_ctas", C.c_int32), ("heap_bytes", C.c_uint64), ("slot_bytes", C.c_uint64),
+                ("timeout_s", C.c_double), ("allgather", ALLGATHER), ("allgather_user", C.c_void_p),
+                ("param_file", C.c_char_p)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libmpx.so (building it in-tree with nvcc first if it is missing/stale)."""
+    global _lib
+    if _lib is None:
+        path = _build.build()
+        L = C.CDLL(path, mode=C.RTLD_GLOBAL)
+        P = C.c_void_p
+        sig = {
+            "mp_init": (C.c_int, [C.POINTER(P), C.POINTER(mp_init_args)]),
+            "mp_finalize": (C.c_int, [P]),
+            "mp_strerror": (C.c_char_p, [C.c_int]),
+            "mp_last_error": (C.c_char_p, [P]),
+            "mp_abi_version": (C.c_int, []),
+            "mp_paths": (C.c_int, [P, C.c_int, C.c_int, C.POINTER(mp_path), C.POINTER(C.c_int)]),
+            "mp_set_model": (C.c_int, [P, C.c_int, C.c_int, C.POINTER(mp_path), C.POINTER(mp_path_params),
+                                       C.c_int, C.POINTER(mp_port_params)]),
+            "mp_get_model": (C.c_int, [P, C.c_int, C.c_int, C.POINTER(mp_path), C.POINTER(mp_path_params),
+                                       C.POINTER(C.c_int), C.POINTER(mp_port_params)]),
+            "mp_set_options": (C.c_int, [P, C.POINTER(mp_model_opts)]),
+            "mp_get_options": (C.c_int, [P, C.POINTER(mp_model_opts)]),
+            "mp_predict": (C.c_int, [P, C.c_int, C.c_int, C.c_uint64, C.POINTER(mp_config),
+                                     C.POINTER(C.c_double)]),
+            "mp_select": (C.c_int, [P, C.c_int, C.c_int, C.c_uint64, C.c_uint32, C.POINTER(mp_config)]),
+            "mp_alloc": (C.c_int, [P, C.c_uint64, C.POINTER(P)]),
+            "mp_free": (C.c_int, [P, P]),
+            "mp_send": (C.c_int, [P, P, C.c_uint64, C.c_int, C.c_int, C.POINTER(mp_config), P]),
+            "mp_recv": (C.c_int, [P, P, C.c_uint64, C.c_int, C.c_int, P]),
+            "mp_xfer": (C.c_int, [P, P, P, C.c_uint64, C.POINTER(mp_config), P]),
+            "mp_sync": (C.c_int, [P]),
+            "mp_calibrate": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int]),
+            "mp_save_params": (C.c_int, [P, C.c_char_p]),
+            "mp_load_params": (C.c_int, [P, C.c_char_p]),
+            "mp_stats": (C.c_int, [P, C.POINTER(C.c_uint64)]),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def exported_symbols() -> List[str]:
+    return ["mp_init", "mp_finalize", "mp_strerror", "mp_last_error", "mp_abi_version", "mp_paths",
+            "mp_set_model", "mp_get_model", "mp_set_options", "mp_get_options", "mp_predict",
+            "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
+            "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats"]
+
+
+def _ptr(x) -> Optional[int]:
+    """Device/host pointer of a torch tensor, an int, or None."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    return x.data_ptr()
+
+
+def _stream(s) -> Optional[int]:
+    if s is None:
+        return None
+    if isinstance(s, int):
+        return s
+    return s.cuda_stream
+
+
+class Context:
+    """One mp_ctx.  Methods mirror the C ABI names and raise MPError on failure."""
+
+    def __init__(self, rank=0, world=1, device=0, model_only=False, calibrate=False,
+                 n_loop_relays=-1, host_path=-1, slots=0, relay_ctas=0, heap_bytes=0,
+                 slot_bytes=0, timeout_s=0.0, allgather=None, param_file=None):
+        L = lib()
+        a = mp_init_args()
+        a.rank, a.world, a.device = rank, world, device
+        a.flags = (MP_INIT_MODEL_ONLY if model_only else 0) | (0 if calibrate else MP_INIT_NO_CALIBRATE)
+        a.n_loop_relays, a.host_path, a.slots, a.relay_ctas = n_loop_relays, host_path, slots, relay_ctas
+        a.heap_bytes, a.slot_bytes, a.timeout_s = heap_bytes, slot_bytes, timeout_s
+        self._ag = ALLGATHER(allgather) if allgather else ALLGATHER()
+        a.allgather = self._ag
+        a.param_file = param_file.encode() if param_file else None
+        h = C.c_void_p()
+        st = L.mp_init(C.byref(h), C.byref(a))
+        if st != 0:
+            raise MPError(st, "mp_init failed")
+        self.h = h
+        self.world, self.rank = world, rank
+
+    def _ck(self, st):
+        if st != 0:
+            raise MPError(st, lib().mp_last_error(self.h).decode())
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().mp_finalize(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---------------------------------------------------------------- model
+    def paths(self, src=0, dst=0):
+        arr = (mp_path * MP_MAX_PATHS)()
+        n = C.c_int()
+        self._ck(lib().mp_paths(self.h, src, dst, arr, C.byref(n)))
+        return [(arr[i].kind, arr[i].via) for i in range(n.value)]
+
+    def set_model(self, src, dst, paths: Sequence, params: Sequence[dict], port: Optional[dict] = None):
+        n = len(paths)
+        pa = (mp_path * MP_MAX_PATHS)(*[mp_path(k, v) for k, v in paths])
+        pr = (mp_path_params * MP_MAX_PATHS)(
+            *[mp_path_params(*[float(p.get(f, d)) for f, d in
+                               (("alpha", 0), ("beta", 0), ("alpha2", 0), ("beta2", 0), ("eps", 0),
+                                ("c", 1), ("sigma", 0), ("w", 0))]) for p in params])
+        po = mp_port_params(port["alpha"], port["beta"]) if port else None
+        self._ck(lib().mp_set_model(self.h, src, dst, pa, pr, n, C.byref(po) if po else None))
+
+    def get_model(self, src=0, dst=0):
+        pa = (mp_path * MP_MAX_PATHS)()
+        pr = (mp_path_params * MP_MAX_PATHS)()
+        n = C.c_int()
+        po = mp_port_params()
+        self._ck(lib().mp_get_model(self.h, src, dst, pa, pr, C.byref(n), C.byref(po)))
+        params = [{f: getattr(pr[i], f) for f, _ in mp_path_params._fields_} for i in range(n.value)]
+        return [(pa[i].kind, pa[i].via) for i in range(n.value)], params, dict(alpha=po.alpha, beta=po.beta)
+
+    def set_options(self, mode=MP_MODEL_PAPER, stagger=1, refine=-1, align=256, c_min=65536,
+                    k_max=1024, slot_bytes=0):
+        o = mp_model_opts(mode, stagger, refine, 0, align, c_min, k_max, slot_bytes)
+        self._ck(lib().mp_set_options(self.h, C.byref(o)))
+
+    def get_options(self):
+        o = mp_model_opts()
+        self._ck(lib().mp_get_options(self.h, C.byref(o)))
+        return {f: getattr(o, f) for f, _ in mp_model_opts._fields_ if f != "reserved"}
+
+    def make_config(self, nbytes: Sequence[int], chunks: Sequence[int], src=0, dst=0) -> mp_config:
+        cfg = mp_config()
+        ps = self.paths(src, dst)
+        assert len(nbytes) == len(ps) == len(chunks)
+        cfg.npaths = len(ps)
+        for i, (k, v) in enumerate(ps):
+            cfg.path[i] = mp_path(k, v)
+            cfg.bytes[i] = int(nbytes[i])
+            cfg.chunks[i] = int(chunks[i])
+        return cfg
+
+    def predict(self, src, dst, n, cfg: mp_config) -> float:
+        t = C.c_double()
+        self._ck(lib().mp_predict(self.h, src, dst, n, C.byref(cfg), C.byref(t)))
+        return t.value
+
+    def select(self, src, dst, n, mask=0) -> mp_config:
+        cfg = mp_config()
+        self._ck(lib().mp_select(self.h, src, dst, n, mask, C.byref(cfg)))
+        return cfg
+
+    # ---------------------------------------------------------------- engine
+    def alloc(self, n) -> int:
+        p = C.c_void_p()
+        self._ck(lib().mp_alloc(self.h, n, C.byref(p)))
+        return p.value
+
+    def free(self, p):
+        self._ck(lib().mp_free(self.h, p))
+
+    def xfer(self, dst, src, n, cfg: Optional[mp_config] = None, stream=None):
+        self._ck(lib().mp_xfer(self.h, _ptr(dst), _ptr(src), n, C.byref(cfg) if cfg else None,
+                               _stream(stream)))
+
+    def send(self, buf, n, dst, tag=0, cfg: Optional[mp_config] = None, stream=None):
+        self._ck(lib().mp_send(self.h, _ptr(buf), n, dst, tag, C.byref(cfg) if cfg else None,
+                               _stream(stream)))
+
+    def recv(self, buf, n, src, tag=0, stream=None):
+        self._ck(lib().mp_recv(self.h, _ptr(buf), n, src, tag, _stream(stream)))
+
+    def sync(self):
+        self._ck(lib().mp_sync(self.h))
+
+    def calibrate(self, sizes: Optional[Sequence[int]] = None, reps=0):
+        if sizes:
+            arr = (C.c_uint64 * len(sizes))(*sizes)
+            self._ck(lib().mp_calibrate(self.h, arr, len(sizes), reps))
+        else:
+            self._ck(lib().mp_calibrate(self.h, None, 0, reps))
+
+    def save_params(self, path):
+        self._ck(lib().mp_save_params(self.h, path.encode()))
+
+    def load_params(self, path):
+        self._ck(lib().mp_load_params(self.h, path.encode()))
+
+    def launches(self) -> int:
+        v = C.c_uint64()
+        self._ck(lib().mp_stats(self.h, C.byref(v)))
+        return v.value

@@ -1,0 +1,126 @@
+"""Parity of the library's model (mp_predict / mp_select, host C++ behind the C ABI)
+with the CPU oracle (oracle/model.py) on seeded synthetic parameter tables.
+
+Bar (BASELINE.json north star + DESIGN.md C17): predictions within 1e-9 relative in
+fp64; selected shares equal up to ±A bytes per path with Σ = n exactly; chunk counts
+equal; the linearised level within 1e-9.  Host-only, runs without a GPU."""
+import math
+import random
+
+import pytest
+
+import synth
+from oracle import model as M
+from paper_conf_sc_sojoodiasfga25_b200 import mp
+
+MiB = 1 << 20
+MODES = [M.PAPER, M.B200]
+
+
+def rel(a, b):
+    return abs(a - b) / max(abs(b), 1e-300)
+
+
+def setup_pair(ctx, tbl, port):
+    paths = [(t["kind"], t["via"]) for t in tbl]
+    params = [{k: t[k] for k in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")} for t in tbl]
+    for p in params:
+        if math.isinf(p["beta2"]):
+            p["beta2"] = 0.0          # unused for the direct path
+    ctx.set_model(0, 1, paths, params, port)
+
+
+def oracle_paths(tbl):
+    return [M.Path(**t) for t in tbl]
+
+
+def opts_for(mode, stagger, refine, slot=64 * MiB):
+    return M.Options(mode=mode, stagger=bool(stagger), refine=refine, slot_bytes=slot)
+
+
+CASES = [(seed, nrel, host, mode, stagger, refine)
+         for seed in range(6) for nrel in (1, 2, 6) for host in (True, False)
+         for mode in MODES for stagger in (0, 1) for refine in (None, False, True)
+         if (seed + nrel + stagger) % 2 == 0]
+
+
+@pytest.mark.parametrize("seed,nrel,host,mode,stagger,refine", CASES)
+def test_select_and_predict_parity(seed, nrel, host, mode, stagger, refine):
+    tbl = synth.topology(1000 + seed, nrel, host)
+    port = dict(alpha=1.5e-6, beta=850e9)
+    paths = oracle_paths(tbl)
+    oport = M.Port(**port)
+    o = opts_for(mode, stagger, refine)
+    with mp.Context(world=8, rank=0, model_only=True) as c:
+        # the C side resolves (0,1) to direct + 6 relays + host; install our table
+        setup_pair(c, tbl, port)
+        c.set_options(mode=mode, stagger=stagger, refine=-1 if refine is None else int(refine),
+                      slot_bytes=o.slot_bytes)
+        rng = random.Random(seed)
+        for n in (1, 4096, MiB + 17, 16 * MiB, 64 * MiB + 3, 1 << 30, (2 << 30) - 1):
+            cfg = c.select(0, 1, n)
+            d = cfg.as_dict()
+            ref = M.select(n, paths, o, oport)
+            assert sum(d["bytes"]) == n
+            for a, b in zip(d["bytes"], ref.bytes):
+                assert abs(a - b) <= o.align
+            assert rel(d["t_level"], ref.t_level) < 1e-9
+            if d["bytes"] == ref.bytes:
+                assert d["chunks"] == ref.chunks
+                assert rel(d["t_pred"], ref.t_pred) < 1e-9
+            # prediction parity on the library's own config and on random configs
+            t_o = M.evaluate(n, d["bytes"], d["chunks"], paths, o, oport)
+            assert rel(d["t_pred"], t_o) < 1e-9
+            for _ in range(3):
+                w = [rng.random() for _ in paths]
+                nb = [int(n * x / sum(w)) for x in w]
+                nb[0] += n - sum(nb)
+                ks = [1] + [rng.randint(1, 64) for _ in paths[1:]]
+                ccfg = c.make_config(nb, ks, 0, 1)
+                assert rel(c.predict(0, 1, n, ccfg), M.evaluate(n, nb, ks, paths, o, oport)) < 1e-9
+
+
+@pytest.mark.parametrize("mask", [0b1, 0b11, 0b101, 0b1001, 0b1111])
+def test_mask_parity(mask):
+    tbl = synth.topology(77, 2, True)
+    paths = oracle_paths(tbl)
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        setup_pair(c, tbl, None)
+        n = 256 * MiB
+        d = c.select(0, 1, n, mask).as_dict()
+        ref = M.select(n, paths, M.Options(), None, [bool(mask >> i & 1) for i in range(4)])
+        for a, b in zip(d["bytes"], ref.bytes):
+            assert abs(a - b) <= 256
+        for i in range(1, 4):
+            if not (mask >> i & 1):
+                assert d["bytes"][i] == 0
+
+
+def test_golden_cases_through_the_abi():
+    # G2 (Eq 8) and G3 (Eq 11) through mp_select / mp_predict
+    us, gbs = 1e-6, 1e9
+    with mp.Context(world=3, rank=0, model_only=True) as c:
+        c.set_options(stagger=0, align=1, c_min=0, refine=0)
+        # G3: direct (1 µs, 100 GB/s) + staged (1, 100, ε 2, α' 1, β' 100), n = 3e6 -> 22 µs.
+        # k = 1 reproduces the unpipelined Eq 2 (Eq 13 with k = 1 is Eq 2).
+        c.set_model(0, 1, [(0, -1), (1, 2)],
+                    [dict(alpha=1 * us, beta=100 * gbs),
+                     dict(alpha=1 * us, beta=100 * gbs, alpha2=1 * us, beta2=100 * gbs, eps=2 * us)])
+        cfg = c.make_config([2_100_000, 900_000], [1, 1], 0, 1)
+        assert rel(c.predict(0, 1, 3_000_000, cfg), 22 * us) < 1e-12
+        # G1 (Eq 1): a single direct path
+        c.set_model(0, 1, [(0, -1)], [dict(alpha=2 * us, beta=50 * gbs)])
+        d = c.select(0, 1, 1_000_000).as_dict()
+        assert d["bytes"] == [1_000_000] and rel(d["t_pred"], 22 * us) < 1e-12
+
+
+def test_cache_invalidation():
+    tbl = synth.topology(5, 2, True)
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        setup_pair(c, tbl, None)
+        a = c.select(0, 1, 64 * MiB).as_dict()
+        assert c.select(0, 1, 64 * MiB).as_dict() == a       # cached (C10)
+        tbl[0]["beta"] *= 2
+        setup_pair(c, tbl, None)
+        b = c.select(0, 1, 64 * MiB).as_dict()
+        assert b["bytes"][0] > a["bytes"][0]
