@@ -1,0 +1,326 @@
+#!/usr/bin/env python3
+"""Benchmark of the multi-path P2P hot path (BASELINE.json metric:
+"P2P GB/s vs msg size (% of path roofline); model-vs-sweep optimum error %").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl mpx|reference]
+                    [--size BYTES] [--mode b200|paper]
+
+One *step* = one message through the whole hot path: mp_select (Alg 1, cached after
+the first call — §8(a) A1-A6) and one fused multi-path transfer launch (A7 direct,
+A8 relay rings, A9 pinned-host PCIe, A10 completion).
+
+N = 1 (default): BASELINE.json config 3 — 1 GiB, direct + 6 relays + pinned host —
+on the single-GPU loopback engine (the relay rings stand in for the intermediate
+GPUs; the host leg is real PCIe); the config is the B200-mode model's pick after an
+init-time calibration (Step 1).  Inputs are 1 GiB (> 126 MB L2), so no flush.
+N > 1 (torchrun): every rank runs its own loopback message (independent replicas,
+"scaling": "weak"); the multi-rank engine is not on the bench path yet.
+
+--impl reference: the CPU oracle (oracle/, fp64 model + memcpy replay) on a bounded
+sample of the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+GiB, MiB = 1 << 30, 1 << 20
+METRIC = "P2P GB/s vs msg size (% of path roofline); model-vs-sweep optimum error %"
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+class Clocks:
+    """Sample nvidia-smi SM clocks and throttle reasons during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index, self.samples, self.stop_ = index, [], threading.Event()
+        self.t = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self.stop_.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.samples.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self.stop_.wait(0.2)
+
+    def __enter__(self):
+        self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop_.set()
+        self.t.join(timeout=10)
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = sorted(float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit())
+        mx = max((float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()), default=None)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for s in self.samples for n, v in zip(names, s[3:7]) if v.strip() == "Active"})
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(self.samples)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def hbm_bytes(d):
+    """Algorithmic HBM bytes of one loopback message: every payload
+    byte is read once from src and written once to dst; a relay byte is also written
+    to and read from its ring slot; a host byte's slot traffic is PCIe/host DRAM."""
+    paths, nb = d["paths"], d["bytes"]
+    relay = sum(b for (k, _), b in zip(paths, nb) if k == 1)
+    return 2 * sum(nb) + 2 * relay
+
+
+def cpu_oracle_run(n, cfg_d, params, budget_s=12.0, sample=256 * MiB):
+    """Time the oracle as it stands (fp64 select + memcpy replay through the split) on a
+    bounded sample of the workload.  Returns (GB/s, description, threads)."""
+    import numpy as np
+    import synth
+    from oracle import model as OM
+    from oracle import transfer as OX
+    scale = sample / n
+    nb = [int(b * scale) // 256 * 256 for b in cfg_d["bytes"]]
+    nb[0] += sample - sum(nb)
+    kinds = [k for k, _ in cfg_d["paths"]]
+    ch = [max(1, min(c, max(1, b // 256))) if b else 0 for b, c in zip(nb, cfg_d["chunks"])]
+    ch[0] = 1
+    src = synth.payload(sample, 0)
+    dst = np.zeros(sample, dtype=np.uint8)
+    paths = [OM.Path(kind=k, via=v, **{f: (p[f] if not (k == 0 and f == "beta2") else float("inf"))
+                                        for f in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")})
+             for (k, v), p in zip(cfg_d["paths"], params)]
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        OM.select(sample, paths, OM.Options(mode=OM.B200))
+        OX.replay(src, nb, ch, kinds, 256, dst)
+        reps += 1
+        if time.perf_counter() - t0 > budget_s or reps >= 50:
+            break
+    dt = time.perf_counter() - t0
+    assert np.array_equal(dst, src)
+    return sample * reps / dt / 1e9, f"{reps} x {sample >> 20} MiB of the {n >> 20} MiB split (same θ, k)", 1
+
+
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    import numpy as np
+    import synth
+    from oracle import model as OM
+    from oracle import transfer as OX
+    n = args.size
+    tbl = synth.topology(0, 6, True)
+    paths = [OM.Path(**t) for t in tbl]
+    opts = OM.Options(mode=OM.B200 if args.mode == "b200" else OM.PAPER, slot_bytes=32 * MiB - 512)
+    cfg = OM.select(n, paths, opts, OM.Port(4e-6, 6.5e12))
+    sample = min(n, 32 * MiB)
+    scale = sample / n
+    nb = [int(b * scale) // 256 * 256 for b in cfg.bytes]
+    nb[0] += sample - sum(nb)
+    ch = [max(1, min(c, max(1, b // 256))) if b else 0 for b, c in zip(nb, cfg.chunks)]
+    ch[0] = 1
+    kinds = [t["kind"] for t in tbl]
+    src = synth.payload(sample, 0)
+    dst = np.zeros(sample, dtype=np.uint8)
+
+    def step():
+        OM.select(sample, paths, opts, OM.Port(4e-6, 6.5e12))
+        OX.replay(src, nb, ch, kinds, 256, dst)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = time.perf_counter() - t0
+    v = sample * args.steps / dt / 1e9
+    desc = f"{sample >> 20} MiB per step of the {n >> 20} MiB config-3 split (numpy memcpy replay + fp64 select)"
+    line = {"metric": METRIC, "value": v, "unit": "GB/s", "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic", "config": workload_config(args, world),
+            "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+            "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def workload_config(args, world):
+    return {"workload": "config3: 1 GiB GPU0->GPU0 loopback, direct + 6 relay rings + pinned-host PCIe, "
+                        "B200-mode model-selected split" if args.size == GiB else
+            f"{args.size} B loopback, direct + 6 relay rings + pinned host, model-selected",
+            "msg_bytes": args.size, "mode": args.mode, "paths": "direct+6relay+host",
+            "l2": "inputs 1 GiB > 126 MB L2 (no flush)", "parallelism": f"replicas{world}"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=400)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="mpx", choices=["mpx", "reference"])
+    ap.add_argument("--size", type=int, default=GiB)
+    ap.add_argument("--mode", default="b200", choices=["b200", "paper"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-calibrate", action="store_true",
+                    help="skip the init-time calibration (default parameters; for ncu runs)")
+    ap.add_argument("--params", default=None, help="load model parameters (Step 2) instead of calibrating")
+    ap.add_argument("--save-params", default=None, help="write the calibrated parameters (Step 1)")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+
+    world, rank, local = dist_env()
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    n = args.size
+    ctx = mp.Context(device=local, calibrate=not (args.no_calibrate or args.params), n_loop_relays=6,
+                     host_path=1, heap_bytes=16 * MiB, param_file=args.params)
+    if args.save_params and rank == 0:
+        ctx.save_params(args.save_params)
+    ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
+    cfg = ctx.select(0, 0, n)
+    d = cfg.as_dict()
+    stream = torch.cuda.Stream()
+    g = torch.Generator(device="cuda").manual_seed(20251116 + rank)
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g)
+    dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+
+    def step():
+        ctx.xfer(dst, src, n, None, stream)   # mp_select (cached) + one fused launch
+
+    with torch.cuda.stream(stream):
+        for _ in range(args.warmup):
+            step()
+    torch.cuda.synchronize()
+    ctx.sync()
+    assert torch.equal(dst, src), "payload mismatch"
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    l0 = ctx.launches()
+    with Clocks(local) as clk:
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for i in range(args.steps):
+            ev[i][0].record(stream)
+            step()
+            ev[i][1].record(stream)
+        t1.record(stream)
+        torch.cuda.synchronize()
+    launches = ctx.launches() - l0
+    ctx.sync()
+    ms = t0.elapsed_time(t1)
+    per_launch = sorted(a.elapsed_time(b) for a, b in ev)
+    ms_t = torch.tensor([ms], device="cuda")
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+        dist.barrier()
+    ms = float(ms_t.item())
+    value = n * world * args.steps / (ms * 1e-3) / 1e9
+
+    # end to end through the public API with host buffers: H2D of the payload from
+    # pinned memory, the transfer, D2H of the received message, every step.
+    h_src = src.cpu().pin_memory()
+    h_dst = torch.empty(n, dtype=torch.uint8).pin_memory()
+    e2e_steps = max(3, args.steps // 4)
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    with torch.cuda.stream(stream):
+        e0.record(stream)
+        for _ in range(e2e_steps):
+            src.copy_(h_src, non_blocking=True)
+            step()
+            h_dst.copy_(dst, non_blocking=True)
+        e1.record(stream)
+    torch.cuda.synchronize()
+    e2e = n * e2e_steps / (e0.elapsed_time(e1) * 1e-3) / 1e9
+    assert torch.equal(h_dst, h_src)
+
+    peak, peak_src = measured_peaks()
+    alg = hbm_bytes(d)
+    avg_launch_ms = sum(per_launch) / len(per_launch)
+    achieved = alg / (avg_launch_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(str(n), {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    _, prm, port = ctx.get_model(0, 0)
+    line = {
+        "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded uniform random bytes)",
+        "config": workload_config(args, world),
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "peak_source": peak_src, "kernel": "xfer_kernel",
+                     "algorithmic_bytes_per_launch": alg},
+        "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n, "d2h_bytes_per_step": n},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+        "model": {"selected": d, "predicted_GBps": n / d["t_pred"] / 1e9 if d["t_pred"] else None,
+                  "E_pred": abs(n / d["t_pred"] / 1e9 - value / world) / (value / world) if d["t_pred"] else None,
+                  "port": port, "direct_params": prm[0], "host_params": prm[-1]},
+        "per_launch_ms": {"min": per_launch[0], "median": per_launch[len(per_launch) // 2],
+                          "max": per_launch[-1]},
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, desc, cores = cpu_oracle_run(n, d, prm)
+        line["cpu_baseline"] = {"value": v, "unit": "GB/s", "cores": cores, "kind": "oracle", "sample": desc}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -136,12 +136,19 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
   if (c->world != 1) return cfail(c, MP_ERR_UNSUPPORTED, "calibration runs on the loopback engine");
   if (reps <= 0) reps = 5;
+  // Default sizes: the asymptotic range (C12).  A local HBM→HBM copy only shows its
+  // steady-state rate once the working set exceeds the 126 MB L2, so the direct link
+  // is fitted on 128 MiB .. 1 GiB; the ring legs on what the ring holds.
   std::vector<uint64_t> sizes;
   if (sizes_in && nsizes > 0)
     sizes.assign(sizes_in, sizes_in + nsizes);
   else
-    for (uint64_t s = 1ull << 20; s <= (256ull << 20); s <<= 1) sizes.push_back(s);
+    for (uint64_t s = 16ull << 20; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
   const uint64_t big = *std::max_element(sizes.begin(), sizes.end());
+  std::vector<uint64_t> direct_sizes;
+  for (uint64_t s : sizes)
+    if (s >= (128ull << 20)) direct_sizes.push_back(s);
+  if (direct_sizes.size() < 2) direct_sizes = sizes;
 
   Bench b;
   b.c = c;
@@ -160,7 +167,7 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
   double eps_dev = 0, eps_host = 0;
   const uint64_t ring_cap = static_cast<uint64_t>(c->slots) * c->slot_bytes;
   do {
-    if ((st = fit_link(b, dst, src, sizes, big, reps, &fd))) break;
+    if ((st = fit_link(b, dst, src, direct_sizes, big, reps, &fd))) break;
     if (c->n_loop_relays > 0) {
       uint8_t *ring = c->rings[0].data;
       if ((st = fit_link(b, ring, src, sizes, ring_cap, reps, &f1))) break;

@@ -220,9 +220,9 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   uint32_t staged_ctas = 0;
   for (int i = 1; i < cfg.npaths; ++i)
     if (cfg.bytes[i]) staged_ctas += 2u * static_cast<uint32_t>(c->relay_ctas);
-  // direct group: up to 4 CTAs per SM, at least 256 KiB per CTA, leaving room
+  // direct group: up to 4 CTAs per SM, at least 32 KiB per CTA, leaving room
   // for every staged group to be co-resident.
-  const uint64_t want = std::max<uint64_t>(1, (cfg.bytes[0] + (256u << 10) - 1) / (256u << 10));
+  const uint64_t want = std::max<uint64_t>(1, (cfg.bytes[0] + (32u << 10) - 1) / (32u << 10));
   const int room = std::max(1, cap - static_cast<int>(staged_ctas));
   const uint32_t g_direct = static_cast<uint32_t>(
       std::min<uint64_t>(want, static_cast<uint64_t>(std::min(room, 4 * c->sms))));

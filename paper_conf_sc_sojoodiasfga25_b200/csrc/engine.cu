@@ -192,7 +192,7 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
   }
 }
 
-__global__ void __launch_bounds__(kThreads) xfer_kernel(const __grid_constant__ XferParams P) {
+__global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant__ XferParams P) {
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();

@@ -1,0 +1,189 @@
+"""GPU parity of the transfer engine (sm_100a kernels through the C ABI) against the
+oracle reference transfer (oracle/transfer.py, O1): bit-exact payloads, canaries
+intact, every path kind, odd sizes and misaligned offsets, the model-selected
+configs, and BASELINE.json's full sizes."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import synth
+from oracle import model as M
+from oracle import transfer as X
+from paper_conf_sc_sojoodiasfga25_b200 import mp
+
+pytestmark = pytest.mark.gpu
+MiB = 1 << 20
+CAN = 4096
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    torch.cuda.init()
+    c = mp.Context(device=0, n_loop_relays=6, host_path=1, slot_bytes=4 * MiB, slots=4,
+                   relay_ctas=8, heap_bytes=64 * MiB, timeout_s=10.0)
+    yield c
+    c.close()
+
+
+def run(ctx, n, nbytes, chunks, src_off=0, dst_off=0, seed=0):
+    host = synth.payload(n + 64, seed)
+    src_full = torch.from_numpy(host).cuda()
+    src = src_full[src_off:src_off + n]
+    dst_full = torch.full((n + 2 * CAN + 64,), 0xA5, dtype=torch.uint8, device="cuda")
+    dst = dst_full[CAN + dst_off:CAN + dst_off + n]
+    cfg = ctx.make_config(nbytes, chunks)
+    ctx.xfer(dst, src, n, cfg, torch.cuda.current_stream())
+    ctx.sync()
+    got = dst_full.cpu().numpy()
+    kinds = [k for k, _ in ctx.paths()]
+    exp = np.full(n, 0, dtype=np.uint8)
+    X.replay(host[src_off:src_off + n], nbytes, chunks, kinds, 256, exp)
+    assert np.array_equal(got[CAN + dst_off:CAN + dst_off + n], exp)
+    assert (got[:CAN + dst_off] == 0xA5).all()
+    assert (got[CAN + dst_off + n:] == 0xA5).all()
+
+
+@pytest.mark.parametrize("n", [1, 15, 16, 17, 255, 4095, 65536 + 3, MiB + 17])
+def test_direct_only(ctx, n):
+    np_ = len(ctx.paths())
+    run(ctx, n, [n] + [0] * (np_ - 1), [1] + [0] * (np_ - 1))
+
+
+@pytest.mark.parametrize("src_off,dst_off", [(0, 0), (1, 1), (8, 8), (15, 15), (16, 0), (1, 0), (3, 7)])
+def test_all_paths_misaligned(ctx, src_off, dst_off):
+    ps = ctx.paths()
+    n = 6 * MiB + 4099
+    per = 512 * 1024
+    nbytes = [0] + [per] * (len(ps) - 1)
+    nbytes[0] = n - sum(nbytes)
+    chunks = [1] + [1 + i % 4 for i in range(len(ps) - 1)]
+    run(ctx, n, nbytes, chunks, src_off, dst_off, seed=3)
+
+
+@pytest.mark.parametrize("kind", ["relay", "host"])
+@pytest.mark.parametrize("k", [1, 2, 3, 7, 16])
+def test_single_staged_path_many_chunks(ctx, kind, k):
+    # a staged path alone (direct gets 0 bytes), more chunks than ring slots: the slot
+    # reuse / generation flags are exercised (S = 4)
+    ps = ctx.paths()
+    i = 1 if kind == "relay" else len(ps) - 1
+    n = 3 * MiB + 256 * 5
+    nbytes = [0] * len(ps)
+    nbytes[i] = n
+    chunks = [1] + [0] * (len(ps) - 1)
+    chunks[i] = k
+    for rep in range(3):                    # repeated messages continue the ring sequence
+        run(ctx, n, nbytes, chunks, seed=rep)
+
+
+def test_ragged_tail_not_multiple_of_align(ctx):
+    ps = ctx.paths()
+    n = 2 * MiB + 100
+    nbytes = [0] * len(ps)
+    nbytes[1] = 1 * MiB + 100        # forced configs may carry a non-multiple of A
+    nbytes[0] = n - nbytes[1]
+    chunks = [1] + [0] * (len(ps) - 1)
+    chunks[1] = 3
+    run(ctx, n, nbytes, chunks)
+
+
+def test_invalid_configs_rejected(ctx):
+    ps = ctx.paths()
+    n = MiB
+    cfg = ctx.make_config([n - 1] + [0] * (len(ps) - 1), [1] + [0] * (len(ps) - 1))
+    src = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    dst = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    with pytest.raises(mp.MPError):                     # Σ bytes != n
+        ctx.xfer(dst, src, n, cfg)
+    nb = [0] * len(ps)
+    nb[0], nb[1] = n - 8192, 8192
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1] = 64                                         # k > ⌊b/A⌋
+    with pytest.raises(mp.MPError):
+        ctx.xfer(dst, src, n, ctx.make_config(nb, ks))
+    nb[1] = 16 * MiB
+    nb[0] = 0
+    ks[1] = 1                                          # chunk larger than a 4 MiB slot
+    with pytest.raises(mp.MPError):
+        ctx.xfer(dst, src, 16 * MiB, ctx.make_config(nb, ks))
+
+
+@pytest.mark.parametrize("mode", [mp.MP_MODEL_PAPER, mp.MP_MODEL_B200])
+@pytest.mark.parametrize("n", [MiB, 16 * MiB + 5, 64 * MiB])
+def test_model_selected_transfer(ctx, mode, n):
+    ctx.set_options(mode=mode)
+    cfg = ctx.select(0, 0, n)
+    d = cfg.as_dict()
+    assert sum(d["bytes"]) == n
+    run(ctx, n, d["bytes"], d["chunks"], seed=5)
+    ctx.set_options()
+
+
+def test_send_recv_loopback(ctx):
+    n = 5 * MiB + 3
+    host = synth.payload(n, 9)
+    src = torch.from_numpy(host).cuda()
+    dst = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    ctx.send(src, n, 0, tag=7, stream=s1)
+    ctx.recv(dst, n, 0, tag=7, stream=s2)
+    s2.synchronize()
+    ctx.sync()
+    assert torch.equal(dst, src)
+    ctx.send(src, n, 0, tag=1)
+    with pytest.raises(mp.MPError) as e:
+        ctx.recv(dst, n, 0, tag=2)
+    assert e.value.status == -8
+
+
+def test_launch_counter(ctx):
+    a = ctx.launches()
+    n = MiB
+    src = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    dst = torch.zeros(n, dtype=torch.uint8, device="cuda")
+    ctx.xfer(dst, src, n)
+    ctx.sync()
+    assert ctx.launches() == a + 1
+
+
+def test_calibration_installs_sane_parameters():
+    c = mp.Context(device=0, n_loop_relays=2, host_path=1, slot_bytes=32 * MiB, heap_bytes=16 * MiB)
+    c.calibrate(sizes=[MiB << i for i in range(0, 8)], reps=3)
+    paths, prm, port = c.get_model(0, 0)
+    assert paths[0] == (0, -1)
+    d = prm[0]
+    assert 5e11 < d["beta"] < 6e12 and 0 < d["alpha"] < 1e-4          # local HBM copy
+    h = prm[-1]
+    assert 5e9 < h["beta"] < 1.5e11 and 5e9 < h["beta2"] < 1.5e11    # PCIe Gen5 legs
+    assert 0 < h["eps"] < 2e-5 and 0 < prm[1]["eps"] < 1e-5
+    assert port["beta"] > d["beta"]
+    c.close()
+
+
+def test_full_size_config3_bit_exact(ctx):
+    # BASELINE.json config 3 at full size (1 GiB, direct + 6 relays + host) on the
+    # loopback engine, in the paper-mode split (every path carries bytes): bit-exact on
+    # the device, plus sampled bytes against the oracle's definition.
+    n = 1 << 30
+    big = mp.Context(device=0, n_loop_relays=6, host_path=1, heap_bytes=16 * MiB)
+    try:
+        big.set_options(mode=mp.MP_MODEL_PAPER)
+        d = big.select(0, 0, n).as_dict()
+        if min(d["bytes"]) == 0:       # force every path on if the model excluded some
+            k = len(d["bytes"])
+            per = (n // (k + 1)) // 256 * 256
+            d["bytes"] = [n - per * (k - 1)] + [per] * (k - 1)
+            d["chunks"] = [1] + [8] * (k - 1)
+        g = torch.Generator(device="cuda").manual_seed(synth.payload_seed(31))
+        src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g)
+        dst = torch.zeros(n, dtype=torch.uint8, device="cuda")
+        big.xfer(dst, src, n, big.make_config(d["bytes"], d["chunks"]))
+        big.sync()
+        assert torch.equal(dst, src)
+        idx = torch.randint(0, n, (4096,), device="cuda")
+        assert torch.equal(dst[idx].cpu(), src[idx].cpu())
+    finally:
+        big.close()
