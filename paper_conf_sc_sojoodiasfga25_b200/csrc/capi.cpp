@@ -3,6 +3,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <limits>
 #include <new>
@@ -185,6 +186,8 @@ int init_engine(mp_ctx *c) {
   CK(cudaSetDevice(c->device));
   if (int e = xfer_capacity(c->device, &c->per_sm, &c->sms))
     return cuda_fail(c, static_cast<cudaError_t>(e), "occupancy query");
+  if (int e = preload_kernels()) return cuda_fail(c, static_cast<cudaError_t>(e), "kernel preload");
+  if (const char *m = std::getenv("MPX_COPY")) c->copy_mode = std::strcmp(m, "reg") == 0 ? 0u : 1u;
   void *p = nullptr;
   CK(cudaMalloc(&p, sizeof(int32_t)));
   c->d_err = static_cast<int32_t *>(p);
@@ -216,6 +219,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   std::memset(&P, 0, sizeof(P));
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.err = c->d_err;
+  P.copy_mode = c->copy_mode;
   const int cap = std::max(1, c->per_sm * c->sms);
   uint32_t staged_ctas = 0;
   for (int i = 1; i < cfg.npaths; ++i)
@@ -367,13 +371,14 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
     delete c;
     return MP_ERR_INVALID;
   }
+  c->allgather = a->allgather;
+  c->allgather_user = a->allgather_user;
   if (!c->model_only) {
-    if (c->world > 1) {
-      delete c;
-      return MP_ERR_UNSUPPORTED;  // multi-process engine: mp_init_world
-    }
-    if (int s = init_engine(c)) {
+    int s = init_engine(c);
+    if (!s && c->world > 1) s = world_init(c);
+    if (s) {
       std::string msg = c->last_error;
+      if (c->world > 1) world_finalize(c);
       free_engine(c);
       delete c;
       std::fprintf(stderr, "mp_init: %s\n", msg.c_str());
@@ -405,6 +410,7 @@ int mp_finalize(mp_ctx *c) {
   if (!c) return MP_OK;
   if (!c->model_only) {
     cudaSetDevice(c->device);
+    if (c->world > 1) world_finalize(c);  // stops the persistent relay kernel first
     cudaDeviceSynchronize();
     free_engine(c);
   }
@@ -588,7 +594,17 @@ int mp_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const 
   if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
   if (dst < 0 || dst >= c->world) return fail(c, MP_ERR_TOPOLOGY, "no such rank");
   if (bytes && !buf) return fail(c, MP_ERR_INVALID, "null buffer");
-  if (c->world != 1) return fail(c, MP_ERR_UNSUPPORTED, "multi-rank send");
+  if (c->world != 1) {
+    if (dst == c->rank) return fail(c, MP_ERR_TOPOLOGY, "send to self needs world == 1 (loopback)");
+    const PairModel *m = pair_model(c, c->rank, dst);
+    mp_config sel;
+    if (!cfg) {
+      if (int s = mp_select(c, c->rank, dst, bytes, 0, &sel)) return s;
+      cfg = &sel;
+    }
+    if (int s = check_config(c, *m, bytes, cfg)) return s;
+    return world_send(c, buf, bytes, dst, tag, *cfg, stream);
+  }
   PendingSend ps;
   ps.buf = buf;
   ps.bytes = bytes;
@@ -608,7 +624,11 @@ int mp_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
   if (src < 0 || src >= c->world) return fail(c, MP_ERR_TOPOLOGY, "no such rank");
-  if (c->world != 1) return fail(c, MP_ERR_UNSUPPORTED, "multi-rank recv");
+  if (c->world != 1) {
+    if (src == c->rank) return fail(c, MP_ERR_TOPOLOGY, "recv from self needs world == 1 (loopback)");
+    if (bytes && !buf) return fail(c, MP_ERR_INVALID, "null buffer");
+    return world_recv(c, buf, bytes, src, tag, stream);
+  }
   if (c->pending.empty()) return fail(c, MP_ERR_STATE, "loopback recv without a posted send");
   PendingSend ps = c->pending.front();
   if (ps.bytes != bytes || ps.tag != tag) {
@@ -626,6 +646,7 @@ int mp_sync(mp_ctx *c) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return MP_OK;
   CK(cudaSetDevice(c->device));
+  if (c->world > 1) return world_sync(c);
   CK(cudaDeviceSynchronize());
   return check_err(c);
 }

@@ -78,6 +78,7 @@ struct mp_ctx {
   uint64_t slot_bytes = 32ull << 20;
   double timeout_s = 20.0;
   int per_sm = 0, sms = 0;
+  uint32_t copy_mode = 1;          // direct-path copy: 1 = TMA bulk, 0 = LDG/STG (env MPX_COPY=reg)
   int32_t *d_err = nullptr;
   std::vector<mpx::Ring> rings;   // loopback: [0..V) relays, [V] host (if enabled)
   mpx::Heap heap;
@@ -85,4 +86,30 @@ struct mp_ctx {
   uint64_t launches = 0;
   uint64_t *d_probe = nullptr;    // calibration flag words (device)
   uint64_t *h_probe = nullptr;    // calibration flag words (mapped host)
+
+  // multi-rank engine (world > 1), see engine.h / world.cpp
+  mp_allgather_fn allgather = nullptr;
+  void *allgather_user = nullptr;
+  uint64_t jobid = 0;
+  mpx::CtrlLayout L;
+  uint8_t *ctrl = nullptr;                  // this rank's control block (device)
+  std::vector<mpx::PeerPtrs> peers;         // [world]: heap/ctrl of every rank (self = local)
+  uint64_t host_stride = 0;
+  uint64_t hseg_per_src = 0;                // bytes of one pair's host ring in a segment
+  size_t hseg_bytes = 0;
+  std::vector<uint8_t *> hseg;              // [world]: mapped host segment of each receiver
+  std::vector<uint64_t> send_seq, recv_seq, relay_q, host_q, done_target;
+  cudaStream_t relay_stream = nullptr;
+  int32_t *stop = nullptr;                  // mapped host word read by the relay kernel
+  bool relay_running = false;
+  std::vector<cudaStream_t> streams;        // user streams seen by mp_send/mp_recv
 };
+
+namespace mpx {
+int world_init(mp_ctx *c);
+int world_finalize(mp_ctx *c);
+int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,
+               void *stream);
+int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream);
+int world_sync(mp_ctx *c);
+}  // namespace mpx

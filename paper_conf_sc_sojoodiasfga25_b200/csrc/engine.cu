@@ -110,35 +110,182 @@ __device__ __forceinline__ void group_copy(uint8_t *dst, const uint8_t *src, uin
   if (gt < len - t0) dst[t0 + gt] = ld1<MODE>(src + t0 + gt);
 }
 
+// ------------------------------------------------------------------ TMA bulk copy
+
+// Bulk-copy engine of one CTA: thread 0 streams 16 KiB blocks global → shared →
+// global with cp.async.bulk (TMA; SASS UBLKCP), kBulkStages blocks in flight, the
+// load of each stage completing on an mbarrier (complete_tx) and each store tracked
+// by a bulk group so a stage is only reloaded once its previous store has finished
+// reading shared memory.  Blocks r, r+G, r+2G, … of the co-aligned 16-B body belong
+// to CTA r; head/tail bytes go through group_copy.  Requires (dst ^ src) % 16 == 0.
+constexpr uint32_t kBulkBlock = 16384;
+constexpr uint32_t kBulkStages = 3;
+constexpr uint32_t kBulkSmem = kBulkBlock * kBulkStages + 64;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint32_t bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(bar) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_load(uint32_t dst_smem, const void *src, uint32_t bytes, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst_smem),
+      "l"(src), "r"(bytes), "r"(bar)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_store(void *dst, uint32_t src_smem, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src_smem), "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
+__device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32_t r, uint32_t G,
+                          uint8_t *smem) {
+  if ((reinterpret_cast<uintptr_t>(dst) ^ reinterpret_cast<uintptr_t>(src)) & 15u) {
+    group_copy<LD_SRC>(dst, src, len, r, G);
+    return;
+  }
+  uint64_t head = (16u - (reinterpret_cast<uintptr_t>(src) & 15u)) & 15u;
+  if (head > len) head = len;
+  const uint64_t body = (len - head) & ~uint64_t(15);
+  const uint64_t tail0 = head + body;
+  // head and tail (< 16 B each) by CTA 0's threads
+  if (r == 0) {
+    if (threadIdx.x < head) dst[threadIdx.x] = src[threadIdx.x];
+    if (threadIdx.x < len - tail0) dst[tail0 + threadIdx.x] = src[tail0 + threadIdx.x];
+  }
+  if (threadIdx.x != 0) return;
+  const uint8_t *s = src + head;
+  uint8_t *d = dst + head;
+  const uint64_t nblk = (body + kBulkBlock - 1) / kBulkBlock;
+  if (r >= nblk) return;
+  const uint64_t mine = (nblk - r + G - 1) / G;  // blocks r, r+G, …
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + kBulkBlock * kBulkStages);
+  for (uint32_t i = 0; i < kBulkStages; ++i) mbar_init(smem_u32(bars + i));
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  auto blk = [&](uint64_t it, uint64_t *off, uint32_t *bytes) {
+    const uint64_t o = (r + it * G) * static_cast<uint64_t>(kBulkBlock);
+    *off = o;
+    *bytes = static_cast<uint32_t>(body - o < kBulkBlock ? body - o : kBulkBlock);
+  };
+  auto issue_load = [&](uint64_t it) {
+    uint64_t o;
+    uint32_t n;
+    blk(it, &o, &n);
+    const uint32_t st = static_cast<uint32_t>(it % kBulkStages);
+    const uint32_t bar = smem_u32(bars + st);
+    mbar_expect_tx(bar, n);
+    bulk_load(smem_u32(smem + st * kBulkBlock), s + o, n, bar);
+  };
+  const uint64_t pro = mine < kBulkStages ? mine : kBulkStages;
+  for (uint64_t it = 0; it < pro; ++it) issue_load(it);
+  for (uint64_t it = 0; it < mine; ++it) {
+    const uint32_t st = static_cast<uint32_t>(it % kBulkStages);
+    mbar_wait(smem_u32(bars + st), static_cast<uint32_t>((it / kBulkStages) & 1));
+    uint64_t o;
+    uint32_t n;
+    blk(it, &o, &n);
+    bulk_store(d + o, smem_u32(smem + st * kBulkBlock), n);
+    // refill the stage used one iteration ago once its store has read shared memory
+    if (it >= 1 && it - 1 + kBulkStages < mine) {
+      bulk_wait_read<1>();
+      issue_load(it - 1 + kBulkStages);
+    }
+  }
+  bulk_wait_all();
+}
+
 // ------------------------------------------------------------------ flags
 
 // Warp 0 polls `n` flag words until every one is >= target (ld.acquire.sys), then
-// the CTA synchronises.  Returns false (and raises DERR_TIMEOUT) on timeout.
+// the CTA synchronises.  Returns false (and raises DERR_TIMEOUT) on timeout, or when
+// the optional host `stop` word becomes non-zero (persistent relay shutdown; then no
+// error is raised and timeout_ns may be 0 = wait forever).
 __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, uint64_t target,
-                                           const XferParams &P, int *s_abort) {
+                                           uint64_t timeout_ns, int32_t *err, int *s_abort,
+                                           const volatile int32_t *stop = nullptr) {
   if (threadIdx.x < 32) {
     const uint32_t lane = threadIdx.x;
     const uint64_t t_start = globaltimer();
-    bool ok = true;
-    for (;;) {
+    int why = 0;
+    for (uint32_t it = 0;; ++it) {
       const bool mine = lane >= n || ld_acquire_sys(flags + lane) >= target;
       if (__all_sync(0xffffffffu, mine)) break;
-      if (globaltimer() - t_start > P.timeout_ns) {
-        ok = false;
+      if (timeout_ns && globaltimer() - t_start > timeout_ns) {
+        why = 1;
         break;
       }
-      __nanosleep(64);
+      if (stop && (it & 255u) == 255u && *stop) {
+        why = 2;
+        break;
+      }
+      __nanosleep(stop ? 256 : 64);
     }
     if (lane == 0) {
-      if (!ok) {
-        atomicExch(P.err, DERR_TIMEOUT);
-        *s_abort = 1;
-      }
+      if (why == 1) atomicExch(err, DERR_TIMEOUT);
+      if (why) *s_abort = 1;
       fence_acq_rel_sys();
     }
   }
   __syncthreads();
   return *s_abort == 0;
+}
+
+// Thread 0 polls one word until it equals / exceeds target, then the CTA syncs.
+__device__ __forceinline__ bool wait_word(const uint64_t *w, uint64_t target, uint64_t timeout_ns,
+                                          int32_t *err, int *s_abort) {
+  if (threadIdx.x == 0) {
+    const uint64_t t_start = globaltimer();
+    while (ld_acquire_sys(w) < target) {
+      if (globaltimer() - t_start > timeout_ns) {
+        atomicExch(err, DERR_TIMEOUT);
+        *s_abort = 1;
+        break;
+      }
+      __nanosleep(64);
+    }
+    fence_acq_rel_sys();
+  }
+  __syncthreads();
+  return *s_abort == 0;
+}
+
+__device__ __forceinline__ void red_add_release_sys(uint64_t *p, uint64_t v) {
+  asm volatile("red.release.sys.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t ld_volatile(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
 }
 
 __device__ __forceinline__ void release_flag(uint64_t *flag, uint64_t value) {
@@ -166,7 +313,7 @@ __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, 
     uint64_t off, len;
     chunk_range(p, j, &off, &len);
     const uint64_t q = p.q0 + j, s = q % p.slots, u = q / p.slots;
-    if (!wait_flags(p.freef + s * kFlagStride, p.g_out, u, P, s_abort)) return;
+    if (!wait_flags(p.freef + s * kFlagStride, p.g_out, u, P.timeout_ns, P.err, s_abort)) return;
     const uint8_t *src = p.src + off;
     uint8_t *slot = p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(src) & 15u);
     // slice r of the chunk, split on 16-byte boundaries of the source
@@ -184,7 +331,7 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
     uint64_t off, len;
     chunk_range(p, j, &off, &len);
     const uint64_t q = p.q0 + j, s = q % p.slots, u = q / p.slots;
-    if (!wait_flags(p.full + s * kFlagStride, p.g_in, u + 1, P, s_abort)) return;
+    if (!wait_flags(p.full + s * kFlagStride, p.g_in, u + 1, P.timeout_ns, P.err, s_abort)) return;
     const uint8_t *slot =
         p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(p.src + off) & 15u);
     group_copy<MODE>(p.dst + off, slot, len, r, p.g_out);
@@ -193,6 +340,7 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
 }
 
 __global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant__ XferParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
@@ -202,7 +350,10 @@ __global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant
     if (p.bytes == 0) continue;
     if (b >= p.cta0_in && b < p.cta0_in + p.g_in) {
       if (p.kind == DK_DIRECT)
-        group_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in);
+        if (P.copy_mode == 1)
+          bulk_copy(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem);
+        else
+          group_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in);
       else
         run_stage_in(p, b - p.cta0_in, P, &s_abort);
       return;
@@ -243,11 +394,243 @@ __global__ void pingpong_kernel(uint64_t *flags, int iters, uint64_t timeout_ns,
   }
 }
 
+
+// ================================================================== multi-rank engine
+
+__device__ __forceinline__ void chunk_of(uint64_t bytes, uint64_t align, uint32_t k, uint32_t j,
+                                         uint64_t *off, uint64_t *len) {
+  const uint64_t U = bytes / align, rem = bytes - U * align;
+  const uint64_t s = align * ((j * U) / k);
+  uint64_t e = align * (((j + 1) * U) / k);
+  if (j + 1 == k) e += rem;
+  *off = s;
+  *len = e - s;
+}
+
+__device__ __forceinline__ MsgEntry *entry_at(uint8_t *ctrl, uint64_t base, uint32_t peer, uint64_t m) {
+  return reinterpret_cast<MsgEntry *>(ctrl + base) + (static_cast<uint64_t>(peer) * kCtsRing + m % kCtsRing);
+}
+
+__device__ __forceinline__ uint64_t *done_at(uint8_t *ctrl, const CtrlLayout &L, uint32_t src) {
+  return reinterpret_cast<uint64_t *>(ctrl + L.done + static_cast<uint64_t>(src) * 128);
+}
+
+__device__ __forceinline__ uint64_t *flags_at(uint8_t *ctrl, uint64_t base, uint32_t who, uint32_t slots,
+                                              uint64_t slot) {
+  return reinterpret_cast<uint64_t *>(ctrl + base) + (static_cast<uint64_t>(who) * slots + slot) * kFlagStride;
+}
+
+// Slice r of G of [0, len), split on 16-byte boundaries.
+__device__ __forceinline__ void slice_of(uint64_t len, uint32_t r, uint32_t G, uint64_t *a, uint64_t *b) {
+  *a = ((len * r / G) + 15) & ~uint64_t(15);
+  uint64_t e = ((len * (r + 1) / G) + 15) & ~uint64_t(15);
+  if (r + 1 == G || e > len) e = len;
+  if (*a > e) *a = e;
+  *b = e;
+}
+
+// After a CTA's stores: make them visible system-wide, count `bytes` into a peer's
+// done counter, optionally release a flag.
+__device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t *flag, uint64_t value) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    fence_acq_rel_sys();
+    if (done && bytes) red_add_release_sys(done, bytes);
+    if (flag) st_release_sys(flag, value);
+  }
+}
+
+__global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant__ SendParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
+  __shared__ int s_abort;
+  __shared__ uint64_t s_off;
+  if (threadIdx.x == 0) s_abort = 0;
+  __syncthreads();
+  // wait for the receiver's clear-to-send (rendezvous, P:62 analogue)
+  MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
+  if (!wait_word(&cts->seq1, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
+  if (threadIdx.x == 0) {
+    const uint64_t off = ld_volatile(&cts->a), n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
+    s_off = off;
+    const bool bad = (n != P.bytes) || (tag != P.tag);
+    if (blockIdx.x == 0) {
+      uint64_t host_k = 0, host_q0 = 0;
+      for (uint32_t i = 0; i < P.npaths; ++i)
+        if (P.sp[i].kind == 2) {
+          host_k = P.sp[i].k;
+          host_q0 = P.sp[i].q0;
+        }
+      MsgEntry *h = entry_at(P.dst_ctrl, P.L.hdr, P.me, P.seq);
+      h->a = bad ? 0 : host_k;
+      h->b = host_q0;
+      h->c = bad ? 2 : 0;
+      fence_acq_rel_sys();
+      st_release_sys(&h->seq1, P.seq + 1);
+    }
+    if (bad) {
+      atomicExch(P.err, DERR_MISMATCH);
+      s_abort = 1;
+    }
+  }
+  __syncthreads();
+  if (s_abort) return;
+  const uint64_t base = s_off;
+  const uint32_t b = blockIdx.x;
+  uint64_t *done = done_at(P.dst_ctrl, P.L, P.me);
+  if (b < P.g_direct) {  // A7: direct NVLink stores into the receiver's heap
+    if (P.copy_mode == 1)
+      bulk_copy(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct, dyn_smem);
+    else
+      group_copy<LD_SRC>(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct);
+    const uint64_t share = P.direct_bytes * (b + 1) / P.g_direct - P.direct_bytes * b / P.g_direct;
+    publish(done, share, nullptr, 0);
+    return;
+  }
+  for (uint32_t i = 0; i < P.npaths; ++i) {
+    const SendParams::StagedDesc &d = P.sp[i];
+    if (b < d.cta0 || b >= d.cta0 + P.g_stage) continue;
+    const uint32_t r = b - d.cta0;
+    for (uint32_t j = 0; j < d.k; ++j) {  // A8/A9 step 1
+      uint64_t off, len;
+      chunk_of(d.bytes, 256, d.k, j, &off, &len);
+      off += d.off;
+      const uint64_t q = d.q0 + j;
+      uint64_t *fr, *fl;
+      uint8_t *slot;
+      uint32_t nfree;
+      if (d.kind == 1) {
+        const uint64_t s = q % P.L.slots;
+        fr = flags_at(P.my_ctrl, P.L.relay_free, d.relay, P.L.slots, s);
+        fl = flags_at(d.ring_ctrl, P.L.ring_full, P.me, P.L.slots, s);
+        slot = d.ring_ctrl + P.L.ring_data + (static_cast<uint64_t>(P.me) * P.L.slots + s) * P.L.stride;
+        nfree = P.g_stage;
+      } else {
+        const uint64_t s = q % P.host_slots;
+        fr = P.host.freef + s * kFlagStride;
+        fl = P.host.full + s * kFlagStride;
+        slot = P.host.data + s * P.host_stride;
+        nfree = P.g_stage;
+      }
+      const uint64_t u = q / (d.kind == 1 ? P.L.slots : P.host_slots);
+      if (!wait_flags(fr, nfree, u, P.timeout_ns, P.err, &s_abort)) return;
+      const uint8_t *src = P.src + off;
+      const uint64_t shift = reinterpret_cast<uintptr_t>(src) & 15u;
+      uint8_t *data = slot + kSlotHdr + shift;
+      uint64_t a, e;
+      slice_of(len, r, P.g_stage, &a, &e);
+      if (a < e) group_copy<LD_SRC>(data + a, src + a, e - a, 0, 1);
+      if (r == 0 && threadIdx.x == 0) {
+        uint64_t *h = reinterpret_cast<uint64_t *>(slot);
+        h[0] = P.dst;
+        h[1] = base + off;
+        h[2] = len;
+        h[3] = shift;
+      }
+      publish(nullptr, 0, fl + r, u + 1);
+    }
+    return;
+  }
+}
+
+__global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant__ RecvParams P) {
+  __shared__ int s_abort;
+  __shared__ uint64_t s_k, s_q0;
+  if (threadIdx.x == 0) s_abort = 0;
+  __syncthreads();
+  MsgEntry *hdr = entry_at(P.my_ctrl, P.L.hdr, P.src, P.seq);
+  if (blockIdx.x == 0) {
+    if (threadIdx.x == 0) {  // post the clear-to-send into the sender's control block
+      MsgEntry *cts = entry_at(P.src_ctrl, P.L.cts, P.me, P.seq);
+      cts->a = P.heap_off;
+      cts->b = P.bytes;
+      cts->c = P.tag;
+      fence_acq_rel_sys();
+      st_release_sys(&cts->seq1, P.seq + 1);
+      // A10: wait until every byte of the message has been counted in
+      const uint64_t *done = done_at(P.my_ctrl, P.L, P.src);
+      const uint64_t t_start = globaltimer();
+      while (ld_acquire_sys(done) < P.done_target) {
+        if (ld_acquire_sys(&hdr->seq1) == P.seq + 1 && ld_volatile(&hdr->c) == 2) {
+          atomicExch(P.err, DERR_MISMATCH);
+          break;
+        }
+        if (globaltimer() - t_start > P.timeout_ns) {
+          atomicExch(P.err, DERR_TIMEOUT);
+          break;
+        }
+        __nanosleep(128);
+      }
+      fence_acq_rel_sys();
+    }
+    return;
+  }
+  // A9 step 3: host-ring consumers
+  const uint32_t r = blockIdx.x - 1;
+  if (!wait_word(&hdr->seq1, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
+  if (threadIdx.x == 0) {
+    s_k = ld_volatile(&hdr->c) ? 0 : ld_volatile(&hdr->a);
+    s_q0 = ld_volatile(&hdr->b);
+  }
+  __syncthreads();
+  uint64_t *done = done_at(P.my_ctrl, P.L, P.src);
+  for (uint64_t j = 0; j < s_k; ++j) {
+    const uint64_t q = s_q0 + j, s = q % P.host_slots, u = q / P.host_slots;
+    if (!wait_flags(P.host.full + s * kFlagStride, P.g_host, u + 1, P.timeout_ns, P.err, &s_abort)) return;
+    uint8_t *slot = P.host.data + s * P.host_stride;
+    const uint64_t *h = reinterpret_cast<const uint64_t *>(slot);
+    const uint64_t off = ld_volatile(h + 1), len = ld_volatile(h + 2), shift = ld_volatile(h + 3);
+    uint64_t a, e;
+    slice_of(len, r, P.g_host, &a, &e);
+    if (a < e) group_copy<LD_HOST>(P.my_heap + off + a, slot + kSlotHdr + shift + a, e - a, 0, 1);
+    publish(done, e - a, P.host.freef + s * kFlagStride + r, u + 1);
+  }
+}
+
+// Persistent relay (A8 step 3): CTA group s (g CTAs) forwards sender s's ring.
+__global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constant__ RelayParams P) {
+  __shared__ int s_abort;
+  __shared__ uint64_t s_h[4];
+  if (threadIdx.x == 0) s_abort = 0;
+  __syncthreads();
+  const uint32_t sender = blockIdx.x / P.g, r = blockIdx.x % P.g;
+  if (sender == P.me || sender >= P.world) return;
+  for (uint64_t q = 0;; ++q) {
+    const uint64_t s = q % P.L.slots, u = q / P.L.slots;
+    uint64_t *fl = flags_at(P.my_ctrl, P.L.ring_full, sender, P.L.slots, s);
+    if (!wait_flags(fl, P.g, u + 1, 0, P.err, &s_abort, P.stop)) return;
+    uint8_t *slot = P.my_ctrl + P.L.ring_data + (static_cast<uint64_t>(sender) * P.L.slots + s) * P.L.stride;
+    if (threadIdx.x < 4) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(slot) + threadIdx.x);
+    __syncthreads();
+    const uint32_t dst = static_cast<uint32_t>(s_h[0]);
+    const uint64_t off = s_h[1], len = s_h[2], shift = s_h[3];
+    uint64_t a, e;
+    slice_of(len, r, P.g, &a, &e);
+    if (a < e) group_copy<LD_RING>(P.peer[dst].heap + off + a, slot + kSlotHdr + shift + a, e - a, 0, 1);
+    uint64_t *fr = flags_at(P.peer[sender].ctrl, P.L.relay_free, P.me, P.L.slots, s);
+    publish(done_at(P.peer[dst].ctrl, P.L, sender), e - a, fr + r, u + 1);
+  }
+}
+
 }  // namespace
 
 int launch_xfer(const XferParams &P, void *stream) {
   if (P.nblocks == 0) return cudaSuccess;
-  xfer_kernel<<<P.nblocks, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
+  xfer_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
+  return static_cast<int>(cudaGetLastError());
+}
+
+int launch_send(const SendParams &P, void *stream) {
+  send_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
+  return static_cast<int>(cudaGetLastError());
+}
+
+int launch_recv(const RecvParams &P, void *stream) {
+  recv_kernel<<<P.nblocks, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
+  return static_cast<int>(cudaGetLastError());
+}
+
+int launch_relay(const RelayParams &P, void *stream) {
+  relay_kernel<<<P.world * P.g, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
 }
 
@@ -256,9 +639,26 @@ int launch_pingpong(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *er
   return static_cast<int>(cudaGetLastError());
 }
 
+int preload_kernels() {
+  // CUDA 12 loads kernels lazily, and loading may need a context synchronisation;
+  // with the persistent relay kernel running that would deadlock the first launch of
+  // any other engine kernel.  Force every kernel of this module to load up front.
+  cudaFuncAttributes a;
+  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, relay_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, pingpong_kernel);
+  return static_cast<int>(e);
+}
+
 int xfer_capacity(int device, int *per_sm, int *sms) {
   int n = 0;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xfer_kernel, kThreads, 0);
+  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e != cudaSuccess) return static_cast<int>(e);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xfer_kernel, kThreads, kBulkSmem);
   if (e != cudaSuccess) return static_cast<int>(e);
   int s = 0;
   e = cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, device);

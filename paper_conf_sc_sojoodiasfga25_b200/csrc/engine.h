@@ -50,6 +50,8 @@ struct DevPath {
 struct XferParams {
   uint32_t npaths;
   uint32_t nblocks;
+  uint32_t copy_mode;    // direct group: 0 = LDG/STG vectors, 1 = TMA bulk (cp.async.bulk)
+  uint32_t pad_;
   uint64_t timeout_ns;
   int32_t *err;          // device (or mapped host) error word
   DevPath p[kMaxPaths];
@@ -58,6 +60,110 @@ struct XferParams {
 // Launch the fused transfer kernel (engine.cu).  Returns a cudaError_t value.
 int launch_xfer(const XferParams &P, void *stream);
 
+// ---------------------------------------------------------------- multi-rank engine
+//
+// One process per GPU.  Every rank exports (cudaIpc) its receive heap and its
+// control block; every rank maps every peer's.  A message src → dst:
+//   receiver (mp_recv):  recv kernel CTA 0 posts a CTS entry {seq+1, heap offset,
+//                        bytes, tag} into the sender's control block, then waits for
+//                        its per-src byte counter `done` to reach the target; CTAs
+//                        1.. consume the message's host-ring chunks (A9 step 3).
+//   sender   (mp_send):  send kernel CTAs wait for the CTS, CTA 0 writes the message
+//                        header {seq+1, host_k, host_q0, status} into the receiver's
+//                        control block; the direct group stores into the peer heap
+//                        (A7), stage-in groups fill relay rings (A8 step 1) and the
+//                        host ring (A9 step 1); every byte delivered is counted into
+//                        the receiver's `done` with red.release.sys.
+//   relay    (persistent, one per rank): per sender ring, forward every landed chunk
+//                        to the destination named in the slot header (A8 step 3).
+// Slot = [kSlotHdr-byte header][data]; header = {dst rank, dst heap offset, len, shift}.
+
+constexpr uint32_t kCtsRing = 64;     // outstanding messages per ordered pair
+constexpr uint32_t kSlotHdr = 256;    // slot header bytes
+
+struct MsgEntry {                      // CTS and message-header entries (32 B)
+  uint64_t seq1;                       // sequence + 1 (written last, with release)
+  uint64_t a, b, c;                    // CTS: heap_off, bytes, tag; HDR: host_k, host_q0, status
+};
+
+struct PeerPtrs {
+  uint8_t *heap;                       // peer's receive heap (mapped)
+  uint8_t *ctrl;                       // peer's control block (mapped)
+};
+
+// Byte offsets inside every rank's control block (identical on all ranks).
+struct CtrlLayout {
+  uint32_t world = 0, slots = 0;
+  uint64_t stride = 0;                 // relay slot stride (kSlotHdr + slot_bytes + kSlotSlack)
+  uint64_t cts = 0;                    // [world(src=receiver)][kCtsRing] MsgEntry — on the sender
+  uint64_t hdr = 0;                    // [world(src=sender)][kCtsRing] MsgEntry   — on the receiver
+  uint64_t done = 0;                   // [world(src)] u64, 128-B padded         — on the receiver
+  uint64_t relay_free = 0;             // [world(relay)][slots][kFlagStride]      — on the sender
+  uint64_t ring_full = 0;              // [world(sender)][slots][kFlagStride]     — on the relay
+  uint64_t ring_data = 0;              // [world(sender)][slots][stride]          — on the relay
+  uint64_t total = 0;
+};
+
+// Host ring of one ordered pair (lives in the receiver's shared pinned segment).
+struct HostRingPtrs {
+  uint8_t *data;                       // [slots][host_stride]
+  uint64_t *full;                      // [slots][kFlagStride]
+  uint64_t *freef;                     // [slots][kFlagStride]
+};
+
+struct SendParams {
+  uint32_t me, dst, nblocks, g_direct, g_stage, npaths, copy_mode, pad0_;
+  uint64_t seq, bytes, tag, timeout_ns;
+  const uint8_t *src;
+  uint8_t *my_ctrl;
+  uint8_t *dst_heap;
+  uint8_t *dst_ctrl;
+  int32_t *err;
+  CtrlLayout L;
+  uint64_t host_stride;
+  uint32_t host_slots;
+  uint32_t pad_;
+  struct StagedDesc {
+    int32_t kind;            // 1 relay, 2 host
+    uint32_t relay;          // relay rank
+    uint32_t k;              // chunks
+    uint32_t cta0;           // first block of the stage-in group
+    uint64_t off, bytes;     // message byte range of this path
+    uint64_t q0;             // ring sequence of chunk 0
+    uint8_t *ring_ctrl;      // relay's control block (relay) — full flags + ring data
+  } sp[kMaxPaths];
+  uint64_t direct_bytes;
+  HostRingPtrs host;         // this pair's host ring (mapped)
+};
+
+struct RecvParams {
+  uint32_t me, src, nblocks, g_host;
+  uint64_t seq, bytes, tag, heap_off, done_target, timeout_ns;
+  uint8_t *my_ctrl;
+  uint8_t *my_heap;
+  uint8_t *src_ctrl;
+  int32_t *err;
+  CtrlLayout L;
+  uint64_t host_stride;
+  uint32_t host_slots;
+  uint32_t pad_;
+  HostRingPtrs host;
+};
+
+struct RelayParams {
+  uint32_t me, world, g;       // g CTAs per sender ring
+  uint32_t pad_;
+  uint8_t *my_ctrl;
+  PeerPtrs peer[kMaxPaths];    // heap/ctrl of every rank (self: local)
+  CtrlLayout L;
+  volatile int32_t *stop;      // mapped host word: != 0 → exit
+  int32_t *err;
+};
+
+int launch_send(const SendParams &P, void *stream);
+int launch_recv(const RecvParams &P, void *stream);
+int launch_relay(const RelayParams &P, void *stream);
+
 // Calibration probes (engine.cu).
 // Flag ping-pong between two CTAs through `flags` (2 words, device or mapped host):
 // `iters` round trips; the measured time is read with events by the caller.
@@ -65,5 +171,8 @@ int launch_pingpong(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *er
 
 // Max co-resident CTAs of the transfer kernel on this device (occupancy × SMs).
 int xfer_capacity(int device, int *per_sm, int *sms);
+
+// Load every engine kernel now (no lazy loading once persistent kernels run).
+int preload_kernels();
 
 }  // namespace mpx

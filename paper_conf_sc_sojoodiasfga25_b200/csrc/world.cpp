@@ -1,0 +1,377 @@
+// world.cpp — multi-rank engine host side (one process per GPU).
+//
+// Bootstrap (§2.1: UCX cuda_ipc exchanges and caches IPC handles;
+// here the exchange is one all-gather at mp_init): every rank exports its receive
+// heap and control block with cudaIpcGetMemHandle and maps every peer's; every rank
+// creates a POSIX shared-memory segment holding the pinned host rings of the
+// messages it receives (A9), registered mapped+portable so both the sending and the
+// receiving GPU address it; ranks >= 3 launch the persistent relay kernel (A8).
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <random>
+#include <string>
+#include <vector>
+
+#include "ctx.h"
+
+namespace mpx {
+
+namespace {
+
+int wfail(mp_ctx *c, int code, const std::string &msg) {
+  c->last_error = msg;
+  return code;
+}
+
+#define CKW(call)                                                                                 \
+  do {                                                                                            \
+    cudaError_t e__ = (call);                                                                     \
+    if (e__ != cudaSuccess) return wfail(c, MP_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e__)); \
+  } while (0)
+
+struct RankInfo {
+  cudaIpcMemHandle_t heap;
+  cudaIpcMemHandle_t ctrl;
+  uint64_t jobid;
+  uint64_t heap_bytes;
+  int32_t device;
+  int32_t relay_ctas;
+  uint64_t slot_bytes;
+  int32_t slots;
+  int32_t host_path;
+};
+
+int allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes) {
+  if (!c->allgather) return wfail(c, MP_ERR_INVALID, "world > 1 needs an allgather callback");
+  if (c->allgather(c->allgather_user, in, out, bytes) != 0)
+    return wfail(c, MP_ERR_INVALID, "bootstrap all-gather failed");
+  return MP_OK;
+}
+
+int barrier(mp_ctx *c) {
+  std::vector<uint8_t> out(c->world);
+  uint8_t one = 1;
+  return allgather(c, &one, out.data(), 1);
+}
+
+CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
+  CtrlLayout L;
+  L.world = world;
+  L.slots = slots;
+  L.stride = kSlotHdr + slot_bytes + kSlotSlack;
+  uint64_t off = 0;
+  auto take = [&](uint64_t bytes) {
+    const uint64_t o = off;
+    off = (off + bytes + 255) & ~uint64_t(255);
+    return o;
+  };
+  L.cts = take(static_cast<uint64_t>(world) * kCtsRing * sizeof(MsgEntry));
+  L.hdr = take(static_cast<uint64_t>(world) * kCtsRing * sizeof(MsgEntry));
+  L.done = take(static_cast<uint64_t>(world) * 128);
+  L.relay_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
+  L.ring_full = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
+  L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
+  L.total = off;
+  return L;
+}
+
+std::string seg_name(uint64_t jobid, int rank) {
+  char b[64];
+  std::snprintf(b, sizeof(b), "/mpx_%016llx_%d", static_cast<unsigned long long>(jobid), rank);
+  return b;
+}
+
+int map_segment(mp_ctx *c, int rank, bool create, uint8_t **out) {
+  const std::string name = seg_name(c->jobid, rank);
+  const int fd = shm_open(name.c_str(), create ? (O_CREAT | O_EXCL | O_RDWR) : O_RDWR, 0600);
+  if (fd < 0) return wfail(c, MP_ERR_NOMEM, "shm_open " + name + " failed");
+  if (create && ftruncate(fd, static_cast<off_t>(c->hseg_bytes)) != 0) {
+    close(fd);
+    return wfail(c, MP_ERR_NOMEM, "ftruncate " + name + " failed");
+  }
+  void *p = mmap(nullptr, c->hseg_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  if (p == MAP_FAILED) return wfail(c, MP_ERR_NOMEM, "mmap " + name + " failed");
+  if (create) std::memset(p, 0, c->hseg_bytes);
+  cudaError_t e = cudaHostRegister(p, c->hseg_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+  if (e != cudaSuccess) {
+    munmap(p, c->hseg_bytes);
+    return wfail(c, MP_ERR_CUDA, std::string("cudaHostRegister: ") + cudaGetErrorString(e));
+  }
+  void *d = nullptr;
+  CKW(cudaHostGetDevicePointer(&d, p, 0));
+  if (d != p) return wfail(c, MP_ERR_UNSUPPORTED, "mapped host pointer differs from its device pointer (no UVA)");
+  *out = static_cast<uint8_t *>(p);
+  return MP_OK;
+}
+
+HostRingPtrs host_ring(const mp_ctx *c, int src, int dst) {
+  uint8_t *base = c->hseg[dst] + static_cast<uint64_t>(src) * c->hseg_per_src;
+  HostRingPtrs h;
+  h.data = base;
+  h.full = reinterpret_cast<uint64_t *>(base + static_cast<uint64_t>(c->slots) * c->host_stride);
+  h.freef = h.full + static_cast<uint64_t>(c->slots) * kFlagStride;
+  return h;
+}
+
+}  // namespace
+
+static bool debug_on() {
+  const char *d = std::getenv("MPX_DEBUG");
+  return d && d[0] == '1';
+}
+
+#define DBG(msg)                                                          \
+  do {                                                                    \
+    if (debug_on()) std::fprintf(stderr, "[mpx %d] %s\n", c->rank, msg); \
+  } while (0)
+
+int world_init(mp_ctx *c) {
+  DBG("world_init begin");
+  CKW(cudaSetDevice(c->device));
+  const int W = c->world;
+  c->L = layout(W, c->slots, c->slot_bytes);
+  void *p = nullptr;
+  CKW(cudaMalloc(&p, c->L.total));
+  c->ctrl = static_cast<uint8_t *>(p);
+  CKW(cudaMemset(c->ctrl, 0, c->L.total));
+
+  RankInfo me;
+  std::memset(&me, 0, sizeof(me));
+  CKW(cudaIpcGetMemHandle(&me.heap, c->heap.base));
+  CKW(cudaIpcGetMemHandle(&me.ctrl, c->ctrl));
+  me.jobid = std::random_device{}() ^ (static_cast<uint64_t>(std::random_device{}()) << 32) ^
+             static_cast<uint64_t>(getpid());
+  me.heap_bytes = c->heap.size;
+  me.device = c->device;
+  me.relay_ctas = c->relay_ctas;
+  me.slot_bytes = c->slot_bytes;
+  me.slots = c->slots;
+  me.host_path = c->host_path ? 1 : 0;
+  std::vector<RankInfo> all(W);
+  if (int s = allgather(c, &me, all.data(), sizeof(RankInfo))) return s;
+  c->jobid = all[0].jobid;
+  for (int r = 0; r < W; ++r)
+    if (all[r].relay_ctas != c->relay_ctas || all[r].slot_bytes != c->slot_bytes ||
+        all[r].slots != c->slots || all[r].host_path != me.host_path)
+      return wfail(c, MP_ERR_INVALID, "ranks disagree on slots / slot_bytes / relay_ctas / host_path");
+
+  DBG("rank info exchanged");
+  c->peers.assign(W, PeerPtrs{nullptr, nullptr});
+  for (int r = 0; r < W; ++r) {
+    if (r == c->rank) {
+      c->peers[r] = PeerPtrs{c->heap.base, c->ctrl};
+      continue;
+    }
+    void *h = nullptr, *k = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&h, all[r].heap, cudaIpcMemLazyEnablePeerAccess);
+    if (e == cudaSuccess) e = cudaIpcOpenMemHandle(&k, all[r].ctrl, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess)
+      return wfail(c, MP_ERR_TOPOLOGY, "cannot map rank " + std::to_string(r) + "'s memory: " + cudaGetErrorString(e));
+    c->peers[r] = PeerPtrs{static_cast<uint8_t *>(h), static_cast<uint8_t *>(k)};
+  }
+
+  // Host rings: one segment per receiving rank, one ring per sender inside it.
+  c->host_stride = kSlotHdr + c->slot_bytes + kSlotSlack;
+  c->hseg_per_src = (static_cast<uint64_t>(c->slots) * c->host_stride +
+                     2ull * c->slots * kFlagStride * 8 + 4095) & ~uint64_t(4095);
+  c->hseg_bytes = static_cast<size_t>(c->hseg_per_src * W);
+  c->hseg.assign(W, nullptr);
+  if (c->host_path) {
+    if (int s = map_segment(c, c->rank, true, &c->hseg[c->rank])) return s;
+    if (int s = barrier(c)) return s;
+    for (int r = 0; r < W; ++r)
+      if (r != c->rank)
+        if (int s = map_segment(c, r, false, &c->hseg[r])) return s;
+    if (int s = barrier(c)) return s;
+    shm_unlink(seg_name(c->jobid, c->rank).c_str());
+  }
+
+  DBG("ipc + host segments mapped");
+  c->send_seq.assign(W, 0);
+  c->recv_seq.assign(W, 0);
+  c->relay_q.assign(W, 0);
+  c->host_q.assign(W, 0);
+  c->done_target.assign(W, 0);
+
+  const char *no_relay = std::getenv("MPX_NO_RELAY");  // diagnostics: no relay kernel
+  if (W >= 3 && !(no_relay && no_relay[0] == '1')) {  // the persistent relay kernel
+    CKW(cudaHostAlloc(&p, 64, cudaHostAllocMapped | cudaHostAllocPortable));
+    c->stop = static_cast<int32_t *>(p);
+    *c->stop = 0;
+    DBG("stop word allocated");
+    CKW(cudaStreamCreateWithFlags(&c->relay_stream, cudaStreamNonBlocking));
+    DBG("relay stream created");
+    RelayParams R{};
+    R.me = static_cast<uint32_t>(c->rank);
+    R.world = static_cast<uint32_t>(W);
+    R.g = static_cast<uint32_t>(c->relay_ctas);
+    R.my_ctrl = c->ctrl;
+    for (int r = 0; r < W; ++r) R.peer[r] = c->peers[r];
+    R.L = c->L;
+    R.stop = c->stop;
+    R.err = c->d_err;
+    if (int e = launch_relay(R, c->relay_stream))
+      return wfail(c, MP_ERR_CUDA, std::string("relay launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+    c->launches += 1;
+    c->relay_running = true;
+  }
+  DBG("relay launched");
+  const int s = barrier(c);
+  DBG("world_init done");
+  return s;
+}
+
+int world_finalize(mp_ctx *c) {
+  int st = MP_OK;
+  if (c->relay_running) {
+    *reinterpret_cast<volatile int32_t *>(c->stop) = 1;
+    cudaStreamSynchronize(c->relay_stream);
+    c->relay_running = false;
+  }
+  for (cudaStream_t s : c->streams) cudaStreamSynchronize(s);
+  if (c->allgather) st = barrier(c);
+  for (int r = 0; r < static_cast<int>(c->peers.size()); ++r) {
+    if (r == c->rank) continue;
+    if (c->peers[r].heap) cudaIpcCloseMemHandle(c->peers[r].heap);
+    if (c->peers[r].ctrl) cudaIpcCloseMemHandle(c->peers[r].ctrl);
+  }
+  c->peers.clear();
+  for (uint8_t *s : c->hseg)
+    if (s) {
+      cudaHostUnregister(s);
+      munmap(s, c->hseg_bytes);
+    }
+  c->hseg.clear();
+  if (c->relay_stream) cudaStreamDestroy(c->relay_stream);
+  c->relay_stream = nullptr;
+  if (c->stop) cudaFreeHost(c->stop);
+  c->stop = nullptr;
+  if (c->ctrl) cudaFree(c->ctrl);
+  c->ctrl = nullptr;
+  return st;
+}
+
+static void note_stream(mp_ctx *c, cudaStream_t s) {
+  if (std::find(c->streams.begin(), c->streams.end(), s) == c->streams.end()) c->streams.push_back(s);
+}
+
+int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,
+               void *stream) {
+  SendParams P{};
+  P.me = static_cast<uint32_t>(c->rank);
+  P.dst = static_cast<uint32_t>(dst);
+  P.seq = c->send_seq[dst];
+  P.bytes = bytes;
+  P.tag = static_cast<uint64_t>(static_cast<int64_t>(tag));
+  P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  P.src = static_cast<const uint8_t *>(buf);
+  P.my_ctrl = c->ctrl;
+  P.dst_heap = c->peers[dst].heap;
+  P.dst_ctrl = c->peers[dst].ctrl;
+  P.err = c->d_err;
+  P.L = c->L;
+  P.host_stride = c->host_stride;
+  P.host_slots = static_cast<uint32_t>(c->slots);
+  P.g_stage = static_cast<uint32_t>(c->relay_ctas);
+  P.copy_mode = c->copy_mode;
+  if (c->host_path) P.host = host_ring(c, c->rank, dst);
+  P.direct_bytes = cfg.bytes[0];
+  const int cap = std::max(1, c->per_sm * c->sms);
+  uint32_t staged = 0;
+  for (int i = 1; i < cfg.npaths; ++i)
+    if (cfg.bytes[i]) staged += P.g_stage;
+  const uint64_t want = std::max<uint64_t>(1, (cfg.bytes[0] + (32u << 10) - 1) / (32u << 10));
+  P.g_direct = static_cast<uint32_t>(
+      std::min<uint64_t>(want, static_cast<uint64_t>(std::max(1, std::min(cap - static_cast<int>(staged), 2 * c->sms)))));
+  uint32_t next = P.g_direct;
+  uint64_t off = cfg.bytes[0];
+  uint32_t np = 0;
+  std::vector<std::pair<int, uint32_t>> advance;
+  for (int i = 1; i < cfg.npaths; ++i) {
+    const uint64_t b = cfg.bytes[i];
+    if (b) {
+      SendParams::StagedDesc &d = P.sp[np++];
+      d.kind = cfg.path[i].kind == MP_PATH_HOST ? 2 : 1;
+      d.relay = d.kind == 1 ? static_cast<uint32_t>(cfg.path[i].via) : 0u;
+      d.k = cfg.chunks[i];
+      d.cta0 = next;
+      next += P.g_stage;
+      d.off = off;
+      d.bytes = b;
+      if (d.kind == 1) {
+        d.q0 = c->relay_q[d.relay];
+        d.ring_ctrl = c->peers[d.relay].ctrl;
+        advance.emplace_back(static_cast<int>(d.relay), d.k);
+      } else {
+        d.q0 = c->host_q[dst];
+        advance.emplace_back(-1, d.k);
+      }
+    }
+    off += b;
+  }
+  P.npaths = np;
+  P.nblocks = next;
+  if (int e = launch_send(P, stream))
+    return wfail(c, MP_ERR_CUDA, std::string("send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  c->launches += 1;
+  c->send_seq[dst] += 1;
+  for (auto &a : advance) {
+    if (a.first < 0)
+      c->host_q[dst] += a.second;
+    else
+      c->relay_q[a.first] += a.second;
+  }
+  note_stream(c, static_cast<cudaStream_t>(stream));
+  return MP_OK;
+}
+
+int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
+  uint8_t *b = static_cast<uint8_t *>(buf);
+  if (bytes && (b < c->heap.base || b + bytes > c->heap.base + c->heap.size))
+    return wfail(c, MP_ERR_INVALID, "mp_recv buffer must come from mp_alloc when world > 1");
+  RecvParams P{};
+  P.me = static_cast<uint32_t>(c->rank);
+  P.src = static_cast<uint32_t>(src);
+  P.seq = c->recv_seq[src];
+  P.bytes = bytes;
+  P.tag = static_cast<uint64_t>(static_cast<int64_t>(tag));
+  P.heap_off = bytes ? static_cast<uint64_t>(b - c->heap.base) : 0;
+  P.done_target = c->done_target[src] + bytes;
+  P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  P.my_ctrl = c->ctrl;
+  P.my_heap = c->heap.base;
+  P.src_ctrl = c->peers[src].ctrl;
+  P.err = c->d_err;
+  P.L = c->L;
+  P.host_stride = c->host_stride;
+  P.host_slots = static_cast<uint32_t>(c->slots);
+  P.g_host = c->host_path ? static_cast<uint32_t>(c->relay_ctas) : 0u;
+  if (c->host_path) P.host = host_ring(c, src, c->rank);
+  P.nblocks = 1 + P.g_host;
+  if (int e = launch_recv(P, stream))
+    return wfail(c, MP_ERR_CUDA, std::string("recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  c->launches += 1;
+  c->recv_seq[src] += 1;
+  c->done_target[src] += bytes;
+  note_stream(c, static_cast<cudaStream_t>(stream));
+  return MP_OK;
+}
+
+int world_sync(mp_ctx *c) {
+  // Never cudaDeviceSynchronize here: the persistent relay kernel never ends.
+  for (cudaStream_t s : c->streams) CKW(cudaStreamSynchronize(s));
+  int32_t e = 0;
+  CKW(cudaMemcpy(&e, c->d_err, sizeof(e), cudaMemcpyDeviceToHost));
+  if (e == DERR_TIMEOUT) return wfail(c, MP_ERR_TIMEOUT, "a device-side wait timed out");
+  if (e == DERR_MISMATCH) return wfail(c, MP_ERR_MISMATCH, "send/recv size or tag mismatch");
+  return MP_OK;
+}
+
+}  // namespace mpx

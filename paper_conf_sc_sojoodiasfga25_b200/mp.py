@@ -179,6 +179,10 @@ class Context:
         self.close()
 
     def __del__(self):
+        # a multi-rank context's mp_finalize is collective: it cannot run from a
+        # garbage-collection finaliser (other ranks may be gone); call close() instead.
+        if getattr(self, "world", 1) > 1:
+            return
         try:
             self.close()
         except Exception:
@@ -281,3 +285,17 @@ class Context:
         v = C.c_uint64()
         self._ck(lib().mp_stats(self.h, C.byref(v)))
         return v.value
+
+
+class _CudaArray:
+    """Minimal __cuda_array_interface__ holder (zero-copy view of device memory)."""
+
+    def __init__(self, ptr: int, n: int):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (ptr, False),
+                                         "version": 3, "strides": None}
+
+
+def as_tensor(ptr: int, n: int):
+    """A torch uint8 tensor viewing n bytes of device memory at ptr (e.g. from mp_alloc)."""
+    import torch
+    return torch.as_tensor(_CudaArray(ptr, n), device="cuda")

@@ -1,0 +1,154 @@
+"""Worker for the multi-rank tests (one process per rank; all ranks may share one GPU).
+
+    python tests/_world_worker.py <rank> <world> <port> <scenario>
+
+Scenario "gloo_model" (CPU): model-only contexts bootstrapped over gloo; every rank
+selects the same configs and the all-gather callback round-trips.
+Scenario "engine" (GPU): real multi-rank engine — IPC-mapped heaps, the persistent
+relay kernel, the shared pinned host ring — with rank 0 → rank 1 messages over every
+path kind, checked byte for byte against the oracle reference transfer.
+"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import ctypes  # noqa: E402
+
+import torch  # noqa: E402
+import torch.distributed as dist  # noqa: E402
+
+MiB = 1 << 20
+
+
+def scenario_gloo_model(rank, world):
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    ag = mdist.torch_allgather()
+    inp = bytes([rank + 1] * 8)
+    out = ctypes.create_string_buffer(8 * world)
+    assert ag(None, inp, ctypes.addressof(out), 8) == 0
+    assert out.raw == b"".join(bytes([r + 1] * 8) for r in range(world))
+    c = mdist.context_from_dist(model_only=True)
+    assert c.world == world and c.rank == rank
+    cfgs = []
+    for dst in range(world):
+        if dst == rank:
+            continue
+        d = c.select(rank, dst, 256 * MiB).as_dict()
+        assert sum(d["bytes"]) == 256 * MiB
+        assert len(d["paths"]) == world  # direct + (world-2) relays + host
+        cfgs.append((rank, dst, d["bytes"], d["chunks"]))
+    # every rank computes the same selection for the same pair (pure function of the model)
+    gathered = [None] * world
+    dist.all_gather_object(gathered, c.select(0, 1, 64 * MiB).as_dict())
+    assert all(g == gathered[0] for g in gathered)
+    c.close()
+
+
+def scenario_engine(rank, world):
+    import numpy as np
+
+    import synth
+    from oracle import transfer as X
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    # Everything CUDA this process will need is initialised BEFORE mp_init: with
+    # world >= 3 the persistent relay kernel runs from then on, and driver calls that
+    # need an idle context (lazy module loading, torch's lazy init, first-use pools)
+    # would wait for it forever.
+    stream = torch.cuda.Stream()
+    src_buf = torch.empty(8 * MiB, dtype=torch.uint8, device="cuda")
+    src_buf.copy_(torch.from_numpy(synth.payload(8 * MiB, 0)))
+    assert int(src_buf[:16].cpu().sum()) >= 0
+    torch.cuda.synchronize()
+    print(f"rank {rank}: init", flush=True)
+    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                timeout_s=60.0)
+    ps = c.paths(0, 1)
+    np_ = len(ps)
+    cases = []
+    n = 3 * MiB + 4099
+    cases.append(([n] + [0] * (np_ - 1), [1] + [0] * (np_ - 1), n))                 # direct only
+    relay_ok = os.environ.get("MPX_NO_RELAY") != "1"
+    if world >= 3 and relay_ok:
+        nb = [0] * np_
+        nb[1] = n                                                               # one relay alone, k = 5
+        ks = [1] + [0] * (np_ - 1)
+        ks[1] = 5
+        cases.append((nb, ks, n))
+    nb = [0] * np_
+    nb[-1] = n                                                                  # host path alone, k = 4
+    ks = [1] + [0] * (np_ - 1)
+    ks[-1] = 4
+    cases.append((nb, ks, n))
+    nb = [0] + [256 * 1024 if (relay_ok or k == 2) else 0 for k, _ in ps[1:]]      # every path at once
+    nb[0] = n - sum(nb)
+    cases.append((nb, [1] + [2 if b else 0 for b in nb[1:]], n))
+    if relay_ok:
+        cases.append((None, None, 5 * MiB + 1))                                 # model-selected
+    else:
+        d = c.select(0, 1, 5 * MiB + 1, 1 | (1 << (np_ - 1))).as_dict()
+        cases.append((d["bytes"], d["chunks"], 5 * MiB + 1))
+    print(f"rank {rank}: context up, {len(cases)} cases", flush=True)
+    for i, (nb, ks, n) in enumerate(cases):
+        print(f"rank {rank}: case {i} {nb} {ks}", flush=True)
+        if rank == 0:
+            host = synth.payload(n, i)
+            src = src_buf[:n]
+            src.copy_(torch.from_numpy(host))
+            cfg = c.make_config(nb, ks, 0, 1) if nb else None
+            c.send(src, n, 1, tag=100 + i, cfg=cfg, stream=stream)
+            stream.synchronize()
+        elif rank == 1:
+            p = c.alloc(n)
+            c.recv(p, n, 0, tag=100 + i, stream=stream)
+            stream.synchronize()
+            got = mp.as_tensor(p, n)
+            host = synth.payload(n, i)
+            exp = np.zeros(n, dtype=np.uint8)
+            if nb:
+                X.replay(host, nb, ks, [k for k, _ in ps], 256, exp)
+            else:
+                exp[:] = host
+            assert np.array_equal(got.cpu().numpy(), exp), f"case {i} mismatch"
+            c.free(p)
+        dist.barrier()
+    # the reverse direction and a tag mismatch are reported, not hung
+    if rank == 1:
+        src = src_buf[:MiB]
+        src.copy_(torch.from_numpy(synth.payload(MiB, 9)))
+        c.send(src, MiB, 0, tag=5, stream=stream)
+        stream.synchronize()
+    elif rank == 0:
+        p = c.alloc(MiB)
+        c.recv(p, MiB, 1, tag=5, stream=stream)
+        stream.synchronize()
+        c.sync()
+        c.free(p)
+    dist.barrier()
+    c.sync()
+    assert c.launches() > 0 or rank >= 2
+    c.close()
+
+
+def main():
+    rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
+    try:
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+        {"gloo_model": scenario_gloo_model, "engine": scenario_engine}[scen](rank, world)
+        dist.barrier()
+        dist.destroy_process_group()
+    except BaseException:
+        import traceback
+        traceback.print_exc()
+        sys.stdout.flush()
+        sys.stderr.flush()
+        os._exit(1)  # skip interpreter teardown (no collective finalisers at exit)
+    print(f"rank {rank} ok", flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,62 @@
+"""Multi-rank paths: world_size-2/3 process groups over gloo on 127.0.0.1.
+
+CPU: the bootstrap all-gather and the per-pair model selection are consistent
+across ranks.  GPU: the real multi-rank engine (IPC-mapped heaps, persistent relay
+kernel, shared pinned host ring) with all ranks on one B200 (same-device CUDA IPC),
+bit-exact against the oracle's reference transfer."""
+import os
+import socket
+import subprocess
+import sys
+
+import pytest
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def run_world(world, scenario, timeout):
+    port = free_port()
+    procs = [subprocess.Popen([sys.executable, os.path.join(HERE, "_world_worker.py"), str(r), str(world),
+                               str(port), scenario], stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)
+             for r in range(world)]
+    outs = []
+    try:
+        for p in procs:
+            out, _ = p.communicate(timeout=timeout)
+            outs.append(out)
+    except subprocess.TimeoutExpired:
+        for p in procs:
+            if p.poll() is None:
+                p.kill()
+        tails = [p.communicate()[0][-2000:] for p in procs]
+        raise AssertionError("timed out; per-rank output tails:\n" +
+                             "\n".join(f"--- rank {r}\n{t}" for r, t in enumerate(tails)))
+    finally:
+        for p in procs:
+            if p.poll() is None:
+                p.kill()
+    for r, (p, out) in enumerate(zip(procs, outs)):
+        assert p.returncode == 0, f"rank {r} failed:\n{out[:3000]}\n...\n{out[-3000:]}"
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_bootstrap_and_consistent_selection(world):
+    run_world(world, "gloo_model", timeout=240)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 3])
+def test_multirank_engine_same_gpu(world):
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(world, "engine", timeout=400)
