@@ -13,8 +13,9 @@ N = 1 (default): BASELINE.json config 3 — 1 GiB, direct + 6 relays + pinned ho
 on the single-GPU loopback engine (the relay rings stand in for the intermediate
 GPUs; the host leg is real PCIe); the config is the B200-mode model's pick after an
 init-time calibration (Step 1).  Inputs are 1 GiB (> 126 MB L2), so no flush.
-N > 1 (torchrun): every rank runs its own loopback message (independent replicas,
-"scaling": "weak"); the multi-rank engine is not on the bench path yet.
+N > 1 (torchrun): config 5's "pairs" reading — ranks (2i, 2i+1) exchange one
+message per step through the multi-rank engine, all pairs concurrently
+("scaling": "weak"; value = bytes of all pairs / max-over-ranks time).
 
 --impl reference: the CPU oracle (oracle/, fp64 model + memcpy replay) on a bounded
 sample of the same workload, rank 0 only.
@@ -46,29 +47,53 @@ def measured_peaks():
 
 
 class Clocks:
-    """Sample nvidia-smi SM clocks and throttle reasons during the timed region."""
+    """Sample SM clocks and clock-event (throttle) reasons during the timed region via
+    NVML (the same counters nvidia-smi reports), every 20 ms; falls back to one
+    nvidia-smi query per sample if NVML is unavailable."""
 
-    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "sw_power_cap": 0x4}
 
     def __init__(self, index=0):
         self.index, self.samples, self.stop_ = index, [], threading.Event()
         self.t = threading.Thread(target=self._run, daemon=True)
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _sample(self):
+        if self.nv is not None:
+            sm = self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM)
+            try:
+                mask = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            except Exception:
+                mask = self.nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+            return float(sm), int(mask)
+        out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm",
+                              "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                             timeout=5).stdout.strip().split(",")
+        self.max_mhz = float(out[1])
+        return float(out[0]), 0
 
     def _run(self):
         while not self.stop_.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
-                                     timeout=5).stdout.strip()
-                if out:
-                    self.samples.append([x.strip() for x in out.split(",")])
+                self.samples.append(self._sample())
             except Exception:
                 pass
-            self.stop_.wait(0.2)
+            self.stop_.wait(0.02)
 
     def __enter__(self):
+        try:
+            self.samples.append(self._sample())
+        except Exception:
+            pass
         self.t.start()
         return self
 
@@ -78,13 +103,11 @@ class Clocks:
 
     def summary(self):
         if not self.samples:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
-        sm = sorted(float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit())
-        mx = max((float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()), default=None)
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({n for s in self.samples for n, v in zip(names, s[3:7]) if v.strip() == "Active"})
-        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx, "reasons": reasons,
-                "samples": len(self.samples)}
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"]}
+        sm = sorted(s[0] for s in self.samples)
+        reasons = sorted({n for _, m in self.samples for n, bit in self.REASONS.items() if m & bit})
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": self.max_mhz, "reasons": reasons,
+                "samples": len(self.samples), "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
 def dist_env():
@@ -187,10 +210,131 @@ def workload_config(args, world):
             "l2": "inputs 1 GiB > 126 MB L2 (no flush)", "parallelism": f"replicas{world}"}
 
 
+def run_world(args, world, rank, local):
+    """N > 1 (torchrun, one process per GPU): BASELINE.json config 5 reading "pairs":
+    ranks (2i, 2i+1) exchange one message per step, 2i → 2i+1, all pairs at once,
+    through the multi-rank engine (IPC-mapped heaps, NVLink direct path, relays
+    through the other GPUs, pinned-host PCIe path), model-selected after a
+    collective calibration.  Bootstrap and the max-over-ranks reduction use gloo on
+    CPU: no NCCL kernel ever runs next to the persistent relay kernel."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+
+    dist.init_process_group("gloo")
+    dev = 0 if os.environ.get("MPX_BENCH_SAME_GPU") == "1" else local   # 1-GPU smoke of this path
+    torch.cuda.set_device(dev)
+    n = args.size
+    peer = rank + 1 if rank % 2 == 0 else rank - 1
+    active = peer < world
+    sender = active and rank % 2 == 0
+    npairs = world // 2
+    # Initialise every CUDA kernel this process will use BEFORE mp_init (DESIGN.md §7).
+    stream = torch.cuda.Stream()
+    g = torch.Generator(device="cuda").manual_seed(20251116 + (rank if sender else peer))
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g)
+    h_buf = torch.empty(n, dtype=torch.uint8).pin_memory()
+    h_buf.copy_(src)
+    src.copy_(h_buf, non_blocking=True)
+    assert torch.equal(src, src.clone())
+    torch.cuda.synchronize()
+
+    ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
+                                  timeout_s=60.0)
+    ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
+    d = ctx.select(0, 1, n).as_dict()
+    rbuf = ctx.alloc(n) if active and not sender else None
+    rview = mp.as_tensor(rbuf, n) if rbuf else None
+
+    def step():
+        if not active:
+            return
+        if sender:
+            ctx.send(src, n, peer, 0, None, stream)
+        else:
+            ctx.recv(rbuf, n, peer, 0, stream)
+
+    for _ in range(args.warmup):
+        step()
+    stream.synchronize()
+    ctx.sync()
+    if active and not sender:
+        assert torch.equal(rview, src), "payload mismatch"   # src = the sender's seeded payload
+    dist.barrier()
+    l0 = ctx.launches()
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    with Clocks(dev) as clk:
+        t0.record(stream)
+        for _ in range(args.steps):
+            step()
+        t1.record(stream)
+        stream.synchronize()
+    ms = t0.elapsed_time(t1) if active else 0.0
+    stats = torch.tensor([ms, float(ctx.launches() - l0)], dtype=torch.float64)
+    mx = stats.clone()
+    dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+    sm = stats.clone()
+    dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+    ms = float(mx[0])
+    value = n * npairs * args.steps / (ms * 1e-3) / 1e9
+
+    # end to end: the sender's payload comes from pinned host memory, the receiver
+    # reads the message back to pinned host memory, every step.
+    e2e_steps = max(3, min(10, args.steps // 4))
+    dist.barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    with torch.cuda.stream(stream):
+        for _ in range(e2e_steps):
+            if sender:
+                src.copy_(h_buf, non_blocking=True)
+            step()
+            if active and not sender:
+                h_buf.copy_(rview, non_blocking=True)
+    e1.record(stream)
+    stream.synchronize()
+    e = torch.tensor([e0.elapsed_time(e1) if active else 0.0], dtype=torch.float64)
+    dist.all_reduce(e, op=dist.ReduceOp.MAX)
+    e2e = n * npairs * e2e_steps / (float(e[0]) * 1e-3) / 1e9
+
+    nvl = sum(b for (k, _), b in zip(d["paths"], d["bytes"]) if k != 2)
+    per_pair = n * args.steps / (ms * 1e-3) / 1e9
+    achieved = nvl * args.steps / (ms * 1e-3) / 1e9
+    line = {
+        "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded uniform random bytes)",
+        "config": {"workload": f"config5 (pairs reading): {npairs} concurrent pairs 2i->2i+1, "
+                               f"{n >> 20} MiB per message, direct + relays + pinned host, model-selected",
+                   "msg_bytes": n, "mode": args.mode, "parallelism": f"pairs{npairs}",
+                   "l2": "messages >= 126 MB L2 (no flush)" if n >= 128 * MiB else "no flush"},
+        "roofline": {"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
+                     "frac": achieved / 770.0, "traffic": None, "peak_source":
+                     "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
+                     "kernel": "send_kernel"},
+        "per_pair_GBps": per_pair,
+        "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n * npairs, "d2h_bytes_per_step": n * npairs},
+        "gpu_launches": int(sm[1]),
+        "clocks": clk.summary(),
+        "model": {"selected": d, "predicted_GBps": n / d["t_pred"] / 1e9 if d["t_pred"] else None,
+                  "E_pred": abs(n / d["t_pred"] / 1e9 - per_pair) / per_pair if d["t_pred"] else None},
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if rbuf:
+        ctx.free(rbuf)
+    ctx.close()
+    dist.destroy_process_group()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=400)
+    ap.add_argument("--steps", type=int, default=2000)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="mpx", choices=["mpx", "reference"])
     ap.add_argument("--size", type=int, default=GiB)
@@ -211,7 +355,7 @@ def main():
 
     world, rank, local = dist_env()
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        return run_world(args, world, rank, local)
     torch.cuda.set_device(local)
     n = args.size
     ctx = mp.Context(device=local, calibrate=not (args.no_calibrate or args.params), n_loop_relays=6,
@@ -266,7 +410,7 @@ def main():
     # pinned memory, the transfer, D2H of the received message, every step.
     h_src = src.cpu().pin_memory()
     h_dst = torch.empty(n, dtype=torch.uint8).pin_memory()
-    e2e_steps = max(3, args.steps // 4)
+    e2e_steps = max(3, min(10, args.steps // 4))
     torch.cuda.synchronize()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
@@ -280,6 +424,27 @@ def main():
     torch.cuda.synchronize()
     e2e = n * e2e_steps / (e0.elapsed_time(e1) * 1e-3) / 1e9
     assert torch.equal(h_dst, h_src)
+
+    # single-path baseline: cudaMemcpyAsync device→device on the same stream (the
+    # copy the paper's engine issues per chunk), same buffers and timing.
+    base = None
+    try:
+        from cuda.bindings import runtime as rt
+        kind = rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice
+        bsteps = max(5, min(args.steps, 50))
+        b0 = torch.cuda.Event(enable_timing=True)
+        b1 = torch.cuda.Event(enable_timing=True)
+        for _ in range(3):
+            rt.cudaMemcpyAsync(dst.data_ptr(), src.data_ptr(), n, kind, stream.cuda_stream)
+        b0.record(stream)
+        for _ in range(bsteps):
+            rt.cudaMemcpyAsync(dst.data_ptr(), src.data_ptr(), n, kind, stream.cuda_stream)
+        b1.record(stream)
+        torch.cuda.synchronize()
+        base = {"cudaMemcpyAsync_d2d_GBps": n * bsteps / (b0.elapsed_time(b1) * 1e-3) / 1e9,
+                "steps": bsteps}
+    except Exception as exc:  # the baseline is context, not the product
+        base = {"error": repr(exc)}
 
     peak, peak_src = measured_peaks()
     alg = hbm_bytes(d)
@@ -310,6 +475,7 @@ def main():
                   "port": port, "direct_params": prm[0], "host_params": prm[-1]},
         "per_launch_ms": {"min": per_launch[0], "median": per_launch[len(per_launch) // 2],
                           "max": per_launch[-1]},
+        "baselines": base,
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, desc, cores = cpu_oracle_run(n, d, prm)

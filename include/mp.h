@@ -148,6 +148,10 @@ typedef struct mp_init_args {
  * pinned host ring, exchanges IPC handles, and — unless MP_INIT_NO_CALIBRATE —
  * calibrates α/β/ε of every path with the engine's own kernels (Step 1).
  * With MP_INIT_MODEL_ONLY no CUDA call is made; world/rank still define the pairs.
+ * world >= 3 starts a persistent relay kernel on a non-blocking stream that runs
+ * until mp_finalize: do not call cudaDeviceSynchronize() meanwhile (use stream
+ * synchronisation / mp_sync), and initialise every CUDA kernel / library the
+ * process will use before mp_init (lazy module loading may need an idle context).
  * Errors: MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_NOMEM, MP_ERR_TOPOLOGY. */
 int mp_init(mp_ctx **ctx, const mp_init_args *args);
 
@@ -233,9 +237,15 @@ int mp_sync(mp_ctx *ctx);
 /* ---------------------------------------------------------------- calibration */
 
 /* Step 1: measure α, β (per link) and ε (per staging device) with the
- * engine's own kernels on this GPU, fit (C12) and install them for (0, 0)
- * loopback, plus the shared port.  sizes: byte counts to sweep (NULL = default),
- * reps: repeats per size (median).  Requires world == 1. */
+ * engine's own kernels, fit T(n) = α + n/β (C12) and install the model of every
+ * pair plus the shared port.  sizes: byte counts to sweep (NULL = default 16 MiB ..
+ * 1 GiB), reps: repeats per size (median).
+ * world == 1: the loopback links (HBM copy, relay-ring legs, pinned-host legs).
+ * world > 1: collective — every rank puts into its successor's heap over NVLink,
+ * times its own host legs and a flag ping-pong through the successor's memory;
+ * the measurements are all-gathered and every ordered pair's model is built from
+ * them.  Requires empty receive heaps on every rank (call before mp_alloc), else
+ * MP_ERR_STATE. */
 int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
 
 /* Save / load the model parameters of every pair (Step 1/2). */

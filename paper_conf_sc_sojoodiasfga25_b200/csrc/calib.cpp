@@ -72,20 +72,11 @@ struct Bench {
 // One direct-only fused launch dst ← src of n bytes; returns seconds.
 int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double *out) {
   mp_ctx *c = b.c;
-  mp_config cfg;
-  std::memset(&cfg, 0, sizeof(cfg));
-  mp_path paths[MP_MAX_PATHS];
-  int np = 0;
-  if (int st = mp_paths(c, 0, 0, paths, &np)) return st;
-  cfg.npaths = np;
-  for (int i = 0; i < np; ++i) cfg.path[i] = paths[i];
-  cfg.bytes[0] = n;
-  cfg.chunks[0] = 1;
   std::vector<double> ts;
   for (int r = 0; r < reps + 1; ++r) {
     CKC(cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s));
     CKC(cudaEventRecord(b.e0, b.s));
-    if (int st = mp_xfer(c, dst, src, n, &cfg, b.s)) return st;
+    if (int st = launch_direct_copy(c, dst, src, n, b.s)) return st;
     CKC(cudaEventRecord(b.e1, b.s));
     CKC(cudaEventSynchronize(b.e1));
     float ms = 0;
@@ -129,13 +120,129 @@ int time_pingpong(Bench &b, uint64_t *flags, bool host, int iters, double *eps) 
   return MP_OK;
 }
 
+// Multi-rank Step 1 (collective): every rank measures its own links — the NVLink
+// put into its successor's heap (direct link and both relay legs, which are the same
+// kind of link through NVSwitch), the host legs into/out of its own pinned segment,
+// ε of a GPU stage by a flag ping-pong through the successor's memory, ε of the host
+// stage through pinned memory — then all ranks exchange their measurements and
+// install a model for every ordered pair (s, d): direct and leg 1 from s, relay leg 2
+// and ε from the relay r, host leg 2 and ε from d; the shared port is s's egress.
+struct LinkMeas {
+  double da, db;          // NVLink put α, β
+  double h1a, h1b;        // GPU → host α, β
+  double h2a, h2b;        // host → GPU α, β
+  double eps_dev, eps_host;
+};
+
+int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
+  const int W = c->world, me = c->rank, succ = (c->rank + 1) % c->world;
+  // the successor's heap is used as the put target: nobody may have live buffers yet
+  int32_t busy = c->heap.used_.empty() ? 0 : 1;
+  std::vector<int32_t> all_busy(W);
+  if (int s = world_allgather(c, &busy, all_busy.data(), sizeof(busy))) return s;
+  for (int32_t v : all_busy)
+    if (v) return cfail(c, MP_ERR_STATE, "multi-rank calibration needs empty receive heaps (call it before mp_alloc)");
+  const uint64_t cap = std::min<uint64_t>(c->heap.size, 1024ull << 20);
+  std::vector<uint64_t> sz;
+  for (uint64_t s : sizes)
+    if (s <= cap) sz.push_back(s);
+  if (sz.size() < 2) sz = {cap / 4, cap / 2, cap};
+  const uint64_t big = *std::max_element(sz.begin(), sz.end());
+
+  Bench b;
+  b.c = c;
+  CKC(cudaSetDevice(c->device));
+  CKC(cudaStreamCreateWithFlags(&b.s, cudaStreamNonBlocking));
+  CKC(cudaEventCreate(&b.e0));
+  CKC(cudaEventCreate(&b.e1));
+  void *src = nullptr;
+  CKC(cudaMalloc(&b.flush, b.flush_bytes));
+  CKC(cudaMalloc(&src, big));
+  CKC(cudaMemset(src, 0x5a, big));
+  LinkMeas m{};
+  int st = MP_OK;
+  do {
+    Fit fd{}, fh1{}, fh2{};
+    if ((st = fit_link(b, c->peers[succ].heap, src, sz, big, reps, &fd))) break;
+    m.da = fd.alpha;
+    m.db = fd.beta;
+    if (c->host_path) {
+      // the own segment's ring of sender == me is never used for traffic
+      uint8_t *hr = c->hseg[me] + static_cast<uint64_t>(me) * c->hseg_per_src;
+      const uint64_t hcap = static_cast<uint64_t>(c->slots) * c->host_stride;
+      std::vector<uint64_t> hs;
+      for (uint64_t s : sz)
+        if (s <= std::min<uint64_t>(hcap, 64ull << 20)) hs.push_back(s);
+      if (hs.size() < 2) hs = {hcap / 4, hcap / 2};
+      if ((st = fit_link(b, hr, src, hs, hcap, std::max(3, reps / 2), &fh1))) break;
+      if ((st = fit_link(b, src, hr, hs, hcap, std::max(3, reps / 2), &fh2))) break;
+      m.h1a = fh1.alpha;
+      m.h1b = fh1.beta;
+      m.h2a = fh2.alpha;
+      m.h2b = fh2.beta;
+      if ((st = time_pingpong(b, c->h_probe, true, 500, &m.eps_host))) break;
+    }
+    uint64_t *pf = reinterpret_cast<uint64_t *>(c->peers[succ].ctrl + c->L.probe);
+    if ((st = time_pingpong(b, pf, false, 1000, &m.eps_dev))) break;
+  } while (false);
+  cudaStreamSynchronize(b.s);
+  cudaFree(src);
+  cudaFree(b.flush);
+  cudaEventDestroy(b.e0);
+  cudaEventDestroy(b.e1);
+  cudaStreamDestroy(b.s);
+  int32_t ok = st == MP_OK ? 0 : 1;
+  std::vector<int32_t> all_ok(W);
+  if (int s = world_allgather(c, &ok, all_ok.data(), sizeof(ok))) return s;
+  if (st) return st;
+  for (int32_t v : all_ok)
+    if (v) return cfail(c, MP_ERR_STATE, "calibration failed on another rank");
+  std::vector<LinkMeas> lm(W);
+  if (int s = world_allgather(c, &m, lm.data(), sizeof(LinkMeas))) return s;
+
+  for (int s = 0; s < W; ++s)
+    for (int d = 0; d < W; ++d) {
+      if (s == d) continue;
+      mp_path paths[MP_MAX_PATHS];
+      mp_path_params prm[MP_MAX_PATHS];
+      int np = 0;
+      paths[np] = mp_path{MP_PATH_DIRECT, -1};
+      prm[np++] = mp_path_params{lm[s].da, lm[s].db, 0, 0, 0, 1, 0, 1};
+      for (int r = 0; r < W; ++r) {
+        if (r == s || r == d) continue;
+        paths[np] = mp_path{MP_PATH_GPU, r};
+        prm[np++] = mp_path_params{lm[s].da, lm[s].db, lm[r].da, lm[r].db, std::max(lm[r].eps_dev, 1e-8), 1, 0, 1};
+      }
+      if (c->host_path) {
+        paths[np] = mp_path{MP_PATH_HOST, -1};
+        prm[np++] = mp_path_params{lm[s].h1a, lm[s].h1b, lm[d].h2a, lm[d].h2b, std::max(lm[d].eps_host, 1e-8),
+                                   1, 0, 0};
+      }
+      mp_port_params port{lm[s].da, lm[s].db};
+      if (int e = mp_set_model(c, s, d, paths, prm, np, &port)) return e;
+    }
+  return world_barrier(c);
+}
+
 }  // namespace
 
 extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
-  if (c->world != 1) return cfail(c, MP_ERR_UNSUPPORTED, "calibration runs on the loopback engine");
   if (reps <= 0) reps = 5;
+  if (c->world != 1) {
+    std::vector<uint64_t> sizes;
+    if (sizes_in && nsizes > 0)
+      sizes.assign(sizes_in, sizes_in + nsizes);
+    else
+      for (uint64_t s = 16ull << 20; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
+    int32_t derr = 0;
+    int s = calibrate_world(c, sizes, reps);
+    if (s) return s;
+    CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
+    if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration probe timed out");
+    return MP_OK;
+  }
   // Default sizes: the asymptotic range (C12).  A local HBM→HBM copy only shows its
   // steady-state rate once the working set exceeds the 126 MB L2, so the direct link
   // is fitted on 128 MiB .. 1 GiB; the ring legs on what the ring holds.

@@ -277,6 +277,28 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
 
 }  // namespace
 
+int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream) {
+  XferParams P;
+  std::memset(&P, 0, sizeof(P));
+  P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  P.err = c->d_err;
+  P.copy_mode = c->copy_mode;
+  P.npaths = 1;
+  DevPath &d = P.p[0];
+  d.kind = DK_DIRECT;
+  d.bytes = n;
+  d.src = static_cast<const uint8_t *>(src);
+  d.dst = static_cast<uint8_t *>(dst);
+  d.align = c->opts.align;
+  const uint64_t want = std::max<uint64_t>(1, (n + (32u << 10) - 1) / (32u << 10));
+  d.g_in = static_cast<uint32_t>(std::min<uint64_t>(want, static_cast<uint64_t>(std::max(1, c->per_sm * c->sms))));
+  P.nblocks = d.g_in;
+  const int e = launch_xfer(P, stream);
+  if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "copy launch");
+  c->launches += 1;
+  return MP_OK;
+}
+
 // ------------------------------------------------------------------ Heap
 
 void mpx::Heap::reset(uint8_t *b, uint64_t n) {
@@ -395,7 +417,7 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
       }
     }
   }
-  if (!c->model_only && !(a->flags & MP_INIT_NO_CALIBRATE) && c->world == 1) {
+  if (!c->model_only && !(a->flags & MP_INIT_NO_CALIBRATE)) {
     if (int s = mp_calibrate(c, nullptr, 0, 0)) {
       std::fprintf(stderr, "mp_init: calibration failed: %s\n", c->last_error.c_str());
       mp_finalize(c);

@@ -106,6 +106,10 @@ struct mp_ctx {
 };
 
 namespace mpx {
+// One direct-path fused launch dst ← src (any world; dst may be peer or mapped host).
+int launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream);
+int world_barrier(mp_ctx *c);
+int world_allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes);
 int world_init(mp_ctx *c);
 int world_finalize(mp_ctx *c);
 int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,

@@ -76,6 +76,7 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.done = take(static_cast<uint64_t>(world) * 128);
   L.relay_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.ring_full = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
+  L.probe = take(64);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
@@ -121,6 +122,9 @@ HostRingPtrs host_ring(const mp_ctx *c, int src, int dst) {
 }
 
 }  // namespace
+
+int world_barrier(mp_ctx *c) { return barrier(c); }
+int world_allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes) { return allgather(c, in, out, bytes); }
 
 static bool debug_on() {
   const char *d = std::getenv("MPX_DEBUG");
