@@ -224,12 +224,9 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   uint32_t staged_ctas = 0;
   for (int i = 1; i < cfg.npaths; ++i)
     if (cfg.bytes[i]) staged_ctas += 2u * static_cast<uint32_t>(c->relay_ctas);
-  // direct group: up to 4 CTAs per SM, at least 32 KiB per CTA, leaving room
-  // for every staged group to be co-resident.
-  const uint64_t want = std::max<uint64_t>(1, (cfg.bytes[0] + (32u << 10) - 1) / (32u << 10));
-  const int room = std::max(1, cap - static_cast<int>(staged_ctas));
-  const uint32_t g_direct = static_cast<uint32_t>(
-      std::min<uint64_t>(want, static_cast<uint64_t>(std::min(room, 4 * c->sms))));
+  // direct group sized by direct_ctas(), leaving room for every staged group to be
+  // co-resident.
+  const uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas));
   uint32_t next = 0;
   uint64_t off = 0;
   P.npaths = static_cast<uint32_t>(cfg.npaths);
@@ -290,8 +287,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   d.src = static_cast<const uint8_t *>(src);
   d.dst = static_cast<uint8_t *>(dst);
   d.align = c->opts.align;
-  const uint64_t want = std::max<uint64_t>(1, (n + (32u << 10) - 1) / (32u << 10));
-  d.g_in = static_cast<uint32_t>(std::min<uint64_t>(want, static_cast<uint64_t>(std::max(1, c->per_sm * c->sms))));
+  d.g_in = direct_ctas(c, n, c->per_sm * c->sms);
   P.nblocks = d.g_in;
   const int e = launch_xfer(P, stream);
   if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "copy launch");
@@ -420,6 +416,13 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
   if (!c->model_only && !(a->flags & MP_INIT_NO_CALIBRATE)) {
     if (int s = mp_calibrate(c, nullptr, 0, 0)) {
       std::fprintf(stderr, "mp_init: calibration failed: %s\n", c->last_error.c_str());
+      mp_finalize(c);
+      return s;
+    }
+  }
+  if (!c->model_only && c->world > 1) {
+    if (int s = world_start_relay(c)) {
+      std::fprintf(stderr, "mp_init: %s\n", c->last_error.c_str());
       mp_finalize(c);
       return s;
     }

@@ -2,6 +2,8 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <algorithm>
+
 #include <cstdint>
 #include <deque>
 #include <map>
@@ -106,11 +108,22 @@ struct mp_ctx {
 };
 
 namespace mpx {
+// CTAs of a direct group: one per 32 KiB, at most 2 per SM with the TMA pipeline (the
+// measured optimum: 2 × 4 × 8 KiB in flight per SM) or 4 per SM with LDG/STG, and at
+// most `room` (what is left of the co-resident capacity).
+inline uint32_t direct_ctas(const mp_ctx *c, uint64_t bytes, int room) {
+  const uint64_t want = bytes ? (bytes + (32u << 10) - 1) / (32u << 10) : 1;
+  const int lim = std::max(1, std::min(room, (c->copy_mode == 1 ? 2 : 4) * c->sms));
+  return static_cast<uint32_t>(std::min<uint64_t>(want, static_cast<uint64_t>(lim)));
+}
+
 // One direct-path fused launch dst ← src (any world; dst may be peer or mapped host).
 int launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream);
 int world_barrier(mp_ctx *c);
 int world_allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes);
 int world_init(mp_ctx *c);
+int world_start_relay(mp_ctx *c);
+int world_stop_relay(mp_ctx *c);
 int world_finalize(mp_ctx *c);
 int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,
                void *stream);

@@ -118,8 +118,10 @@ __device__ __forceinline__ void group_copy(uint8_t *dst, const uint8_t *src, uin
 // by a bulk group so a stage is only reloaded once its previous store has finished
 // reading shared memory.  Blocks r, r+G, r+2G, … of the co-aligned 16-B body belong
 // to CTA r; head/tail bytes go through group_copy.  Requires (dst ^ src) % 16 == 0.
-constexpr uint32_t kBulkBlock = 16384;
-constexpr uint32_t kBulkStages = 3;
+// Sweep on B200 (scripts/copybench.cu, profiles/r01/copybench.jsonl): two pipelines
+// per SM of 4 × 8 KiB beat both deeper/larger pipelines and cudaMemcpyAsync (+3.9 %).
+constexpr uint32_t kBulkBlock = 8192;
+constexpr uint32_t kBulkStages = 4;
 constexpr uint32_t kBulkSmem = kBulkBlock * kBulkStages + 64;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
@@ -594,10 +596,15 @@ __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constan
   __syncthreads();
   const uint32_t sender = blockIdx.x / P.g, r = blockIdx.x % P.g;
   if (sender == P.me || sender >= P.world) return;
-  for (uint64_t q = 0;; ++q) {
+  // ring position survives a stop/restart (mp_calibrate stops the relay)
+  uint64_t *pos = reinterpret_cast<uint64_t *>(P.my_ctrl + P.L.relay_pos) + sender;
+  for (uint64_t q = ld_volatile(pos);; ++q) {
     const uint64_t s = q % P.L.slots, u = q / P.L.slots;
     uint64_t *fl = flags_at(P.my_ctrl, P.L.ring_full, sender, P.L.slots, s);
-    if (!wait_flags(fl, P.g, u + 1, 0, P.err, &s_abort, P.stop)) return;
+    if (!wait_flags(fl, P.g, u + 1, 0, P.err, &s_abort, P.stop)) {
+      if (r == 0 && threadIdx.x == 0) *pos = q;
+      return;
+    }
     uint8_t *slot = P.my_ctrl + P.L.ring_data + (static_cast<uint64_t>(sender) * P.L.slots + s) * P.L.stride;
     if (threadIdx.x < 4) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(slot) + threadIdx.x);
     __syncthreads();

@@ -77,6 +77,7 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.relay_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.ring_full = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.probe = take(64);
+  L.relay_pos = take(static_cast<uint64_t>(world) * 8);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
@@ -204,41 +205,54 @@ int world_init(mp_ctx *c) {
   c->host_q.assign(W, 0);
   c->done_target.assign(W, 0);
 
-  const char *no_relay = std::getenv("MPX_NO_RELAY");  // diagnostics: no relay kernel
-  if (W >= 3 && !(no_relay && no_relay[0] == '1')) {  // the persistent relay kernel
+  if (W >= 3) {  // resources of the persistent relay kernel; it is started by world_start_relay
     CKW(cudaHostAlloc(&p, 64, cudaHostAllocMapped | cudaHostAllocPortable));
     c->stop = static_cast<int32_t *>(p);
     *c->stop = 0;
-    DBG("stop word allocated");
     CKW(cudaStreamCreateWithFlags(&c->relay_stream, cudaStreamNonBlocking));
-    DBG("relay stream created");
-    RelayParams R{};
-    R.me = static_cast<uint32_t>(c->rank);
-    R.world = static_cast<uint32_t>(W);
-    R.g = static_cast<uint32_t>(c->relay_ctas);
-    R.my_ctrl = c->ctrl;
-    for (int r = 0; r < W; ++r) R.peer[r] = c->peers[r];
-    R.L = c->L;
-    R.stop = c->stop;
-    R.err = c->d_err;
-    if (int e = launch_relay(R, c->relay_stream))
-      return wfail(c, MP_ERR_CUDA, std::string("relay launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
-    c->launches += 1;
-    c->relay_running = true;
   }
-  DBG("relay launched");
   const int s = barrier(c);
   DBG("world_init done");
   return s;
 }
 
+// Launch the persistent relay kernel (A8 step 3).  Every allocation / free that may
+// synchronise the device (cudaFree, cudaHostAlloc, ...) must happen before this.
+int world_start_relay(mp_ctx *c) {
+  const char *no_relay = std::getenv("MPX_NO_RELAY");  // diagnostics: no relay kernel
+  if (c->world < 3 || c->relay_running || (no_relay && no_relay[0] == '1')) return MP_OK;
+  *reinterpret_cast<volatile int32_t *>(c->stop) = 0;
+  RelayParams R{};
+  R.me = static_cast<uint32_t>(c->rank);
+  R.world = static_cast<uint32_t>(c->world);
+  R.g = static_cast<uint32_t>(c->relay_ctas);
+  R.my_ctrl = c->ctrl;
+  for (int r = 0; r < c->world; ++r) R.peer[r] = c->peers[r];
+  R.L = c->L;
+  R.stop = c->stop;
+  R.err = c->d_err;
+  if (int e = launch_relay(R, c->relay_stream))
+    return wfail(c, MP_ERR_CUDA, std::string("relay launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  c->launches += 1;
+  c->relay_running = true;
+  DBG("relay launched");
+  return MP_OK;
+}
+
+// Stop it (no transfers may be in flight); its ring positions are kept in the
+// control block, so a restart continues where it stopped.
+int world_stop_relay(mp_ctx *c) {
+  if (!c->relay_running) return MP_OK;
+  *reinterpret_cast<volatile int32_t *>(c->stop) = 1;
+  CKW(cudaStreamSynchronize(c->relay_stream));
+  c->relay_running = false;
+  DBG("relay stopped");
+  return MP_OK;
+}
+
 int world_finalize(mp_ctx *c) {
   int st = MP_OK;
-  if (c->relay_running) {
-    *reinterpret_cast<volatile int32_t *>(c->stop) = 1;
-    cudaStreamSynchronize(c->relay_stream);
-    c->relay_running = false;
-  }
+  world_stop_relay(c);
   for (cudaStream_t s : c->streams) cudaStreamSynchronize(s);
   if (c->allgather) st = barrier(c);
   for (int r = 0; r < static_cast<int>(c->peers.size()); ++r) {
@@ -291,9 +305,7 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   uint32_t staged = 0;
   for (int i = 1; i < cfg.npaths; ++i)
     if (cfg.bytes[i]) staged += P.g_stage;
-  const uint64_t want = std::max<uint64_t>(1, (cfg.bytes[0] + (32u << 10) - 1) / (32u << 10));
-  P.g_direct = static_cast<uint32_t>(
-      std::min<uint64_t>(want, static_cast<uint64_t>(std::max(1, std::min(cap - static_cast<int>(staged), 2 * c->sms)))));
+  P.g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged));
   uint32_t next = P.g_direct;
   uint64_t off = cfg.bytes[0];
   uint32_t np = 0;

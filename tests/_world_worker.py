@@ -67,6 +67,11 @@ def scenario_engine(rank, world):
     print(f"rank {rank}: init", flush=True)
     c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0)
+    if world >= 3:
+        # collective Step 1 with the relay kernel running: stop, measure, restart
+        c.calibrate(sizes=[4 * MiB, 8 * MiB, 16 * MiB], reps=2)
+        _, prm, _ = c.get_model(0, 1)
+        assert prm[0]["beta"] > 0 and prm[1]["eps"] > 0
     ps = c.paths(0, 1)
     np_ = len(ps)
     cases = []
