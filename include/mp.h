@@ -194,7 +194,9 @@ int mp_predict(mp_ctx *ctx, int src, int dst, uint64_t bytes, const mp_config *c
  * Eq 11 then Eq 24 with the two-pass φ (C4) and the active set (C2), k from Eq 19
  * (C5), shares floored to A with the leftover to the direct path (C7), optional
  * pass 3 (C18).  path_mask bit i enables path i of mp_paths() (bit 0, the direct
- * path, is always on; 0 = all paths).  Results are cached (C10).  Host-only. */
+ * path, is always on; 0 = all paths).  The environment variable MPX_PATHS (read at
+ * mp_init; e.g. "direct,host", "direct,gpu", "all") further restricts the path kinds
+ * (P:312-313).  Results are cached (C10).  Host-only. */
 int mp_select(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t path_mask,
               mp_config *out);
 

@@ -389,6 +389,13 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
     delete c;
     return MP_ERR_INVALID;
   }
+  if (const char *ps = std::getenv("MPX_PATHS")) {  // e.g. "direct,host"
+    const std::string s(ps);
+    c->env_kinds = 1u << MP_PATH_DIRECT;
+    if (s.find("gpu") != std::string::npos || s.find("relay") != std::string::npos) c->env_kinds |= 1u << MP_PATH_GPU;
+    if (s.find("host") != std::string::npos) c->env_kinds |= 1u << MP_PATH_HOST;
+    if (s.empty() || s == "all") c->env_kinds = 0x7u;
+  }
   c->allgather = a->allgather;
   c->allgather_user = a->allgather_user;
   if (!c->model_only) {
@@ -569,6 +576,15 @@ int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_con
   if (!c || !out) return fail(c, MP_ERR_INVALID, "null argument");
   if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
   const PairModel *m = pair_model(c, src, dst);
+  // environment variables include/exclude path kinds (MPX_PATHS).
+  if (c->env_kinds != 0x7u) {
+    uint32_t eff = 0;
+    for (size_t i = 0; i < m->paths.size(); ++i) {
+      const bool asked = mask == 0 || ((mask >> i) & 1u);
+      if (i == 0 || (asked && ((c->env_kinds >> m->paths[i].kind) & 1u))) eff |= 1u << i;
+    }
+    mask = eff;
+  }
   const CacheKey key{src, dst, mask, bytes};
   auto it = c->cache.find(key);  // Alg 1 lines 4-6 (C10)
   if (it == c->cache.end()) {

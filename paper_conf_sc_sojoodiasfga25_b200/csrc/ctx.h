@@ -71,6 +71,7 @@ struct mp_ctx {
   mpx::ModelOpts opts;
   std::map<std::pair<int, int>, mpx::PairModel> models;
   std::unordered_map<mpx::CacheKey, mpx::Selection, mpx::CacheKeyHash> cache;
+  uint32_t env_kinds = 0x7u;       // path kinds allowed by MPX_PATHS (bit = MP_PATH_*)
 
   // engine
   int n_loop_relays = 6;

@@ -163,6 +163,36 @@ def test_calibration_installs_sane_parameters():
     c.close()
 
 
+def test_config1_forced_split_and_model(ctx):
+    # BASELINE.json config 1: 1 MiB, direct + 1 relay, 4 chunks; θ forced to (3/4, 1/4)
+    # — 256 KiB on the relay ring in 4 × 64 KiB chunks.  Payload bit-exact
+    # against the oracle replay; mp_predict of that config against the oracle's O2; the
+    # model's own pick (mask = direct + relay) against the oracle brute force.
+    from oracle import optimize as OO
+    n = 1 << 20
+    ps = ctx.paths()
+    nb = [0] * len(ps)
+    nb[0], nb[1] = 3 * n // 4, n // 4
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1] = 4
+    run(ctx, n, nb, ks, seed=11)
+    paths, prm, port = ctx.get_model(0, 0)
+    sub = [M.Path(kind=k, via=v, **{f: (p[f] if not (k == 0 and f == "beta2") else float("inf"))
+                                    for f in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")})
+           for (k, v), p in zip(paths[:2], prm[:2])]
+    o = ctx.get_options()
+    opts = M.Options(mode=o["mode"], stagger=bool(o["stagger"]), align=o["align"], c_min=o["c_min"],
+                     k_max=o["k_max"], slot_bytes=o["slot_bytes"])
+    oport = M.Port(alpha=port["alpha"], beta=port["beta"])
+    t_lib = ctx.predict(0, 0, n, ctx.make_config(nb, ks))
+    t_orc = M.evaluate(n, nb[:2], ks[:2], sub, opts, oport)
+    assert abs(t_lib - t_orc) <= 1e-9 * t_orc
+    t_bf, _, _ = OO.brute_force(n, sub, opts, oport, steps=256, k_values=range(1, 65))
+    pick = ctx.select(0, 0, n, 0b11).as_dict()
+    assert pick["t_pred"] <= t_bf * 1.02
+    run(ctx, n, pick["bytes"], pick["chunks"], seed=12)
+
+
 def test_full_size_config3_bit_exact(ctx):
     # BASELINE.json config 3 at full size (1 GiB, direct + 6 relays + host) on the
     # loopback engine, in the paper-mode split (every path carries bytes): bit-exact on

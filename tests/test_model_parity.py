@@ -124,3 +124,20 @@ def test_cache_invalidation():
         setup_pair(c, tbl, None)
         b = c.select(0, 1, 64 * MiB).as_dict()
         assert b["bytes"][0] > a["bytes"][0]
+
+
+def test_env_path_filter(monkeypatch):
+    # environment variables include / exclude paths (MPX_PATHS, read at mp_init)
+    tbl = synth.topology(11, 2, True)
+    monkeypatch.setenv("MPX_PATHS", "direct,host")
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        setup_pair(c, tbl, None)
+        d = c.select(0, 1, 512 * MiB).as_dict()
+        assert d["bytes"][1] == 0 and d["bytes"][2] == 0 and d["bytes"][3] > 0
+        ref = M.select(512 * MiB, oracle_paths(tbl), M.Options(), None, [True, False, False, True])
+        for a, b in zip(d["bytes"], ref.bytes):
+            assert abs(a - b) <= 256
+    monkeypatch.setenv("MPX_PATHS", "all")
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        setup_pair(c, tbl, None)
+        assert all(b > 0 for b in c.select(0, 1, 512 * MiB).as_dict()["bytes"])
