@@ -220,6 +220,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.err = c->d_err;
   P.copy_mode = c->copy_mode;
+  P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
   const int cap = std::max(1, c->per_sm * c->sms);
   uint32_t staged_ctas = 0;
   for (int i = 1; i < cfg.npaths; ++i)
@@ -280,6 +281,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.err = c->d_err;
   P.copy_mode = c->copy_mode;
+  P.bulk_stages = bulk_stages_for(n);
   P.npaths = 1;
   DevPath &d = P.p[0];
   d.kind = DK_DIRECT;

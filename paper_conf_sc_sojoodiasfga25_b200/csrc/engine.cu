@@ -170,7 +170,7 @@ __device__ __forceinline__ void bulk_wait_all() {
 }
 
 __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32_t r, uint32_t G,
-                          uint8_t *smem) {
+                          uint8_t *smem, uint32_t D) {
   if ((reinterpret_cast<uintptr_t>(dst) ^ reinterpret_cast<uintptr_t>(src)) & 15u) {
     group_copy<LD_SRC>(dst, src, len, r, G);
     return;
@@ -190,8 +190,9 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
   const uint64_t nblk = (body + kBulkBlock - 1) / kBulkBlock;
   if (r >= nblk) return;
   const uint64_t mine = (nblk - r + G - 1) / G;  // blocks r, r+G, …
+  if (D < 1 || D > kBulkStages) D = kBulkStages;
   uint64_t *bars = reinterpret_cast<uint64_t *>(smem + kBulkBlock * kBulkStages);
-  for (uint32_t i = 0; i < kBulkStages; ++i) mbar_init(smem_u32(bars + i));
+  for (uint32_t i = 0; i < D; ++i) mbar_init(smem_u32(bars + i));
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   auto blk = [&](uint64_t it, uint64_t *off, uint32_t *bytes) {
     const uint64_t o = (r + it * G) * static_cast<uint64_t>(kBulkBlock);
@@ -202,24 +203,24 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
     uint64_t o;
     uint32_t n;
     blk(it, &o, &n);
-    const uint32_t st = static_cast<uint32_t>(it % kBulkStages);
+    const uint32_t st = static_cast<uint32_t>(it % D);
     const uint32_t bar = smem_u32(bars + st);
     mbar_expect_tx(bar, n);
     bulk_load(smem_u32(smem + st * kBulkBlock), s + o, n, bar);
   };
-  const uint64_t pro = mine < kBulkStages ? mine : kBulkStages;
+  const uint64_t pro = mine < D ? mine : D;
   for (uint64_t it = 0; it < pro; ++it) issue_load(it);
   for (uint64_t it = 0; it < mine; ++it) {
-    const uint32_t st = static_cast<uint32_t>(it % kBulkStages);
-    mbar_wait(smem_u32(bars + st), static_cast<uint32_t>((it / kBulkStages) & 1));
+    const uint32_t st = static_cast<uint32_t>(it % D);
+    mbar_wait(smem_u32(bars + st), static_cast<uint32_t>((it / D) & 1));
     uint64_t o;
     uint32_t n;
     blk(it, &o, &n);
     bulk_store(d + o, smem_u32(smem + st * kBulkBlock), n);
     // refill the stage used one iteration ago once its store has read shared memory
-    if (it >= 1 && it - 1 + kBulkStages < mine) {
+    if (it >= 1 && it - 1 + D < mine) {
       bulk_wait_read<1>();
-      issue_load(it - 1 + kBulkStages);
+      issue_load(it - 1 + D);
     }
   }
   bulk_wait_all();
@@ -353,7 +354,7 @@ __global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant
     if (b >= p.cta0_in && b < p.cta0_in + p.g_in) {
       if (p.kind == DK_DIRECT)
         if (P.copy_mode == 1)
-          bulk_copy(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem);
+          bulk_copy(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem, P.bulk_stages);
         else
           group_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in);
       else
@@ -481,7 +482,7 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
   uint64_t *done = done_at(P.dst_ctrl, P.L, P.me);
   if (b < P.g_direct) {  // A7: direct NVLink stores into the receiver's heap
     if (P.copy_mode == 1)
-      bulk_copy(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct, dyn_smem);
+      bulk_copy(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct, dyn_smem, P.bulk_stages);
     else
       group_copy<LD_SRC>(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct);
     const uint64_t share = P.direct_bytes * (b + 1) / P.g_direct - P.direct_bytes * b / P.g_direct;

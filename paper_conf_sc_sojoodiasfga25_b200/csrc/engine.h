@@ -51,7 +51,7 @@ struct XferParams {
   uint32_t npaths;
   uint32_t nblocks;
   uint32_t copy_mode;    // direct group: 0 = LDG/STG vectors, 1 = TMA bulk (cp.async.bulk)
-  uint32_t pad_;
+  uint32_t bulk_stages;  // TMA pipeline depth per CTA (1..4)
   uint64_t timeout_ns;
   int32_t *err;          // device (or mapped host) error word
   DevPath p[kMaxPaths];
@@ -114,7 +114,7 @@ struct HostRingPtrs {
 };
 
 struct SendParams {
-  uint32_t me, dst, nblocks, g_direct, g_stage, npaths, copy_mode, pad0_;
+  uint32_t me, dst, nblocks, g_direct, g_stage, npaths, copy_mode, bulk_stages;
   uint64_t seq, bytes, tag, timeout_ns;
   const uint8_t *src;
   uint8_t *my_ctrl;

@@ -299,6 +299,7 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   P.host_slots = static_cast<uint32_t>(c->slots);
   P.g_stage = static_cast<uint32_t>(c->relay_ctas);
   P.copy_mode = c->copy_mode;
+  P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
   if (c->host_path) P.host = host_ring(c, c->rank, dst);
   P.direct_bytes = cfg.bytes[0];
   const int cap = std::max(1, c->per_sm * c->sms);
