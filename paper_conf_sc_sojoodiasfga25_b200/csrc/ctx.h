@@ -109,17 +109,17 @@ struct mp_ctx {
 };
 
 namespace mpx {
-// TMA pipeline shape of a direct group (scripts/copybench.cu sweeps on B200,
-// profiles/r01/copybench*.jsonl): messages that stay L2-resident (≤ 64 MiB) do best with
-// 4 CTAs per SM × 3 stages of 8 KiB, HBM-bound ones with 2 CTAs per SM × 4 stages.
-constexpr uint64_t kL2Resident = 64ull << 20;
-inline uint32_t bulk_stages_for(uint64_t bytes) { return bytes <= kL2Resident ? 3u : 4u; }
+// TMA pipeline shape of a direct group: 2 CTAs per SM × 4 stages of 8 KiB at every
+// size.  (scripts/copybench.cu favoured 4 CTAs/SM × 3 stages for L2-resident sizes in
+// single-launch timings, but inside the engine that shape measured slower at every
+// size in the OMB sweep — profiles/r01/omb_*.jsonl — so it is not used.)
+inline uint32_t bulk_stages_for(uint64_t /*bytes*/) { return 4u; }
 
-// CTAs of a direct group: one per 32 KiB, at most (TMA) 4 or 2 per SM as above, or
-// 4 per SM with LDG/STG, and at most `room` (what is left of the co-resident capacity).
+// CTAs of a direct group: one per 32 KiB, at most 2 per SM (TMA) or 4 per SM
+// (LDG/STG), and at most `room` (what is left of the co-resident capacity).
 inline uint32_t direct_ctas(const mp_ctx *c, uint64_t bytes, int room) {
   const uint64_t want = bytes ? (bytes + (32u << 10) - 1) / (32u << 10) : 1;
-  const int per_sm = c->copy_mode == 1 ? (bytes <= kL2Resident ? 4 : 2) : 4;
+  const int per_sm = c->copy_mode == 1 ? 2 : 4;
   const int lim = std::max(1, std::min(room, per_sm * c->sms));
   return static_cast<uint32_t>(std::min<uint64_t>(want, static_cast<uint64_t>(lim)));
 }
