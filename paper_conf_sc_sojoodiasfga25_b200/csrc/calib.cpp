@@ -120,6 +120,74 @@ int time_pingpong(Bench &b, uint64_t *flags, bool host, int iters, double *eps) 
   return MP_OK;
 }
 
+// Time the staged path `idx` of the loopback pair alone carrying n bytes in k chunks
+// for every k of a grid; return c = k_best / k* (clamped to [0.1, 10]).
+int fit_phi(mp_ctx *c, int idx, uint64_t n, int reps, double *c_out) {
+  mp_path paths[MP_MAX_PATHS];
+  mp_path_params prm[MP_MAX_PATHS];
+  int np = 0;
+  mp_port_params port;
+  if (int s = mp_get_model(c, 0, 0, paths, prm, &np, &port)) return s;
+  PathModel pm;
+  pm.kind = paths[idx].kind;
+  pm.alpha = prm[idx].alpha;
+  pm.beta = prm[idx].beta;
+  pm.alpha2 = prm[idx].alpha2;
+  pm.beta2 = prm[idx].beta2;
+  pm.eps = prm[idx].eps;
+  const double ks = k_star(pm, static_cast<double>(n), M_B200);
+  Bench b;
+  b.c = c;
+  void *src = nullptr, *dst = nullptr;
+  CKC(cudaStreamCreateWithFlags(&b.s, cudaStreamNonBlocking));
+  CKC(cudaEventCreate(&b.e0));
+  CKC(cudaEventCreate(&b.e1));
+  CKC(cudaMalloc(&b.flush, b.flush_bytes));
+  CKC(cudaMalloc(&src, n));
+  CKC(cudaMalloc(&dst, n));
+  mp_config cfg;
+  std::memset(&cfg, 0, sizeof(cfg));
+  cfg.npaths = np;
+  for (int i = 0; i < np; ++i) cfg.path[i] = paths[i];
+  cfg.bytes[idx] = n;
+  double best_t = 1e30;
+  uint32_t best_k = 1;
+  int st = MP_OK;
+  for (uint32_t k : {1u, 2u, 3u, 4u, 6u, 8u, 12u, 16u, 24u, 32u, 48u, 64u}) {
+    const uint64_t A = c->opts.align, U = n / A;
+    if (k > U || A * ((U + k - 1) / k) + (n - U * A) > c->slot_bytes) continue;
+    cfg.chunks[idx] = k;
+    std::vector<double> ts;
+    for (int r = 0; r < reps + 1 && st == MP_OK; ++r) {
+      cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s);
+      cudaEventRecord(b.e0, b.s);
+      st = mp_xfer(c, dst, src, n, &cfg, b.s);
+      cudaEventRecord(b.e1, b.s);
+      cudaEventSynchronize(b.e1);
+      float ms = 0;
+      cudaEventElapsedTime(&ms, b.e0, b.e1);
+      if (r > 0) ts.push_back(ms * 1e-3);
+    }
+    if (st) break;
+    const double t = median(ts);
+    if (t < best_t) {
+      best_t = t;
+      best_k = k;
+    }
+  }
+  cudaStreamSynchronize(b.s);
+  cudaFree(src);
+  cudaFree(dst);
+  cudaFree(b.flush);
+  cudaEventDestroy(b.e0);
+  cudaEventDestroy(b.e1);
+  cudaStreamDestroy(b.s);
+  if (st) return st;
+  const double cc = ks > 0 ? static_cast<double>(best_k) / ks : 1.0;
+  *c_out = std::min(10.0, std::max(0.1, cc));
+  return MP_OK;
+}
+
 // Multi-rank Step 1 (collective): every rank measures its own links — the NVLink
 // put into its successor's heap (direct link and both relay legs, which are the same
 // kind of link through NVSwitch), the host legs into/out of its own pinned segment,
@@ -329,5 +397,20 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
     prm[np++] = mp_path_params{fh1.alpha, fh1.beta, fh2.alpha, fh2.beta, std::max(eps_host, 1e-8), 1, 0, 2};
   }
   mp_port_params port{fd.alpha, 2.0 * fd.beta};
+  if (int s = mp_set_model(c, 0, 0, paths, prm, np, &port)) return s;
+
+  // φ (C4): "topology constants (in the form of c·f(n))", P:275 — the staged path alone
+  // carries n bytes in k chunks over a grid of k; c = k_best / k* (Eq 14/15 with the
+  // fitted α, β, ε), so Eq 19 reproduces the measured optimum at that size.
+  double c_relay = 1.0, c_host = 1.0;
+  if (c->n_loop_relays > 0) {
+    const uint64_t n = std::min<uint64_t>(64ull << 20, static_cast<uint64_t>(c->slots) * c->slot_bytes);
+    if (int s = fit_phi(c, 1, n, reps, &c_relay)) return s;
+    for (int i = 1; i <= c->n_loop_relays; ++i) prm[i].c = c_relay;
+  }
+  if (c->host_path) {
+    if (int s = fit_phi(c, np - 1, 16ull << 20, std::max(3, reps / 2), &c_host)) return s;
+    prm[np - 1].c = c_host;
+  }
   return mp_set_model(c, 0, 0, paths, prm, np, &port);
 }

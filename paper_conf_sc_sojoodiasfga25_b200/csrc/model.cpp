@@ -236,6 +236,11 @@ uint32_t clamp_k(uint64_t k, uint64_t b, const ModelOpts &o) {
 
 bool PairModel::has_port() const { return port_beta > 0.0 && std::isfinite(port_beta); }
 
+double k_star(const PathModel &p, double x, int mode) {
+  if (bottleneck(p, mode) == 1) return std::sqrt(x / (p.alpha * p.beta2));
+  return std::sqrt(x / (p.beta * (p.eps + p.alpha2)));
+}
+
 uint32_t k_from_real(double k_real) {
   // C5: smallest k >= 1 with k(k+1) >= k_real² (1e-12 relative slack for exact ties).
   const double target = k_real * k_real * (1.0 - 1e-12);

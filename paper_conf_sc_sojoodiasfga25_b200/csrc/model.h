@@ -56,4 +56,8 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
 // The C5 integer rule (exposed for tests through the selector only).
 uint32_t k_from_real(double k_real);
 
+// Eq 14 / Eq 15: the real optimal chunk count of a staged path
+// carrying x bytes (used by the φ calibration).
+double k_star(const PathModel &p, double x, int mode);
+
 }  // namespace mpx

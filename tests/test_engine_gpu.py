@@ -160,6 +160,8 @@ def test_calibration_installs_sane_parameters():
     assert 5e9 < h["beta"] < 1.5e11 and 5e9 < h["beta2"] < 1.5e11    # PCIe Gen5 legs
     assert 0 < h["eps"] < 2e-5 and 0 < prm[1]["eps"] < 1e-5
     assert port["beta"] > d["beta"]
+    # φ multipliers (C4) fitted from the measured best chunk counts
+    assert 0.1 <= prm[1]["c"] <= 10 and 0.1 <= h["c"] <= 10
     c.close()
 
 
