@@ -139,11 +139,45 @@ def scenario_engine(rank, world):
     c.close()
 
 
+def scenario_faults(rank, world):
+    """A tag mismatch is reported on both sides as MP_ERR_MISMATCH and a receive that
+    is never matched ends in MP_ERR_TIMEOUT — on the device, bounded by %globaltimer —
+    instead of hanging (failure detection)."""
+    import synth
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    src = torch.empty(MiB, dtype=torch.uint8, device="cuda")
+    src.copy_(torch.from_numpy(synth.payload(MiB, 0)))
+    torch.cuda.synchronize()
+    for fault in ("mismatch", "timeout"):
+        c = mdist.context_from_dist(device=0, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                    timeout_s=3.0)
+        if rank == 0 and fault == "mismatch":
+            c.send(src, MiB, 1, tag=5, stream=stream)
+        elif rank == 1:
+            p = c.alloc(MiB)
+            c.recv(p, MiB, 0, tag=6 if fault == "mismatch" else 7, stream=stream)
+        stream.synchronize()
+        status = 0
+        try:
+            c.sync()
+        except mp.MPError as e:
+            status = e.status
+        expect = {"mismatch": -8, "timeout": -7 if rank == 1 else 0}[fault]
+        assert status == expect, (fault, rank, status)
+        print(f"rank {rank}: {fault} -> {status}", flush=True)
+        dist.barrier()
+        c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     try:
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
-        {"gloo_model": scenario_gloo_model, "engine": scenario_engine}[scen](rank, world)
+        {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
+         "faults": scenario_faults}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

@@ -90,6 +90,22 @@ def test_ragged_tail_not_multiple_of_align(ctx):
     run(ctx, n, nbytes, chunks)
 
 
+def test_random_splits_fuzz(ctx):
+    # 40 seeded random messages: size, offsets, share of every path, chunk counts
+    import random
+    rng = random.Random(20251116)
+    ps = ctx.paths()
+    for it in range(40):
+        n = rng.randint(1, 3 * MiB)
+        w = [rng.random() if rng.random() < 0.7 else 0.0 for _ in ps]
+        tot = sum(w) or 1.0
+        nb = [int(n * x / tot) // 256 * 256 for x in w]
+        nb[0] += n - sum(nb)
+        ks = [1] + [min(max(1, b // 256), rng.randint(1, 9)) if b else 0 for b in nb[1:]]
+        # chunks must fit the 4 MiB test slots
+        run(ctx, n, nb, ks, rng.randint(0, 31), rng.randint(0, 31), seed=it % 20)
+
+
 def test_invalid_configs_rejected(ctx):
     ps = ctx.paths()
     n = MiB

@@ -60,3 +60,12 @@ def test_multirank_engine_same_gpu(world):
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(world, "engine", timeout=400)
+
+
+@pytest.mark.gpu
+def test_multirank_faults_reported_not_hung():
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(2, "faults", timeout=300)
