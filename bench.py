@@ -447,6 +447,52 @@ def main():
     e2e = n * e2e_steps / (e0.elapsed_time(e1) * 1e-3) / 1e9
     assert torch.equal(h_dst[0], h_src) and torch.equal(h_dst[1], h_src)
 
+    # Per-row evidence for the staged legs (§8(a) A8, A9), which the B200-mode pick
+    # leaves idle on this topology: each staged path alone, and the paper-mode pick
+    # (every path carrying bytes), each the median of 5 fused launches.
+    def med(fn, reps=5):
+        ts = []
+        for _ in range(reps + 1):
+            a0 = torch.cuda.Event(enable_timing=True)
+            a1 = torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            fn()
+            a1.record(stream)
+            a1.synchronize()
+            ts.append(a0.elapsed_time(a1) * 1e-3)
+        ts = sorted(ts[1:])
+        return ts[len(ts) // 2]
+
+    per_path = {}
+    peak, peak_src = measured_peaks()
+    paths_ = d["paths"]
+    nstage = 256 * MiB
+    for name, idx in (("relay_ring_alone", 1), ("host_pcie_alone", len(paths_) - 1)):
+        nb = [0] * len(paths_)
+        nb[idx] = nstage
+        ks = [1] + [0] * (len(paths_) - 1)
+        ks[idx] = 16
+        cfg_s = ctx.make_config(nb, ks)
+        t = med(lambda: ctx.xfer(dst, src, nstage, cfg_s, stream))
+        gbs = nstage / t / 1e9
+        if name.startswith("relay"):
+            per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "hbm",
+                              "hbm_GBps": 4 * nstage / t / 1e9, "frac": 4 * nstage / t / 1e9 / peak}
+        else:
+            per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "pcie",
+                              "peak": 64.0, "frac": gbs / 64.0,
+                              "peak_source": "PCIe Gen5 x16 nominal per direction (north star)"}
+    ctx.set_options(mode=mp.MP_MODEL_PAPER)
+    pcfg = ctx.select(0, 0, n)
+    t = med(lambda: ctx.xfer(dst, src, n, pcfg, stream))
+    pd = pcfg.as_dict()
+    per_path["paper_mode_pick_all_paths"] = {"GBps": n / t / 1e9, "bytes": pd["bytes"], "chunks": pd["chunks"],
+                                             "hbm_GBps": hbm_bytes(pd) / t / 1e9,
+                                             "frac": hbm_bytes(pd) / t / 1e9 / peak}
+    ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
+    torch.cuda.synchronize()
+    assert torch.equal(dst, src), "payload mismatch (per-path runs)"
+
     # single-path baseline: cudaMemcpyAsync device→device on the same stream (the
     # copy the paper's engine issues per chunk), same buffers and timing.
     base = None
@@ -498,6 +544,7 @@ def main():
         "per_launch_ms": {"min": per_launch[0], "median": per_launch[len(per_launch) // 2],
                           "max": per_launch[-1]},
         "baselines": base,
+        "per_path": per_path,
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, desc, cores = cpu_oracle_run(n, d, prm)

@@ -121,7 +121,26 @@ def scenario_engine(rank, world):
             assert np.array_equal(got.cpu().numpy(), exp), f"case {i} mismatch"
             c.free(p)
         dist.barrier()
-    # the reverse direction and a tag mismatch are reported, not hung
+    # bidirectional (osu_bibw-style): 0 → 1 and 1 → 0 at once, model-selected, two
+    # streams per rank, a window of 3 messages each way
+    if rank in (0, 1):
+        other = 1 - rank
+        s_tx, s_rx = torch.cuda.Stream(), torch.cuda.Stream()
+        nbi = 2 * MiB + 77
+        bufs = [c.alloc(nbi) for _ in range(3)]
+        with torch.cuda.stream(s_tx):
+            src_buf[:nbi].copy_(torch.from_numpy(synth.payload(nbi, 40 + rank)))
+        for w in range(3):
+            c.recv(bufs[w], nbi, other, tag=900 + w, stream=s_rx)
+            c.send(src_buf[:nbi], nbi, other, tag=900 + w, stream=s_tx)
+        s_tx.synchronize()
+        s_rx.synchronize()
+        exp = torch.from_numpy(synth.payload(nbi, 40 + other))
+        for w in range(3):
+            assert torch.equal(mp.as_tensor(bufs[w], nbi).cpu(), exp), f"bibw window {w}"
+            c.free(bufs[w])
+    dist.barrier()
+    # the reverse direction alone
     if rank == 1:
         src = src_buf[:MiB]
         src.copy_(torch.from_numpy(synth.payload(MiB, 9)))
