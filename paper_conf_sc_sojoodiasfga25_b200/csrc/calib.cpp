@@ -70,13 +70,13 @@ struct Bench {
 };
 
 // One direct-only fused launch dst ← src of n bytes; returns seconds.
-int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double *out) {
+int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double *out, int ctas = 0) {
   mp_ctx *c = b.c;
   std::vector<double> ts;
   for (int r = 0; r < reps + 1; ++r) {
     CKC(cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s));
     CKC(cudaEventRecord(b.e0, b.s));
-    if (int st = launch_direct_copy(c, dst, src, n, b.s)) return st;
+    if (int st = launch_direct_copy(c, dst, src, n, b.s, ctas)) return st;
     CKC(cudaEventRecord(b.e1, b.s));
     CKC(cudaEventSynchronize(b.e1));
     float ms = 0;
@@ -87,13 +87,15 @@ int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double
   return MP_OK;
 }
 
+// Fit one link.  ctas > 0 times the copy with that many CTAs: a staged leg is moved
+// by a stage group of relay_ctas CTAs, so its β is what that group achieves.
 int fit_link(Bench &b, void *dst, const void *src, const std::vector<uint64_t> &sizes, uint64_t cap,
-             int reps, Fit *f) {
+             int reps, Fit *f, int ctas = 0) {
   std::vector<double> n, t;
   for (uint64_t s : sizes) {
     if (s > cap) continue;
     double sec = 0;
-    if (int st = time_copy(b, dst, src, s, reps, &sec)) return st;
+    if (int st = time_copy(b, dst, src, s, reps, &sec, ctas)) return st;
     n.push_back(static_cast<double>(s));
     t.push_back(sec);
   }
@@ -196,7 +198,8 @@ int fit_phi(mp_ctx *c, int idx, uint64_t n, int reps, double *c_out) {
 // install a model for every ordered pair (s, d): direct and leg 1 from s, relay leg 2
 // and ε from the relay r, host leg 2 and ε from d; the shared port is s's egress.
 struct LinkMeas {
-  double da, db;          // NVLink put α, β
+  double da, db;          // NVLink put α, β (direct group)
+  double ra, rb;          // NVLink put α, β with a stage group's CTAs (relay legs)
   double h1a, h1b;        // GPU → host α, β
   double h2a, h2b;        // host → GPU α, β
   double eps_dev, eps_host;
@@ -234,6 +237,10 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
     if ((st = fit_link(b, c->peers[succ].heap, src, sz, big, reps, &fd))) break;
     m.da = fd.alpha;
     m.db = fd.beta;
+    Fit fr{};
+    if ((st = fit_link(b, c->peers[succ].heap, src, sz, big, reps, &fr, c->relay_ctas))) break;
+    m.ra = fr.alpha;
+    m.rb = fr.beta;
     if (c->host_path) {
       // the own segment's ring of sender == me is never used for traffic
       uint8_t *hr = c->hseg[me] + static_cast<uint64_t>(me) * c->hseg_per_src;
@@ -242,8 +249,8 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
       for (uint64_t s : sz)
         if (s <= std::min<uint64_t>(hcap, 64ull << 20)) hs.push_back(s);
       if (hs.size() < 2) hs = {hcap / 4, hcap / 2};
-      if ((st = fit_link(b, hr, src, hs, hcap, std::max(3, reps / 2), &fh1))) break;
-      if ((st = fit_link(b, src, hr, hs, hcap, std::max(3, reps / 2), &fh2))) break;
+      if ((st = fit_link(b, hr, src, hs, hcap, std::max(3, reps / 2), &fh1, c->relay_ctas))) break;
+      if ((st = fit_link(b, src, hr, hs, hcap, std::max(3, reps / 2), &fh2, c->relay_ctas))) break;
       m.h1a = fh1.alpha;
       m.h1b = fh1.beta;
       m.h2a = fh2.alpha;
@@ -279,7 +286,7 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
       for (int r = 0; r < W; ++r) {
         if (r == s || r == d) continue;
         paths[np] = mp_path{MP_PATH_GPU, r};
-        prm[np++] = mp_path_params{lm[s].da, lm[s].db, lm[r].da, lm[r].db, std::max(lm[r].eps_dev, 1e-8), 1, 0, 1};
+        prm[np++] = mp_path_params{lm[s].ra, lm[s].rb, lm[r].ra, lm[r].rb, std::max(lm[r].eps_dev, 1e-8), 1, 0, 1};
       }
       if (c->host_path) {
         paths[np] = mp_path{MP_PATH_HOST, -1};
@@ -353,8 +360,8 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
     if ((st = fit_link(b, dst, src, direct_sizes, big, reps, &fd))) break;
     if (c->n_loop_relays > 0) {
       uint8_t *ring = c->rings[0].data;
-      if ((st = fit_link(b, ring, src, sizes, ring_cap, reps, &f1))) break;
-      if ((st = fit_link(b, dst, ring, sizes, ring_cap, reps, &f2))) break;
+      if ((st = fit_link(b, ring, src, sizes, ring_cap, reps, &f1, c->relay_ctas))) break;
+      if ((st = fit_link(b, dst, ring, sizes, ring_cap, reps, &f2, c->relay_ctas))) break;
       if ((st = time_pingpong(b, c->d_probe, false, 2000, &eps_dev))) break;
     }
     if (c->host_path) {
@@ -362,8 +369,8 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
       std::vector<uint64_t> hs;
       for (uint64_t s : sizes)
         if (s <= std::min<uint64_t>(ring_cap, 64ull << 20)) hs.push_back(s);
-      if ((st = fit_link(b, hr, src, hs, ring_cap, std::max(3, reps / 2), &fh1))) break;
-      if ((st = fit_link(b, dst, hr, hs, ring_cap, std::max(3, reps / 2), &fh2))) break;
+      if ((st = fit_link(b, hr, src, hs, ring_cap, std::max(3, reps / 2), &fh1, c->relay_ctas))) break;
+      if ((st = fit_link(b, dst, hr, hs, ring_cap, std::max(3, reps / 2), &fh2, c->relay_ctas))) break;
       if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) break;
     }
   } while (false);

@@ -275,7 +275,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
 
 }  // namespace
 
-int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream) {
+int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream, int ctas) {
   XferParams P;
   std::memset(&P, 0, sizeof(P));
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
@@ -289,7 +289,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   d.src = static_cast<const uint8_t *>(src);
   d.dst = static_cast<uint8_t *>(dst);
   d.align = c->opts.align;
-  d.g_in = direct_ctas(c, n, c->per_sm * c->sms);
+  d.g_in = ctas > 0 ? static_cast<uint32_t>(ctas) : direct_ctas(c, n, c->per_sm * c->sms);
   P.nblocks = d.g_in;
   const int e = launch_xfer(P, stream);
   if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "copy launch");

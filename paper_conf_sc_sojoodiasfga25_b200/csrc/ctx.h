@@ -125,7 +125,8 @@ inline uint32_t direct_ctas(const mp_ctx *c, uint64_t bytes, int room) {
 }
 
 // One direct-path fused launch dst ← src (any world; dst may be peer or mapped host).
-int launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream);
+// ctas > 0 fixes the CTA count (calibration of a staged leg uses the staged group's).
+int launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, void *stream, int ctas = 0);
 int world_barrier(mp_ctx *c);
 int world_allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes);
 int world_init(mp_ctx *c);

@@ -169,10 +169,11 @@ __device__ __forceinline__ void bulk_wait_all() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
+template <int MODE>
 __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32_t r, uint32_t G,
                           uint8_t *smem, uint32_t D) {
   if ((reinterpret_cast<uintptr_t>(dst) ^ reinterpret_cast<uintptr_t>(src)) & 15u) {
-    group_copy<LD_SRC>(dst, src, len, r, G);
+    group_copy<MODE>(dst, src, len, r, G);
     return;
   }
   uint64_t head = (16u - (reinterpret_cast<uintptr_t>(src) & 15u)) & 15u;
@@ -181,8 +182,8 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
   const uint64_t tail0 = head + body;
   // head and tail (< 16 B each) by CTA 0's threads
   if (r == 0) {
-    if (threadIdx.x < head) dst[threadIdx.x] = src[threadIdx.x];
-    if (threadIdx.x < len - tail0) dst[tail0 + threadIdx.x] = src[tail0 + threadIdx.x];
+    if (threadIdx.x < head) dst[threadIdx.x] = ld1<MODE>(src + threadIdx.x);
+    if (threadIdx.x < len - tail0) dst[tail0 + threadIdx.x] = ld1<MODE>(src + tail0 + threadIdx.x);
   }
   if (threadIdx.x != 0) return;
   const uint8_t *s = src + head;
@@ -256,6 +257,8 @@ __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, ui
       if (why == 1) atomicExch(err, DERR_TIMEOUT);
       if (why) *s_abort = 1;
       fence_acq_rel_sys();
+      // the data behind the flags may next be read by TMA (async proxy) from this thread
+      asm volatile("fence.proxy.async.global;" ::: "memory");
     }
   }
   __syncthreads();
@@ -291,6 +294,17 @@ __device__ __forceinline__ uint64_t ld_volatile(const uint64_t *p) {
   return v;
 }
 
+// One CTA copies its slice of a staged chunk: TMA pipeline (copy_mode 1) or LDG/STG.
+template <int MODE>
+__device__ __forceinline__ void copy_slice(uint8_t *dst, const uint8_t *src, uint64_t len, uint8_t *smem,
+                                           uint32_t copy_mode, uint32_t stages) {
+  if (len == 0) return;
+  if (copy_mode == 1)
+    bulk_copy<MODE>(dst, src, len, 0, 1, smem, stages);
+  else
+    group_copy<MODE>(dst, src, len, 0, 1);
+}
+
 __device__ __forceinline__ void release_flag(uint64_t *flag, uint64_t value) {
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -309,9 +323,18 @@ __device__ __forceinline__ void chunk_range(const DevPath &p, uint32_t j, uint64
   *len = e - s;
 }
 
+// Slice r of G of [0, len), split on 16-byte boundaries.
+__device__ __forceinline__ void slice_of(uint64_t len, uint32_t r, uint32_t G, uint64_t *a, uint64_t *b) {
+  *a = ((len * r / G) + 15) & ~uint64_t(15);
+  uint64_t e = ((len * (r + 1) / G) + 15) & ~uint64_t(15);
+  if (r + 1 == G || e > len) e = len;
+  if (*a > e) *a = e;
+  *b = e;
+}
+
 // ------------------------------------------------------------------ roles
 
-__device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort) {
+__device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
   for (uint32_t j = 0; j < p.k; ++j) {
     uint64_t off, len;
     chunk_range(p, j, &off, &len);
@@ -319,17 +342,15 @@ __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, 
     if (!wait_flags(p.freef + s * kFlagStride, p.g_out, u, P.timeout_ns, P.err, s_abort)) return;
     const uint8_t *src = p.src + off;
     uint8_t *slot = p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(src) & 15u);
-    // slice r of the chunk, split on 16-byte boundaries of the source
-    const uint64_t a = ((len * r / p.g_in) + 15) & ~uint64_t(15);
-    uint64_t b = ((len * (r + 1) / p.g_in) + 15) & ~uint64_t(15);
-    if (r + 1 == p.g_in || b > len) b = len;
-    if (a < b) group_copy<LD_SRC>(slot + a, src + a, b - a, 0, 1);
+    uint64_t a, b;  // slice r of the chunk, split on 16-byte boundaries
+    slice_of(len, r, p.g_in, &a, &b);
+    copy_slice<LD_SRC>(slot + a, src + a, b - a, smem, P.copy_mode, P.bulk_stages);
     release_flag(p.full + s * kFlagStride + r, u + 1);
   }
 }
 
 template <int MODE>
-__device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort) {
+__device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
   for (uint32_t j = 0; j < p.k; ++j) {
     uint64_t off, len;
     chunk_range(p, j, &off, &len);
@@ -337,7 +358,9 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
     if (!wait_flags(p.full + s * kFlagStride, p.g_in, u + 1, P.timeout_ns, P.err, s_abort)) return;
     const uint8_t *slot =
         p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(p.src + off) & 15u);
-    group_copy<MODE>(p.dst + off, slot, len, r, p.g_out);
+    uint64_t a, b;
+    slice_of(len, r, p.g_out, &a, &b);
+    copy_slice<MODE>(p.dst + off + a, slot + a, b - a, smem, P.copy_mode, P.bulk_stages);
     release_flag(p.freef + s * kFlagStride + r, u + 1);
   }
 }
@@ -354,18 +377,18 @@ __global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant
     if (b >= p.cta0_in && b < p.cta0_in + p.g_in) {
       if (p.kind == DK_DIRECT)
         if (P.copy_mode == 1)
-          bulk_copy(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem, P.bulk_stages);
+          bulk_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem, P.bulk_stages);
         else
           group_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in);
       else
-        run_stage_in(p, b - p.cta0_in, P, &s_abort);
+        run_stage_in(p, b - p.cta0_in, P, &s_abort, dyn_smem);
       return;
     }
     if (p.kind == DK_STAGED && b >= p.cta0_out && b < p.cta0_out + p.g_out) {
       if (p.host_ring)
-        run_forward<LD_HOST>(p, b - p.cta0_out, P, &s_abort);
+        run_forward<LD_HOST>(p, b - p.cta0_out, P, &s_abort, dyn_smem);
       else
-        run_forward<LD_RING>(p, b - p.cta0_out, P, &s_abort);
+        run_forward<LD_RING>(p, b - p.cta0_out, P, &s_abort, dyn_smem);
       return;
     }
   }
@@ -423,15 +446,6 @@ __device__ __forceinline__ uint64_t *flags_at(uint8_t *ctrl, uint64_t base, uint
   return reinterpret_cast<uint64_t *>(ctrl + base) + (static_cast<uint64_t>(who) * slots + slot) * kFlagStride;
 }
 
-// Slice r of G of [0, len), split on 16-byte boundaries.
-__device__ __forceinline__ void slice_of(uint64_t len, uint32_t r, uint32_t G, uint64_t *a, uint64_t *b) {
-  *a = ((len * r / G) + 15) & ~uint64_t(15);
-  uint64_t e = ((len * (r + 1) / G) + 15) & ~uint64_t(15);
-  if (r + 1 == G || e > len) e = len;
-  if (*a > e) *a = e;
-  *b = e;
-}
-
 // After a CTA's stores: make them visible system-wide, count `bytes` into a peer's
 // done counter, optionally release a flag.
 __device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t *flag, uint64_t value) {
@@ -482,7 +496,7 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
   uint64_t *done = done_at(P.dst_ctrl, P.L, P.me);
   if (b < P.g_direct) {  // A7: direct NVLink stores into the receiver's heap
     if (P.copy_mode == 1)
-      bulk_copy(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct, dyn_smem, P.bulk_stages);
+      bulk_copy<LD_SRC>(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct, dyn_smem, P.bulk_stages);
     else
       group_copy<LD_SRC>(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct);
     const uint64_t share = P.direct_bytes * (b + 1) / P.g_direct - P.direct_bytes * b / P.g_direct;
@@ -521,7 +535,7 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
       uint8_t *data = slot + kSlotHdr + shift;
       uint64_t a, e;
       slice_of(len, r, P.g_stage, &a, &e);
-      if (a < e) group_copy<LD_SRC>(data + a, src + a, e - a, 0, 1);
+      copy_slice<LD_SRC>(data + a, src + a, e - a, dyn_smem, P.copy_mode, P.bulk_stages);
       if (r == 0 && threadIdx.x == 0) {
         uint64_t *h = reinterpret_cast<uint64_t *>(slot);
         h[0] = P.dst;
@@ -536,6 +550,7 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
 }
 
 __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant__ RecvParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
   __shared__ uint64_t s_k, s_q0;
   if (threadIdx.x == 0) s_abort = 0;
@@ -584,13 +599,15 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
     const uint64_t off = ld_volatile(h + 1), len = ld_volatile(h + 2), shift = ld_volatile(h + 3);
     uint64_t a, e;
     slice_of(len, r, P.g_host, &a, &e);
-    if (a < e) group_copy<LD_HOST>(P.my_heap + off + a, slot + kSlotHdr + shift + a, e - a, 0, 1);
+    copy_slice<LD_HOST>(P.my_heap + off + a, slot + kSlotHdr + shift + a, e - a, dyn_smem, P.copy_mode,
+                        P.bulk_stages);
     publish(done, e - a, P.host.freef + s * kFlagStride + r, u + 1);
   }
 }
 
 // Persistent relay (A8 step 3): CTA group s (g CTAs) forwards sender s's ring.
 __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constant__ RelayParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
   __shared__ uint64_t s_h[4];
   if (threadIdx.x == 0) s_abort = 0;
@@ -613,7 +630,8 @@ __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constan
     const uint64_t off = s_h[1], len = s_h[2], shift = s_h[3];
     uint64_t a, e;
     slice_of(len, r, P.g, &a, &e);
-    if (a < e) group_copy<LD_RING>(P.peer[dst].heap + off + a, slot + kSlotHdr + shift + a, e - a, 0, 1);
+    copy_slice<LD_RING>(P.peer[dst].heap + off + a, slot + kSlotHdr + shift + a, e - a, dyn_smem, P.copy_mode,
+                        P.bulk_stages);
     uint64_t *fr = flags_at(P.peer[sender].ctrl, P.L.relay_free, P.me, P.L.slots, s);
     publish(done_at(P.peer[dst].ctrl, P.L, sender), e - a, fr + r, u + 1);
   }
@@ -633,12 +651,12 @@ int launch_send(const SendParams &P, void *stream) {
 }
 
 int launch_recv(const RecvParams &P, void *stream) {
-  recv_kernel<<<P.nblocks, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
+  recv_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
 }
 
 int launch_relay(const RelayParams &P, void *stream) {
-  relay_kernel<<<P.world * P.g, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
+  relay_kernel<<<P.world * P.g, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
 }
 
@@ -654,6 +672,8 @@ int preload_kernels() {
   cudaFuncAttributes a;
   cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(recv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(relay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);

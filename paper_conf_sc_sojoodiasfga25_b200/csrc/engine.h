@@ -139,7 +139,7 @@ struct SendParams {
 };
 
 struct RecvParams {
-  uint32_t me, src, nblocks, g_host;
+  uint32_t me, src, nblocks, g_host, copy_mode, bulk_stages;
   uint64_t seq, bytes, tag, heap_off, done_target, timeout_ns;
   uint8_t *my_ctrl;
   uint8_t *my_heap;
@@ -154,7 +154,7 @@ struct RecvParams {
 
 struct RelayParams {
   uint32_t me, world, g;       // g CTAs per sender ring
-  uint32_t pad_;
+  uint32_t copy_mode, bulk_stages, pad_;
   uint8_t *my_ctrl;
   PeerPtrs peer[kMaxPaths];    // heap/ctrl of every rank (self: local)
   CtrlLayout L;

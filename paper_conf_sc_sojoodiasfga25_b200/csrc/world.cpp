@@ -226,6 +226,8 @@ int world_start_relay(mp_ctx *c) {
   R.me = static_cast<uint32_t>(c->rank);
   R.world = static_cast<uint32_t>(c->world);
   R.g = static_cast<uint32_t>(c->relay_ctas);
+  R.copy_mode = c->copy_mode;
+  R.bulk_stages = bulk_stages_for(c->slot_bytes);
   R.my_ctrl = c->ctrl;
   for (int r = 0; r < c->world; ++r) R.peer[r] = c->peers[r];
   R.L = c->L;
@@ -370,6 +372,8 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   P.host_stride = c->host_stride;
   P.host_slots = static_cast<uint32_t>(c->slots);
   P.g_host = c->host_path ? static_cast<uint32_t>(c->relay_ctas) : 0u;
+  P.copy_mode = c->copy_mode;
+  P.bulk_stages = bulk_stages_for(bytes);
   if (c->host_path) P.host = host_ring(c, src, c->rank);
   P.nblocks = 1 + P.g_host;
   if (int e = launch_recv(P, stream))

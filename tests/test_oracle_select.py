@@ -39,7 +39,10 @@ def test_select_invariants(seed, nrel, host, n, mode):
         else:
             assert k == 0
     assert cfg.t_pred > 0 and cfg.t_level > 0
-    assert abs(sum(cfg.theta) - 1) < 1e-9 or cfg.bytes[0] == n
+    # θ is informational: paths whose floored share fell below C_min report 0 and their
+    # bytes went to the direct path (Alg 1 lines 27-28), so Σθ <= 1.
+    assert sum(cfg.theta) <= 1 + 1e-9
+    assert all(t >= 0 for t in cfg.theta)
 
 
 @settings(max_examples=40, deadline=None)
