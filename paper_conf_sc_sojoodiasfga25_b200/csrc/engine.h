@@ -101,6 +101,8 @@ struct CtrlLayout {
   uint64_t relay_free = 0;             // [world(relay)][slots][kFlagStride]      — on the sender
   uint64_t ring_full = 0;              // [world(sender)][slots][kFlagStride]     — on the relay
   uint64_t ring_data = 0;              // [world(sender)][slots][stride]          — on the relay
+  uint64_t host_full = 0;              // [world(sender)][slots][kFlagStride]     — on the receiver
+  uint64_t host_free = 0;              // [world(receiver)][slots][kFlagStride]   — on the sender
   uint64_t probe = 0;                  // 64 B of flag words for the ε ping-pong of the predecessor
   uint64_t relay_pos = 0;              // [world(sender)] u64: relay ring position across restarts
   uint64_t total = 0;

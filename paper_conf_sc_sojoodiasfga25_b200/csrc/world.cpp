@@ -76,6 +76,8 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.done = take(static_cast<uint64_t>(world) * 128);
   L.relay_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.ring_full = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
+  L.host_full = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
+  L.host_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.probe = take(64);
   L.relay_pos = take(static_cast<uint64_t>(world) * 8);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
@@ -113,12 +115,17 @@ int map_segment(mp_ctx *c, int rank, bool create, uint8_t **out) {
   return MP_OK;
 }
 
+// The host ring of pair (src, dst): data slots in the receiver's pinned segment; the
+// flags live in device memory of the GPU that polls them — "full" in dst's control
+// block (written by src over NVLink after its PCIe data writes, ordered by a sys-scope
+// fence), "free" in src's (written by dst) — so no flag is ever polled over PCIe.
 HostRingPtrs host_ring(const mp_ctx *c, int src, int dst) {
-  uint8_t *base = c->hseg[dst] + static_cast<uint64_t>(src) * c->hseg_per_src;
   HostRingPtrs h;
-  h.data = base;
-  h.full = reinterpret_cast<uint64_t *>(base + static_cast<uint64_t>(c->slots) * c->host_stride);
-  h.freef = h.full + static_cast<uint64_t>(c->slots) * kFlagStride;
+  h.data = c->hseg[dst] + static_cast<uint64_t>(src) * c->hseg_per_src;
+  h.full = reinterpret_cast<uint64_t *>(c->peers[dst].ctrl + c->L.host_full) +
+           static_cast<uint64_t>(src) * c->slots * kFlagStride;
+  h.freef = reinterpret_cast<uint64_t *>(c->peers[src].ctrl + c->L.host_free) +
+            static_cast<uint64_t>(dst) * c->slots * kFlagStride;
   return h;
 }
 
