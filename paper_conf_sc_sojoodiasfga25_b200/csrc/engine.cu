@@ -171,7 +171,7 @@ __device__ __forceinline__ void bulk_wait_all() {
 
 template <int MODE>
 __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32_t r, uint32_t G,
-                          uint8_t *smem, uint32_t D) {
+                          uint8_t *smem, uint32_t D, bool publish_after = true) {
   if ((reinterpret_cast<uintptr_t>(dst) ^ reinterpret_cast<uintptr_t>(src)) & 15u) {
     group_copy<MODE>(dst, src, len, r, G);
     return;
@@ -194,7 +194,8 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
   if (D < 1 || D > kBulkStages) D = kBulkStages;
   uint64_t *bars = reinterpret_cast<uint64_t *>(smem + kBulkBlock * kBulkStages);
   for (uint32_t i = 0; i < D; ++i) mbar_init(smem_u32(bars + i));
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  // make the initialised barriers visible to the async proxy (no cluster: CTA scope)
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   auto blk = [&](uint64_t it, uint64_t *off, uint32_t *bytes) {
     const uint64_t o = (r + it * G) * static_cast<uint64_t>(kBulkBlock);
     *off = o;
@@ -224,7 +225,13 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
       issue_load(it - 1 + D);
     }
   }
-  bulk_wait_all();
+  if (publish_after) {
+    bulk_wait_all();  // writes complete: a flag / byte count is released next
+  } else {
+    // nothing follows in this launch: only shared memory must outlive the reads
+    // (kernel completion makes the global writes visible), as CUTLASS TMA epilogues do
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+  }
 }
 
 // ------------------------------------------------------------------ flags
@@ -377,7 +384,7 @@ __global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant
     if (b >= p.cta0_in && b < p.cta0_in + p.g_in) {
       if (p.kind == DK_DIRECT)
         if (P.copy_mode == 1)
-          bulk_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem, P.bulk_stages);
+          bulk_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in, dyn_smem, P.bulk_stages, false);
         else
           group_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in);
       else
