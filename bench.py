@@ -533,7 +533,8 @@ def main():
         "config": workload_config(args, world),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
-                     "peak_source": peak_src, "kernel": "xfer_kernel",
+                     "peak_source": peak_src,
+                     "kernel": "direct_kernel" if all(b == 0 for b in d["bytes"][1:]) else "xfer_kernel",
                      "algorithmic_bytes_per_launch": alg},
         "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n, "d2h_bytes_per_step": n},
         "gpu_launches": launches,

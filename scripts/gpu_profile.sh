@@ -10,6 +10,6 @@ timeout 600 python bench.py --save-params $OUT/params.txt > $OUT/bench.log 2>&1;
 timeout 900 python scripts/sweep.py --out $OUT/sweep.json > $OUT/sweep.log 2>&1; echo "rc=$?" >> $OUT/sweep.log
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
   python bench.py --steps 5 --warmup 3 --no-cpu-baseline --params $OUT/params.txt > $OUT/ncu_launch_bench.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:xfer_kernel -s 3 -c 1 -o $OUT/prof \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"xfer_kernel|direct_kernel" -s 3 -c 1 -o $OUT/prof \
   python bench.py --steps 5 --warmup 3 --no-cpu-baseline --params $OUT/params.txt > $OUT/ncu_full.log 2>&1
 echo done
