@@ -658,10 +658,11 @@ struct DirectArgs {
 
 __global__ void __launch_bounds__(kThreads, 4) direct_kernel(const __grid_constant__ DirectArgs A) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
-  if (A.copy_mode == 1)
-    bulk_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
-  else
-    group_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x);
+  bulk_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
+}
+
+__global__ void __launch_bounds__(kThreads, 4) direct_reg_kernel(const __grid_constant__ DirectArgs A) {
+  group_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x);
 }
 
 }  // namespace
@@ -673,7 +674,10 @@ int launch_xfer(const XferParams &P, void *stream) {
     if (P.p[i].bytes) direct_only = false;
   if (direct_only) {
     const DirectArgs A{P.p[0].dst, P.p[0].src, P.p[0].bytes, P.copy_mode, P.bulk_stages};
-    direct_kernel<<<P.nblocks, kThreads, P.copy_mode == 1 ? kBulkSmem : 0, static_cast<cudaStream_t>(stream)>>>(A);
+    if (P.copy_mode == 1)
+      direct_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(A);
+    else
+      direct_reg_kernel<<<P.nblocks, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(A);
     return static_cast<int>(cudaGetLastError());
   }
   xfer_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
@@ -712,6 +716,7 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncSetAttribute(direct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, relay_kernel);
