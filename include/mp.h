@@ -257,6 +257,13 @@ int mp_load_params(mp_ctx *ctx, const char *path);
 /* Launch statistics: number of engine kernels launched by this context so far. */
 int mp_stats(mp_ctx *ctx, uint64_t *kernel_launches);
 
+/* The Hockney fit of Step 1 (reading C12), exposed for parity tests: least squares of
+ * T = α + n/β over m samples (n[i] bytes, t[i] seconds, host arrays), each residual
+ * weighted by 1/t[i]² (relative error).  Clamps: α < 1e-7 s becomes 1e-7 (Eq 14 needs
+ * α > 0); a non-positive slope falls back to β = n[m-1]/t[m-1].  m >= 2, else
+ * MP_ERR_INVALID.  Pure host arithmetic, no context. */
+int mp_fit_hockney(const double *n, const double *t, int m, double *alpha, double *beta);
+
 #ifdef __cplusplus
 }
 #endif

@@ -301,6 +301,16 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
 
 }  // namespace
 
+extern "C" int mp_fit_hockney(const double *n, const double *t, int m, double *alpha, double *beta) {
+  if (!n || !t || !alpha || !beta || m < 2) return MP_ERR_INVALID;
+  for (int i = 0; i < m; ++i)
+    if (!(t[i] > 0.0) || !(n[i] >= 0.0)) return MP_ERR_INVALID;
+  const Fit f = fit_hockney(std::vector<double>(n, n + m), std::vector<double>(t, t + m));
+  *alpha = f.alpha;
+  *beta = f.beta;
+  return MP_OK;
+}
+
 extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");

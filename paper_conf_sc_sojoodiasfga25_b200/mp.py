@@ -108,6 +108,8 @@ def lib():
             "mp_save_params": (C.c_int, [P, C.c_char_p]),
             "mp_load_params": (C.c_int, [P, C.c_char_p]),
             "mp_stats": (C.c_int, [P, C.POINTER(C.c_uint64)]),
+            "mp_fit_hockney": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
+                                         C.POINTER(C.c_double), C.POINTER(C.c_double)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -121,7 +123,17 @@ def exported_symbols() -> List[str]:
     return ["mp_init", "mp_finalize", "mp_strerror", "mp_last_error", "mp_abi_version", "mp_paths",
             "mp_set_model", "mp_get_model", "mp_set_options", "mp_get_options", "mp_predict",
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
-            "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats"]
+            "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney"]
+
+
+def fit_hockney(n: Sequence[float], t: Sequence[float]):
+    """mp_fit_hockney: (α, β) of the Step-1 weighted Hockney fit (reading C12)."""
+    m = len(n)
+    a, b = C.c_double(), C.c_double()
+    st = lib().mp_fit_hockney((C.c_double * m)(*n), (C.c_double * m)(*t), m, C.byref(a), C.byref(b))
+    if st != 0:
+        raise MPError(st, "mp_fit_hockney")
+    return a.value, b.value
 
 
 def _ptr(x) -> Optional[int]:
