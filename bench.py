@@ -240,6 +240,34 @@ def run_world(args, world, rank, local):
     assert torch.equal(src, src.clone())
     torch.cuda.synchronize()
 
+    # Baseline (context, not the product): NCCL send/recv between the same pairs,
+    # measured before mp_init so no NCCL kernel ever runs beside the relay kernel.
+    base = {}
+    if os.environ.get("MPX_BENCH_SAME_GPU") != "1":
+        try:
+            g_nccl = dist.new_group(backend="nccl")
+            nb_steps = max(3, min(args.steps, 20))
+            for it in range(nb_steps + 2):
+                if it == 2:
+                    torch.cuda.synchronize()
+                    b0 = time.perf_counter()
+                if active:
+                    if sender:
+                        dist.send(src, peer, group=g_nccl)
+                    else:
+                        dist.recv(src, peer, group=g_nccl)
+            torch.cuda.synchronize()
+            tb = torch.tensor([time.perf_counter() - b0 if active else 0.0], dtype=torch.float64)
+            dist.all_reduce(tb, op=dist.ReduceOp.MAX)
+            base["nccl_send_recv_GBps_per_pair"] = n * nb_steps / float(tb[0]) / 1e9
+            dist.destroy_process_group(g_nccl)
+            if not sender and active:   # restore the sender's payload on the receiver
+                src.copy_(torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                                        generator=torch.Generator(device="cuda").manual_seed(20251116 + peer)))
+            torch.cuda.synchronize()
+        except Exception as exc:
+            base["nccl_error"] = repr(exc)
+
     ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
                                   timeout_s=60.0)
     ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
@@ -300,6 +328,34 @@ def run_world(args, world, rank, local):
     dist.all_reduce(e, op=dist.ReduceOp.MAX)
     e2e = n * npairs * e2e_steps / (float(e[0]) * 1e-3) / 1e9
 
+    # Baseline: the single-path copy-engine peer copy (what cudaMemcpyPeerAsync does):
+    # cudaMemcpyAsync from the sender's buffer into the receiver's heap buffer through
+    # its IPC mapping.
+    try:
+        from cuda.bindings import runtime as rt
+        offs = [None] * world
+        dist.all_gather_object(offs, (rbuf - ctx.peer_base(rank)) if rbuf else None)
+        ce_t = 0.0
+        if sender:
+            dptr = ctx.peer_base(peer) + offs[peer]
+            kind = rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice
+            c0 = torch.cuda.Event(enable_timing=True)
+            c1 = torch.cuda.Event(enable_timing=True)
+            for _ in range(2):
+                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, stream.cuda_stream)
+            c0.record(stream)
+            nb_steps = max(3, min(args.steps, 20))
+            for _ in range(nb_steps):
+                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, stream.cuda_stream)
+            c1.record(stream)
+            stream.synchronize()
+            ce_t = c0.elapsed_time(c1) * 1e-3 / nb_steps
+        tt = torch.tensor([ce_t], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        base["cudaMemcpy_peer_GBps_per_pair"] = n / float(tt[0]) / 1e9
+    except Exception as exc:
+        base["peer_copy_error"] = repr(exc)
+
     nvl = sum(b for (k, _), b in zip(d["paths"], d["bytes"]) if k != 2)
     per_pair = n * args.steps / (ms * 1e-3) / 1e9
     achieved = nvl * args.steps / (ms * 1e-3) / 1e9
@@ -316,6 +372,7 @@ def run_world(args, world, rank, local):
                      "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
                      "kernel": "send_kernel"},
         "per_pair_GBps": per_pair,
+        "baselines": base,
         "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n * npairs, "d2h_bytes_per_step": n * npairs},
         "gpu_launches": int(sm[1]),
         "clocks": clk.summary(),

@@ -208,6 +208,12 @@ int mp_select(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t path_mask,
 int mp_alloc(mp_ctx *ctx, uint64_t bytes, void **dptr);
 int mp_free(mp_ctx *ctx, void *dptr);
 
+/* The base address, valid in this process, of rank `rank`'s receive heap (its own
+ * heap for rank == ctx's rank; the IPC mapping otherwise).  Lets a caller address a
+ * peer's mp_alloc buffer by (base + offset), e.g. for one-sided copies or baselines.
+ * Errors: MP_ERR_STATE (model-only), MP_ERR_TOPOLOGY (no such rank). */
+int mp_peer_base(mp_ctx *ctx, int rank, void **base);
+
 /* ---------------------------------------------------------------- transfer */
 
 /* Send `bytes` bytes at device pointer `buf` to rank dst with `tag`.  cfg = NULL

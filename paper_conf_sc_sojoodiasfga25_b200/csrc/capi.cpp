@@ -617,6 +617,19 @@ int mp_free(mp_ctx *c, void *dptr) {
   return MP_OK;
 }
 
+int mp_peer_base(mp_ctx *c, int rank, void **base) {
+  if (!c || !base) return fail(c, MP_ERR_INVALID, "null argument");
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  if (rank < 0 || rank >= c->world) return fail(c, MP_ERR_TOPOLOGY, "no such rank");
+  if (rank == c->rank || c->peers.empty()) {
+    if (rank != c->rank) return fail(c, MP_ERR_TOPOLOGY, "no such rank");
+    *base = c->heap.base;
+  } else {
+    *base = c->peers[rank].heap;
+  }
+  return MP_OK;
+}
+
 int mp_xfer(mp_ctx *c, void *dst, const void *src, uint64_t bytes, const mp_config *cfg,
             void *stream) {
   if (!c) return MP_ERR_INVALID;

@@ -108,6 +108,7 @@ def lib():
             "mp_save_params": (C.c_int, [P, C.c_char_p]),
             "mp_load_params": (C.c_int, [P, C.c_char_p]),
             "mp_stats": (C.c_int, [P, C.POINTER(C.c_uint64)]),
+            "mp_peer_base": (C.c_int, [P, C.c_int, C.POINTER(P)]),
             "mp_fit_hockney": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                          C.POINTER(C.c_double), C.POINTER(C.c_double)]),
         }
@@ -123,7 +124,8 @@ def exported_symbols() -> List[str]:
     return ["mp_init", "mp_finalize", "mp_strerror", "mp_last_error", "mp_abi_version", "mp_paths",
             "mp_set_model", "mp_get_model", "mp_set_options", "mp_get_options", "mp_predict",
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
-            "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney"]
+            "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
+            "mp_peer_base"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -265,6 +267,11 @@ class Context:
 
     def free(self, p):
         self._ck(lib().mp_free(self.h, p))
+
+    def peer_base(self, rank) -> int:
+        v = C.c_void_p()
+        self._ck(lib().mp_peer_base(self.h, rank, C.byref(v)))
+        return v.value
 
     def xfer(self, dst, src, n, cfg: Optional[mp_config] = None, stream=None):
         self._ck(lib().mp_xfer(self.h, _ptr(dst), _ptr(src), n, C.byref(cfg) if cfg else None,
