@@ -31,16 +31,17 @@ def main():
     ctx = mdist.context_from_dist(device=dev, heap_bytes=n + 64 * MiB, timeout_s=30.0)
     ps = ctx.paths(0, 1)
     buf = ctx.alloc(n) if rank == 1 else None
-    cases = {"direct": [n] + [0] * (len(ps) - 1)}
+    cases = {"direct": ([n] + [0] * (len(ps) - 1), None)}
     hb = [0] * len(ps)
     hb[-1] = n
-    cases["host"] = hb
+    for k in (1, 2, 4, 8, 16):
+        cases[f"host_k{k}"] = (hb, k)
     if world >= 3:
         rb = [0] * len(ps)
         rb[1] = n
-        cases["relay"] = rb
-    for name, nb in cases.items():
-        ks = [1] + [(max(1, b // (8 * MiB)) if b else 0) for b in nb[1:]]
+        cases["relay"] = (rb, None)
+    for name, (nb, kf) in cases.items():
+        ks = [1] + [((kf or max(1, b // (8 * MiB))) if b else 0) for b in nb[1:]]
         cfg = ctx.make_config(nb, ks, 0, 1)
         dist.barrier()
         t0 = time.perf_counter()
