@@ -1,5 +1,7 @@
 // capi.cpp — the C ABI of include/mp.h: context lifetime, model calls, heap,
 // loopback transfer launcher.  PAPER.md §4 (Steps 1-5; Alg 1).
+#include <sys/mman.h>
+
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
@@ -137,7 +139,12 @@ int check_err(mp_ctx *c) {
 void free_engine(mp_ctx *c) {
   for (auto &r : c->rings) {
     if (r.host) {
-      if (r.data) cudaFreeHost(r.data);
+      if (r.data && r.registered) {
+        cudaHostUnregister(r.data);
+        munmap(r.data, r.data_bytes);
+      } else if (r.data) {
+        cudaFreeHost(r.data);
+      }
       if (r.full) cudaFree(r.full);
     } else {
       if (r.data) cudaFree(r.data);
@@ -167,7 +174,16 @@ int alloc_ring(mp_ctx *c, bool host, Ring *r) {
     // polling never crosses PCIe (measured: host-resident flags polled by 16-32 CTAs
     // cut the host path to 9-22 GB/s, profiles/r01/diag_host.jsonl)
     void *d = nullptr, *f = nullptr;
-    CK(cudaHostAlloc(&d, data_bytes, cudaHostAllocMapped | cudaHostAllocPortable));
+    const char *reg = std::getenv("MPX_HOSTRING_REGISTER");  // diagnostics: shm-like pages
+    if (reg && reg[0] == '1') {
+      d = mmap(nullptr, data_bytes, PROT_READ | PROT_WRITE, MAP_SHARED | MAP_ANONYMOUS, -1, 0);
+      if (d == MAP_FAILED) return fail(c, MP_ERR_NOMEM, "mmap host ring");
+      CK(cudaHostRegister(d, data_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable));
+      r->registered = true;
+    } else {
+      CK(cudaHostAlloc(&d, data_bytes, cudaHostAllocMapped | cudaHostAllocPortable));
+    }
+    r->data_bytes = data_bytes;
     r->data = static_cast<uint8_t *>(d);
     CK(cudaMalloc(&f, flag_bytes));
     CK(cudaMemset(f, 0, flag_bytes));

@@ -23,6 +23,8 @@ struct Ring {
   uint64_t *full = nullptr;    // [slots][kFlagStride]
   uint64_t *freef = nullptr;   // [slots][kFlagStride]
   bool host = false;
+  bool registered = false;     // host data from mmap + cudaHostRegister (diagnostics)
+  uint64_t data_bytes = 0;
   uint64_t q = 0;              // next ring sequence number (chunks issued so far)
 };
 
