@@ -28,7 +28,9 @@ def main():
     s = torch.cuda.Stream()
     src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()
-    ctx = mdist.context_from_dist(device=dev, heap_bytes=n + 64 * MiB, timeout_s=30.0)
+    ctx = mdist.context_from_dist(device=dev, heap_bytes=n + 64 * MiB, timeout_s=30.0,
+                                  relay_ctas=int(os.environ.get("DIAG_CTAS", "16")),
+                                  slots=int(os.environ.get("DIAG_SLOTS", "4")))
     ps = ctx.paths(0, 1)
     buf = ctx.alloc(n) if rank == 1 else None
     cases = {"direct": ([n] + [0] * (len(ps) - 1), None)}
@@ -60,7 +62,7 @@ def main():
         out = [None] * world
         dist.all_gather_object(out, (rank, ms, wall))
         if rank == 0:
-            print(json.dumps({"case": name, "bytes": nb, "chunks": ks, "per_msg_ms": {r: m / K for r, m, _ in out},
+            print(json.dumps({"case": name, "ctas": os.environ.get("DIAG_CTAS", "16"), "slots": os.environ.get("DIAG_SLOTS", "4"), "bytes": nb, "chunks": ks, "per_msg_ms": {r: m / K for r, m, _ in out},
                               "GBps": n * K / (max(m for _, m, _ in out) * 1e-3) / 1e9}), flush=True)
     ctx.sync()
     if buf:
