@@ -186,6 +186,9 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
     if (threadIdx.x < len - tail0) dst[tail0 + threadIdx.x] = ld1<MODE>(src + tail0 + threadIdx.x);
   }
   if (threadIdx.x != 0) return;
+  // data published by another agent (acquired by this CTA before the barrier that
+  // preceded this call) is about to be read through the async proxy
+  if (MODE != LD_SRC) asm volatile("fence.proxy.async.global;" ::: "memory");
   const uint8_t *s = src + head;
   uint8_t *d = dst + head;
   const uint64_t nblk = (body + kBulkBlock - 1) / kBulkBlock;
@@ -263,9 +266,6 @@ __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, ui
     if (lane == 0) {
       if (why == 1) atomicExch(err, DERR_TIMEOUT);
       if (why) *s_abort = 1;
-      fence_acq_rel_sys();
-      // the data behind the flags may next be read by TMA (async proxy) from this thread
-      asm volatile("fence.proxy.async.global;" ::: "memory");
     }
   }
   __syncthreads();
@@ -285,7 +285,6 @@ __device__ __forceinline__ bool wait_word(const uint64_t *w, uint64_t target, ui
       }
       __nanosleep(64);
     }
-    fence_acq_rel_sys();
   }
   __syncthreads();
   return *s_abort == 0;
@@ -314,10 +313,7 @@ __device__ __forceinline__ void copy_slice(uint8_t *dst, const uint8_t *src, uin
 
 __device__ __forceinline__ void release_flag(uint64_t *flag, uint64_t value) {
   __syncthreads();
-  if (threadIdx.x == 0) {
-    fence_acq_rel_sys();
-    st_release_sys(flag, value);
-  }
+  if (threadIdx.x == 0) st_release_sys(flag, value);
 }
 
 // Reading C6: chunk j of a staged share [0, bytes) in units of A.
@@ -455,11 +451,24 @@ __device__ __forceinline__ uint64_t *flags_at(uint8_t *ctrl, uint64_t base, uint
 
 // After a CTA's stores: make them visible system-wide, count `bytes` into a peer's
 // done counter, optionally release a flag.
-__device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t *flag, uint64_t value) {
+// The release operations carry the ordering themselves (bar.sync makes the CTA's
+// prior writes precede thread 0's release, which is cumulative); no separate
+// fence.acq_rel.sys — measured to cost ~18 µs per CTA per chunk on the multi-rank
+// host path.  A byte counter on this same GPU only needs gpu scope.
+__device__ __forceinline__ void red_add_release_gpu(uint64_t *p, uint64_t v) {
+  asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t *flag, uint64_t value,
+                                        bool done_is_local = false) {
   __syncthreads();
   if (threadIdx.x == 0) {
-    fence_acq_rel_sys();
-    if (done && bytes) red_add_release_sys(done, bytes);
+    if (done && bytes) {
+      if (done_is_local)
+        red_add_release_gpu(done, bytes);
+      else
+        red_add_release_sys(done, bytes);
+    }
     if (flag) st_release_sys(flag, value);
   }
 }
@@ -608,7 +617,7 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
     slice_of(len, r, P.g_host, &a, &e);
     copy_slice<LD_HOST>(P.my_heap + off + a, slot + kSlotHdr + shift + a, e - a, dyn_smem, P.copy_mode,
                         P.bulk_stages);
-    publish(done, e - a, P.host.freef + s * kFlagStride + r, u + 1);
+    publish(done, e - a, P.host.freef + s * kFlagStride + r, u + 1, /*done_is_local=*/true);
   }
 }
 
