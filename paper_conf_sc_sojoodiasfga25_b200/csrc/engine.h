@@ -81,9 +81,10 @@ int launch_xfer(const XferParams &P, void *stream);
 constexpr uint32_t kCtsRing = 64;     // outstanding messages per ordered pair
 constexpr uint32_t kSlotHdr = 256;    // slot header bytes
 
-struct MsgEntry {                      // CTS and message-header entries (32 B)
+struct MsgEntry {                      // CTS and message-header entries (64 B)
   uint64_t seq1;                       // sequence + 1 (written last, with release)
   uint64_t a, b, c;                    // CTS: heap_off, bytes, tag; HDR: host_k, host_q0, status
+  uint64_t d, e, f, g;                 // HDR: host range heap offset, host bytes, src shift (mod 16)
 };
 
 struct PeerPtrs {
