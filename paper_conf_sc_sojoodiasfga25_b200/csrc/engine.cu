@@ -473,45 +473,58 @@ __device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t
   }
 }
 
+// The rendezvous (P:62 analogue) runs in its own one-CTA launch ahead of the bulk
+// send kernel on the same stream: the bulk kernel's hundreds of CTAs are only
+// dispatched once the receiver's clear-to-send has arrived, so they never occupy SM
+// slots spinning on it while a receive kernel on this GPU waits for room to run.
+__global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
+  if (threadIdx.x != 0) return;
+  MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
+  const uint64_t t_start = globaltimer();
+  while (ld_acquire_sys(&cts->seq1) < P.seq + 1) {
+    if (globaltimer() - t_start > P.timeout_ns) {
+      atomicExch(P.err, DERR_TIMEOUT);
+      return;
+    }
+    __nanosleep(64);
+  }
+  const uint64_t off = ld_volatile(&cts->a), n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
+  const bool bad = (n != P.bytes) || (tag != P.tag);
+  uint64_t host_k = 0, host_q0 = 0, host_off = 0, host_bytes = 0;
+  for (uint32_t i = 0; i < P.npaths; ++i)
+    if (P.sp[i].kind == 2) {
+      host_k = P.sp[i].k;
+      host_q0 = P.sp[i].q0;
+      host_off = P.sp[i].off;
+      host_bytes = P.sp[i].bytes;
+    }
+  // the receiver's host-ring consumers take the chunk layout from here (device
+  // memory) — never from the slot headers in host memory, whose PCIe reads queue
+  // behind the bulk traffic (measured ~18 µs per CTA per chunk)
+  MsgEntry *h = entry_at(P.dst_ctrl, P.L.hdr, P.me, P.seq);
+  h->a = bad ? 0 : host_k;
+  h->b = host_q0;
+  h->c = bad ? 2 : 0;
+  h->d = off + host_off;
+  h->e = host_bytes;
+  h->f = reinterpret_cast<uintptr_t>(P.src + host_off) & 15u;
+  st_release_sys(&h->seq1, P.seq + 1);
+  if (bad) atomicExch(P.err, DERR_MISMATCH);
+}
+
 __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant__ SendParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
   __shared__ uint64_t s_off;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
-  // wait for the receiver's clear-to-send (rendezvous, P:62 analogue)
+  // the clear-to-send has arrived (send_gate_kernel ran first on this stream)
   MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
   if (!wait_word(&cts->seq1, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
   if (threadIdx.x == 0) {
     const uint64_t off = ld_volatile(&cts->a), n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
     s_off = off;
-    const bool bad = (n != P.bytes) || (tag != P.tag);
-    if (blockIdx.x == 0) {
-      uint64_t host_k = 0, host_q0 = 0, host_off = 0, host_bytes = 0;
-      for (uint32_t i = 0; i < P.npaths; ++i)
-        if (P.sp[i].kind == 2) {
-          host_k = P.sp[i].k;
-          host_q0 = P.sp[i].q0;
-          host_off = P.sp[i].off;
-          host_bytes = P.sp[i].bytes;
-        }
-      // the receiver's host-ring consumers take the chunk layout from here (device
-      // memory) — never from the slot headers in host memory, whose PCIe reads queue
-      // behind the bulk traffic (measured ~18 µs per CTA per chunk)
-      MsgEntry *h = entry_at(P.dst_ctrl, P.L.hdr, P.me, P.seq);
-      h->a = bad ? 0 : host_k;
-      h->b = host_q0;
-      h->c = bad ? 2 : 0;
-      h->d = off + host_off;
-      h->e = host_bytes;
-      h->f = reinterpret_cast<uintptr_t>(P.src + host_off) & 15u;
-      fence_acq_rel_sys();
-      st_release_sys(&h->seq1, P.seq + 1);
-    }
-    if (bad) {
-      atomicExch(P.err, DERR_MISMATCH);
-      s_abort = 1;
-    }
+    if ((n != P.bytes) || (tag != P.tag)) s_abort = 1;  // reported by the gate
   }
   __syncthreads();
   if (s_abort) return;
@@ -705,6 +718,7 @@ int launch_xfer(const XferParams &P, void *stream) {
 }
 
 int launch_send(const SendParams &P, void *stream) {
+  send_gate_kernel<<<1, 32, 0, static_cast<cudaStream_t>(stream)>>>(P);
   send_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
 }
@@ -738,6 +752,7 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_gate_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, relay_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, pingpong_kernel);

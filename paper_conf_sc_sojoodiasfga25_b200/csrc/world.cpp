@@ -346,7 +346,7 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   P.nblocks = next;
   if (int e = launch_send(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
-  c->launches += 1;
+  c->launches += 2;  // rendezvous gate + bulk send kernel
   c->send_seq[dst] += 1;
   for (auto &a : advance) {
     if (a.first < 0)
