@@ -660,6 +660,16 @@ int mp_xfer(mp_ctx *c, void *dst, const void *src, uint64_t bytes, const mp_conf
     cfg = &sel;
   }
   if (int s = check_config(c, *m, bytes, cfg)) return s;
+  // CUDA-graph capture: a direct-only transfer is a pure kernel and replays
+  // correctly; a staged one advances the rings' sequence numbers on the host at
+  // launch, which a replay would not repeat, so it is refused while capturing.
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(static_cast<cudaStream_t>(stream), &cap) == cudaSuccess &&
+      cap != cudaStreamCaptureStatusNone) {
+    for (int i = 1; i < cfg->npaths; ++i)
+      if (cfg->bytes[i])
+        return fail(c, MP_ERR_UNSUPPORTED, "staged paths cannot be captured in a CUDA graph (direct-only can)");
+  }
   return launch_loopback(c, dst, src, bytes, *cfg, stream);
 }
 

@@ -155,6 +155,36 @@ def test_send_recv_loopback(ctx):
     assert e.value.status == -8
 
 
+def test_cuda_graph_capture_direct_only(ctx):
+    # launch-bound windows can be captured in a CUDA graph when the config is
+    # direct-only (a pure kernel); staged configs are refused while capturing
+    n = 3 * MiB + 5
+    ps = ctx.paths()
+    src = torch.from_numpy(synth.payload(n, 21)).cuda()
+    dsts = [torch.zeros(n, dtype=torch.uint8, device="cuda") for _ in range(4)]
+    cfg = ctx.make_config([n] + [0] * (len(ps) - 1), [1] + [0] * (len(ps) - 1))
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for d in dsts:
+            ctx.xfer(d, src, n, cfg, torch.cuda.current_stream())
+    for d in dsts:
+        d.zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    for d in dsts:
+        assert torch.equal(d, src)
+    nb = [0] * len(ps)
+    nb[0], nb[1] = n - 512 * 1024, 512 * 1024
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1] = 2
+    g2 = torch.cuda.CUDAGraph()
+    with pytest.raises(mp.MPError) as e:
+        with torch.cuda.graph(g2, stream=s):
+            ctx.xfer(dsts[0], src, n, ctx.make_config(nb, ks), torch.cuda.current_stream())
+    assert e.value.status == -6
+
+
 def test_launch_counter(ctx):
     a = ctx.launches()
     n = MiB
