@@ -104,6 +104,58 @@ int fit_link(Bench &b, void *dst, const void *src, const std::vector<uint64_t> &
   return MP_OK;
 }
 
+// Two links timed concurrently (dst1 ← src1 on one stream, dst2 ← src2 on another,
+// launched together), each fitted on its own times.
+int fit_links_duplex(Bench &b, void *dst1, const void *src1, void *dst2, const void *src2,
+                     const std::vector<uint64_t> &sizes, int reps, Fit *f1, Fit *f2, int ctas) {
+  mp_ctx *c = b.c;
+  cudaStream_t s2 = nullptr;
+  cudaEvent_t fork = nullptr, e2a = nullptr, e2b = nullptr;
+  CKC(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+  CKC(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming));
+  CKC(cudaEventCreate(&e2a));
+  CKC(cudaEventCreate(&e2b));
+  std::vector<double> n, t1, t2;
+  int st = MP_OK;
+  for (uint64_t s : sizes) {
+    std::vector<double> a, bb;
+    for (int r = 0; r < reps + 1 && st == MP_OK; ++r) {
+      cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s);
+      cudaEventRecord(fork, b.s);
+      cudaStreamWaitEvent(s2, fork, 0);
+      cudaEventRecord(b.e0, b.s);
+      cudaEventRecord(e2a, s2);
+      st = launch_direct_copy(c, dst1, src1, s, b.s, ctas);
+      if (!st) st = launch_direct_copy(c, dst2, src2, s, s2, ctas);
+      cudaEventRecord(b.e1, b.s);
+      cudaEventRecord(e2b, s2);
+      cudaEventSynchronize(b.e1);
+      cudaEventSynchronize(e2b);
+      float ms1 = 0, ms2 = 0;
+      cudaEventElapsedTime(&ms1, b.e0, b.e1);
+      cudaEventElapsedTime(&ms2, e2a, e2b);
+      if (r > 0) {
+        a.push_back(ms1 * 1e-3);
+        bb.push_back(ms2 * 1e-3);
+      }
+    }
+    if (st) break;
+    n.push_back(static_cast<double>(s));
+    t1.push_back(median(a));
+    t2.push_back(median(bb));
+  }
+  cudaStreamSynchronize(s2);
+  cudaStreamDestroy(s2);
+  cudaEventDestroy(fork);
+  cudaEventDestroy(e2a);
+  cudaEventDestroy(e2b);
+  if (st) return st;
+  if (n.size() < 2) return cfail(c, MP_ERR_INVALID, "calibration needs at least two sizes");
+  *f1 = fit_hockney(n, t1);
+  *f2 = fit_hockney(n, t2);
+  return MP_OK;
+}
+
 int time_pingpong(Bench &b, uint64_t *flags, bool host, int iters, double *eps) {
   mp_ctx *c = b.c;
   if (host)
@@ -378,9 +430,14 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
       uint8_t *hr = c->rings[c->n_loop_relays].data;
       std::vector<uint64_t> hs;
       for (uint64_t s : sizes)
-        if (s <= std::min<uint64_t>(ring_cap, 64ull << 20)) hs.push_back(s);
-      if ((st = fit_link(b, hr, src, hs, ring_cap, std::max(3, reps / 2), &fh1, c->relay_ctas))) break;
-      if ((st = fit_link(b, dst, hr, hs, ring_cap, std::max(3, reps / 2), &fh2, c->relay_ctas))) break;
+        if (s <= std::min<uint64_t>(ring_cap / 2, 64ull << 20)) hs.push_back(s);
+      if (hs.size() < 2) hs = {ring_cap / 8, ring_cap / 4};
+      // On one GPU both host legs share its PCIe link (writes up, reads down at the
+      // same time in the pipelined path): time them concurrently, so β and β' are
+      // the full-duplex rates the staged path actually sees.
+      if ((st = fit_links_duplex(b, hr, src, dst, hr + ring_cap / 2, hs, std::max(3, reps / 2), &fh1, &fh2,
+                                 c->relay_ctas)))
+        break;
       if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) break;
     }
   } while (false);
