@@ -13,9 +13,9 @@ N = 1 (default): BASELINE.json config 3 — 1 GiB, direct + 6 relays + pinned ho
 on the single-GPU loopback engine (the relay rings stand in for the intermediate
 GPUs; the host leg is real PCIe); the config is the B200-mode model's pick after an
 init-time calibration (Step 1).  Inputs are 1 GiB (> 126 MB L2), so no flush.
-N > 1 (torchrun): config 5's "pairs" reading — ranks (2i, 2i+1) exchange one
-message per step through the multi-rank engine, all pairs concurrently
-("scaling": "weak"; value = bytes of all pairs / max-over-ranks time).
+N > 1 (torchrun): config 5, disjoint pairs (2i ↔ 2i+1) exchanging one 256 MiB
+message each way per step through the multi-rank engine, all pairs concurrently
+("scaling": "weak"; value = bytes moved by all ranks / max-over-ranks time).
 
 --impl reference: the CPU oracle (oracle/, fp64 model + memcpy replay) on a bounded
 sample of the same workload, rank 0 only.
@@ -211,12 +211,14 @@ def workload_config(args, world):
 
 
 def run_world(args, world, rank, local):
-    """N > 1 (torchrun, one process per GPU): BASELINE.json config 5 reading "pairs":
-    ranks (2i, 2i+1) exchange one message per step, 2i → 2i+1, all pairs at once,
-    through the multi-rank engine (IPC-mapped heaps, NVLink direct path, relays
-    through the other GPUs, pinned-host PCIe path), model-selected after a
-    collective calibration.  Bootstrap and the max-over-ranks reduction use gloo on
-    CPU: no NCCL kernel ever runs next to the persistent relay kernel."""
+    """N > 1 (torchrun, one process per GPU): BASELINE.json config 5, SURVEY §8(d)'s
+    primary reading — disjoint pairs (0↔1, 2↔3, …) exchange one message each way per
+    step, all pairs at once, so every GPU's NVLink egress and ingress are busy and
+    every would-be relay is itself an endpoint.  Messages go through the multi-rank
+    engine (IPC-mapped heaps, direct NVLink path, relays through the other GPUs,
+    pinned-host PCIe path), model-selected after a collective calibration.
+    value = bytes moved by all ranks / max-over-ranks time.  Bootstrap and the
+    reductions use gloo on CPU: no NCCL kernel ever runs beside the relay kernel."""
     import torch
     import torch.distributed as dist
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
@@ -228,42 +230,39 @@ def run_world(args, world, rank, local):
     n = args.size
     peer = rank + 1 if rank % 2 == 0 else rank - 1
     active = peer < world
-    sender = active and rank % 2 == 0
     npairs = world // 2
     # Initialise every CUDA kernel this process will use BEFORE mp_init.
-    stream = torch.cuda.Stream()
-    g = torch.Generator(device="cuda").manual_seed(20251116 + (rank if sender else peer))
-    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g)
-    h_buf = torch.empty(n, dtype=torch.uint8).pin_memory()
-    h_buf.copy_(src)
-    src.copy_(h_buf, non_blocking=True)
+    s_tx, s_rx = torch.cuda.Stream(), torch.cuda.Stream()
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                        generator=torch.Generator(device="cuda").manual_seed(20251116 + rank))
+    expect = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                           generator=torch.Generator(device="cuda").manual_seed(20251116 + peer))
+    h_src = torch.empty(n, dtype=torch.uint8).pin_memory()
+    h_dst = torch.empty(n, dtype=torch.uint8).pin_memory()
+    h_src.copy_(src)
     assert torch.equal(src, src.clone())
     torch.cuda.synchronize()
 
-    # Baseline (context, not the product): NCCL send/recv between the same pairs,
-    # measured before mp_init so no NCCL kernel ever runs beside the relay kernel.
+    # Baseline (context, not the product): NCCL send/recv between the same pairs, both
+    # directions, measured before mp_init so no NCCL kernel runs beside the relay.
     base = {}
-    if os.environ.get("MPX_BENCH_SAME_GPU") != "1":
+    if os.environ.get("MPX_BENCH_SAME_GPU") != "1" and active:
         try:
             g_nccl = dist.new_group(backend="nccl")
+            scratch = torch.empty_like(src)
             nb_steps = max(3, min(args.steps, 20))
             for it in range(nb_steps + 2):
                 if it == 2:
                     torch.cuda.synchronize()
                     b0 = time.perf_counter()
-                if active:
-                    if sender:
-                        dist.send(src, peer, group=g_nccl)
-                    else:
-                        dist.recv(src, peer, group=g_nccl)
+                ops = [dist.P2POp(dist.isend, src, peer, g_nccl), dist.P2POp(dist.irecv, scratch, peer, g_nccl)]
+                for w in dist.batch_isend_irecv(ops):
+                    w.wait()
             torch.cuda.synchronize()
-            tb = torch.tensor([time.perf_counter() - b0 if active else 0.0], dtype=torch.float64)
-            dist.all_reduce(tb, op=dist.ReduceOp.MAX)
-            base["nccl_send_recv_GBps_per_pair"] = n * nb_steps / float(tb[0]) / 1e9
+            tb = time.perf_counter() - b0
+            base["nccl_send_recv_GBps_per_direction"] = n * nb_steps / tb / 1e9
             dist.destroy_process_group(g_nccl)
-            if not sender and active:   # restore the sender's payload on the receiver
-                src.copy_(torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
-                                        generator=torch.Generator(device="cuda").manual_seed(20251116 + peer)))
+            del scratch
             torch.cuda.synchronize()
         except Exception as exc:
             base["nccl_error"] = repr(exc)
@@ -272,33 +271,33 @@ def run_world(args, world, rank, local):
                                   timeout_s=60.0)
     ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
     d = ctx.select(0, 1, n).as_dict()
-    rbuf = ctx.alloc(n) if active and not sender else None
+    rbuf = ctx.alloc(n) if active else None
     rview = mp.as_tensor(rbuf, n) if rbuf else None
 
     def step():
-        if not active:
-            return
-        if sender:
-            ctx.send(src, n, peer, 0, None, stream)
-        else:
-            ctx.recv(rbuf, n, peer, 0, stream)
+        if active:
+            ctx.recv(rbuf, n, peer, 0, s_rx)
+            ctx.send(src, n, peer, 0, None, s_tx)
 
     for _ in range(args.warmup):
         step()
-    stream.synchronize()
+    s_tx.synchronize()
+    s_rx.synchronize()
     ctx.sync()
-    if active and not sender:
-        assert torch.equal(rview, src), "payload mismatch"   # src = the sender's seeded payload
+    if active:
+        assert torch.equal(rview, expect), "payload mismatch"
     dist.barrier()
     l0 = ctx.launches()
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
     with Clocks(dev) as clk:
-        t0.record(stream)
+        t0.record(s_tx)
+        s_rx.wait_event(t0)
         for _ in range(args.steps):
             step()
-        t1.record(stream)
-        stream.synchronize()
+        s_tx.wait_stream(s_rx)
+        t1.record(s_tx)
+        s_tx.synchronize()
     ms = t0.elapsed_time(t1) if active else 0.0
     stats = torch.tensor([ms, float(ctx.launches() - l0)], dtype=torch.float64)
     mx = stats.clone()
@@ -306,78 +305,84 @@ def run_world(args, world, rank, local):
     sm = stats.clone()
     dist.all_reduce(sm, op=dist.ReduceOp.SUM)
     ms = float(mx[0])
-    value = n * npairs * args.steps / (ms * 1e-3) / 1e9
+    value = 2 * n * npairs * args.steps / (ms * 1e-3) / 1e9
 
-    # end to end: the sender's payload comes from pinned host memory, the receiver
-    # reads the message back to pinned host memory, every step.
+    # end to end: every step each sender's payload comes from pinned host memory and
+    # each receiver reads its message back to pinned host memory.
     e2e_steps = max(3, min(10, args.steps // 4))
     dist.barrier()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    with torch.cuda.stream(stream):
-        for _ in range(e2e_steps):
-            if sender:
-                src.copy_(h_buf, non_blocking=True)
-            step()
-            if active and not sender:
-                h_buf.copy_(rview, non_blocking=True)
-    e1.record(stream)
-    stream.synchronize()
+    e0.record(s_tx)
+    s_rx.wait_event(e0)
+    for _ in range(e2e_steps):
+        if active:
+            with torch.cuda.stream(s_tx):
+                src.copy_(h_src, non_blocking=True)
+        step()
+        if active:
+            with torch.cuda.stream(s_rx):
+                h_dst.copy_(rview, non_blocking=True)
+    s_tx.wait_stream(s_rx)
+    e1.record(s_tx)
+    s_tx.synchronize()
     e = torch.tensor([e0.elapsed_time(e1) if active else 0.0], dtype=torch.float64)
     dist.all_reduce(e, op=dist.ReduceOp.MAX)
-    e2e = n * npairs * e2e_steps / (float(e[0]) * 1e-3) / 1e9
+    e2e = 2 * n * npairs * e2e_steps / (float(e[0]) * 1e-3) / 1e9
 
-    # Baseline: the single-path copy-engine peer copy (what cudaMemcpyPeerAsync does):
-    # cudaMemcpyAsync from the sender's buffer into the receiver's heap buffer through
-    # its IPC mapping.
+    # Baseline: the single-path copy-engine peer copy (what cudaMemcpyPeerAsync does),
+    # both directions at once, through the IPC mapping of the partner's heap buffer.
     try:
         from cuda.bindings import runtime as rt
         offs = [None] * world
         dist.all_gather_object(offs, (rbuf - ctx.peer_base(rank)) if rbuf else None)
         ce_t = 0.0
-        if sender:
+        if active:
             dptr = ctx.peer_base(peer) + offs[peer]
             kind = rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice
             c0 = torch.cuda.Event(enable_timing=True)
             c1 = torch.cuda.Event(enable_timing=True)
+            dist.barrier()
             for _ in range(2):
-                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, stream.cuda_stream)
-            c0.record(stream)
+                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, s_tx.cuda_stream)
+            c0.record(s_tx)
             nb_steps = max(3, min(args.steps, 20))
             for _ in range(nb_steps):
-                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, stream.cuda_stream)
-            c1.record(stream)
-            stream.synchronize()
+                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, s_tx.cuda_stream)
+            c1.record(s_tx)
+            s_tx.synchronize()
             ce_t = c0.elapsed_time(c1) * 1e-3 / nb_steps
+        else:
+            dist.barrier()
         tt = torch.tensor([ce_t], dtype=torch.float64)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        base["cudaMemcpy_peer_GBps_per_pair"] = n / float(tt[0]) / 1e9
+        base["cudaMemcpy_peer_GBps_per_direction"] = n / float(tt[0]) / 1e9
     except Exception as exc:
         base["peer_copy_error"] = repr(exc)
 
     nvl = sum(b for (k, _), b in zip(d["paths"], d["bytes"]) if k != 2)
-    per_pair = n * args.steps / (ms * 1e-3) / 1e9
+    per_dir = n * args.steps / (ms * 1e-3) / 1e9
     achieved = nvl * args.steps / (ms * 1e-3) / 1e9
     line = {
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded uniform random bytes)",
-        "config": {"workload": f"config5 (pairs reading): {npairs} concurrent pairs 2i->2i+1, "
+        "config": {"workload": f"config5 (disjoint pairs, both directions): {npairs} pairs 2i<->2i+1, "
                                f"{n >> 20} MiB per message, direct + relays + pinned host, model-selected",
-                   "msg_bytes": n, "mode": args.mode, "parallelism": f"pairs{npairs}",
+                   "msg_bytes": n, "mode": args.mode, "parallelism": f"pairs{npairs}x2dir",
                    "l2": "messages >= 126 MB L2 (no flush)" if n >= 128 * MiB else "no flush"},
         "roofline": {"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
                      "frac": achieved / 770.0, "traffic": None, "peak_source":
                      "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
                      "kernel": "send_kernel"},
-        "per_pair_GBps": per_pair,
+        "per_direction_GBps": per_dir,
         "baselines": base,
-        "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n * npairs, "d2h_bytes_per_step": n * npairs},
+        "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n * 2 * npairs,
+                "d2h_bytes_per_step": n * 2 * npairs},
         "gpu_launches": int(sm[1]),
         "clocks": clk.summary(),
         "model": {"selected": d, "predicted_GBps": n / d["t_pred"] / 1e9 if d["t_pred"] else None,
-                  "E_pred": abs(n / d["t_pred"] / 1e9 - per_pair) / per_pair if d["t_pred"] else None},
+                  "E_pred": abs(n / d["t_pred"] / 1e9 - per_dir) / per_dir if d["t_pred"] else None},
     }
     if rank == 0:
         print(json.dumps(line), flush=True)
@@ -394,7 +399,8 @@ def main():
     ap.add_argument("--steps", type=int, default=2000)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="mpx", choices=["mpx", "reference"])
-    ap.add_argument("--size", type=int, default=GiB)
+    ap.add_argument("--size", type=int, default=None,
+                    help="message bytes (default: 1 GiB at N = 1 — config 3; 256 MiB per message at N > 1 — config 5)")
     ap.add_argument("--mode", default="b200", choices=["b200", "paper"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-calibrate", action="store_true",
@@ -403,6 +409,8 @@ def main():
     ap.add_argument("--save-params", default=None, help="write the calibrated parameters (Step 1)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    if args.size is None:
+        args.size = GiB if int(os.environ.get("WORLD_SIZE", "1")) == 1 else 256 * MiB
     if args.impl == "reference":
         return run_reference(args)
 
