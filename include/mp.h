@@ -200,6 +200,26 @@ int mp_predict(mp_ctx *ctx, int src, int dst, uint64_t bytes, const mp_config *c
 int mp_select(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t path_mask,
               mp_config *out);
 
+/* One of several concurrent messages (NEXT f1). */
+typedef struct mp_flow {
+  int32_t src;
+  int32_t dst;
+  uint32_t path_mask;  /* as in mp_select (0 = all paths of the pair) */
+  uint32_t reserved;
+  uint64_t bytes;
+} mp_flow;
+
+/* mp_select_flows — contention-aware selection for a known set of concurrent flows
+ * ("if the communication pattern … can be known ahead of time,
+ * unused paths can be extracted", P:410 MaxRate for shared links).  Reading C19:
+ * every link used by k of the flows gives each of them 1/k of its bandwidth — the
+ * source egress / destination ingress (port and direct β) by max(k_out, k_in), a
+ * relay's two legs by the number of flows that may use it (and a relay that is itself
+ * an endpoint of a flow is excluded), the host legs by the flows sharing that PCIe
+ * direction — then every flow is selected on its own (mp_select).  out: nflows
+ * configs, caller-allocated.  Not cached.  Host-only. */
+int mp_select_flows(mp_ctx *ctx, int nflows, const mp_flow *flows, mp_config *out);
+
 /* ---------------------------------------------------------------- memory */
 
 /* Allocate / free device memory from this rank's registered heap.  A buffer that

@@ -617,6 +617,26 @@ int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_con
   return MP_OK;
 }
 
+int mp_select_flows(mp_ctx *c, int nflows, const mp_flow *flows, mp_config *out) {
+  if (!c || (nflows > 0 && (!flows || !out)) || nflows < 0) return fail(c, MP_ERR_INVALID, "bad arguments");
+  std::vector<const PairModel *> models;
+  std::vector<FlowSpec> specs;
+  for (int f = 0; f < nflows; ++f) {
+    if (!pair_ok(c, flows[f].src, flows[f].dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+    models.push_back(pair_model(c, flows[f].src, flows[f].dst));
+    FlowSpec s;
+    s.src = flows[f].src;
+    s.dst = flows[f].dst;
+    s.bytes = flows[f].bytes;
+    s.mask = flows[f].path_mask;
+    specs.push_back(s);
+  }
+  std::vector<Selection> sel;
+  select_flows(models, specs, c->opts, &sel);
+  for (int f = 0; f < nflows; ++f) fill_config(*models[f], sel[f], &out[f]);
+  return MP_OK;
+}
+
 int mp_alloc(mp_ctx *c, uint64_t bytes, void **dptr) {
   if (!c || !dptr) return fail(c, MP_ERR_INVALID, "null argument");
   if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");

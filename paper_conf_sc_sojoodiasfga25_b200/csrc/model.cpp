@@ -362,3 +362,73 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
 }
 
 }  // namespace mpx
+
+namespace mpx {
+
+// Reading C19: MaxRate-style fair share for known concurrent flows
+// ("if the communication pattern … can be known ahead of time, unused paths can
+// be extracted"; MaxRate for contention on shared links).  Every link used by
+// k flows gives each 1/k of its bandwidth; then every flow is selected on its own.
+void select_flows(const std::vector<const PairModel *> &models, const std::vector<FlowSpec> &flows,
+                  const ModelOpts &o, std::vector<Selection> *out) {
+  const size_t F = flows.size();
+  auto allowed = [&](size_t f, size_t i) {
+    return i == 0 || flows[f].mask == 0 || ((flows[f].mask >> i) & 1u);
+  };
+  std::vector<int> k_out, k_in, endpoint, relay_users, host_out, host_in;
+  auto grow = [](std::vector<int> &v, int g) {
+    if (static_cast<int>(v.size()) <= g) v.resize(g + 1, 0);
+  };
+  int gmax = 0;
+  for (size_t f = 0; f < F; ++f) {
+    gmax = std::max(gmax, std::max(flows[f].src, flows[f].dst));
+    for (const PathModel &p : models[f]->paths) gmax = std::max(gmax, p.via);
+  }
+  for (auto *v : {&k_out, &k_in, &endpoint, &relay_users, &host_out, &host_in}) grow(*v, gmax);
+  for (size_t f = 0; f < F; ++f) {
+    k_out[flows[f].src] += 1;
+    k_in[flows[f].dst] += 1;
+    endpoint[flows[f].src] = endpoint[flows[f].dst] = 1;
+  }
+  for (size_t f = 0; f < F; ++f) {
+    const auto &paths = models[f]->paths;
+    for (size_t i = 0; i < paths.size(); ++i) {
+      if (!allowed(f, i)) continue;
+      if (paths[i].kind == K_GPU && paths[i].via >= 0) relay_users[paths[i].via] += 1;
+      if (paths[i].kind == K_HOST) {
+        host_out[flows[f].src] += 1;
+        host_in[flows[f].dst] += 1;
+      }
+    }
+  }
+  out->assign(F, Selection());
+  for (size_t f = 0; f < F; ++f) {
+    PairModel m = *models[f];
+    const int s = flows[f].src, d = flows[f].dst;
+    const double pdiv = std::max(k_out[s], k_in[d]);
+    uint32_t mask = 0;
+    for (size_t i = 0; i < m.paths.size(); ++i) {
+      PathModel &p = m.paths[i];
+      bool on = allowed(f, i);
+      if (p.kind == K_DIRECT) {
+        p.beta /= pdiv;
+      } else if (p.kind == K_GPU) {
+        if (p.via < 0 || endpoint[p.via]) {
+          on = false;  // the relay is itself an endpoint: no spare NVLink capacity
+        } else {
+          const double div = std::max(1, relay_users[p.via]);
+          p.beta /= div;
+          p.beta2 /= div;
+        }
+      } else {
+        p.beta /= std::max(1, host_out[s]);
+        p.beta2 /= std::max(1, host_in[d]);
+      }
+      if (on) mask |= 1u << i;
+    }
+    if (m.has_port()) m.port_beta /= pdiv;
+    select(m, flows[f].bytes, mask | 1u, o, &(*out)[f]);
+  }
+}
+
+}  // namespace mpx

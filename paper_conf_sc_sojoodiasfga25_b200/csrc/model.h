@@ -56,6 +56,16 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
 // The C5 integer rule (exposed for tests through the selector only).
 uint32_t k_from_real(double k_real);
 
+// NEXT f1 (reading C19): selection for a known set of concurrent flows with a
+// MaxRate-style fair share of every NVLink / PCIe link among the flows using it.
+struct FlowSpec {
+  int src = 0, dst = 0;
+  uint64_t bytes = 0;
+  uint32_t mask = 0;  // path mask of the pair (0 = all)
+};
+void select_flows(const std::vector<const PairModel *> &models, const std::vector<FlowSpec> &flows,
+                  const ModelOpts &o, std::vector<Selection> *out);
+
 // Eq 14 / Eq 15: the real optimal chunk count of a staged path
 // carrying x bytes (used by the φ calibration).
 double k_star(const PathModel &p, double x, int mode);

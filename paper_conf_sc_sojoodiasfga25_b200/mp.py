@@ -61,6 +61,11 @@ class mp_config(C.Structure):
                     t_pred=self.t_pred, t_level=self.t_level)
 
 
+class mp_flow(C.Structure):
+    _fields_ = [("src", C.c_int32), ("dst", C.c_int32), ("path_mask", C.c_uint32), ("reserved", C.c_uint32),
+                ("bytes", C.c_uint64)]
+
+
 ALLGATHER = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64)
 
 
@@ -109,6 +114,7 @@ def lib():
             "mp_load_params": (C.c_int, [P, C.c_char_p]),
             "mp_stats": (C.c_int, [P, C.POINTER(C.c_uint64)]),
             "mp_peer_base": (C.c_int, [P, C.c_int, C.POINTER(P)]),
+            "mp_select_flows": (C.c_int, [P, C.c_int, C.POINTER(mp_flow), C.POINTER(mp_config)]),
             "mp_fit_hockney": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                          C.POINTER(C.c_double), C.POINTER(C.c_double)]),
         }
@@ -125,7 +131,7 @@ def exported_symbols() -> List[str]:
             "mp_set_model", "mp_get_model", "mp_set_options", "mp_get_options", "mp_predict",
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
             "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
-            "mp_peer_base"]
+            "mp_peer_base", "mp_select_flows"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -258,6 +264,14 @@ class Context:
         cfg = mp_config()
         self._ck(lib().mp_select(self.h, src, dst, n, mask, C.byref(cfg)))
         return cfg
+
+    def select_flows(self, flows):
+        """flows: [(src, dst, bytes, mask)] → [mp_config] (NEXT f1, reading C19)."""
+        n = len(flows)
+        arr = (mp_flow * max(1, n))(*[mp_flow(s, d, m, 0, b) for s, d, b, m in flows])
+        out = (mp_config * max(1, n))()
+        self._ck(lib().mp_select_flows(self.h, n, arr, out))
+        return [out[i] for i in range(n)]
 
     # ---------------------------------------------------------------- engine
     def alloc(self, n) -> int:
