@@ -270,14 +270,19 @@ def run_world(args, world, rank, local):
     ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
                                   timeout_s=60.0)
     ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
-    d = ctx.select(0, 1, n).as_dict()
+    # the communication pattern is known ahead of time: select jointly for all
+    # concurrent flows (NEXT f1, mp_select_flows) — every rank computes the same configs
+    flows = [(r, r ^ 1, n, 0) for r in range(world) if (r ^ 1) < world]
+    cfgs = ctx.select_flows(flows)
+    my_cfg = cfgs[[f[0] for f in flows].index(rank)] if active else None
+    d = (my_cfg or cfgs[0]).as_dict()
     rbuf = ctx.alloc(n) if active else None
     rview = mp.as_tensor(rbuf, n) if rbuf else None
 
     def step():
         if active:
             ctx.recv(rbuf, n, peer, 0, s_rx)
-            ctx.send(src, n, peer, 0, None, s_tx)
+            ctx.send(src, n, peer, 0, my_cfg, s_tx)
 
     for _ in range(args.warmup):
         step()
