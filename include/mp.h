@@ -223,8 +223,9 @@ int mp_select_flows(mp_ctx *ctx, int nflows, const mp_flow *flows, mp_config *ou
 /* ---------------------------------------------------------------- memory */
 
 /* Allocate / free device memory from this rank's registered heap.  A buffer that
- * receives (mp_recv) must come from here when world > 1 (peers address it by heap
- * offset, the analogue of UCX cuda_ipc's cached IPC mappings).  256-B aligned. */
+ * receives (mp_recv) must come from here, or from a region registered with
+ * mp_register, when world > 1 (peers address it by heap offset, the analogue of UCX
+ * cuda_ipc's cached IPC mappings).  256-B aligned. */
 int mp_alloc(mp_ctx *ctx, uint64_t bytes, void **dptr);
 int mp_free(mp_ctx *ctx, void *dptr);
 
@@ -233,6 +234,26 @@ int mp_free(mp_ctx *ctx, void *dptr);
  * peer's mp_alloc buffer by (base + offset), e.g. for one-sided copies or baselines.
  * Errors: MP_ERR_STATE (model-only), MP_ERR_TOPOLOGY (no such rank). */
 int mp_peer_base(mp_ctx *ctx, int rank, void **base);
+
+/* mp_register — make an arbitrary device buffer of this rank a receive target
+ * (UCX cuda_ipc "caches IPC memory handles" so a user buffer is mapped once
+ * and reused).  COLLECTIVE when world > 1: every rank calls it in the
+ * same order (a rank with nothing to register passes buf = NULL, bytes = 0); every
+ * rank exports the allocation holding its buffer (cudaIpcGetMemHandle of the base
+ * found with cuMemGetAddressRange) and maps every peer's, so any rank may later act
+ * as sender or relay for a message into it.  Mappings of one peer allocation are
+ * shared between regions (reference-counted).  *id receives the region id, equal on
+ * every rank (0 is the heap, never returned).  mp_recv into [buf, buf + bytes) then
+ * needs no mp_alloc copy.  The buffer must stay allocated until mp_deregister.
+ * world == 1: nothing to map; returns MP_OK with a local id.
+ * Pauses the persistent relay kernel: no transfer may be in flight on any rank.
+ * Errors: MP_ERR_STATE (model-only), MP_ERR_NOMEM (region table full, 63 regions),
+ * MP_ERR_UNSUPPORTED (the allocation cannot be exported, e.g. VMM / expandable
+ * segments), MP_ERR_CUDA. */
+int mp_register(mp_ctx *ctx, void *buf, uint64_t bytes, int *id);
+
+/* mp_deregister — collective inverse of mp_register (same order on every rank). */
+int mp_deregister(mp_ctx *ctx, int id);
 
 /* ---------------------------------------------------------------- transfer */
 
@@ -246,7 +267,7 @@ int mp_send(mp_ctx *ctx, const void *buf, uint64_t bytes, int dst, int tag,
             const mp_config *cfg, void *stream);
 
 /* Receive `bytes` bytes from rank src with `tag` into device pointer `buf`
- * (heap memory when world > 1).  Matching is FIFO per (src, dst); the tag and the
+ * (heap memory or a registered region — mp_register — when world > 1).  Matching is FIFO per (src, dst); the tag and the
  * size must equal the sender's or the device raises MP_ERR_MISMATCH.  Work after
  * mp_recv on `stream` sees the whole message. */
 int mp_recv(mp_ctx *ctx, void *buf, uint64_t bytes, int src, int tag, void *stream);

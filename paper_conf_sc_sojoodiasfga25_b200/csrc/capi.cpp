@@ -666,6 +666,37 @@ int mp_peer_base(mp_ctx *c, int rank, void **base) {
   return MP_OK;
 }
 
+int mp_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
+  if (!c || !id) return fail(c, MP_ERR_INVALID, "null argument");
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  if ((bytes == 0) != (buf == nullptr)) return fail(c, MP_ERR_INVALID, "buf and bytes must both be set or both 0");
+  if (c->world == 1) {  // loopback receives into any device buffer: nothing to map
+    if (c->regions.empty()) c->regions.assign(mpx::kMaxRegions, mp_ctx::Region{});
+    for (int i = 1; i < static_cast<int>(c->regions.size()); ++i)
+      if (!c->regions[i].used) {
+        c->regions[i].used = true;
+        c->regions[i].base = static_cast<uint8_t *>(buf);
+        c->regions[i].bytes = bytes;
+        *id = i;
+        return MP_OK;
+      }
+    return fail(c, MP_ERR_NOMEM, "mp_register: region table full");
+  }
+  return mpx::world_register(c, buf, bytes, id);
+}
+
+int mp_deregister(mp_ctx *c, int id) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return fail(c, MP_ERR_STATE, "model-only context");
+  if (c->world == 1) {
+    if (id <= 0 || id >= static_cast<int>(c->regions.size()) || !c->regions[id].used)
+      return fail(c, MP_ERR_INVALID, "mp_deregister: unknown region id");
+    c->regions[id] = mp_ctx::Region{};
+    return MP_OK;
+  }
+  return mpx::world_deregister(c, id);
+}
+
 int mp_xfer(mp_ctx *c, void *dst, const void *src, uint64_t bytes, const mp_config *cfg,
             void *stream) {
   if (!c) return MP_ERR_INVALID;

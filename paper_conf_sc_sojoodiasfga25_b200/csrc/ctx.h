@@ -108,6 +108,20 @@ struct mp_ctx {
   int32_t *stop = nullptr;                  // mapped host word read by the relay kernel
   bool relay_running = false;
   std::vector<cudaStream_t> streams;        // user streams seen by mp_send/mp_recv
+  // receive regions (mp_register): [kMaxRegions], region 0 = the heap
+  struct Region {
+    bool used = false;
+    uint8_t *base = nullptr;                // this rank's buffer (nullptr: none registered)
+    uint64_t bytes = 0;
+    std::vector<uint64_t> maps;             // [world]: key into ipc_maps (0 = none)
+  };
+  std::vector<Region> regions;
+  // IPC mapping cache: (rank, remote allocation base) -> {mapped base, refs}
+  struct IpcMap {
+    uint8_t *mapped = nullptr;
+    int refs = 0;
+  };
+  std::map<std::pair<int, uint64_t>, IpcMap> ipc_maps;
 };
 
 namespace mpx {
@@ -139,4 +153,6 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
                void *stream);
 int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream);
 int world_sync(mp_ctx *c);
+int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id);
+int world_deregister(mp_ctx *c, int id);
 }  // namespace mpx

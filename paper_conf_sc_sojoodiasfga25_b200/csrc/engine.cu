@@ -444,6 +444,13 @@ __device__ __forceinline__ uint64_t *done_at(uint8_t *ctrl, const CtrlLayout &L,
   return reinterpret_cast<uint64_t *>(ctrl + L.done + static_cast<uint64_t>(src) * 128);
 }
 
+// Base of rank `rank`'s receive region `region` in this process (see engine.h).
+__device__ __forceinline__ uint8_t *region_base(const uint8_t *ctrl, const CtrlLayout &L, uint64_t region,
+                                                uint32_t rank) {
+  return reinterpret_cast<uint8_t *>(
+      reinterpret_cast<const uint64_t *>(ctrl + L.regions)[region * L.world + rank]);
+}
+
 __device__ __forceinline__ uint64_t *flags_at(uint8_t *ctrl, uint64_t base, uint32_t who, uint32_t slots,
                                               uint64_t slot) {
   return reinterpret_cast<uint64_t *>(ctrl + base) + (static_cast<uint64_t>(who) * slots + slot) * kFlagStride;
@@ -488,7 +495,7 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
     }
     __nanosleep(64);
   }
-  const uint64_t off = ld_volatile(&cts->a), n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
+  const uint64_t n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
   const bool bad = (n != P.bytes) || (tag != P.tag);
   uint64_t host_k = 0, host_q0 = 0, host_off = 0, host_bytes = 0;
   for (uint32_t i = 0; i < P.npaths; ++i)
@@ -505,7 +512,7 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
   h->a = bad ? 0 : host_k;
   h->b = host_q0;
   h->c = bad ? 2 : 0;
-  h->d = off + host_off;
+  h->d = host_off;
   h->e = host_bytes;
   h->f = reinterpret_cast<uintptr_t>(P.src + host_off) & 15u;
   st_release_sys(&h->seq1, P.seq + 1);
@@ -515,7 +522,8 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
 __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant__ SendParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
-  __shared__ uint64_t s_off;
+  __shared__ uint64_t s_off, s_region;
+  __shared__ uint8_t *s_dst;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
   // the clear-to-send has arrived (send_gate_kernel ran first on this stream)
@@ -524,7 +532,9 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
   if (threadIdx.x == 0) {
     const uint64_t off = ld_volatile(&cts->a), n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
     s_off = off;
-    if ((n != P.bytes) || (tag != P.tag)) s_abort = 1;  // reported by the gate
+    s_region = ld_volatile(&cts->d);
+    if ((n != P.bytes) || (tag != P.tag) || s_region >= kMaxRegions) s_abort = 1;  // reported by the gate
+    else s_dst = region_base(P.my_ctrl, P.L, s_region, P.dst) + off;
   }
   __syncthreads();
   if (s_abort) return;
@@ -533,9 +543,9 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
   uint64_t *done = done_at(P.dst_ctrl, P.L, P.me);
   if (b < P.g_direct) {  // A7: direct NVLink stores into the receiver's heap
     if (P.copy_mode == 1)
-      bulk_copy<LD_SRC>(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct, dyn_smem, P.bulk_stages);
+      bulk_copy<LD_SRC>(s_dst, P.src, P.direct_bytes, b, P.g_direct, dyn_smem, P.bulk_stages);
     else
-      group_copy<LD_SRC>(P.dst_heap + base, P.src, P.direct_bytes, b, P.g_direct);
+      group_copy<LD_SRC>(s_dst, P.src, P.direct_bytes, b, P.g_direct);
     const uint64_t share = P.direct_bytes * (b + 1) / P.g_direct - P.direct_bytes * b / P.g_direct;
     publish(done, share, nullptr, 0);
     return;
@@ -579,6 +589,7 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
         h[1] = base + off;
         h[2] = len;
         h[3] = shift;
+        h[4] = s_region;
       }
       publish(nullptr, 0, fl + r, u + 1);
     }
@@ -596,9 +607,10 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
   if (blockIdx.x == 0) {
     if (threadIdx.x == 0) {  // post the clear-to-send into the sender's control block
       MsgEntry *cts = entry_at(P.src_ctrl, P.L.cts, P.me, P.seq);
-      cts->a = P.heap_off;
+      cts->a = P.region_off;
       cts->b = P.bytes;
       cts->c = P.tag;
+      cts->d = P.region;
       fence_acq_rel_sys();
       st_release_sys(&cts->seq1, P.seq + 1);
       // A10: wait until every byte of the message has been counted in
@@ -639,7 +651,7 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
     chunk_of(s_hbytes, 256, static_cast<uint32_t>(s_k), static_cast<uint32_t>(j), &off, &len);
     uint64_t a, e;
     slice_of(len, r, P.g_host, &a, &e);
-    copy_slice<LD_HOST>(P.my_heap + s_hoff + off + a, slot + kSlotHdr + s_shift + a, e - a, dyn_smem,
+    copy_slice<LD_HOST>(P.buf + s_hoff + off + a, slot + kSlotHdr + s_shift + a, e - a, dyn_smem,
                         P.copy_mode, P.bulk_stages);
     publish(done, e - a, P.host.freef + s * kFlagStride + r, u + 1, /*done_is_local=*/true);
   }
@@ -649,7 +661,7 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
 __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constant__ RelayParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
-  __shared__ uint64_t s_h[4];
+  __shared__ uint64_t s_h[5];
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
   const uint32_t sender = blockIdx.x / P.g, r = blockIdx.x % P.g;
@@ -664,13 +676,13 @@ __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constan
       return;
     }
     uint8_t *slot = P.my_ctrl + P.L.ring_data + (static_cast<uint64_t>(sender) * P.L.slots + s) * P.L.stride;
-    if (threadIdx.x < 4) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(slot) + threadIdx.x);
+    if (threadIdx.x < 5) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(slot) + threadIdx.x);
     __syncthreads();
     const uint32_t dst = static_cast<uint32_t>(s_h[0]);
     const uint64_t off = s_h[1], len = s_h[2], shift = s_h[3];
     uint64_t a, e;
     slice_of(len, r, P.g, &a, &e);
-    copy_slice<LD_RING>(P.peer[dst].heap + off + a, slot + kSlotHdr + shift + a, e - a, dyn_smem, P.copy_mode,
+    copy_slice<LD_RING>(region_base(P.my_ctrl, P.L, s_h[4], dst) + off + a, slot + kSlotHdr + shift + a, e - a, dyn_smem, P.copy_mode,
                         P.bulk_stages);
     uint64_t *fr = flags_at(P.peer[sender].ctrl, P.L.relay_free, P.me, P.L.slots, s);
     publish(done_at(P.peer[dst].ctrl, P.L, sender), e - a, fr + r, u + 1);

@@ -64,27 +64,32 @@ int launch_xfer(const XferParams &P, void *stream);
 //
 // One process per GPU.  Every rank exports (cudaIpc) its receive heap and its
 // control block; every rank maps every peer's.  A message src → dst:
-//   receiver (mp_recv):  recv kernel CTA 0 posts a CTS entry {seq+1, heap offset,
-//                        bytes, tag} into the sender's control block, then waits for
+//   receiver (mp_recv):  recv kernel CTA 0 posts a CTS entry {seq+1, region offset,
+//                        bytes, tag, region id} into the sender's control block, then waits for
 //                        its per-src byte counter `done` to reach the target; CTAs
 //                        1.. consume the message's host-ring chunks (A9 step 3).
 //   sender   (mp_send):  send kernel CTAs wait for the CTS, CTA 0 writes the message
 //                        header {seq+1, host_k, host_q0, status} into the receiver's
-//                        control block; the direct group stores into the peer heap
+//                        control block; the direct group stores into the target region
 //                        (A7), stage-in groups fill relay rings (A8 step 1) and the
 //                        host ring (A9 step 1); every byte delivered is counted into
 //                        the receiver's `done` with red.release.sys.
 //   relay    (persistent, one per rank): per sender ring, forward every landed chunk
 //                        to the destination named in the slot header (A8 step 3).
-// Slot = [kSlotHdr-byte header][data]; header = {dst rank, dst heap offset, len, shift}.
+// Slot = [kSlotHdr-byte header][data]; header = {dst rank, region offset, len, shift, region}.
+// A receive target is (region id, offset): every rank's control block holds the table
+// regions[id][rank] = base of rank's region `id` as mapped in THIS process (region 0
+// = the heaps, 1.. = mp_register), so a sender or relay resolves it locally.
 
 constexpr uint32_t kCtsRing = 64;     // outstanding messages per ordered pair
 constexpr uint32_t kSlotHdr = 256;    // slot header bytes
+constexpr uint32_t kMaxRegions = 64;  // receive regions: 0 = heap, 1.. = mp_register
 
 struct MsgEntry {                      // CTS and message-header entries (64 B)
   uint64_t seq1;                       // sequence + 1 (written last, with release)
-  uint64_t a, b, c;                    // CTS: heap_off, bytes, tag; HDR: host_k, host_q0, status
-  uint64_t d, e, f, g;                 // HDR: host range heap offset, host bytes, src shift (mod 16)
+  uint64_t a, b, c;                    // CTS: region offset, bytes, tag; HDR: host_k, host_q0, status
+  uint64_t d, e, f, g;                 // CTS: region id; HDR: host range message offset, host bytes,
+                                       //      src shift (mod 16)
 };
 
 struct PeerPtrs {
@@ -106,6 +111,7 @@ struct CtrlLayout {
   uint64_t host_free = 0;              // [world(receiver)][slots][kFlagStride]   — on the sender
   uint64_t probe = 0;                  // 64 B of flag words for the ε ping-pong of the predecessor
   uint64_t relay_pos = 0;              // [world(sender)] u64: relay ring position across restarts
+  uint64_t regions = 0;                // [kMaxRegions][world] u64: mapped region bases (local)
   uint64_t total = 0;
 };
 
@@ -121,7 +127,6 @@ struct SendParams {
   uint64_t seq, bytes, tag, timeout_ns;
   const uint8_t *src;
   uint8_t *my_ctrl;
-  uint8_t *dst_heap;
   uint8_t *dst_ctrl;
   int32_t *err;
   CtrlLayout L;
@@ -143,9 +148,9 @@ struct SendParams {
 
 struct RecvParams {
   uint32_t me, src, nblocks, g_host, copy_mode, bulk_stages;
-  uint64_t seq, bytes, tag, heap_off, done_target, timeout_ns;
+  uint64_t seq, bytes, tag, region, region_off, done_target, timeout_ns;
   uint8_t *my_ctrl;
-  uint8_t *my_heap;
+  uint8_t *buf;              // the receive buffer (host-ring consumers write here)
   uint8_t *src_ctrl;
   int32_t *err;
   CtrlLayout L;
@@ -159,7 +164,7 @@ struct RelayParams {
   uint32_t me, world, g;       // g CTAs per sender ring
   uint32_t copy_mode, bulk_stages, pad_;
   uint8_t *my_ctrl;
-  PeerPtrs peer[kMaxPaths];    // heap/ctrl of every rank (self: local)
+  PeerPtrs peer[kMaxPaths];    // ctrl of every rank (self: local); targets via regions
   CtrlLayout L;
   volatile int32_t *stop;      // mapped host word: != 0 → exit
   int32_t *err;

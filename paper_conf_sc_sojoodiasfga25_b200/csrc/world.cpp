@@ -39,6 +39,7 @@ struct RankInfo {
   cudaIpcMemHandle_t heap;
   cudaIpcMemHandle_t ctrl;
   uint64_t jobid;
+  uint64_t heap_addr;
   uint64_t heap_bytes;
   int32_t device;
   int32_t relay_ctas;
@@ -80,6 +81,7 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.host_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.probe = take(64);
   L.relay_pos = take(static_cast<uint64_t>(world) * 8);
+  L.regions = take(static_cast<uint64_t>(kMaxRegions) * world * 8);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
@@ -160,6 +162,7 @@ int world_init(mp_ctx *c) {
   CKW(cudaIpcGetMemHandle(&me.ctrl, c->ctrl));
   me.jobid = std::random_device{}() ^ (static_cast<uint64_t>(std::random_device{}()) << 32) ^
              static_cast<uint64_t>(getpid());
+  me.heap_addr = reinterpret_cast<uintptr_t>(c->heap.base);
   me.heap_bytes = c->heap.size;
   me.device = c->device;
   me.relay_ctas = c->relay_ctas;
@@ -187,6 +190,18 @@ int world_init(mp_ctx *c) {
     if (e != cudaSuccess)
       return wfail(c, MP_ERR_TOPOLOGY, "cannot map rank " + std::to_string(r) + "'s memory: " + cudaGetErrorString(e));
     c->peers[r] = PeerPtrs{static_cast<uint8_t *>(h), static_cast<uint8_t *>(k)};
+    c->ipc_maps[{r, all[r].heap_addr}] = mp_ctx::IpcMap{static_cast<uint8_t *>(h), 1};
+  }
+  // region 0 = the heaps
+  c->regions.assign(kMaxRegions, mp_ctx::Region{});
+  c->regions[0].used = true;
+  c->regions[0].base = c->heap.base;
+  c->regions[0].bytes = c->heap.size;
+  c->regions[0].maps.assign(W, 0);
+  {
+    std::vector<uint64_t> row(W);
+    for (int r = 0; r < W; ++r) row[r] = reinterpret_cast<uintptr_t>(c->peers[r].heap);
+    CKW(cudaMemcpy(c->ctrl + c->L.regions, row.data(), W * 8, cudaMemcpyHostToDevice));
   }
 
   // Host rings: one segment per receiving rank, one ring per sender inside it.
@@ -266,9 +281,11 @@ int world_finalize(mp_ctx *c) {
   if (c->allgather) st = barrier(c);
   for (int r = 0; r < static_cast<int>(c->peers.size()); ++r) {
     if (r == c->rank) continue;
-    if (c->peers[r].heap) cudaIpcCloseMemHandle(c->peers[r].heap);
     if (c->peers[r].ctrl) cudaIpcCloseMemHandle(c->peers[r].ctrl);
   }
+  for (auto &m : c->ipc_maps) cudaIpcCloseMemHandle(m.second.mapped);  // heaps + registered regions
+  c->ipc_maps.clear();
+  c->regions.clear();
   c->peers.clear();
   for (uint8_t *s : c->hseg)
     if (s) {
@@ -300,7 +317,6 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.src = static_cast<const uint8_t *>(buf);
   P.my_ctrl = c->ctrl;
-  P.dst_heap = c->peers[dst].heap;
   P.dst_ctrl = c->peers[dst].ctrl;
   P.err = c->d_err;
   P.L = c->L;
@@ -360,19 +376,33 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
 
 int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
   uint8_t *b = static_cast<uint8_t *>(buf);
-  if (bytes && (b < c->heap.base || b + bytes > c->heap.base + c->heap.size))
-    return wfail(c, MP_ERR_INVALID, "mp_recv buffer must come from mp_alloc when world > 1");
+  int region = -1;
+  for (int i = 0; i < static_cast<int>(c->regions.size()) && bytes; ++i) {
+    const mp_ctx::Region &g = c->regions[i];
+    if (g.used && g.base && b >= g.base && b + bytes <= g.base + g.bytes) {
+      region = i;
+      break;
+    }
+  }
+  if (!bytes) region = 0;
+  if (region < 0)
+    return wfail(c, MP_ERR_INVALID, "mp_recv buffer must come from mp_alloc or mp_register when world > 1");
   RecvParams P{};
   P.me = static_cast<uint32_t>(c->rank);
   P.src = static_cast<uint32_t>(src);
   P.seq = c->recv_seq[src];
   P.bytes = bytes;
   P.tag = static_cast<uint64_t>(static_cast<int64_t>(tag));
-  P.heap_off = bytes ? static_cast<uint64_t>(b - c->heap.base) : 0;
+  P.region = static_cast<uint64_t>(region);
+  if (debug_on())
+    std::fprintf(stderr, "[mpx %d] recv %llu B from %d into region %d + %llu\n", c->rank,
+                 static_cast<unsigned long long>(bytes), src, region,
+                 static_cast<unsigned long long>(bytes ? b - c->regions[region].base : 0));
+  P.region_off = bytes ? static_cast<uint64_t>(b - c->regions[region].base) : 0;
   P.done_target = c->done_target[src] + bytes;
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.my_ctrl = c->ctrl;
-  P.my_heap = c->heap.base;
+  P.buf = b;
   P.src_ctrl = c->peers[src].ctrl;
   P.err = c->d_err;
   P.L = c->L;
@@ -390,6 +420,165 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   c->done_target[src] += bytes;
   note_stream(c, static_cast<cudaStream_t>(stream));
   return MP_OK;
+}
+
+// ---------------------------------------------------------------- regions (mp_register)
+
+namespace {
+// cuMemGetAddressRange through the runtime's driver entry point (no -lcuda).
+int alloc_range(mp_ctx *c, const void *p, uint64_t *base, uint64_t *size) {
+  using Fn = int (*)(unsigned long long *, size_t *, unsigned long long);
+  static Fn fn = nullptr;
+  if (!fn) {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q{};
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess || !f)
+      return wfail(c, MP_ERR_CUDA, "cuMemGetAddressRange entry point not found");
+    fn = reinterpret_cast<Fn>(f);
+  }
+  unsigned long long b = 0;
+  size_t n = 0;
+  if (fn(&b, &n, reinterpret_cast<uintptr_t>(p)) != 0)
+    return wfail(c, MP_ERR_INVALID, "mp_register: not a device allocation");
+  *base = b;
+  *size = n;
+  return MP_OK;
+}
+
+struct RegInfo {
+  cudaIpcMemHandle_t h;
+  uint64_t alloc_base, off;
+  int32_t status;   // 0 nothing registered, 1 exported, < 0 MP_ERR_* of a local failure
+  int32_t id;
+};
+
+int write_region_row(mp_ctx *c, int id, const std::vector<uint64_t> &row) {
+  CKW(cudaMemcpy(c->ctrl + c->L.regions + static_cast<uint64_t>(id) * c->world * 8, row.data(),
+                 c->world * 8, cudaMemcpyHostToDevice));
+  // a pageable copy may return before its DMA lands; the relay kernel is stopped here
+  CKW(cudaDeviceSynchronize());
+  return MP_OK;
+}
+
+void unmap(mp_ctx *c, int r, uint64_t key) {
+  auto it = c->ipc_maps.find({r, key});
+  if (it == c->ipc_maps.end()) return;
+  if (--it->second.refs == 0) {
+    cudaIpcCloseMemHandle(it->second.mapped);
+    c->ipc_maps.erase(it);
+  }
+}
+}  // namespace
+
+int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
+  const int W = c->world;
+  int rid = -1;
+  for (int i = 1; i < static_cast<int>(c->regions.size()); ++i)
+    if (!c->regions[i].used) {
+      rid = i;
+      break;
+    }
+  RegInfo me;
+  std::memset(&me, 0, sizeof(me));
+  me.id = rid;
+  std::string local_err;
+  if (buf && bytes) {
+    uint64_t base = 0, size = 0;
+    if (int s = alloc_range(c, buf, &base, &size)) {
+      me.status = s;
+    } else if (reinterpret_cast<uintptr_t>(buf) + bytes > base + size) {
+      me.status = MP_ERR_INVALID;
+      c->last_error = "mp_register: buffer runs past its allocation";
+    } else if (cudaIpcGetMemHandle(&me.h, reinterpret_cast<void *>(base)) != cudaSuccess) {
+      cudaGetLastError();
+      me.status = MP_ERR_UNSUPPORTED;
+      c->last_error = "mp_register: the allocation cannot be exported with cudaIpc (VMM / expandable segment?)";
+    } else {
+      me.status = 1;
+      me.alloc_base = base;
+      me.off = reinterpret_cast<uintptr_t>(buf) - base;
+    }
+  }
+  std::vector<RegInfo> all(W);
+  if (int s = allgather(c, &me, all.data(), sizeof(RegInfo))) return s;
+  for (int r = 0; r < W; ++r) {
+    if (all[r].id != rid) return wfail(c, MP_ERR_STATE, "mp_register / mp_deregister not called collectively");
+    if (all[r].status < 0)
+      return r == c->rank ? all[r].status
+                          : wfail(c, all[r].status, "mp_register failed on rank " + std::to_string(r));
+  }
+  if (rid < 0) return wfail(c, MP_ERR_NOMEM, "mp_register: region table full");
+  const bool relay = c->relay_running;
+  if (int s = world_stop_relay(c)) return s;
+  mp_ctx::Region g;
+  g.used = true;
+  g.base = static_cast<uint8_t *>(bytes ? buf : nullptr);
+  g.bytes = bytes;
+  g.maps.assign(W, 0);
+  std::vector<uint64_t> row(W, 0);
+  int st = MP_OK;
+  for (int r = 0; r < W && st == MP_OK; ++r) {
+    if (all[r].status != 1) continue;
+    if (r == c->rank) {
+      row[r] = reinterpret_cast<uintptr_t>(buf);
+      continue;
+    }
+    auto it = c->ipc_maps.find({r, all[r].alloc_base});
+    if (it == c->ipc_maps.end()) {
+      void *h = nullptr;
+      cudaError_t e = cudaIpcOpenMemHandle(&h, all[r].h, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess) {
+        st = wfail(c, MP_ERR_CUDA, "mp_register: cannot map rank " + std::to_string(r) + ": " + cudaGetErrorString(e));
+        break;
+      }
+      it = c->ipc_maps.emplace(std::make_pair(r, all[r].alloc_base), mp_ctx::IpcMap{static_cast<uint8_t *>(h), 0}).first;
+    }
+    it->second.refs += 1;
+    g.maps[r] = all[r].alloc_base;
+    row[r] = reinterpret_cast<uintptr_t>(it->second.mapped) + all[r].off;
+  }
+  if (st == MP_OK) st = write_region_row(c, rid, row);
+  if (debug_on())
+    for (int r = 0; r < W; ++r)
+      std::fprintf(stderr, "[mpx %d] region %d rank %d -> %p (status %d, alloc %llx + %llu)\n", c->rank, rid, r,
+                   reinterpret_cast<void *>(row[r]), all[r].status,
+                   static_cast<unsigned long long>(all[r].alloc_base), static_cast<unsigned long long>(all[r].off));
+  if (st == MP_OK) {
+    c->regions[rid] = g;
+    *id = rid;
+  } else {
+    for (int r = 0; r < W; ++r)
+      if (g.maps[r]) unmap(c, r, g.maps[r]);
+  }
+  if (relay)
+    if (int s = world_start_relay(c)) return s;
+  // every rank's table holds the row before anyone sends into the region
+  if (int s = barrier(c)) return s;
+  return st;
+}
+
+int world_deregister(mp_ctx *c, int id) {
+  const int W = c->world;
+  if (id <= 0 || id >= static_cast<int>(c->regions.size()) || !c->regions[id].used)
+    return wfail(c, MP_ERR_INVALID, "mp_deregister: unknown region id");
+  RegInfo me;
+  std::memset(&me, 0, sizeof(me));
+  me.id = id;
+  for (cudaStream_t s : c->streams) CKW(cudaStreamSynchronize(s));  // our receives into it are done
+  std::vector<RegInfo> all(W);
+  if (int s = allgather(c, &me, all.data(), sizeof(RegInfo))) return s;
+  for (int r = 0; r < W; ++r)
+    if (all[r].id != id) return wfail(c, MP_ERR_STATE, "mp_register / mp_deregister not called collectively");
+  const bool relay = c->relay_running;
+  if (int s = world_stop_relay(c)) return s;
+  int st = write_region_row(c, id, std::vector<uint64_t>(W, 0));
+  for (int r = 0; r < W; ++r)
+    if (c->regions[id].maps[r]) unmap(c, r, c->regions[id].maps[r]);
+  c->regions[id] = mp_ctx::Region{};
+  if (relay)
+    if (int s = world_start_relay(c)) return s;
+  if (int s = barrier(c)) return s;
+  return st;
 }
 
 int world_sync(mp_ctx *c) {

@@ -114,6 +114,8 @@ def lib():
             "mp_load_params": (C.c_int, [P, C.c_char_p]),
             "mp_stats": (C.c_int, [P, C.POINTER(C.c_uint64)]),
             "mp_peer_base": (C.c_int, [P, C.c_int, C.POINTER(P)]),
+            "mp_register": (C.c_int, [P, P, C.c_uint64, C.POINTER(C.c_int)]),
+            "mp_deregister": (C.c_int, [P, C.c_int]),
             "mp_select_flows": (C.c_int, [P, C.c_int, C.POINTER(mp_flow), C.POINTER(mp_config)]),
             "mp_fit_hockney": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                          C.POINTER(C.c_double), C.POINTER(C.c_double)]),
@@ -131,7 +133,7 @@ def exported_symbols() -> List[str]:
             "mp_set_model", "mp_get_model", "mp_set_options", "mp_get_options", "mp_predict",
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
             "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
-            "mp_peer_base", "mp_select_flows"]
+            "mp_peer_base", "mp_select_flows", "mp_register", "mp_deregister"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -286,6 +288,17 @@ class Context:
         v = C.c_void_p()
         self._ck(lib().mp_peer_base(self.h, rank, C.byref(v)))
         return v.value
+
+    def register(self, buf, n=None) -> int:
+        """mp_register (collective when world > 1): buf = tensor / pointer / None."""
+        if n is None:
+            n = 0 if buf is None else buf.numel() * buf.element_size()
+        v = C.c_int()
+        self._ck(lib().mp_register(self.h, _ptr(buf), n, C.byref(v)))
+        return v.value
+
+    def deregister(self, rid):
+        self._ck(lib().mp_deregister(self.h, rid))
 
     def xfer(self, dst, src, n, cfg: Optional[mp_config] = None, stream=None):
         self._ck(lib().mp_xfer(self.h, _ptr(dst), _ptr(src), n, C.byref(cfg) if cfg else None,

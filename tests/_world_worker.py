@@ -191,12 +191,100 @@ def scenario_faults(rank, world):
         c.close()
 
 
+def scenario_register(rank, world):
+    """mp_register (D7): receive into arbitrary torch tensors — two views of one
+    torch allocation on rank 1 (a shared IPC mapping on every peer), then one tensor
+    per rank in a ring — over every path at once, byte-exact against the oracle
+    replay, bytes outside the views untouched; deregistered regions are refused."""
+    import numpy as np
+
+    import synth
+    from oracle import transfer as X
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    big = torch.zeros(16 * MiB, dtype=torch.uint8, device="cuda")        # rank 1's targets
+    ring = torch.zeros(4 * MiB, dtype=torch.uint8, device="cuda")        # every rank's ring target
+    src_buf = torch.empty(8 * MiB, dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    c = mdist.context_from_dist(device=0, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                timeout_s=60.0)
+    ps = c.paths(0, 1)
+    kinds = [k for k, _ in ps]
+    va, vb = big[MiB + 256: 9 * MiB], big[10 * MiB: 15 * MiB]
+    ida = c.register(va if rank == 1 else None)
+    idb = c.register(vb if rank == 1 else None)
+    idr = c.register(ring)
+    assert len({ida, idb, idr}) == 3 and min(ida, idb, idr) >= 1
+    # (region A) every path at once, explicit config; (region B) model-selected
+    na = 3 * MiB + 4099
+    nb = [256 * 1024] * len(ps)
+    nb[0] = na - 256 * 1024 * (len(ps) - 1)
+    ks = [1] + [2] * (len(ps) - 1)
+    for case, (view, n, cfgb, cfgk) in enumerate([(va, na, nb, ks), (vb, 5 * MiB, None, None)]):
+        host = synth.payload(n, 60 + case)
+        if rank == 0:
+            with torch.cuda.stream(stream):   # never torch.cuda.synchronize(): the relay kernel runs
+                src_buf[:n].copy_(torch.from_numpy(host))
+            c.send(src_buf[:n], n, 1, tag=300 + case, cfg=c.make_config(cfgb, cfgk, 0, 1) if cfgb else None,
+                   stream=stream)
+            stream.synchronize()
+        elif rank == 1:
+            c.recv(view[:n], n, 0, tag=300 + case, stream=stream)
+            stream.synchronize()
+            exp = host.copy()
+            if cfgb:
+                exp = np.zeros(n, dtype=np.uint8)
+                X.replay(host, cfgb, cfgk, kinds, 256, exp)
+            got = view[:n].cpu().numpy()
+            bad = np.nonzero(got != exp)[0]
+            assert bad.size == 0, (f"region case {case}: {bad.size} bytes differ, first {bad[:4]}, "
+                                   f"last {bad[-4:]}, config {cfgb} {cfgk}")
+        dist.barrier()
+    # ring: rank r → r+1 into the peer's registered tensor, at a 4 KiB + 17 offset
+    n = 2 * MiB + 333
+    nxt, prv = (rank + 1) % world, (rank - 1) % world
+    with torch.cuda.stream(stream):
+        src_buf[:n].copy_(torch.from_numpy(synth.payload(n, 70 + rank)))
+    s_rx = torch.cuda.Stream()
+    c.recv(ring[4096 + 17: 4096 + 17 + n], n, prv, tag=400, stream=s_rx)
+    c.send(src_buf[:n], n, nxt, tag=400, stream=stream)
+    stream.synchronize()
+    s_rx.synchronize()
+    c.sync()
+    assert np.array_equal(ring[4096 + 17: 4096 + 17 + n].cpu().numpy(), synth.payload(n, 70 + prv)), "ring"
+    dist.barrier()
+    for rid in (ida, idb, idr):
+        c.deregister(rid)
+    if rank == 1:
+        try:
+            c.recv(va[:MiB], MiB, 0, tag=1, stream=stream)
+            raise AssertionError("recv into a deregistered region was accepted")
+        except mp.MPError:
+            pass
+    # ids are reused after deregistration
+    assert c.register(ring) == ida
+    c.deregister(ida)
+    dist.barrier()
+    c.sync()
+    c.close()
+    # new torch kernels only now: a first launch lazily loads its module, which waits
+    # for the device to idle — never while the persistent relay kernel runs
+    if rank == 1:
+        h = big.cpu().numpy()
+        rest = np.concatenate([h[:MiB + 256], h[MiB + 256 + na: 10 * MiB], h[15 * MiB:]])
+        assert not rest.any(), "bytes outside the registered views were written"
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
+    import faulthandler
+    faulthandler.dump_traceback_later(int(os.environ.get("MPX_TEST_STACKS_S", "280")), exit=False)
     try:
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
-         "faults": scenario_faults}[scen](rank, world)
+         "faults": scenario_faults, "register": scenario_register}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

@@ -38,6 +38,11 @@ def test_model_only_context_rejects_engine_calls():
         assert e.value.status == -5
         with pytest.raises(mp.MPError):
             c.xfer(0, 0, 16)
+        with pytest.raises(mp.MPError) as e:
+            c.register(0x1000, 4096)
+        assert e.value.status == -5
+        with pytest.raises(mp.MPError):
+            c.deregister(1)
 
 
 def test_init_validation():

@@ -155,6 +155,19 @@ def test_send_recv_loopback(ctx):
     assert e.value.status == -8
 
 
+def test_register_loopback(ctx):
+    # world == 1: registration maps nothing but hands out distinct, reusable ids
+    t = torch.zeros(MiB, dtype=torch.uint8, device="cuda")
+    a, b = ctx.register(t), ctx.register(t[4096:])
+    assert a >= 1 and b >= 1 and a != b
+    ctx.deregister(a)
+    assert ctx.register(t[:4096]) == a
+    with pytest.raises(mp.MPError):
+        ctx.deregister(0)
+    ctx.deregister(a)
+    ctx.deregister(b)
+
+
 def test_cuda_graph_capture_direct_only(ctx):
     # launch-bound windows can be captured in a CUDA graph when the config is
     # direct-only (a pure kernel); staged configs are refused while capturing

@@ -69,3 +69,13 @@ def test_multirank_faults_reported_not_hung():
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(2, "faults", timeout=300)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 3])
+def test_multirank_registered_buffers(world):
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(world, "register", timeout=400)
