@@ -179,6 +179,26 @@ int mp_set_model(mp_ctx *ctx, int src, int dst, const mp_path *paths,
 int mp_get_model(mp_ctx *ctx, int src, int dst, mp_path *paths, mp_path_params *params,
                  int *npaths, mp_port_params *port);
 
+/* NEXT f4 size bands (P:360 Observation 4: the linear Hockney model
+ * fitted on the asymptotic bandwidth is less accurate for small messages).  Reading
+ * C20: a pair may carry several complete parameter sets; band j applies to messages
+ * of n bytes with n_min_j <= n < n_min_{j+1}.  Band 0 (n_min = 0) is the model of
+ * mp_set_model.  mp_predict, mp_select and mp_select_flows evaluate Eq 1-24 / Alg 1
+ * unchanged with the parameters of n's band.
+ * mp_set_model_band installs (or replaces, same n_min) band n_min > 0 of (src, dst):
+ * params[npaths] in the order of the pair's paths (npaths must equal the pair's path
+ * count; the path kinds are the base model's), port may be NULL (no shared port).
+ * mp_set_model drops every band of the pair.  Invalidates the config cache.
+ * Errors: MP_ERR_INVALID (n_min == 0, npaths mismatch, invalid parameters as in
+ * mp_set_model), MP_ERR_TOPOLOGY.
+ * mp_get_model_band reads band `band` (0 = base; ascending n_min): any output
+ * pointer may be NULL; *nbands (if not NULL) receives the band count; band < 0
+ * returns only the count.  Errors: MP_ERR_INVALID (band >= count). */
+int mp_set_model_band(mp_ctx *ctx, int src, int dst, uint64_t n_min, const mp_path_params *params,
+                      int npaths, const mp_port_params *port);
+int mp_get_model_band(mp_ctx *ctx, int src, int dst, int band, uint64_t *n_min,
+                      mp_path_params *params, int *npaths, mp_port_params *port, int *nbands);
+
 /* Selector options for this context (invalidates the cache). */
 int mp_set_options(mp_ctx *ctx, const mp_model_opts *opts);
 int mp_get_options(mp_ctx *ctx, mp_model_opts *opts);
@@ -310,6 +330,17 @@ int mp_stats(mp_ctx *ctx, uint64_t *kernel_launches);
  * α > 0); a non-positive slope falls back to β = n[m-1]/t[m-1].  m >= 2, else
  * MP_ERR_INVALID.  Pure host arithmetic, no context. */
 int mp_fit_hockney(const double *n, const double *t, int m, double *alpha, double *beta);
+
+/* The per-band Step-1 fit of reading C20 (NEXT f4), exposed for parity tests.
+ * edges[nedges]: band lower edges in bytes, edges[0] == 0, strictly increasing.
+ * Band j is fitted (as mp_fit_hockney) on the samples with edges[j] <= n[i] <=
+ * edges[j+1] (both inclusive; the last band is unbounded above).  A band with fewer
+ * than two samples takes the fit of the nearest band above it that has two, else of
+ * the nearest below.  alpha[nedges], beta[nedges] receive the fits (host arrays).
+ * Errors: MP_ERR_INVALID (bad edges, t <= 0, no band with two samples).  Pure host
+ * arithmetic, no context. */
+int mp_fit_bands(const double *n, const double *t, int m, const double *edges, int nedges,
+                 double *alpha, double *beta);
 
 #ifdef __cplusplus
 }

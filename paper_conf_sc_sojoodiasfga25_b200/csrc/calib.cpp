@@ -363,6 +363,47 @@ extern "C" int mp_fit_hockney(const double *n, const double *t, int m, double *a
   return MP_OK;
 }
 
+extern "C" int mp_fit_bands(const double *n, const double *t, int m, const double *edges, int nedges,
+                            double *alpha, double *beta) {
+  if (!n || !t || !edges || !alpha || !beta || m < 0 || nedges < 1 || edges[0] != 0.0) return MP_ERR_INVALID;
+  for (int j = 1; j < nedges; ++j)
+    if (!(edges[j] > edges[j - 1])) return MP_ERR_INVALID;
+  for (int i = 0; i < m; ++i)
+    if (!(t[i] > 0.0) || !(n[i] >= 0.0)) return MP_ERR_INVALID;
+  // reading C20: band j is fitted on the sizes in [e_j, e_{j+1}] (both inclusive)
+  std::vector<int> own(nedges, 0);
+  std::vector<Fit> fits(nedges);
+  for (int j = 0; j < nedges; ++j) {
+    const double lo = edges[j], hi = j + 1 < nedges ? edges[j + 1] : HUGE_VAL;
+    std::vector<double> bn, bt;
+    for (int i = 0; i < m; ++i)
+      if (n[i] >= lo && n[i] <= hi) {
+        bn.push_back(n[i]);
+        bt.push_back(t[i]);
+      }
+    if (bn.size() >= 2) {
+      fits[j] = fit_hockney(bn, bt);
+      own[j] = 1;
+    }
+  }
+  // a band without two sizes takes the nearest own fit above it, else below it
+  for (int j = 0; j < nedges; ++j) {
+    if (own[j]) continue;
+    int src = -1;
+    for (int i = j + 1; i < nedges && src < 0; ++i)
+      if (own[i]) src = i;
+    for (int i = j - 1; i >= 0 && src < 0; --i)
+      if (own[i]) src = i;
+    if (src < 0) return MP_ERR_INVALID;
+    fits[j] = fits[src];
+  }
+  for (int j = 0; j < nedges; ++j) {
+    alpha[j] = fits[j].alpha;
+    beta[j] = fits[j].beta;
+  }
+  return MP_OK;
+}
+
 extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");

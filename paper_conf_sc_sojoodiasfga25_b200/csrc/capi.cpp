@@ -90,6 +90,17 @@ PairModel *pair_model(mp_ctx *c, int src, int dst) {
   return &it->second;
 }
 
+// The model of the band holding a message of n bytes (reading C20): the last band
+// with n_min <= n, else the base model.
+const PairModel *model_for(mp_ctx *c, int src, int dst, uint64_t n) {
+  const PairModel *m = pair_model(c, src, dst);
+  auto it = c->bands.find(std::make_pair(src, dst));
+  if (it == c->bands.end()) return m;
+  for (const auto &b : it->second)
+    if (b.first <= n) m = &b.second;
+  return m;
+}
+
 void fill_config(const PairModel &m, const Selection &s, mp_config *out) {
   std::memset(out, 0, sizeof(*out));
   out->npaths = static_cast<int32_t>(m.paths.size());
@@ -517,7 +528,72 @@ int mp_set_model(mp_ctx *c, int src, int dst, const mp_path *paths, const mp_pat
     }
   }
   c->models[std::make_pair(src, dst)] = m;
+  c->bands.erase(std::make_pair(src, dst));  // a new base model drops the pair's bands
   c->cache.clear();
+  return MP_OK;
+}
+
+int mp_set_model_band(mp_ctx *c, int src, int dst, uint64_t n_min, const mp_path_params *prm, int npaths,
+                      const mp_port_params *port) {
+  if (!c || !prm) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  if (n_min == 0) return fail(c, MP_ERR_INVALID, "band n_min must be > 0 (band 0 is mp_set_model)");
+  const PairModel *base = pair_model(c, src, dst);
+  if (npaths != static_cast<int>(base->paths.size()))
+    return fail(c, MP_ERR_INVALID, "band path count must equal the pair's");
+  PairModel m = *base;
+  for (int i = 0; i < npaths; ++i) {
+    PathModel &p = m.paths[i];
+    p.alpha = prm[i].alpha;
+    p.beta = prm[i].beta;
+    p.alpha2 = prm[i].alpha2;
+    p.beta2 = prm[i].beta2;
+    p.eps = prm[i].eps;
+    p.c = prm[i].c;
+    p.sigma = prm[i].sigma;
+    p.w = prm[i].w;
+  }
+  m.port_alpha = port ? port->alpha : 0.0;
+  m.port_beta = port ? port->beta : 0.0;
+  const std::string why = validate_model(m);
+  if (!why.empty()) return fail(c, MP_ERR_INVALID, why);
+  auto &v = c->bands[std::make_pair(src, dst)];
+  auto it = std::find_if(v.begin(), v.end(),
+                         [&](const std::pair<uint64_t, PairModel> &b) { return b.first >= n_min; });
+  if (it != v.end() && it->first == n_min)
+    it->second = m;
+  else
+    v.insert(it, std::make_pair(n_min, m));
+  c->cache.clear();
+  return MP_OK;
+}
+
+int mp_get_model_band(mp_ctx *c, int src, int dst, int band, uint64_t *n_min, mp_path_params *prm,
+                      int *npaths, mp_port_params *port, int *nbands) {
+  if (!c) return MP_ERR_INVALID;
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  auto it = c->bands.find(std::make_pair(src, dst));
+  const int nb = 1 + (it == c->bands.end() ? 0 : static_cast<int>(it->second.size()));
+  if (nbands) *nbands = nb;
+  if (band < 0) return MP_OK;  // count only
+  if (band >= nb) return fail(c, MP_ERR_INVALID, "no such band");
+  uint64_t lo = 0;
+  if (band > 0) {
+    lo = it->second[band - 1].first;
+    m = &it->second[band - 1].second;
+  }
+  if (n_min) *n_min = lo;
+  if (npaths) *npaths = static_cast<int>(m->paths.size());
+  if (prm)
+    for (size_t i = 0; i < m->paths.size(); ++i) {
+      const PathModel &p = m->paths[i];
+      prm[i] = mp_path_params{p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w};
+    }
+  if (port) {
+    port->alpha = m->port_alpha;
+    port->beta = m->port_beta;
+  }
   return MP_OK;
 }
 
@@ -579,7 +655,7 @@ int mp_get_options(mp_ctx *c, mp_model_opts *o) {
 int mp_predict(mp_ctx *c, int src, int dst, uint64_t bytes, const mp_config *cfg, double *seconds) {
   if (!c || !cfg || !seconds) return fail(c, MP_ERR_INVALID, "null argument");
   if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
-  const PairModel *m = pair_model(c, src, dst);
+  const PairModel *m = model_for(c, src, dst, bytes);
   if (cfg->npaths != static_cast<int32_t>(m->paths.size()))
     return fail(c, MP_ERR_INVALID, "config npaths does not match the pair's paths");
   uint64_t sum = 0;
@@ -596,7 +672,7 @@ int mp_predict(mp_ctx *c, int src, int dst, uint64_t bytes, const mp_config *cfg
 int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_config *out) {
   if (!c || !out) return fail(c, MP_ERR_INVALID, "null argument");
   if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
-  const PairModel *m = pair_model(c, src, dst);
+  const PairModel *m = model_for(c, src, dst, bytes);
   // environment variables include/exclude path kinds (MPX_PATHS).
   if (c->env_kinds != 0x7u) {
     uint32_t eff = 0;
@@ -623,7 +699,7 @@ int mp_select_flows(mp_ctx *c, int nflows, const mp_flow *flows, mp_config *out)
   std::vector<FlowSpec> specs;
   for (int f = 0; f < nflows; ++f) {
     if (!pair_ok(c, flows[f].src, flows[f].dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
-    models.push_back(pair_model(c, flows[f].src, flows[f].dst));
+    models.push_back(model_for(c, flows[f].src, flows[f].dst, flows[f].bytes));
     FlowSpec s;
     s.src = flows[f].src;
     s.dst = flows[f].dst;
@@ -805,6 +881,15 @@ int mp_save_params(mp_ctx *c, const char *path) {
     for (const PathModel &p : m.paths)
       std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via,
                    p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
+    auto bt = c->bands.find(kv.first);
+    if (bt == c->bands.end()) continue;
+    for (const auto &b : bt->second) {
+      std::fprintf(f, "band %d %d %zu %llu %.17g %.17g\n", kv.first.first, kv.first.second, b.second.paths.size(),
+                   static_cast<unsigned long long>(b.first), b.second.port_alpha, b.second.port_beta);
+      for (const PathModel &p : b.second.paths)
+        std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via, p.alpha,
+                     p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
+    }
   }
   std::fclose(f);
   return MP_OK;
@@ -822,9 +907,13 @@ int mp_load_params(mp_ctx *c, const char *path) {
   }
   int src, dst;
   size_t np;
+  unsigned long long n_min = 0;
   double pa, pb;
-  while (std::fscanf(f, "%31s %d %d %zu %lf %lf", tag, &src, &dst, &np, &pa, &pb) == 6) {
-    if (std::strcmp(tag, "pair") || np < 1 || np > MP_MAX_PATHS) break;
+  while (std::fscanf(f, "%31s %d %d %zu", tag, &src, &dst, &np) == 4) {
+    const bool band = std::strcmp(tag, "band") == 0;
+    if ((!band && std::strcmp(tag, "pair")) || np < 1 || np > MP_MAX_PATHS) break;
+    if (band && std::fscanf(f, "%llu", &n_min) != 1) break;
+    if (std::fscanf(f, "%lf %lf", &pa, &pb) != 2) break;
     mp_path paths[MP_MAX_PATHS];
     mp_path_params prm[MP_MAX_PATHS];
     for (size_t i = 0; i < np; ++i) {
@@ -837,7 +926,9 @@ int mp_load_params(mp_ctx *c, const char *path) {
     }
     mp_port_params port{pa, pb};
     if (pair_ok(c, src, dst)) {
-      if (int s = mp_set_model(c, src, dst, paths, prm, static_cast<int>(np), &port)) {
+      const int s = band ? mp_set_model_band(c, src, dst, n_min, prm, static_cast<int>(np), &port)
+                         : mp_set_model(c, src, dst, paths, prm, static_cast<int>(np), &port);
+      if (s) {
         std::fclose(f);
         return s;
       }

@@ -72,6 +72,9 @@ struct mp_ctx {
   std::string last_error;
   mpx::ModelOpts opts;
   std::map<std::pair<int, int>, mpx::PairModel> models;
+  // NEXT f4 size bands (reading C20): per pair, (n_min, model) ascending, n_min > 0;
+  // the base model (models) is band 0 with n_min = 0.
+  std::map<std::pair<int, int>, std::vector<std::pair<uint64_t, mpx::PairModel>>> bands;
   std::unordered_map<mpx::CacheKey, mpx::Selection, mpx::CacheKeyHash> cache;
   uint32_t env_kinds = 0x7u;       // path kinds allowed by MPX_PATHS (bit = MP_PATH_*)
 

@@ -119,6 +119,14 @@ def lib():
             "mp_select_flows": (C.c_int, [P, C.c_int, C.POINTER(mp_flow), C.POINTER(mp_config)]),
             "mp_fit_hockney": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                          C.POINTER(C.c_double), C.POINTER(C.c_double)]),
+            "mp_set_model_band": (C.c_int, [P, C.c_int, C.c_int, C.c_uint64, C.POINTER(mp_path_params),
+                                            C.c_int, C.POINTER(mp_port_params)]),
+            "mp_get_model_band": (C.c_int, [P, C.c_int, C.c_int, C.c_int, C.POINTER(C.c_uint64),
+                                            C.POINTER(mp_path_params), C.POINTER(C.c_int),
+                                            C.POINTER(mp_port_params), C.POINTER(C.c_int)]),
+            "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
+                                       C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
+                                       C.POINTER(C.c_double)]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -133,7 +141,8 @@ def exported_symbols() -> List[str]:
             "mp_set_model", "mp_get_model", "mp_set_options", "mp_get_options", "mp_predict",
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
             "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
-            "mp_peer_base", "mp_select_flows", "mp_register", "mp_deregister"]
+            "mp_peer_base", "mp_select_flows", "mp_register", "mp_deregister",
+            "mp_set_model_band", "mp_get_model_band", "mp_fit_bands"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -144,6 +153,24 @@ def fit_hockney(n: Sequence[float], t: Sequence[float]):
     if st != 0:
         raise MPError(st, "mp_fit_hockney")
     return a.value, b.value
+
+
+def fit_bands(n: Sequence[float], t: Sequence[float], edges: Sequence[float]):
+    """mp_fit_bands: [(α_j, β_j)] per size band (reading C20, NEXT f4)."""
+    m, B = len(n), len(edges)
+    a, b = (C.c_double * B)(), (C.c_double * B)()
+    st = lib().mp_fit_bands((C.c_double * max(1, m))(*n), (C.c_double * max(1, m))(*t), m,
+                            (C.c_double * B)(*edges), B, a, b)
+    if st != 0:
+        raise MPError(st, "mp_fit_bands")
+    return [(a[j], b[j]) for j in range(B)]
+
+
+def _params_array(params: Sequence[dict]):
+    return (mp_path_params * MP_MAX_PATHS)(
+        *[mp_path_params(*[float(p.get(f, d)) for f, d in
+                           (("alpha", 0), ("beta", 0), ("alpha2", 0), ("beta2", 0), ("eps", 0),
+                            ("c", 1), ("sigma", 0), ("w", 0))]) for p in params])
 
 
 def _ptr(x) -> Optional[int]:
@@ -220,12 +247,29 @@ class Context:
     def set_model(self, src, dst, paths: Sequence, params: Sequence[dict], port: Optional[dict] = None):
         n = len(paths)
         pa = (mp_path * MP_MAX_PATHS)(*[mp_path(k, v) for k, v in paths])
-        pr = (mp_path_params * MP_MAX_PATHS)(
-            *[mp_path_params(*[float(p.get(f, d)) for f, d in
-                               (("alpha", 0), ("beta", 0), ("alpha2", 0), ("beta2", 0), ("eps", 0),
-                                ("c", 1), ("sigma", 0), ("w", 0))]) for p in params])
+        pr = _params_array(params)
         po = mp_port_params(port["alpha"], port["beta"]) if port else None
         self._ck(lib().mp_set_model(self.h, src, dst, pa, pr, n, C.byref(po) if po else None))
+
+    def set_model_band(self, src, dst, n_min, params: Sequence[dict], port: Optional[dict] = None):
+        """mp_set_model_band (NEXT f4, reading C20)."""
+        po = mp_port_params(port["alpha"], port["beta"]) if port else None
+        self._ck(lib().mp_set_model_band(self.h, src, dst, n_min, _params_array(params), len(params),
+                                         C.byref(po) if po else None))
+
+    def get_model_bands(self, src=0, dst=0):
+        """[(n_min, params, port)] of every band of (src, dst), ascending n_min."""
+        nb = C.c_int()
+        self._ck(lib().mp_get_model_band(self.h, src, dst, -1, None, None, None, None, C.byref(nb)))
+        out = []
+        for j in range(nb.value):
+            lo, n = C.c_uint64(), C.c_int()
+            pr = (mp_path_params * MP_MAX_PATHS)()
+            po = mp_port_params()
+            self._ck(lib().mp_get_model_band(self.h, src, dst, j, C.byref(lo), pr, C.byref(n), C.byref(po), None))
+            out.append((lo.value, [{f: getattr(pr[i], f) for f, _ in mp_path_params._fields_}
+                                   for i in range(n.value)], dict(alpha=po.alpha, beta=po.beta)))
+        return out
 
     def get_model(self, src=0, dst=0):
         pa = (mp_path * MP_MAX_PATHS)()
