@@ -317,6 +317,18 @@ int mp_sync(mp_ctx *ctx);
  * MP_ERR_STATE. */
 int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
 
+/* NEXT f4 (P:360 Observation 4): Step 1 per size band (readings C20, C21).  Every
+ * link is sampled over 4 KiB .. 1 GiB (capped by the rings / heap) with OMB-style
+ * windows of back-to-back copies between the same buffers and fitted
+ * per band (as mp_fit_bands); band 0 replaces the pair's model (mp_set_model), band
+ * j >= 1 is installed with mp_set_model_band(edges[j]).  ε and, when the pair already
+ * has a model, the φ multipliers c are kept (run mp_calibrate first).
+ * edges[nedges]: band lower edges in bytes, edges[0] == 0, strictly increasing; NULL
+ * = {0, 256 KiB, 4 MiB, 32 MiB, 128 MiB}.  reps: windows per size (median).
+ * Collective when world > 1 (same rules as mp_calibrate).
+ * Errors: MP_ERR_STATE (model-only), MP_ERR_INVALID (bad edges), MP_ERR_CUDA. */
+int mp_calibrate_bands(mp_ctx *ctx, const uint64_t *edges, int nedges, int reps);
+
 /* Save / load the model parameters of every pair (Step 1/2). */
 int mp_save_params(mp_ctx *ctx, const char *path);
 int mp_load_params(mp_ctx *ctx, const char *path);

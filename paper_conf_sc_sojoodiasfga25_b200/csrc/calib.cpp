@@ -87,6 +87,88 @@ int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double
   return MP_OK;
 }
 
+// OMB-style timing (reading C21): `W` back-to-back copies of n bytes between the
+// same buffers (no flush — a window of repeated sends), median over
+// `reps` windows; returns seconds per message.
+int time_window(Bench &b, void *dst, const void *src, uint64_t n, int reps, int W, double *out, int ctas = 0) {
+  mp_ctx *c = b.c;
+  std::vector<double> ts;
+  for (int r = 0; r < reps + 1; ++r) {
+    CKC(cudaEventRecord(b.e0, b.s));
+    for (int w = 0; w < W; ++w)
+      if (int st = launch_direct_copy(c, dst, src, n, b.s, ctas)) return st;
+    CKC(cudaEventRecord(b.e1, b.s));
+    CKC(cudaEventSynchronize(b.e1));
+    float ms = 0;
+    CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
+    if (r > 0) ts.push_back(ms * 1e-3 / W);  // first window is a warm-up
+  }
+  *out = median(ts);
+  return MP_OK;
+}
+
+// Samples (n, t) of one link over `sizes` (<= cap): window-timed when `window`,
+// else single copies with the L2 flushed before each.
+int sample_link(Bench &b, void *dst, const void *src, const std::vector<uint64_t> &sizes, uint64_t cap, int reps,
+                int ctas, bool window, std::vector<double> *n, std::vector<double> *t) {
+  for (uint64_t s : sizes) {
+    if (s > cap) continue;
+    double sec = 0;
+    if (window) {
+      const int W = s <= (64ull << 20) ? 16 : 4;
+      if (int st = time_window(b, dst, src, s, reps, W, &sec, ctas)) return st;
+    } else {
+      if (int st = time_copy(b, dst, src, s, reps, &sec, ctas)) return st;
+    }
+    n->push_back(static_cast<double>(s));
+    t->push_back(sec);
+  }
+  return MP_OK;
+}
+
+// Reading C20: band j is fitted on the samples with e_j <= n <= e_{j+1} (both
+// inclusive; the last band unbounded); a band without two samples takes the fit of
+// the nearest band above it that has two, else of the nearest below.  Returns false
+// when no band has two samples.
+bool fit_bands_impl(const std::vector<double> &n, const std::vector<double> &t, const std::vector<double> &edges,
+                    std::vector<Fit> *out) {
+  const int B = static_cast<int>(edges.size());
+  std::vector<int> own(B, 0);
+  std::vector<Fit> fits(B, Fit{0, 0});
+  for (int j = 0; j < B; ++j) {
+    const double lo = edges[j], hi = j + 1 < B ? edges[j + 1] : HUGE_VAL;
+    std::vector<double> bn, bt;
+    for (size_t i = 0; i < n.size(); ++i)
+      if (n[i] >= lo && n[i] <= hi) {
+        bn.push_back(n[i]);
+        bt.push_back(t[i]);
+      }
+    if (bn.size() >= 2) {
+      fits[j] = fit_hockney(bn, bt);
+      own[j] = 1;
+    }
+  }
+  for (int j = 0; j < B; ++j) {
+    if (own[j]) continue;
+    int from = -1;
+    for (int i = j + 1; i < B && from < 0; ++i)
+      if (own[i]) from = i;
+    for (int i = j - 1; i >= 0 && from < 0; --i)
+      if (own[i]) from = i;
+    if (from < 0) return false;
+    fits[j] = fits[from];
+  }
+  *out = fits;
+  return true;
+}
+
+int fit_samples(mp_ctx *c, const std::vector<double> &n, const std::vector<double> &t,
+                const std::vector<double> &edges, std::vector<Fit> *out) {
+  if (!fit_bands_impl(n, t, edges, out))
+    return cfail(c, MP_ERR_INVALID, "calibration needs at least two sizes in some band");
+  return MP_OK;
+}
+
 // Fit one link.  ctas > 0 times the copy with that many CTAs: a staged leg is moved
 // by a stage group of relay_ctas CTAs, so its β is what that group achieves.
 int fit_link(Bench &b, void *dst, const void *src, const std::vector<uint64_t> &sizes, uint64_t cap,
@@ -106,8 +188,9 @@ int fit_link(Bench &b, void *dst, const void *src, const std::vector<uint64_t> &
 
 // Two links timed concurrently (dst1 ← src1 on one stream, dst2 ← src2 on another,
 // launched together), each fitted on its own times.
-int fit_links_duplex(Bench &b, void *dst1, const void *src1, void *dst2, const void *src2,
-                     const std::vector<uint64_t> &sizes, int reps, Fit *f1, Fit *f2, int ctas) {
+int sample_links_duplex(Bench &b, void *dst1, const void *src1, void *dst2, const void *src2,
+                        const std::vector<uint64_t> &sizes, int reps, int ctas, bool flush, std::vector<double> *pn,
+                        std::vector<double> *pt1, std::vector<double> *pt2) {
   mp_ctx *c = b.c;
   cudaStream_t s2 = nullptr;
   cudaEvent_t fork = nullptr, e2a = nullptr, e2b = nullptr;
@@ -120,7 +203,7 @@ int fit_links_duplex(Bench &b, void *dst1, const void *src1, void *dst2, const v
   for (uint64_t s : sizes) {
     std::vector<double> a, bb;
     for (int r = 0; r < reps + 1 && st == MP_OK; ++r) {
-      cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s);
+      if (flush) cudaMemsetAsync(b.flush, r & 0xff, b.flush_bytes, b.s);
       cudaEventRecord(fork, b.s);
       cudaStreamWaitEvent(s2, fork, 0);
       cudaEventRecord(b.e0, b.s);
@@ -150,7 +233,17 @@ int fit_links_duplex(Bench &b, void *dst1, const void *src1, void *dst2, const v
   cudaEventDestroy(e2a);
   cudaEventDestroy(e2b);
   if (st) return st;
-  if (n.size() < 2) return cfail(c, MP_ERR_INVALID, "calibration needs at least two sizes");
+  *pn = n;
+  *pt1 = t1;
+  *pt2 = t2;
+  return MP_OK;
+}
+
+int fit_links_duplex(Bench &b, void *dst1, const void *src1, void *dst2, const void *src2,
+                     const std::vector<uint64_t> &sizes, int reps, Fit *f1, Fit *f2, int ctas) {
+  std::vector<double> n, t1, t2;
+  if (int st = sample_links_duplex(b, dst1, src1, dst2, src2, sizes, reps, ctas, true, &n, &t1, &t2)) return st;
+  if (n.size() < 2) return cfail(b.c, MP_ERR_INVALID, "calibration needs at least two sizes");
   *f1 = fit_hockney(n, t1);
   *f2 = fit_hockney(n, t2);
   return MP_OK;
@@ -257,8 +350,12 @@ struct LinkMeas {
   double eps_dev, eps_host;
 };
 
-int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
+// edges = {0}: the plain Step-1 fit (flushed single copies); more edges: one
+// parameter set per size band (reading C20), window-timed (reading C21).
+int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std::vector<double> &edges,
+                    bool window) {
   const int W = c->world, me = c->rank, succ = (c->rank + 1) % c->world;
+  const int B = static_cast<int>(edges.size());
   // the successor's heap is used as the put target: nobody may have live buffers yet
   int32_t busy = c->heap.used_.empty() ? 0 : 1;
   std::vector<int32_t> all_busy(W);
@@ -282,17 +379,18 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
   CKC(cudaMalloc(&b.flush, b.flush_bytes));
   CKC(cudaMalloc(&src, big));
   CKC(cudaMemset(src, 0x5a, big));
-  LinkMeas m{};
+  std::vector<LinkMeas> m(B, LinkMeas{});
   int st = MP_OK;
   do {
-    Fit fd{}, fh1{}, fh2{};
-    if ((st = fit_link(b, c->peers[succ].heap, src, sz, big, reps, &fd))) break;
-    m.da = fd.alpha;
-    m.db = fd.beta;
-    Fit fr{};
-    if ((st = fit_link(b, c->peers[succ].heap, src, sz, big, reps, &fr, c->relay_ctas))) break;
-    m.ra = fr.alpha;
-    m.rb = fr.beta;
+    std::vector<double> n, t;
+    std::vector<Fit> fd, fr, fh1, fh2;
+    if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, 0, window, &n, &t))) break;
+    if ((st = fit_samples(c, n, t, edges, &fd))) break;
+    n.clear();
+    t.clear();
+    if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, c->relay_ctas, window, &n, &t))) break;
+    if ((st = fit_samples(c, n, t, edges, &fr))) break;
+    double eps_host = 0, eps_dev = 0;
     if (c->host_path) {
       // the own segment's ring of sender == me is never used for traffic
       uint8_t *hr = c->hseg[me] + static_cast<uint64_t>(me) * c->hseg_per_src;
@@ -301,16 +399,33 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
       for (uint64_t s : sz)
         if (s <= std::min<uint64_t>(hcap, 64ull << 20)) hs.push_back(s);
       if (hs.size() < 2) hs = {hcap / 4, hcap / 2};
-      if ((st = fit_link(b, hr, src, hs, hcap, std::max(3, reps / 2), &fh1, c->relay_ctas))) break;
-      if ((st = fit_link(b, src, hr, hs, hcap, std::max(3, reps / 2), &fh2, c->relay_ctas))) break;
-      m.h1a = fh1.alpha;
-      m.h1b = fh1.beta;
-      m.h2a = fh2.alpha;
-      m.h2b = fh2.beta;
-      if ((st = time_pingpong(b, c->h_probe, true, 500, &m.eps_host))) break;
+      const int hr_reps = std::max(3, reps / 2);
+      n.clear();
+      t.clear();
+      if ((st = sample_link(b, hr, src, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) break;
+      if ((st = fit_samples(c, n, t, edges, &fh1))) break;
+      n.clear();
+      t.clear();
+      if ((st = sample_link(b, src, hr, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) break;
+      if ((st = fit_samples(c, n, t, edges, &fh2))) break;
+      if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) break;
     }
     uint64_t *pf = reinterpret_cast<uint64_t *>(c->peers[succ].ctrl + c->L.probe);
-    if ((st = time_pingpong(b, pf, false, 1000, &m.eps_dev))) break;
+    if ((st = time_pingpong(b, pf, false, 1000, &eps_dev))) break;
+    for (int j = 0; j < B; ++j) {
+      m[j].da = fd[j].alpha;
+      m[j].db = fd[j].beta;
+      m[j].ra = fr[j].alpha;
+      m[j].rb = fr[j].beta;
+      if (c->host_path) {
+        m[j].h1a = fh1[j].alpha;
+        m[j].h1b = fh1[j].beta;
+        m[j].h2a = fh2[j].alpha;
+        m[j].h2b = fh2[j].beta;
+      }
+      m[j].eps_dev = eps_dev;
+      m[j].eps_host = eps_host;
+    }
   } while (false);
   cudaStreamSynchronize(b.s);
   cudaFree(src);
@@ -324,34 +439,171 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps) {
   if (st) return st;
   for (int32_t v : all_ok)
     if (v) return cfail(c, MP_ERR_STATE, "calibration failed on another rank");
-  std::vector<LinkMeas> lm(W);
-  if (int s = world_allgather(c, &m, lm.data(), sizeof(LinkMeas))) return s;
+  std::vector<LinkMeas> lm(static_cast<size_t>(W) * B);  // [rank][band]
+  if (int s = world_allgather(c, m.data(), lm.data(), sizeof(LinkMeas) * B)) return s;
 
   for (int s = 0; s < W; ++s)
     for (int d = 0; d < W; ++d) {
       if (s == d) continue;
-      mp_path paths[MP_MAX_PATHS];
-      mp_path_params prm[MP_MAX_PATHS];
-      int np = 0;
-      paths[np] = mp_path{MP_PATH_DIRECT, -1};
-      prm[np++] = mp_path_params{lm[s].da, lm[s].db, 0, 0, 0, 1, 0, 1};
-      for (int r = 0; r < W; ++r) {
-        if (r == s || r == d) continue;
-        paths[np] = mp_path{MP_PATH_GPU, r};
-        prm[np++] = mp_path_params{lm[s].ra, lm[s].rb, lm[r].ra, lm[r].rb, std::max(lm[r].eps_dev, 1e-8), 1, 0, 1};
+      // φ multipliers of an existing model are kept (Step-1 band fits replace α, β only)
+      mp_path_params old[MP_MAX_PATHS];
+      int nold = 0;
+      const bool keep_c = B > 1 && mp_get_model(c, s, d, nullptr, old, &nold, nullptr) == MP_OK;
+      for (int j = 0; j < B; ++j) {
+        const LinkMeas &S = lm[static_cast<size_t>(s) * B + j], &D = lm[static_cast<size_t>(d) * B + j];
+        mp_path paths[MP_MAX_PATHS];
+        mp_path_params prm[MP_MAX_PATHS];
+        int np = 0;
+        paths[np] = mp_path{MP_PATH_DIRECT, -1};
+        prm[np++] = mp_path_params{S.da, S.db, 0, 0, 0, 1, 0, 1};
+        for (int r = 0; r < W; ++r) {
+          if (r == s || r == d) continue;
+          const LinkMeas &R = lm[static_cast<size_t>(r) * B + j];
+          paths[np] = mp_path{MP_PATH_GPU, r};
+          prm[np++] = mp_path_params{S.ra, S.rb, R.ra, R.rb, std::max(R.eps_dev, 1e-8), 1, 0, 1};
+        }
+        if (c->host_path) {
+          paths[np] = mp_path{MP_PATH_HOST, -1};
+          prm[np++] = mp_path_params{S.h1a, S.h1b, D.h2a, D.h2b, std::max(D.eps_host, 1e-8), 1, 0, 0};
+        }
+        if (keep_c && nold == np)
+          for (int i = 0; i < np; ++i) prm[i].c = old[i].c;
+        mp_port_params port{S.da, S.db};
+        const int e = j == 0 ? mp_set_model(c, s, d, paths, prm, np, &port)
+                             : mp_set_model_band(c, s, d, static_cast<uint64_t>(edges[j]), prm, np, &port);
+        if (e) return e;
       }
-      if (c->host_path) {
-        paths[np] = mp_path{MP_PATH_HOST, -1};
-        prm[np++] = mp_path_params{lm[s].h1a, lm[s].h1b, lm[d].h2a, lm[d].h2b, std::max(lm[d].eps_host, 1e-8),
-                                   1, 0, 0};
-      }
-      mp_port_params port{lm[s].da, lm[s].db};
-      if (int e = mp_set_model(c, s, d, paths, prm, np, &port)) return e;
     }
   return world_barrier(c);
 }
 
+// Loopback size bands (reading C20/C21): every link of the pair (0, 0) is sampled
+// window-timed over 4 KiB .. 1 GiB and fitted per band; ε, φ multipliers c, σ and w
+// are kept from the installed model (mp_calibrate / mp_load_params).
+int calibrate_loop_bands(mp_ctx *c, const std::vector<double> &edges, int reps) {
+  const int B = static_cast<int>(edges.size());
+  mp_path paths[MP_MAX_PATHS];
+  mp_path_params base[MP_MAX_PATHS];
+  int np = 0;
+  if (int s = mp_get_model(c, 0, 0, paths, base, &np, nullptr)) return s;
+  std::vector<uint64_t> sizes;
+  for (uint64_t s = 4096; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
+  const uint64_t big = sizes.back();
+  const uint64_t ring_cap = static_cast<uint64_t>(c->slots) * c->slot_bytes;
+  Bench b;
+  b.c = c;
+  CKC(cudaSetDevice(c->device));
+  CKC(cudaStreamCreateWithFlags(&b.s, cudaStreamNonBlocking));
+  CKC(cudaEventCreate(&b.e0));
+  CKC(cudaEventCreate(&b.e1));
+  void *src = nullptr, *dst = nullptr;
+  CKC(cudaMalloc(&b.flush, b.flush_bytes));
+  CKC(cudaMalloc(&src, big));
+  CKC(cudaMalloc(&dst, big));
+  CKC(cudaMemset(src, 0x5a, big));
+  int st = MP_OK;
+  std::vector<Fit> fd, f1, f2, fh1, fh2;
+  do {
+    std::vector<double> n, t, t2;
+    if ((st = sample_link(b, dst, src, sizes, big, reps, 0, true, &n, &t))) break;
+    if ((st = fit_samples(c, n, t, edges, &fd))) break;
+    if (c->n_loop_relays > 0) {
+      uint8_t *ring = c->rings[0].data;
+      n.clear();
+      t.clear();
+      if ((st = sample_link(b, ring, src, sizes, ring_cap, reps, c->relay_ctas, true, &n, &t))) break;
+      if ((st = fit_samples(c, n, t, edges, &f1))) break;
+      n.clear();
+      t.clear();
+      if ((st = sample_link(b, dst, ring, sizes, ring_cap, reps, c->relay_ctas, true, &n, &t))) break;
+      if ((st = fit_samples(c, n, t, edges, &f2))) break;
+    }
+    if (c->host_path) {
+      uint8_t *hr = c->rings[c->n_loop_relays].data;
+      std::vector<uint64_t> hs;
+      for (uint64_t s : sizes)
+        if (s <= std::min<uint64_t>(ring_cap / 2, 64ull << 20)) hs.push_back(s);
+      n.clear();
+      t.clear();
+      if ((st = sample_links_duplex(b, hr, src, dst, hr + ring_cap / 2, hs, std::max(3, reps / 2), c->relay_ctas,
+                                    false, &n, &t, &t2)))
+        break;
+      if ((st = fit_samples(c, n, t, edges, &fh1))) break;
+      if ((st = fit_samples(c, n, t2, edges, &fh2))) break;
+    }
+  } while (false);
+  cudaStreamSynchronize(b.s);
+  cudaFree(src);
+  cudaFree(dst);
+  cudaFree(b.flush);
+  cudaEventDestroy(b.e0);
+  cudaEventDestroy(b.e1);
+  cudaStreamDestroy(b.s);
+  if (st) return st;
+  int32_t derr = 0;
+  CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
+  if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration copy timed out");
+  for (int j = 0; j < B; ++j) {
+    mp_path_params prm[MP_MAX_PATHS];
+    for (int i = 0; i < np; ++i) {
+      prm[i] = base[i];
+      if (paths[i].kind == MP_PATH_DIRECT) {
+        prm[i].alpha = fd[j].alpha;
+        prm[i].beta = fd[j].beta;
+      } else if (paths[i].kind == MP_PATH_GPU) {
+        prm[i].alpha = f1[j].alpha;
+        prm[i].beta = f1[j].beta;
+        prm[i].alpha2 = f2[j].alpha;
+        prm[i].beta2 = f2[j].beta;
+      } else {
+        prm[i].alpha = fh1[j].alpha;
+        prm[i].beta = fh1[j].beta;
+        prm[i].alpha2 = fh2[j].alpha;
+        prm[i].beta2 = fh2[j].beta;
+      }
+    }
+    mp_port_params port{fd[j].alpha, 2.0 * fd[j].beta};  // HBM: read + write per direct byte
+    const int e = j == 0 ? mp_set_model(c, 0, 0, paths, prm, np, &port)
+                         : mp_set_model_band(c, 0, 0, static_cast<uint64_t>(edges[j]), prm, np, &port);
+    if (e) return e;
+  }
+  return MP_OK;
+}
+
 }  // namespace
+
+extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedges, int reps) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (reps <= 0) reps = 5;
+  std::vector<double> edges;
+  if (edges_in && nedges > 0) {
+    if (edges_in[0] != 0) return cfail(c, MP_ERR_INVALID, "band edges must start at 0");
+    for (int j = 0; j < nedges; ++j) {
+      if (j > 0 && edges_in[j] <= edges_in[j - 1]) return cfail(c, MP_ERR_INVALID, "band edges must increase");
+      edges.push_back(static_cast<double>(edges_in[j]));
+    }
+  } else {
+    for (uint64_t e : {0ull, 256ull << 10, 4ull << 20, 32ull << 20, 128ull << 20}) edges.push_back(static_cast<double>(e));
+  }
+  if (c->world != 1) {
+    std::vector<uint64_t> sizes;
+    for (uint64_t s = 4096; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
+    const bool was_running = c->relay_running;
+    if (int s = world_stop_relay(c)) return s;
+    int s = calibrate_world(c, sizes, reps, edges, true);
+    if (was_running) {
+      const int r = world_start_relay(c);
+      if (!s) s = r;
+    }
+    if (s) return s;
+    int32_t derr = 0;
+    CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
+    if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration probe timed out");
+    return MP_OK;
+  }
+  return calibrate_loop_bands(c, edges, reps);
+}
 
 extern "C" int mp_fit_hockney(const double *n, const double *t, int m, double *alpha, double *beta) {
   if (!n || !t || !alpha || !beta || m < 2) return MP_ERR_INVALID;
@@ -370,33 +622,10 @@ extern "C" int mp_fit_bands(const double *n, const double *t, int m, const doubl
     if (!(edges[j] > edges[j - 1])) return MP_ERR_INVALID;
   for (int i = 0; i < m; ++i)
     if (!(t[i] > 0.0) || !(n[i] >= 0.0)) return MP_ERR_INVALID;
-  // reading C20: band j is fitted on the sizes in [e_j, e_{j+1}] (both inclusive)
-  std::vector<int> own(nedges, 0);
-  std::vector<Fit> fits(nedges);
-  for (int j = 0; j < nedges; ++j) {
-    const double lo = edges[j], hi = j + 1 < nedges ? edges[j + 1] : HUGE_VAL;
-    std::vector<double> bn, bt;
-    for (int i = 0; i < m; ++i)
-      if (n[i] >= lo && n[i] <= hi) {
-        bn.push_back(n[i]);
-        bt.push_back(t[i]);
-      }
-    if (bn.size() >= 2) {
-      fits[j] = fit_hockney(bn, bt);
-      own[j] = 1;
-    }
-  }
-  // a band without two sizes takes the nearest own fit above it, else below it
-  for (int j = 0; j < nedges; ++j) {
-    if (own[j]) continue;
-    int src = -1;
-    for (int i = j + 1; i < nedges && src < 0; ++i)
-      if (own[i]) src = i;
-    for (int i = j - 1; i >= 0 && src < 0; --i)
-      if (own[i]) src = i;
-    if (src < 0) return MP_ERR_INVALID;
-    fits[j] = fits[src];
-  }
+  std::vector<Fit> fits;
+  if (!fit_bands_impl(std::vector<double>(n, n + m), std::vector<double>(t, t + m),
+                      std::vector<double>(edges, edges + nedges), &fits))
+    return MP_ERR_INVALID;
   for (int j = 0; j < nedges; ++j) {
     alpha[j] = fits[j].alpha;
     beta[j] = fits[j].beta;
@@ -419,7 +648,7 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
     // kernel must not be running (it resumes at its saved ring positions).
     const bool was_running = c->relay_running;
     if (int s = world_stop_relay(c)) return s;
-    int s = calibrate_world(c, sizes, reps);
+    int s = calibrate_world(c, sizes, reps, std::vector<double>{0.0}, false);
     if (was_running) {
       const int r = world_start_relay(c);
       if (!s) s = r;

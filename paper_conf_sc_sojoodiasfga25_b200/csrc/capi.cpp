@@ -251,6 +251,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   P.err = c->d_err;
   P.copy_mode = c->copy_mode;
   P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
+  P.allow_small = 1;
   const int cap = std::max(1, c->per_sm * c->sms);
   uint32_t staged_ctas = 0;
   for (int i = 1; i < cfg.npaths; ++i)
@@ -312,6 +313,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   P.err = c->d_err;
   P.copy_mode = c->copy_mode;
   P.bulk_stages = bulk_stages_for(n);
+  P.allow_small = ctas > 0 ? 0u : 1u;  // a staged leg's calibration times its group's CTAs
   P.npaths = 1;
   DevPath &d = P.p[0];
   d.kind = DK_DIRECT;

@@ -706,7 +706,27 @@ __global__ void __launch_bounds__(kThreads, 4) direct_kernel(const __grid_consta
   bulk_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
 }
 
-__global__ void __launch_bounds__(kThreads, 4) direct_reg_kernel(const __grid_constant__ DirectArgs A) {
+// One-shot small copy (co-aligned src/dst): thread i of the grid moves vector i of the
+// 16-B body; the last CTA also moves the < 16-byte head and tail.  Kept tiny and
+// branch-light on purpose: at these sizes a launch on a cold SM is bound by its
+// instruction fetches, not by the bytes.
+__global__ void __launch_bounds__(kThreads) direct_small_kernel(uint8_t *dst, const uint8_t *src, uint64_t n) {
+  uint64_t head = (16u - (reinterpret_cast<uintptr_t>(src) & 15u)) & 15u;
+  if (head > n) head = n;
+  const uint64_t nvec = (n - head) >> 4;
+  const uint64_t i = static_cast<uint64_t>(blockIdx.x) * kThreads + threadIdx.x;
+  if (i < nvec)
+    st16(reinterpret_cast<uint4 *>(dst + head) + i, ld16<LD_SRC>(reinterpret_cast<const uint4 *>(src + head) + i));
+  if (blockIdx.x + 1 == gridDim.x) {
+    const uint64_t t0 = head + (nvec << 4);
+    if (threadIdx.x < head) dst[threadIdx.x] = ld1<LD_SRC>(src + threadIdx.x);
+    if (threadIdx.x < n - t0) dst[t0 + threadIdx.x] = ld1<LD_SRC>(src + t0 + threadIdx.x);
+  }
+}
+
+// LDG/STG direct copy (MPX_COPY=reg): no min-blocks bound, so the 4-deep unrolled
+// vector loop gets the registers it needs (a 64-register cap made it spill).
+__global__ void __launch_bounds__(kThreads) direct_reg_kernel(const __grid_constant__ DirectArgs A) {
   group_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x);
 }
 
@@ -717,6 +737,14 @@ int launch_xfer(const XferParams &P, void *stream) {
   bool direct_only = P.p[0].kind == DK_DIRECT && P.p[0].cta0_in == 0 && P.p[0].g_in == P.nblocks;
   for (uint32_t i = 1; i < P.npaths; ++i)
     if (P.p[i].bytes) direct_only = false;
+  if (direct_only && P.allow_small && P.p[0].bytes <= kSmallMax &&
+      ((reinterpret_cast<uintptr_t>(P.p[0].dst) ^ reinterpret_cast<uintptr_t>(P.p[0].src)) & 15u) == 0) {
+    const uint64_t nvec = P.p[0].bytes >> 4;
+    const uint32_t g = static_cast<uint32_t>(nvec ? (nvec + kThreads - 1) / kThreads : 1);
+    direct_small_kernel<<<g, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P.p[0].dst, P.p[0].src,
+                                                                               P.p[0].bytes);
+    return static_cast<int>(cudaGetLastError());
+  }
   if (direct_only) {
     const DirectArgs A{P.p[0].dst, P.p[0].src, P.p[0].bytes, P.copy_mode, P.bulk_stages};
     if (P.copy_mode == 1)
@@ -763,6 +791,7 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_small_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_gate_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);

@@ -52,10 +52,19 @@ struct XferParams {
   uint32_t nblocks;
   uint32_t copy_mode;    // direct group: 0 = LDG/STG vectors, 1 = TMA bulk (cp.async.bulk)
   uint32_t bulk_stages;  // TMA pipeline depth per CTA (1..4)
+  uint32_t allow_small;  // 1: a small direct-only message may use the one-shot kernel
+  uint32_t pad_;
   uint64_t timeout_ns;
   int32_t *err;          // device (or mapped host) error word
   DevPath p[kMaxPaths];
 };
+
+// Direct-only messages up to this size (co-aligned mod 16) go to the one-shot kernel:
+// one 16-B vector per thread, every load in flight at once, ~20 instructions of
+// straight-line code (profiles/r01/smallbench*.jsonl: 2.1-3.1 µs per back-to-back
+// message vs 4.1 µs for the TMA pipeline kernel, whose cold instruction fetches
+// dominate at these sizes).
+constexpr uint64_t kSmallMax = 1ull << 20;
 
 // Launch the fused transfer kernel (engine.cu).  Returns a cudaError_t value.
 int launch_xfer(const XferParams &P, void *stream);

@@ -124,6 +124,7 @@ def lib():
             "mp_get_model_band": (C.c_int, [P, C.c_int, C.c_int, C.c_int, C.POINTER(C.c_uint64),
                                             C.POINTER(mp_path_params), C.POINTER(C.c_int),
                                             C.POINTER(mp_port_params), C.POINTER(C.c_int)]),
+            "mp_calibrate_bands": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
                                        C.POINTER(C.c_double)]),
@@ -142,7 +143,7 @@ def exported_symbols() -> List[str]:
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
             "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
             "mp_peer_base", "mp_select_flows", "mp_register", "mp_deregister",
-            "mp_set_model_band", "mp_get_model_band", "mp_fit_bands"]
+            "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -364,6 +365,14 @@ class Context:
             self._ck(lib().mp_calibrate(self.h, arr, len(sizes), reps))
         else:
             self._ck(lib().mp_calibrate(self.h, None, 0, reps))
+
+    def calibrate_bands(self, edges: Optional[Sequence[int]] = None, reps=0):
+        """mp_calibrate_bands (NEXT f4, readings C20/C21)."""
+        if edges:
+            arr = (C.c_uint64 * len(edges))(*edges)
+            self._ck(lib().mp_calibrate_bands(self.h, arr, len(edges), reps))
+        else:
+            self._ck(lib().mp_calibrate_bands(self.h, None, 0, reps))
 
     def save_params(self, path):
         self._ck(lib().mp_save_params(self.h, path.encode()))

@@ -52,6 +52,14 @@ def test_direct_only(ctx, n):
     run(ctx, n, [n] + [0] * (np_ - 1), [1] + [0] * (np_ - 1))
 
 
+@pytest.mark.parametrize("n", [1, 17, 4096 + 5, 300000, 1 << 20])
+@pytest.mark.parametrize("src_off,dst_off", [(1, 1), (3, 3), (15, 15), (1, 0), (16, 0)])
+def test_direct_only_small_misaligned(ctx, n, src_off, dst_off):
+    # the one-shot small-message kernel (co-aligned) and its fallback (not co-aligned)
+    np_ = len(ctx.paths())
+    run(ctx, n, [n] + [0] * (np_ - 1), [1] + [0] * (np_ - 1), src_off, dst_off)
+
+
 @pytest.mark.parametrize("src_off,dst_off", [(0, 0), (1, 1), (8, 8), (15, 15), (16, 0), (1, 0), (3, 7)])
 def test_all_paths_misaligned(ctx, src_off, dst_off):
     ps = ctx.paths()
@@ -221,6 +229,52 @@ def test_calibration_installs_sane_parameters():
     assert port["beta"] > d["beta"]
     # φ multipliers (C4) fitted from the measured best chunk counts
     assert 0.1 <= prm[1]["c"] <= 10 and 0.1 <= h["c"] <= 10
+    c.close()
+
+
+def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
+    # NEXT f4 (P:360 Observation 4; readings C20/C21): the per-band Step-1 fit installs
+    # one parameter set per band, and the model error at small sizes — where the single
+    # asymptotic Hockney line over-estimates the time — drops.
+    c = mp.Context(device=0, n_loop_relays=2, host_path=1, slot_bytes=32 * MiB, heap_bytes=16 * MiB)
+    c.set_options(mode=mp.MP_MODEL_B200)
+    c.calibrate(reps=3)
+    sizes = [64 << 10, 1 * MiB, 8 * MiB]
+    src = torch.randint(0, 256, (8 * MiB,), dtype=torch.uint8, device="cuda")
+    dst = torch.empty_like(src)
+    s = torch.cuda.Stream()
+
+    def window_time(n, cfg, w=16, reps=5):
+        ts = []
+        for _ in range(reps + 1):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            for _ in range(w):
+                c.xfer(dst, src, n, cfg, s)
+            e1.record(s)
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1) * 1e-3 / w)
+        return sorted(ts[1:])[reps // 2]
+
+    err_base = []
+    for n in sizes:
+        cfg = c.select(0, 0, n)
+        err_base.append(abs(cfg.t_pred - window_time(n, cfg)) / window_time(n, cfg))
+    edges = [0, 256 << 10, 4 * MiB, 32 * MiB, 128 * MiB]
+    c.calibrate_bands(edges, reps=3)
+    bands = c.get_model_bands(0, 0)
+    assert [b[0] for b in bands] == edges
+    for _, prm, port in bands:
+        assert all(p["beta"] > 0 and p["alpha"] > 0 for p in prm) and port["beta"] > 0
+    err_band = []
+    for n in sizes:
+        cfg = c.select(0, 0, n)
+        t = window_time(n, cfg)
+        err_band.append(abs(cfg.t_pred - t) / t)
+    assert max(err_band) < 0.35 and sum(err_band) < sum(err_base), (err_base, err_band)
+    ctx_sum = dict(base=err_base, bands=err_band)
+    print("E_pred base vs banded", ctx_sum)
     c.close()
 
 
