@@ -617,6 +617,17 @@ def main():
         "baselines": base,
         "per_path": per_path,
     }
+    # NEXT f4 (readings C20/C21): the same message modelled with per-band Step-1
+    # parameters (calibrated after the timed region; the pick is unchanged at 1 GiB)
+    if not (args.no_calibrate or args.params):
+        try:
+            ctx.calibrate_bands()
+            bd = ctx.select(0, 0, n).as_dict()
+            pb = n / bd["t_pred"] / 1e9
+            line["model"]["bands"] = {"predicted_GBps": pb, "E_pred": abs(pb - value / world) / (value / world),
+                                      "same_pick": bd["bytes"] == d["bytes"]}
+        except Exception as exc:  # context, not the product
+            line["model"]["bands"] = {"error": repr(exc)}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, desc, cores = cpu_oracle_run(n, d, prm)
         line["cpu_baseline"] = {"value": v, "unit": "GB/s", "cores": cores, "kind": "oracle", "sample": desc}

@@ -60,10 +60,19 @@ def main():
     ap.add_argument("--min", type=int, default=4096)
     ap.add_argument("--max", type=int, default=2 << 30)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "omb.jsonl"))
+    ap.add_argument("--no-bands", action="store_true", help="asymptotic Step-1 model only (no NEXT f4 bands)")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     ctx = mp.Context(device=0, calibrate=True, heap_bytes=16 << 20)
     ctx.set_options(mode=mp.MP_MODEL_B200)
+    # predictions of the single asymptotic Hockney fit (Step 1) before the size bands
+    sizes, n = [], a.min
+    while n <= a.max:
+        sizes.append(n)
+        n *= 2
+    pred_base = {n: n / ctx.select(0, 0, n).t_pred / 1e9 for n in sizes}
+    if not a.no_bands:
+        ctx.calibrate_bands()   # NEXT f4 (readings C20/C21)
     big = a.max
     A = torch.randint(0, 256, (big,), dtype=torch.uint8, device="cuda")
     B = torch.randint(0, 256, (big,), dtype=torch.uint8, device="cuda")
@@ -78,7 +87,7 @@ def main():
         iters = 200 if n <= (1 << 20) else (50 if n <= (64 << 20) else 5)
         skip = 10 if n <= (64 << 20) else 2
         row = {"n": n, "config": {"bytes": d["bytes"], "chunks": d["chunks"]},
-               "pred_GBps": n / d["t_pred"] / 1e9}
+               "pred_GBps": n / d["t_pred"] / 1e9, "pred_base_GBps": pred_base[n]}
         for w in (1, 16, 64):
             def mpw():
                 for _ in range(w):
@@ -106,6 +115,8 @@ def main():
             row["ce_lat_us"] = median_single(
                 lambda: rt.cudaMemcpyAsync(B.data_ptr(), A.data_ptr(), n, kind, s1.cuda_stream), 200, s1) * 1e6
         row["E_pred_w1"] = abs(row["pred_GBps"] - row["bw_w1_GBps"]) / row["bw_w1_GBps"]
+        row["E_pred_base_w1"] = abs(row["pred_base_GBps"] - row["bw_w1_GBps"]) / row["bw_w1_GBps"]
+        row["E_pred_w16"] = abs(row["pred_GBps"] - row["bw_w16_GBps"]) / row["bw_w16_GBps"]
         print(json.dumps(row), flush=True)
         out.write(json.dumps(row) + "\n")
         n *= 2

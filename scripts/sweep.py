@@ -82,6 +82,7 @@ def main():
     ap.add_argument("--sizes", default="16,64,256,1024")
     ap.add_argument("--reps", type=int, default=7)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.json"))
+    ap.add_argument("--no-bands", action="store_true", help="skip the size-band picks (NEXT f4)")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     ctx = mp.Context(device=0, calibrate=True, n_loop_relays=6, host_path=1, heap_bytes=16 * MiB)
@@ -118,6 +119,22 @@ def main():
                           **{f"{k}_GBps": v["GBps"] for k, v in picks.items()},
                           **{f"{k}_E_sel": v["E_sel"] for k, v in picks.items()},
                           **{f"{k}_E_pred": v["E_pred"] for k, v in picks.items()}}), flush=True)
+    if not a.no_bands:
+        # NEXT f4 (readings C20/C21): the B200-mode pick with per-band Step-1 parameters
+        ctx.calibrate_bands()
+        report["bands"] = ctx.get_model_bands(0, 0)
+        ctx.set_options(mode=mp.MP_MODEL_B200)
+        for n in sizes:
+            rs = report["sizes"][str(n)]
+            cfg = ctx.select(0, 0, n)
+            t = measure(ctx, dst, src, n, cfg, a.reps, stream)
+            d = cfg.as_dict()
+            bw, bwp = n / t / 1e9, n / d["t_pred"] / 1e9
+            best = rs["best"]["GBps"]
+            rs["picks"]["b200_bands"] = {"config": d, "t": t, "GBps": bw, "pred_GBps": bwp,
+                                         "E_sel": max(0.0, 1 - bw / best), "E_pred": abs(bwp - best) / best}
+            print(json.dumps({"n": n, "b200_bands_GBps": bw, "b200_bands_E_sel": rs["picks"]["b200_bands"]["E_sel"],
+                              "b200_bands_E_pred": rs["picks"]["b200_bands"]["E_pred"]}), flush=True)
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     with open(a.out, "w") as f:
         json.dump(report, f)
