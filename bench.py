@@ -552,6 +552,31 @@ def main():
             per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "pcie",
                               "peak": 64.0, "frac": gbs / 64.0,
                               "peak_source": "PCIe Gen5 x16 nominal per direction (north star)"}
+    # the practical ceiling of SM-driven PCIe traffic in loopback: both host legs share
+    # this GPU's link, so a full-grid SM copy device→pinned host and one pinned
+    # host→device, run at once, bound what the host path can reach
+    try:
+        hp = torch.empty(nstage, dtype=torch.uint8).pin_memory()
+        hq = torch.empty(nstage, dtype=torch.uint8).pin_memory()
+        s2 = torch.cuda.Stream()
+        dcfg = ctx.make_config([nstage] + [0] * (len(paths_) - 1), [1] + [0] * (len(paths_) - 1))
+
+        def duplex():
+            e = torch.cuda.Event()
+            e.record(stream)
+            s2.wait_event(e)
+            ctx.xfer(hp.data_ptr(), src, nstage, dcfg, stream)
+            ctx.xfer(dst, hq.data_ptr(), nstage, dcfg, s2)
+            e2 = torch.cuda.Event()
+            e2.record(s2)
+            stream.wait_event(e2)
+        ceil = nstage / med(duplex) / 1e9
+        h = per_path["host_pcie_alone"]
+        h["sm_duplex_ceiling_GBps"] = ceil
+        h["frac_of_sm_duplex_ceiling"] = h["GBps"] / ceil
+        del hp, hq
+    except Exception as exc:  # context, not the product
+        per_path["host_pcie_alone"]["sm_duplex_ceiling_error"] = repr(exc)
     ctx.set_options(mode=mp.MP_MODEL_PAPER)
     pcfg = ctx.select(0, 0, n)
     t = med(lambda: ctx.xfer(dst, src, n, pcfg, stream))

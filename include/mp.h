@@ -324,7 +324,7 @@ int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
  * j >= 1 is installed with mp_set_model_band(edges[j]).  ε and, when the pair already
  * has a model, the φ multipliers c are kept (run mp_calibrate first).
  * edges[nedges]: band lower edges in bytes, edges[0] == 0, strictly increasing; NULL
- * = {0, 256 KiB, 4 MiB, 32 MiB, 128 MiB}.  reps: windows per size (median).
+ * = {0, 256 KiB, 4 MiB, 16, 32, 64, 128 MiB}.  reps: windows per size (median).
  * Collective when world > 1 (same rules as mp_calibrate).
  * Errors: MP_ERR_STATE (model-only), MP_ERR_INVALID (bad edges), MP_ERR_CUDA. */
 int mp_calibrate_bands(mp_ctx *ctx, const uint64_t *edges, int nedges, int reps);

@@ -584,7 +584,7 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
       edges.push_back(static_cast<double>(edges_in[j]));
     }
   } else {
-    for (uint64_t e : {0ull, 256ull << 10, 4ull << 20, 32ull << 20, 128ull << 20}) edges.push_back(static_cast<double>(e));
+    for (uint64_t e : {0ull, 256ull << 10, 4ull << 20, 16ull << 20, 32ull << 20, 64ull << 20, 128ull << 20}) edges.push_back(static_cast<double>(e));
   }
   if (c->world != 1) {
     std::vector<uint64_t> sizes;

@@ -30,16 +30,20 @@ MiB = 1 << 20
 
 
 def measure(ctx, dst, src, n, cfg, reps, stream):
+    """OMB-style (reading C21): a window of W back-to-back transfers of
+    the config, seconds per message = window time / W, median over `reps` windows."""
+    W = 8 if n <= 64 * MiB else 2
     ts = []
     for r in range(reps + 1):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        ctx.xfer(dst, src, n, cfg, stream)
+        for _ in range(W):
+            ctx.xfer(dst, src, n, cfg, stream)
         e1.record(stream)
         e1.synchronize()
         if r:
-            ts.append(e0.elapsed_time(e1) * 1e-3)
+            ts.append(e0.elapsed_time(e1) * 1e-3 / W)
     ts.sort()
     return ts[len(ts) // 2]
 
@@ -80,7 +84,7 @@ def grid(n, npaths, host_idx):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--sizes", default="16,64,256,1024")
-    ap.add_argument("--reps", type=int, default=7)
+    ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.json"))
     ap.add_argument("--no-bands", action="store_true", help="skip the size-band picks (NEXT f4)")
     a = ap.parse_args()

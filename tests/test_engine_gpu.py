@@ -239,8 +239,9 @@ def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
     c = mp.Context(device=0, n_loop_relays=2, host_path=1, slot_bytes=32 * MiB, heap_bytes=16 * MiB)
     c.set_options(mode=mp.MP_MODEL_B200)
     c.calibrate(reps=3)
-    sizes = [64 << 10, 1 * MiB, 8 * MiB]
-    src = torch.randint(0, 256, (8 * MiB,), dtype=torch.uint8, device="cuda")
+    # sizes where a window of transfers is GPU-bound (not bound by the Python loop)
+    sizes = [16 * MiB, 32 * MiB, 48 * MiB]
+    src = torch.randint(0, 256, (48 * MiB,), dtype=torch.uint8, device="cuda")
     dst = torch.empty_like(src)
     s = torch.cuda.Stream()
 
@@ -261,7 +262,7 @@ def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
     for n in sizes:
         cfg = c.select(0, 0, n)
         err_base.append(abs(cfg.t_pred - window_time(n, cfg)) / window_time(n, cfg))
-    edges = [0, 256 << 10, 4 * MiB, 32 * MiB, 128 * MiB]
+    edges = [0, 256 << 10, 4 * MiB, 16 * MiB, 32 * MiB, 64 * MiB, 128 * MiB]
     c.calibrate_bands(edges, reps=3)
     bands = c.get_model_bands(0, 0)
     assert [b[0] for b in bands] == edges
@@ -272,7 +273,7 @@ def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
         cfg = c.select(0, 0, n)
         t = window_time(n, cfg)
         err_band.append(abs(cfg.t_pred - t) / t)
-    assert max(err_band) < 0.35 and sum(err_band) < sum(err_base), (err_base, err_band)
+    assert max(err_band) < 0.25 and sum(err_band) < sum(err_base), (err_base, err_band)
     ctx_sum = dict(base=err_base, bands=err_band)
     print("E_pred base vs banded", ctx_sum)
     c.close()
