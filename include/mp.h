@@ -336,10 +336,88 @@ int mp_load_params(mp_ctx *ctx, const char *path);
 /* Launch statistics: number of engine kernels launched by this context so far. */
 int mp_stats(mp_ctx *ctx, uint64_t *kernel_launches);
 
+/* ---------------------------------------------------------------- collectives (NEXT f3)
+ *
+ * PAPER.md §5.3: MPI_Alltoall and MPI_Allreduce as sequences of
+ * model-driven multi-path P2P messages, without the host path (host staging
+ * degrades bidirectional traffic).  Every P2P step of a collective is one
+ * mp_send/mp_recv pair whose config comes from mp_select_flows over the step's
+ * known pattern (all ranks send at once, reading C19).  Algorithms (reading C22):
+ *   Alltoall : MP_ALGO_BRUCK (UCC's; ⌈log2 W⌉ steps, packed blocks) or
+ *              MP_ALGO_PAIRWISE (W−1 steps, one block each).
+ *   Allreduce: MP_ALGO_KNOMIAL (radix-2 K-nomial = recursive halving reduce-scatter +
+ *              recursive doubling allgather; W a power of two) or
+ *              MP_ALGO_RING (any W).
+ *   MP_ALGO_AUTO: Bruck below 256 KiB per block, else pairwise; K-nomial when W is a
+ *              power of two, else ring.
+ * A schedule is data (mp_coll_plan): local copies before, P2P steps, local copies
+ * after.  Buffers named in a plan: MP_BUF_SEND (the caller's send buffer),
+ * MP_BUF_RECV (the caller's receive buffer), MP_BUF_TMP (library scratch, tmp_bytes).
+ * A step sends the concatenation of its send segments to send_to and splits the
+ * message it receives from recv_from over its recv segments, copying or — reduce = 1 —
+ * adding elementwise. */
+enum { MP_COLL_ALLTOALL = 0, MP_COLL_ALLREDUCE = 1 };
+enum { MP_ALGO_AUTO = 0, MP_ALGO_BRUCK = 1, MP_ALGO_PAIRWISE = 2, MP_ALGO_KNOMIAL = 3, MP_ALGO_RING = 4 };
+enum { MP_BUF_SEND = 0, MP_BUF_RECV = 1, MP_BUF_TMP = 2 };
+enum { MP_DT_U8 = 0, MP_DT_I32 = 1, MP_DT_I64 = 2, MP_DT_F32 = 3, MP_DT_F64 = 4, MP_DT_BF16 = 5 };
+enum { MP_OP_SUM = 0 };
+
+#define MP_COLL_MAX_STEPS 64
+#define MP_COLL_MAX_SEGS 512
+#define MP_COLL_MAX_COPIES 64
+
+typedef struct mp_coll_seg { int32_t buf; int32_t reserved; uint64_t off, len; } mp_coll_seg;
+typedef struct mp_coll_copy { int32_t src_buf, dst_buf; uint64_t src_off, dst_off, len; } mp_coll_copy;
+typedef struct mp_coll_step {
+  int32_t send_to, recv_from;    /* ranks (never -1 in the algorithms above) */
+  int32_t reduce, reserved;      /* 1: received data is added into the recv segments */
+  uint32_t send_seg0, send_nseg; /* slice of mp_coll_plan.seg */
+  uint32_t recv_seg0, recv_nseg;
+  uint64_t bytes;                /* message bytes = Σ send lengths (the peer's Σ recv lengths) */
+} mp_coll_step;
+typedef struct mp_coll_plan {
+  int32_t coll, algo, world, rank;
+  uint64_t tmp_bytes;
+  int32_t npre, nsteps, nsegs, npost;
+  mp_coll_copy pre[MP_COLL_MAX_COPIES];
+  mp_coll_step step[MP_COLL_MAX_STEPS];
+  mp_coll_seg seg[MP_COLL_MAX_SEGS];
+  mp_coll_copy post[MP_COLL_MAX_COPIES];
+} mp_coll_plan;
+
+/* Build rank `rank`'s plan of a collective over `world` ranks.  bytes: per destination
+ * block for Alltoall (send and recv buffers hold world·bytes), the whole vector for
+ * Allreduce (elem_size-byte elements; blocks split on element boundaries).  algo is
+ * resolved (AUTO → the concrete algorithm, stored in out->algo).  Pure host function.
+ * Errors: MP_ERR_INVALID (world < 1 or > 16, rank out of range, bytes not a multiple
+ * of elem_size, K-nomial with W not a power of two, plan larger than the caps). */
+int mp_coll_plan_build(int coll, int algo, int world, int rank, uint64_t bytes, uint32_t elem_size,
+                       mp_coll_plan *out);
+
+/* MPI_Alltoall over all ranks of ctx (collective; every rank calls it in the same
+ * order): block s of rank r's send buffer (bytes_per_rank bytes at sendbuf + s·B)
+ * lands at recvbuf + r·B on rank s.  Device buffers; recvbuf must come from mp_alloc
+ * or mp_register when world > 1; sendbuf may be any device buffer.  Stream-ordered on
+ * `stream` (the library forks internal send/receive streams from it and joins them
+ * back).  world == 1: one local copy.  No P2P message of the caller may be in flight
+ * between two ranks while a collective runs (matching is FIFO per pair).
+ * Errors: as mp_send / mp_recv, MP_ERR_NOMEM (heap scratch). */
+int mp_alltoall(mp_ctx *ctx, const void *sendbuf, void *recvbuf, uint64_t bytes_per_rank, int algo,
+                void *stream);
+
+/* MPI_Allreduce(op) of `count` elements of `dtype` (collective): recvbuf = Σ over ranks
+ * of sendbuf, on every rank.  sendbuf == recvbuf is allowed (in place).  Integer sums
+ * are exact (wrapping); floating-point sums are reassociated by the algorithm (bf16:
+ * each addition in fp32, rounded to bf16).  Buffer rules as mp_alltoall.
+ * Errors: MP_ERR_INVALID (dtype, op), as mp_alltoall. */
+int mp_allreduce(mp_ctx *ctx, const void *sendbuf, void *recvbuf, uint64_t count, int dtype, int op,
+                 int algo, void *stream);
+
 /* The Hockney fit of Step 1 (reading C12), exposed for parity tests: least squares of
  * T = α + n/β over m samples (n[i] bytes, t[i] seconds, host arrays), each residual
- * weighted by 1/t[i]² (relative error).  Clamps: α < 1e-7 s becomes 1e-7 (Eq 14 needs
- * α > 0); a non-positive slope falls back to β = n[m-1]/t[m-1].  m >= 2, else
+ * weighted by 1/t[i]² (relative error), subject to α >= 1e-7 s (Eq 14 needs α > 0:
+ * when the free optimum violates it, α = 1e-7 and the slope is refitted for that α);
+ * a non-positive slope falls back to β = n[m-1]/t[m-1].  m >= 2, else
  * MP_ERR_INVALID.  Pure host arithmetic, no context. */
 int mp_fit_hockney(const double *n, const double *t, int m, double *alpha, double *beta);
 

@@ -18,4 +18,8 @@ optimize   Exact optimisers (rational water-filling, continuous-k / integer-k le
            ``model``.
 pipeline   Discrete-event simulation of a two-stage staged path (pins Eq 13).
 transfer   The memcpy reference transfer replayed through a chosen split (O1).
+calibration  The Step-1 Hockney fit (reading C12).
+flows      Concurrent-flow (MaxRate-style) selection, NEXT f1 (reading C19).
+bands      Size bands of the Step-1 parameters, NEXT f4 (reading C20).
+collectives  MPI Alltoall / Allreduce definitions and a plain plan executor, NEXT f3.
 """

@@ -51,8 +51,13 @@ Fit fit_hockney(const std::vector<double> &n, const std::vector<double> &t) {
   const double det = s00 * s11 - s01 * s01;
   double a = (r0 * s11 - r1 * s01) / det;
   double g = (s00 * r1 - s01 * r0) / det;
+  if (!(a > 1e-7)) {
+    // constraint α >= 1e-7 (Eq 14 needs α > 0): the convex objective's constrained
+    // optimum is on the bound — refit the slope with α fixed there
+    a = 1e-7;
+    g = (r1 - a * s01) / s11;
+  }
   if (!(g > 0)) g = t.back() / n.back();
-  if (!(a > 1e-7)) a = 1e-7;  // Eq 14 needs α > 0
   return Fit{a, 1.0 / g};
 }
 

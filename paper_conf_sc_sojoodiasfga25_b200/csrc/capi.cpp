@@ -476,6 +476,7 @@ int mp_finalize(mp_ctx *c) {
   if (!c) return MP_OK;
   if (!c->model_only) {
     cudaSetDevice(c->device);
+    coll_release(c);
     if (c->world > 1) world_finalize(c);  // stops the persistent relay kernel first
     cudaDeviceSynchronize();
     free_engine(c);

@@ -157,5 +157,9 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
 int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream);
 int world_sync(mp_ctx *c);
 int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id);
+// true when [p, p + n) lies in a receive region (heap or mp_register) of this rank
+bool world_receivable(mp_ctx *c, const void *p, uint64_t n);
+// collectives (coll.cpp): release the per-context streams, events and heap scratch
+void coll_release(mp_ctx *c);
 int world_deregister(mp_ctx *c, int id);
 }  // namespace mpx

@@ -11,6 +11,7 @@
 // polls with ld.acquire.sys, then bar.sync.  Ring data is read with L1-bypassing
 // loads (.cg for device rings, .cv for host rings).  Every wait is bounded by
 // %globaltimer and raises DERR_TIMEOUT instead of hanging.
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #include "engine.h"
@@ -730,7 +731,71 @@ __global__ void __launch_bounds__(kThreads) direct_reg_kernel(const __grid_const
   group_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x);
 }
 
+// Elementwise dst += src (Allreduce, NEXT f3): grid-stride over 16-byte vectors when
+// both pointers are 16-B aligned, element tail and unaligned inputs element-wise.
+template <typename T>
+__device__ __forceinline__ T add_elem(T a, T b) { return a + b; }
+template <>
+__device__ __forceinline__ __nv_bfloat16 add_elem(__nv_bfloat16 a, __nv_bfloat16 b) {
+  return __float2bfloat16(__bfloat162float(a) + __bfloat162float(b));
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads) reduce_add_kernel(T *dst, const T *src, uint64_t n) {
+  constexpr int E = 16 / sizeof(T);
+  const uint64_t gt = static_cast<uint64_t>(blockIdx.x) * kThreads + threadIdx.x;
+  const uint64_t GT = static_cast<uint64_t>(gridDim.x) * kThreads;
+  uint64_t done = 0;
+  if (((reinterpret_cast<uintptr_t>(dst) | reinterpret_cast<uintptr_t>(src)) & 15u) == 0) {
+    const uint64_t nv = n / E;
+    for (uint64_t i = gt; i < nv; i += GT) {
+      uint4 a = reinterpret_cast<const uint4 *>(dst)[i];
+      const uint4 b = ld16<LD_RING>(reinterpret_cast<const uint4 *>(src) + i);
+      T *pa = reinterpret_cast<T *>(&a);
+      const T *pb = reinterpret_cast<const T *>(&b);
+#pragma unroll
+      for (int e = 0; e < E; ++e) pa[e] = add_elem(pa[e], pb[e]);
+      reinterpret_cast<uint4 *>(dst)[i] = a;
+    }
+    done = nv * E;
+  }
+  for (uint64_t i = done + gt; i < n; i += GT) dst[i] = add_elem(dst[i], src[i]);
+}
+
 }  // namespace
+
+int launch_reduce(int dtype, void *dst, const void *src, uint64_t bytes, void *stream) {
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  auto grid = [&](uint64_t vec) {
+    const uint64_t g = (vec + kThreads - 1) / kThreads;
+    return static_cast<uint32_t>(g < 1 ? 1 : (g > 1184 ? 1184 : g));
+  };
+  switch (dtype) {
+    case 1:  // MP_DT_I32
+      reduce_add_kernel<int32_t><<<grid(bytes / 16), kThreads, 0, s>>>(
+          static_cast<int32_t *>(dst), static_cast<const int32_t *>(src), bytes / 4);
+      break;
+    case 2:  // MP_DT_I64
+      reduce_add_kernel<long long><<<grid(bytes / 16), kThreads, 0, s>>>(
+          static_cast<long long *>(dst), static_cast<const long long *>(src), bytes / 8);
+      break;
+    case 3:  // MP_DT_F32
+      reduce_add_kernel<float><<<grid(bytes / 16), kThreads, 0, s>>>(static_cast<float *>(dst),
+                                                                      static_cast<const float *>(src), bytes / 4);
+      break;
+    case 4:  // MP_DT_F64
+      reduce_add_kernel<double><<<grid(bytes / 16), kThreads, 0, s>>>(static_cast<double *>(dst),
+                                                                       static_cast<const double *>(src), bytes / 8);
+      break;
+    case 5:  // MP_DT_BF16
+      reduce_add_kernel<__nv_bfloat16><<<grid(bytes / 16), kThreads, 0, s>>>(
+          static_cast<__nv_bfloat16 *>(dst), static_cast<const __nv_bfloat16 *>(src), bytes / 2);
+      break;
+    default:
+      return static_cast<int>(cudaErrorInvalidValue);
+  }
+  return static_cast<int>(cudaGetLastError());
+}
 
 int launch_xfer(const XferParams &P, void *stream) {
   if (P.nblocks == 0) return cudaSuccess;
@@ -792,6 +857,11 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_small_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<int32_t>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<long long>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<float>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<double>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<__nv_bfloat16>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_gate_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);

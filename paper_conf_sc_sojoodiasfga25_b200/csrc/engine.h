@@ -183,6 +183,10 @@ int launch_send(const SendParams &P, void *stream);
 int launch_recv(const RecvParams &P, void *stream);
 int launch_relay(const RelayParams &P, void *stream);
 
+// Collectives (coll.cpp): dst[i] += src[i] over `bytes` bytes of `dtype` elements
+// (MP_DT_* of include/mp.h; bf16 added in fp32 and rounded).  Returns a cudaError_t.
+int launch_reduce(int dtype, void *dst, const void *src, uint64_t bytes, void *stream);
+
 // Calibration probes (engine.cu).
 // Flag ping-pong between two CTAs through `flags` (2 words, device or mapped host):
 // `iters` round trips; the measured time is read with events by the caller.

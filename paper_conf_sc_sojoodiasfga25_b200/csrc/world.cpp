@@ -374,6 +374,13 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   return MP_OK;
 }
 
+bool world_receivable(mp_ctx *c, const void *p, uint64_t n) {
+  const uint8_t *b = static_cast<const uint8_t *>(p);
+  for (const mp_ctx::Region &g : c->regions)
+    if (g.used && g.base && b >= g.base && b + n <= g.base + g.bytes) return true;
+  return false;
+}
+
 int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
   uint8_t *b = static_cast<uint8_t *>(buf);
   int region = -1;

@@ -66,6 +66,37 @@ class mp_flow(C.Structure):
                 ("bytes", C.c_uint64)]
 
 
+MP_COLL_ALLTOALL, MP_COLL_ALLREDUCE = 0, 1
+MP_ALGO_AUTO, MP_ALGO_BRUCK, MP_ALGO_PAIRWISE, MP_ALGO_KNOMIAL, MP_ALGO_RING = 0, 1, 2, 3, 4
+MP_BUF_SEND, MP_BUF_RECV, MP_BUF_TMP = 0, 1, 2
+MP_DT_U8, MP_DT_I32, MP_DT_I64, MP_DT_F32, MP_DT_F64, MP_DT_BF16 = 0, 1, 2, 3, 4, 5
+MP_OP_SUM = 0
+MP_COLL_MAX_STEPS, MP_COLL_MAX_SEGS, MP_COLL_MAX_COPIES = 64, 512, 64
+
+
+class mp_coll_seg(C.Structure):
+    _fields_ = [("buf", C.c_int32), ("reserved", C.c_int32), ("off", C.c_uint64), ("len", C.c_uint64)]
+
+
+class mp_coll_copy(C.Structure):
+    _fields_ = [("src_buf", C.c_int32), ("dst_buf", C.c_int32), ("src_off", C.c_uint64), ("dst_off", C.c_uint64),
+                ("len", C.c_uint64)]
+
+
+class mp_coll_step(C.Structure):
+    _fields_ = [("send_to", C.c_int32), ("recv_from", C.c_int32), ("reduce", C.c_int32), ("reserved", C.c_int32),
+                ("send_seg0", C.c_uint32), ("send_nseg", C.c_uint32), ("recv_seg0", C.c_uint32),
+                ("recv_nseg", C.c_uint32), ("bytes", C.c_uint64)]
+
+
+class mp_coll_plan(C.Structure):
+    _fields_ = [("coll", C.c_int32), ("algo", C.c_int32), ("world", C.c_int32), ("rank", C.c_int32),
+                ("tmp_bytes", C.c_uint64), ("npre", C.c_int32), ("nsteps", C.c_int32), ("nsegs", C.c_int32),
+                ("npost", C.c_int32), ("pre", mp_coll_copy * MP_COLL_MAX_COPIES),
+                ("step", mp_coll_step * MP_COLL_MAX_STEPS), ("seg", mp_coll_seg * MP_COLL_MAX_SEGS),
+                ("post", mp_coll_copy * MP_COLL_MAX_COPIES)]
+
+
 ALLGATHER = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64)
 
 
@@ -124,6 +155,10 @@ def lib():
             "mp_get_model_band": (C.c_int, [P, C.c_int, C.c_int, C.c_int, C.POINTER(C.c_uint64),
                                             C.POINTER(mp_path_params), C.POINTER(C.c_int),
                                             C.POINTER(mp_port_params), C.POINTER(C.c_int)]),
+            "mp_coll_plan_build": (C.c_int, [C.c_int, C.c_int, C.c_int, C.c_int, C.c_uint64, C.c_uint32,
+                                             C.POINTER(mp_coll_plan)]),
+            "mp_alltoall": (C.c_int, [P, P, P, C.c_uint64, C.c_int, P]),
+            "mp_allreduce": (C.c_int, [P, P, P, C.c_uint64, C.c_int, C.c_int, C.c_int, P]),
             "mp_calibrate_bands": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
@@ -143,7 +178,8 @@ def exported_symbols() -> List[str]:
             "mp_select", "mp_alloc", "mp_free", "mp_send", "mp_recv", "mp_xfer", "mp_sync",
             "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
             "mp_peer_base", "mp_select_flows", "mp_register", "mp_deregister",
-            "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands"]
+            "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands",
+            "mp_coll_plan_build", "mp_alltoall", "mp_allreduce"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -165,6 +201,26 @@ def fit_bands(n: Sequence[float], t: Sequence[float], edges: Sequence[float]):
     if st != 0:
         raise MPError(st, "mp_fit_bands")
     return [(a[j], b[j]) for j in range(B)]
+
+
+def coll_plan(coll: int, algo: int, world: int, rank: int, nbytes: int, elem_size: int = 1) -> dict:
+    """mp_coll_plan_build as plain Python data (NEXT f3)."""
+    p = mp_coll_plan()
+    st = lib().mp_coll_plan_build(coll, algo, world, rank, nbytes, elem_size, C.byref(p))
+    if st != 0:
+        raise MPError(st, "mp_coll_plan_build")
+    cp = lambda k: dict(src_buf=k.src_buf, dst_buf=k.dst_buf, src_off=k.src_off, dst_off=k.dst_off,  # noqa: E731
+                        len=k.len)
+    sg = lambda g: dict(buf=g.buf, off=g.off, len=g.len)  # noqa: E731
+    steps = []
+    for j in range(p.nsteps):
+        t = p.step[j]
+        steps.append(dict(send_to=t.send_to, recv_from=t.recv_from, reduce=t.reduce, bytes=t.bytes,
+                          send_segs=[sg(p.seg[t.send_seg0 + k]) for k in range(t.send_nseg)],
+                          recv_segs=[sg(p.seg[t.recv_seg0 + k]) for k in range(t.recv_nseg)]))
+    return dict(coll=p.coll, algo=p.algo, world=p.world, rank=p.rank, tmp_bytes=p.tmp_bytes,
+                pre=[cp(p.pre[i]) for i in range(p.npre)], post=[cp(p.post[i]) for i in range(p.npost)],
+                nsteps=p.nsteps, steps=steps)
 
 
 def _params_array(params: Sequence[dict]):
@@ -355,6 +411,15 @@ class Context:
 
     def recv(self, buf, n, src, tag=0, stream=None):
         self._ck(lib().mp_recv(self.h, _ptr(buf), n, src, tag, _stream(stream)))
+
+    def alltoall(self, sendbuf, recvbuf, bytes_per_rank, algo=MP_ALGO_AUTO, stream=None):
+        """mp_alltoall (collective, NEXT f3)."""
+        self._ck(lib().mp_alltoall(self.h, _ptr(sendbuf), _ptr(recvbuf), bytes_per_rank, algo, _stream(stream)))
+
+    def allreduce(self, sendbuf, recvbuf, count, dtype=MP_DT_F32, algo=MP_ALGO_AUTO, stream=None):
+        """mp_allreduce(MP_OP_SUM) (collective, NEXT f3)."""
+        self._ck(lib().mp_allreduce(self.h, _ptr(sendbuf), _ptr(recvbuf), count, dtype, MP_OP_SUM, algo,
+                                    _stream(stream)))
 
     def sync(self):
         self._ck(lib().mp_sync(self.h))

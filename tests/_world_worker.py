@@ -277,14 +277,92 @@ def scenario_register(rank, world):
         assert not rest.any(), "bytes outside the registered views were written"
 
 
+def scenario_coll(rank, world):
+    """NEXT f3: mp_alltoall (Bruck, pairwise) and mp_allreduce (K-nomial when
+    W is a power of two, ring) through the multi-rank engine against the oracle's MPI
+    definitions: Alltoall and the int32 Allreduce exact; fp32 / bf16 sums within the
+    rounding bound of W − 1 reassociated additions; in place and out of place."""
+    import numpy as np
+
+    from oracle import collectives as OCL
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    BMAX = 300 * 1024 + 5
+    send = torch.zeros(world * BMAX + 64, dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                timeout_s=60.0)
+    rbuf = c.alloc(world * BMAX + 64)
+    rview = mp.as_tensor(rbuf, world * BMAX + 64)
+
+    def put(t, arr):
+        with torch.cuda.stream(stream):   # never torch.cuda.synchronize(): the relay kernel runs
+            t[:arr.nbytes].copy_(torch.from_numpy(arr.view(np.uint8)))
+        stream.synchronize()
+
+    def get(t, nbytes):
+        stream.synchronize()
+        return t[:nbytes].cpu().numpy()
+
+    for algo in (mp.MP_ALGO_BRUCK, mp.MP_ALGO_PAIRWISE):
+        for B in (1000, BMAX):
+            sends = [np.random.default_rng(97 * s + B + algo).integers(0, 256, world * B, dtype=np.uint8)
+                     for s in range(world)]
+            put(send, sends[rank])
+            c.alltoall(send, rview, B, algo, stream)
+            got = get(rview, world * B)
+            exp = OCL.alltoall(sends, B)[rank]
+            bad = np.nonzero(got != exp)[0]
+            assert bad.size == 0, f"alltoall algo {algo} B {B}: {bad.size} bytes differ, first {bad[:4]}"
+            dist.barrier()
+    algos = [mp.MP_ALGO_RING] + ([mp.MP_ALGO_KNOMIAL] if world & (world - 1) == 0 else [])
+    count = 100003
+    for algo in algos:
+        # int32, out of place (send buffer: any device memory; receive buffer: the heap)
+        sends = [np.random.default_rng(31 * s + algo).integers(-2 ** 31, 2 ** 31, count, dtype=np.int64)
+                 .astype(np.int32) for s in range(world)]
+        put(send, sends[rank])
+        c.allreduce(send, rview, count, mp.MP_DT_I32, algo, stream)
+        got = get(rview, 4 * count).view(np.int32)
+        assert np.array_equal(got, OCL.allreduce_sum(sends).astype(np.int32)), f"allreduce i32 algo {algo}"
+        dist.barrier()
+        # fp32 and bf16, in place in the heap buffer
+        for dt, npdt, eps in ((mp.MP_DT_F32, np.float32, 2.0 ** -24), (mp.MP_DT_BF16, None, 2.0 ** -8)):
+            rng = np.random.default_rng(53 * rank + algo + dt)
+            x = rng.standard_normal(count).astype(np.float32)
+            if npdt is None:   # bf16: the upper 16 bits of the fp32 pattern (round to nearest even)
+                u = x.view(np.uint32)
+                u = ((u + 0x7FFF + ((u >> 16) & 1)) >> 16).astype(np.uint16)
+                arr, vals = u, (u.astype(np.uint32) << 16).view(np.float32)
+            else:
+                arr, vals = x, x
+            allv = [None] * world
+            dist.all_gather_object(allv, vals)
+            put(rview, arr)
+            c.allreduce(rview, rview, count, dt, algo, stream)
+            raw = get(rview, arr.nbytes)
+            got = raw.view(np.float32) if npdt is not None else (raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32)
+            exact = OCL.allreduce_sum(allv)
+            bound = (world - 1) * eps * np.sum([np.abs(v.astype(np.float64)) for v in allv], axis=0) * 1.01 + 1e-30
+            err = np.abs(got.astype(np.float64) - exact)
+            assert (err <= bound).all(), f"allreduce dtype {dt} algo {algo}: max err / bound {np.max(err / bound)}"
+            dist.barrier()
+    c.sync()
+    c.free(rbuf)
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
+    faulthandler.enable()
     faulthandler.dump_traceback_later(int(os.environ.get("MPX_TEST_STACKS_S", "280")), exit=False)
     try:
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
-         "faults": scenario_faults, "register": scenario_register}[scen](rank, world)
+         "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

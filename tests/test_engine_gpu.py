@@ -333,3 +333,18 @@ def test_full_size_config3_bit_exact(ctx):
         assert torch.equal(dst[idx].cpu(), src[idx].cpu())
     finally:
         big.close()
+
+
+def test_loopback_collectives_are_local_copies(ctx):
+    # world == 1 (NEXT f3): Alltoall and Allreduce reduce to one local copy
+    n = 3 * MiB + 5
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda")
+    dst = torch.zeros_like(src)
+    ctx.alltoall(src, dst, n)
+    ctx.sync()
+    assert torch.equal(src, dst)
+    x = torch.randn(1000, device="cuda")
+    y = torch.zeros_like(x)
+    ctx.allreduce(x, y, 1000, mp.MP_DT_F32)
+    ctx.sync()
+    assert torch.equal(x, y)

@@ -47,12 +47,45 @@ def test_matches_exact_rational_normal_equations(pts):
         assert abs(1 / b - float(g_ex)) <= 1e-9 * float(g_ex)
 
 
+def objective(n, t, a, g):
+    return sum(((ti - a - ni * g) / ti) ** 2 for ni, ti in zip(n, t))
+
+
 def test_clamps():
-    # negative intercept → 1e-7; decreasing times → slope from the last sample
+    # negative intercept → α = 1e-7 with the slope refitted; decreasing times → slope
+    # from the last sample
     a, b = OC.fit_hockney([1e6, 2e6, 4e6], [1e-6, 3e-6, 7e-6])
     assert a == 1e-7
     a, b = OC.fit_hockney([1e6, 2e6], [2e-5, 1e-5])
     assert b == 2e6 / 1e-5
+
+
+@settings(max_examples=100, deadline=None)
+@given(st.lists(st.tuples(st.integers(1, 4000), st.integers(1, 500)), min_size=2, max_size=8,
+                unique_by=lambda x: x[0]))
+def test_clamped_fit_is_the_constrained_optimum(pts):
+    # the L2 -> HBM cliff of a size band makes times grow faster than linearly, and
+    # the free fit's intercept goes negative; the clamped fit must then be the optimum
+    # of the objective on the constraint α = 1e-7: the exact rational 1-D normal
+    # equation, and no nearby slope does better (convexity)
+    n = [float(p[0] * 65536) for p in pts]
+    t = [float(p[1]) * 1e-6 * (1 + p[0] / 400) for p in pts]   # super-linear in n
+    a_ex, g_ex = exact_weighted_normal_equations(n, t) if len(n) > 2 or n[0] != n[1] else (None, None)
+    a, b = OC.fit_hockney(n, t)
+    if a_ex is None or a_ex > F(1, 10 ** 7):
+        return
+    assert a == 1e-7
+    nF = [F(x) for x in n]
+    tF = [F(x) for x in t]
+    a0 = F(1, 10 ** 7)
+    g1 = sum((ti - a0) * ni / ti ** 2 for ni, ti in zip(nF, tF)) / sum(ni * ni / ti ** 2 for ni, ti in zip(nF, tF))
+    if g1 <= 0:
+        return
+    assert abs(1 / b - float(g1)) <= 1e-9 * float(g1)
+    g = 1 / b
+    f0 = objective(n, t, a, g)
+    for d in (1e-4, -1e-4, 1e-2, -1e-2):
+        assert objective(n, t, a, g * (1 + d)) >= f0 * (1 - 1e-12)
 
 
 @settings(max_examples=200, deadline=None)

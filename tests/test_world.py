@@ -79,3 +79,14 @@ def test_multirank_registered_buffers(world):
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(world, "register", timeout=400)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_multirank_collectives(world):
+    # NEXT f3: mp_alltoall / mp_allreduce through the multi-rank engine, all ranks on one GPU
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(world, "coll", timeout=600)
