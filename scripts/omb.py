@@ -76,6 +76,11 @@ def main():
     big = a.max
     A = torch.randint(0, 256, (big,), dtype=torch.uint8, device="cuda")
     B = torch.randint(0, 256, (big,), dtype=torch.uint8, device="cuda")
+    # osu_bibw: each side sends from its s_buf into the peer's r_buf — the reverse
+    # direction uses its own pair of buffers (a swapped A↔B pair would make each copy
+    # read the lines the other is writing; profiles/r01/bibw.jsonl)
+    Cb = torch.randint(0, 256, (big,), dtype=torch.uint8, device="cuda")
+    D = torch.empty(big, dtype=torch.uint8, device="cuda")
     s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
     kind = rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
@@ -105,7 +110,7 @@ def main():
             ev.record(s1)
             s2.wait_event(ev)
             ctx.xfer(B, A, n, None, s1)
-            ctx.xfer(A, B, n, None, s2)
+            ctx.xfer(D, Cb, n, None, s2)
             ev2 = torch.cuda.Event()
             ev2.record(s2)
             s1.wait_event(ev2)

@@ -72,6 +72,15 @@ def scenario_engine(rank, world):
         c.calibrate(sizes=[4 * MiB, 8 * MiB, 16 * MiB], reps=2)
         _, prm, _ = c.get_model(0, 1)
         assert prm[0]["beta"] > 0 and prm[1]["eps"] > 0
+    # NEXT f4: collective per-band Step 1 (readings C20/C21) on every pair
+    c.calibrate_bands([0, 1 * MiB, 8 * MiB], reps=2)
+    for dst in range(world):
+        if dst == rank:
+            continue
+        bands = c.get_model_bands(rank, dst)
+        assert [b[0] for b in bands] == [0, 1 * MiB, 8 * MiB], bands
+        for _, prm, port in bands:
+            assert all(p["beta"] > 0 and p["alpha"] > 0 for p in prm) and port["beta"] > 0
     ps = c.paths(0, 1)
     np_ = len(ps)
     cases = []
