@@ -173,6 +173,9 @@ void free_engine(mp_ctx *c) {
   c->h_probe = nullptr;
   for (auto &p : c->pending) cudaEventDestroy(p.ready);
   c->pending.clear();
+  if (c->big_ev) cudaEventDestroy(c->big_ev);
+  c->big_ev = nullptr;
+  c->big_valid = false;
 }
 
 int alloc_ring(mp_ctx *c, bool host, Ring *r) {
@@ -258,7 +261,18 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
     if (cfg.bytes[i]) staged_ctas += 2u * static_cast<uint32_t>(c->relay_ctas);
   // direct group sized by direct_ctas(), leaving room for every staged group to be
   // co-resident.
-  const uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas));
+  uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas));
+  // Two large copies running at once (osu_bibw's two directions on two streams) do
+  // best with one TMA pipeline per SM each — 64 KiB in flight per SM in total, as one
+  // copy with two (profiles/r01/bibw.jsonl).  A large direct-only launch that finds
+  // the previous one, from another stream, still running takes one CTA per SM.
+  cudaStreamCaptureStatus capst = cudaStreamCaptureStatusNone;
+  const bool big = staged_ctas == 0 && cfg.bytes[0] >= (16ull << 20) &&
+                   cudaStreamIsCapturing(static_cast<cudaStream_t>(stream), &capst) == cudaSuccess &&
+                   capst == cudaStreamCaptureStatusNone;  // (not inside a CUDA-graph capture)
+  if (big && c->big_valid && c->big_stream != static_cast<cudaStream_t>(stream) &&
+      cudaEventQuery(c->big_ev) == cudaErrorNotReady)
+    g_direct = std::min<uint32_t>(g_direct, static_cast<uint32_t>(c->sms));
   uint32_t next = 0;
   uint64_t off = 0;
   P.npaths = static_cast<uint32_t>(cfg.npaths);
@@ -301,6 +315,12 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   const int e = launch_xfer(P, stream);
   if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "xfer launch");
   c->launches += 1;
+  if (big) {
+    if (!c->big_ev) CK(cudaEventCreateWithFlags(&c->big_ev, cudaEventDisableTiming));
+    CK(cudaEventRecord(c->big_ev, static_cast<cudaStream_t>(stream)));
+    c->big_stream = static_cast<cudaStream_t>(stream);
+    c->big_valid = true;
+  }
   return MP_OK;
 }
 

@@ -92,6 +92,10 @@ struct mp_ctx {
   mpx::Heap heap;
   std::deque<mpx::PendingSend> pending;
   uint64_t launches = 0;
+  // the last large loopback transfer (concurrency-aware direct grid)
+  cudaEvent_t big_ev = nullptr;
+  cudaStream_t big_stream = nullptr;
+  bool big_valid = false;
   uint64_t *d_probe = nullptr;    // calibration flag words (device)
   uint64_t *h_probe = nullptr;    // calibration flag words (mapped host)
 
