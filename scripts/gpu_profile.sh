@@ -8,12 +8,18 @@ mkdir -p $OUT
 nvidia-smi -q -d CLOCK > $OUT/clocks_before.txt 2>&1
 (nproc; grep -m1 "model name" /proc/cpuinfo) > $OUT/host.txt 2>&1
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $OUT/smoke.log 2>&1; echo "smoke rc=$?" >> $OUT/smoke.log
+# tools (not the product): C OMB harness and the copy design sweeps
+[ -x scripts/omb_c ] || g++ -O2 -std=c++17 -I include -I /usr/local/cuda/include scripts/omb_c.cpp \
+  -L paper_conf_sc_sojoodiasfga25_b200/_lib -lmpx -L /usr/local/cuda/lib64 -lcudart \
+  -Wl,-rpath,'$ORIGIN/../paper_conf_sc_sojoodiasfga25_b200/_lib' -o scripts/omb_c
+[ -x scripts/smallbench ] || nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o scripts/smallbench scripts/smallbench.cu
 timeout 900 python -m pytest tests -m gpu -q -p no:cacheprovider > $OUT/pytest_gpu.log 2>&1; echo "rc=$?" >> $OUT/pytest_gpu.log
 timeout 600 python bench.py --save-params $OUT/params.txt > $OUT/bench.log 2>&1; echo "rc=$?" >> $OUT/bench.log
 MPX_COPY=reg timeout 300 python bench.py --no-cpu-baseline --steps 200 --params $OUT/params.txt > $OUT/bench_reg.log 2>&1
 timeout 300 python bench.py --impl reference --steps 20 --warmup 3 > $OUT/bench_reference.log 2>&1
 timeout 900 python scripts/sweep.py --out $OUT/sweep.json > $OUT/sweep.log 2>&1; echo "rc=$?" >> $OUT/sweep.log
 timeout 900 python scripts/omb.py --out $OUT/omb.jsonl > $OUT/omb.log 2>&1
+timeout 900 ./scripts/omb_c > $OUT/omb_c.jsonl 2> $OUT/omb_c.err
 [ -x scripts/smallbench ] && timeout 300 ./scripts/smallbench > $OUT/smallbench.jsonl 2>&1
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
   python bench.py --steps 5 --warmup 3 --no-cpu-baseline --params $OUT/params.txt > $OUT/ncu_launch_bench.log 2>&1
