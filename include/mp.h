@@ -277,6 +277,12 @@ int mp_deregister(mp_ctx *ctx, int id);
 
 /* ---------------------------------------------------------------- transfer */
 
+/* Eager protocol (reading C23; NEXT f4's low-latency protocol): when
+ * world > 1, a message of 1..65536 bytes skips the rendezvous — one kernel per side,
+ * the payload goes over the direct path into a slot the receiver owns (8 slots per
+ * sender), and `cfg`'s split is not used.  Both sides classify by size alone; the
+ * environment variable MPX_EAGER=0 (equal on every rank, read at mp_init) turns it
+ * off. */
 /* Send `bytes` bytes at device pointer `buf` to rank dst with `tag`.  cfg = NULL
  * selects with mp_select(all paths); otherwise cfg->bytes/chunks/path are used as
  * given (validated: Σ bytes == n, 1 <= k <= max(1, ⌊b/A⌋), chunk <= slot_bytes,

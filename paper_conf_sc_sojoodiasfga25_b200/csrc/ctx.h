@@ -111,6 +111,8 @@ struct mp_ctx {
   size_t hseg_bytes = 0;
   std::vector<uint8_t *> hseg;              // [world]: mapped host segment of each receiver
   std::vector<uint64_t> send_seq, recv_seq, relay_q, host_q, done_target;
+  std::vector<uint64_t> eager_send_seq, eager_recv_seq;  // eager protocol (reading C23)
+  uint64_t eager_max = 0;                   // messages of 1..eager_max bytes go eager
   cudaStream_t relay_stream = nullptr;
   int32_t *stop = nullptr;                  // mapped host word read by the relay kernel
   bool relay_running = false;

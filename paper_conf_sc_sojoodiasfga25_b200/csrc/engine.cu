@@ -691,6 +691,57 @@ __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constan
 }
 
 
+// Eager protocol (engine.h, reading C23).  Slot = [kEagerHdr header][shift][data]:
+// header words 0/1 = bytes/tag (CTA 0), 16 + r = source shift of CTA r's slice, 8 + r =
+// CTA r's sequence flag (seq + 1, released after its slice).
+__global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_constant__ EagerParams P) {
+  __shared__ int s_abort;
+  if (threadIdx.x == 0) s_abort = 0;
+  __syncthreads();
+  const uint32_t r = blockIdx.x;
+  // the slot is free once the receiver has returned message seq − kEagerSlots
+  if (P.seq >= kEagerSlots && !wait_word(P.free_ctr, P.seq + 1 - kEagerSlots, P.timeout_ns, P.err, &s_abort))
+    return;
+  uint64_t *hdr = reinterpret_cast<uint64_t *>(P.slot);
+  const uint64_t shift = reinterpret_cast<uintptr_t>(P.src) & 15u;
+  uint8_t *data = P.slot + kEagerHdr + shift;
+  const uint64_t a = static_cast<uint64_t>(r) * kEagerSlice;
+  const uint64_t e = a + kEagerSlice < P.bytes ? a + kEagerSlice : P.bytes;
+  if (a < e) group_copy<LD_SRC>(data + a, P.src + a, e - a, 0, 1);
+  if (threadIdx.x == 0) {
+    if (r == 0) {
+      hdr[0] = P.bytes;
+      hdr[1] = P.tag;
+    }
+    hdr[16 + r] = shift;
+  }
+  __syncthreads();  // the CTA's stores precede thread 0's release (cumulative)
+  if (threadIdx.x == 0) st_release_sys(hdr + 8 + r, P.seq + 1);
+}
+
+__global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_constant__ EagerParams P) {
+  __shared__ int s_abort;
+  if (threadIdx.x == 0) s_abort = 0;
+  __syncthreads();
+  const uint32_t r = blockIdx.x;
+  const uint64_t *hdr = reinterpret_cast<const uint64_t *>(P.slot);
+  if (!wait_word(hdr + 8 + r, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
+  if (r == 0 && threadIdx.x == 0 && (ld_volatile(hdr) != P.bytes || ld_volatile(hdr + 1) != P.tag))
+    atomicExch(P.err, DERR_MISMATCH);
+  const uint8_t *data = P.slot + kEagerHdr + ld_volatile(hdr + 16 + r);
+  const uint64_t a = static_cast<uint64_t>(r) * kEagerSlice;
+  const uint64_t e = a + kEagerSlice < P.bytes ? a + kEagerSlice : P.bytes;
+  if (a < e) group_copy<LD_RING>(P.dst + a, data + a, e - a, 0, 1);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    // the last CTA out returns the slot to the sender
+    if (atomicAdd(P.cnt, 1u) == P.ctas - 1) {
+      atomicExch(P.cnt, 0u);
+      red_add_release_sys(P.free_ctr, 1);
+    }
+  }
+}
+
 // Direct-only messages (the B200-mode pick whenever the shared port is saturated by
 // the direct path, and every calibration copy) get this small kernel instead of the
 // fused one: ~30x less code, so a cold SM starts copying after far fewer instruction
@@ -828,6 +879,16 @@ int launch_send(const SendParams &P, void *stream) {
   return static_cast<int>(cudaGetLastError());
 }
 
+int launch_eager_send(const EagerParams &P, void *stream) {
+  eager_send_kernel<<<P.ctas, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
+  return static_cast<int>(cudaGetLastError());
+}
+
+int launch_eager_recv(const EagerParams &P, void *stream) {
+  eager_recv_kernel<<<P.ctas, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
+  return static_cast<int>(cudaGetLastError());
+}
+
 int launch_recv(const RecvParams &P, void *stream) {
   recv_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
@@ -857,6 +918,8 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_small_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, eager_send_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, eager_recv_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<int32_t>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<long long>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<float>);

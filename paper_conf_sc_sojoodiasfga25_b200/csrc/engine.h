@@ -91,6 +91,17 @@ int launch_xfer(const XferParams &P, void *stream);
 // = the heaps, 1.. = mp_register), so a sender or relay resolves it locally.
 
 constexpr uint32_t kCtsRing = 64;     // outstanding messages per ordered pair
+
+// Eager protocol (NEXT f4's low-latency protocol, reading C23): a message of
+// 1..kEagerMax bytes skips the rendezvous — the sender writes it, with per-CTA
+// sequence flags, into one of kEagerSlots slots the receiver owns per sender, the
+// receiver copies it out and returns the slot with a counter.  One kernel per side,
+// no clear-to-send round trip.
+constexpr uint32_t kEagerSlots = 8;
+constexpr uint64_t kEagerMax = 64ull << 10;
+constexpr uint32_t kEagerSlice = 8192;            // bytes per CTA (kEagerMax / 8 CTAs)
+constexpr uint32_t kEagerHdr = 256;               // {bytes, tag, flags[8]} before the data
+constexpr uint64_t kEagerStride = kEagerHdr + kEagerMax + 256;  // + co-alignment shift
 constexpr uint32_t kSlotHdr = 256;    // slot header bytes
 constexpr uint32_t kMaxRegions = 64;  // receive regions: 0 = heap, 1.. = mp_register
 
@@ -121,6 +132,9 @@ struct CtrlLayout {
   uint64_t probe = 0;                  // 64 B of flag words for the ε ping-pong of the predecessor
   uint64_t relay_pos = 0;              // [world(sender)] u64: relay ring position across restarts
   uint64_t regions = 0;                // [kMaxRegions][world] u64: mapped region bases (local)
+  uint64_t eager = 0;                  // [world(sender)][kEagerSlots][kEagerStride]   — on the receiver
+  uint64_t eager_free = 0;             // [world(receiver)] u64, 128-B padded: slots returned — on the sender
+  uint64_t eager_cnt = 0;              // [world(sender)][kEagerSlots] u32: CTAs done copying out — on the receiver
   uint64_t total = 0;
 };
 
@@ -179,7 +193,22 @@ struct RelayParams {
   int32_t *err;
 };
 
+struct EagerParams {
+  uint32_t peer;             // receiver (send) / sender (recv)
+  uint32_t ctas;             // ⌈bytes / kEagerSlice⌉ (>= 1)
+  uint64_t seq;              // eager sequence number of this message on the pair
+  uint64_t bytes, tag, timeout_ns;
+  const uint8_t *src;        // send: the user buffer
+  uint8_t *dst;              // recv: the user buffer
+  uint8_t *slot;             // the slot (receiver's control block; mapped on the sender)
+  uint64_t *free_ctr;        // eager_free word of the pair (sender's control block)
+  uint32_t *cnt;             // recv: eager_cnt word of the slot (receiver-local)
+  int32_t *err;
+};
+
 int launch_send(const SendParams &P, void *stream);
+int launch_eager_send(const EagerParams &P, void *stream);
+int launch_eager_recv(const EagerParams &P, void *stream);
 int launch_recv(const RecvParams &P, void *stream);
 int launch_relay(const RelayParams &P, void *stream);
 

@@ -46,6 +46,7 @@ struct RankInfo {
   uint64_t slot_bytes;
   int32_t slots;
   int32_t host_path;
+  uint64_t eager_max;
 };
 
 int allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes) {
@@ -82,6 +83,9 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.probe = take(64);
   L.relay_pos = take(static_cast<uint64_t>(world) * 8);
   L.regions = take(static_cast<uint64_t>(kMaxRegions) * world * 8);
+  L.eager = take(static_cast<uint64_t>(world) * kEagerSlots * kEagerStride);
+  L.eager_free = take(static_cast<uint64_t>(world) * 128);
+  L.eager_cnt = take(static_cast<uint64_t>(world) * kEagerSlots * 4);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
@@ -169,13 +173,16 @@ int world_init(mp_ctx *c) {
   me.slot_bytes = c->slot_bytes;
   me.slots = c->slots;
   me.host_path = c->host_path ? 1 : 0;
+  const char *eg = std::getenv("MPX_EAGER");  // "0": every message takes the rendezvous
+  c->eager_max = (eg && eg[0] == '0') ? 0 : kEagerMax;
+  me.eager_max = c->eager_max;
   std::vector<RankInfo> all(W);
   if (int s = allgather(c, &me, all.data(), sizeof(RankInfo))) return s;
   c->jobid = all[0].jobid;
   for (int r = 0; r < W; ++r)
     if (all[r].relay_ctas != c->relay_ctas || all[r].slot_bytes != c->slot_bytes ||
-        all[r].slots != c->slots || all[r].host_path != me.host_path)
-      return wfail(c, MP_ERR_INVALID, "ranks disagree on slots / slot_bytes / relay_ctas / host_path");
+        all[r].slots != c->slots || all[r].host_path != me.host_path || all[r].eager_max != me.eager_max)
+      return wfail(c, MP_ERR_INVALID, "ranks disagree on slots / slot_bytes / relay_ctas / host_path / MPX_EAGER");
 
   DBG("rank info exchanged");
   c->peers.assign(W, PeerPtrs{nullptr, nullptr});
@@ -226,6 +233,8 @@ int world_init(mp_ctx *c) {
   c->relay_q.assign(W, 0);
   c->host_q.assign(W, 0);
   c->done_target.assign(W, 0);
+  c->eager_send_seq.assign(W, 0);
+  c->eager_recv_seq.assign(W, 0);
 
   if (W >= 3) {  // resources of the persistent relay kernel; it is started by world_start_relay
     CKW(cudaHostAlloc(&p, 64, cudaHostAllocMapped | cudaHostAllocPortable));
@@ -306,8 +315,51 @@ static void note_stream(mp_ctx *c, cudaStream_t s) {
   if (std::find(c->streams.begin(), c->streams.end(), s) == c->streams.end()) c->streams.push_back(s);
 }
 
+// Eager protocol (reading C23): 1..eager_max bytes, direct path, no rendezvous.
+static EagerParams eager_params(mp_ctx *c, int sender, int receiver, uint64_t seq, uint64_t bytes, int tag) {
+  EagerParams P{};
+  P.seq = seq;
+  P.bytes = bytes;
+  P.tag = static_cast<uint64_t>(static_cast<int64_t>(tag));
+  P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  P.ctas = static_cast<uint32_t>((bytes + kEagerSlice - 1) / kEagerSlice);
+  const uint64_t slot = seq % kEagerSlots;
+  P.slot = c->peers[receiver].ctrl + c->L.eager + (static_cast<uint64_t>(sender) * kEagerSlots + slot) * kEagerStride;
+  P.free_ctr = reinterpret_cast<uint64_t *>(c->peers[sender].ctrl + c->L.eager_free +
+                                            static_cast<uint64_t>(receiver) * 128);
+  P.cnt = reinterpret_cast<uint32_t *>(c->peers[receiver].ctrl + c->L.eager_cnt) +
+          static_cast<uint64_t>(sender) * kEagerSlots + slot;
+  P.err = c->d_err;
+  return P;
+}
+
+static int eager_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, void *stream) {
+  EagerParams P = eager_params(c, c->rank, dst, c->eager_send_seq[dst], bytes, tag);
+  P.peer = static_cast<uint32_t>(dst);
+  P.src = static_cast<const uint8_t *>(buf);
+  if (int e = launch_eager_send(P, stream))
+    return wfail(c, MP_ERR_CUDA, std::string("eager send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  c->launches += 1;
+  c->eager_send_seq[dst] += 1;
+  note_stream(c, static_cast<cudaStream_t>(stream));
+  return MP_OK;
+}
+
+static int eager_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
+  EagerParams P = eager_params(c, src, c->rank, c->eager_recv_seq[src], bytes, tag);
+  P.peer = static_cast<uint32_t>(src);
+  P.dst = static_cast<uint8_t *>(buf);
+  if (int e = launch_eager_recv(P, stream))
+    return wfail(c, MP_ERR_CUDA, std::string("eager recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  c->launches += 1;
+  c->eager_recv_seq[src] += 1;
+  note_stream(c, static_cast<cudaStream_t>(stream));
+  return MP_OK;
+}
+
 int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,
                void *stream) {
+  if (bytes > 0 && bytes <= c->eager_max) return eager_send(c, buf, bytes, dst, tag, stream);
   SendParams P{};
   P.me = static_cast<uint32_t>(c->rank);
   P.dst = static_cast<uint32_t>(dst);
@@ -394,6 +446,7 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   if (!bytes) region = 0;
   if (region < 0)
     return wfail(c, MP_ERR_INVALID, "mp_recv buffer must come from mp_alloc or mp_register when world > 1");
+  if (bytes > 0 && bytes <= c->eager_max) return eager_recv(c, buf, bytes, src, tag, stream);
   RecvParams P{};
   P.me = static_cast<uint32_t>(c->rank);
   P.src = static_cast<uint32_t>(src);

@@ -95,6 +95,12 @@ int main(int argc, char **argv) {
     for (int i = 0; i < cfg.npaths; ++i)
       std::printf("%s%llu", i ? ", " : "", static_cast<unsigned long long>(cfg.bytes[i]));
     std::printf("], \"pred_GBps\": %.4f", n / cfg.t_pred / 1e9);
+    {  // bibw as two concurrent flows of the same pair (NEXT f1/f2, reading C19)
+      mp_flow fl[2] = {{0, 0, 0, 0, n}, {0, 0, 0, 0, n}};
+      mp_config fc[2];
+      MK(mp_select_flows(ctx, 2, fl, fc));
+      std::printf(", \"pred_bibw_GBps\": %.4f", 2.0 * n / std::max(fc[0].t_pred, fc[1].t_pred) / 1e9);
+    }
     for (int w : {1, 16, 64}) {
       const int it = std::max(2, iters / w);
       std::printf(", \"bw_w%d_GBps\": %.4f, \"ce_bw_w%d_GBps\": %.4f", w, n / timed(mpx, w, it) / 1e9, w,

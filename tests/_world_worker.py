@@ -179,21 +179,23 @@ def scenario_faults(rank, world):
     src = torch.empty(MiB, dtype=torch.uint8, device="cuda")
     src.copy_(torch.from_numpy(synth.payload(MiB, 0)))
     torch.cuda.synchronize()
-    for fault in ("mismatch", "timeout"):
+    for fault in ("mismatch", "timeout", "eager_mismatch"):
         c = mdist.context_from_dist(device=0, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                     timeout_s=3.0)
-        if rank == 0 and fault == "mismatch":
-            c.send(src, MiB, 1, tag=5, stream=stream)
+        nb = 4096 if fault == "eager_mismatch" else MiB
+        if rank == 0 and fault != "timeout":
+            c.send(src[:nb], nb, 1, tag=5, stream=stream)
         elif rank == 1:
-            p = c.alloc(MiB)
-            c.recv(p, MiB, 0, tag=6 if fault == "mismatch" else 7, stream=stream)
+            p = c.alloc(nb)
+            c.recv(p, nb, 0, tag=7 if fault == "timeout" else 6, stream=stream)
         stream.synchronize()
         status = 0
         try:
             c.sync()
         except mp.MPError as e:
             status = e.status
-        expect = {"mismatch": -8, "timeout": -7 if rank == 1 else 0}[fault]
+        expect = {"mismatch": -8, "timeout": -7 if rank == 1 else 0,
+                  "eager_mismatch": -8 if rank == 1 else 0}[fault]
         assert status == expect, (fault, rank, status)
         print(f"rank {rank}: {fault} -> {status}", flush=True)
         dist.barrier()
@@ -286,6 +288,57 @@ def scenario_register(rank, world):
         assert not rest.any(), "bytes outside the registered views were written"
 
 
+def scenario_eager(rank, world):
+    """The eager protocol (reading C23): messages of 1..64 KiB, misaligned sources and
+    destinations, 8-KiB slice edges, the 64 KiB / 64 KiB + 1 boundary to the rendezvous,
+    a window of 20 messages (more than the 8 slots: flow control), and eager and
+    rendezvous messages interleaved on one pair — every byte checked."""
+    import numpy as np
+
+    import synth
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    src_buf = torch.empty(2 * MiB, dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    c = mdist.context_from_dist(device=0, heap_bytes=32 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                timeout_s=60.0)
+    sizes = [1, 17, 4095, 8192, 8193, 3 * 8192 + 5, 65535, 65536, 65537, 300000]
+    offs = [(0, 0), (1, 1), (3, 7), (16, 5)]
+    cases = [(n, so, do) for n in sizes for so, do in offs[: 1 if n > 65536 else 4]]
+    cases += [(777, 0, 0)] * 20                     # a window beyond the 8 slots
+    cases += [(65536 + 4096, 0, 0), (100, 2, 2), (1 << 20, 0, 0), (5, 0, 0)]   # interleaved protocols
+    if rank == 0:
+        for i, (n, so, _) in enumerate(cases):
+            host = synth.payload(n, 500 + i)
+            with torch.cuda.stream(stream):
+                src_buf[so:so + n].copy_(torch.from_numpy(host))
+            c.send(src_buf[so:so + n], n, 1, tag=1000 + i, stream=stream)
+        stream.synchronize()
+    elif rank == 1:
+        bufs = []
+        for i, (n, _, do) in enumerate(cases):
+            p = c.alloc(n + 64)
+            c.recv(p + do, n, 0, tag=1000 + i, stream=stream)
+            bufs.append(p)
+        stream.synchronize()
+        c.sync()
+        for i, ((n, _, do), p) in enumerate(zip(cases, bufs)):
+            got = mp_tensor(p + do, n).cpu().numpy()
+            exp = synth.payload(n, 500 + i)
+            bad = np.nonzero(got != exp)[0]
+            assert bad.size == 0, f"eager case {i} (n={n}, dst+{do}): {bad.size} bytes differ, first {bad[:4]}"
+            c.free(p)
+    dist.barrier()
+    c.sync()
+    c.close()
+
+
+def mp_tensor(ptr, n):
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    return mp.as_tensor(ptr, n)
+
+
 def scenario_coll(rank, world):
     """NEXT f3: mp_alltoall (Bruck, pairwise) and mp_allreduce (K-nomial when
     W is a power of two, ring) through the multi-rank engine against the oracle's MPI
@@ -371,7 +424,8 @@ def main():
     try:
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
-         "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll}[scen](rank, world)
+         "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
+         "eager": scenario_eager}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

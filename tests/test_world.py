@@ -90,3 +90,14 @@ def test_multirank_collectives(world):
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(world, "coll", timeout=600)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 3])
+def test_multirank_eager_protocol(world):
+    # reading C23: small messages skip the rendezvous
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(world, "eager", timeout=400)
