@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cstring>
 #include <map>
+#include <new>
 #include <string>
 #include <tuple>
 #include <vector>
@@ -234,8 +235,7 @@ extern "C" int mp_coll_plan_build(int coll, int algo, int world, int rank, uint6
 
 // ------------------------------------------------------------------ executor
 
-namespace {
-
+namespace mpx {
 struct CollState {
   cudaStream_t s = nullptr, r = nullptr;   // internal send / receive streams
   std::vector<cudaEvent_t> ev;             // event pool
@@ -244,8 +244,9 @@ struct CollState {
   uint64_t seq = 0;
   std::map<std::tuple<int, int, uint64_t, uint32_t>, std::vector<mp_config>> cfgs;  // per-step configs
 };
+}  // namespace mpx
 
-std::map<mp_ctx *, CollState> g_state;  // one per context (contexts are single-threaded)
+namespace {
 
 int ensure(mp_ctx *c, CollState &st, uint64_t need, int nev) {
   if (!st.s) {
@@ -323,7 +324,9 @@ int local_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, cudaStream_t s
 
 int run_plan(mp_ctx *c, const mp_coll_plan &P, const void *sendbuf, void *recvbuf, uint64_t bytes, uint32_t elem,
              int dtype, void *ustream) {
-  CollState &st = g_state[c];
+  if (!c->coll) c->coll = new (std::nothrow) CollState();
+  if (!c->coll) return MP_ERR_NOMEM;
+  CollState &st = *c->coll;
   uint64_t maxmsg = 0;
   for (int j = 0; j < P.nsteps; ++j) maxmsg = std::max(maxmsg, P.step[j].bytes);
   const uint64_t align = 256;
@@ -435,9 +438,8 @@ int collective(mp_ctx *c, int coll, int algo, const void *sendbuf, void *recvbuf
 }  // namespace
 
 void mpx::coll_release(mp_ctx *c) {
-  auto it = g_state.find(c);
-  if (it == g_state.end()) return;
-  CollState &st = it->second;
+  if (!c->coll) return;
+  CollState &st = *c->coll;
   if (st.s) cudaStreamSynchronize(st.s);
   if (st.r) cudaStreamSynchronize(st.r);
   for (cudaEvent_t e : st.ev) cudaEventDestroy(e);
@@ -449,7 +451,8 @@ void mpx::coll_release(mp_ctx *c) {
   if (st.s) cudaStreamDestroy(st.s);
   if (st.r) cudaStreamDestroy(st.r);
   if (st.scratch) mp_free(c, st.scratch);
-  g_state.erase(it);
+  delete c->coll;
+  c->coll = nullptr;
 }
 
 extern "C" int mp_alltoall(mp_ctx *c, const void *sendbuf, void *recvbuf, uint64_t bytes_per_rank, int algo,

@@ -17,6 +17,8 @@
 
 namespace mpx {
 
+struct CollState;  // collectives (coll.cpp): internal streams, events, heap scratch
+
 // A staging ring (D8): S slots of slot_stride bytes + per-CTA flag words.
 struct Ring {
   uint8_t *data = nullptr;     // device memory (relay) or mapped pinned host memory (host)
@@ -111,6 +113,7 @@ struct mp_ctx {
   size_t hseg_bytes = 0;
   std::vector<uint8_t *> hseg;              // [world]: mapped host segment of each receiver
   std::vector<uint64_t> send_seq, recv_seq, relay_q, host_q, done_target;
+  mpx::CollState *coll = nullptr;           // created by the first collective
   std::vector<uint64_t> eager_send_seq, eager_recv_seq;  // eager protocol (reading C23)
   uint64_t eager_max = 0;                   // messages of 1..eager_max bytes go eager
   cudaStream_t relay_stream = nullptr;
