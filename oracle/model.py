@@ -343,7 +343,8 @@ def _solve_level_port(n: float, omegas, deltas, paths, active, opts, port: Port)
 
 
 def select(n: int, paths: Sequence[Path], opts: Options, port: Optional[Port] = None,
-           path_mask: Optional[Sequence[bool]] = None) -> Config:
+           path_mask: Optional[Sequence[bool]] = None,
+           dshift: Optional[Sequence[float]] = None) -> Config:
     """O3 — canonical reading of Algorithm 1 `populate_path_config`.
 
     paths[0] is the direct path (A1 order: direct, GPU-staged by device, host).
@@ -356,7 +357,10 @@ def select(n: int, paths: Sequence[Path], opts: Options, port: Optional[Port] = 
          takes n − Σ (Alg 1 lines 24-28 "give leftover to direct", C7).
       6. [reading C18, B200 mode by default] pass 3: Eq 24 again with the affine
          integer-k coefficients of Eq 13 (``omega_delta_fixed_k``); new shares.
-      7. t_pred = O2 of the config; t_level = the last level solve's finish time."""
+      7. t_pred = O2 of the config; t_level = the last level solve's finish time.
+
+    dshift (NEXT f2, reading C24, oracle/window.py): every level solve uses
+    max(0, Δ_i − dshift_i) in place of Δ_i (the per-message coefficients of a window)."""
     p = len(paths)
     assert paths[0].kind == DIRECT
     mask = list(path_mask) if path_mask is not None else [True] * p
@@ -367,6 +371,8 @@ def select(n: int, paths: Sequence[Path], opts: Options, port: Optional[Port] = 
         port = Port()
 
     def level(om, de, act):
+        if dshift is not None:
+            de = [max(0.0, d - s) for d, s in zip(de, dshift)]
         if opts.mode == B200:
             return _solve_level_port(float(n), om, de, paths, act, opts, port)
         return _solve_level_paper(float(n), om, de, paths, act, opts)
