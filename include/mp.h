@@ -240,6 +240,50 @@ typedef struct mp_flow {
  * configs, caller-allocated.  Not cached.  Host-only. */
 int mp_select_flows(mp_ctx *ctx, int nflows, const mp_flow *flows, mp_config *out);
 
+/* ---------------------------------------------------------------- NEXT f2: windows, BIBW */
+
+/* Window model of the pair (src, dst) (PAPER.md Observation 2, P:358:
+ * "larger window sizes allow for more concurrent transfers, reducing the impact of
+ * latency"; OMB windows).  Reading C24: in a window of w
+ * back-to-back messages with one config, path i's message is an issue phase
+ * a_i = min(h[i], α_i) that may overlap the previous message, then a serve phase
+ * T_i − a_i (T_i = the mp_predict path time), so T_i^w = T_i + (w−1)·max(a_i, T_i − a_i);
+ * the shared port is one more such pipeline (a_S = min(α_S, min a_i of the active paths
+ * through it)); the window adds a fixed completion cost tau (OMB's wait-all + ack):
+ * T^w = tau + max(paths, port).  h[npaths] in seconds, in the order of mp_paths;
+ * npaths must equal the pair's path count; h >= 0, tau >= 0 (defaults 0: h = 0 is the
+ * paper's per-message model, T^w = w·T).  The window parameters apply to every size
+ * band of the pair; mp_set_model with a different path count drops them.
+ * Errors: MP_ERR_INVALID, MP_ERR_TOPOLOGY.  Host-only. */
+int mp_set_window_model(mp_ctx *ctx, int src, int dst, const double *h, int npaths, double tau);
+/* h (MP_MAX_PATHS entries), npaths and tau may each be NULL. */
+int mp_get_window_model(mp_ctx *ctx, int src, int dst, double *h, int *npaths, double *tau);
+
+/* mp_predict_window — T^w of C24 for `window` >= 1 messages of `bytes` each with config
+ * cfg (validated as in mp_predict; window = 1 gives mp_predict + tau).  *seconds = the
+ * whole window.  Errors as mp_predict; MP_ERR_INVALID for window = 0.  Host-only. */
+int mp_predict_window(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t window,
+                      const mp_config *cfg, double *seconds);
+
+/* mp_select_window — Algorithm 1 for a window (reading C24): mp_select on the
+ * window's per-message coefficients (every Δ_i − (1 − 1/w)·a_i, the port's
+ * α_S − (1 − 1/w)·a_S).  out->t_pred = T^w of the result, out->t_level = w·(per-message
+ * level) + tau.  window = 1 returns mp_select's config.  path_mask and MPX_PATHS as in
+ * mp_select.  Not cached.  Host-only. */
+int mp_select_window(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t window,
+                     uint32_t path_mask, mp_config *out);
+
+/* Host duplex factor κ of GPU `gpu` (rank; 0 <= gpu < MP_MAX_PATHS), reading C25
+ * (PAPER.md Observation 5: "contention between the bidirectional transfers
+ * along the host-staged path … the model should be extended to account for host-staged
+ * contention, PCIe configuration").  In mp_select_flows, after C19's fair share, a flow
+ * s -> d (s != d) runs its host up leg at κ_s·β if any flow's host down leg enters s,
+ * and its down leg at κ_d·β' if any flow's host up leg leaves d.  Loopback flows
+ * (s == d) are calibrated duplex and are not scaled.  kappa in (0, 1]; default 1.
+ * Errors: MP_ERR_INVALID (kappa out of range), MP_ERR_TOPOLOGY (gpu out of range). */
+int mp_set_host_duplex(mp_ctx *ctx, int gpu, double kappa);
+int mp_get_host_duplex(mp_ctx *ctx, int gpu, double *kappa);
+
 /* ---------------------------------------------------------------- memory */
 
 /* Allocate / free device memory from this rank's registered heap.  A buffer that

@@ -552,6 +552,8 @@ int mp_set_model(mp_ctx *c, int src, int dst, const mp_path *paths, const mp_pat
   }
   c->models[std::make_pair(src, dst)] = m;
   c->bands.erase(std::make_pair(src, dst));  // a new base model drops the pair's bands
+  auto wt = c->windows.find(std::make_pair(src, dst));  // … and window params of another path list
+  if (wt != c->windows.end() && wt->second.h.size() != m.paths.size()) c->windows.erase(wt);
   c->cache.clear();
   return MP_OK;
 }
@@ -731,8 +733,94 @@ int mp_select_flows(mp_ctx *c, int nflows, const mp_flow *flows, mp_config *out)
     specs.push_back(s);
   }
   std::vector<Selection> sel;
-  select_flows(models, specs, c->opts, &sel);
+  select_flows(models, specs, c->opts, &sel, &c->kappa);
   for (int f = 0; f < nflows; ++f) fill_config(*models[f], sel[f], &out[f]);
+  return MP_OK;
+}
+
+// ------------------------------------------------------------------ NEXT f2 (C24, C25)
+
+int mp_set_window_model(mp_ctx *c, int src, int dst, const double *h, int npaths, double tau) {
+  if (!c || (npaths > 0 && !h)) return fail(c, MP_ERR_INVALID, "null argument");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  if (npaths != static_cast<int>(m->paths.size()))
+    return fail(c, MP_ERR_INVALID, "window npaths must equal the pair's path count");
+  if (!(tau >= 0.0) || !std::isfinite(tau)) return fail(c, MP_ERR_INVALID, "tau must be finite and >= 0");
+  WindowModel w;
+  for (int i = 0; i < npaths; ++i) {
+    if (!(h[i] >= 0.0) || !std::isfinite(h[i])) return fail(c, MP_ERR_INVALID, "h must be finite and >= 0");
+    w.h.push_back(h[i]);
+  }
+  w.tau = tau;
+  c->windows[std::make_pair(src, dst)] = w;
+  return MP_OK;
+}
+
+int mp_get_window_model(mp_ctx *c, int src, int dst, double *h, int *npaths, double *tau) {
+  if (!c) return MP_ERR_INVALID;
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = pair_model(c, src, dst);
+  auto it = c->windows.find(std::make_pair(src, dst));
+  if (npaths) *npaths = static_cast<int>(m->paths.size());
+  if (h)
+    for (size_t i = 0; i < m->paths.size(); ++i)
+      h[i] = (it != c->windows.end() && i < it->second.h.size()) ? it->second.h[i] : 0.0;
+  if (tau) *tau = it != c->windows.end() ? it->second.tau : 0.0;
+  return MP_OK;
+}
+
+static const WindowModel &window_of_pair(mp_ctx *c, int src, int dst) {
+  static const WindowModel none;
+  auto it = c->windows.find(std::make_pair(src, dst));
+  return it == c->windows.end() ? none : it->second;
+}
+
+int mp_predict_window(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t window, const mp_config *cfg,
+                      double *seconds) {
+  if (!c || !cfg || !seconds) return fail(c, MP_ERR_INVALID, "null argument");
+  if (window < 1) return fail(c, MP_ERR_INVALID, "window must be >= 1");
+  double t1 = 0.0;
+  if (int s = mp_predict(c, src, dst, bytes, cfg, &t1)) return s;  // validates the config
+  *seconds = predict_window(*model_for(c, src, dst, bytes), window_of_pair(c, src, dst), bytes, window,
+                            cfg->bytes, cfg->chunks, c->opts);
+  return MP_OK;
+}
+
+int mp_select_window(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t window, uint32_t mask,
+                     mp_config *out) {
+  if (!c || !out) return fail(c, MP_ERR_INVALID, "null argument");
+  if (window < 1) return fail(c, MP_ERR_INVALID, "window must be >= 1");
+  if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
+  const PairModel *m = model_for(c, src, dst, bytes);
+  if (c->env_kinds != 0x7u) {  // MPX_PATHS, as in mp_select
+    uint32_t eff = 0;
+    for (size_t i = 0; i < m->paths.size(); ++i) {
+      const bool asked = mask == 0 || ((mask >> i) & 1u);
+      if (i == 0 || (asked && ((c->env_kinds >> m->paths[i].kind) & 1u))) eff |= 1u << i;
+    }
+    mask = eff;
+  }
+  Selection s;
+  select_window(*m, window_of_pair(c, src, dst), bytes, window, mask, c->opts, &s);
+  fill_config(*m, s, out);
+  return MP_OK;
+}
+
+int mp_set_host_duplex(mp_ctx *c, int gpu, double kappa) {
+  if (!c) return MP_ERR_INVALID;
+  if (gpu < 0 || gpu >= MP_MAX_PATHS) return fail(c, MP_ERR_TOPOLOGY, "gpu out of range");
+  if (!(kappa > 0.0) || !(kappa <= 1.0)) return fail(c, MP_ERR_INVALID, "kappa must be in (0, 1]");
+  if (static_cast<int>(c->kappa.size()) <= gpu) c->kappa.resize(gpu + 1, 1.0);
+  c->kappa[gpu] = kappa;
+  c->cache.clear();
+  return MP_OK;
+}
+
+int mp_get_host_duplex(mp_ctx *c, int gpu, double *kappa) {
+  if (!c || !kappa) return MP_ERR_INVALID;
+  if (gpu < 0 || gpu >= MP_MAX_PATHS) return fail(c, MP_ERR_TOPOLOGY, "gpu out of range");
+  *kappa = gpu < static_cast<int>(c->kappa.size()) ? c->kappa[gpu] : 1.0;
   return MP_OK;
 }
 
@@ -904,6 +992,12 @@ int mp_save_params(mp_ctx *c, const char *path) {
     for (const PathModel &p : m.paths)
       std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via,
                    p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
+    auto wt = c->windows.find(kv.first);
+    if (wt != c->windows.end()) {
+      std::fprintf(f, "window %d %d %zu %.17g", kv.first.first, kv.first.second, wt->second.h.size(), wt->second.tau);
+      for (double h : wt->second.h) std::fprintf(f, " %.17g", h);
+      std::fprintf(f, "\n");
+    }
     auto bt = c->bands.find(kv.first);
     if (bt == c->bands.end()) continue;
     for (const auto &b : bt->second) {
@@ -914,6 +1008,8 @@ int mp_save_params(mp_ctx *c, const char *path) {
                      p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
     }
   }
+  for (size_t g = 0; g < c->kappa.size(); ++g)
+    if (c->kappa[g] != 1.0) std::fprintf(f, "duplex %zu 0 1 %.17g\n", g, c->kappa[g]);
   std::fclose(f);
   return MP_OK;
 }
@@ -933,6 +1029,25 @@ int mp_load_params(mp_ctx *c, const char *path) {
   unsigned long long n_min = 0;
   double pa, pb;
   while (std::fscanf(f, "%31s %d %d %zu", tag, &src, &dst, &np) == 4) {
+    if (std::strcmp(tag, "window") == 0 || std::strcmp(tag, "duplex") == 0) {  // NEXT f2
+      const bool win = tag[0] == 'w';
+      double tau = 0.0, h[MP_MAX_PATHS];
+      if (np < 1 || np > MP_MAX_PATHS || std::fscanf(f, "%lf", &tau) != 1) break;
+      if (win)
+        for (size_t i = 0; i < np; ++i)
+          if (std::fscanf(f, "%lf", &h[i]) != 1) {
+            std::fclose(f);
+            return fail(c, MP_ERR_INVALID, "truncated parameter file");
+          }
+      int s = MP_OK;
+      if (win && pair_ok(c, src, dst)) s = mp_set_window_model(c, src, dst, h, static_cast<int>(np), tau);
+      if (!win) s = mp_set_host_duplex(c, src, tau);
+      if (s) {
+        std::fclose(f);
+        return s;
+      }
+      continue;
+    }
     const bool band = std::strcmp(tag, "band") == 0;
     if ((!band && std::strcmp(tag, "pair")) || np < 1 || np > MP_MAX_PATHS) break;
     if (band && std::fscanf(f, "%llu", &n_min) != 1) break;

@@ -77,6 +77,10 @@ struct mp_ctx {
   // NEXT f4 size bands (reading C20): per pair, (n_min, model) ascending, n_min > 0;
   // the base model (models) is band 0 with n_min = 0.
   std::map<std::pair<int, int>, std::vector<std::pair<uint64_t, mpx::PairModel>>> bands;
+  // NEXT f2 (readings C24, C25): per-pair window parameters and per-GPU host duplex
+  // factors (absent = h 0, τ 0; κ 1).
+  std::map<std::pair<int, int>, mpx::WindowModel> windows;
+  std::vector<double> kappa;
   std::unordered_map<mpx::CacheKey, mpx::Selection, mpx::CacheKeyHash> cache;
   uint32_t env_kinds = 0x7u;       // path kinds allowed by MPX_PATHS (bit = MP_PATH_*)
 

@@ -202,8 +202,15 @@ Level level_port(const PairModel &m, double n, const std::vector<double> &om,
   }
 }
 
+// dshift (NEXT f2, reading C24): the level solves use max(0, Δ_i − dshift_i).
 Level solve(const PairModel &m, double n, const std::vector<double> &om,
-            const std::vector<double> &de, const std::vector<char> &act, const ModelOpts &o) {
+            const std::vector<double> &de, const std::vector<char> &act, const ModelOpts &o,
+            const double *dshift = nullptr) {
+  if (dshift) {
+    std::vector<double> ds(de.size());
+    for (size_t i = 0; i < de.size(); ++i) ds[i] = std::max(0.0, de[i] - dshift[i]);
+    return o.mode == M_B200 ? level_port(m, n, om, ds, act, o) : level_paper(m, n, om, ds, act, o);
+  }
   return o.mode == M_B200 ? level_port(m, n, om, de, act, o) : level_paper(m, n, om, de, act, o);
 }
 
@@ -302,7 +309,8 @@ double predict(const PairModel &m, uint64_t n, const uint64_t *bytes, const uint
   return t;
 }
 
-void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, Selection *out) {
+void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, Selection *out,
+            const double *dshift) {
   const size_t p = m.paths.size();
   out->bytes.assign(p, 0);
   out->chunks.assign(p, 0);
@@ -316,7 +324,7 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
   // Pass 1: unpipelined Ω, Δ; Eq 11 / port level with the active set.
   std::vector<double> om(p), de(p);
   for (size_t i = 0; i < p; ++i) od_unpipelined(m.paths[i], &om[i], &de[i]);
-  Level L0 = solve(m, nd, om, de, act, o);
+  Level L0 = solve(m, nd, om, de, act, o, dshift);
 
   // Pass 2: φ from θ⁽⁰⁾, Eq 22, Eq 24.
   std::vector<double> phi(p, 0.0);
@@ -331,7 +339,7 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
   }
   std::vector<char> act1 = L0.act;
   act1[0] = 1;
-  Level L = solve(m, nd, om, de, act1, o);
+  Level L = solve(m, nd, om, de, act1, o, dshift);
 
   shares_of(n, L, o, &out->bytes);
   out->chunks[0] = 1;
@@ -348,7 +356,7 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
       od_fixed_k(m.paths[i], std::max<uint32_t>(1, out->chunks[i]), o.mode, &om[i], &de[i]);
       act3[i] = (i == 0) || out->bytes[i] > 0;
     }
-    L = solve(m, nd, om, de, act3, o);
+    L = solve(m, nd, om, de, act3, o, dshift);
     std::vector<uint32_t> k_prev = out->chunks;
     shares_of(n, L, o, &out->bytes);
     for (size_t i = 1; i < p; ++i)
@@ -361,6 +369,71 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
   out->t_pred = predict(m, n, out->bytes.data(), out->chunks.data(), o);
 }
 
+// ------------------------------------------------------------------ NEXT f2 (C24)
+// A window of w back-to-back messages with one config (PAPER.md Obs 2).  Path
+// i's message = an issue phase a_i = min(h_i, α_i) that may overlap the previous
+// message's serve phase, then the serve phase T_i − a_i: T_i^w = T_i + (w−1)·max(a_i,
+// T_i − a_i).  The port is one more such pipeline with a_S = min(α_S, min a_i of the
+// active paths through it).  T^w = τ + max(paths, port).
+
+namespace {
+inline double issue_part(const PathModel &p, const WindowModel &wm, size_t i) {
+  const double h = i < wm.h.size() ? wm.h[i] : 0.0;
+  return std::min(std::max(h, 0.0), p.alpha);
+}
+inline double window_of(double t1, double a, uint32_t w) {
+  return t1 + static_cast<double>(w - 1) * std::max(a, t1 - a);
+}
+double port_issue(const PairModel &m, const WindowModel &wm, const std::vector<char> &act) {
+  double a = kInf;
+  for (size_t i = 0; i < m.paths.size(); ++i)
+    if (act[i] && m.paths[i].w > 0.0) a = std::min(a, issue_part(m.paths[i], wm, i));
+  return a == kInf ? 0.0 : std::min(m.port_alpha, a);
+}
+}  // namespace
+
+double predict_window(const PairModel &m, const WindowModel &wm, uint64_t n, uint32_t w,
+                      const uint64_t *bytes, const uint32_t *chunks, const ModelOpts &o) {
+  if (n == 0) return 0.0;
+  const size_t p = m.paths.size();
+  std::vector<char> act(p);
+  for (size_t i = 0; i < p; ++i) act[i] = bytes[i] > 0;
+  std::vector<double> st;
+  stagger_of(m, act, o, &st);
+  double t = 0.0;
+  for (size_t i = 0; i < p; ++i) {
+    if (!act[i]) continue;
+    const PathModel &q = m.paths[i];
+    const double b = static_cast<double>(bytes[i]);
+    const double ti = (q.kind == K_DIRECT) ? q.alpha + b / q.beta : staged_time(q, b, chunks[i], o.mode);
+    t = std::max(t, window_of(ti + st[i], issue_part(q, wm, i), w));
+  }
+  if (o.mode == M_B200 && m.has_port()) {
+    double load = 0.0;
+    for (size_t i = 0; i < p; ++i) load += m.paths[i].w * static_cast<double>(bytes[i]);
+    if (load > 0.0) t = std::max(t, window_of(m.port_alpha + load / m.port_beta, port_issue(m, wm, act), w));
+  }
+  return wm.tau + t;
+}
+
+void select_window(const PairModel &m, const WindowModel &wm, uint64_t n, uint32_t w, uint32_t mask,
+                   const ModelOpts &o, Selection *out) {
+  const size_t p = m.paths.size();
+  const double f = 1.0 - 1.0 / static_cast<double>(w);
+  std::vector<double> shift(p);
+  std::vector<char> allowed(p);
+  for (size_t i = 0; i < p; ++i) {
+    shift[i] = f * issue_part(m.paths[i], wm, i);
+    allowed[i] = (i == 0) || mask == 0 || ((mask >> i) & 1u);
+  }
+  PairModel mw = m;  // per-message port startup of the window
+  if (m.has_port()) mw.port_alpha = m.port_alpha - f * port_issue(m, wm, allowed);
+  select(mw, n, mask, o, out, shift.data());
+  if (n == 0) return;
+  out->t_pred = predict_window(m, wm, n, w, out->bytes.data(), out->chunks.data(), o);
+  out->t_level = static_cast<double>(w) * out->t_level + wm.tau;
+}
+
 }  // namespace mpx
 
 namespace mpx {
@@ -370,7 +443,7 @@ namespace mpx {
 // be extracted"; MaxRate for contention on shared links).  Every link used by
 // k flows gives each 1/k of its bandwidth; then every flow is selected on its own.
 void select_flows(const std::vector<const PairModel *> &models, const std::vector<FlowSpec> &flows,
-                  const ModelOpts &o, std::vector<Selection> *out) {
+                  const ModelOpts &o, std::vector<Selection> *out, const std::vector<double> *kappa) {
   const size_t F = flows.size();
   auto allowed = [&](size_t f, size_t i) {
     return i == 0 || flows[f].mask == 0 || ((flows[f].mask >> i) & 1u);
@@ -423,6 +496,14 @@ void select_flows(const std::vector<const PairModel *> &models, const std::vecto
       } else {
         p.beta /= std::max(1, host_out[s]);
         p.beta2 /= std::max(1, host_in[d]);
+        // C25 (NEXT f2, Obs 5 P:379-385): a leg whose PCIe link also carries the other
+        // direction runs at the duplex factor κ of that GPU; loopback legs are
+        // calibrated duplex already.
+        if (kappa && s != d) {
+          auto kap = [&](int g) { return g < static_cast<int>(kappa->size()) ? (*kappa)[g] : 1.0; };
+          if (host_in[s] > 0) p.beta *= kap(s);
+          if (host_out[d] > 0) p.beta2 *= kap(d);
+        }
       }
       if (on) mask |= 1u << i;
     }

@@ -50,8 +50,24 @@ std::string validate_model(const PairModel &m);
 double predict(const PairModel &m, uint64_t n, const uint64_t *bytes, const uint32_t *chunks,
                const ModelOpts &o);
 
-// O3: Algorithm 1.  mask bit i enables path i (bit 0 forced on).
-void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, Selection *out);
+// O3: Algorithm 1.  mask bit i enables path i (bit 0 forced on).  dshift (NEXT f2,
+// C24): per-path amounts subtracted from every Δ_i of the level solves (may be null).
+void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, Selection *out,
+            const double *dshift = nullptr);
+
+// NEXT f2 (reading C24): window parameters of a pair — h[i] the startup of path i a
+// back-to-back successor overlaps (a_i = min(h_i, α_i); empty = 0), tau the fixed
+// completion cost of a window [s].
+struct WindowModel {
+  std::vector<double> h;
+  double tau = 0.0;
+};
+// Time of w back-to-back messages of n bytes with one config (W1).
+double predict_window(const PairModel &m, const WindowModel &wm, uint64_t n, uint32_t w,
+                      const uint64_t *bytes, const uint32_t *chunks, const ModelOpts &o);
+// Alg 1 on the window's per-message coefficients; t_pred = W1, t_level = w·level + τ.
+void select_window(const PairModel &m, const WindowModel &wm, uint64_t n, uint32_t w, uint32_t mask,
+                   const ModelOpts &o, Selection *out);
 
 // The C5 integer rule (exposed for tests through the selector only).
 uint32_t k_from_real(double k_real);
@@ -63,8 +79,10 @@ struct FlowSpec {
   uint64_t bytes = 0;
   uint32_t mask = 0;  // path mask of the pair (0 = all)
 };
+// kappa (NEXT f2, reading C25): per-GPU host duplex factor (may be null = all 1).
 void select_flows(const std::vector<const PairModel *> &models, const std::vector<FlowSpec> &flows,
-                  const ModelOpts &o, std::vector<Selection> *out);
+                  const ModelOpts &o, std::vector<Selection> *out,
+                  const std::vector<double> *kappa = nullptr);
 
 // Eq 14 / Eq 15: the real optimal chunk count of a staged path
 // carrying x bytes (used by the φ calibration).

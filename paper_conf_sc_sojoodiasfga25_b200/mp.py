@@ -160,6 +160,15 @@ def lib():
             "mp_alltoall": (C.c_int, [P, P, P, C.c_uint64, C.c_int, P]),
             "mp_allreduce": (C.c_int, [P, P, P, C.c_uint64, C.c_int, C.c_int, C.c_int, P]),
             "mp_calibrate_bands": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int]),
+            "mp_set_window_model": (C.c_int, [P, C.c_int, C.c_int, C.POINTER(C.c_double), C.c_int, C.c_double]),
+            "mp_get_window_model": (C.c_int, [P, C.c_int, C.c_int, C.POINTER(C.c_double), C.POINTER(C.c_int),
+                                              C.POINTER(C.c_double)]),
+            "mp_predict_window": (C.c_int, [P, C.c_int, C.c_int, C.c_uint64, C.c_uint32, C.POINTER(mp_config),
+                                            C.POINTER(C.c_double)]),
+            "mp_select_window": (C.c_int, [P, C.c_int, C.c_int, C.c_uint64, C.c_uint32, C.c_uint32,
+                                           C.POINTER(mp_config)]),
+            "mp_set_host_duplex": (C.c_int, [P, C.c_int, C.c_double]),
+            "mp_get_host_duplex": (C.c_int, [P, C.c_int, C.POINTER(C.c_double)]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
                                        C.POINTER(C.c_double)]),
@@ -179,7 +188,9 @@ def exported_symbols() -> List[str]:
             "mp_calibrate", "mp_save_params", "mp_load_params", "mp_stats", "mp_fit_hockney",
             "mp_peer_base", "mp_select_flows", "mp_register", "mp_deregister",
             "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands",
-            "mp_coll_plan_build", "mp_alltoall", "mp_allreduce"]
+            "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
+            "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
+            "mp_set_host_duplex", "mp_get_host_duplex"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -375,6 +386,34 @@ class Context:
         out = (mp_config * max(1, n))()
         self._ck(lib().mp_select_flows(self.h, n, arr, out))
         return [out[i] for i in range(n)]
+
+    # ---------------------------------------------------------------- NEXT f2 (C24, C25)
+    def set_window_model(self, src, dst, h: Sequence[float], tau: float = 0.0):
+        self._ck(lib().mp_set_window_model(self.h, src, dst, (C.c_double * max(1, len(h)))(*h), len(h), tau))
+
+    def get_window_model(self, src=0, dst=0):
+        h = (C.c_double * MP_MAX_PATHS)()
+        n, tau = C.c_int(), C.c_double()
+        self._ck(lib().mp_get_window_model(self.h, src, dst, h, C.byref(n), C.byref(tau)))
+        return [h[i] for i in range(n.value)], tau.value
+
+    def predict_window(self, src, dst, n, window, cfg: mp_config) -> float:
+        t = C.c_double()
+        self._ck(lib().mp_predict_window(self.h, src, dst, n, window, C.byref(cfg), C.byref(t)))
+        return t.value
+
+    def select_window(self, src, dst, n, window, mask=0) -> mp_config:
+        cfg = mp_config()
+        self._ck(lib().mp_select_window(self.h, src, dst, n, window, mask, C.byref(cfg)))
+        return cfg
+
+    def set_host_duplex(self, gpu, kappa):
+        self._ck(lib().mp_set_host_duplex(self.h, gpu, kappa))
+
+    def get_host_duplex(self, gpu) -> float:
+        k = C.c_double()
+        self._ck(lib().mp_get_host_duplex(self.h, gpu, C.byref(k)))
+        return k.value
 
     # ---------------------------------------------------------------- engine
     def alloc(self, n) -> int:

@@ -1,0 +1,142 @@
+"""NEXT f2 — parity of the library's window model (mp_predict_window, mp_select_window,
+reading C24) and host duplex factor (mp_set_host_duplex in mp_select_flows, reading
+C25) with the oracle (oracle/window.py).  CPU only (model-only contexts)."""
+import math
+import os
+import random
+
+import pytest
+
+import synth
+from oracle import model as M
+from oracle import window as WN
+from paper_conf_sc_sojoodiasfga25_b200 import mp
+
+MiB = 1 << 20
+W = 4
+FIELDS = ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")
+
+
+def rel(a, b):
+    return abs(a - b) / max(abs(b), 1e-300)
+
+
+def table(s, d, seed=0):
+    relays = [r for r in range(W) if r not in (s, d)]
+    tbl = synth.topology(seed + 10 * s + d, len(relays), True)
+    for t, r in zip(tbl[1:1 + len(relays)], relays):
+        t["via"] = r
+    return tbl
+
+
+def install(c, s, d, tbl, port):
+    params = [{k: (0.0 if k == "beta2" and math.isinf(t[k]) else t[k]) for k in FIELDS} for t in tbl]
+    c.set_model(s, d, [(t["kind"], t["via"]) for t in tbl], params,
+                None if port is None else dict(alpha=port.alpha, beta=port.beta))
+
+
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("mode", [M.PAPER, M.B200])
+def test_select_and_predict_window_parity(seed, mode):
+    rng = random.Random(seed)
+    tbl = table(0, 1, seed)
+    paths = [M.Path(**t) for t in tbl]
+    port = M.Port(alpha=rng.uniform(1, 4) * 1e-6, beta=850e9)
+    h = [rng.uniform(0, 1.5) * p.alpha for p in paths]
+    tau = rng.uniform(0, 10e-6)
+    opts = M.Options(mode=mode, slot_bytes=64 * MiB)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.set_options(mode=mode, slot_bytes=64 * MiB)
+        install(c, 0, 1, tbl, port)
+        c.set_window_model(0, 1, h, tau)
+        hh, tt = c.get_window_model(0, 1)
+        assert hh == h and tt == tau
+        for n in (1 * MiB + 17, 16 * MiB, 64 * MiB, 1024 * MiB):
+            for w in (1, 2, 16, 64):
+                ref = WN.select_window(n, w, paths, h, opts, port, tau=tau)
+                got = c.select_window(0, 1, n, w).as_dict()
+                assert sum(got["bytes"]) == n
+                for a, b in zip(got["bytes"], ref.bytes):
+                    assert abs(a - b) <= 256
+                assert rel(got["t_level"], ref.t_level) < 1e-9
+                if got["bytes"] == ref.bytes:
+                    assert got["chunks"] == ref.chunks and rel(got["t_pred"], ref.t_pred) < 1e-9
+                # mp_predict_window on the oracle's config
+                cfg = c.make_config(ref.bytes, ref.chunks, 0, 1)
+                t = c.predict_window(0, 1, n, w, cfg)
+                assert rel(t, WN.evaluate_window(n, w, ref.bytes, ref.chunks, paths, h, opts, port, tau)) < 1e-9
+                if w == 1:
+                    assert rel(t, c.predict(0, 1, n, cfg) + tau) < 1e-12
+
+
+def test_window_defaults_and_errors():
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        n = 64 * MiB
+        base = c.select(0, 1, n).as_dict()
+        for w in (1, 8):  # no window model installed: h = 0, τ = 0 → w × the message
+            got = c.select_window(0, 1, n, w).as_dict()
+            assert got["bytes"] == base["bytes"] and rel(got["t_pred"], w * base["t_pred"]) < 1e-12
+        h, tau = c.get_window_model(0, 1)
+        assert h == [0.0] * len(c.paths(0, 1)) and tau == 0.0
+        with pytest.raises(mp.MPError):
+            c.select_window(0, 1, n, 0)
+        with pytest.raises(mp.MPError):
+            c.set_window_model(0, 1, [1e-6], 0.0)           # wrong path count
+        with pytest.raises(mp.MPError):
+            c.set_window_model(0, 1, [-1.0] * len(h), 0.0)  # h < 0
+        with pytest.raises(mp.MPError):
+            c.set_host_duplex(0, 0.0)
+        with pytest.raises(mp.MPError):
+            c.set_host_duplex(0, 1.5)
+        assert c.get_host_duplex(3) == 1.0
+
+
+def test_window_and_duplex_survive_the_params_file(tmp_path):
+    f = str(tmp_path / "p.txt")
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        h = [float(i + 1) * 1e-6 for i in range(len(c.paths(0, 1)))]
+        c.set_window_model(0, 1, h, 3e-6)
+        c.set_host_duplex(2, 0.75)
+        c.save_params(f)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.load_params(f)
+        assert c.get_window_model(0, 1) == (h, 3e-6)
+        assert c.get_host_duplex(2) == 0.75 and c.get_host_duplex(1) == 1.0
+
+
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("mode", [M.PAPER, M.B200])
+def test_select_flows_duplex_parity(seed, mode):
+    rng = random.Random(50 + seed)
+    kappa = {g: rng.choice([1.0, rng.uniform(0.5, 1.0)]) for g in range(W)}
+    flows = []
+    for _ in range(rng.randint(1, 6)):
+        s = rng.randrange(W)
+        d = rng.choice([x for x in range(W) if x != s])
+        mask = [True] + [rng.random() < 0.8 for _ in range(W - 1)]
+        flows.append((s, d, rng.choice([16, 64, 256]) * MiB, mask))
+    if rng.random() < 0.5:  # a bidirectional pair
+        flows.append((flows[0][1], flows[0][0], flows[0][2], flows[0][3]))
+
+    def paths(s, d):
+        return [M.Path(**t) for t in table(s, d, seed)]
+
+    def port(s, d):
+        return M.Port(alpha=1e-6, beta=850e9)
+    opts = M.Options(mode=mode, slot_bytes=64 * MiB)
+    ref = WN.select_flows_duplex(flows, paths, port, opts, kappa.get)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.set_options(mode=mode, slot_bytes=64 * MiB)
+        for g, k in kappa.items():
+            c.set_host_duplex(g, k)
+        for s, d in {(s, d) for s, d, _, _ in flows}:
+            install(c, s, d, table(s, d, seed), port(s, d))
+        got = c.select_flows([(s, d, n, sum(1 << i for i, m in enumerate(mask) if m)) for s, d, n, mask in flows])
+        for g, r in zip(got, ref):
+            gd = g.as_dict()
+            assert sum(gd["bytes"]) == sum(r.bytes)
+            for a, b in zip(gd["bytes"], r.bytes):
+                assert abs(a - b) <= 256
+            assert rel(gd["t_level"], r.t_level) < 1e-9
+            if gd["bytes"] == r.bytes:
+                assert gd["chunks"] == r.chunks and rel(gd["t_pred"], r.t_pred) < 1e-9
