@@ -284,6 +284,19 @@ int mp_select_window(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t win
 int mp_set_host_duplex(mp_ctx *ctx, int gpu, double kappa);
 int mp_get_host_duplex(mp_ctx *ctx, int gpu, double *kappa);
 
+/* mp_calibrate_window — Step 1 for the C24/C25 parameters of the loopback pair
+ * (0, 0).  For every path alone (all bytes on it; staged paths in >= 8 chunks) and
+ * every size (NULL/0 = 4, 16, 64 MiB) it times one message on an idle stream (T1) and
+ * `window` (0 = 16) back-to-back messages (TW), median of `reps` (0 = 7).  Then
+ * tau = max(0, median(T1 − mp_predict) over the direct path's sizes), and h_i = median over sizes of
+ * max(0, T1 − tau − (TW − T1)/(window − 1)) (the serve-bound branch of C24).  κ of
+ * this GPU = the mean of (simplex / duplex time) of the two host legs at 64 MiB, each
+ * leg moved by relay_ctas CTAs as in the engine.  Installs them with
+ * mp_set_window_model / mp_set_host_duplex.  Parameters measured on B200: parity
+ * unpinned (the paper prints none).  Errors: MP_ERR_STATE (model-only),
+ * MP_ERR_UNSUPPORTED (world > 1), MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_TIMEOUT. */
+int mp_calibrate_window(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int window, int reps);
+
 /* ---------------------------------------------------------------- memory */
 
 /* Allocate / free device memory from this rank's registered heap.  A buffer that
@@ -363,7 +376,9 @@ int mp_sync(mp_ctx *ctx);
  * world > 1: collective — every rank puts into its successor's heap over NVLink,
  * times its own host legs and a flag ping-pong through the successor's memory;
  * the measurements are all-gathered and every ordered pair's model is built from
- * them.  Requires empty receive heaps on every rank (call before mp_alloc), else
+ * them; each rank also times its two host legs at once against alone and every
+ * rank's host duplex factor κ (reading C25) is installed (mp_set_host_duplex).
+ * Requires empty receive heaps on every rank (call before mp_alloc), else
  * MP_ERR_STATE. */
 int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
 

@@ -353,6 +353,7 @@ struct LinkMeas {
   double h1a, h1b;        // GPU → host α, β
   double h2a, h2b;        // host → GPU α, β
   double eps_dev, eps_host;
+  double kappa;           // host duplex factor of this GPU (reading C25)
 };
 
 // edges = {0}: the plain Step-1 fit (flushed single copies); more edges: one
@@ -395,7 +396,7 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
     t.clear();
     if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, c->relay_ctas, window, &n, &t))) break;
     if ((st = fit_samples(c, n, t, edges, &fr))) break;
-    double eps_host = 0, eps_dev = 0;
+    double eps_host = 0, eps_dev = 0, kappa = 1.0;
     if (c->host_path) {
       // the own segment's ring of sender == me is never used for traffic
       uint8_t *hr = c->hseg[me] + static_cast<uint64_t>(me) * c->hseg_per_src;
@@ -414,6 +415,19 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
       if ((st = sample_link(b, src, hr, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) break;
       if ((st = fit_samples(c, n, t, edges, &fh2))) break;
       if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) break;
+      // κ (reading C25, NEXT f2): both host legs of this GPU alone, then at once
+      const uint64_t hk = std::min<uint64_t>(hcap / 2, 32ull << 20);
+      if (big >= 2 * hk && hk >= (1u << 20)) {
+        double up = 0, down = 0;
+        std::vector<double> kn, k1, k2;
+        uint8_t *sb = static_cast<uint8_t *>(src);
+        if ((st = time_copy(b, hr, sb, hk, hr_reps, &up, c->relay_ctas))) break;
+        if ((st = time_copy(b, sb + big - hk, hr + hcap / 2, hk, hr_reps, &down, c->relay_ctas))) break;
+        if ((st = sample_links_duplex(b, hr, sb, sb + big - hk, hr + hcap / 2, {hk}, hr_reps, c->relay_ctas, true,
+                                      &kn, &k1, &k2)))
+          break;
+        kappa = std::min(1.0, 0.5 * (up / k1[0] + down / k2[0]));
+      }
     }
     uint64_t *pf = reinterpret_cast<uint64_t *>(c->peers[succ].ctrl + c->L.probe);
     if ((st = time_pingpong(b, pf, false, 1000, &eps_dev))) break;
@@ -430,6 +444,7 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
       }
       m[j].eps_dev = eps_dev;
       m[j].eps_host = eps_host;
+      m[j].kappa = std::max(kappa, 1e-3);
     }
   } while (false);
   cudaStreamSynchronize(b.s);
@@ -447,6 +462,8 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
   std::vector<LinkMeas> lm(static_cast<size_t>(W) * B);  // [rank][band]
   if (int s = world_allgather(c, m.data(), lm.data(), sizeof(LinkMeas) * B)) return s;
 
+  for (int g = 0; g < W; ++g)  // reading C25: every GPU's duplex factor
+    if (int e = mp_set_host_duplex(c, g, lm[static_cast<size_t>(g) * B].kappa)) return e;
   for (int s = 0; s < W; ++s)
     for (int d = 0; d < W; ++d) {
       if (s == d) continue;
@@ -608,6 +625,135 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
     return MP_OK;
   }
   return calibrate_loop_bands(c, edges, reps);
+}
+
+// NEXT f2 window / duplex calibration (readings C24, C25), loopback pair (0, 0).
+// Per path alone and per size: T1 = one message on an idle stream, TW = W back-to-back
+// messages (CUDA events around the enqueue, a stream sync before each window — OMB's
+// wait-all).  τ = median(T1 − mp_predict) over the direct path's sizes, clamped >= 0;
+// the steady per-message
+// time s = (TW − T1)/(W − 1) = max(a, T1 − τ − a), read in the serve-bound branch:
+// a = T1 − τ − s; h_i = median over sizes of max(0, a).  κ of this GPU = the host
+// legs' duplex / simplex rate (D2H and H2D alone, then both at once, 64 MiB).
+extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int window, int reps) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (c->world != 1) return cfail(c, MP_ERR_UNSUPPORTED, "mp_calibrate_window: loopback contexts only");
+  if (window <= 0) window = 16;
+  if (window < 2) return cfail(c, MP_ERR_INVALID, "window must be >= 2");
+  if (reps <= 0) reps = 7;
+  std::vector<uint64_t> sizes;
+  if (sizes_in && nsizes > 0)
+    sizes.assign(sizes_in, sizes_in + nsizes);
+  else
+    sizes = {4ull << 20, 16ull << 20, 64ull << 20};
+  uint64_t big = 0;
+  for (uint64_t s : sizes) big = std::max(big, s);
+  if (big == 0) return cfail(c, MP_ERR_INVALID, "sizes must be > 0");
+  const uint64_t ring_cap = static_cast<uint64_t>(c->slots) * c->slot_bytes;
+  const uint64_t hn = std::min<uint64_t>(64ull << 20, ring_cap / 2);  // κ probe size
+  if (c->host_path) big = std::max(big, hn);
+  mp_path paths[MP_MAX_PATHS];
+  int np = 0;
+  if (int s = mp_paths(c, 0, 0, paths, &np)) return s;
+  Bench b;
+  b.c = c;
+  CKC(cudaSetDevice(c->device));
+  CKC(cudaStreamCreateWithFlags(&b.s, cudaStreamNonBlocking));
+  CKC(cudaEventCreate(&b.e0));
+  CKC(cudaEventCreate(&b.e1));
+  void *src = nullptr, *dst = nullptr;
+  CKC(cudaMalloc(&b.flush, b.flush_bytes));
+  CKC(cudaMalloc(&src, big));
+  CKC(cudaMalloc(&dst, big));
+  CKC(cudaMemset(src, 0x3c, big));
+  CKC(cudaDeviceSynchronize());
+  int st = MP_OK;
+  auto timed = [&](const mp_config &cfg, uint64_t n, int W, double *out) -> int {
+    std::vector<double> ts;
+    for (int r = 0; r < reps + 1; ++r) {
+      CKC(cudaStreamSynchronize(b.s));
+      CKC(cudaEventRecord(b.e0, b.s));
+      for (int w = 0; w < W; ++w)
+        if (int e = mp_xfer(c, dst, src, n, &cfg, b.s)) return e;
+      CKC(cudaEventRecord(b.e1, b.s));
+      CKC(cudaEventSynchronize(b.e1));
+      float ms = 0;
+      CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
+      if (r > 0) ts.push_back(ms * 1e-3);
+    }
+    *out = median(ts);
+    return MP_OK;
+  };
+  struct Sample {
+    int path;
+    double t1, tw, pred;
+  };
+  std::vector<Sample> smp;
+  const uint64_t slot_lim = c->opts.slot_bytes ? c->opts.slot_bytes : c->slot_bytes;
+  for (int i = 0; i < np && st == MP_OK; ++i)
+    for (uint64_t n : sizes) {
+      mp_config cfg;
+      std::memset(&cfg, 0, sizeof(cfg));
+      cfg.npaths = np;
+      for (int j = 0; j < np; ++j) cfg.path[j] = paths[j];
+      cfg.bytes[i] = n;
+      cfg.chunks[0] = 1;
+      if (i > 0) {
+        uint64_t k = std::max<uint64_t>(8, (n + slot_lim - 1) / slot_lim);
+        k = std::min<uint64_t>(k, std::max<uint64_t>(1, n / std::max<uint64_t>(1, c->opts.c_min)));
+        cfg.chunks[i] = static_cast<uint32_t>(std::max<uint64_t>(1, k));
+        if ((n + cfg.chunks[i] - 1) / cfg.chunks[i] > slot_lim) continue;
+      }
+      Sample sm{i, 0, 0, 0};
+      if ((st = mp_predict(c, 0, 0, n, &cfg, &sm.pred))) break;
+      if ((st = timed(cfg, n, 1, &sm.t1))) break;
+      if ((st = timed(cfg, n, window, &sm.tw))) break;
+      smp.push_back(sm);
+    }
+  // κ: host legs alone and at once (reading C25)
+  double kappa = 1.0;
+  if (st == MP_OK && c->host_path) {
+    uint8_t *hr = c->rings[c->n_loop_relays].data;
+    double up = 0, down = 0;
+    std::vector<double> n, t1, t2;
+    if (!(st = time_copy(b, hr, src, hn, reps, &up, c->relay_ctas)) &&
+        !(st = time_copy(b, dst, hr + ring_cap / 2, hn, reps, &down, c->relay_ctas)) &&
+        !(st = sample_links_duplex(b, hr, src, dst, hr + ring_cap / 2, {hn}, reps, c->relay_ctas, true, &n, &t1,
+                                   &t2)))
+      kappa = std::min(1.0, 0.5 * (up / t1[0] + down / t2[0]));
+  }
+  cudaStreamSynchronize(b.s);
+  cudaFree(src);
+  cudaFree(dst);
+  cudaFree(b.flush);
+  cudaEventDestroy(b.e0);
+  cudaEventDestroy(b.e1);
+  cudaStreamDestroy(b.s);
+  if (st) return st;
+  int32_t derr = 0;
+  CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
+  if (derr) return cfail(c, MP_ERR_TIMEOUT, "window calibration transfer timed out");
+  if (smp.empty()) return cfail(c, MP_ERR_INVALID, "no calibration sample fits the staging rings");
+  // τ is a property of the window (idle-stream launch + the host wait), the same for
+  // every config: read it off the direct path, which carries no staging-model error.
+  std::vector<double> taus;
+  for (const Sample &sm : smp)
+    if (sm.path == 0) taus.push_back(sm.t1 - sm.pred);
+  const double tau = taus.empty() ? 0.0 : std::max(0.0, median(taus));
+  double h[MP_MAX_PATHS];
+  for (int i = 0; i < np; ++i) {
+    std::vector<double> as;
+    for (const Sample &sm : smp)
+      if (sm.path == i) {
+        const double steady = (sm.tw - sm.t1) / static_cast<double>(window - 1);
+        as.push_back(std::max(0.0, sm.t1 - tau - steady));
+      }
+    h[i] = as.empty() ? 0.0 : median(as);
+  }
+  if (int e = mp_set_window_model(c, 0, 0, h, np, tau)) return e;
+  if (int e = mp_set_host_duplex(c, c->rank, std::max(kappa, 1e-3))) return e;
+  return MP_OK;
 }
 
 extern "C" int mp_fit_hockney(const double *n, const double *t, int m, double *alpha, double *beta) {

@@ -168,6 +168,7 @@ def lib():
             "mp_select_window": (C.c_int, [P, C.c_int, C.c_int, C.c_uint64, C.c_uint32, C.c_uint32,
                                            C.POINTER(mp_config)]),
             "mp_set_host_duplex": (C.c_int, [P, C.c_int, C.c_double]),
+            "mp_calibrate_window": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int, C.c_int]),
             "mp_get_host_duplex": (C.c_int, [P, C.c_int, C.POINTER(C.c_double)]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
@@ -190,7 +191,7 @@ def exported_symbols() -> List[str]:
             "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands",
             "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
-            "mp_set_host_duplex", "mp_get_host_duplex"]
+            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -409,6 +410,11 @@ class Context:
 
     def set_host_duplex(self, gpu, kappa):
         self._ck(lib().mp_set_host_duplex(self.h, gpu, kappa))
+
+    def calibrate_window(self, sizes: Optional[Sequence[int]] = None, window=16, reps=7):
+        """mp_calibrate_window (loopback; readings C24, C25)."""
+        arr = (C.c_uint64 * len(sizes))(*sizes) if sizes else None
+        self._ck(lib().mp_calibrate_window(self.h, arr, len(sizes) if sizes else 0, window, reps))
 
     def get_host_duplex(self, gpu) -> float:
         k = C.c_double()

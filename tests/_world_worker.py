@@ -72,6 +72,8 @@ def scenario_engine(rank, world):
         c.calibrate(sizes=[4 * MiB, 8 * MiB, 16 * MiB], reps=2)
         _, prm, _ = c.get_model(0, 1)
         assert prm[0]["beta"] > 0 and prm[1]["eps"] > 0
+        # NEXT f2 (reading C25): every rank's host duplex factor is measured and shared
+        assert all(0 < c.get_host_duplex(g) <= 1 for g in range(world))
     # NEXT f4: collective per-band Step 1 (readings C20/C21) on every pair
     c.calibrate_bands([0, 1 * MiB, 8 * MiB], reps=2)
     for dst in range(world):

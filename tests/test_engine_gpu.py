@@ -232,6 +232,34 @@ def test_calibration_installs_sane_parameters():
     c.close()
 
 
+def test_calibrate_window_installs_sane_parameters_and_window_selection_is_bit_exact():
+    # NEXT f2 (readings C24, C25): h_i, τ and κ measured on the loopback engine, and a
+    # transfer with the window-selected config stays bit-exact.
+    c = mp.Context(device=0, n_loop_relays=2, host_path=1, slot_bytes=32 * MiB, heap_bytes=16 * MiB)
+    c.set_options(mode=mp.MP_MODEL_B200)
+    c.calibrate(reps=3)
+    c.calibrate_window(sizes=[4 * MiB, 16 * MiB], window=8, reps=3)
+    h, tau = c.get_window_model(0, 0)
+    _, prm, _ = c.get_model(0, 0)
+    assert len(h) == len(prm)
+    assert all(0.0 <= x < 1e-3 for x in h) and 0.0 <= tau < 1e-3
+    assert 0.2 < c.get_host_duplex(0) <= 1.0
+    n = 16 * MiB + 4096 + 17
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                        generator=torch.Generator("cuda").manual_seed(5))
+    dst = torch.zeros_like(src)
+    for w in (1, 16):
+        cfg = c.select_window(0, 0, n, w)
+        assert sum(cfg.as_dict()["bytes"]) == n
+        c.xfer(dst, src, n, cfg)
+        torch.cuda.synchronize()
+        assert torch.equal(dst, src)
+        dst.zero_()
+        t1 = c.predict(0, 0, n, cfg)
+        assert c.predict_window(0, 0, n, w, cfg) <= w * t1 + tau + 1e-12
+    c.close()
+
+
 def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
     # NEXT f4 (P:360 Observation 4; readings C20/C21): the per-band Step-1 fit installs
     # one parameter set per band, and the model error at small sizes — where the single
