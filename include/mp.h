@@ -99,7 +99,9 @@ typedef struct mp_model_opts {
   int32_t mode;        /* MP_MODEL_PAPER | MP_MODEL_B200 */
   int32_t stagger;     /* 1: Alg 1 line 17 issue stagger; 0: off */
   int32_t refine;      /* pass 3 (C18): 1 on, 0 off, -1 = mode default (B200 on) */
-  int32_t reserved;
+  int32_t window;      /* NEXT f2 (C24): the window mp_select assumes — > 1 makes mp_select
+                          (and so mp_send / mp_xfer with cfg = NULL) return
+                          mp_select_window's config; 0 or 1 = per message (default) */
   uint64_t align;      /* A: share alignment and chunk unit, >= 1 (default 256) */
   uint64_t c_min;      /* smallest staged share and chunk (default 65536) */
   uint64_t k_max;      /* chunk-count cap (default 1024) */
@@ -216,7 +218,8 @@ int mp_predict(mp_ctx *ctx, int src, int dst, uint64_t bytes, const mp_config *c
  * pass 3 (C18).  path_mask bit i enables path i of mp_paths() (bit 0, the direct
  * path, is always on; 0 = all paths).  The environment variable MPX_PATHS (read at
  * mp_init; e.g. "direct,host", "direct,gpu", "all") further restricts the path kinds
- * (P:312-313).  Results are cached (C10).  Host-only. */
+ * (P:312-313).  Results are cached (C10).  With mp_model_opts.window > 1 it returns
+ * mp_select_window's config for that window (NEXT f2, C24).  Host-only. */
 int mp_select(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t path_mask,
               mp_config *out);
 

@@ -655,6 +655,8 @@ int mp_set_options(mp_ctx *c, const mp_model_opts *o) {
   m.c_min = o->c_min;
   m.k_max = o->k_max;
   m.slot_bytes = o->slot_bytes;
+  if (o->window < 0) return fail(c, MP_ERR_INVALID, "window must be >= 0");
+  m.window = o->window > 1 ? static_cast<uint32_t>(o->window) : 1u;
   if (!c->model_only) {  // chunks must fit the engine's staging slots
     const uint64_t lim = c->slot_bytes > 2 * m.align ? c->slot_bytes - 2 * m.align : 1;
     if (m.slot_bytes == 0 || m.slot_bytes > lim) m.slot_bytes = lim;
@@ -674,6 +676,7 @@ int mp_get_options(mp_ctx *c, mp_model_opts *o) {
   o->c_min = c->opts.c_min;
   o->k_max = c->opts.k_max;
   o->slot_bytes = c->opts.slot_bytes;
+  o->window = static_cast<int32_t>(c->opts.window);
   return MP_OK;
 }
 
@@ -694,6 +697,12 @@ int mp_predict(mp_ctx *c, int src, int dst, uint64_t bytes, const mp_config *cfg
   return MP_OK;
 }
 
+static const WindowModel &window_of_pair(mp_ctx *c, int src, int dst) {
+  static const WindowModel none;
+  auto it = c->windows.find(std::make_pair(src, dst));
+  return it == c->windows.end() ? none : it->second;
+}
+
 int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_config *out) {
   if (!c || !out) return fail(c, MP_ERR_INVALID, "null argument");
   if (!pair_ok(c, src, dst)) return fail(c, MP_ERR_TOPOLOGY, "no such pair");
@@ -711,7 +720,10 @@ int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_con
   auto it = c->cache.find(key);  // Alg 1 lines 4-6 (C10)
   if (it == c->cache.end()) {
     Selection s;
-    select(*m, bytes, mask, c->opts, &s);
+    if (c->opts.window > 1)  // NEXT f2: window-aware auto-selection (C24)
+      select_window(*m, window_of_pair(c, src, dst), bytes, c->opts.window, mask, c->opts, &s);
+    else
+      select(*m, bytes, mask, c->opts, &s);
     it = c->cache.emplace(key, std::move(s)).first;  // Alg 1 line 29
   }
   fill_config(*m, it->second, out);
@@ -754,6 +766,7 @@ int mp_set_window_model(mp_ctx *c, int src, int dst, const double *h, int npaths
   }
   w.tau = tau;
   c->windows[std::make_pair(src, dst)] = w;
+  c->cache.clear();  // mp_select depends on it when opts.window > 1
   return MP_OK;
 }
 
@@ -768,12 +781,6 @@ int mp_get_window_model(mp_ctx *c, int src, int dst, double *h, int *npaths, dou
       h[i] = (it != c->windows.end() && i < it->second.h.size()) ? it->second.h[i] : 0.0;
   if (tau) *tau = it != c->windows.end() ? it->second.tau : 0.0;
   return MP_OK;
-}
-
-static const WindowModel &window_of_pair(mp_ctx *c, int src, int dst) {
-  static const WindowModel none;
-  auto it = c->windows.find(std::make_pair(src, dst));
-  return it == c->windows.end() ? none : it->second;
 }
 
 int mp_predict_window(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t window, const mp_config *cfg,

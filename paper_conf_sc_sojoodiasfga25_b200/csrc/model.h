@@ -33,6 +33,7 @@ struct ModelOpts {
   uint64_t c_min = 65536;
   uint64_t k_max = 1024;
   uint64_t slot_bytes = 0;
+  uint32_t window = 1;  // NEXT f2: the window mp_select assumes (C24)
 };
 
 struct Selection {

@@ -42,7 +42,7 @@ class mp_port_params(C.Structure):
 
 class mp_model_opts(C.Structure):
     _fields_ = [("mode", C.c_int32), ("stagger", C.c_int32), ("refine", C.c_int32),
-                ("reserved", C.c_int32), ("align", C.c_uint64), ("c_min", C.c_uint64),
+                ("window", C.c_int32), ("align", C.c_uint64), ("c_min", C.c_uint64),
                 ("k_max", C.c_uint64), ("slot_bytes", C.c_uint64)]
 
 
@@ -350,14 +350,14 @@ class Context:
         return [(pa[i].kind, pa[i].via) for i in range(n.value)], params, dict(alpha=po.alpha, beta=po.beta)
 
     def set_options(self, mode=MP_MODEL_PAPER, stagger=1, refine=-1, align=256, c_min=65536,
-                    k_max=1024, slot_bytes=0):
-        o = mp_model_opts(mode, stagger, refine, 0, align, c_min, k_max, slot_bytes)
+                    k_max=1024, slot_bytes=0, window=1):
+        o = mp_model_opts(mode, stagger, refine, window, align, c_min, k_max, slot_bytes)
         self._ck(lib().mp_set_options(self.h, C.byref(o)))
 
     def get_options(self):
         o = mp_model_opts()
         self._ck(lib().mp_get_options(self.h, C.byref(o)))
-        return {f: getattr(o, f) for f, _ in mp_model_opts._fields_ if f != "reserved"}
+        return {f: getattr(o, f) for f, _ in mp_model_opts._fields_}
 
     def make_config(self, nbytes: Sequence[int], chunks: Sequence[int], src=0, dst=0) -> mp_config:
         cfg = mp_config()

@@ -69,6 +69,29 @@ def test_select_and_predict_window_parity(seed, mode):
                     assert rel(t, c.predict(0, 1, n, cfg) + tau) < 1e-12
 
 
+def test_window_option_makes_mp_select_window_aware():
+    tbl = table(0, 1, 3)
+    paths = [M.Path(**t) for t in tbl]
+    h = [0.8 * p.alpha for p in paths]
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        install(c, 0, 1, tbl, M.Port(alpha=2e-6, beta=850e9))
+        c.set_window_model(0, 1, h, 1e-6)
+        n = 8 * MiB
+        per_msg = c.select(0, 1, n).as_dict()
+        c.set_options(window=16)
+        assert c.get_options()["window"] == 16
+        got = c.select(0, 1, n).as_dict()
+        want = c.select_window(0, 1, n, 16).as_dict()
+        assert got == want
+        ref = WN.select_window(n, 16, paths, h, M.Options(), M.Port(alpha=2e-6, beta=850e9), tau=1e-6)
+        for a, b in zip(got["bytes"], ref.bytes):
+            assert abs(a - b) <= 256
+        c.set_window_model(0, 1, [0.0] * len(h), 0.0)   # invalidates the cache
+        assert c.select(0, 1, n).as_dict()["bytes"] == per_msg["bytes"]
+        c.set_options(window=1)
+        assert c.select(0, 1, n).as_dict() == per_msg
+
+
 def test_window_defaults_and_errors():
     with mp.Context(world=W, rank=0, model_only=True) as c:
         n = 64 * MiB
