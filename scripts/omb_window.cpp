@@ -135,6 +135,66 @@ int main(int argc, char **argv) {
       std::fflush(stdout);
     }
   }
+
+  // osu_bibw (Obs 1 and 5): both directions at once, four buffers, windows of
+  // 16 per direction then a host wait.  Configs: the two flows selected jointly
+  // (mp_select_flows, C19/C25) vs each selected alone (mp_select, the paper's
+  // per-message model), with all paths and with {direct, host} only.
+  uint8_t *Cb = nullptr, *D = nullptr;
+  CK(cudaMalloc(&Cb, maxn));
+  CK(cudaMalloc(&D, maxn));
+  CK(cudaMemset(Cb, 0x3c, maxn));
+  cudaStream_t s2;
+  CK(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+  cudaEvent_t fork, join;
+  CK(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&join, cudaEventDisableTiming));
+  mp_path ps[MP_MAX_PATHS];
+  int np = 0;
+  MK(mp_paths(ctx, 0, 0, ps, &np));
+  const uint32_t host_mask = 1u | (1u << (np - 1));
+  auto bibw = [&](const mp_config &c1, const mp_config &c2, uint64_t n, int w, int it) {
+    auto iter = [&] {
+      CK(cudaEventRecord(fork, s1));
+      CK(cudaStreamWaitEvent(s2, fork, 0));
+      for (int k = 0; k < w; ++k) {
+        MK(mp_xfer(ctx, B, A, n, &c1, s1));
+        MK(mp_xfer(ctx, D, Cb, n, &c2, s2));
+      }
+      CK(cudaEventRecord(join, s2));
+      CK(cudaStreamWaitEvent(s1, join, 0));
+      CK(cudaStreamSynchronize(s1));
+    };
+    for (int i = 0; i < 2; ++i) iter();
+    std::vector<double> ts;
+    for (int r = 0; r < 3; ++r) {
+      const auto t0 = std::chrono::steady_clock::now();
+      for (int i = 0; i < it; ++i) iter();
+      const auto t1 = std::chrono::steady_clock::now();
+      ts.push_back(std::chrono::duration<double>(t1 - t0).count() / it);
+    }
+    std::sort(ts.begin(), ts.end());
+    return 2.0 * static_cast<double>(n) * w / ts[1] / 1e9;
+  };
+  for (uint64_t n = 16ull << 20; n <= maxn; n <<= 2)
+    for (uint32_t mask : {0u, host_mask}) {
+      const int w = 16;
+      const int it = std::max(2, static_cast<int>(std::min(100.0, 4e9 / (2.0 * n * w))));
+      mp_flow fl[2] = {{0, 0, mask, 0, n}, {0, 0, mask, 0, n}};
+      mp_config fc[2], ind;
+      MK(mp_select_flows(ctx, 2, fl, fc));
+      MK(mp_select(ctx, 0, 0, n, mask, &ind));
+      const double b_joint = bibw(fc[0], fc[1], n, w, it);
+      const double b_ind = bibw(ind, ind, n, w, it);
+      std::printf("{\"bibw\": true, \"n\": %llu, \"w\": %d, \"mask\": \"%s\", \"bibw_joint_GBps\": %.4f, "
+                  "\"pred_joint_GBps\": %.4f, \"bibw_independent_GBps\": %.4f, \"pred_independent_GBps\": %.4f",
+                  static_cast<unsigned long long>(n), w, mask ? "direct+host" : "all", b_joint,
+                  2.0 * n / std::max(fc[0].t_pred, fc[1].t_pred) / 1e9, b_ind, 2.0 * n / ind.t_pred / 1e9);
+      print_cfg("cfg_joint", fc[0]);
+      print_cfg("cfg_independent", ind);
+      std::printf("}\n");
+      std::fflush(stdout);
+    }
   MK(mp_sync(ctx));
   mp_finalize(ctx);
   return 0;
