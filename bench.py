@@ -398,6 +398,24 @@ def run_world(args, world, rank, local):
     return 0
 
 
+def selector_overhead(ctx, n, gbps):
+    """E5 (the model's runtime overhead, "<0.1 % of the total execution
+    time" for large messages): mp_select per call through the binding, on a cache
+    miss (every call a new size) and a hit, against the message's measured time."""
+    k = 2000
+    t0 = time.perf_counter()
+    for i in range(k):
+        ctx.select(0, 0, n + 256 * (i + 1))
+    miss = (time.perf_counter() - t0) / k
+    t0 = time.perf_counter()
+    for _ in range(k):
+        ctx.select(0, 0, n)
+    hit = (time.perf_counter() - t0) / k
+    t_msg = n / (gbps * 1e9)
+    return {"miss_us": miss * 1e6, "hit_us": hit * 1e6, "miss_frac_of_message": miss / t_msg,
+            "note": "Python ctypes call included; the message is the timed 1 GiB transfer"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -546,8 +564,11 @@ def main():
         t = med(lambda: ctx.xfer(dst, src, nstage, cfg_s, stream))
         gbs = nstage / t / 1e9
         if name.startswith("relay"):
+            # a staged path is two stage groups of relay_ctas (16) CTAs each, sized for
+            # a relay's NVLink share beside the direct group, not for loopback HBM
             per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "hbm",
-                              "hbm_GBps": 4 * nstage / t / 1e9, "frac": 4 * nstage / t / 1e9 / peak}
+                              "hbm_GBps": 4 * nstage / t / 1e9, "frac": 4 * nstage / t / 1e9 / peak,
+                              "ctas": 32, "hbm_GBps_per_cta": 4 * nstage / t / 1e9 / 32}
         else:
             per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "pcie",
                               "peak": 64.0, "frac": gbs / 64.0,
@@ -641,6 +662,7 @@ def main():
                           "max": per_launch[-1]},
         "baselines": base,
         "per_path": per_path,
+        "select_overhead": selector_overhead(ctx, n, value / world),
     }
     # NEXT f4 (readings C20/C21): the same message modelled with per-band Step-1
     # parameters (calibrated after the timed region; the pick is unchanged at 1 GiB)

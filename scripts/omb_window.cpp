@@ -74,6 +74,21 @@ int main(int argc, char **argv) {
     for (int i = 0; i < np; ++i) std::printf("%s%.3f", i ? ", " : "", h[i] * 1e6);
     std::printf("]}\n");
   }
+  {  // E5: the selector's own cost per call from C, cache miss / hit
+    mp_config t;
+    const int K = 20000;
+    auto t0 = std::chrono::steady_clock::now();
+    for (int i = 0; i < K; ++i) MK(mp_select(ctx, 0, 0, (1ull << 30) + 256ull * (i + 1), 0, &t));
+    auto t1 = std::chrono::steady_clock::now();
+    for (int i = 0; i < K; ++i) MK(mp_select(ctx, 0, 0, 1ull << 30, 0, &t));
+    auto t2 = std::chrono::steady_clock::now();
+    for (int i = 0; i < K; ++i) MK(mp_select_window(ctx, 0, 0, (1ull << 30) + 256ull * (i + 1), 16, 0, &t));
+    auto t3 = std::chrono::steady_clock::now();
+    std::printf("{\"select_miss_us\": %.3f, \"select_hit_us\": %.3f, \"select_window_us\": %.3f}\n",
+                std::chrono::duration<double>(t1 - t0).count() / K * 1e6,
+                std::chrono::duration<double>(t2 - t1).count() / K * 1e6,
+                std::chrono::duration<double>(t3 - t2).count() / K * 1e6);
+  }
   uint8_t *A = nullptr, *B = nullptr, *ack_s = nullptr, *ack_r = nullptr;
   CK(cudaMalloc(&A, maxn));
   CK(cudaMalloc(&B, maxn));
