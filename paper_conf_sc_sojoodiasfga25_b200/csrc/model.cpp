@@ -141,24 +141,38 @@ Level level_paper(const PairModel &m, double n, const std::vector<double> &om,
 
 // B200 mode (C14): bytes deliverable by time T; fractional knapsack on the shared
 // port, paths in ascending (w, index).
+// *slope (if not null) receives d(total)/dT on T's linear piece: total is piecewise
+// linear in T (a path contributes 1/Ω while it is below the port cap, the path the
+// cap cuts (β_S − Σ_{earlier} w_j/Ω_j)/w, the paths after it 0).
 double port_fill(const PairModel &m, double T, const std::vector<double> &om,
                  const std::vector<double> &de, const std::vector<char> &act,
-                 const std::vector<size_t> &order, std::vector<double> *x) {
+                 const std::vector<size_t> &order, std::vector<double> *x, double *slope = nullptr) {
   const bool port = m.has_port();
+  const bool port_open = port && T > m.port_alpha;
   double room = port ? std::max(0.0, T - m.port_alpha) * m.port_beta : kInf;
-  double total = 0.0;
+  double room_slope = port_open ? m.port_beta : 0.0;  // d(room)/dT while no path is cut
+  bool cut = false;
+  double total = 0.0, ds = 0.0;
   if (x) x->assign(m.paths.size(), 0.0);
   for (size_t i : order) {
     if (!act[i]) continue;
     double u = std::max(0.0, (T - de[i]) / om[i]);
+    double du = u > 0.0 ? 1.0 / om[i] : 0.0;
     const double w = m.paths[i].w;
     if (w > 0.0 && port) {
-      u = std::min(u, room / w);
+      if (cut || room / w < u) {  // the port cap binds on this path
+        u = cut ? 0.0 : room / w;
+        du = cut ? 0.0 : room_slope / w;
+        cut = true;
+      }
       room -= w * u;
+      room_slope -= w * du;
     }
     if (x) (*x)[i] = u;
     total += u;
+    ds += du;
   }
+  if (slope) *slope = ds;
   return total;
 }
 
@@ -173,14 +187,30 @@ Level level_port(const PairModel &m, double n, const std::vector<double> &om,
   for (;;) {
     stagger_of(m, act, o, &st);
     for (size_t i = 0; i < p; ++i) ds[i] = de[i] + st[i];
-    double lo = 0.0, hi = 1e-9;
-    while (port_fill(m, hi, om, ds, act, order, nullptr) < n) hi *= 2.0;
-    for (int it = 0; it < 200; ++it) {
-      const double mid = 0.5 * (lo + hi);
-      if (port_fill(m, mid, om, ds, act, order, nullptr) >= n)
-        hi = mid;
+    // smallest T with capacity(T) >= n: capacity is monotone and piecewise linear, so
+    // a bracketed Newton step lands on the root of its piece (bisection as the
+    // safeguard) — the same T as plain bisection, in a handful of evaluations.
+    double lo = 0.0, hi = kInf;  // start: any one active path carrying everything
+    for (size_t i = 0; i < p; ++i)
+      if (act[i]) hi = std::min(hi, ds[i] + n * om[i]);
+    if (!(hi > 1e-9) || !std::isfinite(hi)) hi = 1e-9;
+    while (port_fill(m, hi, om, ds, act, order, nullptr) < n) {
+      lo = hi;
+      hi *= 2.0;
+    }
+    double T = hi;
+    for (int it = 0; it < 400 && hi - lo > 4e-16 * hi; ++it) {
+      double a = 0.0;
+      const double c = port_fill(m, T, om, ds, act, order, nullptr, &a);
+      if (c >= n)
+        hi = T;
       else
-        lo = mid;
+        lo = T;
+      if (c == n) break;
+      double next = a > 0.0 ? T + (n - c) / a : 0.5 * (lo + hi);
+      if (!(next > lo && next < hi)) next = 0.5 * (lo + hi);
+      if (next == T) break;
+      T = next;
     }
     port_fill(m, hi, om, ds, act, order, &x);
     bool changed = false;
