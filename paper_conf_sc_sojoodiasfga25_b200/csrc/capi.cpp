@@ -176,6 +176,9 @@ void free_engine(mp_ctx *c) {
   if (c->big_ev) cudaEventDestroy(c->big_ev);
   c->big_ev = nullptr;
   c->big_valid = false;
+  if (c->ring_ev) cudaEventDestroy(c->ring_ev);
+  c->ring_ev = nullptr;
+  c->ring_valid = false;
 }
 
 int alloc_ring(mp_ctx *c, bool host, Ring *r) {
@@ -312,9 +315,17 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
     r.q += d.k;
   }
   P.nblocks = next;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (staged_ctas && c->ring_valid && c->ring_stream != st) CK(cudaStreamWaitEvent(st, c->ring_ev, 0));
   const int e = launch_xfer(P, stream);
   if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "xfer launch");
   c->launches += 1;
+  if (staged_ctas) {
+    if (!c->ring_ev) CK(cudaEventCreateWithFlags(&c->ring_ev, cudaEventDisableTiming));
+    CK(cudaEventRecord(c->ring_ev, st));
+    c->ring_stream = st;
+    c->ring_valid = true;
+  }
   if (big) {
     if (!c->big_ev) CK(cudaEventCreateWithFlags(&c->big_ev, cudaEventDisableTiming));
     CK(cudaEventRecord(c->big_ev, static_cast<cudaStream_t>(stream)));

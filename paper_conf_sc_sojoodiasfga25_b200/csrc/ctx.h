@@ -102,6 +102,12 @@ struct mp_ctx {
   cudaEvent_t big_ev = nullptr;
   cudaStream_t big_stream = nullptr;
   bool big_valid = false;
+  // the last loopback launch that used the staging rings: ring slots are handed out in
+  // launch order, so a staged launch on another stream runs after it (no two kernels
+  // ever wait on each other's ring slots)
+  cudaEvent_t ring_ev = nullptr;
+  cudaStream_t ring_stream = nullptr;
+  bool ring_valid = false;
   uint64_t *d_probe = nullptr;    // calibration flag words (device)
   uint64_t *h_probe = nullptr;    // calibration flag words (mapped host)
 

@@ -206,6 +206,33 @@ def test_cuda_graph_capture_direct_only(ctx):
     assert e.value.status == -6
 
 
+def test_staged_transfers_on_two_streams(ctx):
+    # osu_bibw with staged paths: both directions share the relay and host rings; a
+    # staged launch on one stream is ordered after the other stream's last staged
+    # launch (ring slots are handed out in launch order), so neither waits on slots the
+    # other holds.  Every payload arrives bit-exact, nothing times out.
+    n = 8 * MiB + 4099
+    ps = ctx.paths()
+    nb = [0] * len(ps)
+    nb[1], nb[-1] = 2 * MiB, 1 * MiB
+    nb[0] = n - sum(nb)
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1], ks[-1] = 4, 3
+    cfg = ctx.make_config(nb, ks)
+    srcs = [torch.from_numpy(synth.payload(n, 30 + i)).cuda() for i in range(2)]
+    dsts = [[torch.zeros(n, dtype=torch.uint8, device="cuda") for _ in range(4)] for _ in range(2)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    torch.cuda.synchronize()
+    for j in range(4):
+        for i in range(2):
+            ctx.xfer(dsts[i][j], srcs[i], n, cfg, streams[i])
+    torch.cuda.synchronize()
+    ctx.sync()
+    for i in range(2):
+        for d in dsts[i]:
+            assert torch.equal(d, srcs[i])
+
+
 def test_launch_counter(ctx):
     a = ctx.launches()
     n = MiB
