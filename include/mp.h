@@ -300,6 +300,16 @@ int mp_get_host_duplex(mp_ctx *ctx, int gpu, double *kappa);
  * MP_ERR_UNSUPPORTED (world > 1), MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_TIMEOUT. */
 int mp_calibrate_window(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int window, int reps);
 
+/* mp_fit_window — the estimator of mp_calibrate_window on given samples (for parity):
+ * sample j of path[j] (0 <= path < npaths; path 0 = direct) has T1 = t1[j] (one message
+ * on an idle stream), TW = tw[j] (`window` >= 2 back-to-back messages) and the model's
+ * time pred[j] of one message.  *tau = max(0, median over path-0 samples of
+ * t1 − pred) (0 without one); h[i] = median over path i's samples of
+ * max(0, t1 − tau − (tw − t1)/(window − 1)) (0 without one); h has npaths entries.
+ * Medians of an even count take the upper middle value.  Errors: MP_ERR_INVALID. */
+int mp_fit_window(const int *path, const double *t1, const double *tw, const double *pred, int m,
+                  int window, int npaths, double *h, double *tau);
+
 /* ---------------------------------------------------------------- memory */
 
 /* Allocate / free device memory from this rank's registered heap.  A buffer that

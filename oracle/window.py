@@ -148,3 +148,22 @@ def select_flows_duplex(flows, pair_paths, pair_port, opts: M.Options, kappa) ->
                  for p in paths]
         out.append(M.select(n, paths, opts, port, m))
     return out
+
+
+# ----------------------------------------------------------------------------- C24 fit
+
+def fit_window(samples, window: int, npaths: int):
+    """The C24 estimator of Step 1 (mp_calibrate_window): samples = [(path, T1, TW, pred)]
+    with T1 one message on an idle stream, TW `window` back-to-back messages, pred the
+    model's one-message time.  τ = max(0, median(T1 − pred) over the direct path's
+    samples); h_i = median over path i's samples of max(0, T1 − τ − (TW − T1)/(W − 1))
+    (the serve-bound branch of W1: TW − T1 = (W − 1)·(T_i − a_i)).  Medians of an even
+    count take the upper middle value."""
+    from statistics import median_high
+    d = [t1 - pred for p, t1, _, pred in samples if p == 0]
+    tau = max(0.0, median_high(d)) if d else 0.0
+    h = []
+    for i in range(npaths):
+        a = [max(0.0, t1 - tau - (tw - t1) / (window - 1)) for p, t1, tw, _ in samples if p == i]
+        h.append(median_high(a) if a else 0.0)
+    return h, tau

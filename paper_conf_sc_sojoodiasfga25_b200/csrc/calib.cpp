@@ -735,24 +735,47 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
   CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
   if (derr) return cfail(c, MP_ERR_TIMEOUT, "window calibration transfer timed out");
   if (smp.empty()) return cfail(c, MP_ERR_INVALID, "no calibration sample fits the staging rings");
-  // τ is a property of the window (idle-stream launch + the host wait), the same for
-  // every config: read it off the direct path, which carries no staging-model error.
+  std::vector<int> sp;
+  std::vector<double> s1, sw, spred;
+  for (const Sample &sm : smp) {
+    sp.push_back(sm.path);
+    s1.push_back(sm.t1);
+    sw.push_back(sm.tw);
+    spred.push_back(sm.pred);
+  }
+  double h[MP_MAX_PATHS], tau = 0.0;
+  if (int e = mp_fit_window(sp.data(), s1.data(), sw.data(), spred.data(), static_cast<int>(smp.size()), window, np,
+                            h, &tau))
+    return cfail(c, e, "window fit failed");
+  if (int e = mp_set_window_model(c, 0, 0, h, np, tau)) return e;
+  if (int e = mp_set_host_duplex(c, c->rank, std::max(kappa, 1e-3))) return e;
+  return MP_OK;
+}
+
+// The C24 estimator of mp_calibrate_window on given samples (pure host arithmetic).
+// τ is a property of the window (idle-stream launch + the host wait), the same for
+// every config: it is read off the direct path (path 0), which carries no
+// staging-model error.  Per path, the steady per-message time s = (TW − T1)/(W − 1) =
+// max(a, T1 − τ − a), read in the serve-bound branch: a = T1 − τ − s.
+extern "C" int mp_fit_window(const int *path, const double *t1, const double *tw, const double *pred, int m,
+                             int window, int npaths, double *h, double *tau) {
+  if (!path || !t1 || !tw || !pred || !h || !tau || m < 1 || window < 2 || npaths < 1 || npaths > MP_MAX_PATHS)
+    return MP_ERR_INVALID;
   std::vector<double> taus;
-  for (const Sample &sm : smp)
-    if (sm.path == 0) taus.push_back(sm.t1 - sm.pred);
-  const double tau = taus.empty() ? 0.0 : std::max(0.0, median(taus));
-  double h[MP_MAX_PATHS];
-  for (int i = 0; i < np; ++i) {
+  for (int j = 0; j < m; ++j) {
+    if (path[j] < 0 || path[j] >= npaths || !(t1[j] > 0.0) || !(tw[j] > 0.0)) return MP_ERR_INVALID;
+    if (path[j] == 0) taus.push_back(t1[j] - pred[j]);
+  }
+  *tau = taus.empty() ? 0.0 : std::max(0.0, median(taus));
+  for (int i = 0; i < npaths; ++i) {
     std::vector<double> as;
-    for (const Sample &sm : smp)
-      if (sm.path == i) {
-        const double steady = (sm.tw - sm.t1) / static_cast<double>(window - 1);
-        as.push_back(std::max(0.0, sm.t1 - tau - steady));
+    for (int j = 0; j < m; ++j)
+      if (path[j] == i) {
+        const double steady = (tw[j] - t1[j]) / static_cast<double>(window - 1);
+        as.push_back(std::max(0.0, t1[j] - *tau - steady));
       }
     h[i] = as.empty() ? 0.0 : median(as);
   }
-  if (int e = mp_set_window_model(c, 0, 0, h, np, tau)) return e;
-  if (int e = mp_set_host_duplex(c, c->rank, std::max(kappa, 1e-3))) return e;
   return MP_OK;
 }
 

@@ -169,6 +169,9 @@ def lib():
                                            C.POINTER(mp_config)]),
             "mp_set_host_duplex": (C.c_int, [P, C.c_int, C.c_double]),
             "mp_calibrate_window": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int, C.c_int]),
+            "mp_fit_window": (C.c_int, [C.POINTER(C.c_int), C.POINTER(C.c_double), C.POINTER(C.c_double),
+                                        C.POINTER(C.c_double), C.c_int, C.c_int, C.c_int, C.POINTER(C.c_double),
+                                        C.POINTER(C.c_double)]),
             "mp_get_host_duplex": (C.c_int, [P, C.c_int, C.POINTER(C.c_double)]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
@@ -191,7 +194,7 @@ def exported_symbols() -> List[str]:
             "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands",
             "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
-            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window"]
+            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_fit_window"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -202,6 +205,18 @@ def fit_hockney(n: Sequence[float], t: Sequence[float]):
     if st != 0:
         raise MPError(st, "mp_fit_hockney")
     return a.value, b.value
+
+
+def fit_window(path: Sequence[int], t1: Sequence[float], tw: Sequence[float], pred: Sequence[float],
+               window: int, npaths: int):
+    """mp_fit_window: (h[npaths], τ) of the C24 estimator (NEXT f2)."""
+    m = len(path)
+    h, tau = (C.c_double * max(1, npaths))(), C.c_double()
+    st = lib().mp_fit_window((C.c_int * m)(*path), (C.c_double * m)(*t1), (C.c_double * m)(*tw),
+                             (C.c_double * m)(*pred), m, window, npaths, h, C.byref(tau))
+    if st != 0:
+        raise MPError(st, "mp_fit_window")
+    return [h[i] for i in range(npaths)], tau.value
 
 
 def fit_bands(n: Sequence[float], t: Sequence[float], edges: Sequence[float]):

@@ -267,3 +267,51 @@ def test_duplex_shares_never_oversubscribe_a_duplex_link(seed):
             k = kappa[g] if g in other else 1.0
             # every user's rate is at most κ·β / (number of users); Σ <= κ·max β
             assert sum(r for r, _ in users) <= k * max(b for _, b in users) * (1 + 1e-9)
+
+
+# ------------------------------------------------------------------ C24 Step-1 fit
+
+def window_samples(paths, h, tau, W, sizes):
+    """Noiseless samples from (W1): each path alone carrying n bytes."""
+    out = []
+    opts = M.Options(stagger=False)
+    for i, p in enumerate(paths):
+        for n in sizes:
+            nb = [0] * len(paths)
+            nb[i] = n
+            ks = [1 if j == 0 else (8 if j == i else 0) for j in range(len(paths))]
+            pred = M.evaluate(n, nb, ks, paths, opts)
+            t1 = WN.evaluate_window(n, 1, nb, ks, paths, h, opts, None, tau)
+            tw = WN.evaluate_window(n, W, nb, ks, paths, h, opts, None, tau)
+            out.append((i, t1, tw, pred))
+    return out
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_window_fit_recovers_h_and_tau_in_the_serve_bound_regime(seed):
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    rng = random.Random(seed)
+    paths = paths_from(synth.topology(seed, 2, True))
+    h = [rng.uniform(0, 1) * p.alpha for p in paths]
+    tau = rng.uniform(0, 10) * US
+    smp = window_samples(paths, h, tau, 16, [4 * MiB, 16 * MiB, 64 * MiB])
+    got_h, got_tau = WN.fit_window(smp, 16, len(paths))
+    assert abs(got_tau - tau) < 1e-15
+    for a, b in zip(got_h, h):
+        assert abs(a - b) < 1e-15
+    # the library's estimator on the same samples
+    lh, lt = mp.fit_window([s[0] for s in smp], [s[1] for s in smp], [s[2] for s in smp],
+                           [s[3] for s in smp], 16, len(paths))
+    assert abs(lt - got_tau) <= 1e-18 and all(abs(a - b) <= 1e-18 for a, b in zip(lh, got_h))
+
+
+def test_window_fit_reads_the_serve_bound_branch():
+    # Issue-bound samples (a > T − a) are ambiguous under W1 (TW − T1 = (W−1)·a): the
+    # estimator reads the serve-bound branch and returns the mirror T − a.
+    p = M.Path(M.DIRECT, 10 * US, 1e12)
+    n = 1 << 20                                       # T = 10 µs + 1.05 µs
+    t = p.alpha + n / p.beta
+    a = 9 * US
+    smp = [(0, t, WN.path_window_time(t, a, 8), t)]
+    h, tau = WN.fit_window(smp, 8, 1)
+    assert tau == 0.0 and abs(h[0] - (t - a)) < 1e-15
