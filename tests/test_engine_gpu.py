@@ -403,3 +403,31 @@ def test_loopback_collectives_are_local_copies(ctx):
     ctx.allreduce(x, y, 1000, mp.MP_DT_F32)
     ctx.sync()
     assert torch.equal(x, y)
+
+
+def test_message_beyond_4_gib_all_path_kinds(ctx):
+    # Offsets past 2^32 on every path kind: a 4 GiB + 4099-byte message over the direct
+    # path, one relay ring and the host ring (O1: dst == src byte for byte, canaries on
+    # both sides intact).
+    n = (4 << 30) + 4099
+    g = torch.Generator("cuda").manual_seed(20251116)
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g)
+    dst_full = torch.full((n + 2 * CAN,), 0xA5, dtype=torch.uint8, device="cuda")
+    dst = dst_full[CAN:CAN + n]
+    ps = ctx.paths()
+    nb = [0] * len(ps)
+    nb[1], nb[-1] = 64 * MiB, 16 * MiB
+    nb[0] = n - sum(nb)
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1], ks[-1] = 32, 8
+    ctx.xfer(dst, src, n, ctx.make_config(nb, ks), torch.cuda.current_stream())
+    ctx.sync()
+    assert torch.equal(dst, src)
+    assert bool((dst_full[:CAN] == 0xA5).all()) and bool((dst_full[CAN + n:] == 0xA5).all())
+    # the same message direct-only through the model-selected path (one fused launch)
+    dst.zero_()
+    ctx.xfer(dst, src, n, None, torch.cuda.current_stream())
+    ctx.sync()
+    assert torch.equal(dst, src)
+    del src, dst, dst_full
+    torch.cuda.empty_cache()
