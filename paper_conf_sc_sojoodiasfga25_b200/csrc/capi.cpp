@@ -224,6 +224,7 @@ int init_engine(mp_ctx *c) {
     return cuda_fail(c, static_cast<cudaError_t>(e), "occupancy query");
   if (int e = preload_kernels()) return cuda_fail(c, static_cast<cudaError_t>(e), "kernel preload");
   if (const char *m = std::getenv("MPX_COPY")) c->copy_mode = std::strcmp(m, "reg") == 0 ? 0u : 1u;
+  if (const char *m = std::getenv("MPX_PDL")) c->pdl = std::strcmp(m, "0") == 0 ? 0u : 1u;
   void *p = nullptr;
   CK(cudaMalloc(&p, sizeof(int32_t)));
   c->d_err = static_cast<int32_t *>(p);
@@ -256,6 +257,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.err = c->d_err;
   P.copy_mode = c->copy_mode;
+  P.pdl = c->pdl;
   P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
   P.allow_small = 1;
   const int cap = std::max(1, c->per_sm * c->sms);
@@ -264,7 +266,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
     if (cfg.bytes[i]) staged_ctas += 2u * static_cast<uint32_t>(c->relay_ctas);
   // direct group sized by direct_ctas(), leaving room for every staged group to be
   // co-resident.
-  uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas));
+  uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas), c->pdl != 0);
   // Two large copies running at once (osu_bibw's two directions on two streams) do
   // best with one TMA pipeline per SM each — 64 KiB in flight per SM in total, as one
   // copy with two (profiles/r01/bibw.jsonl).  A large direct-only launch that finds
@@ -343,6 +345,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   P.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
   P.err = c->d_err;
   P.copy_mode = c->copy_mode;
+  P.pdl = c->pdl;
   P.bulk_stages = bulk_stages_for(n);
   P.allow_small = ctas > 0 ? 0u : 1u;  // a staged leg's calibration times its group's CTAs
   P.npaths = 1;
@@ -352,7 +355,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   d.src = static_cast<const uint8_t *>(src);
   d.dst = static_cast<uint8_t *>(dst);
   d.align = c->opts.align;
-  d.g_in = ctas > 0 ? static_cast<uint32_t>(ctas) : direct_ctas(c, n, c->per_sm * c->sms);
+  d.g_in = ctas > 0 ? static_cast<uint32_t>(ctas) : direct_ctas(c, n, c->per_sm * c->sms, c->pdl != 0);
   P.nblocks = d.g_in;
   const int e = launch_xfer(P, stream);
   if (e != cudaSuccess) return cuda_fail(c, static_cast<cudaError_t>(e), "copy launch");

@@ -92,6 +92,7 @@ struct mp_ctx {
   uint64_t slot_bytes = 32ull << 20;
   double timeout_s = 20.0;
   int per_sm = 0, sms = 0;
+  uint32_t pdl = 1;                // loopback launches use PDL (env MPX_PDL=0: off)
   uint32_t copy_mode = 1;          // direct-path copy: 1 = TMA bulk, 0 = LDG/STG (env MPX_COPY=reg)
   int32_t *d_err = nullptr;
   std::vector<mpx::Ring> rings;   // loopback: [0..V) relays, [V] host (if enabled)
@@ -154,11 +155,15 @@ namespace mpx {
 inline uint32_t bulk_stages_for(uint64_t /*bytes*/) { return 4u; }
 
 // CTAs of a direct group: one per 32 KiB, at most 2 per SM (TMA) or 4 per SM
-// (LDG/STG), and at most `room` (what is left of the co-resident capacity).
-inline uint32_t direct_ctas(const mp_ctx *c, uint64_t bytes, int room) {
-  const uint64_t want = bytes ? (bytes + (32u << 10) - 1) / (32u << 10) : 1;
+// (LDG/STG), and at most `room` (what is left of the co-resident capacity).  With PDL
+// (full_grid: loopback launches) a TMA group always takes the full 2 per SM: a grid that is not a multiple of the SM
+// count lands unevenly on the SMs its predecessor still occupies (8 MiB, 256 CTAs:
+// 5.2 µs per back-to-back message vs 3.1 µs with 296; scripts/pdlbench.cu).
+inline uint32_t direct_ctas(const mp_ctx *c, uint64_t bytes, int room, bool full_grid = false) {
+  uint64_t want = bytes ? (bytes + (32u << 10) - 1) / (32u << 10) : 1;
   const int per_sm = c->copy_mode == 1 ? 2 : 4;
   const int lim = std::max(1, std::min(room, per_sm * c->sms));
+  if (full_grid && c->copy_mode == 1) want = static_cast<uint64_t>(lim);
   return static_cast<uint32_t>(std::min<uint64_t>(want, static_cast<uint64_t>(lim)));
 }
 

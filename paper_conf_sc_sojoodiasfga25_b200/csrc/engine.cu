@@ -14,6 +14,8 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <utility>
+
 #include "engine.h"
 
 namespace mpx {
@@ -336,6 +338,16 @@ __device__ __forceinline__ void slice_of(uint64_t len, uint32_t r, uint32_t G, u
   *b = e;
 }
 
+// Programmatic dependent launch (PDL): let the stream's next kernel launch now (its
+// CTAs become resident while this one runs), then wait until the stream's previous
+// kernel has completed and its memory operations are visible.  Back-to-back messages
+// (an OMB window, reading C24) then pay no launch gap.  Both instructions are no-ops
+// for a kernel launched without the attribute.
+__device__ __forceinline__ void pdl_enter() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+
 // ------------------------------------------------------------------ roles
 
 __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
@@ -371,6 +383,7 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
 
 __global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant__ XferParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
+  pdl_enter();
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
@@ -755,6 +768,7 @@ struct DirectArgs {
 
 __global__ void __launch_bounds__(kThreads, 4) direct_kernel(const __grid_constant__ DirectArgs A) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
+  pdl_enter();
   bulk_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
 }
 
@@ -763,6 +777,7 @@ __global__ void __launch_bounds__(kThreads, 4) direct_kernel(const __grid_consta
 // branch-light on purpose: at these sizes a launch on a cold SM is bound by its
 // instruction fetches, not by the bytes.
 __global__ void __launch_bounds__(kThreads) direct_small_kernel(uint8_t *dst, const uint8_t *src, uint64_t n) {
+  pdl_enter();
   uint64_t head = (16u - (reinterpret_cast<uintptr_t>(src) & 15u)) & 15u;
   if (head > n) head = n;
   const uint64_t nvec = (n - head) >> 4;
@@ -779,6 +794,7 @@ __global__ void __launch_bounds__(kThreads) direct_small_kernel(uint8_t *dst, co
 // LDG/STG direct copy (MPX_COPY=reg): no min-blocks bound, so the 4-deep unrolled
 // vector loop gets the registers it needs (a 64-register cap made it spill).
 __global__ void __launch_bounds__(kThreads) direct_reg_kernel(const __grid_constant__ DirectArgs A) {
+  pdl_enter();
   group_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x);
 }
 
@@ -848,8 +864,27 @@ int launch_reduce(int dtype, void *dst, const void *src, uint64_t bytes, void *s
   return static_cast<int>(cudaGetLastError());
 }
 
+namespace {
+// <<<>>> with the PDL attribute when asked (cudaLaunchKernelEx).
+template <typename... KArgs, typename... Args>
+int launch_k(bool pdl, void (*kern)(KArgs...), uint32_t grid, uint32_t smem, void *stream, Args &&...args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = static_cast<cudaStream_t>(stream);
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return static_cast<int>(cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...));
+}
+}  // namespace
+
 int launch_xfer(const XferParams &P, void *stream) {
   if (P.nblocks == 0) return cudaSuccess;
+  const bool pdl = P.pdl != 0;
   bool direct_only = P.p[0].kind == DK_DIRECT && P.p[0].cta0_in == 0 && P.p[0].g_in == P.nblocks;
   for (uint32_t i = 1; i < P.npaths; ++i)
     if (P.p[i].bytes) direct_only = false;
@@ -857,20 +892,15 @@ int launch_xfer(const XferParams &P, void *stream) {
       ((reinterpret_cast<uintptr_t>(P.p[0].dst) ^ reinterpret_cast<uintptr_t>(P.p[0].src)) & 15u) == 0) {
     const uint64_t nvec = P.p[0].bytes >> 4;
     const uint32_t g = static_cast<uint32_t>(nvec ? (nvec + kThreads - 1) / kThreads : 1);
-    direct_small_kernel<<<g, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P.p[0].dst, P.p[0].src,
-                                                                               P.p[0].bytes);
-    return static_cast<int>(cudaGetLastError());
+    return launch_k(pdl, direct_small_kernel, g, 0, stream, P.p[0].dst, static_cast<const uint8_t *>(P.p[0].src),
+                    P.p[0].bytes);
   }
   if (direct_only) {
     const DirectArgs A{P.p[0].dst, P.p[0].src, P.p[0].bytes, P.copy_mode, P.bulk_stages};
-    if (P.copy_mode == 1)
-      direct_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(A);
-    else
-      direct_reg_kernel<<<P.nblocks, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(A);
-    return static_cast<int>(cudaGetLastError());
+    if (P.copy_mode == 1) return launch_k(pdl, direct_kernel, P.nblocks, kBulkSmem, stream, A);
+    return launch_k(pdl, direct_reg_kernel, P.nblocks, 0, stream, A);
   }
-  xfer_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
-  return static_cast<int>(cudaGetLastError());
+  return launch_k(pdl, xfer_kernel, P.nblocks, kBulkSmem, stream, P);
 }
 
 int launch_send(const SendParams &P, void *stream) {

@@ -53,7 +53,7 @@ struct XferParams {
   uint32_t copy_mode;    // direct group: 0 = LDG/STG vectors, 1 = TMA bulk (cp.async.bulk)
   uint32_t bulk_stages;  // TMA pipeline depth per CTA (1..4)
   uint32_t allow_small;  // 1: a small direct-only message may use the one-shot kernel
-  uint32_t pad_;
+  uint32_t pdl;          // 1: launched with programmatic stream serialization (PDL)
   uint64_t timeout_ns;
   int32_t *err;          // device (or mapped host) error word
   DevPath p[kMaxPaths];
@@ -64,7 +64,7 @@ struct XferParams {
 // straight-line code (profiles/r01/smallbench*.jsonl: 2.1-3.1 µs per back-to-back
 // message vs 4.1 µs for the TMA pipeline kernel, whose cold instruction fetches
 // dominate at these sizes).
-constexpr uint64_t kSmallMax = 1ull << 20;
+constexpr uint64_t kSmallMax = 4ull << 20;
 
 // Launch the fused transfer kernel (engine.cu).  Returns a cudaError_t value.
 int launch_xfer(const XferParams &P, void *stream);
