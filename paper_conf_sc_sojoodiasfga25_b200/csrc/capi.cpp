@@ -922,13 +922,13 @@ int mp_xfer(mp_ctx *c, void *dst, const void *src, uint64_t bytes, const mp_conf
   // CUDA-graph capture: a direct-only transfer is a pure kernel and replays
   // correctly; a staged one advances the rings' sequence numbers on the host at
   // launch, which a replay would not repeat, so it is refused while capturing.
+  // (only staged configs need the query: it costs host time on every small message)
+  bool staged = false;
+  for (int i = 1; i < cfg->npaths; ++i) staged = staged || cfg->bytes[i] != 0;
   cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
-  if (cudaStreamIsCapturing(static_cast<cudaStream_t>(stream), &cap) == cudaSuccess &&
-      cap != cudaStreamCaptureStatusNone) {
-    for (int i = 1; i < cfg->npaths; ++i)
-      if (cfg->bytes[i])
-        return fail(c, MP_ERR_UNSUPPORTED, "staged paths cannot be captured in a CUDA graph (direct-only can)");
-  }
+  if (staged && cudaStreamIsCapturing(static_cast<cudaStream_t>(stream), &cap) == cudaSuccess &&
+      cap != cudaStreamCaptureStatusNone)
+    return fail(c, MP_ERR_UNSUPPORTED, "staged paths cannot be captured in a CUDA graph (direct-only can)");
   return launch_loopback(c, dst, src, bytes, *cfg, stream);
 }
 
