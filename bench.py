@@ -663,7 +663,9 @@ def main():
                      "frac": achieved / peak, "traffic": traffic,
                      "peak_source": peak_src,
                      "kernel": "direct_kernel" if all(b == 0 for b in d["bytes"][1:]) else "xfer_kernel",
-                     "algorithmic_bytes_per_launch": alg},
+                     "algorithmic_bytes_per_launch": alg,
+                     "note": "achieved = algorithmic bytes / (timed region / steps); the peak is "
+                             "torch copy_ timed alone, this kernel runs back to back under PDL"},
         "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n, "d2h_bytes_per_step": n},
         "gpu_launches": launches,
         "clocks": clk.summary(),
