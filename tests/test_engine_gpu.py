@@ -431,3 +431,28 @@ def test_message_beyond_4_gib_all_path_kinds(ctx):
     assert torch.equal(dst, src)
     del src, dst, dst_full
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("n", [4096 + 16, 3 * MiB, 64 * MiB + 256])
+def test_back_to_back_dependent_chain(ctx, n):
+    # PDL: each launch lets its successor start early, and the successor
+    # waits (griddepcontrol.wait) before touching memory.  A chain in which every
+    # message reads what the previous one wrote — b0 → b1 → … → b8, back to back on one
+    # stream, no sync in between — arrives intact only if that wait holds.  The
+    # middle link is a staged config (relay + host rings).
+    g = torch.Generator("cuda").manual_seed(n)
+    bufs = [torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g)]
+    bufs += [torch.zeros(n, dtype=torch.uint8, device="cuda") for _ in range(8)]
+    ps = ctx.paths()
+    nb = [0] * len(ps)
+    nb[1] = nb[-1] = (n // 4) // 256 * 256
+    nb[0] = n - nb[1] - nb[-1]
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1] = ks[-1] = max(2, -(-nb[1] // (2 * MiB)))   # chunks fit the fixture's 4 MiB slots
+    staged = ctx.make_config(nb, ks) if nb[1] >= 64 * 1024 else None
+    s = torch.cuda.current_stream()
+    torch.cuda.synchronize()
+    for i in range(8):
+        ctx.xfer(bufs[i + 1], bufs[i], n, staged if i == 4 else None, s)
+    ctx.sync()
+    assert torch.equal(bufs[8], bufs[0])
