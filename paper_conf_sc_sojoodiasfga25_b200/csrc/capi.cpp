@@ -225,6 +225,9 @@ int init_engine(mp_ctx *c) {
   if (int e = preload_kernels()) return cuda_fail(c, static_cast<cudaError_t>(e), "kernel preload");
   if (const char *m = std::getenv("MPX_COPY")) c->copy_mode = std::strcmp(m, "reg") == 0 ? 0u : 1u;
   if (const char *m = std::getenv("MPX_PDL")) c->pdl = std::strcmp(m, "0") == 0 ? 0u : 1u;
+  // multi-rank PDL is opt-in: with both ranks on one GPU under MPS it cost 10-18 % on
+  // direct messages of 1-16 MiB (profiles/r01/world_pdl); unmeasured across GPUs
+  if (const char *m = std::getenv("MPX_PDL_WORLD")) c->pdl_world = std::strcmp(m, "1") == 0 ? 1u : 0u;
   void *p = nullptr;
   CK(cudaMalloc(&p, sizeof(int32_t)));
   c->d_err = static_cast<int32_t *>(p);

@@ -93,6 +93,7 @@ struct mp_ctx {
   double timeout_s = 20.0;
   int per_sm = 0, sms = 0;
   uint32_t pdl = 1;                // loopback launches use PDL (env MPX_PDL=0: off)
+  uint32_t pdl_world = 0;          // multi-rank launches use PDL (env MPX_PDL_WORLD=1: on)
   uint32_t copy_mode = 1;          // direct-path copy: 1 = TMA bulk, 0 = LDG/STG (env MPX_COPY=reg)
   int32_t *d_err = nullptr;
   std::vector<mpx::Ring> rings;   // loopback: [0..V) relays, [V] host (if enabled)

@@ -498,7 +498,12 @@ __device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t
 // send kernel on the same stream: the bulk kernel's hundreds of CTAs are only
 // dispatched once the receiver's clear-to-send has arrived, so they never occupy SM
 // slots spinning on it while a receive kernel on this GPU waits for room to run.
+// PDL in the multi-rank engine: the gate waits for the stream's previous kernel, and
+// lets the bulk send kernel launch only once the clear-to-send has arrived (no bulk
+// CTA is ever resident during the rendezvous); send, receive and eager kernels let
+// their successor launch at once and wait for their predecessor (pdl_enter).
 __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   if (threadIdx.x != 0) return;
   MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
   const uint64_t t_start = globaltimer();
@@ -531,10 +536,12 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
   h->f = reinterpret_cast<uintptr_t>(P.src + host_off) & 15u;
   st_release_sys(&h->seq1, P.seq + 1);
   if (bad) atomicExch(P.err, DERR_MISMATCH);
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
 __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant__ SendParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
+  pdl_enter();
   __shared__ int s_abort;
   __shared__ uint64_t s_off, s_region;
   __shared__ uint8_t *s_dst;
@@ -613,6 +620,7 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
 
 __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant__ RecvParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
+  pdl_enter();
   __shared__ int s_abort;
   __shared__ uint64_t s_k, s_q0, s_hoff, s_hbytes, s_shift;
   if (threadIdx.x == 0) s_abort = 0;
@@ -708,6 +716,7 @@ __global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constan
 // header words 0/1 = bytes/tag (CTA 0), 16 + r = source shift of CTA r's slice, 8 + r =
 // CTA r's sequence flag (seq + 1, released after its slice).
 __global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_constant__ EagerParams P) {
+  pdl_enter();
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
@@ -733,6 +742,7 @@ __global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_const
 }
 
 __global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_constant__ EagerParams P) {
+  pdl_enter();
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
@@ -904,24 +914,30 @@ int launch_xfer(const XferParams &P, void *stream) {
 }
 
 int launch_send(const SendParams &P, void *stream) {
-  send_gate_kernel<<<1, 32, 0, static_cast<cudaStream_t>(stream)>>>(P);
-  send_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
-  return static_cast<int>(cudaGetLastError());
+  const bool pdl = P.pdl != 0;
+  cudaLaunchConfig_t cfg = {};  // the gate is one warp
+  cfg.gridDim = dim3(1);
+  cfg.blockDim = dim3(32);
+  cfg.stream = static_cast<cudaStream_t>(stream);
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
+  if (int e = static_cast<int>(cudaLaunchKernelEx(&cfg, send_gate_kernel, P))) return e;
+  return launch_k(pdl, send_kernel, P.nblocks, kBulkSmem, stream, P);
 }
 
 int launch_eager_send(const EagerParams &P, void *stream) {
-  eager_send_kernel<<<P.ctas, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
-  return static_cast<int>(cudaGetLastError());
+  return launch_k(P.pdl != 0, eager_send_kernel, P.ctas, 0, stream, P);
 }
 
 int launch_eager_recv(const EagerParams &P, void *stream) {
-  eager_recv_kernel<<<P.ctas, kThreads, 0, static_cast<cudaStream_t>(stream)>>>(P);
-  return static_cast<int>(cudaGetLastError());
+  return launch_k(P.pdl != 0, eager_recv_kernel, P.ctas, 0, stream, P);
 }
 
 int launch_recv(const RecvParams &P, void *stream) {
-  recv_kernel<<<P.nblocks, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
-  return static_cast<int>(cudaGetLastError());
+  return launch_k(P.pdl != 0, recv_kernel, P.nblocks, kBulkSmem, stream, P);
 }
 
 int launch_relay(const RelayParams &P, void *stream) {

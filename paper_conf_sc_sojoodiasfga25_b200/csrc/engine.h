@@ -155,7 +155,7 @@ struct SendParams {
   CtrlLayout L;
   uint64_t host_stride;
   uint32_t host_slots;
-  uint32_t pad_;
+  uint32_t pdl;          // 1: launched with programmatic stream serialization (PDL)
   struct StagedDesc {
     int32_t kind;            // 1 relay, 2 host
     uint32_t relay;          // relay rank
@@ -179,7 +179,7 @@ struct RecvParams {
   CtrlLayout L;
   uint64_t host_stride;
   uint32_t host_slots;
-  uint32_t pad_;
+  uint32_t pdl;          // 1: launched with programmatic stream serialization (PDL)
   HostRingPtrs host;
 };
 
@@ -204,6 +204,7 @@ struct EagerParams {
   uint64_t *free_ctr;        // eager_free word of the pair (sender's control block)
   uint32_t *cnt;             // recv: eager_cnt word of the slot (receiver-local)
   int32_t *err;
+  uint32_t pdl;              // 1: launched with programmatic stream serialization (PDL)
 };
 
 int launch_send(const SendParams &P, void *stream);

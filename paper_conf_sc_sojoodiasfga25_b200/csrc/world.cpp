@@ -330,6 +330,7 @@ static EagerParams eager_params(mp_ctx *c, int sender, int receiver, uint64_t se
   P.cnt = reinterpret_cast<uint32_t *>(c->peers[receiver].ctrl + c->L.eager_cnt) +
           static_cast<uint64_t>(sender) * kEagerSlots + slot;
   P.err = c->d_err;
+  P.pdl = c->pdl_world;
   return P;
 }
 
@@ -376,6 +377,7 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   P.host_slots = static_cast<uint32_t>(c->slots);
   P.g_stage = static_cast<uint32_t>(c->relay_ctas);
   P.copy_mode = c->copy_mode;
+  P.pdl = c->pdl_world;
   P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
   if (c->host_path) P.host = host_ring(c, c->rank, dst);
   P.direct_bytes = cfg.bytes[0];
@@ -470,6 +472,7 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   P.host_slots = static_cast<uint32_t>(c->slots);
   P.g_host = c->host_path ? static_cast<uint32_t>(c->relay_ctas) : 0u;
   P.copy_mode = c->copy_mode;
+  P.pdl = c->pdl_world;
   P.bulk_stages = bulk_stages_for(bytes);
   if (c->host_path) P.host = host_ring(c, src, c->rank);
   P.nblocks = 1 + P.g_host;

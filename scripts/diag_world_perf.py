@@ -24,7 +24,7 @@ def main():
     dev = 0 if os.environ.get("MPX_BENCH_SAME_GPU") == "1" else int(os.environ.get("LOCAL_RANK", 0))
     torch.cuda.set_device(dev)
     n = int(os.environ.get("DIAG_BYTES", 64 * MiB))
-    K = 20
+    K = int(os.environ.get("DIAG_K", "20"))
     s = torch.cuda.Stream()
     src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()

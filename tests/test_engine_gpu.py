@@ -294,21 +294,27 @@ def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
     c = mp.Context(device=0, n_loop_relays=2, host_path=1, slot_bytes=32 * MiB, heap_bytes=16 * MiB)
     c.set_options(mode=mp.MP_MODEL_B200)
     c.calibrate(reps=3)
-    # sizes where a window of transfers is GPU-bound (not bound by the Python loop)
     sizes = [16 * MiB, 32 * MiB, 48 * MiB]
     src = torch.randint(0, 256, (48 * MiB,), dtype=torch.uint8, device="cuda")
     dst = torch.empty_like(src)
     s = torch.cuda.Stream()
 
     def window_time(n, cfg, w=16, reps=5):
+        # the window is captured in a CUDA graph so that it is GPU-bound: under PDL a
+        # back-to-back 16 MiB message takes ~4 µs, about one Python-loop iteration
+        assert sum(cfg.as_dict()["bytes"][1:]) == 0, "B200 mode picks direct-only here"
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(w):
+                c.xfer(dst, src, n, cfg, torch.cuda.current_stream())
         ts = []
         for _ in range(reps + 1):
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
-            e0.record(s)
-            for _ in range(w):
-                c.xfer(dst, src, n, cfg, s)
-            e1.record(s)
+            with torch.cuda.stream(s):
+                e0.record(s)
+                g.replay()
+                e1.record(s)
             e1.synchronize()
             ts.append(e0.elapsed_time(e1) * 1e-3 / w)
         return sorted(ts[1:])[reps // 2]
