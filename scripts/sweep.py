@@ -37,6 +37,11 @@ def measure(ctx, dst, src, n, cfg, reps, stream):
     for r in range(reps + 1):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
+        # a ~100 µs spin kernel first, so that the whole window is enqueued before the
+        # GPU reaches it: the window is then timed at GPU speed, not at the Python
+        # loop's (a back-to-back 16 MiB message takes ~4 µs under PDL)
+        with torch.cuda.stream(stream):
+            torch.cuda._sleep(200_000)
         e0.record(stream)
         for _ in range(W):
             ctx.xfer(dst, src, n, cfg, stream)
