@@ -577,10 +577,15 @@ def main():
         gbs = nstage / t / 1e9
         if name.startswith("relay"):
             # a staged path is two stage groups of relay_ctas (16) CTAs each, sized for
-            # a relay's NVLink share beside the direct group, not for loopback HBM
+            # a relay's NVLink share beside the direct group, not for loopback HBM: its
+            # ceiling is the slower leg as Step 1 measured it with that group
+            # (calibrated β, β' of the path)
+            lp = ctx.get_model(0, 0)[1][idx]
+            ceil_ = min(lp["beta"], lp["beta2"]) / 1e9
             per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "hbm",
                               "hbm_GBps": 4 * nstage / t / 1e9, "frac": 4 * nstage / t / 1e9 / peak,
-                              "ctas": 32, "hbm_GBps_per_cta": 4 * nstage / t / 1e9 / 32}
+                              "ctas": 32, "hbm_GBps_per_cta": 4 * nstage / t / 1e9 / 32,
+                              "stage_group_ceiling_GBps": ceil_, "frac_of_stage_group_ceiling": gbs / ceil_}
         else:
             per_path[name] = {"GBps": gbs, "bytes": nstage, "chunks": 16, "bound": "pcie",
                               "peak": 64.0, "frac": gbs / 64.0,
