@@ -163,3 +163,51 @@ def test_select_flows_duplex_parity(seed, mode):
             assert rel(gd["t_level"], r.t_level) < 1e-9
             if gd["bytes"] == r.bytes:
                 assert gd["chunks"] == r.chunks and rel(gd["t_pred"], r.t_pred) < 1e-9
+
+
+@pytest.mark.parametrize("mode", [M.PAPER, M.B200])
+def test_window_model_applies_to_every_size_band(mode):
+    # C24 with C20: the pair's h and τ hold for every band; a_i = min(h_i, α_i) takes
+    # the α of n's band (oracle: oracle/bands.band_index + oracle/window.select_window).
+    from oracle import bands as OB
+    rng = random.Random(7)
+    base = [M.Path(**t) for t in table(0, 1, 11)]
+    scaled = [M.Path(**{**t, "alpha": t["alpha"] * 0.3, "alpha2": t["alpha2"] * 0.3}) for t in table(0, 1, 11)]
+    bands = [(0, scaled, M.Port(1e-6, 8e11)), (16 * MiB, base, M.Port(3e-6, 9e11))]
+    h = [rng.uniform(0.2, 1.2) * p.alpha for p in base]
+    tau = 2e-6
+    opts = M.Options(mode=mode, slot_bytes=64 * MiB)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.set_options(mode=mode, slot_bytes=64 * MiB)
+        install(c, 0, 1, table(0, 1, 11), None)
+        prm = [{k: (0.0 if k == "beta2" and math.isinf(getattr(p, k)) else getattr(p, k)) for k in FIELDS}
+               for p in scaled]
+        c.set_model(0, 1, [(p.kind, p.via) for p in scaled], prm, dict(alpha=1e-6, beta=8e11))
+        prm = [{k: (0.0 if k == "beta2" and math.isinf(getattr(p, k)) else getattr(p, k)) for k in FIELDS}
+               for p in base]
+        c.set_model_band(0, 1, 16 * MiB, prm, dict(alpha=3e-6, beta=9e11))
+        c.set_window_model(0, 1, h, tau)
+        for n in (4 * MiB, 16 * MiB - 256, 16 * MiB, 256 * MiB):
+            j = OB.band_index([b[0] for b in bands], n)
+            _, ps, port = bands[j]
+            for w in (1, 8):
+                ref = WN.select_window(n, w, ps, h, opts, port, tau=tau)
+                got = c.select_window(0, 1, n, w).as_dict()
+                for a, b in zip(got["bytes"], ref.bytes):
+                    assert abs(a - b) <= 256
+                assert rel(got["t_level"], ref.t_level) < 1e-9
+                if got["bytes"] == ref.bytes:
+                    assert rel(got["t_pred"], ref.t_pred) < 1e-9
+
+
+def test_predict_window_rejects_bad_configs():
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        n = 8 * MiB
+        ps = c.paths(0, 1)
+        bad = c.make_config([n - 1] + [0] * (len(ps) - 1), [1] + [0] * (len(ps) - 1), 0, 1)
+        with pytest.raises(mp.MPError):
+            c.predict_window(0, 1, n, 4, bad)                   # bytes do not sum to n
+        ok = c.make_config([n] + [0] * (len(ps) - 1), [1] + [0] * (len(ps) - 1), 0, 1)
+        with pytest.raises(mp.MPError):
+            c.predict_window(0, 1, n, 0, ok)                    # window 0
+        assert c.predict_window(0, 1, n, 4, ok) == pytest.approx(4 * c.predict(0, 1, n, ok), rel=1e-12)
