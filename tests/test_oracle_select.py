@@ -159,3 +159,19 @@ def test_mask_excludes_paths():
     paths = paths_from(synth.topology(11, 2, host=True))
     cfg = M.select(512 * MiB, paths, M.Options(), path_mask=[True, False, True, False])
     assert cfg.bytes[1] == 0 and cfg.bytes[3] == 0 and cfg.bytes[2] > 0
+
+
+@settings(max_examples=40, deadline=None)
+@given(st.integers(0, 10_000), st.integers(1, 6), st.integers(16, 2048).map(lambda m: m * MiB),
+       st.floats(400, 1200))
+def test_b200_prediction_never_exceeds_the_port_plus_unported_paths(seed, nrel, n, port_gbs):
+    # C14: every NVLink path (w = 1) leaves through the same egress port, so no
+    # B200-mode prediction exceeds β_port plus the rates of the paths that bypass it
+    # (the host path, w = 0: at most its slower leg).  The paper's private-link model
+    # has no such bound, and the NVSwitch case is where it breaks.
+    paths = paths_from(synth.topology(seed, nrel, host=True))
+    port = M.Port(alpha=2 * US, beta=port_gbs * GBS)
+    cfg = M.select(n, paths, M.Options(mode=M.B200, slot_bytes=64 * MiB), port)
+    h = paths[-1]
+    bound = port.beta + min(h.beta, h.beta2)
+    assert n / cfg.t_pred <= bound * (1 + 1e-9)
