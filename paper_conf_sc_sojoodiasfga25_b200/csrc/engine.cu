@@ -260,6 +260,14 @@ __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, ui
         why = 1;
         break;
       }
+      // fail fast: once any wait of this context has failed (sticky error word), the
+      // flags this CTA waits for may never come — abort now instead of timing out in
+      // turn behind it (the persistent relay, which passes `stop`, keeps serving)
+      if (!stop && (it & 63u) == 63u &&
+          __any_sync(0xffffffffu, lane == 0 && *reinterpret_cast<volatile int32_t *>(err) != 0)) {
+        why = 3;
+        break;
+      }
       if (stop && (it & 255u) == 255u && *stop) {
         why = 2;
         break;
@@ -280,9 +288,13 @@ __device__ __forceinline__ bool wait_word(const uint64_t *w, uint64_t target, ui
                                           int32_t *err, int *s_abort) {
   if (threadIdx.x == 0) {
     const uint64_t t_start = globaltimer();
-    while (ld_acquire_sys(w) < target) {
+    for (uint32_t it = 0; ld_acquire_sys(w) < target; ++it) {
       if (globaltimer() - t_start > timeout_ns) {
         atomicExch(err, DERR_TIMEOUT);
+        *s_abort = 1;
+        break;
+      }
+      if ((it & 63u) == 63u && *reinterpret_cast<volatile int32_t *>(err) != 0) {  // fail fast
         *s_abort = 1;
         break;
       }
