@@ -376,10 +376,17 @@ def run_world(args, world, rank, local):
                                f"{n >> 20} MiB per message, direct + relays + pinned host, model-selected",
                    "msg_bytes": n, "mode": args.mode, "parallelism": f"pairs{npairs}x2dir",
                    "l2": "messages >= 126 MB L2 (no flush)" if n >= 128 * MiB else "no flush"},
-        "roofline": {"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
-                     "frac": achieved / 770.0, "traffic": None, "peak_source":
-                     "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
-                     "kernel": "send_kernel"},
+        "roofline": ({"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
+                      "frac": achieved / 770.0, "traffic": None, "peak_source":
+                      "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
+                      "kernel": "send_kernel"}
+                     if os.environ.get("MPX_BENCH_SAME_GPU") != "1" else
+                     # every rank on one GPU (diagnostic): the shared resource is that
+                     # GPU's HBM, 2 bytes per payload byte, both directions at once
+                     {"bound": "hbm", "achieved": 2 * achieved * world, "peak": measured_peaks()[0],
+                      "unit": "GB/s", "frac": 2 * achieved * world / measured_peaks()[0],
+                      "traffic": None, "peak_source": "MEASURED_PEAKS.json HBM copy (all ranks on one GPU)",
+                      "kernel": "send_kernel"}),
         "per_direction_GBps": per_dir,
         "baselines": base,
         "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n * 2 * npairs,
