@@ -34,7 +34,7 @@
 extern "C" {
 #endif
 
-#define MP_ABI_VERSION 1
+#define MP_ABI_VERSION 2  /* 2: NEXT f2 calls; mp_model_opts.window (was reserved) */
 #define MP_MAX_PATHS 16
 
 /* Status codes. */
