@@ -239,8 +239,9 @@ typedef struct mp_flow {
  * source egress / destination ingress (port and direct β) by max(k_out, k_in), a
  * relay's two legs by the number of flows that may use it (and a relay that is itself
  * an endpoint of a flow is excluded), the host legs by the flows sharing that PCIe
- * direction — then every flow is selected on its own (mp_select).  out: nflows
- * configs, caller-allocated.  Not cached.  Host-only. */
+ * direction — then every flow is selected on its own (mp_select; with
+ * mp_model_opts.window > 1, mp_select_window with the pair's window model, NEXT f2).
+ * out: nflows configs, caller-allocated.  Not cached.  Host-only. */
 int mp_select_flows(mp_ctx *ctx, int nflows, const mp_flow *flows, mp_config *out);
 
 /* ---------------------------------------------------------------- NEXT f2: windows, BIBW */

@@ -135,9 +135,12 @@ def duplex_flags(flows, paths_of):
     return out
 
 
-def select_flows_duplex(flows, pair_paths, pair_port, opts: M.Options, kappa) -> list:
+def select_flows_duplex(flows, pair_paths, pair_port, opts: M.Options, kappa, window: int = 1,
+                        window_of=None) -> list:
     """C19 fair share, then C25's duplex factor κ_g on the host legs, then O3 per flow.
-    kappa(g) -> κ_g."""
+    kappa(g) -> κ_g.  window > 1 (C24): every flow sends a window of that many messages,
+    so each is selected with select_window and its pair's window model,
+    window_of(s, d) -> (h, τ)."""
     facs = F.share_factors(flows, lambda f: pair_paths(flows[f][0], flows[f][1]))
     dup = duplex_flags(flows, lambda f: pair_paths(flows[f][0], flows[f][1]))
     out = []
@@ -146,7 +149,11 @@ def select_flows_duplex(flows, pair_paths, pair_port, opts: M.Options, kappa) ->
         paths = [replace(p, beta=p.beta * (kappa(s) if up else 1.0),
                          beta2=p.beta2 * (kappa(d) if down else 1.0)) if p.kind == M.HOST_STAGED else p
                  for p in paths]
-        out.append(M.select(n, paths, opts, port, m))
+        if window > 1 and window_of is not None:
+            h, tau = window_of(s, d)
+            out.append(select_window(n, window, paths, h, opts, port, m, tau))
+        else:
+            out.append(M.select(n, paths, opts, port, m))
     return out
 
 

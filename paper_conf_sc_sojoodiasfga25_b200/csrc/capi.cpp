@@ -761,8 +761,10 @@ int mp_select_flows(mp_ctx *c, int nflows, const mp_flow *flows, mp_config *out)
     s.mask = flows[f].path_mask;
     specs.push_back(s);
   }
+  std::vector<const WindowModel *> wms;
+  for (int f = 0; f < nflows; ++f) wms.push_back(&window_of_pair(c, flows[f].src, flows[f].dst));
   std::vector<Selection> sel;
-  select_flows(models, specs, c->opts, &sel, &c->kappa);
+  select_flows(models, specs, c->opts, &sel, &c->kappa, &wms);
   for (int f = 0; f < nflows; ++f) fill_config(*models[f], sel[f], &out[f]);
   return MP_OK;
 }

@@ -303,7 +303,12 @@ int step_configs(mp_ctx *c, CollState &st, const mp_coll_plan &me, uint64_t byte
       flows.push_back(mp_flow{r, s.send_to, mask, 0, s.bytes});
     }
     std::vector<mp_config> cf(flows.size());
-    if (int e = mp_select_flows(c, static_cast<int>(flows.size()), flows.data(), cf.data())) return e;
+    // one message per pair and step: never the window-aware selection (C24)
+    const uint32_t w = c->opts.window;
+    c->opts.window = 1;
+    const int e = mp_select_flows(c, static_cast<int>(flows.size()), flows.data(), cf.data());
+    c->opts.window = w;
+    if (e) return e;
     mine[j] = cf[my];
   }
   *out = &st.cfgs.emplace(key, std::move(mine)).first->second;

@@ -473,7 +473,8 @@ namespace mpx {
 // be extracted"; MaxRate for contention on shared links).  Every link used by
 // k flows gives each 1/k of its bandwidth; then every flow is selected on its own.
 void select_flows(const std::vector<const PairModel *> &models, const std::vector<FlowSpec> &flows,
-                  const ModelOpts &o, std::vector<Selection> *out, const std::vector<double> *kappa) {
+                  const ModelOpts &o, std::vector<Selection> *out, const std::vector<double> *kappa,
+                  const std::vector<const WindowModel *> *windows) {
   const size_t F = flows.size();
   auto allowed = [&](size_t f, size_t i) {
     return i == 0 || flows[f].mask == 0 || ((flows[f].mask >> i) & 1u);
@@ -538,7 +539,10 @@ void select_flows(const std::vector<const PairModel *> &models, const std::vecto
       if (on) mask |= 1u << i;
     }
     if (m.has_port()) m.port_beta /= pdiv;
-    select(m, flows[f].bytes, mask | 1u, o, &(*out)[f]);
+    if (o.window > 1 && windows && (*windows)[f])  // C24: every flow sends a window
+      select_window(m, *(*windows)[f], flows[f].bytes, o.window, mask | 1u, o, &(*out)[f]);
+    else
+      select(m, flows[f].bytes, mask | 1u, o, &(*out)[f]);
   }
 }
 

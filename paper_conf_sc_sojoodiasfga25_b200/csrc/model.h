@@ -81,9 +81,11 @@ struct FlowSpec {
   uint32_t mask = 0;  // path mask of the pair (0 = all)
 };
 // kappa (NEXT f2, reading C25): per-GPU host duplex factor (may be null = all 1).
+// windows (NEXT f2, C24): per-flow window model, used when o.window > 1 (may be null).
 void select_flows(const std::vector<const PairModel *> &models, const std::vector<FlowSpec> &flows,
                   const ModelOpts &o, std::vector<Selection> *out,
-                  const std::vector<double> *kappa = nullptr);
+                  const std::vector<double> *kappa = nullptr,
+                  const std::vector<const WindowModel *> *windows = nullptr);
 
 // Eq 14 / Eq 15: the real optimal chunk count of a staged path
 // carrying x bytes (used by the φ calibration).

@@ -211,3 +211,46 @@ def test_predict_window_rejects_bad_configs():
         with pytest.raises(mp.MPError):
             c.predict_window(0, 1, n, 0, ok)                    # window 0
         assert c.predict_window(0, 1, n, 4, ok) == pytest.approx(4 * c.predict(0, 1, n, ok), rel=1e-12)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_select_flows_with_window_option_parity(seed):
+    # mp_model_opts.window > 1 makes mp_select_flows window-aware too (C24 with C19/C25)
+    rng = random.Random(300 + seed)
+    flows = []
+    for _ in range(rng.randint(1, 5)):
+        s = rng.randrange(W)
+        d = rng.choice([x for x in range(W) if x != s])
+        flows.append((s, d, rng.choice([4, 16, 64]) * MiB, [True] * W))
+    kappa = {g: rng.uniform(0.6, 1.0) for g in range(W)}
+    wins = {}
+
+    def paths(s, d):
+        return [M.Path(**t) for t in table(s, d, seed)]
+
+    def port(s, d):
+        return M.Port(alpha=1e-6, beta=850e9)
+
+    def window_of(s, d):
+        if (s, d) not in wins:
+            r = random.Random(1000 * s + d + seed)
+            wins[(s, d)] = ([r.uniform(0, 1.2) * p.alpha for p in paths(s, d)], r.uniform(0, 5e-6))
+        return wins[(s, d)]
+    opts = M.Options(mode=M.B200, slot_bytes=64 * MiB)
+    ref = WN.select_flows_duplex(flows, paths, port, opts, kappa.get, window=8, window_of=window_of)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.set_options(mode=M.B200, slot_bytes=64 * MiB, window=8)
+        for g, k in kappa.items():
+            c.set_host_duplex(g, k)
+        for s, d in {(s, d) for s, d, _, _ in flows}:
+            install(c, s, d, table(s, d, seed), port(s, d))
+            h, tau = window_of(s, d)
+            c.set_window_model(s, d, h, tau)
+        got = c.select_flows([(s, d, n, 0) for s, d, n, _ in flows])
+        for g, r in zip(got, ref):
+            gd = g.as_dict()
+            for a, b in zip(gd["bytes"], r.bytes):
+                assert abs(a - b) <= 256
+            assert rel(gd["t_level"], r.t_level) < 1e-9
+            if gd["bytes"] == r.bytes:
+                assert gd["chunks"] == r.chunks and rel(gd["t_pred"], r.t_pred) < 1e-9
