@@ -462,3 +462,21 @@ def test_back_to_back_dependent_chain(ctx, n):
         ctx.xfer(bufs[i + 1], bufs[i], n, staged if i == 4 else None, s)
     ctx.sync()
     assert torch.equal(bufs[8], bufs[0])
+
+
+def test_window_option_drives_unconfigured_transfers(ctx):
+    # mp_model_opts.window > 1: mp_xfer with no config uses mp_select_window's config
+    # (C24); the payload stays bit-exact.
+    o = ctx.get_options()
+    n = 24 * MiB + 99
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                        generator=torch.Generator("cuda").manual_seed(9))
+    dst = torch.zeros_like(src)
+    try:
+        ctx.set_options(**{**o, "window": 16})
+        assert ctx.select(0, 0, n).as_dict() == ctx.select_window(0, 0, n, 16).as_dict()
+        ctx.xfer(dst, src, n, None, torch.cuda.current_stream())
+        ctx.sync()
+        assert torch.equal(dst, src)
+    finally:
+        ctx.set_options(**o)

@@ -254,3 +254,24 @@ def test_select_flows_with_window_option_parity(seed):
             assert rel(gd["t_level"], r.t_level) < 1e-9
             if gd["bytes"] == r.bytes:
                 assert gd["chunks"] == r.chunks and rel(gd["t_pred"], r.t_pred) < 1e-9
+
+
+def test_params_file_with_bands_window_and_duplex(tmp_path):
+    f = str(tmp_path / "p.txt")
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        tbl = table(0, 1, 5)
+        install(c, 0, 1, tbl, M.Port(alpha=1e-6, beta=8e11))
+        prm = [{k: (0.0 if k == "beta2" and math.isinf(t[k]) else t[k] * (0.5 if k == "alpha" else 1.0))
+                for k in FIELDS} for t in tbl]
+        c.set_model_band(0, 1, 8 * MiB, prm, dict(alpha=2e-6, beta=9e11))
+        h = [0.5 * t["alpha"] for t in tbl]
+        c.set_window_model(0, 1, h, 1.5e-6)
+        c.set_host_duplex(3, 0.6)
+        want = [c.select_window(0, 1, n, 16).as_dict() for n in (2 * MiB, 64 * MiB)]
+        c.save_params(f)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.load_params(f)
+        assert [b[0] for b in c.get_model_bands(0, 1)] == [0, 8 * MiB]
+        assert c.get_window_model(0, 1) == (h, 1.5e-6) and c.get_host_duplex(3) == 0.6
+        got = [c.select_window(0, 1, n, 16).as_dict() for n in (2 * MiB, 64 * MiB)]
+        assert got == want
