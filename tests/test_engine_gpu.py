@@ -480,3 +480,16 @@ def test_window_option_drives_unconfigured_transfers(ctx):
         assert torch.equal(dst, src)
     finally:
         ctx.set_options(**o)
+
+
+def test_zero_byte_message_is_a_no_op(ctx):
+    # bytes == 0 is allowed and moves nothing; no kernel is launched
+    dst = torch.full((4096,), 0xA5, dtype=torch.uint8, device="cuda")
+    src = torch.zeros(4096, dtype=torch.uint8, device="cuda")
+    a = ctx.launches()
+    ctx.xfer(dst, src, 0, None, torch.cuda.current_stream())
+    ctx.sync()
+    assert ctx.launches() == a
+    assert bool((dst == 0xA5).all())
+    d = ctx.select(0, 0, 0).as_dict()
+    assert sum(d["bytes"]) == 0 and d["t_pred"] == 0.0
