@@ -132,6 +132,22 @@ def scenario_engine(rank, world):
             assert np.array_equal(got.cpu().numpy(), exp), f"case {i} mismatch"
             c.free(p)
         dist.barrier()
+    # a zero-byte message (allowed, moves nothing) completes and keeps
+    # the pair's FIFO matching in step: the next message still arrives intact
+    if rank == 0:
+        src_buf[:4096].copy_(torch.from_numpy(synth.payload(4096, 77)))
+        c.send(src_buf[:0], 0, 1, tag=90, stream=stream)
+        c.send(src_buf[:4096], 4096, 1, tag=91, stream=stream)
+        stream.synchronize()
+    elif rank == 1:
+        p = c.alloc(4096)
+        c.recv(p, 0, 0, tag=90, stream=stream)
+        c.recv(p, 4096, 0, tag=91, stream=stream)
+        stream.synchronize()
+        assert np.array_equal(mp.as_tensor(p, 4096).cpu().numpy(), synth.payload(4096, 77)), \
+            "after a zero-byte message"
+        c.free(p)
+    dist.barrier()
     # bidirectional (osu_bibw-style): 0 → 1 and 1 → 0 at once, model-selected, two
     # streams per rank, a window of 3 messages each way
     if rank in (0, 1):
