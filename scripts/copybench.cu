@@ -3,12 +3,15 @@
 // different block sizes / depths / CTAs per SM / L2 hints, vs cudaMemcpyAsync.
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o copybench scripts/copybench.cu
 //   ./copybench [bytes]     → one line per variant: GB/s (payload) and % of memcpy
+//   ./copybench [bytes] few → per-CTA rate of small grids (8/16/32 CTAs, as a staged
+//                             stage group) vs issuing warps per CTA
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <string>
 #include <vector>
 
 #define CK(x)                                                                   \
@@ -146,6 +149,20 @@ int main(int argc, char **argv) {
     }
   }
   CK(cudaFuncSetAttribute(tma_copy, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+  if (argc > 2 && std::string(argv[2]) == "few") {
+    for (uint32_t grid : {8u, 16u, 32u})
+      for (uint32_t B : {8192u, 16384u})
+        for (uint32_t D : {4u, 8u})
+          for (uint32_t lanes : {1u, 2u, 4u}) {
+            const uint64_t smem = static_cast<uint64_t>(B) * D * lanes + 8ull * D * lanes;
+            if (smem > 220 * 1024) continue;
+            const double g = timeit([&] { tma_copy<<<grid, 256, smem, st>>>(d, s, n, B, D, lanes, 0); });
+            CK(cudaGetLastError());
+            std::printf("{\"variant\": \"few grid=%u B=%u D=%u warps=%u\", \"GBps\": %.1f, \"GBps_per_cta\": %.2f}\n",
+                        grid, B, D, lanes, g, g / grid);
+          }
+    return 0;
+  }
   struct V {
     uint32_t B, D, lanes, per_sm;
     int hint;
