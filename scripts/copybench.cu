@@ -105,6 +105,52 @@ __global__ void __launch_bounds__(256) tma_copy(uint8_t *d, const uint8_t *s, ui
   asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
+// Same pipeline, one issuing thread per CTA, but the stage of block it-L is refilled
+// after the store of block it (L stores may still be reading shared memory; loads run
+// D-L blocks ahead).  L = 1 is tma_copy's schedule.
+template <int L>
+__global__ void __launch_bounds__(256) tma_lag(uint8_t *d, const uint8_t *s, uint64_t n, uint32_t B, uint32_t D) {
+  extern __shared__ __align__(128) uint8_t sm[];
+  if (threadIdx.x) return;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(sm + static_cast<uint64_t>(B) * D);
+  for (uint32_t i = 0; i < D; ++i) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(su32(bars + i)));
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  const uint64_t nblk = (n + B - 1) / B, me = blockIdx.x, G = gridDim.x;
+  if (me >= nblk) return;
+  const uint64_t mine = (nblk - me + G - 1) / G;
+  auto load = [&](uint64_t it) {
+    const uint64_t o = (me + it * G) * B;
+    const uint32_t len = static_cast<uint32_t>(n - o < B ? n - o : B);
+    const uint32_t bar = su32(bars + it % D);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(len) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     su32(sm + (it % D) * B)),
+                 "l"(s + o), "r"(len), "r"(bar)
+                 : "memory");
+  };
+  const uint64_t pro = mine < D ? mine : D;
+  for (uint64_t it = 0; it < pro; ++it) load(it);
+  for (uint64_t it = 0; it < mine; ++it) {
+    const uint32_t st = it % D;
+    asm volatile(
+        "{\n\t.reg .pred p;\nW_%=:\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t@!p bra W_%=;\n}" ::"r"(
+            su32(bars + st)),
+        "r"(static_cast<uint32_t>((it / D) & 1))
+        : "memory");
+    const uint64_t o = (me + it * G) * B;
+    const uint32_t len = static_cast<uint32_t>(n - o < B ? n - o : B);
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(d + o), "r"(su32(sm + st * B)),
+                 "r"(len)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    if (it >= L && it - L + D < mine) {
+      asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(L) : "memory");
+      load(it - L + D);
+    }
+  }
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
 int main(int argc, char **argv) {
   const uint64_t n = argc > 1 ? std::strtoull(argv[1], nullptr, 0) : (1ull << 30);
   int sms = 0;
@@ -150,9 +196,9 @@ int main(int argc, char **argv) {
   }
   CK(cudaFuncSetAttribute(tma_copy, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
   if (argc > 2 && std::string(argv[2]) == "few") {
-    for (uint32_t grid : {8u, 16u, 32u})
+    for (uint32_t grid : {16u, 148u})
       for (uint32_t B : {8192u, 16384u})
-        for (uint32_t D : {4u, 8u})
+        for (uint32_t D : {2u, 3u, 4u, 8u})
           for (uint32_t lanes : {1u, 2u, 4u}) {
             const uint64_t smem = static_cast<uint64_t>(B) * D * lanes + 8ull * D * lanes;
             if (smem > 220 * 1024) continue;
@@ -160,6 +206,24 @@ int main(int argc, char **argv) {
             CK(cudaGetLastError());
             std::printf("{\"variant\": \"few grid=%u B=%u D=%u warps=%u\", \"GBps\": %.1f, \"GBps_per_cta\": %.2f}\n",
                         grid, B, D, lanes, g, g / grid);
+          }
+    CK(cudaFuncSetAttribute(tma_lag<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    CK(cudaFuncSetAttribute(tma_lag<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    CK(cudaFuncSetAttribute(tma_lag<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    for (uint32_t grid : {16u, 148u, 296u})
+      for (uint32_t B : {4096u, 8192u})
+        for (uint32_t D : {4u, 8u})
+          for (int L : {1, 2, 3}) {
+            if (B * D > 32768u || L >= static_cast<int>(D)) continue;
+            const uint64_t smem = static_cast<uint64_t>(B) * D + 8ull * D;
+            const double g = timeit([&] {
+              if (L == 1) tma_lag<1><<<grid, 256, smem, st>>>(d, s, n, B, D);
+              if (L == 2) tma_lag<2><<<grid, 256, smem, st>>>(d, s, n, B, D);
+              if (L == 3) tma_lag<3><<<grid, 256, smem, st>>>(d, s, n, B, D);
+            });
+            CK(cudaGetLastError());
+            std::printf("{\"variant\": \"lag grid=%u B=%u D=%u L=%d\", \"GBps\": %.1f, \"GBps_per_cta\": %.2f}\n",
+                        grid, B, D, L, g, g / grid);
           }
     return 0;
   }
