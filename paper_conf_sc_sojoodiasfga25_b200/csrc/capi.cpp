@@ -351,6 +351,8 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   P.pdl = c->pdl;
   P.bulk_stages = bulk_stages_for(n);
   P.allow_small = ctas > 0 ? 0u : 1u;  // a staged leg's calibration times its group's CTAs
+  // loopback staged legs move 16 KiB TMA blocks (xfer_kernel); multi-rank ones 8 KiB
+  P.staged_blk = ctas > 0 && c->world == 1 ? 1u : 0u;
   P.npaths = 1;
   DevPath &d = P.p[0];
   d.kind = DK_DIRECT;

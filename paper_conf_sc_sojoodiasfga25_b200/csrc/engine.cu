@@ -115,7 +115,7 @@ __device__ __forceinline__ void group_copy(uint8_t *dst, const uint8_t *src, uin
 
 // ------------------------------------------------------------------ TMA bulk copy
 
-// Bulk-copy engine of one CTA: thread 0 streams 16 KiB blocks global → shared →
+// Bulk-copy engine of one CTA: thread 0 streams BLK-byte blocks (8 KiB by default) global → shared →
 // global with cp.async.bulk (TMA; SASS UBLKCP), kBulkStages blocks in flight, the
 // load of each stage completing on an mbarrier (complete_tx) and each store tracked
 // by a bulk group so a stage is only reloaded once its previous store has finished
@@ -126,6 +126,13 @@ __device__ __forceinline__ void group_copy(uint8_t *dst, const uint8_t *src, uin
 constexpr uint32_t kBulkBlock = 8192;
 constexpr uint32_t kBulkStages = 4;
 constexpr uint32_t kBulkSmem = kBulkBlock * kBulkStages + 64;
+// Staged legs of the loopback transfer kernel use 16 KiB blocks: one CTA's TMA rate is
+// bound by the shared memory it keeps in flight (~32 KiB per ~1.5 µs round trip;
+// few-CTA sweep, profiles/r01/copybench_few*.jsonl: 20 GB/s at 4 × 8 KiB, 40 GB/s at
+// 4 × 16 KiB).  xfer_kernel launches with kXferSmem; residency drops from 4 to 3 CTAs
+// per SM, and xfer_capacity() reports that, so the co-residency cap follows.
+constexpr uint32_t kStagedBlock = 16384;
+constexpr uint32_t kXferSmem = kStagedBlock * kBulkStages + 64;
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -172,7 +179,7 @@ __device__ __forceinline__ void bulk_wait_all() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
-template <int MODE>
+template <int MODE, uint32_t BLK = kBulkBlock>
 __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32_t r, uint32_t G,
                           uint8_t *smem, uint32_t D, bool publish_after = true) {
   if ((reinterpret_cast<uintptr_t>(dst) ^ reinterpret_cast<uintptr_t>(src)) & 15u) {
@@ -194,18 +201,18 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
   if (MODE != LD_SRC) asm volatile("fence.proxy.async.global;" ::: "memory");
   const uint8_t *s = src + head;
   uint8_t *d = dst + head;
-  const uint64_t nblk = (body + kBulkBlock - 1) / kBulkBlock;
+  const uint64_t nblk = (body + BLK - 1) / BLK;
   if (r >= nblk) return;
   const uint64_t mine = (nblk - r + G - 1) / G;  // blocks r, r+G, …
   if (D < 1 || D > kBulkStages) D = kBulkStages;
-  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + kBulkBlock * kBulkStages);
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + BLK * kBulkStages);
   for (uint32_t i = 0; i < D; ++i) mbar_init(smem_u32(bars + i));
   // make the initialised barriers visible to the async proxy (no cluster: CTA scope)
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   auto blk = [&](uint64_t it, uint64_t *off, uint32_t *bytes) {
-    const uint64_t o = (r + it * G) * static_cast<uint64_t>(kBulkBlock);
+    const uint64_t o = (r + it * G) * static_cast<uint64_t>(BLK);
     *off = o;
-    *bytes = static_cast<uint32_t>(body - o < kBulkBlock ? body - o : kBulkBlock);
+    *bytes = static_cast<uint32_t>(body - o < BLK ? body - o : BLK);
   };
   auto issue_load = [&](uint64_t it) {
     uint64_t o;
@@ -214,7 +221,7 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
     const uint32_t st = static_cast<uint32_t>(it % D);
     const uint32_t bar = smem_u32(bars + st);
     mbar_expect_tx(bar, n);
-    bulk_load(smem_u32(smem + st * kBulkBlock), s + o, n, bar);
+    bulk_load(smem_u32(smem + st * BLK), s + o, n, bar);
   };
   const uint64_t pro = mine < D ? mine : D;
   for (uint64_t it = 0; it < pro; ++it) issue_load(it);
@@ -224,7 +231,7 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
     uint64_t o;
     uint32_t n;
     blk(it, &o, &n);
-    bulk_store(d + o, smem_u32(smem + st * kBulkBlock), n);
+    bulk_store(d + o, smem_u32(smem + st * BLK), n);
     // refill the stage used one iteration ago once its store has read shared memory
     if (it >= 1 && it - 1 + D < mine) {
       bulk_wait_read<1>();
@@ -316,12 +323,12 @@ __device__ __forceinline__ uint64_t ld_volatile(const uint64_t *p) {
 }
 
 // One CTA copies its slice of a staged chunk: TMA pipeline (copy_mode 1) or LDG/STG.
-template <int MODE>
+template <int MODE, uint32_t BLK = kBulkBlock>
 __device__ __forceinline__ void copy_slice(uint8_t *dst, const uint8_t *src, uint64_t len, uint8_t *smem,
                                            uint32_t copy_mode, uint32_t stages) {
   if (len == 0) return;
   if (copy_mode == 1)
-    bulk_copy<MODE>(dst, src, len, 0, 1, smem, stages);
+    bulk_copy<MODE, BLK>(dst, src, len, 0, 1, smem, stages);
   else
     group_copy<MODE>(dst, src, len, 0, 1);
 }
@@ -372,7 +379,7 @@ __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, 
     uint8_t *slot = p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(src) & 15u);
     uint64_t a, b;  // slice r of the chunk, split on 16-byte boundaries
     slice_of(len, r, p.g_in, &a, &b);
-    copy_slice<LD_SRC>(slot + a, src + a, b - a, smem, P.copy_mode, P.bulk_stages);
+    copy_slice<LD_SRC, kStagedBlock>(slot + a, src + a, b - a, smem, P.copy_mode, P.bulk_stages);
     release_flag(p.full + s * kFlagStride + r, u + 1);
   }
 }
@@ -388,7 +395,7 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
         p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(p.src + off) & 15u);
     uint64_t a, b;
     slice_of(len, r, p.g_out, &a, &b);
-    copy_slice<MODE>(p.dst + off + a, slot + a, b - a, smem, P.copy_mode, P.bulk_stages);
+    copy_slice<MODE, kStagedBlock>(p.dst + off + a, slot + a, b - a, smem, P.copy_mode, P.bulk_stages);
     release_flag(p.freef + s * kFlagStride + r, u + 1);
   }
 }
@@ -794,6 +801,15 @@ __global__ void __launch_bounds__(kThreads, 4) direct_kernel(const __grid_consta
   bulk_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
 }
 
+// Step 1's timing copy of a loopback staged leg: the same striped TMA pipeline as
+// direct_kernel, with the staged legs' block size (kStagedBlock), so the calibrated
+// leg β is what a stage group of that many CTAs moves.
+__global__ void __launch_bounds__(kThreads, 4) direct_leg_kernel(const __grid_constant__ DirectArgs A) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
+  pdl_enter();
+  bulk_copy<LD_SRC, kStagedBlock>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
+}
+
 // One-shot small copy (co-aligned src/dst): thread i of the grid moves vector i of the
 // 16-B body; the last CTA also moves the < 16-byte head and tail.  Kept tiny and
 // branch-light on purpose: at these sizes a launch on a cold SM is bound by its
@@ -919,10 +935,11 @@ int launch_xfer(const XferParams &P, void *stream) {
   }
   if (direct_only) {
     const DirectArgs A{P.p[0].dst, P.p[0].src, P.p[0].bytes, P.copy_mode, P.bulk_stages};
+    if (P.copy_mode == 1 && P.staged_blk) return launch_k(pdl, direct_leg_kernel, P.nblocks, kXferSmem, stream, A);
     if (P.copy_mode == 1) return launch_k(pdl, direct_kernel, P.nblocks, kBulkSmem, stream, A);
     return launch_k(pdl, direct_reg_kernel, P.nblocks, 0, stream, A);
   }
-  return launch_k(pdl, xfer_kernel, P.nblocks, kBulkSmem, stream, P);
+  return launch_k(pdl, xfer_kernel, P.nblocks, kXferSmem, stream, P);
 }
 
 int launch_send(const SendParams &P, void *stream) {
@@ -967,11 +984,14 @@ int preload_kernels() {
   // with the persistent relay kernel running that would deadlock the first launch of
   // any other engine kernel.  Force every kernel of this module to load up front.
   cudaFuncAttributes a;
-  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(recv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(relay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(direct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(direct_leg_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_leg_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
@@ -993,9 +1013,9 @@ int preload_kernels() {
 
 int xfer_capacity(int device, int *per_sm, int *sms) {
   int n = 0;
-  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
   if (e != cudaSuccess) return static_cast<int>(e);
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xfer_kernel, kThreads, kBulkSmem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xfer_kernel, kThreads, kXferSmem);
   if (e != cudaSuccess) return static_cast<int>(e);
   int s = 0;
   e = cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, device);

@@ -54,6 +54,9 @@ struct XferParams {
   uint32_t bulk_stages;  // TMA pipeline depth per CTA (1..4)
   uint32_t allow_small;  // 1: a small direct-only message may use the one-shot kernel
   uint32_t pdl;          // 1: launched with programmatic stream serialization (PDL)
+  uint32_t staged_blk;   // 1: a direct-only copy timing a loopback staged leg (Step 1):
+                         //    moved with the staged legs' TMA block size
+  uint32_t pad_;
   uint64_t timeout_ns;
   int32_t *err;          // device (or mapped host) error word
   DevPath p[kMaxPaths];
