@@ -493,3 +493,22 @@ def test_zero_byte_message_is_a_no_op(ctx):
     assert bool((dst == 0xA5).all())
     d = ctx.select(0, 0, 0).as_dict()
     assert sum(d["bytes"]) == 0 and d["t_pred"] == 0.0
+
+
+@pytest.mark.parametrize("kind", ["relay", "host"])
+@pytest.mark.parametrize("per_cta", [16384 - 16, 16384, 16384 + 16, 3 * 16384 + 4097])
+@pytest.mark.parametrize("src_off,dst_off", [(0, 0), (5, 5), (3, 11)])
+def test_staged_slices_around_16k_blocks(ctx, kind, per_cta, src_off, dst_off):
+    # loopback staged legs move 16 KiB TMA blocks (engine.cu kStagedBlock): each stage
+    # group CTA's slice of a chunk is sized to end just before, on and just after a
+    # block boundary, co-aligned and not (the LDG/STG fallback), two messages in a row
+    # with different chunk counts so one slot carries chunks of different lengths
+    ps = ctx.paths()
+    i = 1 if kind == "relay" else len(ps) - 1
+    for k in (2, 3):
+        n = per_cta * 8 * k + 7
+        nbytes = [0] * len(ps)
+        nbytes[i] = n
+        chunks = [1] + [0] * (len(ps) - 1)
+        chunks[i] = k
+        run(ctx, n, nbytes, chunks, src_off, dst_off, seed=k)
