@@ -614,14 +614,7 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
   if (c->world != 1) {
     std::vector<uint64_t> sizes;
     for (uint64_t s = 4096; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
-    const bool was_running = c->relay_running;
-    if (int s = world_stop_relay(c)) return s;
-    int s = calibrate_world(c, sizes, reps, edges, true);
-    if (was_running) {
-      const int r = world_start_relay(c);
-      if (!s) s = r;
-    }
-    if (s) return s;
+    if (int s = calibrate_world(c, sizes, reps, edges, true)) return s;
     int32_t derr = 0;
     CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
     if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration probe timed out");
@@ -821,16 +814,7 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
     else
       for (uint64_t s = 16ull << 20; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
     int32_t derr = 0;
-    // cudaFree inside the calibration synchronises the device: the persistent relay
-    // kernel must not be running (it resumes at its saved ring positions).
-    const bool was_running = c->relay_running;
-    if (int s = world_stop_relay(c)) return s;
-    int s = calibrate_world(c, sizes, reps, std::vector<double>{0.0}, false);
-    if (was_running) {
-      const int r = world_start_relay(c);
-      if (!s) s = r;
-    }
-    if (s) return s;
+    if (int s = calibrate_world(c, sizes, reps, std::vector<double>{0.0}, false)) return s;
     CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
     if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration probe timed out");
     return MP_OK;

@@ -308,6 +308,7 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
     d.host_ring = r.host ? 1u : 0u;
     d.q0 = r.q;
     d.slot_stride = c->slot_bytes + kSlotSlack;
+    d.lane = lane_stride(c->slot_bytes, static_cast<uint32_t>(c->relay_ctas));
     d.ring = r.data;
     d.full = r.full;
     d.freef = r.freef;
@@ -1004,7 +1005,7 @@ int mp_sync(mp_ctx *c) {
 
 int mp_stats(mp_ctx *c, uint64_t *launches) {
   if (!c || !launches) return MP_ERR_INVALID;
-  *launches = c->launches;
+  *launches = c->launches + (c->world > 1 && !c->model_only ? world_relay_launches(c) : 0);
   return MP_OK;
 }
 

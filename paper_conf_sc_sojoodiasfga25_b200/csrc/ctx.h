@@ -17,7 +17,8 @@
 
 namespace mpx {
 
-struct CollState;  // collectives (coll.cpp): internal streams, events, heap scratch
+struct CollState;     // collectives (coll.cpp): internal streams, events, heap scratch
+struct RelayService;  // world.cpp: the relay rank's doorbell thread and streams
 
 // A staging ring (D8): S slots of slot_stride bytes + per-CTA flag words.
 struct Ring {
@@ -125,12 +126,12 @@ struct mp_ctx {
   size_t hseg_bytes = 0;
   std::vector<uint8_t *> hseg;              // [world]: mapped host segment of each receiver
   std::vector<uint64_t> send_seq, recv_seq, relay_q, host_q, done_target;
+  std::vector<uint64_t> relay_m;            // [world(relay)]: relayed messages sent via each relay
   mpx::CollState *coll = nullptr;           // created by the first collective
   std::vector<uint64_t> eager_send_seq, eager_recv_seq;  // eager protocol (reading C23)
   uint64_t eager_max = 0;                   // messages of 1..eager_max bytes go eager
-  cudaStream_t relay_stream = nullptr;
-  int32_t *stop = nullptr;                  // mapped host word read by the relay kernel
-  bool relay_running = false;
+  mpx::RelayService *relay_svc = nullptr;   // world >= 3: launches relay kernels on doorbells
+  uint64_t relay_launches_done = 0;         // relay launches of stopped services
   std::vector<cudaStream_t> streams;        // user streams seen by mp_send/mp_recv
   // receive regions (mp_register): [kMaxRegions], region 0 = the heap
   struct Region {
@@ -176,6 +177,8 @@ int world_allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes);
 int world_init(mp_ctx *c);
 int world_start_relay(mp_ctx *c);
 int world_stop_relay(mp_ctx *c);
+uint64_t world_relay_launches(const mp_ctx *c);  // relay kernels this rank launched
+int world_relay_error(const mp_ctx *c);          // cudaError_t of a failed relay launch, 0 if none
 int world_finalize(mp_ctx *c);
 int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,
                void *stream);

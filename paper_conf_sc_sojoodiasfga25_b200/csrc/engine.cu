@@ -250,12 +250,10 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
 // ------------------------------------------------------------------ flags
 
 // Warp 0 polls `n` flag words until every one is >= target (ld.acquire.sys), then
-// the CTA synchronises.  Returns false (and raises DERR_TIMEOUT) on timeout, or when
-// the optional host `stop` word becomes non-zero (persistent relay shutdown; then no
-// error is raised and timeout_ns may be 0 = wait forever).
+// the CTA synchronises.  Returns false (and raises DERR_TIMEOUT) on timeout, or once
+// any other wait of the context has failed (the sticky error word is set).
 __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, uint64_t target,
-                                           uint64_t timeout_ns, int32_t *err, int *s_abort,
-                                           const volatile int32_t *stop = nullptr) {
+                                           uint64_t timeout_ns, int32_t *err, int *s_abort) {
   if (threadIdx.x < 32) {
     const uint32_t lane = threadIdx.x;
     const uint64_t t_start = globaltimer();
@@ -263,23 +261,19 @@ __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, ui
     for (uint32_t it = 0;; ++it) {
       const bool mine = lane >= n || ld_acquire_sys(flags + lane) >= target;
       if (__all_sync(0xffffffffu, mine)) break;
-      if (timeout_ns && globaltimer() - t_start > timeout_ns) {
+      if (globaltimer() - t_start > timeout_ns) {
         why = 1;
         break;
       }
       // fail fast: once any wait of this context has failed (sticky error word), the
       // flags this CTA waits for may never come — abort now instead of timing out in
-      // turn behind it (the persistent relay, which passes `stop`, keeps serving)
-      if (!stop && (it & 63u) == 63u &&
+      // turn behind it
+      if ((it & 63u) == 63u &&
           __any_sync(0xffffffffu, lane == 0 && *reinterpret_cast<volatile int32_t *>(err) != 0)) {
         why = 3;
         break;
       }
-      if (stop && (it & 255u) == 255u && *stop) {
-        why = 2;
-        break;
-      }
-      __nanosleep(stop ? 256 : 64);
+      __nanosleep(64);
     }
     if (lane == 0) {
       if (why == 1) atomicExch(err, DERR_TIMEOUT);
@@ -367,40 +361,433 @@ __device__ __forceinline__ void pdl_enter() {
   asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
+// ------------------------------------------------------------------ streamed lanes
+//
+// One lane of a staged path (engine.h, lane_stride) moved through one TMA pipeline
+// that runs across chunk boundaries: the loads of chunk j+1 are issued while the
+// stores of chunk j are still in flight, and a chunk's flag is published once its
+// stores have completed (a lag of kStreamLag store groups, or at once when the storer
+// would otherwise block), so the pipeline never drains between chunks.  The handoff
+// protocol is unchanged — chunk granularity: the full flag of a lane is released
+// when its whole slice has landed and the free flag when it has been read (Eq 12-13's
+// two-stage pipeline) — only the per-chunk restart and drain of the copy
+// (profiles/r01 relay_sweep: ~5.6 µs per chunk per lane) are gone.
+// Requires co-aligned source and destination slices (else the CTA-wide per-chunk
+// path, copy_slice, is used).  A Role supplies, per chunk j:
+//   int  wait(j)               watcher: block until chunk j may be read (consumer:
+//                              full flag) / written (producer: free flag); 1 or -1
+//   int  fetch(j, w)           watcher, after wait: up to 5 words for geom / stored
+//                              (the relay's lane header); 1, or -1 when invalid
+//   SliceGeo geom(j, w)        loader: source / destination / length of slice j
+//   void before_store(j)       storer, producer: lane header (relay) — after wait
+//   void loaded(j)             publisher: every load of slice j has landed
+//                              (consumer: free flag)
+//   void stored(j, w)          publisher: every store of slice j is complete and
+//                              visible (producer: full flag; consumer: byte counters)
+// Four threads, each one lane of its own warp: the loader (thread 0) enters chunks
+// and issues the TMA loads, the storer (thread 96) issues the TMA stores and hands
+// each stage back through an "empty" mbarrier once its store has read it out (the
+// usual warp-specialised TMA pipeline: neither issue stream waits on the other's
+// latencies), the watcher (thread 32) waits on the flags, the publisher (thread 64)
+// issues the system-scope releases (each a MEMBAR.SYS of several µs).
+constexpr uint32_t kStreamLag = 6;
+constexpr uint32_t kStreamAhead = 8;  // chunks the watcher may run ahead of the publisher
+
+struct SliceGeo {
+  const uint8_t *src;
+  uint8_t *dst;
+  uint64_t len;
+};
+
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+
+// Non-blocking: has the phase with this parity completed?
+__device__ __forceinline__ bool mbar_test(uint32_t bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(bar), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+
+// Wait for the phase, giving up (false) once *stop is set.
+__device__ __forceinline__ bool mbar_wait_or_stop(uint32_t bar, uint32_t parity, const uint32_t *stop) {
+  while (!mbar_test(bar, parity)) {
+    if (*reinterpret_cast<const volatile uint32_t *>(stop)) return false;
+    __nanosleep(20);
+  }
+  return true;
+}
+
+__device__ __forceinline__ uint64_t ld_relaxed_sys(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Block one thread until *f >= target: 1, or -1 on timeout (DERR_TIMEOUT raised) or
+// once the context's error word is set.  Polls relaxed (an acquire load invalidates
+// the SM's L1 every time); one acquire on success.
+__device__ __forceinline__ int poll_flag(const uint64_t *f, uint64_t target, uint64_t timeout_ns, int32_t *err) {
+  const uint64_t t0 = globaltimer();
+  for (uint32_t it = 0;; ++it) {
+    if (ld_relaxed_sys(f) >= target && ld_acquire_sys(f) >= target) return 1;
+    if (globaltimer() - t0 > timeout_ns) {
+      atomicExch(err, DERR_TIMEOUT);
+      return -1;
+    }
+    if ((it & 63u) == 63u && *reinterpret_cast<volatile int32_t *>(err) != 0) return -1;
+    __nanosleep(128);
+  }
+}
+
+__device__ __forceinline__ uint32_t ld_acquire_cta_shared(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void st_release_cta_shared(uint32_t *p, uint32_t v) {
+  asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+
+template <int MODE>
+__device__ __forceinline__ void bytes_copy(uint8_t *d, const uint8_t *s, uint64_t n) {
+  for (uint64_t i = 0; i < n; ++i) d[i] = ld1<MODE>(s + i);
+}
+
+// Called by every thread of the CTA; threads other than 0, 32, 64 and 96 return at once.
+template <int MODE, class Role>
+__device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
+  __shared__ uint32_t s_ready;    // chunks the watcher has found ready
+  __shared__ uint32_t s_taken;    // chunks taken up (consumer: loader read the words; producer: storer)
+  __shared__ uint32_t s_loaded;   // chunks whose loads have all landed (storer → publisher)
+  __shared__ uint32_t s_stored;   // chunks whose stores are complete (storer → publisher)
+  __shared__ uint32_t s_pub;      // chunks the publisher has finished (their words free)
+  __shared__ uint32_t s_stop;     // 1: a wait failed
+  __shared__ uint64_t s_words[kStreamAhead][5];
+  constexpr uint32_t BLK = kStagedBlock, D = kBulkStages;
+  static_assert(D == 4, "stage arithmetic below assumes 4 stages");
+  uint64_t *full = reinterpret_cast<uint64_t *>(smem + BLK * D);  // [D] loaded
+  uint64_t *empty = full + D;                                      // [D] read out by its store
+  const uint32_t full0 = smem_u32(full), empty0 = smem_u32(empty), smem0 = smem_u32(smem);
+  if (threadIdx.x == 0) {
+    s_ready = 0;
+    s_taken = 0;
+    s_loaded = 0;
+    s_stored = 0;
+    s_pub = 0;
+    s_stop = 0;
+    for (uint32_t i = 0; i < D; ++i) {
+      mbar_init(full0 + 8 * i);
+      mbar_init(empty0 + 8 * i);
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x == 32) {  // the watcher: flag waits (a global round trip per poll)
+    for (uint32_t j = 0; j < nchunks; ++j) {
+      while (ld_acquire_cta_shared(&s_pub) + kStreamAhead <= j) {
+        if (*reinterpret_cast<volatile uint32_t *>(&s_stop)) return;
+        __nanosleep(64);
+      }
+      if (R.wait(j) < 0 || R.fetch(j, s_words[j % kStreamAhead]) < 0) {
+        st_release_cta_shared(&s_stop, 1);
+        return;
+      }
+      st_release_cta_shared(&s_ready, j + 1);
+    }
+    return;
+  }
+  if (threadIdx.x == 64) {  // the publisher: system-scope releases (MEMBAR.SYS each) off the TMA issue
+    uint32_t pl = 0, ps = 0;
+    while (ps < nchunks || pl < nchunks) {
+      const uint32_t a = ld_acquire_cta_shared(&s_loaded);
+      const uint32_t b = ld_acquire_cta_shared(&s_stored);
+      if (pl == a && ps == b) {
+        if (*reinterpret_cast<volatile uint32_t *>(&s_stop)) return;
+        __nanosleep(32);
+        continue;
+      }
+      for (; pl < a; ++pl) R.loaded(pl);
+      for (; ps < b; ++ps) R.stored(ps, s_words[ps % kStreamAhead]);
+      st_release_cta_shared(&s_pub, ps);
+    }
+    return;
+  }
+  struct Geo {
+    const uint8_t *s0;  // slice start (source), for the producer's head/tail
+    const uint8_t *s;   // 16-B aligned body start (source)
+    uint8_t *d;         // body start (destination)
+    uint64_t len;       // slice bytes
+    uint64_t body;      // body bytes (a multiple of 16)
+    uint32_t steps;     // max(1, blocks of the body): a chunk without a body takes one empty step
+  };
+  // the geometry of the chunks between the store and the load cursor (<= D + 1),
+  // written by the loader before it arms a chunk's first stage (mbarrier arrive =
+  // release, the storer's wait = acquire)
+  __shared__ Geo geo[kStreamAhead];
+  if (threadIdx.x == 0) {
+    // ---- the loader: chunk entry (consumer: readiness, geometry, head/tail), loads
+    uint32_t gl = 0;
+    for (uint32_t lc = 0; lc < nchunks; ++lc) {
+      if (!R.producer) {
+        // block: the storer publishes on its own (never waits on us with publications pending)
+        int rdy = ld_acquire_cta_shared(&s_ready) > lc ? 1 : 0;
+        while (!rdy) {
+          if (*reinterpret_cast<volatile uint32_t *>(&s_stop)) rdy = -1;
+          else if (ld_acquire_cta_shared(&s_ready) > lc) rdy = 1;
+          else __nanosleep(32);
+        }
+        if (rdy < 0) return;
+        asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA reads what was acquired
+      }
+      const SliceGeo g = R.geom(lc, s_words[lc % kStreamAhead]);
+      if (!R.producer) st_release_cta_shared(&s_taken, lc + 1);
+      uint64_t h = (16u - (reinterpret_cast<uintptr_t>(g.src) & 15u)) & 15u;
+      if (h > g.len) h = g.len;
+      const uint64_t body = (g.len - h) & ~uint64_t(15);
+      const uint32_t nblk = static_cast<uint32_t>((body + BLK - 1) / BLK);
+      if (!R.producer) {  // consumer: head / tail bytes now (the lane is acquired)
+        bytes_copy<MODE>(g.dst, g.src, h);
+        bytes_copy<MODE>(g.dst + h + body, g.src + h + body, g.len - h - body);
+      }
+      // the stage of this chunk's first step is free (the store of step gl - D has read
+      // it out); geo[lc % 8] was last read for chunk lc - 8, which the storer left
+      // more than D steps ago
+      if (gl >= D && !mbar_wait_or_stop(empty0 + 8 * (gl & 3u), ((gl >> 2) - 1) & 1u, &s_stop)) return;
+      Geo &e = geo[lc % kStreamAhead];
+      e.s0 = g.src;
+      e.s = g.src + h;
+      e.d = g.dst + h;
+      e.len = g.len;
+      e.body = body;
+      e.steps = nblk ? nblk : 1;
+      const uint8_t *src = g.src + h;
+      uint64_t rem = body;
+      for (uint32_t b = 0; b < e.steps; ++b, ++gl) {
+        const uint32_t fb = full0 + 8 * (gl & 3u);
+        if (b > 0 && gl >= D && !mbar_wait_or_stop(empty0 + 8 * (gl & 3u), ((gl >> 2) - 1) & 1u, &s_stop))
+          return;
+        if (rem) {
+          const uint32_t n = rem < BLK ? static_cast<uint32_t>(rem) : BLK;
+          mbar_expect_tx(fb, n);
+          bulk_load(smem0 + (gl & 3u) * BLK, src, n, fb);
+          src += n;
+          rem -= n;
+        } else {
+          mbar_arrive(fb);
+        }
+      }
+    }
+    return;
+  }
+  if (threadIdx.x != 96) return;
+  // ---- the storer: producer readiness + head/tail + lane header, stores, stage
+  // release, publication of completed chunks
+  // chunks [ph, pt) have their stores issued but are not yet published; the last
+  // store step of chunk c is pend_last[c % 16] (at most kStreamLag + 1 are pending)
+  __shared__ uint32_t pend_last[16];
+  uint32_t ph = 0, pt = 0;
+  uint32_t pub_at = 0xffffffffu;  // store step after which chunk ph is published
+  auto flush = [&]() {            // every issued store complete; the publisher releases the chunks
+    if (ph == pt) return;
+    bulk_wait_all();
+    ph = pt;
+    st_release_cta_shared(&s_stored, pt);
+    pub_at = 0xffffffffu;
+  };
+  uint32_t gs = 0;
+  bool ok = true;
+  for (uint32_t sc = 0; sc < nchunks && ok; ++sc) {
+    if (R.producer) {
+      if (ld_acquire_cta_shared(&s_ready) <= sc) {
+        flush();  // never block with publications pending (the other side may wait on them)
+        while (ld_acquire_cta_shared(&s_ready) <= sc) {
+          if (*reinterpret_cast<volatile uint32_t *>(&s_stop)) {
+            ok = false;
+            break;
+          }
+          __nanosleep(32);
+        }
+        if (!ok) break;
+      }
+      st_release_cta_shared(&s_taken, sc + 1);
+    }
+    // the chunk's geometry: written by the loader before it armed this first step
+    uint32_t fb = full0 + 8 * (gs & 3u);
+    if (!mbar_test(fb, (gs >> 2) & 1u)) {
+      flush();
+      if (!mbar_wait_or_stop(fb, (gs >> 2) & 1u, &s_stop)) {
+        ok = false;
+        break;
+      }
+    }
+    const Geo &e = geo[sc % kStreamAhead];
+    if (R.producer) {
+      const uint64_t h = static_cast<uint64_t>(e.s - e.s0);
+      bytes_copy<MODE>(e.d - h, e.s0, h);
+      bytes_copy<MODE>(e.d + e.body, e.s + e.body, e.len - h - e.body);
+      R.before_store(sc);
+    }
+    uint8_t *dst = e.d;
+    uint64_t rem = e.body;
+    const uint32_t steps = e.steps;
+    for (uint32_t b = 0; b < steps; ++b, ++gs) {
+      fb = full0 + 8 * (gs & 3u);
+      if (b > 0 && !mbar_test(fb, (gs >> 2) & 1u)) {
+        flush();
+        if (!mbar_wait_or_stop(fb, (gs >> 2) & 1u, &s_stop)) {
+          ok = false;
+          break;
+        }
+      }
+      if (rem) {
+        const uint32_t n = rem < BLK ? static_cast<uint32_t>(rem) : BLK;
+        bulk_store(dst, smem0 + (gs & 3u) * BLK, n);
+        dst += n;
+        rem -= n;
+      } else {
+        bulk_commit();  // an empty group keeps group index == step index
+      }
+      // the previous step's store has read its stage: hand the stage back to the loader
+      if (gs > 0) {
+        bulk_wait_read<1>();
+        mbar_arrive(empty0 + 8 * ((gs - 1) & 3u));
+      }
+      if (gs >= pub_at) {  // the oldest pending chunk's stores are kStreamLag groups back
+        asm volatile("cp.async.bulk.wait_group %0;" ::"n"(kStreamLag) : "memory");
+        asm volatile("fence.proxy.async.global;" ::: "memory");
+        while (ph != pt && pend_last[ph % 16] + kStreamLag <= gs) ++ph;
+        st_release_cta_shared(&s_stored, ph);
+        pub_at = ph != pt ? pend_last[ph % 16] + kStreamLag : 0xffffffffu;
+      }
+    }
+    if (!ok) break;
+    // chunk sc fully loaded and its stores issued
+    st_release_cta_shared(&s_loaded, sc + 1);
+    pend_last[pt % 16] = gs - 1;  // pt == sc
+    if (ph == pt) pub_at = gs - 1 + kStreamLag;
+    ++pt;
+  }
+  if (ok) {
+    flush();
+    bulk_wait_read<0>();
+  } else {
+    st_release_cta_shared(&s_stop, 1);  // the watcher, loader and publisher stop too
+    bulk_wait_all();
+  }
+}
+
 // ------------------------------------------------------------------ roles
 
+// Lane r of a staged path (stage-in CTA r and forward CTA r): slice r of every chunk
+// goes through lane r of the chunk's slot, handed over by lane r's own full/free flag
+// (engine.h, lane_stride) — an independent two-stage pipeline per lane.
+__device__ __forceinline__ uint8_t *lane_at(const DevPath &p, uint64_t s, uint32_t r, const uint8_t *src) {
+  return p.ring + s * p.slot_stride + r * p.lane + (reinterpret_cast<uintptr_t>(src) & 15u);
+}
+
+// Streamed roles of the loopback rings (lane_stream).
+struct LoopProducer {
+  static constexpr bool producer = true;
+  const DevPath *p;
+  uint32_t r;
+  uint64_t timeout_ns;
+  int32_t *err;
+  __device__ SliceGeo geom(uint32_t j, const uint64_t *) const {
+    uint64_t off, len, a, b;
+    chunk_range(*p, j, &off, &len);
+    slice_of(len, r, p->g_in, &a, &b);
+    const uint8_t *src = p->src + off;
+    return SliceGeo{src + a, lane_at(*p, (p->q0 + j) % p->slots, r, src), b - a};
+  }
+  __device__ int wait(uint32_t j) {
+    const uint64_t q = p->q0 + j;
+    return poll_flag(p->freef + (q % p->slots) * kFlagStride + r, q / p->slots, timeout_ns, err);
+  }
+  __device__ int fetch(uint32_t, uint64_t *) { return 1; }
+  __device__ void before_store(uint32_t) {}
+  __device__ void loaded(uint32_t) {}
+  __device__ void stored(uint32_t j, const uint64_t *) {
+    const uint64_t q = p->q0 + j;
+    st_release_sys(p->full + (q % p->slots) * kFlagStride + r, q / p->slots + 1);
+  }
+};
+
+struct LoopConsumer {
+  static constexpr bool producer = false;
+  const DevPath *p;
+  uint32_t r;
+  uint64_t timeout_ns;
+  int32_t *err;
+  __device__ SliceGeo geom(uint32_t j, const uint64_t *) const {
+    uint64_t off, len, a, b;
+    chunk_range(*p, j, &off, &len);
+    slice_of(len, r, p->g_out, &a, &b);
+    return SliceGeo{lane_at(*p, (p->q0 + j) % p->slots, r, p->src + off), p->dst + off + a, b - a};
+  }
+  __device__ int wait(uint32_t j) {
+    const uint64_t q = p->q0 + j;
+    return poll_flag(p->full + (q % p->slots) * kFlagStride + r, q / p->slots + 1, timeout_ns, err);
+  }
+  __device__ int fetch(uint32_t, uint64_t *) { return 1; }
+  __device__ void before_store(uint32_t) {}
+  __device__ void loaded(uint32_t j) {
+    const uint64_t q = p->q0 + j;
+    st_release_sys(p->freef + (q % p->slots) * kFlagStride + r, q / p->slots + 1);
+  }
+  __device__ void stored(uint32_t, const uint64_t *) {}
+};
+
 __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
+  if (P.copy_mode == 1) {  // streamed lane (the source slice and its lane are co-aligned)
+    LoopProducer R{&p, r, P.timeout_ns, P.err};
+    lane_stream<LD_SRC>(R, p.k, smem);
+    return;
+  }
   for (uint32_t j = 0; j < p.k; ++j) {
     uint64_t off, len;
     chunk_range(p, j, &off, &len);
     const uint64_t q = p.q0 + j, s = q % p.slots, u = q / p.slots;
-    if (!wait_flags(p.freef + s * kFlagStride, p.g_out, u, P.timeout_ns, P.err, s_abort)) return;
+    if (!wait_flags(p.freef + s * kFlagStride + r, 1, u, P.timeout_ns, P.err, s_abort)) return;
     const uint8_t *src = p.src + off;
-    uint8_t *slot = p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(src) & 15u);
     uint64_t a, b;  // slice r of the chunk, split on 16-byte boundaries
     slice_of(len, r, p.g_in, &a, &b);
-    copy_slice<LD_SRC, kStagedBlock>(slot + a, src + a, b - a, smem, P.copy_mode, P.bulk_stages);
+    copy_slice<LD_SRC, kStagedBlock>(lane_at(p, s, r, src), src + a, b - a, smem, P.copy_mode, P.bulk_stages);
     release_flag(p.full + s * kFlagStride + r, u + 1);
   }
 }
 
 template <int MODE>
 __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
+  if (P.copy_mode == 1 && ((reinterpret_cast<uintptr_t>(p.src) ^ reinterpret_cast<uintptr_t>(p.dst)) & 15u) == 0) {
+    LoopConsumer R{&p, r, P.timeout_ns, P.err};
+    lane_stream<MODE>(R, p.k, smem);
+    return;
+  }
   for (uint32_t j = 0; j < p.k; ++j) {
     uint64_t off, len;
     chunk_range(p, j, &off, &len);
     const uint64_t q = p.q0 + j, s = q % p.slots, u = q / p.slots;
-    if (!wait_flags(p.full + s * kFlagStride, p.g_in, u + 1, P.timeout_ns, P.err, s_abort)) return;
-    const uint8_t *slot =
-        p.ring + s * p.slot_stride + (reinterpret_cast<uintptr_t>(p.src + off) & 15u);
+    if (!wait_flags(p.full + s * kFlagStride + r, 1, u + 1, P.timeout_ns, P.err, s_abort)) return;
     uint64_t a, b;
     slice_of(len, r, p.g_out, &a, &b);
-    copy_slice<MODE, kStagedBlock>(p.dst + off + a, slot + a, b - a, smem, P.copy_mode, P.bulk_stages);
+    copy_slice<MODE, kStagedBlock>(p.dst + off + a, lane_at(p, s, r, p.src + off), b - a, smem, P.copy_mode,
+                                   P.bulk_stages);
     release_flag(p.freef + s * kFlagStride + r, u + 1);
   }
 }
 
-__global__ void __launch_bounds__(kThreads, 4) xfer_kernel(const __grid_constant__ XferParams P) {
+__global__ void __launch_bounds__(kThreads, 3) xfer_kernel(const __grid_constant__ XferParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
   __shared__ int s_abort;
@@ -513,10 +900,151 @@ __device__ __forceinline__ void publish(uint64_t *done, uint64_t bytes, uint64_t
   }
 }
 
+// Streamed roles of the multi-rank engine (lane_stream).
+// Sender stage-in lane r of a relay or host path (A8/A9 step 1).
+struct SendProducer {
+  static constexpr bool producer = true;
+  const SendParams *P;
+  const SendParams::StagedDesc *d;
+  uint32_t r;
+  uint64_t lstride, base, region;
+  __device__ void chunk(uint32_t j, uint64_t *off, uint64_t *a, uint64_t *e) const {
+    uint64_t len;
+    chunk_of(d->bytes, P->align, d->k, j, off, &len);
+    *off += d->off;
+    slice_of(len, r, d->g, a, e);
+  }
+  __device__ uint64_t slot(uint32_t j) const {
+    const uint64_t q = d->q0 + j;
+    return d->kind == 1 ? q % P->L.slots : q % P->host_slots;
+  }
+  __device__ uint64_t gen(uint32_t j) const {
+    const uint64_t q = d->q0 + j;
+    return d->kind == 1 ? q / P->L.slots : q / P->host_slots;
+  }
+  __device__ uint8_t *lane(uint32_t j) const {
+    const uint64_t s = slot(j);
+    return d->kind == 1 ? d->ring_ctrl + P->L.ring_data + (static_cast<uint64_t>(P->me) * P->L.slots + s) * P->L.stride +
+                              r * lstride
+                        : P->host.data + s * P->host_stride + r * lstride;
+  }
+  __device__ SliceGeo geom(uint32_t j, const uint64_t *) const {
+    uint64_t off, a, e;
+    chunk(j, &off, &a, &e);
+    const uint8_t *src = P->src + off;
+    return SliceGeo{src + a, lane(j) + kLaneHdr + (reinterpret_cast<uintptr_t>(src) & 15u), e - a};
+  }
+  __device__ int wait(uint32_t j) {
+    const uint64_t *fr = d->kind == 1 ? flags_at(P->my_ctrl, P->L.relay_free, d->relay, P->L.slots, slot(j)) + r
+                                      : P->host.freef + slot(j) * kFlagStride + r;
+    return poll_flag(fr, gen(j), P->timeout_ns, P->err);
+  }
+  __device__ int fetch(uint32_t, uint64_t *) { return 1; }
+  __device__ void before_store(uint32_t j) {
+    if (d->kind != 1) return;
+    uint64_t off, a, e;
+    chunk(j, &off, &a, &e);
+    uint64_t *h = reinterpret_cast<uint64_t *>(lane(j));  // the lane header the relay forwards by
+    h[0] = P->dst;
+    h[1] = base + off + a;
+    h[2] = e - a;
+    h[3] = reinterpret_cast<uintptr_t>(P->src + off) & 15u;
+    h[4] = region;
+  }
+  __device__ void loaded(uint32_t) {}
+  __device__ void stored(uint32_t j, const uint64_t *) {
+    uint64_t *fl = d->kind == 1 ? flags_at(d->ring_ctrl, P->L.ring_full, P->me, P->L.slots, slot(j)) + r
+                                : P->host.full + slot(j) * kFlagStride + r;
+    st_release_sys(fl, gen(j) + 1);
+  }
+};
+
+// Relay forward lane r (A8 step 3): the lane header names the destination.  The
+// watcher copies it to shared memory (words: dst, region offset, len, shift, region).
+struct RelayConsumer {
+  static constexpr bool producer = false;
+  const RelayParams *P;
+  uint32_t r;
+  uint64_t lstride;
+  __device__ uint8_t *lane(uint32_t j) const {
+    const uint64_t s = (P->q0 + j) % P->L.slots;
+    return P->my_ctrl + P->L.ring_data + (static_cast<uint64_t>(P->sender) * P->L.slots + s) * P->L.stride +
+           r * lstride;
+  }
+  __device__ int wait(uint32_t j) {
+    const uint64_t q = P->q0 + j;
+    return poll_flag(flags_at(P->my_ctrl, P->L.ring_full, P->sender, P->L.slots, q % P->L.slots) + r,
+                     q / P->L.slots + 1, P->timeout_ns, P->err);
+  }
+  __device__ int fetch(uint32_t j, uint64_t *w) {
+    const uint64_t *h = reinterpret_cast<const uint64_t *>(lane(j));
+    for (int i = 0; i < 5; ++i) w[i] = ld_volatile(h + i);
+    if (w[0] >= P->L.world || w[4] >= kMaxRegions || w[3] > 15) {  // never write through a torn lane
+      atomicExch(P->err, DERR_MISMATCH);
+      return -1;
+    }
+    return 1;
+  }
+  __device__ SliceGeo geom(uint32_t j, const uint64_t *w) const {
+    return SliceGeo{lane(j) + kLaneHdr + w[3], region_base(P->my_ctrl, P->L, w[4], static_cast<uint32_t>(w[0])) + w[1],
+                    w[2]};
+  }
+  __device__ void before_store(uint32_t) {}
+  __device__ void loaded(uint32_t j) {
+    const uint64_t q = P->q0 + j;
+    st_release_sys(flags_at(P->sender_ctrl, P->L.relay_free, P->me, P->L.slots, q % P->L.slots) + r,
+                   q / P->L.slots + 1);
+  }
+  __device__ void stored(uint32_t, const uint64_t *w) {
+    red_add_release_sys(done_at(P->peer[w[0]].ctrl, P->L, P->sender), w[2]);
+  }
+};
+
+// Receiver's host-ring consumer lane r (A9 step 3); the chunk layout comes from the
+// message header in device memory.
+struct HostConsumer {
+  static constexpr bool producer = false;
+  const RecvParams *P;
+  uint32_t r;
+  uint64_t lstride, k, q0, hoff, hbytes, shift, align;
+  uint64_t *done;
+  __device__ void chunk(uint32_t j, uint64_t *off, uint64_t *a, uint64_t *e) const {
+    uint64_t len;
+    chunk_of(hbytes, align, static_cast<uint32_t>(k), j, off, &len);
+    slice_of(len, r, P->g_host, a, e);
+  }
+  __device__ SliceGeo geom(uint32_t j, const uint64_t *) const {
+    uint64_t off, a, e;
+    chunk(j, &off, &a, &e);
+    const uint64_t s = (q0 + j) % P->host_slots;
+    return SliceGeo{P->host.data + s * P->host_stride + r * lstride + kLaneHdr + ((shift + off) & 15u),
+                    P->buf + hoff + off + a, e - a};
+  }
+  __device__ int wait(uint32_t j) {
+    const uint64_t q = q0 + j;
+    return poll_flag(P->host.full + (q % P->host_slots) * kFlagStride + r, q / P->host_slots + 1, P->timeout_ns,
+                     P->err);
+  }
+  __device__ int fetch(uint32_t, uint64_t *) { return 1; }
+  __device__ void before_store(uint32_t) {}
+  __device__ void loaded(uint32_t j) {
+    const uint64_t q = q0 + j;
+    st_release_sys(P->host.freef + (q % P->host_slots) * kFlagStride + r, q / P->host_slots + 1);
+  }
+  __device__ void stored(uint32_t j, const uint64_t *) {
+    uint64_t off, a, e;
+    chunk(j, &off, &a, &e);
+    red_add_release_gpu(done, e - a);
+  }
+};
+
 // The rendezvous (P:62 analogue) runs in its own one-CTA launch ahead of the bulk
 // send kernel on the same stream: the bulk kernel's hundreds of CTAs are only
 // dispatched once the receiver's clear-to-send has arrived, so they never occupy SM
 // slots spinning on it while a receive kernel on this GPU waits for room to run.
+// The gate also rings the doorbell of every relay the message uses (engine.h): the
+// relay rank's host thread then launches the relay kernel for the message's chunks,
+// so a relay kernel only runs while the data it forwards is flowing.
 // PDL in the multi-rank engine: the gate waits for the stream's previous kernel, and
 // lets the bulk send kernel launch only once the clear-to-send has arrived (no bulk
 // CTA is ever resident during the rendezvous); send, receive and eager kernels let
@@ -526,7 +1054,8 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
   if (threadIdx.x != 0) return;
   MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
   const uint64_t t_start = globaltimer();
-  while (ld_acquire_sys(&cts->seq1) < P.seq + 1) {
+  uint64_t seen;
+  while ((seen = ld_acquire_sys(&cts->seq1)) < P.seq + 1) {
     if (globaltimer() - t_start > P.timeout_ns) {
       atomicExch(P.err, DERR_TIMEOUT);
       return;
@@ -534,7 +1063,10 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
     __nanosleep(64);
   }
   const uint64_t n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
-  const bool bad = (n != P.bytes) || (tag != P.tag);
+  // seen > seq + 1: the receiver posted a later receive into this CTS entry before
+  // this send consumed it (more than kCtsRing outstanding receives from one peer) —
+  // the entry no longer describes this message
+  const bool bad = (n != P.bytes) || (tag != P.tag) || seen != P.seq + 1;
   uint64_t host_k = 0, host_q0 = 0, host_off = 0, host_bytes = 0;
   for (uint32_t i = 0; i < P.npaths; ++i)
     if (P.sp[i].kind == 2) {
@@ -553,12 +1085,32 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
   h->d = host_off;
   h->e = host_bytes;
   h->f = reinterpret_cast<uintptr_t>(P.src + host_off) & 15u;
+  h->g = P.align;
   st_release_sys(&h->seq1, P.seq + 1);
-  if (bad) atomicExch(P.err, DERR_MISMATCH);
+  if (bad) {
+    atomicExch(P.err, DERR_MISMATCH);
+  } else {
+    for (uint32_t i = 0; i < P.npaths; ++i) {  // doorbells (relay rank's host thread)
+      const SendParams::StagedDesc &d = P.sp[i];
+      if (d.kind != 1) continue;
+      BellEntry *e = d.bell + d.m % kBellRing;
+      // co-alignment of source and target (mod 16 is the same in every process's
+      // mapping: mapped bases are >= 256-B aligned) lets the relay stream its lanes
+      const uint64_t region = ld_volatile(&cts->d);
+      const bool aligned = region < kMaxRegions &&
+                           ((reinterpret_cast<uintptr_t>(P.src) ^
+                             (reinterpret_cast<uintptr_t>(region_base(P.my_ctrl, P.L, region, P.dst)) + ld_volatile(&cts->a))) &
+                            15u) == 0;
+      e->q0 = d.q0;
+      e->k = d.k;
+      e->g = d.g | (aligned ? (1ull << 32) : 0ull);
+      st_release_sys(&e->tag, d.m + 1);
+    }
+  }
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
-__global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant__ SendParams P) {
+__global__ void __launch_bounds__(kThreads, 3) send_kernel(const __grid_constant__ SendParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
   __shared__ int s_abort;
@@ -573,8 +1125,10 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
     const uint64_t off = ld_volatile(&cts->a), n = ld_volatile(&cts->b), tag = ld_volatile(&cts->c);
     s_off = off;
     s_region = ld_volatile(&cts->d);
-    if ((n != P.bytes) || (tag != P.tag) || s_region >= kMaxRegions) s_abort = 1;  // reported by the gate
-    else s_dst = region_base(P.my_ctrl, P.L, s_region, P.dst) + off;
+    if ((n != P.bytes) || (tag != P.tag) || s_region >= kMaxRegions || ld_volatile(&cts->seq1) != P.seq + 1)
+      s_abort = 1;  // reported by the gate
+    else
+      s_dst = region_base(P.my_ctrl, P.L, s_region, P.dst) + off;
   }
   __syncthreads();
   if (s_abort) return;
@@ -592,56 +1146,61 @@ __global__ void __launch_bounds__(kThreads, 4) send_kernel(const __grid_constant
   }
   for (uint32_t i = 0; i < P.npaths; ++i) {
     const SendParams::StagedDesc &d = P.sp[i];
-    if (b < d.cta0 || b >= d.cta0 + P.g_stage) continue;
-    const uint32_t r = b - d.cta0;
+    if (b < d.cta0 || b >= d.cta0 + d.g) continue;
+    const uint32_t r = b - d.cta0;  // lane r of every slot of this path
+    const uint64_t lstride = lane_stride(P.L.slot_bytes, d.g);
+    if (P.copy_mode == 1) {  // streamed lane (source slice and lane are co-aligned)
+      SendProducer R{&P, &d, r, lstride, base, s_region};
+      lane_stream<LD_SRC>(R, d.k, dyn_smem);
+      return;
+    }
     for (uint32_t j = 0; j < d.k; ++j) {  // A8/A9 step 1
       uint64_t off, len;
-      chunk_of(d.bytes, 256, d.k, j, &off, &len);
+      chunk_of(d.bytes, P.align, d.k, j, &off, &len);
       off += d.off;
       const uint64_t q = d.q0 + j;
       uint64_t *fr, *fl;
-      uint8_t *slot;
-      uint32_t nfree;
+      uint8_t *lane;
+      uint64_t u;
       if (d.kind == 1) {
         const uint64_t s = q % P.L.slots;
-        fr = flags_at(P.my_ctrl, P.L.relay_free, d.relay, P.L.slots, s);
-        fl = flags_at(d.ring_ctrl, P.L.ring_full, P.me, P.L.slots, s);
-        slot = d.ring_ctrl + P.L.ring_data + (static_cast<uint64_t>(P.me) * P.L.slots + s) * P.L.stride;
-        nfree = P.g_stage;
+        u = q / P.L.slots;
+        fr = flags_at(P.my_ctrl, P.L.relay_free, d.relay, P.L.slots, s) + r;
+        fl = flags_at(d.ring_ctrl, P.L.ring_full, P.me, P.L.slots, s) + r;
+        lane = d.ring_ctrl + P.L.ring_data + (static_cast<uint64_t>(P.me) * P.L.slots + s) * P.L.stride + r * lstride;
       } else {
         const uint64_t s = q % P.host_slots;
-        fr = P.host.freef + s * kFlagStride;
-        fl = P.host.full + s * kFlagStride;
-        slot = P.host.data + s * P.host_stride;
-        nfree = P.g_stage;
+        u = q / P.host_slots;
+        fr = P.host.freef + s * kFlagStride + r;
+        fl = P.host.full + s * kFlagStride + r;
+        lane = P.host.data + s * P.host_stride + r * lstride;
       }
-      const uint64_t u = q / (d.kind == 1 ? P.L.slots : P.host_slots);
-      if (!wait_flags(fr, nfree, u, P.timeout_ns, P.err, &s_abort)) return;
+      if (!wait_flags(fr, 1, u, P.timeout_ns, P.err, &s_abort)) return;
       const uint8_t *src = P.src + off;
       const uint64_t shift = reinterpret_cast<uintptr_t>(src) & 15u;
-      uint8_t *data = slot + kSlotHdr + shift;
       uint64_t a, e;
-      slice_of(len, r, P.g_stage, &a, &e);
-      copy_slice<LD_SRC>(data + a, src + a, e - a, dyn_smem, P.copy_mode, P.bulk_stages);
-      if (r == 0 && threadIdx.x == 0) {
-        uint64_t *h = reinterpret_cast<uint64_t *>(slot);
+      slice_of(len, r, d.g, &a, &e);
+      copy_slice<LD_SRC, kStagedBlock>(lane + kLaneHdr + shift, src + a, e - a, dyn_smem, P.copy_mode,
+                                       P.bulk_stages);
+      if (d.kind == 1 && threadIdx.x == 0) {  // the lane header the relay forwards by
+        uint64_t *h = reinterpret_cast<uint64_t *>(lane);
         h[0] = P.dst;
-        h[1] = base + off;
-        h[2] = len;
+        h[1] = base + off + a;
+        h[2] = e - a;
         h[3] = shift;
         h[4] = s_region;
       }
-      publish(nullptr, 0, fl + r, u + 1);
+      publish(nullptr, 0, fl, u + 1);
     }
     return;
   }
 }
 
-__global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant__ RecvParams P) {
+__global__ void __launch_bounds__(kThreads, 3) recv_kernel(const __grid_constant__ RecvParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
   __shared__ int s_abort;
-  __shared__ uint64_t s_k, s_q0, s_hoff, s_hbytes, s_shift;
+  __shared__ uint64_t s_k, s_q0, s_hoff, s_hbytes, s_shift, s_align;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
   MsgEntry *hdr = entry_at(P.my_ctrl, P.L.hdr, P.src, P.seq);
@@ -672,7 +1231,7 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
     }
     return;
   }
-  // A9 step 3: host-ring consumers
+  // A9 step 3: host-ring consumers, CTA r = lane r of every host slot
   const uint32_t r = blockIdx.x - 1;
   if (!wait_word(&hdr->seq1, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
   if (threadIdx.x == 0) {
@@ -681,52 +1240,65 @@ __global__ void __launch_bounds__(kThreads, 4) recv_kernel(const __grid_constant
     s_hoff = ld_volatile(&hdr->d);
     s_hbytes = ld_volatile(&hdr->e);
     s_shift = ld_volatile(&hdr->f);
+    s_align = ld_volatile(&hdr->g);
   }
   __syncthreads();
   uint64_t *done = done_at(P.my_ctrl, P.L, P.src);
+  const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g_host);
+  if (P.copy_mode == 1 && ((reinterpret_cast<uintptr_t>(P.buf) + s_hoff) & 15u) == s_shift) {
+    // streamed lane: the host slices and their destination are co-aligned
+    HostConsumer R{&P, r, lstride, s_k, s_q0, s_hoff, s_hbytes, s_shift, s_align, done};
+    lane_stream<LD_HOST>(R, static_cast<uint32_t>(s_k), dyn_smem);
+    return;
+  }
   for (uint64_t j = 0; j < s_k; ++j) {
     const uint64_t q = s_q0 + j, s = q % P.host_slots, u = q / P.host_slots;
-    if (!wait_flags(P.host.full + s * kFlagStride, P.g_host, u + 1, P.timeout_ns, P.err, &s_abort)) return;
-    uint8_t *slot = P.host.data + s * P.host_stride;
+    if (!wait_flags(P.host.full + s * kFlagStride + r, 1, u + 1, P.timeout_ns, P.err, &s_abort)) return;
+    uint8_t *lane = P.host.data + s * P.host_stride + r * lstride;
     uint64_t off, len;
-    chunk_of(s_hbytes, 256, static_cast<uint32_t>(s_k), static_cast<uint32_t>(j), &off, &len);
+    chunk_of(s_hbytes, s_align, static_cast<uint32_t>(s_k), static_cast<uint32_t>(j), &off, &len);
     uint64_t a, e;
     slice_of(len, r, P.g_host, &a, &e);
-    copy_slice<LD_HOST>(P.buf + s_hoff + off + a, slot + kSlotHdr + s_shift + a, e - a, dyn_smem,
-                        P.copy_mode, P.bulk_stages);
+    copy_slice<LD_HOST, kStagedBlock>(P.buf + s_hoff + off + a, lane + kLaneHdr + ((s_shift + off) & 15u), e - a,
+                                      dyn_smem, P.copy_mode, P.bulk_stages);
     publish(done, e - a, P.host.freef + s * kFlagStride + r, u + 1, /*done_is_local=*/true);
   }
 }
 
-// Persistent relay (A8 step 3): CTA group s (g CTAs) forwards sender s's ring.
-__global__ void __launch_bounds__(kThreads, 4) relay_kernel(const __grid_constant__ RelayParams P) {
+// Relay (A8 step 3), one bounded launch per relayed message: CTA r forwards lane r of
+// chunks [q0, q0 + k) of the sender's ring to the destination its lane header names,
+// counts the bytes into the destination's `done` and returns the lane to the sender.
+__global__ void __launch_bounds__(kThreads, 3) relay_kernel(const __grid_constant__ RelayParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
   __shared__ uint64_t s_h[5];
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
-  const uint32_t sender = blockIdx.x / P.g, r = blockIdx.x % P.g;
-  if (sender == P.me || sender >= P.world) return;
-  // ring position survives a stop/restart (mp_calibrate stops the relay)
-  uint64_t *pos = reinterpret_cast<uint64_t *>(P.my_ctrl + P.L.relay_pos) + sender;
-  for (uint64_t q = ld_volatile(pos);; ++q) {
-    const uint64_t s = q % P.L.slots, u = q / P.L.slots;
-    uint64_t *fl = flags_at(P.my_ctrl, P.L.ring_full, sender, P.L.slots, s);
-    if (!wait_flags(fl, P.g, u + 1, 0, P.err, &s_abort, P.stop)) {
-      if (r == 0 && threadIdx.x == 0) *pos = q;
-      return;
-    }
-    uint8_t *slot = P.my_ctrl + P.L.ring_data + (static_cast<uint64_t>(sender) * P.L.slots + s) * P.L.stride;
-    if (threadIdx.x < 5) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(slot) + threadIdx.x);
+  const uint32_t r = blockIdx.x;
+  const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g);
+  if (P.copy_mode == 1 && P.aligned) {  // streamed lane (the sender found source and target co-aligned)
+    RelayConsumer R{&P, r, lstride};
+    lane_stream<LD_RING>(R, static_cast<uint32_t>(P.k), dyn_smem);
+    return;
+  }
+  for (uint64_t j = 0; j < P.k; ++j) {
+    const uint64_t q = P.q0 + j, s = q % P.L.slots, u = q / P.L.slots;
+    uint64_t *fl = flags_at(P.my_ctrl, P.L.ring_full, P.sender, P.L.slots, s) + r;
+    if (!wait_flags(fl, 1, u + 1, P.timeout_ns, P.err, &s_abort)) return;
+    uint8_t *lane =
+        P.my_ctrl + P.L.ring_data + (static_cast<uint64_t>(P.sender) * P.L.slots + s) * P.L.stride + r * lstride;
+    if (threadIdx.x < 5) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(lane) + threadIdx.x);
     __syncthreads();
     const uint32_t dst = static_cast<uint32_t>(s_h[0]);
-    const uint64_t off = s_h[1], len = s_h[2], shift = s_h[3];
-    uint64_t a, e;
-    slice_of(len, r, P.g, &a, &e);
-    copy_slice<LD_RING>(region_base(P.my_ctrl, P.L, s_h[4], dst) + off + a, slot + kSlotHdr + shift + a, e - a, dyn_smem, P.copy_mode,
-                        P.bulk_stages);
-    uint64_t *fr = flags_at(P.peer[sender].ctrl, P.L.relay_free, P.me, P.L.slots, s);
-    publish(done_at(P.peer[dst].ctrl, P.L, sender), e - a, fr + r, u + 1);
+    const uint64_t off = s_h[1], len = s_h[2], shift = s_h[3], region = s_h[4];
+    if (dst >= P.L.world || region >= kMaxRegions) {  // a torn or foreign lane: never write through it
+      if (threadIdx.x == 0) atomicExch(P.err, DERR_MISMATCH);
+      return;
+    }
+    copy_slice<LD_RING, kStagedBlock>(region_base(P.my_ctrl, P.L, region, dst) + off, lane + kLaneHdr + shift, len,
+                                      dyn_smem, P.copy_mode, kBulkStages);
+    uint64_t *fr = flags_at(P.sender_ctrl, P.L.relay_free, P.me, P.L.slots, s) + r;
+    publish(done_at(P.peer[dst].ctrl, P.L, P.sender), len, fr, u + 1);
   }
 }
 
@@ -954,7 +1526,7 @@ int launch_send(const SendParams &P, void *stream) {
   cfg.attrs = at;
   cfg.numAttrs = pdl ? 1 : 0;
   if (int e = static_cast<int>(cudaLaunchKernelEx(&cfg, send_gate_kernel, P))) return e;
-  return launch_k(pdl, send_kernel, P.nblocks, kBulkSmem, stream, P);
+  return launch_k(pdl, send_kernel, P.nblocks, kXferSmem, stream, P);
 }
 
 int launch_eager_send(const EagerParams &P, void *stream) {
@@ -966,11 +1538,11 @@ int launch_eager_recv(const EagerParams &P, void *stream) {
 }
 
 int launch_recv(const RecvParams &P, void *stream) {
-  return launch_k(P.pdl != 0, recv_kernel, P.nblocks, kBulkSmem, stream, P);
+  return launch_k(P.pdl != 0, recv_kernel, P.nblocks, kXferSmem, stream, P);
 }
 
 int launch_relay(const RelayParams &P, void *stream) {
-  relay_kernel<<<P.world * P.g, kThreads, kBulkSmem, static_cast<cudaStream_t>(stream)>>>(P);
+  relay_kernel<<<P.g, kThreads, kXferSmem, static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
 }
 
@@ -985,9 +1557,9 @@ int preload_kernels() {
   // any other engine kernel.  Force every kernel of this module to load up front.
   cudaFuncAttributes a;
   cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(recv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(relay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(recv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(relay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(direct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(direct_leg_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);

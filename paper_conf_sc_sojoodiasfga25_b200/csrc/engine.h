@@ -15,12 +15,31 @@
 #pragma once
 #include <cstdint>
 
+#ifdef __CUDACC__
+#define MPX_HD __host__ __device__
+#else
+#define MPX_HD
+#endif
+
 namespace mpx {
 
 constexpr int kMaxPaths = 16;
 constexpr int kFlagStride = 32;    // flag words per slot (max CTAs per staged group)
 constexpr int kThreads = 256;      // threads per CTA of every engine kernel
-constexpr uint32_t kSlotSlack = 256;  // bytes of slack per slot (co-alignment shift)
+// A staging slot is cut into per-lane regions, one per CTA of the stage group (see
+// lane_stride): lane r of a slot only ever holds slice r of a chunk, written by
+// stage-in CTA r and read by forward CTA r, so each lane is an independent two-stage
+// pipeline with its own full/free flag (no CTA waits for another CTA's slice).
+// Slack per slot: lanes round up (<= 144 B each for <= kFlagStride lanes).
+constexpr uint32_t kSlotSlack = 8192;
+constexpr uint32_t kLaneHdr = 64;     // per-lane header (multi-rank relay rings)
+
+// Bytes between lanes of a slot of slot_bytes payload cut into g lanes: a slice of a
+// chunk <= slot_bytes is at most ceil(slot_bytes/g) + 16 bytes (slice_of rounds its
+// ends up to 16 B), plus the <= 15-byte co-alignment shift and the lane header.
+MPX_HD inline uint64_t lane_stride(uint64_t slot_bytes, uint32_t g) {
+  return (((slot_bytes + g - 1) / g + 15) / 16) * 16 + 128;
+}
 
 enum : int32_t { DK_DIRECT = 0, DK_STAGED = 1 };
 
@@ -29,8 +48,8 @@ enum : int32_t { DERR_NONE = 0, DERR_TIMEOUT = 1, DERR_MISMATCH = 2 };
 
 struct DevPath {
   int32_t kind;          // DK_DIRECT / DK_STAGED
-  uint32_t g_in;         // direct: CTAs; staged: stage-in CTAs (<= kFlagStride)
-  uint32_t g_out;        // staged: forward CTAs (<= kFlagStride)
+  uint32_t g_in;         // direct: CTAs; staged: stage-in CTAs = lanes (<= kFlagStride)
+  uint32_t g_out;        // staged: forward CTAs (== g_in: lane r is served by CTA r of each)
   uint32_t cta0_in;      // first blockIdx.x of the direct / stage-in group
   uint32_t cta0_out;     // first blockIdx.x of the forward group
   uint32_t k;            // chunks
@@ -40,6 +59,7 @@ struct DevPath {
   uint64_t bytes;        // bytes on this path
   uint64_t align;        // chunk unit A (reading C6)
   uint64_t slot_stride;  // bytes between slots (slot_bytes + kSlotSlack)
+  uint64_t lane;         // bytes between the lanes of a slot (lane_stride(slot_bytes, g))
   const uint8_t *src;    // source + path offset
   uint8_t *dst;          // destination + path offset (local, peer or mapped)
   uint8_t *ring;         // slot 0
@@ -80,20 +100,30 @@ int launch_xfer(const XferParams &P, void *stream);
 //                        bytes, tag, region id} into the sender's control block, then waits for
 //                        its per-src byte counter `done` to reach the target; CTAs
 //                        1.. consume the message's host-ring chunks (A9 step 3).
-//   sender   (mp_send):  send kernel CTAs wait for the CTS, CTA 0 writes the message
-//                        header {seq+1, host_k, host_q0, status} into the receiver's
-//                        control block; the direct group stores into the target region
-//                        (A7), stage-in groups fill relay rings (A8 step 1) and the
-//                        host ring (A9 step 1); every byte delivered is counted into
-//                        the receiver's `done` with red.release.sys.
-//   relay    (persistent, one per rank): per sender ring, forward every landed chunk
-//                        to the destination named in the slot header (A8 step 3).
-// Slot = [kSlotHdr-byte header][data]; header = {dst rank, region offset, len, shift, region}.
+//   sender   (mp_send):  a one-CTA gate kernel waits for the CTS, writes the message
+//                        header {seq+1, host_k, host_q0, status, ...} into the
+//                        receiver's control block and rings the doorbell of every
+//                        relay the message uses; then the bulk send kernel's direct
+//                        group stores into the target region (A7), its stage-in
+//                        groups fill relay rings (A8 step 1) and the host ring (A9
+//                        step 1); every byte delivered is counted into the
+//                        receiver's `done` with red.release.sys.
+//   relay    (on demand): a host thread of the relay rank watches its doorbells (in
+//                        its shared pinned segment, written by the senders' gate
+//                        kernels over PCIe) and launches one bounded relay kernel per
+//                        relayed message range, on a per-sender stream; CTA r forwards
+//                        lane r of every chunk of the range to the destination named
+//                        in the lane header (A8 step 3), then the kernel ends.  No
+//                        kernel outlives the traffic it serves, so a device-wide
+//                        synchronisation on any rank completes.
+// Relay slot = kFlagStride-many lanes (lane_stride); lane header = {dst rank, region
+// offset of the slice, slice length, shift, region}.
 // A receive target is (region id, offset): every rank's control block holds the table
 // regions[id][rank] = base of rank's region `id` as mapped in THIS process (region 0
 // = the heaps, 1.. = mp_register), so a sender or relay resolves it locally.
 
 constexpr uint32_t kCtsRing = 64;     // outstanding messages per ordered pair
+constexpr uint32_t kBellRing = 64;    // outstanding relayed messages per (sender, relay)
 
 // Eager protocol (NEXT f4's low-latency protocol, reading C23): a message of
 // 1..kEagerMax bytes skips the rendezvous — the sender writes it, with per-CTA
@@ -105,15 +135,27 @@ constexpr uint64_t kEagerMax = 64ull << 10;
 constexpr uint32_t kEagerSlice = 8192;            // bytes per CTA (kEagerMax / 8 CTAs)
 constexpr uint32_t kEagerHdr = 256;               // {bytes, tag, flags[8]} before the data
 constexpr uint64_t kEagerStride = kEagerHdr + kEagerMax + 256;  // + co-alignment shift
-constexpr uint32_t kSlotHdr = 256;    // slot header bytes
 constexpr uint32_t kMaxRegions = 64;  // receive regions: 0 = heap, 1.. = mp_register
 
 struct MsgEntry {                      // CTS and message-header entries (64 B)
   uint64_t seq1;                       // sequence + 1 (written last, with release)
   uint64_t a, b, c;                    // CTS: region offset, bytes, tag; HDR: host_k, host_q0, status
   uint64_t d, e, f, g;                 // CTS: region id; HDR: host range message offset, host bytes,
-                                       //      src shift (mod 16)
+                                       //      src shift (mod 16), chunk unit A
 };
+
+// Doorbell of one relayed message (sender → relay rank's host thread), in the relay's
+// shared pinned segment.  Written by the sender's gate kernel; tag last (release).
+struct BellEntry {
+  uint64_t tag;                        // message index on (sender, relay) + 1
+  uint64_t q0;                         // ring sequence of the message's first chunk
+  uint64_t k;                          // chunks
+  uint64_t g;                          // lanes (stage-group CTAs); bit 32: source and
+                                       // target co-aligned mod 16
+};
+inline uint64_t bell_bytes(uint32_t world) {
+  return (static_cast<uint64_t>(world) * kBellRing * sizeof(BellEntry) + 4095) & ~uint64_t(4095);
+}
 
 struct PeerPtrs {
   uint8_t *heap;                       // peer's receive heap (mapped)
@@ -123,7 +165,8 @@ struct PeerPtrs {
 // Byte offsets inside every rank's control block (identical on all ranks).
 struct CtrlLayout {
   uint32_t world = 0, slots = 0;
-  uint64_t stride = 0;                 // relay slot stride (kSlotHdr + slot_bytes + kSlotSlack)
+  uint64_t stride = 0;                 // relay slot stride (slot_bytes + kSlotSlack)
+  uint64_t slot_bytes = 0;             // payload bytes per relay slot (lane_stride input)
   uint64_t cts = 0;                    // [world(src=receiver)][kCtsRing] MsgEntry — on the sender
   uint64_t hdr = 0;                    // [world(src=sender)][kCtsRing] MsgEntry   — on the receiver
   uint64_t done = 0;                   // [world(src)] u64, 128-B padded         — on the receiver
@@ -133,7 +176,6 @@ struct CtrlLayout {
   uint64_t host_full = 0;              // [world(sender)][slots][kFlagStride]     — on the receiver
   uint64_t host_free = 0;              // [world(receiver)][slots][kFlagStride]   — on the sender
   uint64_t probe = 0;                  // 64 B of flag words for the ε ping-pong of the predecessor
-  uint64_t relay_pos = 0;              // [world(sender)] u64: relay ring position across restarts
   uint64_t regions = 0;                // [kMaxRegions][world] u64: mapped region bases (local)
   uint64_t eager = 0;                  // [world(sender)][kEagerSlots][kEagerStride]   — on the receiver
   uint64_t eager_free = 0;             // [world(receiver)] u64, 128-B padded: slots returned — on the sender
@@ -149,8 +191,8 @@ struct HostRingPtrs {
 };
 
 struct SendParams {
-  uint32_t me, dst, nblocks, g_direct, g_stage, npaths, copy_mode, bulk_stages;
-  uint64_t seq, bytes, tag, timeout_ns;
+  uint32_t me, dst, nblocks, g_direct, npaths, copy_mode, bulk_stages, g_host;
+  uint64_t seq, bytes, tag, timeout_ns, align;
   const uint8_t *src;
   uint8_t *my_ctrl;
   uint8_t *dst_ctrl;
@@ -164,9 +206,13 @@ struct SendParams {
     uint32_t relay;          // relay rank
     uint32_t k;              // chunks
     uint32_t cta0;           // first block of the stage-in group
+    uint32_t g;              // CTAs of the stage-in group = lanes of the ring slots
+    uint32_t pad_;
     uint64_t off, bytes;     // message byte range of this path
     uint64_t q0;             // ring sequence of chunk 0
+    uint64_t m;              // relay: message index on (me, relay) (doorbell entry)
     uint8_t *ring_ctrl;      // relay's control block (relay) — full flags + ring data
+    BellEntry *bell;         // relay: the doorbell ring for (me) in the relay's segment (mapped)
   } sp[kMaxPaths];
   uint64_t direct_bytes;
   HostRingPtrs host;         // this pair's host ring (mapped)
@@ -186,13 +232,16 @@ struct RecvParams {
   HostRingPtrs host;
 };
 
+// One bounded relay launch: forward chunks [q0, q0 + k) of `sender`'s ring, g lanes
+// (grid = g CTAs, CTA r = lane r).
 struct RelayParams {
-  uint32_t me, world, g;       // g CTAs per sender ring
-  uint32_t copy_mode, bulk_stages, pad_;
+  uint32_t me, sender, g, copy_mode;
+  uint32_t aligned, pad_;      // 1: source and target co-aligned (streamed lanes)
+  uint64_t q0, k, timeout_ns;
   uint8_t *my_ctrl;
-  PeerPtrs peer[kMaxPaths];    // ctrl of every rank (self: local); targets via regions
+  uint8_t *sender_ctrl;        // the sender's control block (mapped): relay_free flags
+  PeerPtrs peer[kMaxPaths];    // ctrl of every rank (self: local): destinations' done counters
   CtrlLayout L;
-  volatile int32_t *stop;      // mapped host word: != 0 → exit
   int32_t *err;
 };
 

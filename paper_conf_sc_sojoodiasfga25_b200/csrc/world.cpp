@@ -5,12 +5,19 @@
 // heap and control block with cudaIpcGetMemHandle and maps every peer's; every rank
 // creates a POSIX shared-memory segment holding the pinned host rings of the
 // messages it receives (A9), registered mapped+portable so both the sending and the
-// receiving GPU address it; ranks >= 3 launch the persistent relay kernel (A8).
+// receiving GPU address it, preceded by the rank's relay doorbells; with world >= 3
+// every rank runs a relay service thread that launches bounded relay kernels (A8 step
+// 3) when a sender's gate kernel rings one of its doorbells.
 #include <fcntl.h>
 #include <sys/mman.h>
+#include <sys/prctl.h>
+#include <time.h>
 #include <unistd.h>
 
 #include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <thread>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -66,7 +73,8 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   CtrlLayout L;
   L.world = world;
   L.slots = slots;
-  L.stride = kSlotHdr + slot_bytes + kSlotSlack;
+  L.stride = slot_bytes + kSlotSlack;
+  L.slot_bytes = slot_bytes;
   uint64_t off = 0;
   auto take = [&](uint64_t bytes) {
     const uint64_t o = off;
@@ -81,7 +89,6 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.host_full = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.host_free = take(static_cast<uint64_t>(world) * slots * kFlagStride * 8);
   L.probe = take(64);
-  L.relay_pos = take(static_cast<uint64_t>(world) * 8);
   L.regions = take(static_cast<uint64_t>(kMaxRegions) * world * 8);
   L.eager = take(static_cast<uint64_t>(world) * kEagerSlots * kEagerStride);
   L.eager_free = take(static_cast<uint64_t>(world) * 128);
@@ -127,7 +134,7 @@ int map_segment(mp_ctx *c, int rank, bool create, uint8_t **out) {
 // fence), "free" in src's (written by dst) — so no flag is ever polled over PCIe.
 HostRingPtrs host_ring(const mp_ctx *c, int src, int dst) {
   HostRingPtrs h;
-  h.data = c->hseg[dst] + static_cast<uint64_t>(src) * c->hseg_per_src;
+  h.data = c->hseg[dst] + bell_bytes(c->world) + static_cast<uint64_t>(src) * c->hseg_per_src;
   h.full = reinterpret_cast<uint64_t *>(c->peers[dst].ctrl + c->L.host_full) +
            static_cast<uint64_t>(src) * c->slots * kFlagStride;
   h.freef = reinterpret_cast<uint64_t *>(c->peers[src].ctrl + c->L.host_free) +
@@ -211,13 +218,13 @@ int world_init(mp_ctx *c) {
     CKW(cudaMemcpy(c->ctrl + c->L.regions, row.data(), W * 8, cudaMemcpyHostToDevice));
   }
 
-  // Host rings: one segment per receiving rank, one ring per sender inside it.
-  c->host_stride = kSlotHdr + c->slot_bytes + kSlotSlack;
-  c->hseg_per_src = (static_cast<uint64_t>(c->slots) * c->host_stride +
-                     2ull * c->slots * kFlagStride * 8 + 4095) & ~uint64_t(4095);
-  c->hseg_bytes = static_cast<size_t>(c->hseg_per_src * W);
+  // One shared pinned segment per rank: its relay doorbells, then (host path) the host
+  // rings of the messages it receives, one ring per sender.
+  c->host_stride = c->slot_bytes + kSlotSlack;
+  c->hseg_per_src = (static_cast<uint64_t>(c->slots) * c->host_stride + 4095) & ~uint64_t(4095);
+  c->hseg_bytes = static_cast<size_t>(bell_bytes(W) + (c->host_path ? c->hseg_per_src * W : 0));
   c->hseg.assign(W, nullptr);
-  if (c->host_path) {
+  if (c->host_path || W >= 3) {
     if (int s = map_segment(c, c->rank, true, &c->hseg[c->rank])) return s;
     if (int s = barrier(c)) return s;
     for (int r = 0; r < W; ++r)
@@ -231,57 +238,132 @@ int world_init(mp_ctx *c) {
   c->send_seq.assign(W, 0);
   c->recv_seq.assign(W, 0);
   c->relay_q.assign(W, 0);
+  c->relay_m.assign(W, 0);
   c->host_q.assign(W, 0);
   c->done_target.assign(W, 0);
   c->eager_send_seq.assign(W, 0);
   c->eager_recv_seq.assign(W, 0);
-
-  if (W >= 3) {  // resources of the persistent relay kernel; it is started by world_start_relay
-    CKW(cudaHostAlloc(&p, 64, cudaHostAllocMapped | cudaHostAllocPortable));
-    c->stop = static_cast<int32_t *>(p);
-    *c->stop = 0;
-    CKW(cudaStreamCreateWithFlags(&c->relay_stream, cudaStreamNonBlocking));
-  }
   const int s = barrier(c);
   DBG("world_init done");
   return s;
 }
 
-// Launch the persistent relay kernel (A8 step 3).  Every allocation / free that may
-// synchronise the device (cudaFree, cudaHostAlloc, ...) must happen before this.
+// ---------------------------------------------------------------- relay service (A8 step 3)
+//
+// The relay rank's side of a GPU-staged path.  A sender's gate kernel rings a doorbell
+// in this rank's shared pinned segment (BellEntry: ring sequence q0, chunk count k,
+// lanes g) once the message's clear-to-send has arrived; this thread sees it and
+// launches one relay kernel of g CTAs for those chunks on the sender's stream (stream
+// order keeps a sender's ring positions in order).  Every relay kernel ends when its
+// chunks are forwarded, so nothing runs on this GPU without traffic to serve, and a
+// device-wide synchronisation (torch.cuda.synchronize, cudaDeviceSynchronize, lazy
+// module loading) completes on every rank.  The thread spins while traffic is recent
+// and polls every ~20 µs after 50 ms of quiet.
+struct RelayService {
+  std::thread th;
+  std::atomic<bool> stop{false};
+  std::atomic<int> error{0};           // cudaError_t of a failed relay launch (sticky)
+  std::atomic<uint64_t> launches{0};
+  std::vector<cudaStream_t> streams;   // [world(sender)]
+  std::vector<uint64_t> next;          // [world(sender)] next doorbell index
+  BellEntry *bells = nullptr;          // this rank's doorbells [world(sender)][kBellRing]
+};
+
+namespace {
+void relay_loop(mp_ctx *c, RelayService *S) {
+  cudaSetDevice(c->device);
+  prctl(PR_SET_TIMERSLACK, 1000UL);  // 1 µs: the idle poll's sleep stays short
+  RelayParams base{};
+  base.me = static_cast<uint32_t>(c->rank);
+  base.copy_mode = c->copy_mode;
+  base.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  base.my_ctrl = c->ctrl;
+  for (int r = 0; r < c->world; ++r) base.peer[r] = c->peers[r];
+  base.L = c->L;
+  base.err = c->d_err;
+  auto last = std::chrono::steady_clock::now();
+  while (!S->stop.load(std::memory_order_acquire)) {
+    bool any = false;
+    for (int s = 0; s < c->world; ++s) {
+      if (s == c->rank) continue;
+      for (;;) {
+        BellEntry *e = S->bells + static_cast<uint64_t>(s) * kBellRing + S->next[s] % kBellRing;
+        if (__atomic_load_n(&e->tag, __ATOMIC_ACQUIRE) != S->next[s] + 1) break;
+        RelayParams P = base;
+        P.sender = static_cast<uint32_t>(s);
+        P.sender_ctrl = c->peers[s].ctrl;
+        P.q0 = __atomic_load_n(&e->q0, __ATOMIC_RELAXED);
+        P.k = __atomic_load_n(&e->k, __ATOMIC_RELAXED);
+        const uint64_t g = __atomic_load_n(&e->g, __ATOMIC_RELAXED);
+        P.g = static_cast<uint32_t>(g & 0xffffffffu);
+        P.aligned = static_cast<uint32_t>((g >> 32) & 1u);
+        if (P.g < 1 || P.g > static_cast<uint32_t>(kFlagStride)) {
+          S->error.store(static_cast<int>(cudaErrorInvalidValue));
+        } else if (int rc = launch_relay(P, S->streams[s])) {
+          S->error.store(rc);
+        }
+        S->launches.fetch_add(1, std::memory_order_relaxed);
+        S->next[s] += 1;
+        any = true;
+      }
+    }
+    const auto now = std::chrono::steady_clock::now();
+    if (any) {
+      last = now;
+    } else if (now - last > std::chrono::milliseconds(50)) {
+      timespec ts{0, 20000};
+      nanosleep(&ts, nullptr);
+    }
+  }
+}
+}  // namespace
+
 int world_start_relay(mp_ctx *c) {
-  const char *no_relay = std::getenv("MPX_NO_RELAY");  // diagnostics: no relay kernel
-  if (c->world < 3 || c->relay_running || (no_relay && no_relay[0] == '1')) return MP_OK;
-  *reinterpret_cast<volatile int32_t *>(c->stop) = 0;
-  RelayParams R{};
-  R.me = static_cast<uint32_t>(c->rank);
-  R.world = static_cast<uint32_t>(c->world);
-  R.g = static_cast<uint32_t>(c->relay_ctas);
-  R.copy_mode = c->copy_mode;
-  R.bulk_stages = bulk_stages_for(c->slot_bytes);
-  R.my_ctrl = c->ctrl;
-  for (int r = 0; r < c->world; ++r) R.peer[r] = c->peers[r];
-  R.L = c->L;
-  R.stop = c->stop;
-  R.err = c->d_err;
-  if (int e = launch_relay(R, c->relay_stream))
-    return wfail(c, MP_ERR_CUDA, std::string("relay launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
-  c->launches += 1;
-  c->relay_running = true;
-  DBG("relay launched");
+  const char *no_relay = std::getenv("MPX_NO_RELAY");  // diagnostics: no relay service
+  if (c->world < 3 || c->relay_svc || (no_relay && no_relay[0] == '1')) return MP_OK;
+  RelayService *S = new RelayService();
+  S->streams.assign(c->world, nullptr);
+  S->next.assign(c->world, 0);
+  S->bells = reinterpret_cast<BellEntry *>(c->hseg[c->rank]);
+  for (int r = 0; r < c->world; ++r) {
+    if (r == c->rank) continue;
+    cudaError_t e = cudaStreamCreateWithFlags(&S->streams[r], cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+      for (cudaStream_t st : S->streams)
+        if (st) cudaStreamDestroy(st);
+      delete S;
+      return wfail(c, MP_ERR_CUDA, std::string("relay stream: ") + cudaGetErrorString(e));
+    }
+  }
+  c->relay_svc = S;
+  S->th = std::thread(relay_loop, c, S);
+  DBG("relay service started");
   return MP_OK;
 }
 
-// Stop it (no transfers may be in flight); its ring positions are kept in the
-// control block, so a restart continues where it stopped.
+// Stop the service thread (finalize) and wait for every relay kernel it launched.
 int world_stop_relay(mp_ctx *c) {
-  if (!c->relay_running) return MP_OK;
-  *reinterpret_cast<volatile int32_t *>(c->stop) = 1;
-  CKW(cudaStreamSynchronize(c->relay_stream));
-  c->relay_running = false;
-  DBG("relay stopped");
+  RelayService *S = c->relay_svc;
+  if (!S) return MP_OK;
+  S->stop.store(true, std::memory_order_release);
+  if (S->th.joinable()) S->th.join();
+  for (cudaStream_t st : S->streams)
+    if (st) {
+      cudaStreamSynchronize(st);
+      cudaStreamDestroy(st);
+    }
+  c->relay_launches_done += S->launches.load();
+  c->relay_svc = nullptr;
+  delete S;
+  DBG("relay service stopped");
   return MP_OK;
 }
+
+uint64_t world_relay_launches(const mp_ctx *c) {
+  return c->relay_launches_done + (c->relay_svc ? c->relay_svc->launches.load() : 0);
+}
+
+int world_relay_error(const mp_ctx *c) { return c->relay_svc ? c->relay_svc->error.load() : 0; }
 
 int world_finalize(mp_ctx *c) {
   int st = MP_OK;
@@ -302,10 +384,6 @@ int world_finalize(mp_ctx *c) {
       munmap(s, c->hseg_bytes);
     }
   c->hseg.clear();
-  if (c->relay_stream) cudaStreamDestroy(c->relay_stream);
-  c->relay_stream = nullptr;
-  if (c->stop) cudaFreeHost(c->stop);
-  c->stop = nullptr;
   if (c->ctrl) cudaFree(c->ctrl);
   c->ctrl = nullptr;
   return st;
@@ -375,16 +453,20 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   P.L = c->L;
   P.host_stride = c->host_stride;
   P.host_slots = static_cast<uint32_t>(c->slots);
-  P.g_stage = static_cast<uint32_t>(c->relay_ctas);
+  P.align = c->opts.align;
   P.copy_mode = c->copy_mode;
   P.pdl = c->pdl_world;
   P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
   if (c->host_path) P.host = host_ring(c, c->rank, dst);
   P.direct_bytes = cfg.bytes[0];
+  // Every staged path gets a stage group of relay_ctas CTAs (= lanes of its ring
+  // slots; the receiver's host consumers and Step 1's leg timing use the same count).
+  const uint32_t g_stage = static_cast<uint32_t>(c->relay_ctas);
+  P.g_host = g_stage;
   const int cap = std::max(1, c->per_sm * c->sms);
   uint32_t staged = 0;
   for (int i = 1; i < cfg.npaths; ++i)
-    if (cfg.bytes[i]) staged += P.g_stage;
+    if (cfg.bytes[i]) staged += g_stage;
   P.g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged));
   uint32_t next = P.g_direct;
   uint64_t off = cfg.bytes[0];
@@ -397,13 +479,17 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
       d.kind = cfg.path[i].kind == MP_PATH_HOST ? 2 : 1;
       d.relay = d.kind == 1 ? static_cast<uint32_t>(cfg.path[i].via) : 0u;
       d.k = cfg.chunks[i];
+      d.g = g_stage;
       d.cta0 = next;
-      next += P.g_stage;
+      next += d.g;
       d.off = off;
       d.bytes = b;
       if (d.kind == 1) {
+        if (!c->hseg[d.relay]) return wfail(c, MP_ERR_TOPOLOGY, "relay rank has no doorbell segment");
         d.q0 = c->relay_q[d.relay];
         d.ring_ctrl = c->peers[d.relay].ctrl;
+        d.m = c->relay_m[d.relay];
+        d.bell = reinterpret_cast<BellEntry *>(c->hseg[d.relay]) + static_cast<uint64_t>(c->rank) * kBellRing;
         advance.emplace_back(static_cast<int>(d.relay), d.k);
       } else {
         d.q0 = c->host_q[dst];
@@ -419,10 +505,12 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   c->launches += 2;  // rendezvous gate + bulk send kernel
   c->send_seq[dst] += 1;
   for (auto &a : advance) {
-    if (a.first < 0)
+    if (a.first < 0) {
       c->host_q[dst] += a.second;
-    else
+    } else {
       c->relay_q[a.first] += a.second;
+      c->relay_m[a.first] += 1;
+    }
   }
   note_stream(c, static_cast<cudaStream_t>(stream));
   return MP_OK;
@@ -518,7 +606,8 @@ struct RegInfo {
 int write_region_row(mp_ctx *c, int id, const std::vector<uint64_t> &row) {
   CKW(cudaMemcpy(c->ctrl + c->L.regions + static_cast<uint64_t>(id) * c->world * 8, row.data(),
                  c->world * 8, cudaMemcpyHostToDevice));
-  // a pageable copy may return before its DMA lands; the relay kernel is stopped here
+  // a pageable copy may return before its DMA lands (registration is collective and
+  // no transfer is in flight, so no relay kernel runs: the device goes idle)
   CKW(cudaDeviceSynchronize());
   return MP_OK;
 }
@@ -571,8 +660,6 @@ int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
                           : wfail(c, all[r].status, "mp_register failed on rank " + std::to_string(r));
   }
   if (rid < 0) return wfail(c, MP_ERR_NOMEM, "mp_register: region table full");
-  const bool relay = c->relay_running;
-  if (int s = world_stop_relay(c)) return s;
   mp_ctx::Region g;
   g.used = true;
   g.base = static_cast<uint8_t *>(bytes ? buf : nullptr);
@@ -613,8 +700,6 @@ int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
     for (int r = 0; r < W; ++r)
       if (g.maps[r]) unmap(c, r, g.maps[r]);
   }
-  if (relay)
-    if (int s = world_start_relay(c)) return s;
   // every rank's table holds the row before anyone sends into the region
   if (int s = barrier(c)) return s;
   return st;
@@ -632,21 +717,18 @@ int world_deregister(mp_ctx *c, int id) {
   if (int s = allgather(c, &me, all.data(), sizeof(RegInfo))) return s;
   for (int r = 0; r < W; ++r)
     if (all[r].id != id) return wfail(c, MP_ERR_STATE, "mp_register / mp_deregister not called collectively");
-  const bool relay = c->relay_running;
-  if (int s = world_stop_relay(c)) return s;
   int st = write_region_row(c, id, std::vector<uint64_t>(W, 0));
   for (int r = 0; r < W; ++r)
     if (c->regions[id].maps[r]) unmap(c, r, c->regions[id].maps[r]);
   c->regions[id] = mp_ctx::Region{};
-  if (relay)
-    if (int s = world_start_relay(c)) return s;
   if (int s = barrier(c)) return s;
   return st;
 }
 
 int world_sync(mp_ctx *c) {
-  // Never cudaDeviceSynchronize here: the persistent relay kernel never ends.
   for (cudaStream_t s : c->streams) CKW(cudaStreamSynchronize(s));
+  if (int e = world_relay_error(c))
+    return wfail(c, MP_ERR_CUDA, std::string("relay launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   int32_t e = 0;
   CKW(cudaMemcpy(&e, c->d_err, sizeof(e), cudaMemcpyDeviceToHost));
   if (e == DERR_TIMEOUT) return wfail(c, MP_ERR_TIMEOUT, "a device-side wait timed out");

@@ -29,6 +29,7 @@ def main():
     src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()
     ctx = mdist.context_from_dist(device=dev, heap_bytes=n + 64 * MiB, timeout_s=30.0,
+                                  calibrate=os.environ.get("DIAG_CALIBRATE", "1") == "1",
                                   relay_ctas=int(os.environ.get("DIAG_CTAS", "16")),
                                   slots=int(os.environ.get("DIAG_SLOTS", "4")))
     ps = ctx.paths(0, 1)
@@ -36,12 +37,22 @@ def main():
     cases = {"direct": ([n] + [0] * (len(ps) - 1), None)}
     hb = [0] * len(ps)
     hb[-1] = n
-    for k in (2, 4, 8, 16):        # 64 MiB over 32 MiB slots needs k >= 2
+    kmin = -(-n // (32 * MiB - 512))  # chunks must fit the 32 MiB slots
+    for k in sorted({max(kmin, k) for k in (2, 4, 8, 16)}):
         cases[f"host_k{k}"] = (hb, k)
     if world >= 3:
         rb = [0] * len(ps)
         rb[1] = n
-        cases["relay"] = (rb, None)
+        for k in sorted({max(kmin, k) for k in (4, 8, 16)}):
+            cases[f"relay_k{k}"] = (rb, k)
+    _, prm, _ = ctx.get_model(0, 1)
+
+    def ceiling(nb):
+        # the stage-group ceiling of a staged path alone: the slower of its two legs as
+        # Step 1 timed them (plain copies with the stage group's CTAs)
+        i = next((j for j, b in enumerate(nb) if b), 0)
+        return None if i == 0 else min(prm[i]["beta"], prm[i]["beta2"]) / 1e9
+
     for name, (nb, kf) in cases.items():
         ks = [1] + [((kf or max(1, b // (8 * MiB))) if b else 0) for b in nb[1:]]
         cfg = ctx.make_config(nb, ks, 0, 1)
@@ -62,8 +73,13 @@ def main():
         out = [None] * world
         dist.all_gather_object(out, (rank, ms, wall))
         if rank == 0:
-            print(json.dumps({"case": name, "ctas": os.environ.get("DIAG_CTAS", "16"), "slots": os.environ.get("DIAG_SLOTS", "4"), "bytes": nb, "chunks": ks, "per_msg_ms": {r: m / K for r, m, _ in out},
-                              "GBps": n * K / (max(m for _, m, _ in out) * 1e-3) / 1e9}), flush=True)
+            gbs = n * K / (max(m for _, m, _ in out) * 1e-3) / 1e9
+            ce = ceiling(nb)
+            print(json.dumps({"case": name, "ctas": os.environ.get("DIAG_CTAS", "16"),
+                              "slots": os.environ.get("DIAG_SLOTS", "4"), "bytes": nb, "chunks": ks,
+                              "per_msg_ms": {r: m / K for r, m, _ in out}, "GBps": gbs,
+                              "stage_group_ceiling_GBps": ce,
+                              "frac_of_stage_group_ceiling": gbs / ce if ce else None}), flush=True)
     ctx.sync()
     if buf:
         ctx.free(buf)

@@ -434,6 +434,70 @@ def scenario_coll(rank, world):
     c.close()
 
 
+def scenario_devsync(rank, world):
+    """The relay needs no idle device: relay kernels are launched
+    per relayed message by the relay rank's doorbell thread and end with it, so every
+    rank may device-synchronise (torch.cuda.synchronize), allocate and load new CUDA
+    kernels at any time after mp_init — here between messages and, on the relay rank,
+    while a relayed message is in flight.  Payloads bit-exact against the oracle."""
+    import numpy as np
+
+    import synth
+    from oracle import transfer as X
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                timeout_s=60.0, calibrate=False)
+    # CUDA work created only now, after mp_init: a fresh allocation, a generator kernel
+    src_buf = torch.empty(8 * MiB, dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    ps = c.paths(0, 1)
+    np_ = len(ps)
+    n = 6 * MiB + 4099
+    for i in range(4):
+        nb = [0] * np_
+        ks = [1] + [0] * (np_ - 1)
+        if i % 2 == 0:       # every relay alone, k = 7
+            for j in range(1, np_ - 1):
+                nb[j] = (n // (np_ - 2)) // 256 * 256
+                ks[j] = 7
+            nb[-2] += n - sum(nb)
+        else:                # direct + relays + host
+            for j in range(1, np_):
+                nb[j] = 1 * MiB
+                ks[j] = 3
+            nb[0] = n - sum(nb)
+        host = synth.payload(n, 300 + i)
+        if rank == 0:
+            src = src_buf[:n]
+            src.copy_(torch.from_numpy(host))
+            torch.cuda.synchronize()
+            c.send(src, n, 1, tag=7, cfg=c.make_config(nb, ks, 0, 1), stream=stream)
+        elif rank == 1:
+            p = c.alloc(n)
+            c.recv(p, n, 0, tag=7, stream=stream)
+        else:
+            # the relay rank device-synchronises while the message may be in flight
+            # and launches a kernel it never ran before
+            torch.cuda.synchronize()
+            x = torch.randint(0, 256, (1 << 20,), dtype=torch.uint8, device="cuda",
+                              generator=torch.Generator(device="cuda").manual_seed(i))
+            assert int(x.sum().item()) > 0
+        torch.cuda.synchronize()   # every rank, device-wide, between messages
+        if rank == 1:
+            exp = np.zeros(n, dtype=np.uint8)
+            X.replay(host, nb, ks, [k for k, _ in ps], 256, exp)
+            assert np.array_equal(mp.as_tensor(p, n).cpu().numpy(), exp), f"message {i} mismatch"
+            c.free(p)
+        c.sync()
+        dist.barrier()
+    if rank >= 2:
+        assert c.launches() >= 4, c.launches()   # one relay kernel per relayed message
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
@@ -443,7 +507,7 @@ def main():
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
          "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
-         "eager": scenario_eager}[scen](rank, world)
+         "eager": scenario_eager, "devsync": scenario_devsync}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

@@ -101,3 +101,14 @@ def test_multirank_eager_protocol(world):
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(world, "eager", timeout=400)
+
+
+@pytest.mark.gpu
+def test_multirank_device_sync_with_relays():
+    # relay kernels are bounded launches (doorbell thread), so
+    # torch.cuda.synchronize() between messages and during a relayed message is safe
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(3, "devsync", timeout=400)
