@@ -3,22 +3,26 @@
 "P2P GB/s vs msg size (% of path roofline); model-vs-sweep optimum error %").
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl mpx|reference]
-                    [--size BYTES] [--mode b200|paper]
+                    [--size BYTES] [--mode b200|paper] [--workload config3|config5]
 
 One *step* = one message through the whole hot path: mp_select (Alg 1, cached after
-the first call — §8(a) A1-A6) and one fused multi-path transfer launch (A7 direct,
-A8 relay rings, A9 pinned-host PCIe, A10 completion).
+the first call — §8(a) A1-A6) and the transfer launches (A7 direct, A8 relays, A9
+pinned-host PCIe, A10 completion).
 
 N = 1 (default): BASELINE.json config 3 — 1 GiB, direct + 6 relays + pinned host —
 on the single-GPU loopback engine (the relay rings stand in for the intermediate
 GPUs; the host leg is real PCIe); the config is the B200-mode model's pick after an
 init-time calibration (Step 1).  Inputs are 1 GiB (> 126 MB L2), so no flush.
-N > 1 (torchrun): config 5, disjoint pairs (2i ↔ 2i+1) exchanging one 256 MiB
-message each way per step through the multi-rank engine, all pairs concurrently
-("scaling": "weak"; value = bytes moved by all ranks / max-over-ranks time).
+config.selected names the split that executed.
+N > 1 (torchrun): config 3 proper — one 1 GiB message GPU0 → GPU1 over the direct
+NVLink path, the relays GPU2..GPU{N-1} and the pinned-host path ("scaling":
+"strong"; value = GPU0→GPU1 payload GB/s, max-over-ranks device time), with NCCL
+send/recv and copy-engine peer-copy baselines on the same pair, every path alone,
+and the roofline against the source GPU's NVLink egress + PCIe.  --workload
+config5: disjoint pairs (2i ↔ 2i+1) exchanging 256 MiB each way, every GPU busy.
 
 --impl reference: the CPU oracle (oracle/, fp64 model + memcpy replay) on a bounded
-sample of the same workload, rank 0 only.
+sample of the same workload, one piece per host core, rank 0 only.
 """
 from __future__ import annotations
 
@@ -126,42 +130,90 @@ def hbm_bytes(d):
     return 2 * sum(nb) + 2 * relay
 
 
-def cpu_oracle_run(n, cfg_d, params, budget_s=12.0, sample=256 * MiB):
-    """Time the oracle as it stands (fp64 select + memcpy replay through the split) on a
-    bounded sample of the workload.  Returns (GB/s, description, threads)."""
-    import numpy as np
-    import synth
-    from oracle import model as OM
-    from oracle import transfer as OX
+def host_cpu():
+    """(threads this process may run on, CPU model) of the host."""
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+    model = "unknown"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return cores, model
+
+
+def _oracle_split(cfg_d, sample, n):
+    """The selected split scaled to a sample of `sample` bytes (same θ, same k)."""
     scale = sample / n
     nb = [int(b * scale) // 256 * 256 for b in cfg_d["bytes"]]
     nb[0] += sample - sum(nb)
-    kinds = [k for k, _ in cfg_d["paths"]]
     ch = [max(1, min(c, max(1, b // 256))) if b else 0 for b, c in zip(nb, cfg_d["chunks"])]
     ch[0] = 1
-    src = synth.payload(sample, 0)
-    dst = np.zeros(sample, dtype=np.uint8)
+    return nb, ch
+
+
+def cpu_oracle_run(n, cfg_d, params, budget_s=8.0, sample=256 * MiB):
+    """Time the oracle as it stands (fp64 Alg 1 select + numpy memcpy replay through the
+    split; never tuned) on a bounded sample of the workload: single-threaded, then on
+    every host core (the sample cut into one piece per core, each piece replayed by
+    its own thread through the same split — numpy releases the GIL in the copies).
+    Returns the cpu_baseline dict (value = the all-core rate)."""
+    import numpy as np
+    from concurrent.futures import ThreadPoolExecutor
+
+    import synth
+    from oracle import model as OM
+    from oracle import transfer as OX
+    kinds = [k for k, _ in cfg_d["paths"]]
     paths = [OM.Path(kind=k, via=v, **{f: (p[f] if not (k == 0 and f == "beta2") else float("inf"))
                                         for f in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")})
              for (k, v), p in zip(cfg_d["paths"], params)]
-    t0 = time.perf_counter()
-    reps = 0
-    while True:
-        OM.select(sample, paths, OM.Options(mode=OM.B200))
-        OX.replay(src, nb, ch, kinds, 256, dst)
-        reps += 1
-        if time.perf_counter() - t0 > budget_s or reps >= 50:
-            break
-    dt = time.perf_counter() - t0
-    assert np.array_equal(dst, src)
-    return sample * reps / dt / 1e9, f"{reps} x {sample >> 20} MiB of the {n >> 20} MiB split (same θ, k)", 1
+    cores, model = host_cpu()
+
+    def rate(threads):
+        piece = sample // threads // 256 * 256
+        nb, ch = _oracle_split(cfg_d, piece, n)
+        srcs = [synth.payload(piece, t) for t in range(threads)]
+        dsts = [np.zeros(piece, dtype=np.uint8) for _ in range(threads)]
+
+        def one(t):
+            OM.select(piece, paths, OM.Options(mode=OM.B200))
+            OX.replay(srcs[t], nb, ch, kinds, 256, dsts[t])
+
+        with ThreadPoolExecutor(threads) as ex:
+            list(ex.map(one, range(threads)))          # warm (page faults)
+            t0 = time.perf_counter()
+            reps = 0
+            while True:
+                list(ex.map(one, range(threads)))
+                reps += 1
+                if time.perf_counter() - t0 > budget_s / 2 or reps >= 50:
+                    break
+            dt = time.perf_counter() - t0
+        assert all(np.array_equal(d, s_) for d, s_ in zip(dsts, srcs))
+        return piece * threads * reps / dt / 1e9, reps, piece
+
+    v1, r1, p1 = rate(1)
+    vN, rN, pN = rate(cores) if cores > 1 else (v1, r1, p1)
+    return {"value": vN, "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "sample": f"all cores: {rN} x {cores} pieces of {pN >> 20} MiB; single thread: {r1} x {p1 >> 20} MiB; "
+                      f"each piece the {n >> 20} MiB split scaled (same θ, k), fp64 select + numpy replay",
+            "single_thread_GBps": v1, "cpu_model": model}
 
 
 def run_reference(args):
+    """--impl reference: the CPU oracle as it stands (fp64 Alg 1 + numpy memcpy replay of
+    the config-3 split), one bounded sample per step cut into one piece per host core
+    (a thread each), rank 0 only."""
     world, rank, _ = dist_env()
     if rank != 0:
         return 0
     import numpy as np
+    from concurrent.futures import ThreadPoolExecutor
+
     import synth
     from oracle import model as OM
     from oracle import transfer as OX
@@ -170,48 +222,368 @@ def run_reference(args):
     paths = [OM.Path(**t) for t in tbl]
     opts = OM.Options(mode=OM.B200 if args.mode == "b200" else OM.PAPER, slot_bytes=32 * MiB - 512)
     cfg = OM.select(n, paths, opts, OM.Port(4e-6, 6.5e12))
+    cores, model = host_cpu()
     sample = min(n, 32 * MiB)
-    scale = sample / n
-    nb = [int(b * scale) // 256 * 256 for b in cfg.bytes]
-    nb[0] += sample - sum(nb)
-    ch = [max(1, min(c, max(1, b // 256))) if b else 0 for b, c in zip(nb, cfg.chunks)]
-    ch[0] = 1
+    piece = sample // cores // 256 * 256
+    nb, ch = _oracle_split({"bytes": cfg.bytes, "chunks": cfg.chunks}, piece, n)
     kinds = [t["kind"] for t in tbl]
-    src = synth.payload(sample, 0)
-    dst = np.zeros(sample, dtype=np.uint8)
+    srcs = [synth.payload(piece, t) for t in range(cores)]
+    dsts = [np.zeros(piece, dtype=np.uint8) for _ in range(cores)]
 
-    def step():
-        OM.select(sample, paths, opts, OM.Port(4e-6, 6.5e12))
-        OX.replay(src, nb, ch, kinds, 256, dst)
+    def one(t):
+        OM.select(piece, paths, opts, OM.Port(4e-6, 6.5e12))
+        OX.replay(srcs[t], nb, ch, kinds, 256, dsts[t])
 
-    for _ in range(args.warmup):
-        step()
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        step()
-    dt = time.perf_counter() - t0
-    v = sample * args.steps / dt / 1e9
-    desc = f"{sample >> 20} MiB per step of the {n >> 20} MiB config-3 split (numpy memcpy replay + fp64 select)"
+    with ThreadPoolExecutor(cores) as ex:
+        def step():
+            list(ex.map(one, range(cores)))
+
+        for _ in range(args.warmup):
+            step()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            step()
+        dt = time.perf_counter() - t0
+    assert all(np.array_equal(d, s_) for d, s_ in zip(dsts, srcs))
+    v = piece * cores * args.steps / dt / 1e9
+    desc = (f"{cores} pieces x {piece >> 20} MiB per step (one thread per host core) of the {n >> 20} MiB "
+            f"config-3 split (numpy memcpy replay + fp64 select)")
     line = {"metric": METRIC, "value": v, "unit": "GB/s", "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
-            "data": "synthetic", "config": workload_config(args, world),
-            "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": desc},
+            "higher_is_better": True, "scaling": "weak" if world == 1 else "strong", "vs_baseline": None,
+            "dtype": "u8", "data": "synthetic", "config": workload_config(args, world),
+            "cpu_baseline": {"value": v, "unit": "GB/s", "cores": cores, "kind": "oracle", "sample": desc,
+                             "cpu_model": model},
             "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
 
 
-def workload_config(args, world):
+def split_label(d):
+    """The executed split in words, e.g. "direct-only" or
+    "direct 61.2% + relays 2,3 38.8% (k 8,8)"."""
+    n = sum(d["bytes"]) or 1
+    used = [(k, v, b, c) for (k, v), b, c in zip(d["paths"], d["bytes"], d["chunks"]) if b]
+    if len(used) == 1 and used[0][0] == 0:
+        return "direct-only"
+    parts = []
+    for kind, name in ((0, "direct"), (1, "relays"), (2, "host")):
+        sel = [(v, b, c) for k, v, b, c in used if k == kind]
+        if not sel:
+            continue
+        share = 100.0 * sum(b for _, b, _ in sel) / n
+        if kind == 0:
+            parts.append(f"direct {share:.1f}%")
+        elif kind == 1:
+            parts.append(f"relays {','.join(str(v) for v, _, _ in sel)} {share:.1f}% "
+                         f"(k {','.join(str(c) for _, _, c in sel)})")
+        else:
+            parts.append(f"host {share:.1f}% (k {sel[0][2]})")
+    return " + ".join(parts)
+
+
+def workload_config(args, world, d=None):
+    if world > 1 and args.workload == "config5":
+        return {"workload": f"config5 (disjoint pairs, both directions): {world // 2} pairs 2i<->2i+1, "
+                            f"{args.size >> 20} MiB per message, direct + relays + pinned host, model-selected",
+                "msg_bytes": args.size, "mode": args.mode, "parallelism": f"pairs{world // 2}x2dir",
+                "selected": split_label(d) if d else None,
+                "l2": "messages >= 126 MB L2 (no flush)" if args.size >= 128 * MiB else "no flush"}
+    if world > 1:
+        return {"workload": f"config3: {args.size >> 20} MiB GPU0->GPU1, direct + relays GPU2..GPU{world - 1} "
+                            f"+ pinned-host PCIe, {args.mode}-mode model-selected split"
+                            if world > 2 else
+                            f"config3 at N=2: {args.size >> 20} MiB GPU0->GPU1, direct + pinned-host PCIe "
+                            f"(no relay GPU), {args.mode}-mode model-selected split",
+                "msg_bytes": args.size, "mode": args.mode, "paths": f"direct+{world - 2}relay+host",
+                "selected": split_label(d) if d else None,
+                "parallelism": f"p2p-1pair+{world - 2}relays",
+                "l2": "message 1 GiB > 126 MB L2 (no flush)" if args.size >= 128 * MiB else "no flush"}
     return {"workload": "config3: 1 GiB GPU0->GPU0 loopback, direct + 6 relay rings + pinned-host PCIe, "
                         "B200-mode model-selected split" if args.size == GiB else
             f"{args.size} B loopback, direct + 6 relay rings + pinned host, model-selected",
-            "msg_bytes": args.size, "mode": args.mode, "paths": "direct+6relay+host",
+            "msg_bytes": args.size, "mode": args.mode, "paths": "direct+6relay+host (available)",
+            "selected": split_label(d) if d else None,
             "l2": "inputs 1 GiB > 126 MB L2 (no flush)", "parallelism": f"replicas{world}"}
 
 
+def p2p_roles(world):
+    """Config 3 on N GPUs (BASELINE.json configs[2]; P:352's 2_GPUs / 3_GPUs setups):
+    rank 0 sends one message to rank 1; ranks 2..N-1 are the relay GPUs; the host
+    path is the pinned-host PCIe path."""
+    return ["sender" if r == 0 else "receiver" if r == 1 else "relay" for r in range(world)]
+
+
+def p2p_plan(ctx, world, n, mode):
+    """Roles and the model's config for config 3 (every rank computes the same)."""
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    ctx.set_options(mode=mp.MP_MODEL_B200 if mode == "b200" else mp.MP_MODEL_PAPER)
+    return p2p_roles(world), ctx.select(0, 1, n)
+
+
 def run_world(args, world, rank, local):
-    """N > 1 (torchrun, one process per GPU): BASELINE.json config 5, SURVEY §8(d)'s
+    if args.workload == "config5":
+        return run_world_pairs(args, world, rank, local)
+    return run_world_p2p(args, world, rank, local)
+
+
+def _gather_max(x):
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(x)], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t[0])
+
+
+def _gather_sum(x):
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(x)], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t[0])
+
+
+def run_world_p2p(args, world, rank, local):
+    """N > 1 (torchrun, one process per GPU), the primary multi-GPU line: BASELINE.json
+    config 3 — one message of --size bytes (default 1 GiB) from GPU0 to GPU1, split by
+    the model (Alg 1, B200 mode after the collective Step-1 calibration) over the
+    direct NVLink path, the relays GPU2..GPU{N-1} and the pinned-host PCIe path (P:352's
+    2_GPUs / 3_GPUs / 3_GPUs_w_host setups grown to N GPUs).  "scaling": "strong" — the
+    message is fixed and N adds relay GPUs.  value = payload GB/s GPU0 → GPU1 over K
+    back-to-back messages, max-over-ranks device time.  Baselines on the same pair:
+    NCCL send/recv (before mp_init) and a copy-engine peer copy (cudaMemcpyAsync into
+    the IPC-mapped receive buffer — what cudaMemcpyPeerAsync does).  Bootstrap and
+    reductions use gloo on the CPU."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+
+    dist.init_process_group("gloo")
+    same_gpu = os.environ.get("MPX_BENCH_SAME_GPU") == "1"   # 1-GPU smoke of this path (MPS)
+    dev = 0 if same_gpu else local
+    torch.cuda.set_device(dev)
+    n = args.size
+    roles = p2p_roles(world)
+    role = roles[rank]
+    s_tx, s_rx = torch.cuda.Stream(), torch.cuda.Stream()
+    src = expect = None
+    if role == "sender":
+        src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                            generator=torch.Generator(device="cuda").manual_seed(20251116))
+    if role == "receiver":
+        expect = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                               generator=torch.Generator(device="cuda").manual_seed(20251116))
+    torch.cuda.synchronize()
+    base = {}
+
+    # NCCL send/recv on the same pair (context, not the product), before mp_init
+    if not same_gpu:
+        try:
+            g_nccl = dist.new_group(backend="nccl")
+            buf = src if role == "sender" else torch.empty(n, dtype=torch.uint8, device="cuda")
+            nb_steps = max(3, min(args.steps, 20))
+            tb = 0.0
+            for it in range(nb_steps + 2):
+                if it == 2:
+                    torch.cuda.synchronize()
+                    b0 = time.perf_counter()
+                if role == "sender":
+                    dist.send(buf, 1, group=g_nccl)
+                elif role == "receiver":
+                    dist.recv(buf, 0, group=g_nccl)
+            torch.cuda.synchronize()
+            tb = time.perf_counter() - b0 if role in ("sender", "receiver") else 0.0
+            tb = _gather_max(tb)
+            base["nccl_send_recv_GBps"] = n * nb_steps / tb / 1e9
+            dist.destroy_process_group(g_nccl)
+            del buf
+            torch.cuda.synchronize()
+        except Exception as exc:
+            base["nccl_error"] = repr(exc)
+
+    ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
+                                  timeout_s=60.0, param_file=args.params)
+    _, cfg = p2p_plan(ctx, world, n, args.mode)
+    d = cfg.as_dict()
+    topo = ctx.topology()
+    rbuf = ctx.alloc(n) if role == "receiver" else None
+    rview = mp.as_tensor(rbuf, n) if rbuf else None
+
+    def message(c, tag):
+        if role == "sender":
+            ctx.send(src, n, 1, tag, c, s_tx)
+        elif role == "receiver":
+            ctx.recv(rbuf, n, 0, tag, s_rx)
+
+    def timed(c, k, tag0=0):
+        """k messages with config c: max-over-ranks device time (s) between two events
+        on each endpoint's stream, after a barrier."""
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        st = s_tx if role == "sender" else s_rx
+        e0.record(st)
+        for i in range(k):
+            message(c, tag0 + i)
+        e1.record(st)
+        st.synchronize()
+        ms = e0.elapsed_time(e1) if role in ("sender", "receiver") else 0.0
+        return _gather_max(ms) * 1e-3
+
+    for i in range(args.warmup):
+        message(cfg, i)
+    s_tx.synchronize()
+    s_rx.synchronize()
+    ctx.sync()
+    if role == "receiver":
+        assert torch.equal(rview, expect), "payload mismatch"
+    dist.barrier()
+    l0 = ctx.launches()
+    with Clocks(dev) as clk:
+        t = timed(cfg, args.steps)
+    launches = int(_gather_sum(ctx.launches() - l0))
+    ctx.sync()
+    if role == "receiver":
+        assert torch.equal(rview, expect), "payload mismatch (timed)"
+    value = n * args.steps / t / 1e9
+
+    # end to end through the public API: the sender's payload comes from pinned host
+    # memory every step (H2D on its stream), the receiver reads every message back
+    h_src = src.cpu().pin_memory() if role == "sender" else None
+    h_dst = torch.empty(n, dtype=torch.uint8).pin_memory() if role == "receiver" else None
+    e2e_steps = max(3, min(10, args.steps // 4))
+    dist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    st = s_tx if role == "sender" else s_rx
+    e0.record(st)
+    for i in range(e2e_steps):
+        if role == "sender":
+            with torch.cuda.stream(s_tx):
+                src.copy_(h_src, non_blocking=True)
+        message(cfg, 1000 + i)
+        if role == "receiver":
+            with torch.cuda.stream(s_rx):
+                h_dst.copy_(rview, non_blocking=True)
+    e1.record(st)
+    st.synchronize()
+    te = _gather_max(e0.elapsed_time(e1) if role in ("sender", "receiver") else 0.0) * 1e-3
+    e2e = n * e2e_steps / te / 1e9
+    if role == "receiver":
+        assert torch.equal(h_dst, expect.cpu()), "payload mismatch (e2e)"
+
+    # every path alone (A7-A9 evidence), a few messages each, same pair
+    per_path = {}
+    paths_ = d["paths"]
+    kp = max(3, min(args.steps, 10))
+    _, prm, _ = ctx.get_model(0, 1)
+    for i, (kind, via) in enumerate(paths_):
+        nb = [0] * len(paths_)
+        nb[i] = n
+        ks = [1] + [0] * (len(paths_) - 1)
+        if i:
+            ks[i] = max(16, -(-n // (32 * MiB - 512)))
+        ti = timed(ctx.make_config(nb, ks, 0, 1), kp, 5000 + 100 * i)
+        gbs = n / (ti / kp) / 1e9
+        name = "direct" if kind == 0 else (f"relay_gpu{via}" if kind == 1 else "host_pcie")
+        row = {"GBps": gbs, "chunks": ks[i]}
+        if kind == 0:
+            row.update({"frac_of_nvlink_nominal": gbs / 900.0, "frac_of_measured_peer_copy": gbs / 770.0})
+        else:
+            ceil = min(prm[i]["beta"], prm[i]["beta2"]) / 1e9
+            row.update({"stage_group_ceiling_GBps": ceil, "frac_of_stage_group_ceiling": gbs / ceil})
+            if kind == 2:
+                row["frac_of_pcie_nominal"] = gbs / 64.0
+        per_path[name] = row
+    if role == "receiver":
+        assert torch.equal(rview, expect), "payload mismatch (per-path)"
+
+    # copy-engine peer copy GPU0 -> GPU1's receive buffer (what cudaMemcpyPeerAsync does)
+    try:
+        from cuda.bindings import runtime as rt
+        offs = [None] * world
+        dist.all_gather_object(offs, (rbuf - ctx.peer_base(rank)) if rbuf else None)
+        ce_t = 0.0
+        nb_steps = max(3, min(args.steps, 20))
+        dist.barrier()
+        if role == "sender":
+            dptr = ctx.peer_base(1) + offs[1]
+            kind = rt.cudaMemcpyKind.cudaMemcpyDeviceToDevice
+            c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            for _ in range(2):
+                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, s_tx.cuda_stream)
+            c0.record(s_tx)
+            for _ in range(nb_steps):
+                rt.cudaMemcpyAsync(dptr, src.data_ptr(), n, kind, s_tx.cuda_stream)
+            c1.record(s_tx)
+            s_tx.synchronize()
+            ce_t = c0.elapsed_time(c1) * 1e-3 / nb_steps
+        ce_t = _gather_max(ce_t)
+        base["cudaMemcpyPeer_ce_GBps"] = n / ce_t / 1e9
+        base["mp_over_cudaMemcpyPeer"] = value / base["cudaMemcpyPeer_ce_GBps"]
+    except Exception as exc:
+        base["peer_copy_error"] = repr(exc)
+    if "nccl_send_recv_GBps" in base:
+        base["mp_over_nccl"] = value / base["nccl_send_recv_GBps"]
+
+    nvl = sum(b for (k, _), b in zip(paths_, d["bytes"]) if k != 2)
+    host = n - nvl
+    per_s = args.steps / t
+    nvl_gbs, pcie_gbs = nvl * per_s / 1e9, host * per_s / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_nvlink.json")
+    if os.path.exists(tp):  # scripts/ncu_rank.sh + scripts/nvlink_summary.py
+        try:
+            traffic = json.load(open(tp))[f"{world}:{n}"]["rank0:send_kernel"]["nvlink_tx_bytes_per_launch"]
+        except Exception:
+            traffic = None
+    if not same_gpu:
+        roofline = {"bound": "nvlink+pcie", "achieved": value, "peak": 964.0, "unit": "GB/s",
+                    "frac": value / 964.0, "traffic": traffic,
+                    "peak_source": "nominal summed path roofline of the source GPU: NVLink 5 egress 900 GB/s "
+                                   "+ PCIe Gen5 x16 64 GB/s (north star); measured peer copy 770 GB/s "
+                                   "(B200_PROFILING.md) alongside",
+                    "nvlink_egress_GBps": nvl_gbs, "frac_of_nvlink_nominal": nvl_gbs / 900.0,
+                    "frac_of_measured_peer_copy": nvl_gbs / 770.0, "pcie_GBps": pcie_gbs,
+                    "frac_of_pcie_nominal": pcie_gbs / 64.0, "kernel": "send_kernel + relay_kernel + recv_kernel"}
+    else:  # every rank on one GPU (diagnostic): the shared resource is that GPU's HBM
+        hbm = 2 * n + 2 * sum(b for (k, _), b in zip(paths_, d["bytes"]) if k == 1)
+        peak = measured_peaks()[0]
+        roofline = {"bound": "hbm", "achieved": hbm * per_s / 1e9, "peak": peak, "unit": "GB/s",
+                    "frac": hbm * per_s / 1e9 / peak, "traffic": None,
+                    "peak_source": "MEASURED_PEAKS.json HBM copy (all ranks on one GPU: not an NVLink number)",
+                    "kernel": "send_kernel + relay_kernel + recv_kernel"}
+    clk_all = [None] * world
+    dist.all_gather_object(clk_all, clk.summary())
+    pred = n / d["t_pred"] / 1e9 if d["t_pred"] else None
+    line = {
+        "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t / args.steps * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+        "data": "synthetic (seeded uniform random bytes)", "config": workload_config(args, world, d),
+        "roofline": roofline,
+        "e2e": {"value": e2e, "unit": "GB/s", "h2d_bytes_per_step": n, "d2h_bytes_per_step": n},
+        "gpu_launches": launches,
+        "clocks": clk_all[0], "clocks_all_ranks": clk_all,
+        "baselines": base, "per_path": per_path,
+        "model": {"selected": d, "split": split_label(d), "predicted_GBps": pred,
+                  "E_pred": abs(pred - value) / value if pred else None},
+        "topology": {"fingerprint": topo["fingerprint"],
+                     "gpus": [{k: g[k] for k in ("numa_node", "pcie_gen", "pcie_width", "nvlinks", "sms")}
+                              for g in topo["gpus"]],
+                     "peer_access_all": all(all(r) for r in topo["peer_access"]),
+                     "same_gpu_diagnostic": same_gpu},
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if rbuf:
+        ctx.free(rbuf)
+    ctx.close()
+    dist.destroy_process_group()
+    return 0
+
+
+def run_world_pairs(args, world, rank, local):
+    """N > 1 with --workload config5 (secondary line): BASELINE.json config 5, SURVEY §8(d)'s
     primary reading — disjoint pairs (0↔1, 2↔3, …) exchange one message each way per
     step, all pairs at once, so every GPU's NVLink egress and ingress are busy and
     every would-be relay is itself an endpoint.  Messages go through the multi-rank
@@ -372,10 +744,7 @@ def run_world(args, world, rank, local):
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded uniform random bytes)",
-        "config": {"workload": f"config5 (disjoint pairs, both directions): {npairs} pairs 2i<->2i+1, "
-                               f"{n >> 20} MiB per message, direct + relays + pinned host, model-selected",
-                   "msg_bytes": n, "mode": args.mode, "parallelism": f"pairs{npairs}x2dir",
-                   "l2": "messages >= 126 MB L2 (no flush)" if n >= 128 * MiB else "no flush"},
+        "config": workload_config(args, world, d),
         "roofline": ({"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
                       "frac": achieved / 770.0, "traffic": None, "peak_source":
                       "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
@@ -430,8 +799,11 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="mpx", choices=["mpx", "reference"])
     ap.add_argument("--size", type=int, default=None,
-                    help="message bytes (default: 1 GiB at N = 1 — config 3; 256 MiB per message at N > 1 — config 5)")
+                    help="message bytes (default: 1 GiB — config 3; 256 MiB per message with --workload config5)")
     ap.add_argument("--mode", default="b200", choices=["b200", "paper"])
+    ap.add_argument("--workload", default="config3", choices=["config3", "config5"],
+                    help="N > 1: config3 (GPU0 -> GPU1 over direct + relays GPU2.. + host; default) or "
+                         "config5 (disjoint pairs exchanging, every GPU busy)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-calibrate", action="store_true",
                     help="skip the init-time calibration (default parameters; for ncu runs)")
@@ -440,7 +812,7 @@ def main():
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.size is None:
-        args.size = GiB if int(os.environ.get("WORLD_SIZE", "1")) == 1 else 256 * MiB
+        args.size = 256 * MiB if (args.workload == "config5" and int(os.environ.get("WORLD_SIZE", "1")) > 1) else GiB
     if args.impl == "reference":
         return run_reference(args)
 
@@ -627,8 +999,10 @@ def main():
     t = med(lambda: ctx.xfer(dst, src, n, pcfg, stream))
     pd = pcfg.as_dict()
     per_path["paper_mode_pick_all_paths"] = {"GBps": n / t / 1e9, "bytes": pd["bytes"], "chunks": pd["chunks"],
+                                             "split": split_label(pd), "kernel": "xfer_kernel",
                                              "hbm_GBps": hbm_bytes(pd) / t / 1e9,
-                                             "frac": hbm_bytes(pd) / t / 1e9 / peak}
+                                             "frac": hbm_bytes(pd) / t / 1e9 / peak,
+                                             "vs_b200_pick": (n / t / 1e9) / (value / world)}
     ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
     torch.cuda.synchronize()
     assert torch.equal(dst, src), "payload mismatch (per-path runs)"
@@ -670,7 +1044,7 @@ def main():
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic (seeded uniform random bytes)",
-        "config": workload_config(args, world),
+        "config": workload_config(args, world, d),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "peak_source": peak_src,
@@ -690,6 +1064,7 @@ def main():
         "baselines": base,
         "per_path": per_path,
         "select_overhead": selector_overhead(ctx, n, value / world),
+        "topology": {k: v for k, v in ctx.topology().items() if k in ("fingerprint", "gpus")},
     }
     # NEXT f4 (readings C20/C21): the same message modelled with per-band Step-1
     # parameters (calibrated after the timed region; the pick is unchanged at 1 GiB)
@@ -703,8 +1078,7 @@ def main():
         except Exception as exc:  # context, not the product
             line["model"]["bands"] = {"error": repr(exc)}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        v, desc, cores = cpu_oracle_run(n, d, prm)
-        line["cpu_baseline"] = {"value": v, "unit": "GB/s", "cores": cores, "kind": "oracle", "sample": desc}
+        line["cpu_baseline"] = cpu_oracle_run(n, d, prm)
     if rank == 0:
         print(json.dumps(line), flush=True)
     ctx.close()

@@ -34,7 +34,8 @@
 extern "C" {
 #endif
 
-#define MP_ABI_VERSION 2  /* 2: NEXT f2 calls; mp_model_opts.window (was reserved) */
+#define MP_ABI_VERSION 3  /* 3: topology (mp_get/set_topology), fingerprinted parameter files;
+                             2: NEXT f2 calls; mp_model_opts.window (was reserved) */
 #define MP_MAX_PATHS 16
 
 /* Status codes. */
@@ -145,21 +146,77 @@ typedef struct mp_init_args {
 
 /* ---------------------------------------------------------------- lifetime */
 
-/* Create a context.  Collective over all ranks when world > 1.  Discovers the
- * topology (peer access, PCIe host path), allocates the heap, relay rings and the
- * pinned host ring, exchanges IPC handles, and — unless MP_INIT_NO_CALIBRATE —
- * calibrates α/β/ε of every path with the engine's own kernels (Step 1).
- * With MP_INIT_MODEL_ONLY no CUDA call is made; world/rank still define the pairs.
- * world >= 3 starts a persistent relay kernel on a non-blocking stream that runs
- * until mp_finalize: do not call cudaDeviceSynchronize() meanwhile (use stream
- * synchronisation / mp_sync), and initialise every CUDA kernel / library the
- * process will use before mp_init (lazy module loading may need an idle context).
- * Errors: MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_NOMEM, MP_ERR_TOPOLOGY. */
+/* Create a context — the paper's Steps 1-2 (parameters "extracted once per
+ * system topology and stored on each compute node", loaded at start-up).  Collective
+ * over all ranks when world > 1.  mp_init:
+ *   - discovers the topology (mp_get_topology): every GPU's UUID, PCI location, NUMA
+ *     node (sysfs), PCIe link and active NVLink links (NVML, loaded with dlopen; 0 =
+ *     unknown), and per ordered pair of GPUs peer access, P2P performance rank and
+ *     native atomics (cudaDeviceCanAccessPeer / cudaDeviceGetP2PAttribute where the
+ *     peer GPU is visible in this process, else the outcome of the IPC mapping);
+ *     a pair's relays (A1) are the ranks with peer access from the source and to the
+ *     destination;
+ *   - allocates the receive heap and control block, exchanges IPC handles, creates
+ *     the shared pinned segments (relay doorbells, host rings) bound to their GPU's
+ *     NUMA node (host-path quality depends on "PCIe configuration,
+ *     and NUMA effects");
+ *   - loads param_file if it exists (Step 2; refused with MP_ERR_TOPOLOGY when its
+ *     topology fingerprint differs from this job's), and — unless
+ *     MP_INIT_NO_CALIBRATE — calibrates α/β/ε of every path with the engine's own
+ *     kernels (Step 1);
+ *   - world >= 3: starts the relay service thread (launches a bounded relay kernel
+ *     for each relayed message a sender announces; no kernel outlives its traffic,
+ *     so device-wide synchronisation is allowed at any time).
+ * With MP_INIT_MODEL_ONLY no CUDA call is made; world/rank still define the pairs
+ * (topology unknown: every path assumed; mp_set_topology injects one).
+ * Errors: MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_NOMEM, MP_ERR_TOPOLOGY (a peer's memory
+ * cannot be mapped; a parameter file from another topology). */
 int mp_init(mp_ctx **ctx, const mp_init_args *args);
 
-/* Destroy a context: waits for outstanding work, stops relay kernels, unmaps and
- * frees everything.  Collective when world > 1.  ctx may be NULL. */
+/* Destroy a context (the end of the Step 5 engine's lifetime): waits for
+ * outstanding work on the streams it has seen, stops the relay service (waits for
+ * the relay kernels it launched), unmaps and frees everything.  Collective when
+ * world > 1.  ctx may be NULL.  Always returns MP_OK or the barrier's failure. */
 int mp_finalize(mp_ctx *ctx);
+
+/* ---------------------------------------------------------------- topology (Step 1) */
+
+/* One GPU of the job.  0 / -1 = unknown (NVML or sysfs unavailable). */
+typedef struct mp_gpu_info {
+  char uuid[16];          /* cudaDeviceProp.uuid */
+  int32_t device;         /* CUDA ordinal in the owning process */
+  int32_t pci_domain, pci_bus, pci_device;
+  int32_t numa_node;      /* NUMA node of the GPU's PCIe root (-1 unknown) */
+  int32_t pcie_gen, pcie_width;  /* maximum PCIe link generation / width (NVML) */
+  int32_t pcie_gen_cur;   /* current PCIe generation (power-managed; informational) */
+  int32_t nvlinks;        /* active NVLink links (NVML) */
+  int32_t sms;            /* streaming multiprocessors */
+  int32_t reserved;
+} mp_gpu_info;
+
+/* The job's topology: gpu[r] is rank r's GPU; [s][d] matrices by rank. */
+typedef struct mp_topology {
+  int32_t world;
+  int32_t reserved;
+  uint64_t fingerprint;   /* FNV-1a of the GPUs (UUID, SMs, PCIe link, NVLinks, NUMA) and
+                             the peer-access matrix; 0 = no topology known */
+  mp_gpu_info gpu[MP_MAX_PATHS];
+  int32_t peer_access[MP_MAX_PATHS][MP_MAX_PATHS];   /* 1: s can load/store d's memory */
+  int32_t p2p_perf_rank[MP_MAX_PATHS][MP_MAX_PATHS]; /* cudaDevP2PAttrPerformanceRank */
+  int32_t p2p_atomics[MP_MAX_PATHS][MP_MAX_PATHS];   /* cudaDevP2PAttrNativeAtomicSupported */
+} mp_topology;
+
+/* The topology found by mp_init (or injected).  A model-only context without one
+ * reports fingerprint 0 and full peer access.  Host-only. */
+int mp_get_topology(mp_ctx *ctx, mp_topology *out);
+
+/* Inject a topology into a MODEL-ONLY context (tests, planning for another node):
+ * in->world must equal the context's; the fingerprint is recomputed; every pair's
+ * model returns to the default paths of that topology (relays need peer access from
+ * the source and to the destination; a pair without peer access s -> d has no
+ * direct path and is reported as MP_ERR_TOPOLOGY).  Errors: MP_ERR_STATE (not
+ * model-only), MP_ERR_INVALID. */
+int mp_set_topology(mp_ctx *ctx, const mp_topology *in);
 
 const char *mp_strerror(int status);
 const char *mp_last_error(mp_ctx *ctx);
@@ -354,7 +411,10 @@ int mp_deregister(mp_ctx *ctx, int id);
  * sender), and `cfg`'s split is not used.  Both sides classify by size alone; the
  * environment variable MPX_EAGER=0 (equal on every rank, read at mp_init) turns it
  * off. */
-/* Send `bytes` bytes at device pointer `buf` to rank dst with `tag`.  cfg = NULL
+/* mp_send — Step 5 (the pipeline engine moves "the number of chunks and the
+ * size of each chunk per path" the model chose) under MPI point-to-point semantics
+ * (OMB's MPI_Isend / MPI_Irecv windows; matching FIFO per pair as in MPI).
+ * Send `bytes` bytes at device pointer `buf` to rank dst with `tag`.  cfg = NULL
  * selects with mp_select(all paths); otherwise cfg->bytes/chunks/path are used as
  * given (validated: Σ bytes == n, 1 <= k <= max(1, ⌊b/A⌋), chunk <= slot_bytes,
  * paths available).  Stream-ordered: the send kernel waits on the device for the
@@ -363,7 +423,8 @@ int mp_deregister(mp_ctx *ctx, int id);
 int mp_send(mp_ctx *ctx, const void *buf, uint64_t bytes, int dst, int tag,
             const mp_config *cfg, void *stream);
 
-/* Receive `bytes` bytes from rank src with `tag` into device pointer `buf`
+/* mp_recv — the receiving side of Step 5 with MPI semantics.
+ * Receive `bytes` bytes from rank src with `tag` into device pointer `buf`
  * (heap memory or a registered region — mp_register — when world > 1).  Matching is FIFO per (src, dst); the tag and the
  * size must equal the sender's or the device raises MP_ERR_MISMATCH.  Work after
  * mp_recv on `stream` sees the whole message. */
@@ -408,7 +469,12 @@ int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
  * Errors: MP_ERR_STATE (model-only), MP_ERR_INVALID (bad edges), MP_ERR_CUDA. */
 int mp_calibrate_bands(mp_ctx *ctx, const uint64_t *edges, int nedges, int reps);
 
-/* Save / load the model parameters of every pair (Step 1/2). */
+/* Save / load the model parameters of every pair (Step 1/2: "once per system
+ * topology and stored on each compute node").  The file carries the topology
+ * fingerprint and one line per GPU (UUID, NVLinks, PCIe link, NUMA node); loading a
+ * file whose fingerprint differs from the context's known topology fails with
+ * MP_ERR_TOPOLOGY and installs nothing (a file without a fingerprint, or a context
+ * without a topology, is accepted). */
 int mp_save_params(mp_ctx *ctx, const char *path);
 int mp_load_params(mp_ctx *ctx, const char *path);
 

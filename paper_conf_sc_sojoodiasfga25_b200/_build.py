@@ -19,7 +19,7 @@ OUT_DIR = os.path.join(PKG, "_lib")
 LIB = os.path.join(OUT_DIR, "libmpx.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["model.cpp", "capi.cpp", "calib.cpp", "world.cpp", "coll.cpp", "engine.cu"]
+SOURCES = ["model.cpp", "capi.cpp", "calib.cpp", "world.cpp", "coll.cpp", "topo.cpp", "engine.cu"]
 HEADERS = ["model.h", "engine.h", "ctx.h"]
 
 

@@ -69,8 +69,11 @@ PairModel default_pair(const mp_ctx *c, int src, int dst) {
   if (loop) {
     for (int r = 0; r < c->n_loop_relays; ++r) m.paths.push_back(default_path(K_GPU, r, true));
   } else {
+    // a relay r needs peer access src -> r and r -> dst (topology, mp_init)
     for (int r = 0; r < c->world; ++r)
-      if (r != src && r != dst) m.paths.push_back(default_path(K_GPU, r, false));
+      if (r != src && r != dst &&
+          (!c->have_topo || (c->topo.peer_access[src][r] && c->topo.peer_access[r][dst])))
+        m.paths.push_back(default_path(K_GPU, r, false));
   }
   if (c->host_path) m.paths.push_back(default_path(K_HOST, -1, loop));
   m.port_alpha = 4e-6;
@@ -80,6 +83,7 @@ PairModel default_pair(const mp_ctx *c, int src, int dst) {
 
 bool pair_ok(const mp_ctx *c, int src, int dst) {
   if (src < 0 || dst < 0 || src >= c->world || dst >= c->world) return false;
+  if (src != dst && c->have_topo && !c->topo.peer_access[src][dst]) return false;  // no direct path
   return true;
 }
 
@@ -242,7 +246,10 @@ int init_engine(mp_ctx *c) {
     if (e != cudaSuccess) return fail(c, MP_ERR_NOMEM, "heap allocation failed");
     c->heap.reset(static_cast<uint8_t *>(h), c->heap.size);
   }
-  if (c->world == 1) {
+  if (c->world == 1) {  // topology of the loopback job: this GPU alone
+    std::vector<mp_gpu_info> g(1);
+    if (int s = topo_local(c, &g[0])) return s;
+    if (int s = topo_discover(c, g, std::vector<int>(1, 1))) return s;
     c->rings.resize(c->n_loop_relays + (c->host_path ? 1 : 0));
     for (int r = 0; r < c->n_loop_relays; ++r)
       if (int s = alloc_ring(c, false, &c->rings[r])) return s;
@@ -1014,6 +1021,16 @@ int mp_save_params(mp_ctx *c, const char *path) {
   FILE *f = std::fopen(path, "w");
   if (!f) return fail(c, MP_ERR_INVALID, std::string("cannot write ") + path);
   std::fprintf(f, "mpx-params 1\n");
+  if (c->have_topo) {  // Step 1's parameters belong to this topology
+    const mp_topology &T = c->topo;
+    std::fprintf(f, "topology %016llx %d\n", static_cast<unsigned long long>(T.fingerprint), T.world);
+    for (int r = 0; r < T.world; ++r) {
+      const mp_gpu_info &g = T.gpu[r];
+      std::fprintf(f, "gpu %d ", r);
+      for (int i = 0; i < 16; ++i) std::fprintf(f, "%02x", static_cast<unsigned char>(g.uuid[i]));
+      std::fprintf(f, " %d %d %d %d %d\n", g.sms, g.nvlinks, g.pcie_gen, g.pcie_width, g.numa_node);
+    }
+  }
   for (const auto &kv : c->models) {
     const PairModel &m = kv.second;
     std::fprintf(f, "pair %d %d %zu %.17g %.17g\n", kv.first.first, kv.first.second, m.paths.size(),
@@ -1047,61 +1064,86 @@ int mp_load_params(mp_ctx *c, const char *path) {
   if (!c || !path) return MP_ERR_INVALID;
   FILE *f = std::fopen(path, "r");
   if (!f) return fail(c, MP_ERR_INVALID, std::string("cannot read ") + path);
+  std::vector<std::string> lines;
+  char buf[4096];
+  while (std::fgets(buf, sizeof(buf), f)) lines.push_back(buf);
+  std::fclose(f);
   char tag[32];
   int ver = 0;
-  if (std::fscanf(f, "%31s %d", tag, &ver) != 2 || std::strcmp(tag, "mpx-params") != 0 || ver != 1) {
-    std::fclose(f);
+  if (lines.empty() || std::sscanf(lines[0].c_str(), "%31s %d", tag, &ver) != 2 || std::strcmp(tag, "mpx-params") != 0 ||
+      ver != 1)
     return fail(c, MP_ERR_INVALID, "not an mpx parameter file");
+  // Step 2 loads only what Step 1 measured on this topology
+  for (const std::string &ln : lines) {
+    unsigned long long fp = 0;
+    int w = 0;
+    if (std::sscanf(ln.c_str(), "topology %llx %d", &fp, &w) == 2 && c->have_topo &&
+        (fp != c->topo.fingerprint || w != c->topo.world)) {
+      char msg[160];
+      std::snprintf(msg, sizeof(msg), "parameter file topology %016llx (world %d) is not this job's %016llx (world %d)",
+                    fp, w, static_cast<unsigned long long>(c->topo.fingerprint), c->topo.world);
+      return fail(c, MP_ERR_TOPOLOGY, msg);
+    }
   }
-  int src, dst;
-  size_t np;
-  unsigned long long n_min = 0;
-  double pa, pb;
-  while (std::fscanf(f, "%31s %d %d %zu", tag, &src, &dst, &np) == 4) {
-    if (std::strcmp(tag, "window") == 0 || std::strcmp(tag, "duplex") == 0) {  // NEXT f2
+  auto truncated = [&]() { return fail(c, MP_ERR_INVALID, "truncated parameter file"); };
+  size_t i = 1;
+  while (i < lines.size()) {
+    const char *ln = lines[i].c_str();
+    int src = 0, dst = 0;
+    size_t np = 0;
+    if (std::sscanf(ln, "%31s", tag) != 1) {
+      ++i;
+      continue;
+    }
+    if (!std::strcmp(tag, "topology") || !std::strcmp(tag, "gpu")) {
+      ++i;
+      continue;
+    }
+    if (!std::strcmp(tag, "window") || !std::strcmp(tag, "duplex")) {  // NEXT f2
       const bool win = tag[0] == 'w';
       double tau = 0.0, h[MP_MAX_PATHS];
-      if (np < 1 || np > MP_MAX_PATHS || std::fscanf(f, "%lf", &tau) != 1) break;
-      if (win)
-        for (size_t i = 0; i < np; ++i)
-          if (std::fscanf(f, "%lf", &h[i]) != 1) {
-            std::fclose(f);
-            return fail(c, MP_ERR_INVALID, "truncated parameter file");
-          }
+      int used = 0;
+      if (std::sscanf(ln, "%31s %d %d %zu %lf%n", tag, &src, &dst, &np, &tau, &used) != 5 || np < 1 ||
+          np > MP_MAX_PATHS)
+        return truncated();
+      if (win) {
+        const char *q = ln + used;
+        for (size_t k = 0; k < np; ++k) {
+          int u = 0;
+          if (std::sscanf(q, "%lf%n", &h[k], &u) != 1) return truncated();
+          q += u;
+        }
+      }
       int s = MP_OK;
       if (win && pair_ok(c, src, dst)) s = mp_set_window_model(c, src, dst, h, static_cast<int>(np), tau);
       if (!win) s = mp_set_host_duplex(c, src, tau);
-      if (s) {
-        std::fclose(f);
-        return s;
-      }
+      if (s) return s;
+      ++i;
       continue;
     }
-    const bool band = std::strcmp(tag, "band") == 0;
-    if ((!band && std::strcmp(tag, "pair")) || np < 1 || np > MP_MAX_PATHS) break;
-    if (band && std::fscanf(f, "%llu", &n_min) != 1) break;
-    if (std::fscanf(f, "%lf %lf", &pa, &pb) != 2) break;
+    const bool band = !std::strcmp(tag, "band");
+    if (!band && std::strcmp(tag, "pair")) return fail(c, MP_ERR_INVALID, std::string("unknown line: ") + tag);
+    unsigned long long n_min = 0;
+    double pa = 0.0, pb = 0.0;
+    const int got = band ? std::sscanf(ln, "%31s %d %d %zu %llu %lf %lf", tag, &src, &dst, &np, &n_min, &pa, &pb)
+                         : std::sscanf(ln, "%31s %d %d %zu %lf %lf", tag, &src, &dst, &np, &pa, &pb);
+    if (got != (band ? 7 : 6) || np < 1 || np > MP_MAX_PATHS || i + np >= lines.size()) return truncated();
     mp_path paths[MP_MAX_PATHS];
     mp_path_params prm[MP_MAX_PATHS];
-    for (size_t i = 0; i < np; ++i) {
-      mp_path_params &q = prm[i];
-      if (std::fscanf(f, "%31s %d %d %lf %lf %lf %lf %lf %lf %lf %lf", tag, &paths[i].kind, &paths[i].via,
-                      &q.alpha, &q.beta, &q.alpha2, &q.beta2, &q.eps, &q.c, &q.sigma, &q.w) != 11) {
-        std::fclose(f);
-        return fail(c, MP_ERR_INVALID, "truncated parameter file");
-      }
+    for (size_t k = 0; k < np; ++k) {
+      mp_path_params &q = prm[k];
+      if (std::sscanf(lines[i + 1 + k].c_str(), "%31s %d %d %lf %lf %lf %lf %lf %lf %lf %lf", tag, &paths[k].kind,
+                      &paths[k].via, &q.alpha, &q.beta, &q.alpha2, &q.beta2, &q.eps, &q.c, &q.sigma, &q.w) != 11)
+        return truncated();
     }
     mp_port_params port{pa, pb};
     if (pair_ok(c, src, dst)) {
       const int s = band ? mp_set_model_band(c, src, dst, n_min, prm, static_cast<int>(np), &port)
                          : mp_set_model(c, src, dst, paths, prm, static_cast<int>(np), &port);
-      if (s) {
-        std::fclose(f);
-        return s;
-      }
+      if (s) return s;
     }
+    i += 1 + np;
   }
-  std::fclose(f);
   return MP_OK;
 }
 

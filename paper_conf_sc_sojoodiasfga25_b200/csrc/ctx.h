@@ -83,6 +83,8 @@ struct mp_ctx {
   std::map<std::pair<int, int>, mpx::WindowModel> windows;
   std::vector<double> kappa;
   std::unordered_map<mpx::CacheKey, mpx::Selection, mpx::CacheKeyHash> cache;
+  mp_topology topo{};              // topo.cpp: found by mp_init or injected (model-only)
+  bool have_topo = false;
   uint32_t env_kinds = 0x7u;       // path kinds allowed by MPX_PATHS (bit = MP_PATH_*)
 
   // engine
@@ -190,4 +192,9 @@ bool world_receivable(mp_ctx *c, const void *p, uint64_t n);
 // collectives (coll.cpp): release the per-context streams, events and heap scratch
 void coll_release(mp_ctx *c);
 int world_deregister(mp_ctx *c, int id);
+// topology (topo.cpp)
+int topo_local(mp_ctx *c, mp_gpu_info *g);
+int topo_discover(mp_ctx *c, const std::vector<mp_gpu_info> &gpus, const std::vector<int> &mapped);
+uint64_t topo_fingerprint(const mp_topology &t);
+void numa_prefer(void *p, size_t n, int node);
 }  // namespace mpx

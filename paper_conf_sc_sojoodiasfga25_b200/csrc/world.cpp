@@ -54,6 +54,7 @@ struct RankInfo {
   int32_t slots;
   int32_t host_path;
   uint64_t eager_max;
+  mp_gpu_info gpu;   // topology (topo.cpp)
 };
 
 int allgather(mp_ctx *c, const void *in, void *out, uint64_t bytes) {
@@ -115,7 +116,12 @@ int map_segment(mp_ctx *c, int rank, bool create, uint8_t **out) {
   void *p = mmap(nullptr, c->hseg_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
   close(fd);
   if (p == MAP_FAILED) return wfail(c, MP_ERR_NOMEM, "mmap " + name + " failed");
-  if (create) std::memset(p, 0, c->hseg_bytes);
+  if (create) {
+    // the segment holds the host rings this rank's GPU reads (A9 step 3): first touch
+    // on its NUMA node (NUMA effects on the host path)
+    numa_prefer(p, c->hseg_bytes, c->topo.gpu[c->rank].numa_node);
+    std::memset(p, 0, c->hseg_bytes);
+  }
   cudaError_t e = cudaHostRegister(p, c->hseg_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
   if (e != cudaSuccess) {
     munmap(p, c->hseg_bytes);
@@ -183,6 +189,7 @@ int world_init(mp_ctx *c) {
   const char *eg = std::getenv("MPX_EAGER");  // "0": every message takes the rendezvous
   c->eager_max = (eg && eg[0] == '0') ? 0 : kEagerMax;
   me.eager_max = c->eager_max;
+  if (int s = topo_local(c, &me.gpu)) return s;
   std::vector<RankInfo> all(W);
   if (int s = allgather(c, &me, all.data(), sizeof(RankInfo))) return s;
   c->jobid = all[0].jobid;
@@ -205,6 +212,13 @@ int world_init(mp_ctx *c) {
       return wfail(c, MP_ERR_TOPOLOGY, "cannot map rank " + std::to_string(r) + "'s memory: " + cudaGetErrorString(e));
     c->peers[r] = PeerPtrs{static_cast<uint8_t *>(h), static_cast<uint8_t *>(k)};
     c->ipc_maps[{r, all[r].heap_addr}] = mp_ctx::IpcMap{static_cast<uint8_t *>(h), 1};
+  }
+  // topology: GPUs, peer access (mapping every peer above succeeded, else
+  // mp_init already failed with MP_ERR_TOPOLOGY), PCIe / NVLink / NUMA
+  {
+    std::vector<mp_gpu_info> gpus(W);
+    for (int r = 0; r < W; ++r) gpus[r] = all[r].gpu;
+    if (int s = topo_discover(c, gpus, std::vector<int>(W, 1))) return s;
   }
   // region 0 = the heaps
   c->regions.assign(kMaxRegions, mp_ctx::Region{});

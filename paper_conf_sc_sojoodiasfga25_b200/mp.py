@@ -16,6 +16,8 @@ MP_MAX_PATHS = 16
 MP_PATH_DIRECT, MP_PATH_GPU, MP_PATH_HOST = 0, 1, 2
 MP_MODEL_PAPER, MP_MODEL_B200 = 0, 1
 MP_INIT_MODEL_ONLY, MP_INIT_NO_CALIBRATE = 1, 2
+MP_OK, MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_TOPOLOGY, MP_ERR_NOMEM, MP_ERR_STATE = 0, -1, -2, -3, -4, -5
+MP_ERR_UNSUPPORTED, MP_ERR_TIMEOUT, MP_ERR_MISMATCH = -6, -7, -8
 
 STATUS = {0: "MP_OK", -1: "MP_ERR_INVALID", -2: "MP_ERR_CUDA", -3: "MP_ERR_TOPOLOGY",
           -4: "MP_ERR_NOMEM", -5: "MP_ERR_STATE", -6: "MP_ERR_UNSUPPORTED",
@@ -97,6 +99,20 @@ class mp_coll_plan(C.Structure):
                 ("post", mp_coll_copy * MP_COLL_MAX_COPIES)]
 
 
+class mp_gpu_info(C.Structure):
+    _fields_ = [("uuid", C.c_char * 16)] + [(n, C.c_int32) for n in (
+        "device", "pci_domain", "pci_bus", "pci_device", "numa_node", "pcie_gen", "pcie_width", "pcie_gen_cur",
+        "nvlinks", "sms", "reserved")]
+
+
+class mp_topology(C.Structure):
+    _fields_ = [("world", C.c_int32), ("reserved", C.c_int32), ("fingerprint", C.c_uint64),
+                ("gpu", mp_gpu_info * MP_MAX_PATHS),
+                ("peer_access", (C.c_int32 * MP_MAX_PATHS) * MP_MAX_PATHS),
+                ("p2p_perf_rank", (C.c_int32 * MP_MAX_PATHS) * MP_MAX_PATHS),
+                ("p2p_atomics", (C.c_int32 * MP_MAX_PATHS) * MP_MAX_PATHS)]
+
+
 ALLGATHER = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64)
 
 
@@ -173,6 +189,8 @@ def lib():
                                         C.POINTER(C.c_double), C.c_int, C.c_int, C.c_int, C.POINTER(C.c_double),
                                         C.POINTER(C.c_double)]),
             "mp_get_host_duplex": (C.c_int, [P, C.c_int, C.POINTER(C.c_double)]),
+            "mp_get_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
+            "mp_set_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
                                        C.POINTER(C.c_double)]),
@@ -194,7 +212,8 @@ def exported_symbols() -> List[str]:
             "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands",
             "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
-            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_fit_window"]
+            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_fit_window",
+            "mp_get_topology", "mp_set_topology"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -504,6 +523,38 @@ class Context:
 
     def load_params(self, path):
         self._ck(lib().mp_load_params(self.h, path.encode()))
+
+    def topology(self) -> dict:
+        """mp_get_topology: the job's GPUs (UUID, PCI, NUMA, PCIe link, NVLinks) and the
+        per-pair peer access / P2P attributes (Step 1)."""
+        t = mp_topology()
+        self._ck(lib().mp_get_topology(self.h, C.byref(t)))
+        w = t.world
+        gpus = [{"uuid": bytes(g.uuid).hex(), "device": g.device,
+                 "pci": f"{g.pci_domain:04x}:{g.pci_bus:02x}:{g.pci_device:02x}.0", "numa_node": g.numa_node,
+                 "pcie_gen": g.pcie_gen, "pcie_width": g.pcie_width, "pcie_gen_cur": g.pcie_gen_cur,
+                 "nvlinks": g.nvlinks, "sms": g.sms} for g in list(t.gpu)[:w]]
+        mat = lambda m: [[m[a][b] for b in range(w)] for a in range(w)]  # noqa: E731
+        return {"world": w, "fingerprint": f"{t.fingerprint:016x}", "gpus": gpus,
+                "peer_access": mat(t.peer_access), "p2p_perf_rank": mat(t.p2p_perf_rank),
+                "p2p_atomics": mat(t.p2p_atomics)}
+
+    def set_topology(self, topo: dict):
+        """mp_set_topology (model-only contexts): inject a topology dict as returned by
+        topology() (missing keys default to 0 / full peer access)."""
+        t = mp_topology()
+        w = int(topo["world"])
+        t.world = w
+        for r, g in enumerate(topo.get("gpus", [])[:w]):
+            t.gpu[r].uuid = bytes.fromhex(g.get("uuid", "00" * 16))[:16]
+            for k in ("device", "numa_node", "pcie_gen", "pcie_width", "pcie_gen_cur", "nvlinks", "sms"):
+                setattr(t.gpu[r], k, int(g.get(k, 0)))
+        for key in ("peer_access", "p2p_perf_rank", "p2p_atomics"):
+            m = topo.get(key)
+            for a in range(w):
+                for b in range(w):
+                    getattr(t, key)[a][b] = int(m[a][b]) if m else (1 if key == "peer_access" else 0)
+        self._ck(lib().mp_set_topology(self.h, C.byref(t)))
 
     def launches(self) -> int:
         v = C.c_uint64()

@@ -498,6 +498,33 @@ def scenario_devsync(rank, world):
     c.close()
 
 
+def scenario_bench_plan(rank, world):
+    """bench.py --gpus N (config 3) on CPU: rank roles (0 sends, 1 receives, 2.. relay),
+    every rank derives the same model config for GPU0 -> GPU1 over direct + relays
+    GPU2..GPU{N-1} + host, and the workload label names the executed split."""
+    import argparse
+
+    import bench
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    roles = bench.p2p_roles(world)
+    assert roles[0] == "sender" and roles[1] == "receiver" and roles[2:] == ["relay"] * (world - 2)
+    c = mdist.context_from_dist(model_only=True)
+    n = 1 << 30
+    r2, cfg = bench.p2p_plan(c, world, n, "b200")
+    d = cfg.as_dict()
+    assert r2 == roles
+    assert d["paths"] == [(0, -1)] + [(1, r) for r in range(2, world)] + [(2, -1)], d["paths"]
+    assert sum(d["bytes"]) == n
+    out = [None] * world
+    dist.all_gather_object(out, (d["bytes"], d["chunks"]))
+    assert all(o == out[0] for o in out)
+    args = argparse.Namespace(size=n, mode="b200", workload="config3")
+    w = bench.workload_config(args, world, d)
+    assert w["paths"] == f"direct+{world - 2}relay+host" and w["selected"] == bench.split_label(d)
+    assert w["parallelism"] == f"p2p-1pair+{world - 2}relays"
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
@@ -507,7 +534,8 @@ def main():
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
          "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
-         "eager": scenario_eager, "devsync": scenario_devsync}[scen](rank, world)
+         "eager": scenario_eager, "devsync": scenario_devsync,
+         "bench_plan": scenario_bench_plan}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

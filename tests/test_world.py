@@ -52,6 +52,12 @@ def test_gloo_bootstrap_and_consistent_selection(world):
     run_world(world, "gloo_model", timeout=240)
 
 
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_bench_config3_roles_and_plan(world):
+    # bench.py --gpus N: rank roles and the shared config-3 plan, gloo on CPU
+    run_world(world, "bench_plan", timeout=240)
+
+
 @pytest.mark.gpu
 @pytest.mark.parametrize("world", [2, 3])
 def test_multirank_engine_same_gpu(world):
