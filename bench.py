@@ -404,9 +404,12 @@ def run_world_p2p(args, world, rank, local):
 
     ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
                                   timeout_s=60.0, param_file=args.params)
+    if args.save_params and rank == 0:
+        ctx.save_params(args.save_params)
     _, cfg = p2p_plan(ctx, world, n, args.mode)
     d = cfg.as_dict()
     topo = ctx.topology()
+    _, prm01, port01 = ctx.get_model(0, 1)
     rbuf = ctx.alloc(n) if role == "receiver" else None
     rview = mp.as_tensor(rbuf, n) if rbuf else None
 
@@ -566,7 +569,7 @@ def run_world_p2p(args, world, rank, local):
         "clocks": clk_all[0], "clocks_all_ranks": clk_all,
         "baselines": base, "per_path": per_path,
         "model": {"selected": d, "split": split_label(d), "predicted_GBps": pred,
-                  "E_pred": abs(pred - value) / value if pred else None},
+                  "E_pred": abs(pred - value) / value if pred else None, "params": prm01, "port": port01},
         "topology": {"fingerprint": topo["fingerprint"],
                      "gpus": [{k: g[k] for k in ("numa_node", "pcie_gen", "pcie_width", "nvlinks", "sms")}
                               for g in topo["gpus"]],

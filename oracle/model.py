@@ -77,6 +77,7 @@ class Config:
     theta: List[float] = field(default_factory=list)
     t_pred: float = 0.0         # O2 evaluation of this config
     t_level: float = 0.0        # linearised common finish time (Eq 21 level)
+    theta_level: List[float] = field(default_factory=list)  # θ of the last level solve (Σ = 1)
 
 
 # ----------------------------------------------------------------------------- §3.1
@@ -411,6 +412,41 @@ def select(n: int, paths: Sequence[Path], opts: Options, port: Optional[Port] = 
     # Δ = kα + ε + α'; case 2 Ω = 1/(kβ) + 1/β', Δ = α + k(ε + α') — so Eq 24 is
     # solved once more with those coefficients, equalising the integer-k finish times.
     refine = opts.refine if opts.refine is not None else (opts.mode == B200)
+    if refine and opts.mode == B200:
+        # Reading C26 (B200 mode): the exact pipeline T(x, k) = max(T1, T2) (C3)
+        # picks its bottleneck stage per chunk size, so k_i is the exact integer
+        # argmin of T at the path's share (``k_exact``) and the affine piece of Eq 13
+        # used for Eq 24 is the one that is binding there (``piece_exact``); two
+        # rounds of (k, piece, Eq 24, shares), then k once more for the final shares.
+        for _round in range(2):
+            om3, de3 = [], []
+            for i, q in enumerate(paths):
+                if q.kind == DIRECT or nbytes[i] == 0:
+                    om, de = omega_delta_unpipelined(q) if q.kind == DIRECT else (1.0, 0.0)
+                else:
+                    chunks[i] = k_exact(float(nbytes[i]), q, nbytes[i], opts)
+                    om, de = piece_exact(float(nbytes[i]), chunks[i], q)
+                om3.append(om)
+                de3.append(de)
+            act3 = [i == 0 or nbytes[i] > 0 for i in range(p)]
+            theta, t_level, act3 = level(om3, de3, act3)
+            nbytes = _shares(n, theta, act3, opts)
+        chunks = [1] + [k_exact(float(nbytes[i]), paths[i], nbytes[i], opts) if nbytes[i] else 0
+                        for i in range(1, p)]
+        cfg = Config(nbytes, chunks, [theta[i] if nbytes[i] > 0 or i == 0 else 0.0 for i in range(p)])
+        cfg.t_pred = evaluate(n, nbytes, chunks, paths, opts, port)
+        cfg.t_level = t_level
+        cfg.theta_level = list(theta)
+        # Reading C26, last step: the model's own prediction decides between this
+        # split and the direct path alone (any path but the direct one may be
+        # excluded), for plain messages (not a window's shifted coefficients).
+        if dshift is None:
+            direct = [n] + [0] * (p - 1)
+            t_direct = evaluate(n, direct, [1] + [0] * (p - 1), paths, opts, port)
+            if t_direct < cfg.t_pred:
+                return Config(direct, [1] + [0] * (p - 1), [1.0] + [0.0] * (p - 1), t_direct, t_direct,
+                              [1.0] + [0.0] * (p - 1))
+        return cfg
     if refine:
         om3, de3 = [], []
         for i, q in enumerate(paths):
@@ -426,7 +462,48 @@ def select(n: int, paths: Sequence[Path], opts: Options, port: Optional[Port] = 
     cfg = Config(nbytes, chunks, [theta[i] if nbytes[i] > 0 or i == 0 else 0.0 for i in range(p)])
     cfg.t_pred = evaluate(n, nbytes, chunks, paths, opts, port)
     cfg.t_level = t_level
+    cfg.theta_level = list(theta)
     return cfg
+
+
+def k_exact(x: float, p: Path, b: int, opts: Options) -> int:
+    """Reading C26 (B200 mode): the integer k in C5's clamp range minimising the exact
+    two-stage pipeline time of x bytes (C3).  With s1 = α + x/(kβ) and
+    s2 = ε + α' + x/(kβ'), T(k) = s1 + s2 + (k−1)·max(s1, s2) = max(T1, T2) where
+    T1 = k·s1 + s2 (Eq 13 case 1) and T2 = s1 + k·s2 (case 2), both convex in k, so
+    T is convex and its real minimiser is the minimiser of T1 (Eq 14), of T2 (Eq 15)
+    or the stage crossover s1 = s2; the integer argmin is the floor or ceiling of one
+    of them (or a bound of the range).  Ties go to the smaller k (C5)."""
+    lo = _clamp_k(1, b, opts)
+    hi = max(lo, _clamp_k(10 ** 9, b, opts))
+    e = p.eps + p.alpha2
+    cands = {lo, hi}
+    reals = [math.sqrt(x / (p.alpha * p.beta2)), math.sqrt(x / (p.beta * e))]
+    if p.alpha != e:
+        kc = x * (1.0 / p.beta2 - 1.0 / p.beta) / (p.alpha - e)
+        if kc > 0:
+            reals.append(kc)
+    for r in reals:
+        for k in (math.floor(r), math.ceil(r)):
+            cands.add(min(hi, max(lo, int(k))))
+    best = None
+    for k in sorted(cands):
+        t = pipelined_time(x, k, p, B200)
+        if best is None or t < best[0]:
+            best = (t, k)
+    return best[1]
+
+
+def piece_exact(x: float, k: int, p: Path):
+    """Reading C26: the affine piece (Ω, Δ) of the exact pipeline time at k chunks
+    that binds at x bytes — case 1 (Ω = 1/β + 1/(kβ'), Δ = kα + ε + α') when
+    T1 >= T2, else case 2 (Ω = 1/(kβ) + 1/β', Δ = α + k(ε + α'))."""
+    m = x / k
+    s1 = p.alpha + m / p.beta
+    s2 = p.eps + p.alpha2 + m / p.beta2
+    if s1 >= s2:
+        return 1.0 / p.beta + 1.0 / (k * p.beta2), k * p.alpha + p.eps + p.alpha2
+    return 1.0 / (k * p.beta) + 1.0 / p.beta2, p.alpha + k * (p.eps + p.alpha2)
 
 
 def omega_delta_fixed_k(p: Path, k: int, mode: int = PAPER):

@@ -116,6 +116,38 @@ def level_integer_k(n: float, paths: Sequence[M.Path], k_max=64, mode=M.PAPER, i
     return hi
 
 
+def level_integer_k_b200(n: float, paths: Sequence[M.Path], k_max=256, iters=300):
+    """Exact optimum of Eq 5 over real x and integer k in 1..k_max with the B200-mode
+    exact pipeline time (C3): T = max(T1, T2), T1 = kα + ε + α' + x(1/β + 1/(kβ')),
+    T2 = α + k(ε + α') + x(1/(kβ) + 1/β').  At level T path i carries
+    max_k min((T − c1)/s1, (T − c2)/s2) bytes (or 0), increasing in T; bisect on
+    Σ cap_i = n.  (No issue stagger, no shared port.)"""
+    def pieces(p):
+        if p.kind == M.DIRECT:
+            return [((1.0 / p.beta, p.alpha),)]
+        out = []
+        for k in range(1, k_max + 1):
+            out.append(((1.0 / p.beta + 1.0 / (k * p.beta2), k * p.alpha + p.eps + p.alpha2),
+                        (1.0 / (k * p.beta) + 1.0 / p.beta2, p.alpha + k * (p.eps + p.alpha2))))
+        return out
+
+    lines = [pieces(p) for p in paths]
+
+    def cap(T, ls):
+        return max(0.0, max(min((T - c) / s for s, c in pc) for pc in ls))
+
+    lo, hi = 0.0, 1e-9
+    while sum(cap(hi, ls) for ls in lines) < n:
+        hi *= 2.0
+    for _ in range(iters):
+        mid = 0.5 * (lo + hi)
+        if sum(cap(mid, ls) for ls in lines) >= n:
+            hi = mid
+        else:
+            lo = mid
+    return hi
+
+
 def lp_port_exact(n: float, omegas, deltas, weights, port_alpha, port_beta):
     """B200 mode (C14): min T s.t. Ω_i x_i + Δ_i <= T (i in A), Σ w_i x_i <= (T − α_S) β_S,
     Σ x_i = n, x >= 0, minimised over every non-empty active subset A (scipy HiGHS).

@@ -269,6 +269,51 @@ uint32_t clamp_k(uint64_t k, uint64_t b, const ModelOpts &o) {
   return static_cast<uint32_t>(std::max<uint64_t>(1, k));
 }
 
+// Reading C26 (B200 mode): the integer k in C5's clamp range minimising the exact
+// pipeline time T(k) = max(k·s1 + s2, s1 + k·s2) (convex in k): the floor / ceiling of
+// the minimiser of either piece (Eq 14, Eq 15) or of the stage crossover s1 = s2, or
+// a bound of the range; ties to the smaller k.
+uint32_t k_exact(const PathModel &p, double x, uint64_t b, const ModelOpts &o) {
+  const uint32_t lo = clamp_k(1, b, o);
+  const uint32_t hi = std::max(lo, clamp_k(1000000000ull, b, o));
+  const double e = p.eps + p.alpha2;
+  double reals[3] = {std::sqrt(x / (p.alpha * p.beta2)), std::sqrt(x / (p.beta * e)), -1.0};
+  if (p.alpha != e) reals[2] = x * (1.0 / p.beta2 - 1.0 / p.beta) / (p.alpha - e);
+  uint32_t cand[8] = {lo, hi, lo, lo, lo, lo, lo, lo};
+  int nc = 2;
+  for (double r : reals) {
+    if (!(r > 0.0)) continue;
+    for (double f : {std::floor(r), std::ceil(r)}) {
+      const double c = std::min(static_cast<double>(hi), std::max(static_cast<double>(lo), f));
+      cand[nc++] = static_cast<uint32_t>(c);
+    }
+  }
+  std::sort(cand, cand + nc);
+  uint32_t best = cand[0];
+  double tb = staged_time(p, x, best, M_B200);
+  for (int i = 1; i < nc; ++i) {
+    const double t = staged_time(p, x, cand[i], M_B200);
+    if (t < tb) {
+      tb = t;
+      best = cand[i];
+    }
+  }
+  return best;
+}
+
+// Reading C26: the affine piece of the exact pipeline time at k chunks binding at x.
+void piece_exact(const PathModel &p, double x, uint32_t k, double *om, double *de) {
+  const double kd = static_cast<double>(k), m = x / kd;
+  const double s1 = p.alpha + m / p.beta, s2 = p.eps + p.alpha2 + m / p.beta2;
+  if (s1 >= s2) {
+    *om = 1.0 / p.beta + 1.0 / (kd * p.beta2);
+    *de = kd * p.alpha + p.eps + p.alpha2;
+  } else {
+    *om = 1.0 / (kd * p.beta) + 1.0 / p.beta2;
+    *de = p.alpha + kd * (p.eps + p.alpha2);
+  }
+}
+
 }  // namespace
 
 bool PairModel::has_port() const { return port_beta > 0.0 && std::isfinite(port_beta); }
@@ -380,7 +425,48 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
   }
 
   const bool refine = o.refine >= 0 ? o.refine != 0 : o.mode == M_B200;
-  if (refine) {  // pass 3 (C18)
+  if (refine && o.mode == M_B200) {  // pass 3, reading C26: exact-pipeline k and piece
+    std::vector<char> act3(p);
+    for (int round = 0; round < 2; ++round) {
+      for (size_t i = 0; i < p; ++i) {
+        const PathModel &q = m.paths[i];
+        if (q.kind == K_DIRECT) {
+          od_unpipelined(q, &om[i], &de[i]);
+        } else if (out->bytes[i] == 0) {
+          om[i] = 1.0;
+          de[i] = 0.0;
+        } else {
+          const double x = static_cast<double>(out->bytes[i]);
+          out->chunks[i] = k_exact(q, x, out->bytes[i], o);
+          piece_exact(q, x, out->chunks[i], &om[i], &de[i]);
+        }
+        act3[i] = (i == 0) || out->bytes[i] > 0;
+      }
+      L = solve(m, nd, om, de, act3, o, dshift);
+      shares_of(n, L, o, &out->bytes);
+    }
+    for (size_t i = 1; i < p; ++i)
+      out->chunks[i] = out->bytes[i] ? k_exact(m.paths[i], static_cast<double>(out->bytes[i]), out->bytes[i], o) : 0;
+    for (size_t i = 0; i < p; ++i) out->theta[i] = (i == 0 || out->bytes[i] > 0) ? L.theta[i] : 0.0;
+    out->t_level = L.t;
+    out->t_pred = predict(m, n, out->bytes.data(), out->chunks.data(), o);
+    if (!dshift) {  // C26: the model decides between this split and the direct path alone
+      std::vector<uint64_t> db(p, 0);
+      std::vector<uint32_t> dk(p, 0);
+      db[0] = n;
+      dk[0] = 1;
+      const double td = predict(m, n, db.data(), dk.data(), o);
+      if (td < out->t_pred) {
+        out->bytes = db;
+        out->chunks = dk;
+        out->theta.assign(p, 0.0);
+        out->theta[0] = 1.0;
+        out->t_pred = out->t_level = td;
+      }
+    }
+    return;
+  }
+  if (refine) {  // pass 3 (C18), PAPER mode when asked for
     std::vector<char> act3(p);
     for (size_t i = 0; i < p; ++i) {
       od_fixed_k(m.paths[i], std::max<uint32_t>(1, out->chunks[i]), o.mode, &om[i], &de[i]);

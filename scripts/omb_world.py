@@ -3,7 +3,7 @@
 osu_bibw / osu_latency, 4 KiB - 2 GiB, single pair GPU0 <-> GPU1, vs cudaMemcpyPeer
 and NCCL send/recv; the paper's OMB methodology).
 
-    torchrun --nproc-per-node N scripts/omb_world.py [--min 4096] [--max 1073741824]
+    torchrun --nproc-per-node N scripts/omb_world.py [--min-bytes 4096] [--max-bytes 1073741824]
              [--windows 1,16,64] [--out gpurun_out/omb_world.jsonl]
 
 Ranks 0 and 1 are the pair; ranks 2.. serve as relay GPUs for the model's configs.
@@ -41,8 +41,8 @@ def main():
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
     ap = argparse.ArgumentParser()
-    ap.add_argument("--min", type=int, default=4096)
-    ap.add_argument("--max", type=int, default=1 << 30)
+    ap.add_argument("--min-bytes", type=int, default=4096)
+    ap.add_argument("--max-bytes", type=int, default=1 << 30)
     ap.add_argument("--windows", default="1,16,64")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "omb_world.jsonl"))
     a = ap.parse_args()
@@ -53,8 +53,8 @@ def main():
     torch.cuda.set_device(dev)
     windows = [int(w) for w in a.windows.split(",")]
     sizes = []
-    n = a.min
-    while n <= a.max:
+    n = a.min_bytes
+    while n <= a.max_bytes:
         sizes.append(n)
         n *= 2
     big = sizes[-1]

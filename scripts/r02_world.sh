@@ -16,5 +16,5 @@ for N in 2 3 4; do
   run $N $((29600 + N)) bench_n$N bench.py --gpus $N --steps ${STEPS:-20} --warmup 3
 done
 TMO=900 run 4 29611 sweep_world scripts/sweep_world.py --sizes ${SWEEP_SIZES:-16,64} --step ${SWEEP_STEP:-16} --reps 3 --out $OUT/sweep_world.json
-TMO=900 run 3 29612 omb_world scripts/omb_world.py --max ${OMB_MAX:-268435456} --windows 1,16 --out $OUT/omb_world_full.jsonl
+TMO=900 run 3 29612 omb_world scripts/omb_world.py --max-bytes ${OMB_MAX:-268435456} --windows 1,16 --out $OUT/omb_world_full.jsonl
 echo done

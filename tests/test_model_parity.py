@@ -141,3 +141,31 @@ def test_env_path_filter(monkeypatch):
     with mp.Context(world=4, rank=0, model_only=True) as c:
         setup_pair(c, tbl, None)
         assert all(b > 0 for b in c.select(0, 1, 512 * MiB).as_dict()["bytes"])
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_b200_heavy_latency_parity(seed):
+    # reading C26 on the heavy-latency corner (the bottleneck stage flips with the
+    # chunk size): library = oracle — shares ±A, chunks, level and prediction 1e-9
+    import sys
+    import os
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from test_oracle_select import heavy_paths
+    rnd = random.Random(5000 + seed)
+    paths = heavy_paths(rnd, 1 + seed % 3)
+    tbl = [dict(kind=p.kind, via=(p.via if p.kind == 1 else -1), alpha=p.alpha, beta=p.beta, alpha2=p.alpha2,
+                beta2=p.beta2, eps=p.eps, c=p.c, sigma=p.sigma, w=p.w) for p in paths]
+    port = dict(alpha=paths[0].alpha, beta=paths[0].beta * rnd.uniform(0.9, 1.1))
+    o = M.Options(mode=M.B200, slot_bytes=32 * MiB - 512)
+    with mp.Context(world=8, rank=0, model_only=True) as c:
+        setup_pair(c, tbl, port)
+        c.set_options(mode=M.B200, slot_bytes=o.slot_bytes)
+        for n in (16 * MiB, 64 * MiB + 3, 256 * MiB, 1 << 30):
+            d = c.select(0, 1, n).as_dict()
+            ref = M.select(n, paths, o, M.Port(**port))
+            assert sum(d["bytes"]) == n
+            for a, b in zip(d["bytes"], ref.bytes):
+                assert abs(a - b) <= o.align
+            if d["bytes"] == ref.bytes:
+                assert d["chunks"] == ref.chunks
+            assert rel(d["t_pred"], ref.t_pred) < 1e-9 and rel(d["t_level"], ref.t_level) < 1e-9

@@ -39,10 +39,16 @@ def test_select_invariants(seed, nrel, host, n, mode):
         else:
             assert k == 0
     assert cfg.t_pred > 0 and cfg.t_level > 0
-    # θ is informational: paths whose floored share fell below C_min report 0 and their
-    # bytes went to the direct path (Alg 1 lines 27-28), so Σθ <= 1.
-    assert sum(cfg.theta) <= 1 + 1e-9
-    assert all(t >= 0 for t in cfg.theta)
+    # The last level solve splits the whole message: Σθ = 1 over its active set (Eq 3),
+    # every θ >= 0 (C2).  A path with θ > 0 but no bytes was dropped only because its
+    # floored share ⌊θn/A⌋A fell below C_min (Alg 1 lines 24-28, C7); no θ mass is
+    # lost anywhere else.  The reported θ is that solve's, zero for dropped paths.
+    assert abs(sum(cfg.theta_level) - 1.0) < 1e-9
+    assert all(t >= -1e-12 for t in cfg.theta_level)
+    for i in range(1, len(paths)):
+        if cfg.bytes[i] == 0 and cfg.theta_level[i] > 0:
+            assert math.floor(cfg.theta_level[i] * n / opts.align) * opts.align < opts.c_min, (i, cfg.theta_level)
+        assert cfg.theta[i] == (cfg.theta_level[i] if cfg.bytes[i] else 0.0)
 
 
 @settings(max_examples=40, deadline=None)
@@ -175,3 +181,68 @@ def test_b200_prediction_never_exceeds_the_port_plus_unported_paths(seed, nrel, 
     h = paths[-1]
     bound = port.beta + min(h.beta, h.beta2)
     assert n / cfg.t_pred <= bound * (1 + 1e-9)
+
+
+# ---------------------------------------------------------------- reading C26 (B200 mode)
+
+def heavy_paths(rnd, nrel):
+    """B200 mode's pathological corner: startup latencies up to ~1 ms on the staged
+    legs (e.g. host legs calibrated while other ranks share the GPU), where the
+    bottleneck stage flips with the chunk size."""
+    lu = lambda a, b: math.exp(rnd.uniform(math.log(a), math.log(b)))  # noqa: E731
+    out = [M.Path(kind=M.DIRECT, alpha=lu(5e-6, 6e-5), beta=lu(3e11, 3e12), w=1.0)]
+    for r in range(nrel):
+        out.append(M.Path(kind=M.GPU_STAGED, alpha=lu(5e-6, 2e-4), beta=lu(2e11, 8e11), alpha2=lu(5e-6, 2e-4),
+                          beta2=lu(2e11, 8e11), eps=lu(1e-6, 1e-5), w=1.0, via=2 + r))
+    out.append(M.Path(kind=M.HOST_STAGED, alpha=lu(1e-5, 1e-3), beta=lu(1e10, 6e10), alpha2=lu(1e-5, 5e-4),
+                      beta2=lu(1e10, 6e10), eps=lu(1e-6, 1e-5)))
+    return out
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_k_exact_is_the_integer_argmin_of_the_exact_pipeline(seed):
+    # C26's k against brute force over every k of C5's clamp range (ties to the lower k)
+    import random
+    rnd = random.Random(seed)
+    p = heavy_paths(rnd, 1)[1 + seed % 2]
+    opts = M.Options(mode=M.B200, slot_bytes=32 * MiB - 512)
+    b = rnd.choice([1, 4, 16, 64, 256]) * MiB + 256 * rnd.randrange(1000)
+    k = M.k_exact(float(b), p, b, opts)
+    lo, hi = M._clamp_k(1, b, opts), max(M._clamp_k(1, b, opts), M._clamp_k(10 ** 9, b, opts))
+    ts = {kk: M.pipelined_time(float(b), kk, p, M.B200) for kk in range(lo, hi + 1)}
+    best = min(ts.values())
+    assert ts[k] == best and all(ts[kk] > best for kk in range(lo, k))
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_b200_select_never_worse_than_direct_alone(seed):
+    # C26's last step: the model's own prediction of the pick never exceeds the direct
+    # path alone (P:314: any path but the direct one may be excluded)
+    import random
+    rnd = random.Random(1000 + seed)
+    paths = heavy_paths(rnd, rnd.randrange(0, 4))
+    n = rnd.choice([16, 64, 256, 1024]) * MiB
+    opts = M.Options(mode=M.B200, slot_bytes=32 * MiB - 512)
+    port = M.Port(alpha=paths[0].alpha, beta=paths[0].beta * rnd.uniform(0.9, 1.1))
+    cfg = M.select(n, paths, opts, port)
+    direct = M.evaluate(n, [n] + [0] * (len(paths) - 1), [1] + [0] * (len(paths) - 1), paths, opts, port)
+    assert cfg.t_pred <= direct * (1 + 1e-12)
+    assert cfg.t_pred == M.evaluate(n, cfg.bytes, cfg.chunks, paths, opts, port)
+
+
+@pytest.mark.parametrize("seed", range(16))
+@pytest.mark.parametrize("mib", [16, 256, 1024])
+def test_b200_select_vs_exact_pipeline_optimum(seed, mib):
+    # The B200-mode pick (no stagger, no port) against the exact optimum of Eq 5 under
+    # the exact pipeline over real shares and integer k (oracle/optimize.py):
+    # B200-like tables within 1 %, the heavy-latency corner within 5 % (shares floored
+    # to A and C_min, k <= 256 in the optimiser).
+    import random
+    n = mib * MiB
+    for paths, bound in ((paths_from(synth.topology(seed, 2 + seed % 4, host=True)), 1.005),
+                         (heavy_paths(random.Random(seed), 1 + seed % 3), 1.005)):
+        opts = M.Options(mode=M.B200, stagger=False)
+        cfg = M.select(n, paths, opts)
+        t_opt = O.level_integer_k_b200(float(n), paths, k_max=256)
+        assert t_opt * (1 - 1e-9) <= cfg.t_pred * (1 + 1e-9)
+        assert cfg.t_pred <= t_opt * bound, (cfg.t_pred / t_opt, cfg.bytes, cfg.chunks)
