@@ -94,20 +94,40 @@ int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double
 
 // OMB-style timing (reading C21): `W` back-to-back copies of n bytes between the
 // same buffers (no flush — a window of repeated sends), median over
-// `reps` windows; returns seconds per message.
+// `reps` windows; returns seconds per message.  The window is captured once in a CUDA
+// graph and replayed, so it is timed at GPU speed: enqueued from the host, a small
+// message costs 2-3 µs of host submission per call, more than its 1-2 µs on the GPU
+// (DESIGN §6), and the bands would fit the host instead of the link.  (Thread-local
+// capture: the relay service thread keeps launching on its own streams meanwhile.)
 int time_window(Bench &b, void *dst, const void *src, uint64_t n, int reps, int W, double *out, int ctas = 0) {
   mp_ctx *c = b.c;
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  CKC(cudaStreamBeginCapture(b.s, cudaStreamCaptureModeThreadLocal));
+  int st = MP_OK;
+  for (int w = 0; w < W && st == MP_OK; ++w) st = launch_direct_copy(c, dst, src, n, b.s, ctas);
+  const cudaError_t ce = cudaStreamEndCapture(b.s, &g);
+  if (st) {
+    if (g) cudaGraphDestroy(g);
+    return st;
+  }
+  CKC(ce);
+  const cudaError_t ie = cudaGraphInstantiate(&ge, g, 0);
+  cudaGraphDestroy(g);
+  CKC(ie);
   std::vector<double> ts;
-  for (int r = 0; r < reps + 1; ++r) {
-    CKC(cudaEventRecord(b.e0, b.s));
-    for (int w = 0; w < W; ++w)
-      if (int st = launch_direct_copy(c, dst, src, n, b.s, ctas)) return st;
-    CKC(cudaEventRecord(b.e1, b.s));
-    CKC(cudaEventSynchronize(b.e1));
+  for (int r = 0; r < reps + 1 && st == MP_OK; ++r) {
+    cudaError_t e = cudaEventRecord(b.e0, b.s);
+    if (e == cudaSuccess) e = cudaGraphLaunch(ge, b.s);
+    if (e == cudaSuccess) e = cudaEventRecord(b.e1, b.s);
+    if (e == cudaSuccess) e = cudaEventSynchronize(b.e1);
     float ms = 0;
-    CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, b.e0, b.e1);
+    if (e != cudaSuccess) st = cfail(c, MP_ERR_CUDA, std::string("window graph: ") + cudaGetErrorString(e));
     if (r > 0) ts.push_back(ms * 1e-3 / W);  // first window is a warm-up
   }
+  cudaGraphExecDestroy(ge);
+  if (st) return st;
   *out = median(ts);
   return MP_OK;
 }
@@ -402,7 +422,7 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
     double eps_host = 0, eps_dev = 0, kappa = 1.0;
     if (c->host_path) {
       // the own segment's ring of sender == me is never used for traffic
-      uint8_t *hr = c->hseg[me] + static_cast<uint64_t>(me) * c->hseg_per_src;
+      uint8_t *hr = c->hseg[me] + bell_bytes(static_cast<uint32_t>(W)) + static_cast<uint64_t>(me) * c->hseg_per_src;
       const uint64_t hcap = static_cast<uint64_t>(c->slots) * c->host_stride;
       std::vector<uint64_t> hs;
       for (uint64_t s : sz)

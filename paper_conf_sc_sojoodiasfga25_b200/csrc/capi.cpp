@@ -277,6 +277,10 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   // direct group sized by direct_ctas(), leaving room for every staged group to be
   // co-resident.
   uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas), c->pdl != 0);
+  // beside staged groups, a whole number of CTAs per SM (an uneven grid lands unevenly
+  // on the SMs a PDL predecessor still holds)
+  if (staged_ctas && g_direct > static_cast<uint32_t>(c->sms))
+    g_direct = g_direct / static_cast<uint32_t>(c->sms) * static_cast<uint32_t>(c->sms);
   // Two large copies running at once (osu_bibw's two directions on two streams) do
   // best with one TMA pipeline per SM each — 64 KiB in flight per SM in total, as one
   // copy with two (profiles/r01/bibw.jsonl).  A large direct-only launch that finds
@@ -359,8 +363,7 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   P.pdl = c->pdl;
   P.bulk_stages = bulk_stages_for(n);
   P.allow_small = ctas > 0 ? 0u : 1u;  // a staged leg's calibration times its group's CTAs
-  // loopback staged legs move 16 KiB TMA blocks (xfer_kernel); multi-rank ones 8 KiB
-  P.staged_blk = ctas > 0 && c->world == 1 ? 1u : 0u;
+  P.staged_blk = ctas > 0 ? 1u : 0u;  // staged lanes move 16 KiB TMA blocks in every engine
   P.npaths = 1;
   DevPath &d = P.p[0];
   d.kind = DK_DIRECT;

@@ -1339,9 +1339,14 @@ __global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_const
   __syncthreads();
   const uint32_t r = blockIdx.x;
   const uint64_t *hdr = reinterpret_cast<const uint64_t *>(P.slot);
-  if (!wait_word(hdr + 8 + r, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
-  if (r == 0 && threadIdx.x == 0 && (ld_volatile(hdr) != P.bytes || ld_volatile(hdr + 1) != P.tag))
-    atomicExch(P.err, DERR_MISMATCH);
+  // every CTA first checks the sender's size and tag (CTA 0's flag): a receive posted
+  // larger than the message would otherwise wait for slices that never come
+  if (!wait_word(hdr + 8, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
+  if (ld_volatile(hdr) != P.bytes || ld_volatile(hdr + 1) != P.tag) {
+    if (threadIdx.x == 0) atomicExch(P.err, DERR_MISMATCH);
+    return;
+  }
+  if (r > 0 && !wait_word(hdr + 8 + r, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
   const uint8_t *data = P.slot + kEagerHdr + ld_volatile(hdr + 16 + r);
   const uint64_t a = static_cast<uint64_t>(r) * kEagerSlice;
   const uint64_t e = a + kEagerSlice < P.bytes ? a + kEagerSlice : P.bytes;

@@ -482,6 +482,8 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   for (int i = 1; i < cfg.npaths; ++i)
     if (cfg.bytes[i]) staged += g_stage;
   P.g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged));
+  if (staged && P.g_direct > static_cast<uint32_t>(c->sms))  // whole CTAs per SM beside staged groups
+    P.g_direct = P.g_direct / static_cast<uint32_t>(c->sms) * static_cast<uint32_t>(c->sms);
   uint32_t next = P.g_direct;
   uint64_t off = cfg.bytes[0];
   uint32_t np = 0;

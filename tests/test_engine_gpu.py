@@ -288,20 +288,22 @@ def test_calibrate_window_installs_sane_parameters_and_window_selection_is_bit_e
 
 
 def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
-    # NEXT f4 (P:360 Observation 4; readings C20/C21): the per-band Step-1 fit installs
-    # one parameter set per band, and the model error at small sizes — where the single
-    # asymptotic Hockney line over-estimates the time — drops.
+    # NEXT f4 (P:360 Observation 4: "less accurate for smaller message sizes"; readings
+    # C20/C21): the per-band Step-1 fit installs one parameter set per band, and the
+    # model error at small sizes — 64 KiB, 1 MiB, 2 MiB, where the single asymptotic
+    # Hockney line mispredicts the time — drops below 15 %.
     c = mp.Context(device=0, n_loop_relays=2, host_path=1, slot_bytes=32 * MiB, heap_bytes=16 * MiB)
     c.set_options(mode=mp.MP_MODEL_B200)
     c.calibrate(reps=3)
-    sizes = [16 * MiB, 32 * MiB, 48 * MiB]
-    src = torch.randint(0, 256, (48 * MiB,), dtype=torch.uint8, device="cuda")
+    sizes = [64 * 1024, 1 * MiB, 2 * MiB]
+    src = torch.randint(0, 256, (2 * MiB,), dtype=torch.uint8, device="cuda")
     dst = torch.empty_like(src)
     s = torch.cuda.Stream()
 
-    def window_time(n, cfg, w=16, reps=5):
-        # the window is captured in a CUDA graph so that it is GPU-bound: under PDL a
-        # back-to-back 16 MiB message takes ~4 µs, about one Python-loop iteration
+    def window_time(n, cfg, w=64, reps=7):
+        # the window is captured in a CUDA graph so that it is GPU-bound (Step 1 times
+        # its band windows the same way, reading C21): enqueued from Python a small
+        # message costs more host time than its ~1-2 µs on the GPU
         assert sum(cfg.as_dict()["bytes"][1:]) == 0, "B200 mode picks direct-only here"
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
@@ -334,7 +336,7 @@ def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
         cfg = c.select(0, 0, n)
         t = window_time(n, cfg)
         err_band.append(abs(cfg.t_pred - t) / t)
-    assert max(err_band) < 0.25 and sum(err_band) < sum(err_base), (err_base, err_band)
+    assert max(err_band) < 0.15 and sum(err_band) < sum(err_base), (err_base, err_band)
     ctx_sum = dict(base=err_base, bands=err_band)
     print("E_pred base vs banded", ctx_sum)
     c.close()
