@@ -345,12 +345,16 @@ int mp_select_window(mp_ctx *ctx, int src, int dst, uint64_t bytes, uint32_t win
 int mp_set_host_duplex(mp_ctx *ctx, int gpu, double kappa);
 int mp_get_host_duplex(mp_ctx *ctx, int gpu, double *kappa);
 
-/* mp_calibrate_window — Step 1 for the C24/C25 parameters of the loopback pair
- * (0, 0).  For every path alone (all bytes on it; staged paths in >= 8 chunks) and
- * every size (NULL/0 = 4, 16, 64 MiB) it times one message on an idle stream (T1) and
- * `window` (0 = 16) back-to-back messages (TW), median of `reps` (0 = 7).  Then
- * tau = max(0, median(T1 − mp_predict) over the direct path's sizes), and h_i = median over sizes of
- * max(0, T1 − tau − (TW − T1)/(window − 1)) (the serve-bound branch of C24).  κ of
+/* mp_calibrate_window — Step 1 for the C24/C25/C27 parameters of the loopback
+ * pair (0, 0), timed as osu_bw times a window: the host clock around the
+ * mp_xfer enqueues and the stream synchronisation that completes them.  First the host
+ * submission time per call (C27; the marginal host-clock cost of one more 64 KiB
+ * direct-only message in an OMB-style window, mp_set_submit_time).  Then, for every path alone (all bytes on it; staged
+ * paths in >= 8 chunks) and every size (NULL/0 = 64 KiB, 1, 4, 16, 64 MiB), one message
+ * on an idle stream (T1) and `window` (0 = 16) back-to-back messages (TW), median of
+ * `reps` (0 = 7); tau = max(0, median(T1 − mp_predict) over the direct path's sizes),
+ * h_i = median over the serve-bound sizes of max(0, T1 − tau − (TW − T1)/(window − 1))
+ * (mp_fit_window with h_sub).  κ of
  * this GPU = the mean of (simplex / duplex time) of the two host legs at 64 MiB, each
  * leg moved by relay_ctas CTAs as in the engine.  Installs them with
  * mp_set_window_model / mp_set_host_duplex.  Parameters measured on B200: parity
@@ -363,10 +367,22 @@ int mp_calibrate_window(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int wind
  * on an idle stream), TW = tw[j] (`window` >= 2 back-to-back messages) and the model's
  * time pred[j] of one message.  *tau = max(0, median over path-0 samples of
  * t1 − pred) (0 without one); h[i] = median over path i's samples of
- * max(0, t1 − tau − (tw − t1)/(window − 1)) (0 without one); h has npaths entries.
- * Medians of an even count take the upper middle value.  Errors: MP_ERR_INVALID. */
+ * max(0, t1 − tau − (tw − t1)/(window − 1)) (0 without one), skipping the samples whose
+ * steady per-message time (tw − t1)/(window − 1) is <= h_sub·(1 + 1e-6) (submission-
+ * bound, reading C27; h_sub = 0 keeps every sample); h has npaths entries.  Medians of
+ * an even count take the upper middle value.  Errors: MP_ERR_INVALID. */
 int mp_fit_window(const int *path, const double *t1, const double *tw, const double *pred, int m,
-                  int window, int npaths, double *h, double *tau);
+                  int window, int npaths, double h_sub, double *h, double *tau);
+
+/* Host submission time per message (reading C27; NEXT f4 — P:360/P:375: small messages
+ * behave differently; their windows are bound by the host's cost per call): the messages
+ * of a window are enqueued h_sub seconds apart, so in mp_predict_window /
+ * mp_select_window every path's (and the port's) per-message step is
+ * max(a_i, T_i − a_i, h_sub).  One value per context (the caller's cost per mp_send /
+ * mp_xfer call); mp_calibrate_window measures it from C; 0 by default.
+ * Errors: MP_ERR_INVALID (negative or not finite). */
+int mp_set_submit_time(mp_ctx *ctx, double seconds);
+int mp_get_submit_time(mp_ctx *ctx, double *seconds);
 
 /* ---------------------------------------------------------------- memory */
 

@@ -41,3 +41,14 @@ def stage_times(x: float, k: int, alpha: float, beta: float, eps: float, alpha2:
     """Per-chunk stage times of Eq 12, m = x/k."""
     m = x / k
     return alpha + m / beta, eps + alpha2 + (m / beta2 if beta2 != math.inf else 0.0)
+
+
+def simulate_window(w: int, a: float, b: float, h_sub: float = 0.0) -> float:
+    """Finish time of w messages through a two-stage pipeline (reading C24: an issue
+    phase a that may overlap the previous message, then a serve phase b), message j
+    released by the host at (j − 1)·h_sub (reading C27)."""
+    f1 = f2 = 0.0
+    for j in range(w):
+        f1 = max(f1, j * h_sub) + a       # issue: after the previous issue and the release
+        f2 = max(f2, f1) + b              # serve: after its issue and the previous serve
+    return f2

@@ -28,6 +28,18 @@ active paths with w_i > 0).  A window also pays a fixed completion cost τ
 
 w = 1 gives O2 (+ τ); h = 0 gives w·T (+ τ), the paper's per-message model.
 
+C27 — host submission (NEXT f4's small-message regime): the messages of a
+window are enqueued by the host one call at a time, h_sub seconds apart (the caller's
+cost per mp_send / mp_xfer call, calibrated), so message j cannot start before
+(j − 1)·h_sub.  For the two-stage pipeline with those release times the finish of the
+last message is (a flow-shop argument on the release-time grid; pinned against the
+event simulation of oracle/pipeline.py)
+
+    T_i^w = T_i + (w − 1)·max(a_i, T_i − a_i, h_sub),
+
+the same for the port; h_sub = 0 is C24.  Small messages, whose GPU time is below the
+host's cost per call, are submission-bound: T^w ≈ τ + T_1 + (w − 1)·h_sub.
+
 Selection for a window (``select_window``): while serve >= issue on every path,
 T_i^w / w = T_i − (1 − 1/w)·a_i, i.e. each path's per-message Δ_i drops by
 (1 − 1/w)·a_i and the port's α_S by (1 − 1/w)·a_S (a_S over the paths the mask
@@ -66,15 +78,18 @@ def port_issue_part(port: M.Port, paths, h, active) -> float:
     return min([port.alpha] + a) if a else 0.0
 
 
-def path_window_time(t1: float, a: float, w: int) -> float:
+def path_window_time(t1: float, a: float, w: int, h_sub: float = 0.0) -> float:
     """C24: two-stage pipeline (issue a, serve t1 − a) over w messages:
-    T^w = t1 + (w − 1)·max(a, t1 − a)."""
-    return t1 + (w - 1) * max(a, t1 - a)
+    T^w = t1 + (w − 1)·max(a, t1 − a); C27: messages released h_sub apart,
+    T^w = t1 + (w − 1)·max(a, t1 − a, h_sub)."""
+    return t1 + (w - 1) * max(a, t1 - a, h_sub)
 
 
 def evaluate_window(n: int, w: int, nbytes, chunks, paths: Sequence[M.Path], h: Sequence[float],
-                    opts: M.Options, port: Optional[M.Port] = None, tau: float = 0.0) -> float:
-    """(W1): time of w back-to-back messages of n bytes with the config (nbytes, chunks)."""
+                    opts: M.Options, port: Optional[M.Port] = None, tau: float = 0.0,
+                    h_sub: float = 0.0) -> float:
+    """(W1): time of w back-to-back messages of n bytes with the config (nbytes, chunks);
+    h_sub = the host's submission time per message (C27)."""
     assert w >= 1 and sum(nbytes) == n
     if n == 0:
         return 0.0
@@ -88,19 +103,22 @@ def evaluate_window(n: int, w: int, nbytes, chunks, paths: Sequence[M.Path], h: 
             ti = p.alpha + b / p.beta                          # Eq 6
         else:
             ti = M.pipelined_time(float(b), int(k), p, opts.mode)  # Eq 13
-        t = max(t, path_window_time(ti + s, issue_part(p, hi), w))
+        t = max(t, path_window_time(ti + s, issue_part(p, hi), w, h_sub))
     if opts.mode == M.B200 and port is not None and port.beta != M.INF:
         load = sum(p.w * b for p, b in zip(paths, nbytes))
         if load > 0:
             a_s = port_issue_part(port, paths, h, active)
-            t = max(t, path_window_time(port.alpha + load / port.beta, a_s, w))
+            t = max(t, path_window_time(port.alpha + load / port.beta, a_s, w, h_sub))
     return tau + t
 
 
 def select_window(n: int, w: int, paths: Sequence[M.Path], h: Sequence[float], opts: M.Options,
-                  port: Optional[M.Port] = None, path_mask=None, tau: float = 0.0) -> M.Config:
+                  port: Optional[M.Port] = None, path_mask=None, tau: float = 0.0,
+                  h_sub: float = 0.0) -> M.Config:
     """C24 selection: O3 on the per-message coefficients of a window (Δ_i − (1 − 1/w)·a_i,
-    port α_S − (1 − 1/w)·a_S over the mask's paths); t_pred = (W1) of the result, t_level = w·(per-message level) + τ."""
+    port α_S − (1 − 1/w)·a_S over the mask's paths); t_pred = (W1) of the result (with
+    C27's h_sub), t_level = w·(per-message level) + τ.  (A submission-bound window's
+    time does not depend on the split; the split is chosen for the serve-bound case.)"""
     assert w >= 1
     shift = [(1.0 - 1.0 / w) * issue_part(p, hi) for p, hi in zip(paths, h)]
     wport = None
@@ -111,7 +129,7 @@ def select_window(n: int, w: int, paths: Sequence[M.Path], h: Sequence[float], o
     cfg = M.select(n, paths, opts, wport, path_mask, dshift=shift)
     if n == 0:
         return cfg
-    cfg.t_pred = evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, tau)
+    cfg.t_pred = evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, tau, h_sub)
     cfg.t_level = w * cfg.t_level + tau
     return cfg
 
@@ -159,18 +177,21 @@ def select_flows_duplex(flows, pair_paths, pair_port, opts: M.Options, kappa, wi
 
 # ----------------------------------------------------------------------------- C24 fit
 
-def fit_window(samples, window: int, npaths: int):
+def fit_window(samples, window: int, npaths: int, h_sub: float = 0.0):
     """The C24 estimator of Step 1 (mp_calibrate_window): samples = [(path, T1, TW, pred)]
     with T1 one message on an idle stream, TW `window` back-to-back messages, pred the
     model's one-message time.  τ = max(0, median(T1 − pred) over the direct path's
     samples); h_i = median over path i's samples of max(0, T1 − τ − (TW − T1)/(W − 1))
-    (the serve-bound branch of W1: TW − T1 = (W − 1)·(T_i − a_i)).  Medians of an even
-    count take the upper middle value."""
+    (the serve-bound branch of W1: TW − T1 = (W − 1)·(T_i − a_i)).  C27: a sample whose
+    steady per-message time (TW − T1)/(W − 1) does not exceed the host's submission time
+    h_sub·(1 + 1e-6) is submission-bound and says nothing about a_i — it is skipped.
+    Medians of an even count take the upper middle value."""
     from statistics import median_high
     d = [t1 - pred for p, t1, _, pred in samples if p == 0]
     tau = max(0.0, median_high(d)) if d else 0.0
     h = []
     for i in range(npaths):
-        a = [max(0.0, t1 - tau - (tw - t1) / (window - 1)) for p, t1, tw, _ in samples if p == i]
+        a = [max(0.0, t1 - tau - (tw - t1) / (window - 1)) for p, t1, tw, _ in samples
+             if p == i and (tw - t1) / (window - 1) > h_sub * (1 + 1e-6)]
         h.append(median_high(a) if a else 0.0)
     return h, tau

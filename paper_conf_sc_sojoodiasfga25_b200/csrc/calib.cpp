@@ -11,6 +11,7 @@
 // ε of a staging device is half the round trip of a flag ping-pong between two CTAs
 // through that device's flag memory (the same release/acquire the pipeline uses).
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstring>
 #include <string>
@@ -643,14 +644,21 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
   return calibrate_loop_bands(c, edges, reps);
 }
 
-// NEXT f2 window / duplex calibration (readings C24, C25), loopback pair (0, 0).
-// Per path alone and per size: T1 = one message on an idle stream, TW = W back-to-back
-// messages (CUDA events around the enqueue, a stream sync before each window — OMB's
-// wait-all).  τ = median(T1 − mp_predict) over the direct path's sizes, clamped >= 0;
-// the steady per-message
-// time s = (TW − T1)/(W − 1) = max(a, T1 − τ − a), read in the serve-bound branch:
-// a = T1 − τ − s; h_i = median over sizes of max(0, a).  κ of this GPU = the host
-// legs' duplex / simplex rate (D2H and H2D alone, then both at once, 64 MiB).
+// NEXT f2 window / duplex calibration (readings C24, C25, C27), loopback pair (0, 0).
+//   h_sub (C27) = the host's time per mp_xfer call: the marginal host-clock cost of
+//                 one more 64 KiB direct-only message in an OMB-style window (enqueue,
+//                 wait): (t(64 calls) − t(16 calls)) / 48, medians of 2·reps;
+//   per path alone and per size: T1 = one message on an idle stream, TW = W messages
+//   back to back (CUDA events around the enqueue, a stream sync before each window);
+//   (h_i, τ) = mp_fit_window(h_sub): τ = median(T1 − mp_predict) over the direct
+//   path's sizes, clamped >= 0; the steady per-message time s = (TW − T1)/(W − 1) =
+//   max(a, T1 − τ − a, h_sub), read in the serve-bound branch (s > h_sub):
+//   a = T1 − τ − s; h_i = median over those sizes of max(0, a);
+//   then τ += the host's completion overhead of a window, as osu_bw sees it (its
+//   wait-all): the median over the direct path's sizes of the host-clock time
+//   of one message (enqueue + stream synchronisation) minus its device time.
+// κ of this GPU = the host legs' duplex / simplex rate (D2H and H2D alone, then both at
+// once, 64 MiB).
 extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int window, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
@@ -662,7 +670,7 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
   if (sizes_in && nsizes > 0)
     sizes.assign(sizes_in, sizes_in + nsizes);
   else
-    sizes = {4ull << 20, 16ull << 20, 64ull << 20};
+    sizes = {64ull << 10, 1ull << 20, 4ull << 20, 16ull << 20, 64ull << 20};
   uint64_t big = 0;
   for (uint64_t s : sizes) big = std::max(big, s);
   if (big == 0) return cfail(c, MP_ERR_INVALID, "sizes must be > 0");
@@ -685,6 +693,7 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
   CKC(cudaMemset(src, 0x3c, big));
   CKC(cudaDeviceSynchronize());
   int st = MP_OK;
+  using clk = std::chrono::steady_clock;
   auto timed = [&](const mp_config &cfg, uint64_t n, int W, double *out) -> int {
     std::vector<double> ts;
     for (int r = 0; r < reps + 1; ++r) {
@@ -701,9 +710,65 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
     *out = median(ts);
     return MP_OK;
   };
+  auto timed_host = [&](const mp_config &cfg, uint64_t n, double *out) -> int {  // enqueue + wait-all
+    std::vector<double> ts;
+    for (int r = 0; r < reps + 1; ++r) {
+      CKC(cudaStreamSynchronize(b.s));
+      const auto t0 = clk::now();
+      if (int e = mp_xfer(c, dst, src, n, &cfg, b.s)) return e;
+      CKC(cudaStreamSynchronize(b.s));
+      if (r > 0) ts.push_back(std::chrono::duration<double>(clk::now() - t0).count());
+    }
+    *out = median(ts);
+    return MP_OK;
+  };
+  // C27: the host's submission time per call
+  double h_sub = 0.0;
+  {
+    mp_config d4;
+    std::memset(&d4, 0, sizeof(d4));
+    d4.npaths = np;
+    for (int j = 0; j < np; ++j) d4.path[j] = paths[j];
+    d4.bytes[0] = 65536;
+    d4.chunks[0] = 1;
+    // the marginal host-clock cost of one more call in an OMB-style window (enqueue
+    // W calls, wait for them): (t(64) − t(16)) / 48 — fixed costs (the first launch on
+    // an idle stream, the wait) cancel.  64 KiB messages: their GPU time is below the
+    // host's, and long enough for the next launch to overlap them (a 4 KiB kernel is
+    // launch-bound on the GPU itself: ~2.9 µs per message vs ~2.0 µs from 64 KiB up)
+    // Each t(W) is the mean over 50 consecutive windows, after 0.2 s of them: a
+    // sustained window loop runs at the GPU's boost clock, isolated bursts do not (and
+    // take ~2.9 µs per message instead of ~2.0).
+    auto burst = [&](int W, double *out) -> int {
+      std::vector<double> ts;
+      const auto warm = clk::now();
+      while (std::chrono::duration<double>(clk::now() - warm).count() < 0.2) {
+        for (int w = 0; w < W; ++w)
+          if (int e = mp_xfer(c, dst, src, 65536, &d4, b.s)) return e;
+        CKC(cudaStreamSynchronize(b.s));
+      }
+      for (int r = 0; r < reps; ++r) {
+        const auto t0 = clk::now();
+        for (int it = 0; it < 50; ++it) {
+          for (int w = 0; w < W; ++w)
+            if (int e = mp_xfer(c, dst, src, 65536, &d4, b.s)) return e;
+          CKC(cudaStreamSynchronize(b.s));
+        }
+        ts.push_back(std::chrono::duration<double>(clk::now() - t0).count() / 50);
+      }
+      *out = median(ts);
+      return MP_OK;
+    };
+    double t16 = 0.0, t64 = 0.0;
+    if ((st = burst(16, &t16)) || (st = burst(64, &t64))) return st;
+    std::vector<double> hs{std::max(0.0, (t64 - t16) / 48.0)};
+    CKC(cudaStreamSynchronize(b.s));
+    if (st) return st;
+    h_sub = median(hs);
+  }
   struct Sample {
     int path;
-    double t1, tw, pred;
+    double t1, tw, pred, t1_host;
   };
   std::vector<Sample> smp;
   const uint64_t slot_lim = c->opts.slot_bytes ? c->opts.slot_bytes : c->slot_bytes;
@@ -721,10 +786,11 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
         cfg.chunks[i] = static_cast<uint32_t>(std::max<uint64_t>(1, k));
         if ((n + cfg.chunks[i] - 1) / cfg.chunks[i] > slot_lim) continue;
       }
-      Sample sm{i, 0, 0, 0};
+      Sample sm{i, 0, 0, 0, 0};
       if ((st = mp_predict(c, 0, 0, n, &cfg, &sm.pred))) break;
       if ((st = timed(cfg, n, 1, &sm.t1))) break;
       if ((st = timed(cfg, n, window, &sm.tw))) break;
+      if (i == 0 && (st = timed_host(cfg, n, &sm.t1_host))) break;
       smp.push_back(sm);
     }
   // κ: host legs alone and at once (reading C25)
@@ -761,9 +827,14 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
   }
   double h[MP_MAX_PATHS], tau = 0.0;
   if (int e = mp_fit_window(sp.data(), s1.data(), sw.data(), spred.data(), static_cast<int>(smp.size()), window, np,
-                            h, &tau))
+                            h_sub, h, &tau))
     return cfail(c, e, "window fit failed");
+  std::vector<double> sync;
+  for (const Sample &sm : smp)
+    if (sm.path == 0) sync.push_back(sm.t1_host - sm.t1);
+  if (!sync.empty()) tau += std::max(0.0, median(sync));
   if (int e = mp_set_window_model(c, 0, 0, h, np, tau)) return e;
+  if (int e = mp_set_submit_time(c, h_sub)) return e;
   if (int e = mp_set_host_duplex(c, c->rank, std::max(kappa, 1e-3))) return e;
   return MP_OK;
 }
@@ -774,7 +845,7 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
 // staging-model error.  Per path, the steady per-message time s = (TW − T1)/(W − 1) =
 // max(a, T1 − τ − a), read in the serve-bound branch: a = T1 − τ − s.
 extern "C" int mp_fit_window(const int *path, const double *t1, const double *tw, const double *pred, int m,
-                             int window, int npaths, double *h, double *tau) {
+                             int window, int npaths, double h_sub, double *h, double *tau) {
   if (!path || !t1 || !tw || !pred || !h || !tau || m < 1 || window < 2 || npaths < 1 || npaths > MP_MAX_PATHS)
     return MP_ERR_INVALID;
   std::vector<double> taus;
@@ -788,6 +859,7 @@ extern "C" int mp_fit_window(const int *path, const double *t1, const double *tw
     for (int j = 0; j < m; ++j)
       if (path[j] == i) {
         const double steady = (tw[j] - t1[j]) / static_cast<double>(window - 1);
+        if (!(steady > h_sub * (1.0 + 1e-6))) continue;  // submission-bound (C27): no information on a_i
         as.push_back(std::max(0.0, t1[j] - *tau - steady));
       }
     h[i] = as.empty() ? 0.0 : median(as);

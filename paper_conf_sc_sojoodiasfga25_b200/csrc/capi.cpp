@@ -727,10 +727,12 @@ int mp_predict(mp_ctx *c, int src, int dst, uint64_t bytes, const mp_config *cfg
   return MP_OK;
 }
 
-static const WindowModel &window_of_pair(mp_ctx *c, int src, int dst) {
-  static const WindowModel none;
+// The pair's window model with the context's host submission time (reading C27).
+static WindowModel window_of_pair(mp_ctx *c, int src, int dst) {
   auto it = c->windows.find(std::make_pair(src, dst));
-  return it == c->windows.end() ? none : it->second;
+  WindowModel w = it == c->windows.end() ? WindowModel() : it->second;
+  w.submit = c->submit;
+  return w;
 }
 
 int mp_select(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t mask, mp_config *out) {
@@ -774,8 +776,10 @@ int mp_select_flows(mp_ctx *c, int nflows, const mp_flow *flows, mp_config *out)
     s.mask = flows[f].path_mask;
     specs.push_back(s);
   }
+  std::vector<WindowModel> wcopy;
+  for (int f = 0; f < nflows; ++f) wcopy.push_back(window_of_pair(c, flows[f].src, flows[f].dst));
   std::vector<const WindowModel *> wms;
-  for (int f = 0; f < nflows; ++f) wms.push_back(&window_of_pair(c, flows[f].src, flows[f].dst));
+  for (int f = 0; f < nflows; ++f) wms.push_back(&wcopy[f]);
   std::vector<Selection> sel;
   select_flows(models, specs, c->opts, &sel, &c->kappa, &wms);
   for (int f = 0; f < nflows; ++f) fill_config(*models[f], sel[f], &out[f]);
@@ -843,6 +847,20 @@ int mp_select_window(mp_ctx *c, int src, int dst, uint64_t bytes, uint32_t windo
   Selection s;
   select_window(*m, window_of_pair(c, src, dst), bytes, window, mask, c->opts, &s);
   fill_config(*m, s, out);
+  return MP_OK;
+}
+
+int mp_set_submit_time(mp_ctx *c, double seconds) {
+  if (!c) return MP_ERR_INVALID;
+  if (!(seconds >= 0.0) || !std::isfinite(seconds)) return fail(c, MP_ERR_INVALID, "submit time must be finite and >= 0");
+  c->submit = seconds;
+  c->cache.clear();  // mp_select depends on it when opts.window > 1
+  return MP_OK;
+}
+
+int mp_get_submit_time(mp_ctx *c, double *seconds) {
+  if (!c || !seconds) return MP_ERR_INVALID;
+  *seconds = c->submit;
   return MP_OK;
 }
 
@@ -1059,6 +1077,7 @@ int mp_save_params(mp_ctx *c, const char *path) {
   }
   for (size_t g = 0; g < c->kappa.size(); ++g)
     if (c->kappa[g] != 1.0) std::fprintf(f, "duplex %zu 0 1 %.17g\n", g, c->kappa[g]);
+  if (c->submit > 0.0) std::fprintf(f, "submit %.17g\n", c->submit);
   std::fclose(f);
   return MP_OK;
 }
@@ -1099,6 +1118,13 @@ int mp_load_params(mp_ctx *c, const char *path) {
       continue;
     }
     if (!std::strcmp(tag, "topology") || !std::strcmp(tag, "gpu")) {
+      ++i;
+      continue;
+    }
+    if (!std::strcmp(tag, "submit")) {  // reading C27
+      double v = 0.0;
+      if (std::sscanf(ln, "%31s %lf", tag, &v) != 2) return truncated();
+      if (int s = mp_set_submit_time(c, v)) return s;
       ++i;
       continue;
     }

@@ -82,6 +82,7 @@ struct mp_ctx {
   // factors (absent = h 0, τ 0; κ 1).
   std::map<std::pair<int, int>, mpx::WindowModel> windows;
   std::vector<double> kappa;
+  double submit = 0.0;             // reading C27: host submission time per message [s]
   std::unordered_map<mpx::CacheKey, mpx::Selection, mpx::CacheKeyHash> cache;
   mp_topology topo{};              // topo.cpp: found by mp_init or injected (model-only)
   bool have_topo = false;

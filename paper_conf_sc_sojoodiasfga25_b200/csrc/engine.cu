@@ -817,6 +817,12 @@ __global__ void __launch_bounds__(kThreads, 3) xfer_kernel(const __grid_constant
   }
 }
 
+// Holds a stream for `ns` nanoseconds (calibration of the host submission time, C27).
+__global__ void spin_kernel(uint64_t ns) {
+  const uint64_t t0 = globaltimer();
+  while (globaltimer() - t0 < ns) __nanosleep(1000);
+}
+
 // Flag ping-pong between block 0 and block 1: ε probe (calibration, C12).
 __global__ void pingpong_kernel(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *err) {
   if (threadIdx.x != 0) return;
@@ -1551,6 +1557,11 @@ int launch_relay(const RelayParams &P, void *stream) {
   return static_cast<int>(cudaGetLastError());
 }
 
+int launch_spin(uint64_t ns, void *stream) {
+  spin_kernel<<<1, 32, 0, static_cast<cudaStream_t>(stream)>>>(ns);
+  return static_cast<int>(cudaGetLastError());
+}
+
 int launch_pingpong(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *err, void *stream) {
   pingpong_kernel<<<2, 32, 0, static_cast<cudaStream_t>(stream)>>>(flags, iters, timeout_ns, err);
   return static_cast<int>(cudaGetLastError());
@@ -1585,6 +1596,7 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, relay_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, pingpong_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, spin_kernel);
   return static_cast<int>(e);
 }
 

@@ -273,6 +273,8 @@ int launch_reduce(int dtype, void *dst, const void *src, uint64_t bytes, void *s
 // Flag ping-pong between two CTAs through `flags` (2 words, device or mapped host):
 // `iters` round trips; the measured time is read with events by the caller.
 int launch_pingpong(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *err, void *stream);
+// A one-warp kernel that holds `stream` for `ns` nanoseconds (Step 1 of C27).
+int launch_spin(uint64_t ns, void *stream);
 
 // Max co-resident CTAs of the transfer kernel on this device (occupancy × SMs).
 int xfer_capacity(int device, int *per_sm, int *sms);

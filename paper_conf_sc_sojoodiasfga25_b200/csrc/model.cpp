@@ -490,15 +490,17 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
 // i's message = an issue phase a_i = min(h_i, α_i) that may overlap the previous
 // message's serve phase, then the serve phase T_i − a_i: T_i^w = T_i + (w−1)·max(a_i,
 // T_i − a_i).  The port is one more such pipeline with a_S = min(α_S, min a_i of the
-// active paths through it).  T^w = τ + max(paths, port).
+// active paths through it).  T^w = τ + max(paths, port).  Reading C27: the host enqueues
+// the messages h_sub apart, so the per-message step is max(a_i, T_i − a_i, h_sub).
 
 namespace {
 inline double issue_part(const PathModel &p, const WindowModel &wm, size_t i) {
   const double h = i < wm.h.size() ? wm.h[i] : 0.0;
   return std::min(std::max(h, 0.0), p.alpha);
 }
-inline double window_of(double t1, double a, uint32_t w) {
-  return t1 + static_cast<double>(w - 1) * std::max(a, t1 - a);
+// C24, with C27's host submission: message j is released (j − 1)·h_sub after the first
+inline double window_of(double t1, double a, uint32_t w, double h_sub) {
+  return t1 + static_cast<double>(w - 1) * std::max(std::max(a, t1 - a), h_sub);
 }
 double port_issue(const PairModel &m, const WindowModel &wm, const std::vector<char> &act) {
   double a = kInf;
@@ -522,12 +524,13 @@ double predict_window(const PairModel &m, const WindowModel &wm, uint64_t n, uin
     const PathModel &q = m.paths[i];
     const double b = static_cast<double>(bytes[i]);
     const double ti = (q.kind == K_DIRECT) ? q.alpha + b / q.beta : staged_time(q, b, chunks[i], o.mode);
-    t = std::max(t, window_of(ti + st[i], issue_part(q, wm, i), w));
+    t = std::max(t, window_of(ti + st[i], issue_part(q, wm, i), w, wm.submit));
   }
   if (o.mode == M_B200 && m.has_port()) {
     double load = 0.0;
     for (size_t i = 0; i < p; ++i) load += m.paths[i].w * static_cast<double>(bytes[i]);
-    if (load > 0.0) t = std::max(t, window_of(m.port_alpha + load / m.port_beta, port_issue(m, wm, act), w));
+    if (load > 0.0)
+      t = std::max(t, window_of(m.port_alpha + load / m.port_beta, port_issue(m, wm, act), w, wm.submit));
   }
   return wm.tau + t;
 }

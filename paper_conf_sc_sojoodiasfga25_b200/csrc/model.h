@@ -62,6 +62,7 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
 struct WindowModel {
   std::vector<double> h;
   double tau = 0.0;
+  double submit = 0.0;  // reading C27: host submission time per message (the context's)
 };
 // Time of w back-to-back messages of n bytes with one config (W1).
 double predict_window(const PairModel &m, const WindowModel &wm, uint64_t n, uint32_t w,

@@ -186,8 +186,10 @@ def lib():
             "mp_set_host_duplex": (C.c_int, [P, C.c_int, C.c_double]),
             "mp_calibrate_window": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int, C.c_int]),
             "mp_fit_window": (C.c_int, [C.POINTER(C.c_int), C.POINTER(C.c_double), C.POINTER(C.c_double),
-                                        C.POINTER(C.c_double), C.c_int, C.c_int, C.c_int, C.POINTER(C.c_double),
-                                        C.POINTER(C.c_double)]),
+                                        C.POINTER(C.c_double), C.c_int, C.c_int, C.c_int, C.c_double,
+                                        C.POINTER(C.c_double), C.POINTER(C.c_double)]),
+            "mp_set_submit_time": (C.c_int, [P, C.c_double]),
+            "mp_get_submit_time": (C.c_int, [P, C.POINTER(C.c_double)]),
             "mp_get_host_duplex": (C.c_int, [P, C.c_int, C.POINTER(C.c_double)]),
             "mp_get_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
             "mp_set_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
@@ -213,7 +215,7 @@ def exported_symbols() -> List[str]:
             "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
             "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_fit_window",
-            "mp_get_topology", "mp_set_topology"]
+            "mp_get_topology", "mp_set_topology", "mp_set_submit_time", "mp_get_submit_time"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -227,12 +229,12 @@ def fit_hockney(n: Sequence[float], t: Sequence[float]):
 
 
 def fit_window(path: Sequence[int], t1: Sequence[float], tw: Sequence[float], pred: Sequence[float],
-               window: int, npaths: int):
-    """mp_fit_window: (h[npaths], τ) of the C24 estimator (NEXT f2)."""
+               window: int, npaths: int, h_sub: float = 0.0):
+    """mp_fit_window: (h[npaths], τ) of the C24 estimator (NEXT f2; C27's h_sub)."""
     m = len(path)
     h, tau = (C.c_double * max(1, npaths))(), C.c_double()
     st = lib().mp_fit_window((C.c_int * m)(*path), (C.c_double * m)(*t1), (C.c_double * m)(*tw),
-                             (C.c_double * m)(*pred), m, window, npaths, h, C.byref(tau))
+                             (C.c_double * m)(*pred), m, window, npaths, h_sub, h, C.byref(tau))
     if st != 0:
         raise MPError(st, "mp_fit_window")
     return [h[i] for i in range(npaths)], tau.value
@@ -449,6 +451,15 @@ class Context:
         """mp_calibrate_window (loopback; readings C24, C25)."""
         arr = (C.c_uint64 * len(sizes))(*sizes) if sizes else None
         self._ck(lib().mp_calibrate_window(self.h, arr, len(sizes) if sizes else 0, window, reps))
+
+    def set_submit_time(self, seconds: float):
+        """mp_set_submit_time (reading C27): the host's time per enqueued message."""
+        self._ck(lib().mp_set_submit_time(self.h, seconds))
+
+    def get_submit_time(self) -> float:
+        v = C.c_double()
+        self._ck(lib().mp_get_submit_time(self.h, C.byref(v)))
+        return v.value
 
     def get_host_duplex(self, gpu) -> float:
         k = C.c_double()

@@ -8,7 +8,8 @@
 //   g++ -O2 -std=c++17 -I include -I /usr/local/cuda/include scripts/omb_window.cpp \
 //       -L paper_conf_sc_sojoodiasfga25_b200/_lib -lmpx -L /usr/local/cuda/lib64 -lcudart \
 //       -Wl,-rpath,'$ORIGIN/../paper_conf_sc_sojoodiasfga25_b200/_lib' -o scripts/omb_window
-//   ./scripts/omb_window [bands]   → one JSON line of calibrated parameters, then one per (size, window)
+//   ./scripts/omb_window [bands|asym] [max_bytes] [nobibw]
+//       → one JSON line of calibrated parameters, then one per (size, window)
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -47,7 +48,8 @@ static void print_cfg(const char *key, const mp_config &c) {
 
 int main(int argc, char **argv) {
   const bool bands = argc > 1 && std::strcmp(argv[1], "bands") == 0;
-  const uint64_t maxn = 1ull << 30;
+  const uint64_t maxn = argc > 2 ? std::strtoull(argv[2], nullptr, 10) : 1ull << 30;  // largest message
+  const bool skip_bibw = argc > 3 && std::strcmp(argv[3], "nobibw") == 0;
   mp_init_args a{};
   a.world = 1;
   a.n_loop_relays = 6;
@@ -65,12 +67,13 @@ int main(int argc, char **argv) {
   if (bands) MK(mp_calibrate_bands(ctx, nullptr, 0, 5));
   MK(mp_calibrate_window(ctx, nullptr, 0, 16, 7));
   {
-    double h[MP_MAX_PATHS], tau = 0, kappa = 0;
+    double h[MP_MAX_PATHS], tau = 0, kappa = 0, sub = 0;
     int np = 0;
     MK(mp_get_window_model(ctx, 0, 0, h, &np, &tau));
     MK(mp_get_host_duplex(ctx, 0, &kappa));
-    std::printf("{\"calibrated\": true, \"bands\": %s, \"tau_us\": %.3f, \"kappa\": %.4f, \"h_us\": [", bands ? "true" : "false",
-                tau * 1e6, kappa);
+    MK(mp_get_submit_time(ctx, &sub));
+    std::printf("{\"calibrated\": true, \"bands\": %s, \"tau_us\": %.3f, \"submit_us\": %.3f, \"kappa\": %.4f, \"h_us\": [",
+                bands ? "true" : "false", tau * 1e6, sub * 1e6, kappa);
     for (int i = 0; i < np; ++i) std::printf("%s%.3f", i ? ", " : "", h[i] * 1e6);
     std::printf("]}\n");
   }
@@ -105,6 +108,26 @@ int main(int argc, char **argv) {
   MK(mp_predict_window(ctx, 0, 0, 4, 1, &ack, &ack1));
   MK(mp_predict_window(ctx, 0, 0, 4, 2, &ack, &ack2));
   const double ack_inc = ack2 - ack1;  // one more (back-to-back) 4-byte message
+
+  {  // C27 cross-check: the marginal host cost of one more 64 KiB message, this process's loop
+    mp_config c64;
+    MK(mp_select(ctx, 0, 0, 65536, 1, &c64));
+    auto burst = [&](int W) {  // mean of 100 consecutive windows (the loop osu_bw runs)
+      for (int it = 0; it < 20; ++it) {
+        for (int w = 0; w < W; ++w) MK(mp_xfer(ctx, B, A, 65536, &c64, s1));
+        CK(cudaStreamSynchronize(s1));
+      }
+      const auto t0 = std::chrono::steady_clock::now();
+      for (int it = 0; it < 100; ++it) {
+        for (int w = 0; w < W; ++w) MK(mp_xfer(ctx, B, A, 65536, &c64, s1));
+        CK(cudaStreamSynchronize(s1));
+      }
+      return std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() / 100;
+    };
+    const double t16 = burst(16), t64 = burst(64);
+    std::printf("{\"submit_check_us\": %.3f, \"t16_us\": %.3f, \"t64_us\": %.3f}\n", (t64 - t16) / 48 * 1e6,
+                t16 * 1e6, t64 * 1e6);
+  }
 
   auto omb = [&](const mp_config &cfg, uint64_t n, int w, int it) {
     auto iter = [&] {
@@ -191,7 +214,7 @@ int main(int argc, char **argv) {
     std::sort(ts.begin(), ts.end());
     return 2.0 * static_cast<double>(n) * w / ts[1] / 1e9;
   };
-  for (uint64_t n = 16ull << 20; n <= maxn; n <<= 2)
+  for (uint64_t n = 16ull << 20; n <= maxn && !skip_bibw; n <<= 2)
     for (uint32_t mask : {0u, host_mask}) {
       const int w = 16;
       const int it = std::max(2, static_cast<int>(std::min(100.0, 4e9 / (2.0 * n * w))));

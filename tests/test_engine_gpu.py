@@ -2,6 +2,7 @@
 oracle reference transfer (oracle/transfer.py, O1): bit-exact payloads, canaries
 intact, every path kind, odd sizes and misaligned offsets, the model-selected
 configs, and BASELINE.json's full sizes."""
+import os
 import numpy as np
 import pytest
 
@@ -514,3 +515,34 @@ def test_staged_slices_around_16k_blocks(ctx, kind, per_cta, src_off, dst_off):
         chunks = [1] + [0] * (len(ps) - 1)
         chunks[i] = k
         run(ctx, n, nbytes, chunks, src_off, dst_off, seed=k)
+
+
+def test_window_model_predicts_small_osu_bw_windows():
+    # NEXT f4 with NEXT f2's window model: osu_bw's own loop (a window of
+    # w back-to-back messages, a 4-byte ack, a host wait; host clock) from C through the
+    # ABI, against mp_predict_window after mp_calibrate_bands + mp_calibrate_window —
+    # size bands (C20/C21) and the host-submission term (C27): within 10 % for every
+    # window of 64 KiB - 1 MiB messages (scripts/omb_window.cpp)
+    import json
+    import shutil
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    exe = os.path.join(root, "scripts", "omb_window")
+    if not os.path.exists(exe):
+        if not shutil.which("g++"):
+            pytest.skip("no g++ to build scripts/omb_window")
+        subprocess.run(["g++", "-O2", "-std=c++17", "-I", os.path.join(root, "include"), "-I", "/usr/local/cuda/include",
+                        os.path.join(root, "scripts", "omb_window.cpp"), "-L",
+                        os.path.join(root, "paper_conf_sc_sojoodiasfga25_b200", "_lib"), "-lmpx", "-L",
+                        "/usr/local/cuda/lib64", "-lcudart", "-Wl,-rpath," +
+                        os.path.join(root, "paper_conf_sc_sojoodiasfga25_b200", "_lib"), "-o", exe], check=True)
+    out = subprocess.run([exe, "bands", str(1 << 20), "nobibw"], capture_output=True, text=True, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    rows = [json.loads(x) for x in out.stdout.splitlines() if x.startswith("{")]
+    cal = rows[0]
+    assert cal["calibrated"] and 0.5 < cal["submit_us"] < 20, cal
+    win = [r for r in rows if "w" in r and r["n"] <= 1 << 20]
+    assert len(win) >= 6
+    for r in win:
+        err = abs(r["pred_win_GBps"] - r["bw_window_cfg_GBps"]) / r["bw_window_cfg_GBps"]
+        assert err < 0.10, (r["n"], r["w"], r["pred_win_GBps"], r["bw_window_cfg_GBps"])

@@ -315,3 +315,63 @@ def test_window_fit_reads_the_serve_bound_branch():
     smp = [(0, t, WN.path_window_time(t, a, 8), t)]
     h, tau = WN.fit_window(smp, 8, 1)
     assert tau == 0.0 and abs(h[0] - (t - a)) < 1e-15
+
+
+# ------------------------------------------------------------------ C27 host submission
+
+@settings(max_examples=300, deadline=None)
+@given(st.floats(1e-7, 1e-2), st.floats(0.0, 1.0), st.integers(1, 64), st.floats(0.0, 2e-3))
+def test_submission_bound_window_is_the_release_time_simulation(t1, frac, w, h_sub):
+    # C27: message j released by the host at (j − 1)·h_sub; the two-stage pipeline with
+    # those release times, simulated event by event, finishes at
+    # t1 + (w − 1)·max(a, t1 − a, h_sub)
+    a = frac * t1
+    assert rel(WN.path_window_time(t1, a, w, h_sub), P.simulate_window(w, a, t1 - a, h_sub)) < 1e-12
+    assert P.simulate_window(w, a, t1 - a, 0.0) == pytest.approx(P.simulate_two_stage(w, a, t1 - a), rel=1e-12)
+
+
+def test_submission_bound_closed_form_and_reduction():
+    # h_sub above every phase: T^w = τ + T_1 + (w − 1)·h_sub (the split does not matter);
+    # h_sub = 0: the C24 window unchanged
+    paths = paths_from(synth.topology(4, 2, True))
+    opts = M.Options(mode=M.B200)
+    port = M.Port(2 * US, 850 * GBS)
+    n = 1 * MiB
+    cfg = M.select(n, paths, opts, port)
+    h = [0.5 * p.alpha for p in paths]
+    t1 = M.evaluate(n, cfg.bytes, cfg.chunks, paths, opts, port)
+    for w in (2, 16, 64):
+        big = 10 * t1
+        got = WN.evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, tau=3 * US, h_sub=big)
+        assert rel(got, 3 * US + t1 + (w - 1) * big) < 1e-12
+        assert WN.evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, 3 * US, 0.0) == \
+            WN.evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, 3 * US)
+        # never below the per-message window without submission cost
+        assert got >= WN.evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, 3 * US)
+
+
+def test_fit_window_skips_submission_bound_samples():
+    # C27 in Step 1: samples whose steady per-message time is the host's submission
+    # time carry no information on the issue overlap a_i
+    t, a, W, hs = 10 * US, 4 * US, 16, 12 * US
+    serve_bound = (0, 4 * t, WN.path_window_time(4 * t, a, W, hs), 4 * t)  # steady = 4t − a = 36 µs
+    sub_bound = (0, t, WN.path_window_time(t, a, W, hs), t)                # steady = 12 µs = h_sub
+    h, tau = WN.fit_window([serve_bound, sub_bound, serve_bound], W, 1, h_sub=hs)
+    assert tau == 0.0 and h[0] == pytest.approx(a, rel=1e-9)
+    h, _ = WN.fit_window([sub_bound], W, 1, h_sub=hs)
+    assert h == [0.0]
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_window_fit_with_submission_time_library_parity(seed):
+    # C27 in the estimator: library mp_fit_window(h_sub) = oracle fit_window(h_sub)
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    rng = random.Random(50 + seed)
+    paths = paths_from(synth.topology(seed, 2, True))
+    h = [rng.uniform(0, 1) * p.alpha for p in paths]
+    tau, hs = rng.uniform(0, 10) * US, rng.uniform(1, 30) * US
+    smp = window_samples(paths, h, tau, 16, [64 * 1024, 1 * MiB, 4 * MiB, 16 * MiB, 64 * MiB])
+    got_h, got_tau = WN.fit_window(smp, 16, len(paths), h_sub=hs)
+    lh, lt = mp.fit_window([s[0] for s in smp], [s[1] for s in smp], [s[2] for s in smp],
+                           [s[3] for s in smp], 16, len(paths), hs)
+    assert abs(lt - got_tau) <= 1e-18 and all(abs(a - b) <= 1e-18 for a, b in zip(lh, got_h))

@@ -275,3 +275,46 @@ def test_params_file_with_bands_window_and_duplex(tmp_path):
         assert c.get_window_model(0, 1) == (h, 1.5e-6) and c.get_host_duplex(3) == 0.6
         got = [c.select_window(0, 1, n, 16).as_dict() for n in (2 * MiB, 64 * MiB)]
         assert got == want
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("mode", [M.PAPER, M.B200])
+def test_submission_time_parity(seed, mode):
+    # reading C27: the context's host submission time enters every window prediction
+    # (mp_predict_window, mp_select_window's t_pred) as the oracle's h_sub; it survives
+    # the parameter file; 0 is C24
+    rng = random.Random(100 + seed)
+    tbl = table(0, 1, seed)
+    paths = [M.Path(**t) for t in tbl]
+    port = M.Port(alpha=2e-6, beta=850e9)
+    h = [rng.uniform(0, 1.5) * p.alpha for p in paths]
+    tau, h_sub = rng.uniform(0, 10e-6), rng.choice([0.0, 1.5e-6, 3e-6, 40e-6])
+    opts = M.Options(mode=mode, slot_bytes=64 * MiB)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.set_options(mode=mode, slot_bytes=64 * MiB)
+        install(c, 0, 1, tbl, port)
+        c.set_window_model(0, 1, h, tau)
+        c.set_submit_time(h_sub)
+        assert c.get_submit_time() == h_sub
+        for n in (64 * 1024, 1 * MiB, 16 * MiB):
+            for w in (2, 16, 64):
+                ref = WN.select_window(n, w, paths, h, opts, port, tau=tau, h_sub=h_sub)
+                got = c.select_window(0, 1, n, w).as_dict()
+                if got["bytes"] == ref.bytes:
+                    assert rel(got["t_pred"], ref.t_pred) < 1e-9
+                cfg = c.make_config(ref.bytes, ref.chunks, 0, 1)
+                want = WN.evaluate_window(n, w, ref.bytes, ref.chunks, paths, h, opts, port, tau, h_sub)
+                assert rel(c.predict_window(0, 1, n, w, cfg), want) < 1e-9
+    with pytest.raises(mp.MPError):
+        with mp.Context(world=W, rank=0, model_only=True) as c:
+            c.set_submit_time(-1.0)
+
+
+def test_submission_time_survives_the_params_file(tmp_path):
+    f = str(tmp_path / "p.txt")
+    with mp.Context(world=2, rank=0, model_only=True) as c:
+        c.set_submit_time(2.5e-6)
+        c.save_params(f)
+    with mp.Context(world=2, rank=0, model_only=True) as c:
+        c.load_params(f)
+        assert c.get_submit_time() == 2.5e-6
