@@ -1,7 +1,7 @@
 """Host-side cost per mp_xfer call from Python (ctypes) vs cudaMemcpyAsync through
 cuda-python, for small messages: is the OMB small-size window loop host-bound?"""
 import os, sys, time, json
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 import torch
 from cuda.bindings import runtime as rt

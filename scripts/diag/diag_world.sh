@@ -1,6 +1,6 @@
 #!/bin/bash
 # Diagnose the multi-rank engine with all ranks on one GPU (under gpurun).
-# Usage: bash scripts/diag_world.sh <outdir> <world> [MPX_NO_RELAY=0|1]
+# Usage: bash scripts/diag/diag_world.sh <outdir> <world> [MPX_NO_RELAY=0|1]
 OUT=${1:-gpurun_out/diag}; W=${2:-3}; NR=${3:-0}
 mkdir -p $OUT
 PORT=$((20000 + RANDOM % 20000))
