@@ -410,7 +410,7 @@ int mp_peer_base(mp_ctx *ctx, int rank, void **base);
  * every rank (0 is the heap, never returned).  mp_recv into [buf, buf + bytes) then
  * needs no mp_alloc copy.  The buffer must stay allocated until mp_deregister.
  * world == 1: nothing to map; returns MP_OK with a local id.
- * Pauses the persistent relay kernel: no transfer may be in flight on any rank.
+ * No transfer may be in flight on any rank (the region table is rewritten).
  * Errors: MP_ERR_STATE (model-only), MP_ERR_NOMEM (region table full, 63 regions),
  * MP_ERR_UNSUPPORTED (the allocation cannot be exported, e.g. VMM / expandable
  * segments), MP_ERR_CUDA. */

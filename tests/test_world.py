@@ -1,8 +1,8 @@
 """Multi-rank paths: world_size-2/3 process groups over gloo on 127.0.0.1.
 
 CPU: the bootstrap all-gather and the per-pair model selection are consistent
-across ranks.  GPU: the real multi-rank engine (IPC-mapped heaps, persistent relay
-kernel, shared pinned host ring) with all ranks on one B200 (same-device CUDA IPC),
+across ranks.  GPU: the real multi-rank engine (IPC-mapped heaps, on-demand relay
+kernels, shared pinned host ring) with all ranks on one B200 (same-device CUDA IPC),
 bit-exact against the oracle's reference transfer."""
 import os
 import socket
