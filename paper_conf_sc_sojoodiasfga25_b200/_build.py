@@ -37,30 +37,35 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(f) <= t for f in _inputs())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    """Build libmpx.so (default: the in-tree product library).  `out` + `defines`
+    (e.g. ["MPX_STREAM_STAGES=6"]) build a variant elsewhere for design experiments;
+    load it with MPX_LIB=<out>."""
+    lib_path = out or LIB
+    if not force and out is None and up_to_date():
         return LIB
-    os.makedirs(OUT_DIR, exist_ok=True)
+    out_dir = os.path.dirname(lib_path)
+    os.makedirs(out_dir, exist_ok=True)
     objs = []
     common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
-              "-I", os.path.join(ROOT, "include")]
+              "-I", os.path.join(ROOT, "include")] + [f"-D{d}" for d in defines]
     for s in SOURCES:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(OUT_DIR, s + ".o")
+        obj = os.path.join(out_dir, s + ".o")
         cmd = [NVCC] + ARCH + common + ["-lineinfo", "-c", src, "-o", obj]
         if s.endswith(".cu"):
             cmd += ["-Xptxas", "-v"] if verbose else []
         else:
             cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-Wall", "-I", os.path.join(ROOT, "include"),
-                   "-I", "/usr/local/cuda/include", "-c", src, "-o", obj]
+                   "-I", "/usr/local/cuda/include", "-c", src, "-o", obj] + [f"-D{d}" for d in defines]
         subprocess.run(cmd, check=True)
         objs.append(obj)
-    tmp = LIB + ".tmp"
+    tmp = lib_path + ".tmp"
     subprocess.run([NVCC] + ARCH + ["-shared", "-cudart", "static", "-o", tmp] + objs, check=True)
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib_path)
     for o in objs:
         os.remove(o)
-    return LIB
+    return lib_path
 
 
 if __name__ == "__main__":

@@ -224,8 +224,10 @@ int alloc_ring(mp_ctx *c, bool host, Ring *r) {
 
 int init_engine(mp_ctx *c) {
   CK(cudaSetDevice(c->device));
-  if (int e = xfer_capacity(c->device, &c->per_sm, &c->sms))
+  if (int e = xfer_capacity(c->device, &c->per_sm, &c->per_sm_deep, &c->sms))
     return cuda_fail(c, static_cast<cudaError_t>(e), "occupancy query");
+  if (const char *m = std::getenv("MPX_STAGES"))  // design experiments: one staged depth for every launch
+    c->force_stages = std::strcmp(m, "4") == 0 ? shallow_stages() : (std::strcmp(m, "6") == 0 ? deep_stages() : 0u);
   if (int e = preload_kernels()) return cuda_fail(c, static_cast<cudaError_t>(e), "kernel preload");
   if (const char *m = std::getenv("MPX_COPY")) c->copy_mode = std::strcmp(m, "reg") == 0 ? 0u : 1u;
   if (const char *m = std::getenv("MPX_PDL")) c->pdl = std::strcmp(m, "0") == 0 ? 0u : 1u;
@@ -270,10 +272,11 @@ int launch_loopback(mp_ctx *c, void *dst, const void *src, uint64_t n, const mp_
   P.pdl = c->pdl;
   P.bulk_stages = bulk_stages_for(cfg.bytes[0]);
   P.allow_small = 1;
-  const int cap = std::max(1, c->per_sm * c->sms);
   uint32_t staged_ctas = 0;
   for (int i = 1; i < cfg.npaths; ++i)
     if (cfg.bytes[i]) staged_ctas += 2u * static_cast<uint32_t>(c->relay_ctas);
+  P.stages = stages_for(c, staged_ctas);
+  const int cap = std::max(1, per_sm_at(c, P.stages) * c->sms);
   // direct group sized by direct_ctas(), leaving room for every staged group to be
   // co-resident.
   uint32_t g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged_ctas), c->pdl != 0);
@@ -364,6 +367,8 @@ int mpx::launch_direct_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, v
   P.bulk_stages = bulk_stages_for(n);
   P.allow_small = ctas > 0 ? 0u : 1u;  // a staged leg's calibration times its group's CTAs
   P.staged_blk = ctas > 0 ? 1u : 0u;  // staged lanes move 16 KiB TMA blocks in every engine
+  // a staged leg is timed at the depth a staged path alone runs at (one group of CTAs)
+  P.stages = ctas > 0 ? stages_for(c, 2u * static_cast<uint32_t>(ctas)) : shallow_stages();
   P.npaths = 1;
   DevPath &d = P.p[0];
   d.kind = DK_DIRECT;

@@ -95,7 +95,8 @@ struct mp_ctx {
   int relay_ctas = 16;
   uint64_t slot_bytes = 32ull << 20;
   double timeout_s = 20.0;
-  int per_sm = 0, sms = 0;
+  int per_sm = 0, per_sm_deep = 0, sms = 0;  // co-resident staged-kernel CTAs per SM (4 / 6 stages)
+  uint32_t force_stages = 0;       // env MPX_STAGES=4|6: every staged launch at that depth
   uint32_t pdl = 1;                // loopback launches use PDL (env MPX_PDL=0: off)
   uint32_t pdl_world = 0;          // multi-rank launches use PDL (env MPX_PDL_WORLD=1: on)
   uint32_t copy_mode = 1;          // direct-path copy: 1 = TMA bulk, 0 = LDG/STG (env MPX_COPY=reg)
@@ -171,6 +172,16 @@ inline uint32_t direct_ctas(const mp_ctx *c, uint64_t bytes, int room, bool full
   if (full_grid && c->copy_mode == 1) want = static_cast<uint64_t>(lim);
   return static_cast<uint32_t>(std::min<uint64_t>(want, static_cast<uint64_t>(lim)));
 }
+
+// Staged pipeline depth of a launch with `staged` staged CTAs (engine.cu): the deep
+// pipeline (6 × 16 KiB, 2 CTAs per SM) when those CTAs leave every SM room for at least
+// one more CTA (the direct group), else 4 stages (3 CTAs per SM).
+inline uint32_t stages_for(const mp_ctx *c, uint32_t staged) {
+  if (c->force_stages) return c->force_stages;
+  return staged + static_cast<uint32_t>(c->sms) <= static_cast<uint32_t>(c->per_sm_deep * c->sms) ? deep_stages()
+                                                                                                    : shallow_stages();
+}
+inline int per_sm_at(const mp_ctx *c, uint32_t stages) { return stages == deep_stages() ? c->per_sm_deep : c->per_sm; }
 
 // One direct-path fused launch dst ← src (any world; dst may be peer or mapped host).
 // ctas > 0 fixes the CTA count (calibration of a staged leg uses the staged group's).

@@ -129,10 +129,22 @@ constexpr uint32_t kBulkSmem = kBulkBlock * kBulkStages + 64;
 // Staged legs of the loopback transfer kernel use 16 KiB blocks: one CTA's TMA rate is
 // bound by the shared memory it keeps in flight (~32 KiB per ~1.5 µs round trip;
 // few-CTA sweep, profiles/r01/copybench_few*.jsonl: 20 GB/s at 4 × 8 KiB, 40 GB/s at
-// 4 × 16 KiB).  xfer_kernel launches with kXferSmem; residency drops from 4 to 3 CTAs
-// per SM, and xfer_capacity() reports that, so the co-residency cap follows.
+// 4 × 16 KiB).  Kernels with staged CTAs launch with staged_smem<D>() (below); their
+// residency (3 CTAs per SM at 4 stages, 2 at 6) comes from xfer_capacity().
 constexpr uint32_t kStagedBlock = 16384;
-constexpr uint32_t kXferSmem = kStagedBlock * kBulkStages + 64;
+// Stages of a staged lane's streamed pipeline (lane_stream) and of Step 1's staged-leg
+// timing copy (direct_leg_kernel).  Deep (6 × 16 KiB = 96 KiB in flight per CTA) moves a
+// lane ~19 % faster than 4 stages (relay ring alone, 16 lanes: 590-604 → 703-718 GB/s;
+// profiles/r02/stages) but leaves 2 CTAs per SM instead of 3, so the host picks the
+// depth per launch (deep when the staged CTAs leave every SM room for a direct CTA).
+constexpr uint32_t kDeepStages = 6;
+static_assert(kDeepStages >= kBulkStages, "staged CTAs also run the 4-stage per-chunk path");
+// dynamic shared memory of a kernel with staged CTAs of depth D: the stages, then a
+// full and an empty mbarrier per stage
+template <uint32_t D>
+constexpr uint32_t staged_smem() {
+  return kStagedBlock * D + 16 * D + 64;
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -179,7 +191,7 @@ __device__ __forceinline__ void bulk_wait_all() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
-template <int MODE, uint32_t BLK = kBulkBlock>
+template <int MODE, uint32_t BLK = kBulkBlock, uint32_t MAXD = kBulkStages>
 __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32_t r, uint32_t G,
                           uint8_t *smem, uint32_t D, bool publish_after = true) {
   if ((reinterpret_cast<uintptr_t>(dst) ^ reinterpret_cast<uintptr_t>(src)) & 15u) {
@@ -204,8 +216,8 @@ __device__ void bulk_copy(uint8_t *dst, const uint8_t *src, uint64_t len, uint32
   const uint64_t nblk = (body + BLK - 1) / BLK;
   if (r >= nblk) return;
   const uint64_t mine = (nblk - r + G - 1) / G;  // blocks r, r+G, …
-  if (D < 1 || D > kBulkStages) D = kBulkStages;
-  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + BLK * kBulkStages);
+  if (D < 1 || D > MAXD) D = MAXD;
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + BLK * MAXD);
   for (uint32_t i = 0; i < D; ++i) mbar_init(smem_u32(bars + i));
   // make the initialised barriers visible to the async proxy (no cluster: CTA scope)
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -465,7 +477,7 @@ __device__ __forceinline__ void bytes_copy(uint8_t *d, const uint8_t *s, uint64_
 }
 
 // Called by every thread of the CTA; threads other than 0, 32, 64 and 96 return at once.
-template <int MODE, class Role>
+template <int MODE, uint32_t D, class Role>
 __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
   __shared__ uint32_t s_ready;    // chunks the watcher has found ready
   __shared__ uint32_t s_taken;    // chunks taken up (consumer: loader read the words; producer: storer)
@@ -474,8 +486,7 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
   __shared__ uint32_t s_pub;      // chunks the publisher has finished (their words free)
   __shared__ uint32_t s_stop;     // 1: a wait failed
   __shared__ uint64_t s_words[kStreamAhead][5];
-  constexpr uint32_t BLK = kStagedBlock, D = kBulkStages;
-  static_assert(D == 4, "stage arithmetic below assumes 4 stages");
+  constexpr uint32_t BLK = kStagedBlock;
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + BLK * D);  // [D] loaded
   uint64_t *empty = full + D;                                      // [D] read out by its store
   const uint32_t full0 = smem_u32(full), empty0 = smem_u32(empty), smem0 = smem_u32(smem);
@@ -563,7 +574,7 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
       // the stage of this chunk's first step is free (the store of step gl - D has read
       // it out); geo[lc % 8] was last read for chunk lc - 8, which the storer left
       // more than D steps ago
-      if (gl >= D && !mbar_wait_or_stop(empty0 + 8 * (gl & 3u), ((gl >> 2) - 1) & 1u, &s_stop)) return;
+      if (gl >= D && !mbar_wait_or_stop(empty0 + 8 * (gl % D), ((gl / D) - 1) & 1u, &s_stop)) return;
       Geo &e = geo[lc % kStreamAhead];
       e.s0 = g.src;
       e.s = g.src + h;
@@ -574,13 +585,13 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
       const uint8_t *src = g.src + h;
       uint64_t rem = body;
       for (uint32_t b = 0; b < e.steps; ++b, ++gl) {
-        const uint32_t fb = full0 + 8 * (gl & 3u);
-        if (b > 0 && gl >= D && !mbar_wait_or_stop(empty0 + 8 * (gl & 3u), ((gl >> 2) - 1) & 1u, &s_stop))
+        const uint32_t fb = full0 + 8 * (gl % D);
+        if (b > 0 && gl >= D && !mbar_wait_or_stop(empty0 + 8 * (gl % D), ((gl / D) - 1) & 1u, &s_stop))
           return;
         if (rem) {
           const uint32_t n = rem < BLK ? static_cast<uint32_t>(rem) : BLK;
           mbar_expect_tx(fb, n);
-          bulk_load(smem0 + (gl & 3u) * BLK, src, n, fb);
+          bulk_load(smem0 + (gl % D) * BLK, src, n, fb);
           src += n;
           rem -= n;
         } else {
@@ -623,10 +634,10 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
       st_release_cta_shared(&s_taken, sc + 1);
     }
     // the chunk's geometry: written by the loader before it armed this first step
-    uint32_t fb = full0 + 8 * (gs & 3u);
-    if (!mbar_test(fb, (gs >> 2) & 1u)) {
+    uint32_t fb = full0 + 8 * (gs % D);
+    if (!mbar_test(fb, (gs / D) & 1u)) {
       flush();
-      if (!mbar_wait_or_stop(fb, (gs >> 2) & 1u, &s_stop)) {
+      if (!mbar_wait_or_stop(fb, (gs / D) & 1u, &s_stop)) {
         ok = false;
         break;
       }
@@ -642,17 +653,17 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
     uint64_t rem = e.body;
     const uint32_t steps = e.steps;
     for (uint32_t b = 0; b < steps; ++b, ++gs) {
-      fb = full0 + 8 * (gs & 3u);
-      if (b > 0 && !mbar_test(fb, (gs >> 2) & 1u)) {
+      fb = full0 + 8 * (gs % D);
+      if (b > 0 && !mbar_test(fb, (gs / D) & 1u)) {
         flush();
-        if (!mbar_wait_or_stop(fb, (gs >> 2) & 1u, &s_stop)) {
+        if (!mbar_wait_or_stop(fb, (gs / D) & 1u, &s_stop)) {
           ok = false;
           break;
         }
       }
       if (rem) {
         const uint32_t n = rem < BLK ? static_cast<uint32_t>(rem) : BLK;
-        bulk_store(dst, smem0 + (gs & 3u) * BLK, n);
+        bulk_store(dst, smem0 + (gs % D) * BLK, n);
         dst += n;
         rem -= n;
       } else {
@@ -661,7 +672,7 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
       // the previous step's store has read its stage: hand the stage back to the loader
       if (gs > 0) {
         bulk_wait_read<1>();
-        mbar_arrive(empty0 + 8 * ((gs - 1) & 3u));
+        mbar_arrive(empty0 + 8 * ((gs - 1) % D));
       }
       if (gs >= pub_at) {  // the oldest pending chunk's stores are kStreamLag groups back
         asm volatile("cp.async.bulk.wait_group %0;" ::"n"(kStreamLag) : "memory");
@@ -748,10 +759,11 @@ struct LoopConsumer {
   __device__ void stored(uint32_t, const uint64_t *) {}
 };
 
+template <uint32_t D>
 __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
   if (P.copy_mode == 1) {  // streamed lane (the source slice and its lane are co-aligned)
     LoopProducer R{&p, r, P.timeout_ns, P.err};
-    lane_stream<LD_SRC>(R, p.k, smem);
+    lane_stream<LD_SRC, D>(R, p.k, smem);
     return;
   }
   for (uint32_t j = 0; j < p.k; ++j) {
@@ -767,11 +779,11 @@ __device__ void run_stage_in(const DevPath &p, uint32_t r, const XferParams &P, 
   }
 }
 
-template <int MODE>
+template <int MODE, uint32_t D>
 __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, int *s_abort, uint8_t *smem) {
   if (P.copy_mode == 1 && ((reinterpret_cast<uintptr_t>(p.src) ^ reinterpret_cast<uintptr_t>(p.dst)) & 15u) == 0) {
     LoopConsumer R{&p, r, P.timeout_ns, P.err};
-    lane_stream<MODE>(R, p.k, smem);
+    lane_stream<MODE, D>(R, p.k, smem);
     return;
   }
   for (uint32_t j = 0; j < p.k; ++j) {
@@ -787,7 +799,8 @@ __device__ void run_forward(const DevPath &p, uint32_t r, const XferParams &P, i
   }
 }
 
-__global__ void __launch_bounds__(kThreads, 3) xfer_kernel(const __grid_constant__ XferParams P) {
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) xfer_kernel(const __grid_constant__ XferParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
   __shared__ int s_abort;
@@ -804,14 +817,14 @@ __global__ void __launch_bounds__(kThreads, 3) xfer_kernel(const __grid_constant
         else
           group_copy<LD_SRC>(p.dst, p.src, p.bytes, b - p.cta0_in, p.g_in);
       else
-        run_stage_in(p, b - p.cta0_in, P, &s_abort, dyn_smem);
+        run_stage_in<D>(p, b - p.cta0_in, P, &s_abort, dyn_smem);
       return;
     }
     if (p.kind == DK_STAGED && b >= p.cta0_out && b < p.cta0_out + p.g_out) {
       if (p.host_ring)
-        run_forward<LD_HOST>(p, b - p.cta0_out, P, &s_abort, dyn_smem);
+        run_forward<LD_HOST, D>(p, b - p.cta0_out, P, &s_abort, dyn_smem);
       else
-        run_forward<LD_RING>(p, b - p.cta0_out, P, &s_abort, dyn_smem);
+        run_forward<LD_RING, D>(p, b - p.cta0_out, P, &s_abort, dyn_smem);
       return;
     }
   }
@@ -1116,7 +1129,8 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
-__global__ void __launch_bounds__(kThreads, 3) send_kernel(const __grid_constant__ SendParams P) {
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) send_kernel(const __grid_constant__ SendParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
   __shared__ int s_abort;
@@ -1157,7 +1171,7 @@ __global__ void __launch_bounds__(kThreads, 3) send_kernel(const __grid_constant
     const uint64_t lstride = lane_stride(P.L.slot_bytes, d.g);
     if (P.copy_mode == 1) {  // streamed lane (source slice and lane are co-aligned)
       SendProducer R{&P, &d, r, lstride, base, s_region};
-      lane_stream<LD_SRC>(R, d.k, dyn_smem);
+      lane_stream<LD_SRC, D>(R, d.k, dyn_smem);
       return;
     }
     for (uint32_t j = 0; j < d.k; ++j) {  // A8/A9 step 1
@@ -1202,7 +1216,8 @@ __global__ void __launch_bounds__(kThreads, 3) send_kernel(const __grid_constant
   }
 }
 
-__global__ void __launch_bounds__(kThreads, 3) recv_kernel(const __grid_constant__ RecvParams P) {
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kernel(const __grid_constant__ RecvParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
   __shared__ int s_abort;
@@ -1254,7 +1269,7 @@ __global__ void __launch_bounds__(kThreads, 3) recv_kernel(const __grid_constant
   if (P.copy_mode == 1 && ((reinterpret_cast<uintptr_t>(P.buf) + s_hoff) & 15u) == s_shift) {
     // streamed lane: the host slices and their destination are co-aligned
     HostConsumer R{&P, r, lstride, s_k, s_q0, s_hoff, s_hbytes, s_shift, s_align, done};
-    lane_stream<LD_HOST>(R, static_cast<uint32_t>(s_k), dyn_smem);
+    lane_stream<LD_HOST, D>(R, static_cast<uint32_t>(s_k), dyn_smem);
     return;
   }
   for (uint64_t j = 0; j < s_k; ++j) {
@@ -1274,7 +1289,8 @@ __global__ void __launch_bounds__(kThreads, 3) recv_kernel(const __grid_constant
 // Relay (A8 step 3), one bounded launch per relayed message: CTA r forwards lane r of
 // chunks [q0, q0 + k) of the sender's ring to the destination its lane header names,
 // counts the bytes into the destination's `done` and returns the lane to the sender.
-__global__ void __launch_bounds__(kThreads, 3) relay_kernel(const __grid_constant__ RelayParams P) {
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kernel(const __grid_constant__ RelayParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   __shared__ int s_abort;
   __shared__ uint64_t s_h[5];
@@ -1284,7 +1300,7 @@ __global__ void __launch_bounds__(kThreads, 3) relay_kernel(const __grid_constan
   const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g);
   if (P.copy_mode == 1 && P.aligned) {  // streamed lane (the sender found source and target co-aligned)
     RelayConsumer R{&P, r, lstride};
-    lane_stream<LD_RING>(R, static_cast<uint32_t>(P.k), dyn_smem);
+    lane_stream<LD_RING, D>(R, static_cast<uint32_t>(P.k), dyn_smem);
     return;
   }
   for (uint64_t j = 0; j < P.k; ++j) {
@@ -1387,10 +1403,11 @@ __global__ void __launch_bounds__(kThreads, 4) direct_kernel(const __grid_consta
 // Step 1's timing copy of a loopback staged leg: the same striped TMA pipeline as
 // direct_kernel, with the staged legs' block size (kStagedBlock), so the calibrated
 // leg β is what a stage group of that many CTAs moves.
-__global__ void __launch_bounds__(kThreads, 4) direct_leg_kernel(const __grid_constant__ DirectArgs A) {
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) direct_leg_kernel(const __grid_constant__ DirectArgs A) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
-  bulk_copy<LD_SRC, kStagedBlock>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, A.stages, false);
+  bulk_copy<LD_SRC, kStagedBlock, D>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x, dyn_smem, D, false);
 }
 
 // One-shot small copy (co-aligned src/dst): thread i of the grid moves vector i of the
@@ -1503,9 +1520,12 @@ int launch_k(bool pdl, void (*kern)(KArgs...), uint32_t grid, uint32_t smem, voi
 }
 }  // namespace
 
+// The kernels with staged CTAs come in two depths (kBulkStages = 4 / kDeepStages = 6):
+// `stages` of the parameter block picks the instance and its shared memory.
 int launch_xfer(const XferParams &P, void *stream) {
   if (P.nblocks == 0) return cudaSuccess;
   const bool pdl = P.pdl != 0;
+  const bool deep = P.stages == kDeepStages;
   bool direct_only = P.p[0].kind == DK_DIRECT && P.p[0].cta0_in == 0 && P.p[0].g_in == P.nblocks;
   for (uint32_t i = 1; i < P.npaths; ++i)
     if (P.p[i].bytes) direct_only = false;
@@ -1518,11 +1538,14 @@ int launch_xfer(const XferParams &P, void *stream) {
   }
   if (direct_only) {
     const DirectArgs A{P.p[0].dst, P.p[0].src, P.p[0].bytes, P.copy_mode, P.bulk_stages};
-    if (P.copy_mode == 1 && P.staged_blk) return launch_k(pdl, direct_leg_kernel, P.nblocks, kXferSmem, stream, A);
+    if (P.copy_mode == 1 && P.staged_blk)
+      return deep ? launch_k(pdl, direct_leg_kernel<kDeepStages>, P.nblocks, staged_smem<kDeepStages>(), stream, A)
+                  : launch_k(pdl, direct_leg_kernel<kBulkStages>, P.nblocks, staged_smem<kBulkStages>(), stream, A);
     if (P.copy_mode == 1) return launch_k(pdl, direct_kernel, P.nblocks, kBulkSmem, stream, A);
     return launch_k(pdl, direct_reg_kernel, P.nblocks, 0, stream, A);
   }
-  return launch_k(pdl, xfer_kernel, P.nblocks, kXferSmem, stream, P);
+  return deep ? launch_k(pdl, xfer_kernel<kDeepStages>, P.nblocks, staged_smem<kDeepStages>(), stream, P)
+              : launch_k(pdl, xfer_kernel<kBulkStages>, P.nblocks, staged_smem<kBulkStages>(), stream, P);
 }
 
 int launch_send(const SendParams &P, void *stream) {
@@ -1537,7 +1560,9 @@ int launch_send(const SendParams &P, void *stream) {
   cfg.attrs = at;
   cfg.numAttrs = pdl ? 1 : 0;
   if (int e = static_cast<int>(cudaLaunchKernelEx(&cfg, send_gate_kernel, P))) return e;
-  return launch_k(pdl, send_kernel, P.nblocks, kXferSmem, stream, P);
+  return P.stages == kDeepStages
+             ? launch_k(pdl, send_kernel<kDeepStages>, P.nblocks, staged_smem<kDeepStages>(), stream, P)
+             : launch_k(pdl, send_kernel<kBulkStages>, P.nblocks, staged_smem<kBulkStages>(), stream, P);
 }
 
 int launch_eager_send(const EagerParams &P, void *stream) {
@@ -1549,11 +1574,16 @@ int launch_eager_recv(const EagerParams &P, void *stream) {
 }
 
 int launch_recv(const RecvParams &P, void *stream) {
-  return launch_k(P.pdl != 0, recv_kernel, P.nblocks, kXferSmem, stream, P);
+  return P.stages == kDeepStages
+             ? launch_k(P.pdl != 0, recv_kernel<kDeepStages>, P.nblocks, staged_smem<kDeepStages>(), stream, P)
+             : launch_k(P.pdl != 0, recv_kernel<kBulkStages>, P.nblocks, staged_smem<kBulkStages>(), stream, P);
 }
 
 int launch_relay(const RelayParams &P, void *stream) {
-  relay_kernel<<<P.g, kThreads, kXferSmem, static_cast<cudaStream_t>(stream)>>>(P);
+  if (P.stages == kDeepStages)
+    relay_kernel<kDeepStages><<<P.g, kThreads, staged_smem<kDeepStages>(), static_cast<cudaStream_t>(stream)>>>(P);
+  else
+    relay_kernel<kBulkStages><<<P.g, kThreads, staged_smem<kBulkStages>(), static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
 }
 
@@ -1567,20 +1597,42 @@ int launch_pingpong(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *er
   return static_cast<int>(cudaGetLastError());
 }
 
-int preload_kernels() {
-  // CUDA 12 loads kernels lazily, and loading may need a context synchronisation;
-  // with the persistent relay kernel running that would deadlock the first launch of
-  // any other engine kernel.  Force every kernel of this module to load up front.
+namespace {
+template <uint32_t D>
+cudaError_t preload_staged() {
   cudaFuncAttributes a;
-  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(recv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(relay_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(direct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
+  const int smem = static_cast<int>(staged_smem<D>());
+  cudaError_t e = cudaFuncSetAttribute(xfer_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(send_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(recv_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(relay_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(direct_leg_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_leg_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel);
+    e = cudaFuncSetAttribute(direct_leg_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, xfer_kernel<D>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel<D>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel<D>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, relay_kernel<D>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_leg_kernel<D>);
+  return e;
+}
+
+template <uint32_t D>
+cudaError_t occupancy(int *n) {
+  const int smem = static_cast<int>(staged_smem<D>());
+  cudaError_t e = cudaFuncSetAttribute(xfer_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(n, xfer_kernel<D>, kThreads, smem);
+}
+}  // namespace
+
+int preload_kernels() {
+  // CUDA 12 loads kernels lazily, and a first load may wait for the device to idle;
+  // load every kernel of this module up front (the relay service thread launches
+  // relay kernels while the user's streams are busy).
+  cudaFuncAttributes a;
+  cudaError_t e = preload_staged<kBulkStages>();
+  if (e == cudaSuccess) e = preload_staged<kDeepStages>();
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(direct_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kBulkSmem);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_reg_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, direct_small_kernel);
@@ -1591,27 +1643,27 @@ int preload_kernels() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<float>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<double>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_add_kernel<__nv_bfloat16>);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, send_gate_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, recv_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, relay_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, pingpong_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, spin_kernel);
   return static_cast<int>(e);
 }
 
-int xfer_capacity(int device, int *per_sm, int *sms) {
-  int n = 0;
-  cudaError_t e = cudaFuncSetAttribute(xfer_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kXferSmem);
-  if (e != cudaSuccess) return static_cast<int>(e);
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xfer_kernel, kThreads, kXferSmem);
+int xfer_capacity(int device, int *per_sm, int *per_sm_deep, int *sms) {
+  int n = 0, nd = 0;
+  cudaError_t e = occupancy<kBulkStages>(&n);
+  if (e == cudaSuccess) e = occupancy<kDeepStages>(&nd);
   if (e != cudaSuccess) return static_cast<int>(e);
   int s = 0;
   e = cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, device);
   if (e != cudaSuccess) return static_cast<int>(e);
   *per_sm = n;
+  *per_sm_deep = nd;
   *sms = s;
   return cudaSuccess;
 }
+
+uint32_t deep_stages() { return kDeepStages; }
+uint32_t shallow_stages() { return kBulkStages; }
 
 }  // namespace mpx

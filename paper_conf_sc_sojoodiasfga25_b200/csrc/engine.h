@@ -76,7 +76,7 @@ struct XferParams {
   uint32_t pdl;          // 1: launched with programmatic stream serialization (PDL)
   uint32_t staged_blk;   // 1: a direct-only copy timing a loopback staged leg (Step 1):
                          //    moved with the staged legs' TMA block size
-  uint32_t pad_;
+  uint32_t stages;       // staged pipeline depth: shallow_stages() or deep_stages()
   uint64_t timeout_ns;
   int32_t *err;          // device (or mapped host) error word
   DevPath p[kMaxPaths];
@@ -192,6 +192,7 @@ struct HostRingPtrs {
 
 struct SendParams {
   uint32_t me, dst, nblocks, g_direct, npaths, copy_mode, bulk_stages, g_host;
+  uint32_t stages, pad_;     // staged pipeline depth (shallow_stages() / deep_stages())
   uint64_t seq, bytes, tag, timeout_ns, align;
   const uint8_t *src;
   uint8_t *my_ctrl;
@@ -220,6 +221,7 @@ struct SendParams {
 
 struct RecvParams {
   uint32_t me, src, nblocks, g_host, copy_mode, bulk_stages;
+  uint32_t stages, pad_;     // staged pipeline depth
   uint64_t seq, bytes, tag, region, region_off, done_target, timeout_ns;
   uint8_t *my_ctrl;
   uint8_t *buf;              // the receive buffer (host-ring consumers write here)
@@ -236,7 +238,8 @@ struct RecvParams {
 // (grid = g CTAs, CTA r = lane r).
 struct RelayParams {
   uint32_t me, sender, g, copy_mode;
-  uint32_t aligned, pad_;      // 1: source and target co-aligned (streamed lanes)
+  uint32_t aligned;            // 1: source and target co-aligned (streamed lanes)
+  uint32_t stages;             // staged pipeline depth
   uint64_t q0, k, timeout_ns;
   uint8_t *my_ctrl;
   uint8_t *sender_ctrl;        // the sender's control block (mapped): relay_free flags
@@ -276,8 +279,13 @@ int launch_pingpong(uint64_t *flags, int iters, uint64_t timeout_ns, int32_t *er
 // A one-warp kernel that holds `stream` for `ns` nanoseconds (Step 1 of C27).
 int launch_spin(uint64_t ns, void *stream);
 
-// Max co-resident CTAs of the transfer kernel on this device (occupancy × SMs).
-int xfer_capacity(int device, int *per_sm, int *sms);
+// Co-resident CTAs per SM of the kernels with staged CTAs at 4 stages (per_sm) and at
+// the deep 6 (per_sm_deep), and the SM count.
+int xfer_capacity(int device, int *per_sm, int *per_sm_deep, int *sms);
+// The two staged-pipeline depths (engine.cu): `stages` of XferParams / SendParams /
+// RecvParams / RelayParams must be one of them.
+uint32_t deep_stages();
+uint32_t shallow_stages();
 
 // Load every engine kernel now (no lazy loading once persistent kernels run).
 int preload_kernels();

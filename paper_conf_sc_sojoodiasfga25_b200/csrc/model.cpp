@@ -288,12 +288,11 @@ uint32_t k_exact(const PathModel &p, double x, uint64_t b, const ModelOpts &o) {
       cand[nc++] = static_cast<uint32_t>(c);
     }
   }
-  std::sort(cand, cand + nc);
   uint32_t best = cand[0];
   double tb = staged_time(p, x, best, M_B200);
   for (int i = 1; i < nc; ++i) {
     const double t = staged_time(p, x, cand[i], M_B200);
-    if (t < tb) {
+    if (t < tb || (t == tb && cand[i] < best)) {  // ties to the smaller k
       tb = t;
       best = cand[i];
     }

@@ -291,6 +291,7 @@ void relay_loop(mp_ctx *c, RelayService *S) {
   base.me = static_cast<uint32_t>(c->rank);
   base.copy_mode = c->copy_mode;
   base.timeout_ns = static_cast<uint64_t>(c->timeout_s * 1e9);
+  base.stages = stages_for(c, static_cast<uint32_t>(c->relay_ctas));
   base.my_ctrl = c->ctrl;
   for (int r = 0; r < c->world; ++r) base.peer[r] = c->peers[r];
   base.L = c->L;
@@ -477,10 +478,11 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   // slots; the receiver's host consumers and Step 1's leg timing use the same count).
   const uint32_t g_stage = static_cast<uint32_t>(c->relay_ctas);
   P.g_host = g_stage;
-  const int cap = std::max(1, c->per_sm * c->sms);
   uint32_t staged = 0;
   for (int i = 1; i < cfg.npaths; ++i)
     if (cfg.bytes[i]) staged += g_stage;
+  P.stages = stages_for(c, staged);
+  const int cap = std::max(1, per_sm_at(c, P.stages) * c->sms);
   P.g_direct = direct_ctas(c, cfg.bytes[0], cap - static_cast<int>(staged));
   if (staged && P.g_direct > static_cast<uint32_t>(c->sms))  // whole CTAs per SM beside staged groups
     P.g_direct = P.g_direct / static_cast<uint32_t>(c->sms) * static_cast<uint32_t>(c->sms);
@@ -575,6 +577,7 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   P.host_stride = c->host_stride;
   P.host_slots = static_cast<uint32_t>(c->slots);
   P.g_host = c->host_path ? static_cast<uint32_t>(c->relay_ctas) : 0u;
+  P.stages = stages_for(c, P.g_host);
   P.copy_mode = c->copy_mode;
   P.pdl = c->pdl_world;
   P.bulk_stages = bulk_stages_for(bytes);

@@ -131,7 +131,9 @@ def lib():
     """Load libmpx.so (building it in-tree with nvcc first if it is missing/stale)."""
     global _lib
     if _lib is None:
-        path = _build.build()
+        # MPX_LIB: an alternative in-tree build (design experiments, e.g. a variant
+        # compiled with other MPX_* defines by _build.build(out=..., defines=...))
+        path = os.environ.get("MPX_LIB") or _build.build()
         L = C.CDLL(path, mode=C.RTLD_GLOBAL)
         P = C.c_void_p
         sig = {

