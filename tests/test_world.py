@@ -22,10 +22,12 @@ def free_port():
     return p
 
 
-def run_world(world, scenario, timeout):
+def run_world(world, scenario, timeout, env=None):
     port = free_port()
+    penv = dict(os.environ, **(env or {}))
     procs = [subprocess.Popen([sys.executable, os.path.join(HERE, "_world_worker.py"), str(r), str(world),
-                               str(port), scenario], stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)
+                               str(port), scenario], stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True,
+                              env=penv)
              for r in range(world)]
     outs = []
     try:
@@ -118,3 +120,14 @@ def test_multirank_device_sync_with_relays():
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(3, "devsync", timeout=400)
+
+
+@pytest.mark.gpu
+def test_multirank_engine_shallow_staged_pipelines():
+    # every staged launch at 4 stages (MPX_STAGES=4): the send / recv / relay kernel
+    # instances a sender with many relays gets (the default picks 6 when room allows)
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(3, "engine", timeout=400, env={"MPX_STAGES": "4"})
