@@ -378,7 +378,98 @@ struct LinkMeas {
   double h2a, h2b;        // host → GPU α, β
   double eps_dev, eps_host;
   double kappa;           // host duplex factor of this GPU (reading C25)
+  double egress_b;        // C14 shared port: this GPU writing to every peer at once [B/s]
+  double ingress_b;       // every peer writing into this GPU at once [B/s]
 };
+
+// Reading C14's shared port across GPUs: on NVSwitch every NVLink path of a pair leaves
+// through the source's egress and enters through the destination's ingress, so the
+// port of (s, d) is min(egress(s), ingress(d)) — measured here as aggregates, not as
+// the one-destination direct copy (which would leave no room for a relay even where
+// one peer stream cannot fill the links).  Egress of rank s: s copies n bytes into
+// every peer's heap at once (one stream per peer), rounds serialised over s.  Ingress
+// of rank d: every other rank copies n bytes into d's heap at once after a barrier;
+// the aggregate is (W − 1)·n over the slowest copy.  Medians of `reps` rounds.
+int aggregate_ports(mp_ctx *c, uint64_t n, int reps, double *egress, double *ingress) {
+  const int W = c->world, me = c->rank;
+  *egress = *ingress = 0.0;
+  if (W < 2 || n == 0) return MP_OK;
+  std::vector<cudaStream_t> st(W, nullptr);
+  std::vector<cudaEvent_t> e0(W, nullptr), e1(W, nullptr);
+  void *src = nullptr;
+  int rc = MP_OK;
+  auto ck = [&](cudaError_t e, const char *what) {
+    if (e != cudaSuccess && rc == MP_OK) rc = cfail(c, MP_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+    return e == cudaSuccess;
+  };
+  ck(cudaMalloc(&src, n), "cudaMalloc");
+  for (int r = 0; r < W && rc == MP_OK; ++r) {
+    ck(cudaStreamCreateWithFlags(&st[r], cudaStreamNonBlocking), "stream");
+    ck(cudaEventCreate(&e0[r]), "event");
+    ck(cudaEventCreate(&e1[r]), "event");
+  }
+  if (rc == MP_OK) ck(cudaMemset(src, 0x6b, n), "memset");
+  if (rc == MP_OK) ck(cudaDeviceSynchronize(), "sync");
+  // every rank takes part in every barrier, even after a local failure (no hang)
+  std::vector<double> eg, in;
+  for (int rep = 0; rep < reps; ++rep) {
+    for (int s = 0; s < W; ++s) {  // egress rounds
+      if (int b = world_barrier(c)) return b;
+      double t = 0.0;
+      if (me == s && rc == MP_OK) {
+        for (int r = 0; r < W; ++r)
+          if (r != me) {
+            ck(cudaEventRecord(e0[r], st[r]), "record");
+            if (rc == MP_OK) rc = launch_direct_copy(c, c->peers[r].heap, src, n, st[r]);
+            ck(cudaEventRecord(e1[r], st[r]), "record");
+          }
+        for (int r = 0; r < W; ++r)
+          if (r != me && rc == MP_OK) ck(cudaEventSynchronize(e1[r]), "sync");
+        // first start to last end across the streams
+        float lo = 0, hi = 0;
+        int first = -1;
+        for (int r = 0; r < W && rc == MP_OK; ++r) {
+          if (r == me) continue;
+          if (first < 0) first = r;
+          float a = 0, b = 0;
+          ck(cudaEventElapsedTime(&a, e0[first], e0[r]), "elapsed");
+          ck(cudaEventElapsedTime(&b, e0[first], e1[r]), "elapsed");
+          lo = std::min(lo, a);
+          hi = std::max(hi, b);
+        }
+        t = (hi - lo) * 1e-3;
+        if (t > 0) eg.push_back(static_cast<double>(W - 1) * n / t);
+      }
+    }
+    for (int d = 0; d < W; ++d) {  // ingress rounds
+      if (int b = world_barrier(c)) return b;
+      double t = 0.0;
+      if (me != d && rc == MP_OK) {
+        ck(cudaEventRecord(e0[d], st[d]), "record");
+        if (rc == MP_OK) rc = launch_direct_copy(c, c->peers[d].heap, src, n, st[d]);
+        ck(cudaEventRecord(e1[d], st[d]), "record");
+        ck(cudaEventSynchronize(e1[d]), "sync");
+        float ms = 0;
+        ck(cudaEventElapsedTime(&ms, e0[d], e1[d]), "elapsed");
+        t = ms * 1e-3;
+      }
+      std::vector<double> all(W);
+      if (int b = world_allgather(c, &t, all.data(), sizeof(double))) return b;
+      const double tmax = *std::max_element(all.begin(), all.end());
+      if (me == d && tmax > 0) in.push_back(static_cast<double>(W - 1) * n / tmax);
+    }
+  }
+  if (src) cudaFree(src);
+  for (int r = 0; r < W; ++r) {
+    if (st[r]) cudaStreamDestroy(st[r]);
+    if (e0[r]) cudaEventDestroy(e0[r]);
+    if (e1[r]) cudaEventDestroy(e1[r]);
+  }
+  if (rc) return rc;
+  *egress = eg.empty() ? 0.0 : median(eg);
+  *ingress = in.empty() ? 0.0 : median(in);
+  return MP_OK;
+}
 
 // edges = {0}: the plain Step-1 fit (flushed single copies); more edges: one
 // parameter set per size band (reading C20), window-timed (reading C21).
@@ -483,6 +574,15 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
   if (st) return st;
   for (int32_t v : all_ok)
     if (v) return cfail(c, MP_ERR_STATE, "calibration failed on another rank");
+  {  // C14's shared port as aggregates (egress, ingress); heaps are still empty
+    double eg = 0.0, in = 0.0;
+    const uint64_t n_each = std::min<uint64_t>(cap, 256ull << 20);
+    if (int e = aggregate_ports(c, n_each, std::max(3, reps / 2), &eg, &in)) return e;
+    for (int j = 0; j < B; ++j) {
+      m[j].egress_b = eg;
+      m[j].ingress_b = in;
+    }
+  }
   std::vector<LinkMeas> lm(static_cast<size_t>(W) * B);  // [rank][band]
   if (int s = world_allgather(c, m.data(), lm.data(), sizeof(LinkMeas) * B)) return s;
 
@@ -514,7 +614,11 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
         }
         if (keep_c && nold == np)
           for (int i = 0; i < np; ++i) prm[i].c = old[i].c;
-        mp_port_params port{S.da, S.db};
+        // the port of (s, d): min(egress(s), ingress(d)) (C14); the direct copy's β when
+        // an aggregate is missing or lower (the port is never below one stream)
+        double pb = S.db;
+        if (S.egress_b > 0 && D.ingress_b > 0) pb = std::max(S.db, std::min(S.egress_b, D.ingress_b));
+        mp_port_params port{S.da, pb};
         const int e = j == 0 ? mp_set_model(c, s, d, paths, prm, np, &port)
                              : mp_set_model_band(c, s, d, static_cast<uint64_t>(edges[j]), prm, np, &port);
         if (e) return e;
