@@ -985,13 +985,14 @@ struct RelayConsumer {
   const RelayParams *P;
   uint32_t r;
   uint64_t lstride;
+  uint64_t q0;  // the message's first ring sequence
   __device__ uint8_t *lane(uint32_t j) const {
-    const uint64_t s = (P->q0 + j) % P->L.slots;
+    const uint64_t s = (q0 + j) % P->L.slots;
     return P->my_ctrl + P->L.ring_data + (static_cast<uint64_t>(P->sender) * P->L.slots + s) * P->L.stride +
            r * lstride;
   }
   __device__ int wait(uint32_t j) {
-    const uint64_t q = P->q0 + j;
+    const uint64_t q = q0 + j;
     return poll_flag(flags_at(P->my_ctrl, P->L.ring_full, P->sender, P->L.slots, q % P->L.slots) + r,
                      q / P->L.slots + 1, P->timeout_ns, P->err);
   }
@@ -1010,7 +1011,7 @@ struct RelayConsumer {
   }
   __device__ void before_store(uint32_t) {}
   __device__ void loaded(uint32_t j) {
-    const uint64_t q = P->q0 + j;
+    const uint64_t q = q0 + j;
     st_release_sys(flags_at(P->sender_ctrl, P->L.relay_free, P->me, P->L.slots, q % P->L.slots) + r,
                    q / P->L.slots + 1);
   }
@@ -1286,27 +1287,27 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kerne
   }
 }
 
-// Relay (A8 step 3), one bounded launch per relayed message: CTA r forwards lane r of
-// chunks [q0, q0 + k) of the sender's ring to the destination its lane header names,
-// counts the bytes into the destination's `done` and returns the lane to the sender.
+// Relay (A8 step 3): CTA r forwards lane r of chunks [q0, q0 + k) of the sender's ring
+// to the destination its lane header names, counts the bytes into the destination's
+// `done` and returns the lane to the sender — for the launch's first message, then
+// (lingering) for each next message of the sender whose doorbell CTA 0 sees within
+// linger_ns, so back-to-back relayed messages pay no relaunch.  A relay kernel still
+// ends once its sender goes quiet: nothing outlives the traffic by more than the linger.
 template <uint32_t D>
-__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kernel(const __grid_constant__ RelayParams P) {
-  extern __shared__ __align__(128) uint8_t dyn_smem[];
-  __shared__ int s_abort;
-  __shared__ uint64_t s_h[5];
-  if (threadIdx.x == 0) s_abort = 0;
-  __syncthreads();
+__device__ bool relay_message(const RelayParams &P, uint64_t q0, uint64_t k, uint32_t aligned, int *s_abort,
+                              uint8_t *smem) {
   const uint32_t r = blockIdx.x;
   const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g);
-  if (P.copy_mode == 1 && P.aligned) {  // streamed lane (the sender found source and target co-aligned)
-    RelayConsumer R{&P, r, lstride};
-    lane_stream<LD_RING, D>(R, static_cast<uint32_t>(P.k), dyn_smem);
-    return;
+  if (P.copy_mode == 1 && aligned) {  // streamed lane (the sender found source and target co-aligned)
+    RelayConsumer R{&P, r, lstride, q0};
+    lane_stream<LD_RING, D>(R, static_cast<uint32_t>(k), smem);
+    return *reinterpret_cast<volatile int32_t *>(P.err) == 0;
   }
-  for (uint64_t j = 0; j < P.k; ++j) {
-    const uint64_t q = P.q0 + j, s = q % P.L.slots, u = q / P.L.slots;
+  __shared__ uint64_t s_h[5];
+  for (uint64_t j = 0; j < k; ++j) {
+    const uint64_t q = q0 + j, s = q % P.L.slots, u = q / P.L.slots;
     uint64_t *fl = flags_at(P.my_ctrl, P.L.ring_full, P.sender, P.L.slots, s) + r;
-    if (!wait_flags(fl, 1, u + 1, P.timeout_ns, P.err, &s_abort)) return;
+    if (!wait_flags(fl, 1, u + 1, P.timeout_ns, P.err, s_abort)) return false;
     uint8_t *lane =
         P.my_ctrl + P.L.ring_data + (static_cast<uint64_t>(P.sender) * P.L.slots + s) * P.L.stride + r * lstride;
     if (threadIdx.x < 5) s_h[threadIdx.x] = ld_volatile(reinterpret_cast<const uint64_t *>(lane) + threadIdx.x);
@@ -1315,12 +1316,88 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kern
     const uint64_t off = s_h[1], len = s_h[2], shift = s_h[3], region = s_h[4];
     if (dst >= P.L.world || region >= kMaxRegions) {  // a torn or foreign lane: never write through it
       if (threadIdx.x == 0) atomicExch(P.err, DERR_MISMATCH);
-      return;
+      return false;
     }
     copy_slice<LD_RING, kStagedBlock>(region_base(P.my_ctrl, P.L, region, dst) + off, lane + kLaneHdr + shift, len,
-                                      dyn_smem, P.copy_mode, kBulkStages);
+                                      smem, P.copy_mode, kBulkStages);
     uint64_t *fr = flags_at(P.sender_ctrl, P.L.relay_free, P.me, P.L.slots, s) + r;
     publish(done_at(P.peer[dst].ctrl, P.L, P.sender), len, fr, u + 1);
+    __syncthreads();
+  }
+  return true;
+}
+
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kernel(const __grid_constant__ RelayParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
+  __shared__ int s_abort;
+  __shared__ uint64_t s_next[4];  // next message: tag, q0, k, flags (bit 0 aligned, bit 1 stop)
+  if (threadIdx.x == 0) s_abort = 0;
+  __syncthreads();
+  uint64_t m = P.m0, q0 = P.q0, k = P.k;
+  uint32_t aligned = P.aligned;
+  for (;;) {
+    if (!relay_message<D>(P, q0, k, aligned, &s_abort, dyn_smem)) break;
+    // the sender's next message: CTA 0 looks for its doorbell for up to linger_ns and
+    // publishes the decision; every CTA follows it
+    uint64_t *dec = P.dec + ((m + 1) % kBellRing) * 4;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      const BellEntry *e = P.bells + (m + 1) % kBellRing;
+      const uint64_t t0 = globaltimer();
+      bool found = false;
+      while (P.linger_ns && globaltimer() - t0 < P.linger_ns) {
+        if (ld_relaxed_sys(&e->tag) == m + 2) {
+          found = ld_acquire_sys(&e->tag) == m + 2;
+          break;
+        }
+        __nanosleep(256);
+      }
+      uint64_t nq = 0, nk = 0, flags = 2;  // stop
+      if (found) {
+        const uint64_t g = ld_volatile(&e->g);
+        if (static_cast<uint32_t>(g & 0xffffffffu) == P.g) {  // same lanes: this launch serves it
+          nq = ld_volatile(&e->q0);
+          nk = ld_volatile(&e->k);
+          flags = (g >> 32) & 1u;
+        }
+      }
+      dec[1] = nq;
+      dec[2] = nk;
+      dec[3] = flags;
+      st_release_sys(dec, m + 2);
+    }
+    if (threadIdx.x == 0) {
+      const uint64_t t0 = globaltimer();
+      while (ld_acquire_sys(dec) != m + 2) {
+        if (globaltimer() - t0 > P.linger_ns + P.timeout_ns) {
+          atomicExch(P.err, DERR_TIMEOUT);
+          s_abort = 1;
+          break;
+        }
+        __nanosleep(128);
+      }
+      s_next[1] = ld_volatile(dec + 1);
+      s_next[2] = ld_volatile(dec + 2);
+      s_next[3] = ld_volatile(dec + 3);
+    }
+    __syncthreads();
+    if (s_abort || (s_next[3] & 2u)) break;
+    m += 1;
+    q0 = s_next[1];
+    k = s_next[2];
+    aligned = static_cast<uint32_t>(s_next[3] & 1u);
+    __syncthreads();
+  }
+  // the last CTA out hands the sender's doorbell position back to the host thread
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence_system();
+    if (atomicAdd(P.exit_cnt, 1u) == P.g - 1) {
+      atomicExch(P.exit_cnt, 0u);
+      volatile uint64_t *st = P.state;
+      st[0] = m + 1;                     // first message this launch did not serve
+      st_release_sys(P.state + 1, 0);    // alive = 0
+    }
   }
 }
 

@@ -180,6 +180,8 @@ struct CtrlLayout {
   uint64_t eager = 0;                  // [world(sender)][kEagerSlots][kEagerStride]   — on the receiver
   uint64_t eager_free = 0;             // [world(receiver)] u64, 128-B padded: slots returned — on the sender
   uint64_t eager_cnt = 0;              // [world(sender)][kEagerSlots] u32: CTAs done copying out — on the receiver
+  uint64_t relay_dec = 0;              // [world(sender)][kBellRing][4] u64: a relay kernel's next-message decisions
+  uint64_t relay_exit = 0;             // [world(sender)] u32, 128-B padded: relay CTAs that have left
   uint64_t total = 0;
 };
 
@@ -234,13 +236,21 @@ struct RecvParams {
   HostRingPtrs host;
 };
 
-// One bounded relay launch: forward chunks [q0, q0 + k) of `sender`'s ring, g lanes
-// (grid = g CTAs, CTA r = lane r).
+// One relay launch: forward chunks [q0, q0 + k) of `sender`'s ring (its doorbell
+// message m0), g lanes (grid = g CTAs, CTA r = lane r); then, while the sender's next
+// doorbell arrives within linger_ns with the same g, its message too, and so on; the
+// last CTA out records the first message it did not serve and clears `alive`.
 struct RelayParams {
   uint32_t me, sender, g, copy_mode;
   uint32_t aligned;            // 1: source and target co-aligned (streamed lanes)
   uint32_t stages;             // staged pipeline depth
   uint64_t q0, k, timeout_ns;
+  uint64_t m0;                 // doorbell index of the first message
+  uint64_t linger_ns;          // how long CTA 0 waits for the next doorbell (0: one message)
+  const BellEntry *bells;      // the sender's doorbell row in this rank's segment (mapped host)
+  uint64_t *dec;               // [kBellRing][4] device words: CTA 0's next-message decisions
+  uint32_t *exit_cnt;          // device word: CTAs that have left
+  uint64_t *state;             // mapped host [2]: first unserved message, alive (host sets 1)
   uint8_t *my_ctrl;
   uint8_t *sender_ctrl;        // the sender's control block (mapped): relay_free flags
   PeerPtrs peer[kMaxPaths];    // ctrl of every rank (self: local): destinations' done counters

@@ -94,6 +94,8 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.eager = take(static_cast<uint64_t>(world) * kEagerSlots * kEagerStride);
   L.eager_free = take(static_cast<uint64_t>(world) * 128);
   L.eager_cnt = take(static_cast<uint64_t>(world) * kEagerSlots * 4);
+  L.relay_dec = take(static_cast<uint64_t>(world) * kBellRing * 32);
+  L.relay_exit = take(static_cast<uint64_t>(world) * 128);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
@@ -267,20 +269,26 @@ int world_init(mp_ctx *c) {
 // The relay rank's side of a GPU-staged path.  A sender's gate kernel rings a doorbell
 // in this rank's shared pinned segment (BellEntry: ring sequence q0, chunk count k,
 // lanes g) once the message's clear-to-send has arrived; this thread sees it and
-// launches one relay kernel of g CTAs for those chunks on the sender's stream (stream
-// order keeps a sender's ring positions in order).  Every relay kernel ends when its
-// chunks are forwarded, so nothing runs on this GPU without traffic to serve, and a
-// device-wide synchronisation (torch.cuda.synchronize, cudaDeviceSynchronize, lazy
-// module loading) completes on every rank.  The thread spins while traffic is recent
-// and polls every ~20 µs after 50 ms of quiet.
+// launches a relay kernel of g CTAs for those chunks on the sender's stream (stream
+// order keeps a sender's ring positions in order).  The kernel also serves the
+// sender's following messages whose doorbells arrive within the linger (200 µs;
+// MPX_RELAY_LINGER_US), so back-to-back relayed messages pay no relaunch; its last
+// CTA then records the first doorbell it left and clears `alive`, and this thread
+// takes over from there.  Every relay kernel ends at most a linger after its sender's
+// traffic, so nothing runs on this GPU without traffic to serve, and a device-wide
+// synchronisation (torch.cuda.synchronize, cudaDeviceSynchronize, lazy module
+// loading) completes on every rank.  The thread spins while traffic is recent and
+// polls every ~20 µs after 50 ms of quiet.
 struct RelayService {
   std::thread th;
   std::atomic<bool> stop{false};
   std::atomic<int> error{0};           // cudaError_t of a failed relay launch (sticky)
   std::atomic<uint64_t> launches{0};
   std::vector<cudaStream_t> streams;   // [world(sender)]
-  std::vector<uint64_t> next;          // [world(sender)] next doorbell index
   BellEntry *bells = nullptr;          // this rank's doorbells [world(sender)][kBellRing]
+  uint64_t *state = nullptr;           // mapped host [world(sender)][2]: first unserved
+                                       // doorbell, a relay kernel alive (host sets, kernel clears)
+  uint64_t linger_ns = 200000;         // a relay kernel waits this long for the next doorbell
 };
 
 namespace {
@@ -296,31 +304,45 @@ void relay_loop(mp_ctx *c, RelayService *S) {
   for (int r = 0; r < c->world; ++r) base.peer[r] = c->peers[r];
   base.L = c->L;
   base.err = c->d_err;
+  base.linger_ns = S->linger_ns;
   auto last = std::chrono::steady_clock::now();
   while (!S->stop.load(std::memory_order_acquire)) {
     bool any = false;
     for (int s = 0; s < c->world; ++s) {
       if (s == c->rank) continue;
-      for (;;) {
-        BellEntry *e = S->bells + static_cast<uint64_t>(s) * kBellRing + S->next[s] % kBellRing;
-        if (__atomic_load_n(&e->tag, __ATOMIC_ACQUIRE) != S->next[s] + 1) break;
-        RelayParams P = base;
-        P.sender = static_cast<uint32_t>(s);
-        P.sender_ctrl = c->peers[s].ctrl;
-        P.q0 = __atomic_load_n(&e->q0, __ATOMIC_RELAXED);
-        P.k = __atomic_load_n(&e->k, __ATOMIC_RELAXED);
-        const uint64_t g = __atomic_load_n(&e->g, __ATOMIC_RELAXED);
-        P.g = static_cast<uint32_t>(g & 0xffffffffu);
-        P.aligned = static_cast<uint32_t>((g >> 32) & 1u);
-        if (P.g < 1 || P.g > static_cast<uint32_t>(kFlagStride)) {
-          S->error.store(static_cast<int>(cudaErrorInvalidValue));
-        } else if (int rc = launch_relay(P, S->streams[s])) {
-          S->error.store(rc);
-        }
-        S->launches.fetch_add(1, std::memory_order_relaxed);
-        S->next[s] += 1;
+      uint64_t *st = S->state + 2 * static_cast<uint64_t>(s);
+      if (__atomic_load_n(st + 1, __ATOMIC_ACQUIRE)) {  // a lingering relay kernel serves this sender
         any = true;
+        continue;
       }
+      const uint64_t n = __atomic_load_n(st, __ATOMIC_RELAXED);
+      const BellEntry *e = S->bells + static_cast<uint64_t>(s) * kBellRing + n % kBellRing;
+      if (__atomic_load_n(&e->tag, __ATOMIC_ACQUIRE) != n + 1) continue;
+      RelayParams P = base;
+      P.sender = static_cast<uint32_t>(s);
+      P.sender_ctrl = c->peers[s].ctrl;
+      P.m0 = n;
+      P.q0 = __atomic_load_n(&e->q0, __ATOMIC_RELAXED);
+      P.k = __atomic_load_n(&e->k, __ATOMIC_RELAXED);
+      const uint64_t g = __atomic_load_n(&e->g, __ATOMIC_RELAXED);
+      P.g = static_cast<uint32_t>(g & 0xffffffffu);
+      P.aligned = static_cast<uint32_t>((g >> 32) & 1u);
+      P.bells = S->bells + static_cast<uint64_t>(s) * kBellRing;
+      P.dec = reinterpret_cast<uint64_t *>(c->ctrl + c->L.relay_dec) + static_cast<uint64_t>(s) * kBellRing * 4;
+      P.exit_cnt = reinterpret_cast<uint32_t *>(c->ctrl + c->L.relay_exit + static_cast<uint64_t>(s) * 128);
+      P.state = st;
+      if (P.g < 1 || P.g > static_cast<uint32_t>(kFlagStride)) {
+        S->error.store(static_cast<int>(cudaErrorInvalidValue));
+        __atomic_store_n(st, n + 1, __ATOMIC_RELAXED);  // skip the malformed doorbell
+        continue;
+      }
+      __atomic_store_n(st + 1, 1, __ATOMIC_RELEASE);
+      if (int rc = launch_relay(P, S->streams[s])) {
+        S->error.store(rc);
+        __atomic_store_n(st + 1, 0, __ATOMIC_RELEASE);
+      }
+      S->launches.fetch_add(1, std::memory_order_relaxed);
+      any = true;
     }
     const auto now = std::chrono::steady_clock::now();
     if (any) {
@@ -338,8 +360,18 @@ int world_start_relay(mp_ctx *c) {
   if (c->world < 3 || c->relay_svc || (no_relay && no_relay[0] == '1')) return MP_OK;
   RelayService *S = new RelayService();
   S->streams.assign(c->world, nullptr);
-  S->next.assign(c->world, 0);
   S->bells = reinterpret_cast<BellEntry *>(c->hseg[c->rank]);
+  if (const char *l = std::getenv("MPX_RELAY_LINGER_US")) S->linger_ns = static_cast<uint64_t>(std::atof(l) * 1e3);
+  {
+    void *p = nullptr;
+    cudaError_t e = cudaHostAlloc(&p, 16ull * c->world, cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e != cudaSuccess) {
+      delete S;
+      return wfail(c, MP_ERR_CUDA, std::string("relay state: ") + cudaGetErrorString(e));
+    }
+    std::memset(p, 0, 16ull * c->world);
+    S->state = static_cast<uint64_t *>(p);
+  }
   for (int r = 0; r < c->world; ++r) {
     if (r == c->rank) continue;
     cudaError_t e = cudaStreamCreateWithFlags(&S->streams[r], cudaStreamNonBlocking);
@@ -367,6 +399,7 @@ int world_stop_relay(mp_ctx *c) {
       cudaStreamSynchronize(st);
       cudaStreamDestroy(st);
     }
+  if (S->state) cudaFreeHost(S->state);
   c->relay_launches_done += S->launches.load();
   c->relay_svc = nullptr;
   delete S;

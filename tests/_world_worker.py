@@ -495,7 +495,7 @@ def scenario_devsync(rank, world):
         c.sync()
         dist.barrier()
     if rank >= 2:
-        assert c.launches() >= 4, c.launches()   # one relay kernel per relayed message
+        assert c.launches() >= 1, c.launches()   # relay kernels ran (one serves a burst of messages)
     c.close()
 
 
