@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round-2 GPU session: tests, bench (both arms), ncu launch list + full captures of the
-# top kernels, multi-rank harness under MPS, per-rank NVLink ncu pass (N = 2, one GPU,
-# time-sliced: checks the wrapper, counters are 0 without NVLink traffic), loopback sweep.
+# top kernels, multi-rank harness under MPS, per-rank NVLink ncu pass (only on a box
+# with >= 2 GPUs), loopback sweep.
 # Usage (under gpurun): bash scripts/r02_profile.sh <tag>
 TAG=${1:-r02/prof}
 OUT=gpurun_out/$TAG
@@ -19,9 +19,13 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"dir
 RELAY_K=32 timeout 600 ncu --set full --clock-control none --import-source on -k regex:xfer_kernel -s 2 -c 1 \
   -o $OUT/relay_full python scripts/relay_one.py > $OUT/ncu_relay.log 2>&1
 STEPS=20 TMO=600 bash scripts/r02_world.sh $TAG/world
-NCU_OUT=$OUT/ncu_world MPX_BENCH_SAME_GPU=1 timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 \
-  --master-addr 127.0.0.1 --master-port 29650 --no-python scripts/ncu_rank.sh bench.py --gpus 2 --steps 5 --warmup 3 \
-  --size 268435456 > $OUT/ncu_world_bench.jsonl 2> $OUT/ncu_world_bench.err; echo "ncu_world rc=$?" >> $OUT/ncu_world_bench.err
+NG=$(nvidia-smi -L | wc -l)
+if [ "$NG" -ge 2 ]; then  # per-rank NVLink counters need one GPU per rank (ncu serialises a shared device)
+  NCU_OUT=$OUT/ncu_world timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node $NG \
+    --master-addr 127.0.0.1 --master-port 29650 --no-python scripts/ncu_rank.sh bench.py --gpus $NG --steps 5 \
+    --warmup 3 > $OUT/ncu_world_bench.jsonl 2> $OUT/ncu_world_bench.err; echo "ncu_world rc=$?" >> $OUT/ncu_world_bench.err
+  python scripts/nvlink_summary.py $OUT/ncu_world $NG 1073741824 --out profiles/ncu_nvlink.json > $OUT/nvlink_summary.json
+fi
 timeout 900 python scripts/sweep.py --out $OUT/sweep.json > $OUT/sweep.log 2>&1; echo "rc=$?" >> $OUT/sweep.log
 nvidia-smi -q -d CLOCK > $OUT/clocks_after.txt 2>&1
 echo done
