@@ -476,9 +476,10 @@ __device__ __forceinline__ void bytes_copy(uint8_t *d, const uint8_t *s, uint64_
   for (uint64_t i = 0; i < n; ++i) d[i] = ld1<MODE>(s + i);
 }
 
-// Called by every thread of the CTA; threads other than 0, 32, 64 and 96 return at once.
+// The four roles; a thread returns from here when its role is done (threads other than
+// 0, 32, 64 and 96 at once).
 template <int MODE, uint32_t D, class Role>
-__device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
+__device__ void lane_stream_roles(Role &R, uint32_t nchunks, uint8_t *smem) {
   __shared__ uint32_t s_ready;    // chunks the watcher has found ready
   __shared__ uint32_t s_taken;    // chunks taken up (consumer: loader read the words; producer: storer)
   __shared__ uint32_t s_loaded;   // chunks whose loads have all landed (storer → publisher)
@@ -696,6 +697,20 @@ __device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
     st_release_cta_shared(&s_stop, 1);  // the watcher, loader and publisher stop too
     bulk_wait_all();
   }
+}
+
+// Called by every thread of the CTA: the roles, then every thread meets again and the
+// stage barriers are invalidated, so the next call (a relay kernel streams one message
+// after another) initialises fresh ones.
+template <int MODE, uint32_t D, class Role>
+__device__ void lane_stream(Role &R, uint32_t nchunks, uint8_t *smem) {
+  lane_stream_roles<MODE, D>(R, nchunks, smem);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t bars = smem_u32(smem + static_cast<uint64_t>(kStagedBlock) * D);
+    for (uint32_t i = 0; i < 2 * D; ++i) asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(bars + 8 * i) : "memory");
+  }
+  __syncthreads();
 }
 
 // ------------------------------------------------------------------ roles
