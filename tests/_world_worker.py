@@ -526,6 +526,65 @@ def scenario_bench_plan(rank, world):
     c.close()
 
 
+def scenario_relay_burst(rank, world):
+    """Doorbell and lingering-relay bookkeeping under load: 160 relayed messages rank 0
+    → rank 1 through relay rank 2 (2.5 doorbell rings of 64), windows of 8 in flight,
+    alternating co-aligned and misaligned sources (a lingering relay kernel switches
+    between its streamed and per-chunk paths message by message), with pauses longer
+    than the linger between some windows (the host thread relaunches).  Every message
+    bit-exact against the oracle replay."""
+    import time
+
+    import numpy as np
+
+    import synth
+    from oracle import transfer as X
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+                                timeout_s=60.0, calibrate=False)
+    ps = c.paths(0, 1)
+    n = 1 * MiB + 4099
+    W = 8
+    src_buf = torch.empty(W * (n + 64), dtype=torch.uint8, device="cuda")
+    bufs = [c.alloc(n) for _ in range(W)] if rank == 1 else []
+    nb = [0] * len(ps)
+    nb[1] = n
+    ks = [1] + [0] * (len(ps) - 1)
+    ks[1] = 3
+    cfg = c.make_config(nb, ks, 0, 1)
+    for win in range(20):
+        payloads = [synth.payload(n, 1000 + win * W + i) for i in range(W)]
+        if rank == 0:
+            views = []
+            for i in range(W):
+                off = i * (n + 64) + (0 if (win + i) % 2 == 0 else 7)  # co-aligned, then misaligned
+                v = src_buf[off:off + n]
+                v.copy_(torch.from_numpy(payloads[i]))
+                views.append(v)
+            torch.cuda.synchronize()
+            for i in range(W):
+                c.send(views[i], n, 1, tag=win * W + i, cfg=cfg, stream=stream)
+            stream.synchronize()
+        elif rank == 1:
+            for i in range(W):
+                c.recv(bufs[i], n, 0, tag=win * W + i, stream=stream)
+            stream.synchronize()
+            for i in range(W):
+                exp = np.zeros(n, dtype=np.uint8)
+                X.replay(payloads[i], nb, ks, [k for k, _ in ps], 256, exp)
+                assert np.array_equal(mp.as_tensor(bufs[i], n).cpu().numpy(), exp), f"window {win} message {i}"
+        if win % 5 == 4:
+            time.sleep(0.002)  # > the 200 µs linger: the relay kernel ends, the host thread relaunches
+        dist.barrier()
+    c.sync()
+    for b in bufs:
+        c.free(b)
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
@@ -536,7 +595,7 @@ def main():
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
          "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
          "eager": scenario_eager, "devsync": scenario_devsync,
-         "bench_plan": scenario_bench_plan}[scen](rank, world)
+         "bench_plan": scenario_bench_plan, "relay_burst": scenario_relay_burst}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

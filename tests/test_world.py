@@ -131,3 +131,14 @@ def test_multirank_engine_shallow_staged_pipelines():
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(3, "engine", timeout=400, env={"MPX_STAGES": "4"})
+
+
+@pytest.mark.gpu
+def test_multirank_relay_burst_doorbell_wrap_and_linger():
+    # 160 relayed messages: doorbell / decision rings wrap, lingering relay kernels
+    # switch between streamed and per-chunk lanes, relaunch after quiet periods
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(3, "relay_burst", timeout=400)
