@@ -585,6 +585,50 @@ def scenario_relay_burst(rank, world):
     c.close()
 
 
+def scenario_full_size(rank, world):
+    """BASELINE.json config 3 at full size through the multi-rank engine, in bench.py's
+    launch configuration (default slots / lanes / heap, deep staged pipelines): one
+    1 GiB + 4099-byte message rank 0 → rank 1 with the B200-mode pick, then with the
+    paper-mode pick (every path: direct, relays 2.., host) and every path forced at
+    once; payloads compared whole on the device against the source (O1: dst == src)."""
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    n = (1 << 30) + 4099
+    stream = torch.cuda.Stream()
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                        generator=torch.Generator(device="cuda").manual_seed(20251116)) if rank in (0, 1) else None
+    torch.cuda.synchronize()
+    c = mdist.context_from_dist(device=0, heap_bytes=n + 64 * MiB, timeout_s=120.0, calibrate=False)
+    rbuf = c.alloc(n) if rank == 1 else None
+    ps = c.paths(0, 1)
+    cfgs = []
+    for mode in (mp.MP_MODEL_B200, mp.MP_MODEL_PAPER):
+        c.set_options(mode=mode)
+        cfgs.append(c.select(0, 1, n).as_dict())
+    nb = [0] * len(ps)
+    for j in range(1, len(ps)):
+        nb[j] = (64 if ps[j][0] == 1 else 16) * MiB + 256 * j
+    nb[0] = n - sum(nb)
+    cfgs.append({"bytes": nb, "chunks": [1] + [8] * (len(ps) - 1)})
+    for i, d in enumerate(cfgs):
+        if rank == 0:
+            c.send(src, n, 1, tag=i, cfg=c.make_config(d["bytes"], d["chunks"], 0, 1), stream=stream)
+            stream.synchronize()
+        elif rank == 1:
+            view = mp.as_tensor(rbuf, n)
+            view.zero_()
+            torch.cuda.synchronize()
+            c.recv(rbuf, n, 0, tag=i, stream=stream)
+            stream.synchronize()
+            assert torch.equal(view, src), f"config {i}: {d['bytes']}"
+        dist.barrier()
+    c.sync()
+    if rbuf:
+        c.free(rbuf)
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
@@ -595,7 +639,8 @@ def main():
         {"gloo_model": scenario_gloo_model, "engine": scenario_engine,
          "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
          "eager": scenario_eager, "devsync": scenario_devsync,
-         "bench_plan": scenario_bench_plan, "relay_burst": scenario_relay_burst}[scen](rank, world)
+         "bench_plan": scenario_bench_plan, "relay_burst": scenario_relay_burst,
+         "full_size": scenario_full_size}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

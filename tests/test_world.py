@@ -142,3 +142,14 @@ def test_multirank_relay_burst_doorbell_wrap_and_linger():
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(3, "relay_burst", timeout=400)
+
+
+@pytest.mark.gpu
+def test_multirank_config3_full_size_bit_exact():
+    # BASELINE.json config 3 (1 GiB + 4099 B) through the multi-rank engine in the bench's
+    # launch configuration: B200 pick, paper pick, every path at once; world 3 on one GPU
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(3, "full_size", timeout=600)
