@@ -422,11 +422,11 @@ int mp_deregister(mp_ctx *ctx, int id);
 /* ---------------------------------------------------------------- transfer */
 
 /* Eager protocol (reading C23; NEXT f4's low-latency protocol): when
- * world > 1, a message of 1..65536 bytes skips the rendezvous — one kernel per side,
+ * world > 1, a message of 1..1048576 bytes skips the rendezvous — one kernel per side,
  * the payload goes over the direct path into a slot the receiver owns (8 slots per
  * sender), and `cfg`'s split is not used.  Both sides classify by size alone; the
- * environment variable MPX_EAGER=0 (equal on every rank, read at mp_init) turns it
- * off. */
+ * environment variable MPX_EAGER (equal on every rank, read at mp_init) sets the limit
+ * in bytes (0 = off; at most 1 MiB). */
 /* mp_send — Step 5 (the pipeline engine moves "the number of chunks and the
  * size of each chunk per path" the model chose) under MPI point-to-point semantics
  * (OMB's MPI_Isend / MPI_Irecv windows; matching FIFO per pair as in MPI).

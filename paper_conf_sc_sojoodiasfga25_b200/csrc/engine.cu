@@ -1418,8 +1418,8 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kern
 
 
 // Eager protocol (engine.h, reading C23).  Slot = [kEagerHdr header][shift][data]:
-// header words 0/1 = bytes/tag (CTA 0), 16 + r = source shift of CTA r's slice, 8 + r =
-// CTA r's sequence flag (seq + 1, released after its slice).
+// header words 0/1 = bytes/tag (CTA 0), kEagerShift0 + r = source shift of CTA r's
+// slice, kEagerFlag0 + r = CTA r's sequence flag (seq + 1, released after its slice).
 __global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_constant__ EagerParams P) {
   pdl_enter();
   __shared__ int s_abort;
@@ -1440,10 +1440,10 @@ __global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_const
       hdr[0] = P.bytes;
       hdr[1] = P.tag;
     }
-    hdr[16 + r] = shift;
+    hdr[kEagerShift0 + r] = shift;
   }
   __syncthreads();  // the CTA's stores precede thread 0's release (cumulative)
-  if (threadIdx.x == 0) st_release_sys(hdr + 8 + r, P.seq + 1);
+  if (threadIdx.x == 0) st_release_sys(hdr + kEagerFlag0 + r, P.seq + 1);
 }
 
 __global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_constant__ EagerParams P) {
@@ -1455,13 +1455,13 @@ __global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_const
   const uint64_t *hdr = reinterpret_cast<const uint64_t *>(P.slot);
   // every CTA first checks the sender's size and tag (CTA 0's flag): a receive posted
   // larger than the message would otherwise wait for slices that never come
-  if (!wait_word(hdr + 8, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
+  if (!wait_word(hdr + kEagerFlag0, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
   if (ld_volatile(hdr) != P.bytes || ld_volatile(hdr + 1) != P.tag) {
     if (threadIdx.x == 0) atomicExch(P.err, DERR_MISMATCH);
     return;
   }
-  if (r > 0 && !wait_word(hdr + 8 + r, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
-  const uint8_t *data = P.slot + kEagerHdr + ld_volatile(hdr + 16 + r);
+  if (r > 0 && !wait_word(hdr + kEagerFlag0 + r, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
+  const uint8_t *data = P.slot + kEagerHdr + ld_volatile(hdr + kEagerShift0 + r);
   const uint64_t a = static_cast<uint64_t>(r) * kEagerSlice;
   const uint64_t e = a + kEagerSlice < P.bytes ? a + kEagerSlice : P.bytes;
   if (a < e) group_copy<LD_RING>(P.dst + a, data + a, e - a, 0, 1);

@@ -130,11 +130,18 @@ constexpr uint32_t kBellRing = 64;    // outstanding relayed messages per (sende
 // sequence flags, into one of kEagerSlots slots the receiver owns per sender, the
 // receiver copies it out and returns the slot with a counter.  One kernel per side,
 // no clear-to-send round trip.
+// Round 2 raised kEagerMax from 64 KiB to 1 MiB: a rendezvous costs a clear-to-send
+// round trip per message (the receive holds its stream until the message lands), far
+// more than the eager copy-out of ≤ 1 MiB.
 constexpr uint32_t kEagerSlots = 8;
-constexpr uint64_t kEagerMax = 64ull << 10;
-constexpr uint32_t kEagerSlice = 8192;            // bytes per CTA (kEagerMax / 8 CTAs)
-constexpr uint32_t kEagerHdr = 256;               // {bytes, tag, flags[8]} before the data
+constexpr uint64_t kEagerMax = 1ull << 20;
+constexpr uint32_t kEagerSlice = 16384;           // bytes per CTA (≤ 64 CTAs)
+constexpr uint32_t kEagerCtas = kEagerMax / kEagerSlice;
+constexpr uint32_t kEagerFlag0 = 64;              // header word of CTA r's sequence flag: 64 + r
+constexpr uint32_t kEagerShift0 = 128;            // header word of CTA r's source shift: 128 + r
+constexpr uint32_t kEagerHdr = 2048;              // {bytes, tag, …, flags[64], shifts[64]} before the data
 constexpr uint64_t kEagerStride = kEagerHdr + kEagerMax + 256;  // + co-alignment shift
+static_assert(kEagerCtas <= 64, "eager header holds 64 flags and 64 shifts");
 constexpr uint32_t kMaxRegions = 64;  // receive regions: 0 = heap, 1.. = mp_register
 
 struct MsgEntry {                      // CTS and message-header entries (64 B)

@@ -188,8 +188,11 @@ int world_init(mp_ctx *c) {
   me.slot_bytes = c->slot_bytes;
   me.slots = c->slots;
   me.host_path = c->host_path ? 1 : 0;
-  const char *eg = std::getenv("MPX_EAGER");  // "0": every message takes the rendezvous
-  c->eager_max = (eg && eg[0] == '0') ? 0 : kEagerMax;
+  // MPX_EAGER: "0" = every message takes the rendezvous; a byte count = the eager limit
+  // (<= kEagerMax); unset = kEagerMax
+  const char *eg = std::getenv("MPX_EAGER");
+  c->eager_max = kEagerMax;
+  if (eg && eg[0]) c->eager_max = std::min<uint64_t>(kEagerMax, std::strtoull(eg, nullptr, 10));
   me.eager_max = c->eager_max;
   if (int s = topo_local(c, &me.gpu)) return s;
   std::vector<RankInfo> all(W);

@@ -195,13 +195,13 @@ def scenario_faults(rank, world):
     from paper_conf_sc_sojoodiasfga25_b200 import mp
     torch.cuda.set_device(0)
     stream = torch.cuda.Stream()
-    src = torch.empty(MiB, dtype=torch.uint8, device="cuda")
-    src.copy_(torch.from_numpy(synth.payload(MiB, 0)))
+    src = torch.empty(2 * MiB, dtype=torch.uint8, device="cuda")
+    src.copy_(torch.from_numpy(synth.payload(2 * MiB, 0)))
     torch.cuda.synchronize()
     for fault in ("mismatch", "timeout", "eager_mismatch"):
         c = mdist.context_from_dist(device=0, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                     timeout_s=3.0)
-        nb = 4096 if fault == "eager_mismatch" else MiB
+        nb = 4096 if fault == "eager_mismatch" else 2 * MiB   # 2 MiB: past the eager limit (rendezvous)
         if rank == 0 and fault != "timeout":
             c.send(src[:nb], nb, 1, tag=5, stream=stream)
         elif rank == 1:
@@ -308,8 +308,8 @@ def scenario_register(rank, world):
 
 
 def scenario_eager(rank, world):
-    """The eager protocol (reading C23): messages of 1..64 KiB, misaligned sources and
-    destinations, 8-KiB slice edges, the 64 KiB / 64 KiB + 1 boundary to the rendezvous,
+    """The eager protocol (reading C23): messages of 1 B..1 MiB, misaligned sources and
+    destinations, 16-KiB slice edges, the 1 MiB / 1 MiB + 1 boundary to the rendezvous,
     a window of 20 messages (more than the 8 slots: flow control), and eager and
     rendezvous messages interleaved on one pair — every byte checked."""
     import numpy as np
@@ -318,15 +318,15 @@ def scenario_eager(rank, world):
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     torch.cuda.set_device(0)
     stream = torch.cuda.Stream()
-    src_buf = torch.empty(2 * MiB, dtype=torch.uint8, device="cuda")
+    src_buf = torch.empty(3 * MiB, dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=32 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0)
-    sizes = [1, 17, 4095, 8192, 8193, 3 * 8192 + 5, 65535, 65536, 65537, 300000]
+    sizes = [1, 17, 4095, 16384, 16385, 3 * 16384 + 5, 65537, 300000, MiB - 1, MiB, MiB + 1]
     offs = [(0, 0), (1, 1), (3, 7), (16, 5)]
-    cases = [(n, so, do) for n in sizes for so, do in offs[: 1 if n > 65536 else 4]]
+    cases = [(n, so, do) for n in sizes for so, do in offs[: 1 if n > MiB else 4]]
     cases += [(777, 0, 0)] * 20                     # a window beyond the 8 slots
-    cases += [(65536 + 4096, 0, 0), (100, 2, 2), (1 << 20, 0, 0), (5, 0, 0)]   # interleaved protocols
+    cases += [(2 * MiB + 4096, 0, 0), (100, 2, 2), (MiB, 0, 0), (5, 0, 0)]   # interleaved protocols
     if rank == 0:
         for i, (n, so, _) in enumerate(cases):
             host = synth.payload(n, 500 + i)
