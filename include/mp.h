@@ -34,7 +34,8 @@
 extern "C" {
 #endif
 
-#define MP_ABI_VERSION 3  /* 3: topology (mp_get/set_topology), fingerprinted parameter files;
+#define MP_ABI_VERSION 4  /* 4: mp_path_params.wake (reading C28);
+                             3: topology (mp_get/set_topology), fingerprinted parameter files;
                              2: NEXT f2 calls; mp_model_opts.window (was reserved) */
 #define MP_MAX_PATHS 16
 
@@ -86,6 +87,9 @@ typedef struct mp_path_params {
   double c;       /* multiplier of the topology constant φ_i (C4; 1 = Eq 14/15 at θ⁽⁰⁾) */
   double sigma;   /* issue latency counted by the stagger in B200 mode (C8) [s] */
   double w;       /* bytes of shared-port traffic per payload byte (C14) */
+  double wake;    /* B200 mode (C28): earliest start of the second stage after the message
+                     starts [s] — a relay rank's kernel launch through its doorbell thread;
+                     0 = stage 2 ready at once.  T = max(C3's pipeline, wake + k·s2). */
 } mp_path_params;
 
 /* The shared port of B200 mode (C14): T >= alpha + Σ_i w_i b_i / beta.
@@ -362,6 +366,20 @@ int mp_get_host_duplex(mp_ctx *ctx, int gpu, double *kappa);
  * MP_ERR_UNSUPPORTED (world > 1), MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_TIMEOUT. */
 int mp_calibrate_window(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int window, int reps);
 
+/* mp_calibrate_wake — reading C28: measure, per relay rank r, the time A_r
+ * from a message's start to its relay kernel's start when r's relay service is idle
+ * (doorbell → service thread → kernel launch), and install it as `wake` of every
+ * GPU-staged path via r in every pair model and band.  Collective over the world
+ * (world >= 3; a no-op below), after the relay service is up and with no traffic in
+ * flight; mp_init calls it after Step 1 when it calibrates.  Probe: pair (r+1, r+2)
+ * sends two relay-only messages of `bytes` (0 = 2 MiB; raised above the eager limit)
+ * through r after linger + 1 ms of quiet, timed back to back on the receiver;
+ * A_r = T − k·s2 + median(t1 − t2) over `reps` (0 = 7) with T, s2 of the pair's model
+ * (k = 1: s1 + the median), or 0 when that difference is below 1 µs.  MPX_RELAY_WAKE_US (equal on every
+ * rank) installs that value instead of probing.  Returns MP_ERR_STATE without a relay
+ * service, MP_ERR_TOPOLOGY if a pair lacks the path via r. */
+int mp_calibrate_wake(mp_ctx *ctx, uint64_t bytes, int reps);
+
 /* mp_fit_window — the estimator of mp_calibrate_window on given samples (for parity):
  * sample j of path[j] (0 <= path < npaths; path 0 = direct) has T1 = t1[j] (one message
  * on an idle stream), TW = tw[j] (`window` >= 2 back-to-back messages) and the model's
@@ -454,7 +472,9 @@ int mp_xfer(mp_ctx *ctx, void *dst, const void *src, uint64_t bytes, const mp_co
             void *stream);
 
 /* Block until all work this context enqueued has finished, then report any
- * sticky device error (MP_ERR_TIMEOUT / MP_ERR_MISMATCH). */
+ * sticky device error (MP_ERR_TIMEOUT / MP_ERR_MISMATCH).  A device-wide wait
+ * (cudaDeviceSynchronize): it covers every stream the caller passed, including ones
+ * destroyed since, and also waits for other work of this process on the device. */
 int mp_sync(mp_ctx *ctx);
 
 /* ---------------------------------------------------------------- calibration */

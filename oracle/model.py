@@ -49,6 +49,7 @@ class Path:
     sigma: float = 0.0      # issue latency counted by the stagger in B200 mode (C8)
     w: float = 0.0          # bytes of shared-port traffic per payload byte (C14)
     via: int = -1           # relay device (GPU-staged) or -1
+    wake: float = 0.0       # B200 mode (C28): earliest start of stage 2 after the message starts [s]
 
 
 @dataclass
@@ -154,12 +155,14 @@ def pipelined_time(x: float, k: int, p: Path, mode: int = PAPER) -> float:
 
     Per chunk m = x/k (Eq 12); stage 1 s1 = α + m/β, stage 2 s2 = ε + α' + m/β'.
     PAPER mode, Eq 13:  case 1: k·s1 + s2;  case 2: s1 + k·s2.
-    B200 mode (C3): the exact two-stage pipeline, s1 + s2 + (k−1)·max(s1, s2)."""
+    B200 mode (C3): the exact two-stage pipeline, s1 + s2 + (k−1)·max(s1, s2); with a
+    stage-2 availability time A = p.wake (C28: the relay kernel starts A after the
+    message), max(s1 + s2 + (k−1)·max(s1, s2), A + k·s2)."""
     m = x / k
     s1 = p.alpha + m / p.beta
     s2 = p.eps + p.alpha2 + m / p.beta2
     if mode == B200:
-        return s1 + s2 + (k - 1) * max(s1, s2)
+        return max(s1 + s2 + (k - 1) * max(s1, s2), p.wake + k * s2)
     if bottleneck_case(p, PAPER) == 1:
         return k * (p.alpha + m / p.beta) + p.eps + p.alpha2 + m / p.beta2
     return p.alpha + m / p.beta + k * (p.eps + p.alpha2 + m / p.beta2)
@@ -483,7 +486,24 @@ def k_exact(x: float, p: Path, b: int, opts: Options) -> int:
         kc = x * (1.0 / p.beta2 - 1.0 / p.beta) / (p.alpha - e)
         if kc > 0:
             reals.append(kc)
+    A = p.wake
+    if A > 0:
+        # C28: T3 = A + k·e + x/β' (increasing in k) joins the max; the new crossovers:
+        # T3 = T2 at A − α = x/(kβ); T3 = T1 at (e − α)k² + (A − e + x/β' − x/β)k − x/β' = 0
+        if A > p.alpha:
+            reals.append(x / (p.beta * (A - p.alpha)))
+        qa, qb, qc = e - p.alpha, A - e + x / p.beta2 - x / p.beta, -x / p.beta2
+        if qa == 0.0:
+            if qb != 0.0:
+                reals.append(-qc / qb)
+        else:
+            disc = qb * qb - 4.0 * qa * qc
+            if disc >= 0.0:
+                for sgn in (1.0, -1.0):
+                    reals.append((-qb + sgn * math.sqrt(disc)) / (2.0 * qa))
     for r in reals:
+        if not (r > 0.0) or r > 1e12:
+            continue
         for k in (math.floor(r), math.ceil(r)):
             cands.add(min(hi, max(lo, int(k))))
     best = None
@@ -497,10 +517,14 @@ def k_exact(x: float, p: Path, b: int, opts: Options) -> int:
 def piece_exact(x: float, k: int, p: Path):
     """Reading C26: the affine piece (Ω, Δ) of the exact pipeline time at k chunks
     that binds at x bytes — case 1 (Ω = 1/β + 1/(kβ'), Δ = kα + ε + α') when
-    T1 >= T2, else case 2 (Ω = 1/(kβ) + 1/β', Δ = α + k(ε + α'))."""
+    T1 >= T2, else case 2 (Ω = 1/(kβ) + 1/β', Δ = α + k(ε + α')); C28: the
+    availability piece (Ω = 1/β', Δ = A + k(ε + α')) when it is the largest."""
     m = x / k
     s1 = p.alpha + m / p.beta
     s2 = p.eps + p.alpha2 + m / p.beta2
+    t12 = s1 + s2 + (k - 1) * max(s1, s2)
+    if p.wake > 0 and p.wake + k * s2 > t12:
+        return 1.0 / p.beta2, p.wake + k * (p.eps + p.alpha2)
     if s1 >= s2:
         return 1.0 / p.beta + 1.0 / (k * p.beta2), k * p.alpha + p.eps + p.alpha2
     return 1.0 / (k * p.beta) + 1.0 / p.beta2, p.alpha + k * (p.eps + p.alpha2)

@@ -121,14 +121,18 @@ def level_integer_k_b200(n: float, paths: Sequence[M.Path], k_max=256, iters=300
     exact pipeline time (C3): T = max(T1, T2), T1 = kα + ε + α' + x(1/β + 1/(kβ')),
     T2 = α + k(ε + α') + x(1/(kβ) + 1/β').  At level T path i carries
     max_k min((T − c1)/s1, (T − c2)/s2) bytes (or 0), increasing in T; bisect on
-    Σ cap_i = n.  (No issue stagger, no shared port.)"""
+    Σ cap_i = n.  (No issue stagger, no shared port.)  Reading C28: a path with a
+    stage-2 availability time A adds T3 = A + k(ε + α') + x/β' to the max."""
     def pieces(p):
         if p.kind == M.DIRECT:
             return [((1.0 / p.beta, p.alpha),)]
         out = []
         for k in range(1, k_max + 1):
-            out.append(((1.0 / p.beta + 1.0 / (k * p.beta2), k * p.alpha + p.eps + p.alpha2),
-                        (1.0 / (k * p.beta) + 1.0 / p.beta2, p.alpha + k * (p.eps + p.alpha2))))
+            pc = ((1.0 / p.beta + 1.0 / (k * p.beta2), k * p.alpha + p.eps + p.alpha2),
+                  (1.0 / (k * p.beta) + 1.0 / p.beta2, p.alpha + k * (p.eps + p.alpha2)))
+            if p.wake > 0:  # reading C28: T3 = A + k(ε + α') + x/β'
+                pc += ((1.0 / p.beta2, p.wake + k * (p.eps + p.alpha2)),)
+            out.append(pc)
         return out
 
     lines = [pieces(p) for p in paths]

@@ -16,14 +16,15 @@ from __future__ import annotations
 import math
 
 
-def simulate_two_stage(k: int, s1: float, s2: float, slots: int = 0) -> float:
+def simulate_two_stage(k: int, s1: float, s2: float, slots: int = 0, start2: float = 0.0) -> float:
     """Finish time of k chunks through a two-stage pipeline with per-chunk stage
     times s1 (first link incl. its α) and s2 (ε + α' + second link).  slots = 0
-    means unlimited staging buffers."""
+    means unlimited staging buffers.  start2: the second stage is not available before
+    this time (reading C28: the relay kernel's start)."""
     f1 = [0.0] * k      # stage-1 finish of each chunk
     f2 = [0.0] * k      # stage-2 finish of each chunk
     link1_free = 0.0
-    link2_free = 0.0
+    link2_free = start2
     for c in range(k):
         start1 = link1_free
         if slots and c >= slots:

@@ -89,7 +89,8 @@ def evaluate_window(n: int, w: int, nbytes, chunks, paths: Sequence[M.Path], h: 
                     opts: M.Options, port: Optional[M.Port] = None, tau: float = 0.0,
                     h_sub: float = 0.0) -> float:
     """(W1): time of w back-to-back messages of n bytes with the config (nbytes, chunks);
-    h_sub = the host's submission time per message (C27)."""
+    h_sub = the host's submission time per message (C27); a relay's start A (C28) delays
+    the window once."""
     assert w >= 1 and sum(nbytes) == n
     if n == 0:
         return 0.0
@@ -101,9 +102,16 @@ def evaluate_window(n: int, w: int, nbytes, chunks, paths: Sequence[M.Path], h: 
             continue
         if p.kind == M.DIRECT:
             ti = p.alpha + b / p.beta                          # Eq 6
+            t = max(t, path_window_time(ti + s, issue_part(p, hi), w, h_sub))
+        elif opts.mode == M.B200 and p.wake > 0:
+            # C28: the relay starts A late once and then lingers through the window:
+            # the wake-free message's window plus the first message's delay
+            t0 = M.pipelined_time(float(b), int(k), replace(p, wake=0.0), opts.mode)
+            t1 = M.pipelined_time(float(b), int(k), p, opts.mode)
+            t = max(t, path_window_time(t0 + s, issue_part(p, hi), w, h_sub) + (t1 - t0))
         else:
             ti = M.pipelined_time(float(b), int(k), p, opts.mode)  # Eq 13
-        t = max(t, path_window_time(ti + s, issue_part(p, hi), w, h_sub))
+            t = max(t, path_window_time(ti + s, issue_part(p, hi), w, h_sub))
     if opts.mode == M.B200 and port is not None and port.beta != M.INF:
         load = sum(p.w * b for p, b in zip(paths, nbytes))
         if load > 0:
@@ -126,7 +134,9 @@ def select_window(n: int, w: int, paths: Sequence[M.Path], h: Sequence[float], o
         allowed = [True] * len(paths) if path_mask is None else [i == 0 or bool(m) for i, m in enumerate(path_mask)]
         a_s = port_issue_part(port, paths, h, allowed)
         wport = M.Port(alpha=port.alpha - (1.0 - 1.0 / w) * a_s, beta=port.beta)
-    cfg = M.select(n, paths, opts, wport, path_mask, dshift=shift)
+    # C28: one relay start per window, spread over its w messages in the selection
+    wpaths = [replace(p, wake=p.wake / w) for p in paths]
+    cfg = M.select(n, wpaths, opts, wport, path_mask, dshift=shift)
     if n == 0:
         return cfg
     cfg.t_pred = evaluate_window(n, w, cfg.bytes, cfg.chunks, paths, h, opts, port, tau, h_sub)

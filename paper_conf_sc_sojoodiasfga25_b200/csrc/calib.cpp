@@ -15,6 +15,7 @@
 #include <cmath>
 #include <cstring>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "ctx.h"
@@ -624,6 +625,7 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
         if (e) return e;
       }
     }
+  if (c->relay_svc && W >= 3) return mp_calibrate_wake(c, 0, 0);  // C28 (mp_init: after the service starts)
   return world_barrier(c);
 }
 
@@ -941,6 +943,149 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
   if (int e = mp_set_submit_time(c, h_sub)) return e;
   if (int e = mp_set_host_duplex(c, c->rank, std::max(kappa, 1e-3))) return e;
   return MP_OK;
+}
+
+// Reading C28: the relay wake A of every relay rank r (multi-rank, collective, after
+// the relay service is up, no traffic in flight).  Pair (s, d) = (r + 1, r + 2) mod W
+// sends two relay-only messages of `bytes` (k = 1, above the eager limit) through r
+// right after r's relay kernels have gone idle (linger + 1 ms of quiet).  The sender
+// enqueues both first (its gate kernels wait on the device for the clear-to-send);
+// after a barrier the receiver times recv 1 and recv 2 back to back on its stream,
+// so no host skew enters.  Message 1 pays the relay's start (doorbell → service thread
+// → kernel launch), message 2 finds the kernel lingering: t1 = O + max(T, A + k·s2),
+// t2 = O + T (T = C3's time of the pair's model, O = per-message costs both pay), so
+// when the wake binds (median(t1 − t2) > 1 µs) A = T − k·s2 + median(t1 − t2) (k = 1
+// unless a slot is smaller than n: A = s1 + the median), else A = 0 (a wake that never
+// binds changes no prediction).  Every
+// GPU-staged path via r of every pair model and band takes wake = A_r;
+// MPX_RELAY_WAKE_US overrides the probe.  calibrate_world re-runs it (its fresh models
+// start at wake 0) when the relay service is up.
+extern "C" int mp_calibrate_wake(mp_ctx *c, uint64_t bytes, int reps) {
+  if (!c) return MP_ERR_INVALID;
+  if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  const int W = c->world, me = c->rank;
+  if (W < 3) return MP_OK;  // no relay ranks
+  if (reps <= 0) reps = 7;
+  if (bytes == 0) bytes = 2ull << 20;
+  const uint64_t A = c->opts.align;
+  bytes = std::max<uint64_t>(bytes, (c->eager_max / A + 1) * A);
+  // chunks of at most a staging slot (k = 1 unless the slots are small)
+  const uint64_t per = std::max<uint64_t>(A, (c->slot_bytes - A) / A * A);
+  const uint32_t k = static_cast<uint32_t>((bytes + per - 1) / per);
+  std::vector<double> wake(W, 0.0);
+  if (const char *e = std::getenv("MPX_RELAY_WAKE_US")) {
+    for (double &w : wake) w = std::max(0.0, std::atof(e) / 1e6);
+  } else {
+    if (!c->relay_svc) return cfail(c, MP_ERR_STATE, "mp_calibrate_wake: no relay service");
+    const auto quiet = std::chrono::nanoseconds(world_relay_linger_ns(c)) + std::chrono::milliseconds(1);
+    void *rbuf = nullptr, *src = nullptr;
+    cudaStream_t st = nullptr;
+    cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
+    // every rank needs a probe buffer in its heap; a heap too small for one leaves
+    // every wake at 0 (decided collectively: a rank that skips would strand its peers)
+    int32_t no_room = mp_alloc(c, bytes, &rbuf) == MP_OK ? 0 : 1;
+    c->last_error.clear();
+    std::vector<int32_t> rooms(W);
+    if (int e = world_allgather(c, &no_room, rooms.data(), sizeof(no_room))) return e;
+    bool skip = false;
+    for (int32_t v : rooms) skip = skip || v;
+    int rc = MP_OK;
+    double mine = 0.0;  // this rank's result as the receiver of relay (me − 2) mod W
+    do {
+      if (skip) break;
+      if (cudaMalloc(&src, bytes) != cudaSuccess || cudaMemset(src, 0x3c, bytes) != cudaSuccess ||
+          cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) {
+        rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: buffers");
+        break;
+      }
+      for (cudaEvent_t &e : ev)
+        if (cudaEventCreate(&e) != cudaSuccess) rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: events");
+      if (rc) break;
+      for (int r = 0; r < W && !rc; ++r) {
+        const int s = (r + 1) % W, d = (r + 2) % W;
+        mp_config cfg{};
+        mp_path_params prm[MP_MAX_PATHS];
+        int np = 0, idx = -1;
+        if ((me == s || me == d) && (rc = mp_get_model(c, s, d, cfg.path, prm, &np, nullptr))) break;
+        for (int i = 0; i < np; ++i)
+          if (cfg.path[i].kind == MP_PATH_GPU && cfg.path[i].via == r) idx = i;
+        if ((me == s || me == d) && idx < 0) {
+          rc = cfail(c, MP_ERR_TOPOLOGY, "mp_calibrate_wake: pair has no path via relay " + std::to_string(r));
+          break;
+        }
+        if (me == s) {
+          cfg.npaths = np;
+          cfg.bytes[idx] = bytes;
+          cfg.chunks[0] = 1;
+          cfg.chunks[idx] = k;
+        }
+        std::vector<double> diffs;
+        for (int i = 0; i < reps && !rc; ++i) {
+          if ((rc = world_barrier(c))) break;
+          std::this_thread::sleep_for(quiet);
+          if (me == s)
+            for (int j = 0; j < 2 && !rc; ++j) rc = mp_send(c, src, bytes, d, -1000 - j, &cfg, st);
+          if (rc) break;
+          if ((rc = world_barrier(c))) break;
+          if (me == d) {
+            cudaEventRecord(ev[0], st);
+            rc = mp_recv(c, rbuf, bytes, s, -1000, st);
+            cudaEventRecord(ev[1], st);
+            if (!rc) rc = mp_recv(c, rbuf, bytes, s, -1001, st);
+            cudaEventRecord(ev[2], st);
+          }
+          if (rc) break;
+          if (cudaStreamSynchronize(st) != cudaSuccess) {
+            rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: stream");
+            break;
+          }
+          if (me == d) {
+            float t1 = 0, t2 = 0;
+            cudaEventElapsedTime(&t1, ev[0], ev[1]);
+            cudaEventElapsedTime(&t2, ev[1], ev[2]);
+            if (std::getenv("MPX_WAKE_DEBUG"))
+              std::fprintf(stderr, "wake probe relay %d rep %d: t1 %.2f us t2 %.2f us (k %u)\n", r, i, t1 * 1e3,
+                           t2 * 1e3, k);
+            diffs.push_back((static_cast<double>(t1) - static_cast<double>(t2)) * 1e-3);
+          }
+        }
+        if (!rc && me == d && !diffs.empty()) {
+          // t1 − t2 = max(0, A + k·s2 − T) with T = C3's time of the pair's model (the
+          // fixed per-message costs — clear-to-send, launches — cancel in the difference)
+          const mp_path_params &q = prm[idx];
+          const double m = static_cast<double>(bytes) / k;
+          const double s1 = q.alpha + m / q.beta, s2 = q.eps + q.alpha2 + m / q.beta2;
+          const double T = s1 + s2 + (k - 1) * std::max(s1, s2);
+          const double delta = median(diffs);
+          mine = delta > 1e-6 ? std::max(0.0, T - k * s2 + delta) : 0.0;
+        }
+      }
+    } while (false);
+    if (st) cudaStreamSynchronize(st);
+    for (cudaEvent_t e : ev)
+      if (e) cudaEventDestroy(e);
+    if (st) cudaStreamDestroy(st);
+    if (src) cudaFree(src);
+    if (rbuf) mp_free(c, rbuf);
+    int32_t ok = rc ? 1 : 0;
+    std::vector<int32_t> all_ok(W);
+    if (int e = world_allgather(c, &ok, all_ok.data(), sizeof(ok))) return e;
+    if (rc) return rc;
+    for (int32_t v : all_ok)
+      if (v) return cfail(c, MP_ERR_STATE, "wake calibration failed on another rank");
+    std::vector<double> got(W);
+    if (int e = world_allgather(c, &mine, got.data(), sizeof(double))) return e;
+    for (int d = 0; d < W; ++d) wake[(d - 2 + W) % W] = got[d];  // rank d measured relay d − 2
+  }
+  auto apply = [&](PairModel &m) {
+    for (PathModel &q : m.paths)
+      if (q.kind == K_GPU && q.via >= 0 && q.via < W) q.wake = wake[q.via];
+  };
+  for (auto &kv : c->models) apply(kv.second);
+  for (auto &kv : c->bands)
+    for (auto &b : kv.second) apply(b.second);
+  c->cache.clear();
+  return world_barrier(c);
 }
 
 // The C24 estimator of mp_calibrate_window on given samples (pure host arithmetic).

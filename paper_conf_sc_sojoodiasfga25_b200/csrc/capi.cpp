@@ -522,6 +522,14 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
       mp_finalize(c);
       return s;
     }
+    // reading C28: the relays' start time, once their service runs
+    if (c->world >= 3 && !(a->flags & MP_INIT_NO_CALIBRATE) && c->relay_svc) {
+      if (int s = mp_calibrate_wake(c, 0, 0)) {
+        std::fprintf(stderr, "mp_init: wake calibration failed: %s\n", c->last_error.c_str());
+        mp_finalize(c);
+        return s;
+      }
+    }
   }
   *out = c;
   return MP_OK;
@@ -570,6 +578,7 @@ int mp_set_model(mp_ctx *c, int src, int dst, const mp_path *paths, const mp_pat
     p.c = prm[i].c;
     p.sigma = prm[i].sigma;
     p.w = prm[i].w;
+    p.wake = prm[i].wake;
     m.paths.push_back(p);
   }
   if (port) {
@@ -612,6 +621,7 @@ int mp_set_model_band(mp_ctx *c, int src, int dst, uint64_t n_min, const mp_path
     p.c = prm[i].c;
     p.sigma = prm[i].sigma;
     p.w = prm[i].w;
+    p.wake = prm[i].wake;
   }
   m.port_alpha = port ? port->alpha : 0.0;
   m.port_beta = port ? port->beta : 0.0;
@@ -648,7 +658,7 @@ int mp_get_model_band(mp_ctx *c, int src, int dst, int band, uint64_t *n_min, mp
   if (prm)
     for (size_t i = 0; i < m->paths.size(); ++i) {
       const PathModel &p = m->paths[i];
-      prm[i] = mp_path_params{p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w};
+      prm[i] = mp_path_params{p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w, p.wake};
     }
   if (port) {
     port->alpha = m->port_alpha;
@@ -669,7 +679,7 @@ int mp_get_model(mp_ctx *c, int src, int dst, mp_path *paths, mp_path_params *pr
       paths[i].kind = p.kind;
       paths[i].via = p.via;
     }
-    if (prm) prm[i] = mp_path_params{p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w};
+    if (prm) prm[i] = mp_path_params{p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w, p.wake};
   }
   if (port) {
     port->alpha = m->port_alpha;
@@ -1062,8 +1072,8 @@ int mp_save_params(mp_ctx *c, const char *path) {
     std::fprintf(f, "pair %d %d %zu %.17g %.17g\n", kv.first.first, kv.first.second, m.paths.size(),
                  m.port_alpha, m.port_beta);
     for (const PathModel &p : m.paths)
-      std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via,
-                   p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
+      std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via,
+                   p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w, p.wake);
     auto wt = c->windows.find(kv.first);
     if (wt != c->windows.end()) {
       std::fprintf(f, "window %d %d %zu %.17g", kv.first.first, kv.first.second, wt->second.h.size(), wt->second.tau);
@@ -1076,8 +1086,8 @@ int mp_save_params(mp_ctx *c, const char *path) {
       std::fprintf(f, "band %d %d %zu %llu %.17g %.17g\n", kv.first.first, kv.first.second, b.second.paths.size(),
                    static_cast<unsigned long long>(b.first), b.second.port_alpha, b.second.port_beta);
       for (const PathModel &p : b.second.paths)
-        std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via, p.alpha,
-                     p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w);
+        std::fprintf(f, "path %d %d %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g %.17g\n", p.kind, p.via,
+                     p.alpha, p.beta, p.alpha2, p.beta2, p.eps, p.c, p.sigma, p.w, p.wake);
     }
   }
   for (size_t g = 0; g < c->kappa.size(); ++g)
@@ -1166,9 +1176,11 @@ int mp_load_params(mp_ctx *c, const char *path) {
     mp_path_params prm[MP_MAX_PATHS];
     for (size_t k = 0; k < np; ++k) {
       mp_path_params &q = prm[k];
-      if (std::sscanf(lines[i + 1 + k].c_str(), "%31s %d %d %lf %lf %lf %lf %lf %lf %lf %lf", tag, &paths[k].kind,
-                      &paths[k].via, &q.alpha, &q.beta, &q.alpha2, &q.beta2, &q.eps, &q.c, &q.sigma, &q.w) != 11)
-        return truncated();
+      q.wake = 0.0;  // a round-2 file has no 12th field (C28)
+      const int got_p = std::sscanf(lines[i + 1 + k].c_str(), "%31s %d %d %lf %lf %lf %lf %lf %lf %lf %lf %lf", tag,
+                                    &paths[k].kind, &paths[k].via, &q.alpha, &q.beta, &q.alpha2, &q.beta2, &q.eps,
+                                    &q.c, &q.sigma, &q.w, &q.wake);
+      if (got_p != 11 && got_p != 12) return truncated();
     }
     mp_port_params port{pa, pb};
     if (pair_ok(c, src, dst)) {

@@ -448,11 +448,6 @@ void mpx::coll_release(mp_ctx *c) {
   if (st.s) cudaStreamSynchronize(st.s);
   if (st.r) cudaStreamSynchronize(st.r);
   for (cudaEvent_t e : st.ev) cudaEventDestroy(e);
-  // the engine remembers every stream it enqueued on (mp_sync / finalize synchronise
-  // them): forget the internal ones before destroying them
-  c->streams.erase(std::remove_if(c->streams.begin(), c->streams.end(),
-                                  [&](cudaStream_t x) { return x == st.s || x == st.r; }),
-                   c->streams.end());
   if (st.s) cudaStreamDestroy(st.s);
   if (st.r) cudaStreamDestroy(st.r);
   if (st.scratch) mp_free(c, st.scratch);

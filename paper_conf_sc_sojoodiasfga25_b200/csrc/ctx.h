@@ -136,7 +136,6 @@ struct mp_ctx {
   uint64_t eager_max = 0;                   // messages of 1..eager_max bytes go eager
   mpx::RelayService *relay_svc = nullptr;   // world >= 3: launches relay kernels on doorbells
   uint64_t relay_launches_done = 0;         // relay launches of stopped services
-  std::vector<cudaStream_t> streams;        // user streams seen by mp_send/mp_recv
   // receive regions (mp_register): [kMaxRegions], region 0 = the heap
   struct Region {
     bool used = false;
@@ -193,6 +192,7 @@ int world_start_relay(mp_ctx *c);
 int world_stop_relay(mp_ctx *c);
 uint64_t world_relay_launches(const mp_ctx *c);  // relay kernels this rank launched
 int world_relay_error(const mp_ctx *c);          // cudaError_t of a failed relay launch, 0 if none
+uint64_t world_relay_linger_ns(const mp_ctx *c);  // the relay kernels' linger, 0 without a service
 int world_finalize(mp_ctx *c);
 int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, const mp_config &cfg,
                void *stream);

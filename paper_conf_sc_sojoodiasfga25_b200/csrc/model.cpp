@@ -25,12 +25,14 @@ inline int bottleneck(const PathModel &p, int mode) {
 
 // Staged path carrying x bytes in k chunks.  m = x/k (Eq 12);
 // s1 = α + m/β, s2 = ε + α' + m/β'.  PAPER: Eq 13 (case 1 k·s1 + s2, case 2
-// s1 + k·s2).  B200: s1 + s2 + (k−1)·max(s1, s2) (C3).
+// s1 + k·s2).  B200: s1 + s2 + (k−1)·max(s1, s2) (C3), and no earlier than the
+// relay's start A plus k stage-2 services, A + k·s2 (C28).
 inline double staged_time(const PathModel &p, double x, uint32_t k, int mode) {
   const double m = x / static_cast<double>(k);
   const double s1 = p.alpha + m / p.beta;
   const double s2 = p.eps + p.alpha2 + m / p.beta2;
-  if (mode == M_B200) return s1 + s2 + static_cast<double>(k - 1) * std::max(s1, s2);
+  if (mode == M_B200)
+    return std::max(s1 + s2 + static_cast<double>(k - 1) * std::max(s1, s2), p.wake + static_cast<double>(k) * s2);
   if (bottleneck(p, M_PAPER) == 1) return static_cast<double>(k) * s1 + s2;
   return s1 + static_cast<double>(k) * s2;
 }
@@ -272,14 +274,30 @@ uint32_t clamp_k(uint64_t k, uint64_t b, const ModelOpts &o) {
 // Reading C26 (B200 mode): the integer k in C5's clamp range minimising the exact
 // pipeline time T(k) = max(k·s1 + s2, s1 + k·s2) (convex in k): the floor / ceiling of
 // the minimiser of either piece (Eq 14, Eq 15) or of the stage crossover s1 = s2, or
-// a bound of the range; ties to the smaller k.
+// a bound of the range; ties to the smaller k.  C28: with a relay start A the third
+// piece A + k·s2 (increasing in k) adds its crossovers with the other two.
 uint32_t k_exact(const PathModel &p, double x, uint64_t b, const ModelOpts &o) {
   const uint32_t lo = clamp_k(1, b, o);
   const uint32_t hi = std::max(lo, clamp_k(1000000000ull, b, o));
   const double e = p.eps + p.alpha2;
-  double reals[3] = {std::sqrt(x / (p.alpha * p.beta2)), std::sqrt(x / (p.beta * e)), -1.0};
+  double reals[6] = {std::sqrt(x / (p.alpha * p.beta2)), std::sqrt(x / (p.beta * e)), -1.0, -1.0, -1.0, -1.0};
   if (p.alpha != e) reals[2] = x * (1.0 / p.beta2 - 1.0 / p.beta) / (p.alpha - e);
-  uint32_t cand[8] = {lo, hi, lo, lo, lo, lo, lo, lo};
+  if (p.wake > 0.0) {
+    // A + k·e + x/β' = α + x/(kβ) + k·e + x/β'  ⇔  k = x / (β(A − α))
+    if (p.wake > p.alpha) reals[3] = x / (p.beta * (p.wake - p.alpha));
+    // A + k·e + x/β' = k·α + x/β + e + x/(kβ')  ⇔  (e − α)k² + (A − e + x/β' − x/β)k − x/β' = 0
+    const double qa = e - p.alpha, qb = p.wake - e + x / p.beta2 - x / p.beta, qc = -x / p.beta2;
+    if (qa == 0.0) {
+      if (qb != 0.0) reals[4] = -qc / qb;
+    } else {
+      const double disc = qb * qb - 4.0 * qa * qc;
+      if (disc >= 0.0) {
+        reals[4] = (-qb + std::sqrt(disc)) / (2.0 * qa);
+        reals[5] = (-qb - std::sqrt(disc)) / (2.0 * qa);
+      }
+    }
+  }
+  uint32_t cand[14] = {lo, hi, lo, lo, lo, lo, lo, lo, lo, lo, lo, lo, lo, lo};
   int nc = 2;
   for (double r : reals) {
     if (!(r > 0.0)) continue;
@@ -300,11 +318,16 @@ uint32_t k_exact(const PathModel &p, double x, uint64_t b, const ModelOpts &o) {
   return best;
 }
 
-// Reading C26: the affine piece of the exact pipeline time at k chunks binding at x.
+// Reading C26: the affine piece of the exact pipeline time at k chunks binding at x
+// (C28: the availability piece Ω = 1/β', Δ = A + k(ε + α') when it is the largest).
 void piece_exact(const PathModel &p, double x, uint32_t k, double *om, double *de) {
   const double kd = static_cast<double>(k), m = x / kd;
   const double s1 = p.alpha + m / p.beta, s2 = p.eps + p.alpha2 + m / p.beta2;
-  if (s1 >= s2) {
+  const double t12 = s1 + s2 + static_cast<double>(k - 1) * std::max(s1, s2);
+  if (p.wake > 0.0 && p.wake + kd * s2 > t12) {
+    *om = 1.0 / p.beta2;
+    *de = p.wake + kd * (p.eps + p.alpha2);
+  } else if (s1 >= s2) {
     *om = 1.0 / p.beta + 1.0 / (kd * p.beta2);
     *de = kd * p.alpha + p.eps + p.alpha2;
   } else {
@@ -346,6 +369,7 @@ std::string validate_model(const PairModel &m) {
     if (!(p.beta > 0.0) || !std::isfinite(p.beta)) return "beta must be finite and > 0";
     if (!(p.alpha >= 0.0) || !std::isfinite(p.alpha)) return "alpha must be finite and >= 0";
     if (!(p.w >= 0.0) || !(p.sigma >= 0.0)) return "w and sigma must be >= 0";
+    if (!(p.wake >= 0.0) || !std::isfinite(p.wake)) return "wake must be finite and >= 0";
     if (p.kind != K_DIRECT) {
       if (!(p.beta2 > 0.0) || !std::isfinite(p.beta2)) return "staged beta2 must be finite and > 0";
       if (!(p.alpha2 >= 0.0) || !(p.eps >= 0.0)) return "staged alpha2/eps must be >= 0";
@@ -491,6 +515,8 @@ void select(const PairModel &m, uint64_t n, uint32_t mask, const ModelOpts &o, S
 // T_i − a_i).  The port is one more such pipeline with a_S = min(α_S, min a_i of the
 // active paths through it).  T^w = τ + max(paths, port).  Reading C27: the host enqueues
 // the messages h_sub apart, so the per-message step is max(a_i, T_i − a_i, h_sub).
+// Reading C28: a relay's start A delays the window once (the relay then lingers); the
+// selection spreads it over the window (A/w per message).
 
 namespace {
 inline double issue_part(const PathModel &p, const WindowModel &wm, size_t i) {
@@ -522,8 +548,18 @@ double predict_window(const PairModel &m, const WindowModel &wm, uint64_t n, uin
     if (!act[i]) continue;
     const PathModel &q = m.paths[i];
     const double b = static_cast<double>(bytes[i]);
-    const double ti = (q.kind == K_DIRECT) ? q.alpha + b / q.beta : staged_time(q, b, chunks[i], o.mode);
-    t = std::max(t, window_of(ti + st[i], issue_part(q, wm, i), w, wm.submit));
+    if (q.kind == K_DIRECT || o.mode != M_B200 || q.wake <= 0.0) {
+      const double ti = (q.kind == K_DIRECT) ? q.alpha + b / q.beta : staged_time(q, b, chunks[i], o.mode);
+      t = std::max(t, window_of(ti + st[i], issue_part(q, wm, i), w, wm.submit));
+    } else {
+      // C28 in a window: the relay starts late once, then lingers through the window —
+      // the steady pipeline of the wake-free message plus the first message's delay
+      PathModel q0 = q;
+      q0.wake = 0.0;
+      const double t0 = staged_time(q0, b, chunks[i], o.mode);
+      const double t1 = staged_time(q, b, chunks[i], o.mode);
+      t = std::max(t, window_of(t0 + st[i], issue_part(q, wm, i), w, wm.submit) + (t1 - t0));
+    }
   }
   if (o.mode == M_B200 && m.has_port()) {
     double load = 0.0;
@@ -546,6 +582,7 @@ void select_window(const PairModel &m, const WindowModel &wm, uint64_t n, uint32
   }
   PairModel mw = m;  // per-message port startup of the window
   if (m.has_port()) mw.port_alpha = m.port_alpha - f * port_issue(m, wm, allowed);
+  for (PathModel &q : mw.paths) q.wake /= static_cast<double>(w);  // C28: one relay start per window
   select(mw, n, mask, o, out, shift.data());
   if (n == 0) return;
   out->t_pred = predict_window(m, wm, n, w, out->bytes.data(), out->chunks.data(), o);

@@ -16,6 +16,7 @@ struct PathModel {
   int kind = K_DIRECT;
   int via = -1;
   double alpha = 0, beta = 0, alpha2 = 0, beta2 = 0, eps = 0, c = 1, sigma = 0, w = 0;
+  double wake = 0;  // B200 mode (C28): earliest start of stage 2 after the message starts [s]
 };
 
 struct PairModel {

@@ -416,10 +416,13 @@ uint64_t world_relay_launches(const mp_ctx *c) {
 
 int world_relay_error(const mp_ctx *c) { return c->relay_svc ? c->relay_svc->error.load() : 0; }
 
+uint64_t world_relay_linger_ns(const mp_ctx *c) { return c->relay_svc ? c->relay_svc->linger_ns : 0; }
+
 int world_finalize(mp_ctx *c) {
   int st = MP_OK;
   world_stop_relay(c);
-  for (cudaStream_t s : c->streams) cudaStreamSynchronize(s);
+  cudaDeviceSynchronize();  // every stream this process enqueued on (not a list of handles
+                            // the caller may have destroyed since)
   if (c->allgather) st = barrier(c);
   for (int r = 0; r < static_cast<int>(c->peers.size()); ++r) {
     if (r == c->rank) continue;
@@ -440,9 +443,6 @@ int world_finalize(mp_ctx *c) {
   return st;
 }
 
-static void note_stream(mp_ctx *c, cudaStream_t s) {
-  if (std::find(c->streams.begin(), c->streams.end(), s) == c->streams.end()) c->streams.push_back(s);
-}
 
 // Eager protocol (reading C23): 1..eager_max bytes, direct path, no rendezvous.
 static EagerParams eager_params(mp_ctx *c, int sender, int receiver, uint64_t seq, uint64_t bytes, int tag) {
@@ -471,7 +471,6 @@ static int eager_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int t
     return wfail(c, MP_ERR_CUDA, std::string("eager send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   c->launches += 1;
   c->eager_send_seq[dst] += 1;
-  note_stream(c, static_cast<cudaStream_t>(stream));
   return MP_OK;
 }
 
@@ -483,7 +482,6 @@ static int eager_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, vo
     return wfail(c, MP_ERR_CUDA, std::string("eager recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   c->launches += 1;
   c->eager_recv_seq[src] += 1;
-  note_stream(c, static_cast<cudaStream_t>(stream));
   return MP_OK;
 }
 
@@ -566,7 +564,6 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
       c->relay_m[a.first] += 1;
     }
   }
-  note_stream(c, static_cast<cudaStream_t>(stream));
   return MP_OK;
 }
 
@@ -624,7 +621,6 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   c->launches += 1;
   c->recv_seq[src] += 1;
   c->done_target[src] += bytes;
-  note_stream(c, static_cast<cudaStream_t>(stream));
   return MP_OK;
 }
 
@@ -767,7 +763,7 @@ int world_deregister(mp_ctx *c, int id) {
   RegInfo me;
   std::memset(&me, 0, sizeof(me));
   me.id = id;
-  for (cudaStream_t s : c->streams) CKW(cudaStreamSynchronize(s));  // our receives into it are done
+  CKW(cudaDeviceSynchronize());  // our receives into it are done
   std::vector<RegInfo> all(W);
   if (int s = allgather(c, &me, all.data(), sizeof(RegInfo))) return s;
   for (int r = 0; r < W; ++r)
@@ -780,8 +776,12 @@ int world_deregister(mp_ctx *c, int id) {
   return st;
 }
 
+// A device-wide wait: every stream this process used (relay kernels are bounded
+// launches, §7, so nothing outlives the traffic by more than the linger).  The engine
+// keeps no list of the caller's streams: a handle destroyed after mp_send would make
+// such a list unusable.
 int world_sync(mp_ctx *c) {
-  for (cudaStream_t s : c->streams) CKW(cudaStreamSynchronize(s));
+  CKW(cudaDeviceSynchronize());
   if (int e = world_relay_error(c))
     return wfail(c, MP_ERR_CUDA, std::string("relay launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   int32_t e = 0;

@@ -35,7 +35,7 @@ class mp_path(C.Structure):
 
 
 class mp_path_params(C.Structure):
-    _fields_ = [(n, C.c_double) for n in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")]
+    _fields_ = [(n, C.c_double) for n in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w", "wake")]
 
 
 class mp_port_params(C.Structure):
@@ -187,6 +187,7 @@ def lib():
                                            C.POINTER(mp_config)]),
             "mp_set_host_duplex": (C.c_int, [P, C.c_int, C.c_double]),
             "mp_calibrate_window": (C.c_int, [P, C.POINTER(C.c_uint64), C.c_int, C.c_int, C.c_int]),
+            "mp_calibrate_wake": (C.c_int, [P, C.c_uint64, C.c_int]),
             "mp_fit_window": (C.c_int, [C.POINTER(C.c_int), C.POINTER(C.c_double), C.POINTER(C.c_double),
                                         C.POINTER(C.c_double), C.c_int, C.c_int, C.c_int, C.c_double,
                                         C.POINTER(C.c_double), C.POINTER(C.c_double)]),
@@ -216,7 +217,7 @@ def exported_symbols() -> List[str]:
             "mp_set_model_band", "mp_get_model_band", "mp_fit_bands", "mp_calibrate_bands",
             "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
-            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_fit_window",
+            "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_calibrate_wake", "mp_fit_window",
             "mp_get_topology", "mp_set_topology", "mp_set_submit_time", "mp_get_submit_time"]
 
 
@@ -277,7 +278,7 @@ def _params_array(params: Sequence[dict]):
     return (mp_path_params * MP_MAX_PATHS)(
         *[mp_path_params(*[float(p.get(f, d)) for f, d in
                            (("alpha", 0), ("beta", 0), ("alpha2", 0), ("beta2", 0), ("eps", 0),
-                            ("c", 1), ("sigma", 0), ("w", 0))]) for p in params])
+                            ("c", 1), ("sigma", 0), ("w", 0), ("wake", 0))]) for p in params])
 
 
 def _ptr(x) -> Optional[int]:
@@ -453,6 +454,10 @@ class Context:
         """mp_calibrate_window (loopback; readings C24, C25)."""
         arr = (C.c_uint64 * len(sizes))(*sizes) if sizes else None
         self._ck(lib().mp_calibrate_window(self.h, arr, len(sizes) if sizes else 0, window, reps))
+
+    def calibrate_wake(self, nbytes=0, reps=0):
+        """mp_calibrate_wake (reading C28; collective, world >= 3)."""
+        self._ck(lib().mp_calibrate_wake(self.h, nbytes, reps))
 
     def set_submit_time(self, seconds: float):
         """mp_set_submit_time (reading C27): the host's time per enqueued message."""

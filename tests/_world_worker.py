@@ -629,6 +629,81 @@ def scenario_full_size(rank, world):
     c.close()
 
 
+def scenario_wake(rank, world):
+    """Reading C28: mp_calibrate_wake measures each relay rank's start time and every
+    GPU-staged path via that relay carries it in every pair model (all ranks agree);
+    the MPX_RELAY_WAKE_US override installs its value exactly; relayed messages stay
+    bit-exact and the B200 pick's prediction includes the wake."""
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    n = 8 * MiB + 4099
+    src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                        generator=torch.Generator(device="cuda").manual_seed(7)) if rank == 0 else None
+    torch.cuda.synchronize()
+    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, timeout_s=60.0, calibrate=False)
+    c.calibrate(sizes=[4 * MiB, 8 * MiB, 16 * MiB], reps=2)   # Step 1, then the wake probe
+    wakes = {}
+    for s_ in range(world):
+        for d_ in range(world):
+            if s_ == d_:
+                continue
+            paths, prm, _ = c.get_model(s_, d_)
+            for (kind, via), p in zip(paths, prm):
+                if kind == mp.MP_PATH_GPU:
+                    # every rank on one GPU: µs under MPS, a scheduling time slice (ms) without
+                    assert 0.0 <= p["wake"] < 0.1, (s_, d_, via, p["wake"])
+                    assert wakes.setdefault(via, p["wake"]) == p["wake"]   # one value per relay
+                else:
+                    assert p["wake"] == 0.0
+    allw = [None] * world
+    dist.all_gather_object(allw, wakes)
+    assert all(w == allw[0] for w in allw), allw
+    print(f"rank {rank}: measured relay wakes [us] " + str({k: round(v * 1e6, 2) for k, v in wakes.items()}),
+          flush=True)
+    os.environ["MPX_RELAY_WAKE_US"] = "50"
+    c.calibrate_wake()
+    del os.environ["MPX_RELAY_WAKE_US"]
+    paths, prm, _ = c.get_model(0, 1)
+    for (kind, _), p in zip(paths, prm):
+        assert p["wake"] == (50e-6 if kind == mp.MP_PATH_GPU else 0.0)
+    c.set_options(mode=mp.MP_MODEL_B200)
+    nb = [0] * len(paths)
+    nb[1] = n
+    ks = [1] + [0] * (len(paths) - 1)
+    ks[1] = 4
+    cfg = c.make_config(nb, ks, 0, 1)
+    p1 = prm[1]
+    s2 = p1["eps"] + p1["alpha2"] + n / 4 / p1["beta2"]
+    assert c.predict(0, 1, n, cfg) >= 50e-6 + 4 * s2 - 1e-12
+    rbuf = c.alloc(n) if rank == 1 else None
+    if rank == 0:
+        c.send(src, n, 1, tag=5, cfg=cfg, stream=stream)
+        c.send(src, n, 1, tag=6, cfg=None, stream=stream)
+        stream.synchronize()
+        dist.send(torch.tensor([1]), 1)
+    elif rank == 1:
+        view = mp.as_tensor(rbuf, n)
+        ref = torch.empty(n, dtype=torch.uint8, device="cuda")
+        for t in (5, 6):
+            view.zero_()
+            torch.cuda.synchronize()
+            c.recv(rbuf, n, 0, tag=t, stream=stream)
+            stream.synchronize()
+            if t == 5:
+                ref.copy_(view)
+        dist.recv(torch.tensor([0]), 0)
+        exp = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
+                            generator=torch.Generator(device="cuda").manual_seed(7))
+        assert torch.equal(ref, exp) and torch.equal(view, exp)
+    dist.barrier()
+    c.sync()
+    if rbuf:
+        c.free(rbuf)
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
@@ -640,7 +715,7 @@ def main():
          "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
          "eager": scenario_eager, "devsync": scenario_devsync,
          "bench_plan": scenario_bench_plan, "relay_burst": scenario_relay_burst,
-         "full_size": scenario_full_size}[scen](rank, world)
+         "full_size": scenario_full_size, "wake": scenario_wake}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

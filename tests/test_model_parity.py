@@ -169,3 +169,75 @@ def test_b200_heavy_latency_parity(seed):
             if d["bytes"] == ref.bytes:
                 assert d["chunks"] == ref.chunks
             assert rel(d["t_pred"], ref.t_pred) < 1e-9 and rel(d["t_level"], ref.t_level) < 1e-9
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_c28_wake_parity(seed):
+    # reading C28 (a relay that starts A after the message): library = oracle for the
+    # pick (shares ±A, chunks, level, prediction 1e-9) and for mp_predict of any config
+    import sys
+    import os
+    import dataclasses
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from test_oracle_select import heavy_paths, with_wake
+    rnd = random.Random(6000 + seed)
+    base = heavy_paths(rnd, 1 + seed % 3) if seed % 2 else [M.Path(**t) for t in synth.topology(seed, 3, True)]
+    paths = [with_wake(p, rnd) for p in base]
+    tbl = [dict(kind=p.kind, via=(p.via if p.kind == 1 else -1), alpha=p.alpha, beta=p.beta, alpha2=p.alpha2,
+                beta2=p.beta2, eps=p.eps, c=p.c, sigma=p.sigma, w=p.w) for p in paths]
+    port = dict(alpha=paths[0].alpha, beta=paths[0].beta * rnd.uniform(0.9, 1.6))
+    o = M.Options(mode=M.B200, slot_bytes=32 * MiB - 512)
+    with mp.Context(world=8, rank=0, model_only=True) as c:
+        params = [{k: t[k] for k in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")} for t in tbl]
+        for p, q in zip(params, paths):
+            p["wake"] = q.wake
+            if math.isinf(p["beta2"]):
+                p["beta2"] = 0.0
+        c.set_model(0, 1, [(t["kind"], t["via"]) for t in tbl], params, port)
+        assert [p["wake"] for p in c.get_model(0, 1)[1]] == [q.wake for q in paths]
+        c.set_options(mode=M.B200, slot_bytes=o.slot_bytes)
+        for n in (4 * MiB, 16 * MiB, 64 * MiB + 3, 256 * MiB, 1 << 30):
+            d = c.select(0, 1, n).as_dict()
+            ref = M.select(n, paths, o, M.Port(**port))
+            assert sum(d["bytes"]) == n
+            for a, b in zip(d["bytes"], ref.bytes):
+                assert abs(a - b) <= o.align
+            if d["bytes"] == ref.bytes:
+                assert d["chunks"] == ref.chunks
+            assert rel(d["t_pred"], ref.t_pred) < 1e-9 and rel(d["t_level"], ref.t_level) < 1e-9
+            # mp_predict of an arbitrary config: every staged path at k = 1..8 chunks
+            nb = [n - sum(n // (2 * len(paths)) // 256 * 256 for _ in paths[1:])] + \
+                 [n // (2 * len(paths)) // 256 * 256] * (len(paths) - 1)
+            ch = [1] + [1 + rnd.randrange(8)] * (len(paths) - 1)
+            cfg = c.make_config(nb, ch, 0, 1)
+            assert rel(c.predict(0, 1, n, cfg), M.evaluate(n, nb, ch, paths, o, M.Port(**port))) < 1e-9
+        # wake = 0 is C26 exactly
+        c.set_model(0, 1, [(t["kind"], t["via"]) for t in tbl], [dict(p, wake=0.0) for p in params], port)
+        d = c.select(0, 1, 256 * MiB).as_dict()
+        ref = M.select(256 * MiB, [dataclasses.replace(p, wake=0.0) for p in paths], o, M.Port(**port))
+        assert rel(d["t_pred"], ref.t_pred) < 1e-9
+
+
+def test_c28_wake_validation_and_params_file(tmp_path):
+    tbl = synth.topology(3, 2, True)
+    paths = [(t["kind"], t["via"]) for t in tbl]
+    params = [{k: (0.0 if k == "beta2" and math.isinf(t[k]) else t[k])
+               for k in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")} for t in tbl]
+    params[1]["wake"] = 17e-6
+    f = str(tmp_path / "p.txt")
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        for bad in (-1e-6, math.inf, math.nan):
+            with pytest.raises(mp.MPError):
+                c.set_model(0, 1, paths, [dict(p, wake=bad) if i == 1 else p for i, p in enumerate(params)])
+        c.set_model(0, 1, paths, params)
+        c.save_params(f)
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        c.load_params(f)
+        assert c.get_model(0, 1)[1][1]["wake"] == 17e-6
+    # a round-2 file (11 fields per path line) still loads, with wake = 0
+    txt = open(f).read().splitlines()
+    old = [" ".join(ln.split()[:11]) if ln.startswith("path ") else ln for ln in txt]
+    open(f, "w").write("\n".join(old) + "\n")
+    with mp.Context(world=4, rank=0, model_only=True) as c:
+        c.load_params(f)
+        assert c.get_model(0, 1)[1][1]["wake"] == 0.0

@@ -282,3 +282,34 @@ def test_des_finite_ring_never_faster():
             inf = simulate_two_stage(k, s1, s2)
             assert simulate_two_stage(k, s1, s2, slots=2) >= inf - 1e-15
             assert simulate_two_stage(k, s1, s2, slots=k) == inf
+
+
+# ------------------------------------------------- reading C28: stage-2 availability (wake)
+
+@settings(max_examples=200, deadline=None)
+@given(staged, st.floats(1e5, 2e9), st.integers(1, 64), st.floats(0, 500))
+def test_c28_wake_matches_pipeline_simulation(p, x, k, wake_us):
+    # B200 mode with a relay that starts A after the message: the closed form
+    # max(s1 + s2 + (k−1)·max(s1, s2), A + k·s2) against the event simulation whose
+    # second link is busy until A (oracle/pipeline.py, chunk by chunk)
+    import dataclasses
+    q = dataclasses.replace(p, wake=wake_us * US)
+    s1, s2 = stage_times(x, k, q.alpha, q.beta, q.eps, q.alpha2, q.beta2)
+    assert rel(M.pipelined_time(x, k, q, M.B200), simulate_two_stage(k, s1, s2, start2=q.wake)) < 1e-12
+    # the wake only ever delays, and A = 0 is C3 exactly
+    assert M.pipelined_time(x, k, q, M.B200) >= M.pipelined_time(x, k, p, M.B200)
+    assert simulate_two_stage(k, s1, s2, start2=0.0) == simulate_two_stage(k, s1, s2)
+
+
+def test_c28_wake_special_cases():
+    # A huge wake: the second link alone after A, k·s2; k = 1 store-and-forward: s1 + s2
+    # unless the relay is not up yet (max(s1, A) + s2)
+    p = M.Path(M.GPU_STAGED, 2 * US, 400 * GBS, 3 * US, 500 * GBS, 1 * US, wake=10e-3)
+    x = 64 * 2 ** 20
+    for k in (1, 4, 32):
+        s2 = p.eps + p.alpha2 + x / k / p.beta2
+        assert M.pipelined_time(x, k, p, M.B200) == pytest.approx(p.wake + k * s2, rel=1e-15)
+    p = M.Path(M.GPU_STAGED, 2 * US, 400 * GBS, 3 * US, 500 * GBS, 1 * US, wake=5 * US)
+    s1 = p.alpha + x / p.beta
+    s2 = p.eps + p.alpha2 + x / p.beta2
+    assert M.pipelined_time(x, 1, p, M.B200) == pytest.approx(max(s1, p.wake) + s2, rel=1e-15)

@@ -246,3 +246,76 @@ def test_b200_select_vs_exact_pipeline_optimum(seed, mib):
         t_opt = O.level_integer_k_b200(float(n), paths, k_max=256)
         assert t_opt * (1 - 1e-9) <= cfg.t_pred * (1 + 1e-9)
         assert cfg.t_pred <= t_opt * bound, (cfg.t_pred / t_opt, cfg.bytes, cfg.chunks)
+
+
+# ---------------------------------------------------------------- reading C28 (relay wake)
+
+def with_wake(p, rnd):
+    import dataclasses
+    if p.kind != M.GPU_STAGED:
+        return p
+    return dataclasses.replace(p, wake=math.exp(rnd.uniform(math.log(1e-6), math.log(2e-3))))
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_c28_k_exact_is_the_integer_argmin_with_wake(seed):
+    # the availability piece A + k·s2 adds two crossovers to C26's candidates; brute
+    # force over C5's clamp range still agrees (ties to the lower k)
+    import random
+    rnd = random.Random(7000 + seed)
+    p = with_wake(heavy_paths(rnd, 1)[1], rnd)
+    opts = M.Options(mode=M.B200, slot_bytes=32 * MiB - 512)
+    b = rnd.choice([1, 4, 16, 64, 256]) * MiB + 256 * rnd.randrange(1000)
+    k = M.k_exact(float(b), p, b, opts)
+    lo, hi = M._clamp_k(1, b, opts), max(M._clamp_k(1, b, opts), M._clamp_k(10 ** 9, b, opts))
+    ts = {kk: M.pipelined_time(float(b), kk, p, M.B200) for kk in range(lo, hi + 1)}
+    best = min(ts.values())
+    assert ts[k] == best and all(ts[kk] > best for kk in range(lo, k))
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_c28_piece_is_the_binding_affine_piece(seed):
+    # piece_exact's (Ω, Δ) reproduces the exact time at x and bounds it from below at
+    # every other x (the max of affine pieces at fixed k)
+    import random
+    rnd = random.Random(8000 + seed)
+    p = with_wake(heavy_paths(rnd, 1)[1], rnd)
+    x = rnd.choice([1, 16, 256]) * MiB
+    k = rnd.randrange(1, 64)
+    om, de = M.piece_exact(float(x), k, p)
+    assert om * x + de == pytest.approx(M.pipelined_time(float(x), k, p, M.B200), rel=1e-12)
+    for y in (x / 7, x / 2, 2 * x, 9 * x):
+        assert om * y + de <= M.pipelined_time(y, k, p, M.B200) * (1 + 1e-12)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_c28_select_with_wake(seed):
+    # a late relay: the pick never predicts worse than direct alone, its prediction is
+    # its own evaluation, and a relay that wakes after the direct path would have
+    # finished carries nothing
+    import random
+    rnd = random.Random(9000 + seed)
+    paths = [with_wake(p, rnd) for p in heavy_paths(rnd, rnd.randrange(1, 4))]
+    n = rnd.choice([4, 16, 64, 256]) * MiB
+    opts = M.Options(mode=M.B200, slot_bytes=32 * MiB - 512)
+    cfg = M.select(n, paths, opts)
+    direct = M.evaluate(n, [n] + [0] * (len(paths) - 1), [1] + [0] * (len(paths) - 1), paths, opts)
+    assert cfg.t_pred <= direct * (1 + 1e-12)
+    assert cfg.t_pred == M.evaluate(n, cfg.bytes, cfg.chunks, paths, opts)
+    for i, p in enumerate(paths):
+        if p.kind == M.GPU_STAGED and p.wake >= direct:
+            assert cfg.bytes[i] == 0
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_c28_select_vs_exact_optimum_with_wake(seed):
+    # against the exact optimum over real shares and integer k with the wake in the
+    # path time (oracle/optimize.py evaluates pipelined_time)
+    import random
+    rnd = random.Random(9500 + seed)
+    paths = [with_wake(p, rnd) for p in paths_from(synth.topology(seed, 2 + seed % 3, host=True))]
+    n = rnd.choice([16, 64, 256]) * MiB
+    cfg = M.select(n, paths, M.Options(mode=M.B200, stagger=False))
+    t_opt = O.level_integer_k_b200(float(n), paths, k_max=256)
+    assert t_opt * (1 - 1e-9) <= cfg.t_pred * (1 + 1e-9)
+    assert cfg.t_pred <= t_opt * 1.01, (cfg.t_pred / t_opt, cfg.bytes, cfg.chunks)

@@ -318,3 +318,41 @@ def test_submission_time_survives_the_params_file(tmp_path):
     with mp.Context(world=2, rank=0, model_only=True) as c:
         c.load_params(f)
         assert c.get_submit_time() == 2.5e-6
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_c28_window_parity(seed):
+    # reading C28 in a window: the relay's start delays the window once (library =
+    # oracle for mp_select_window and mp_predict_window); w = 1 is the single message
+    import dataclasses
+    rng = random.Random(300 + seed)
+    tbl = table(0, 1, seed)
+    paths = [M.Path(**t) for t in tbl]
+    paths = [dataclasses.replace(p, wake=rng.uniform(2e-6, 300e-6)) if p.kind == M.GPU_STAGED else p
+             for p in paths]
+    port = M.Port(alpha=2e-6, beta=850e9)
+    h = [rng.uniform(0, 1.5) * p.alpha for p in paths]
+    tau = rng.uniform(0, 10e-6)
+    opts = M.Options(mode=M.B200, slot_bytes=64 * MiB)
+    with mp.Context(world=W, rank=0, model_only=True) as c:
+        c.set_options(mode=M.B200, slot_bytes=64 * MiB)
+        params = [{k: (0.0 if k == "beta2" and math.isinf(t[k]) else t[k]) for k in FIELDS} for t in tbl]
+        for p, q in zip(params, paths):
+            p["wake"] = q.wake
+        c.set_model(0, 1, [(t["kind"], t["via"]) for t in tbl], params, dict(alpha=port.alpha, beta=port.beta))
+        c.set_window_model(0, 1, h, tau)
+        for n in (1 * MiB + 17, 16 * MiB, 64 * MiB, 1024 * MiB):
+            for w in (1, 2, 16, 64):
+                ref = WN.select_window(n, w, paths, h, opts, port, tau=tau)
+                got = c.select_window(0, 1, n, w).as_dict()
+                assert sum(got["bytes"]) == n
+                for a, b in zip(got["bytes"], ref.bytes):
+                    assert abs(a - b) <= 256
+                assert rel(got["t_level"], ref.t_level) < 1e-9
+                if got["bytes"] == ref.bytes:
+                    assert got["chunks"] == ref.chunks and rel(got["t_pred"], ref.t_pred) < 1e-9
+                cfg = c.make_config(ref.bytes, ref.chunks, 0, 1)
+                t = c.predict_window(0, 1, n, w, cfg)
+                assert rel(t, WN.evaluate_window(n, w, ref.bytes, ref.chunks, paths, h, opts, port, tau)) < 1e-9
+                if w == 1:
+                    assert rel(t, c.predict(0, 1, n, cfg) + tau) < 1e-12

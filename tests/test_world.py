@@ -153,3 +153,14 @@ def test_multirank_config3_full_size_bit_exact():
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(3, "full_size", timeout=600)
+
+
+@pytest.mark.gpu
+def test_multirank_relay_wake_calibration():
+    # reading C28: the collective wake probe after Step 1, the env override, and
+    # relayed messages after it (world 3 on one GPU)
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(3, "wake", timeout=400)
