@@ -502,16 +502,25 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
   CKC(cudaMalloc(&src, big));
   CKC(cudaMemset(src, 0x5a, big));
   std::vector<LinkMeas> m(B, LinkMeas{});
-  int st = MP_OK;
-  do {
+  // Ranks sharing one GPU (several processes per device, e.g. under MPS) measure in
+  // turn: measured at once they would share its HBM and every link would be fitted
+  // at a fraction of its rate.  Ranks on distinct GPUs measure concurrently (each
+  // link is used once: rank r puts into r + 1).
+  bool shared_gpu = false;
+  if (c->have_topo)
+    for (int r = 0; r < W; ++r)
+      for (int q = r + 1; q < W; ++q)
+        shared_gpu = shared_gpu || std::memcmp(c->topo.gpu[r].uuid, c->topo.gpu[q].uuid, 16) == 0;
+  auto measure = [&]() -> int {
+    int st = MP_OK;
     std::vector<double> n, t;
     std::vector<Fit> fd, fr, fh1, fh2;
-    if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, 0, window, &n, &t))) break;
-    if ((st = fit_samples(c, n, t, edges, &fd))) break;
+    if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, 0, window, &n, &t))) return st;
+    if ((st = fit_samples(c, n, t, edges, &fd))) return st;
     n.clear();
     t.clear();
-    if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, c->relay_ctas, window, &n, &t))) break;
-    if ((st = fit_samples(c, n, t, edges, &fr))) break;
+    if ((st = sample_link(b, c->peers[succ].heap, src, sz, big, reps, c->relay_ctas, window, &n, &t))) return st;
+    if ((st = fit_samples(c, n, t, edges, &fr))) return st;
     double eps_host = 0, eps_dev = 0, kappa = 1.0;
     if (c->host_path) {
       // the own segment's ring of sender == me is never used for traffic
@@ -524,29 +533,29 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
       const int hr_reps = std::max(3, reps / 2);
       n.clear();
       t.clear();
-      if ((st = sample_link(b, hr, src, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) break;
-      if ((st = fit_samples(c, n, t, edges, &fh1))) break;
+      if ((st = sample_link(b, hr, src, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) return st;
+      if ((st = fit_samples(c, n, t, edges, &fh1))) return st;
       n.clear();
       t.clear();
-      if ((st = sample_link(b, src, hr, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) break;
-      if ((st = fit_samples(c, n, t, edges, &fh2))) break;
-      if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) break;
+      if ((st = sample_link(b, src, hr, hs, hcap, hr_reps, c->relay_ctas, window, &n, &t))) return st;
+      if ((st = fit_samples(c, n, t, edges, &fh2))) return st;
+      if ((st = time_pingpong(b, c->h_probe, true, 500, &eps_host))) return st;
       // κ (reading C25, NEXT f2): both host legs of this GPU alone, then at once
       const uint64_t hk = std::min<uint64_t>(hcap / 2, 32ull << 20);
       if (big >= 2 * hk && hk >= (1u << 20)) {
         double up = 0, down = 0;
         std::vector<double> kn, k1, k2;
         uint8_t *sb = static_cast<uint8_t *>(src);
-        if ((st = time_copy(b, hr, sb, hk, hr_reps, &up, c->relay_ctas))) break;
-        if ((st = time_copy(b, sb + big - hk, hr + hcap / 2, hk, hr_reps, &down, c->relay_ctas))) break;
+        if ((st = time_copy(b, hr, sb, hk, hr_reps, &up, c->relay_ctas))) return st;
+        if ((st = time_copy(b, sb + big - hk, hr + hcap / 2, hk, hr_reps, &down, c->relay_ctas))) return st;
         if ((st = sample_links_duplex(b, hr, sb, sb + big - hk, hr + hcap / 2, {hk}, hr_reps, c->relay_ctas, true,
                                       &kn, &k1, &k2)))
-          break;
+          return st;
         kappa = std::min(1.0, 0.5 * (up / k1[0] + down / k2[0]));
       }
     }
     uint64_t *pf = reinterpret_cast<uint64_t *>(c->peers[succ].ctrl + c->L.probe);
-    if ((st = time_pingpong(b, pf, false, 1000, &eps_dev))) break;
+    if ((st = time_pingpong(b, pf, false, 1000, &eps_dev))) return st;
     for (int j = 0; j < B; ++j) {
       m[j].da = fd[j].alpha;
       m[j].db = fd[j].beta;
@@ -562,7 +571,18 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
       m[j].eps_host = eps_host;
       m[j].kappa = std::max(kappa, 1e-3);
     }
-  } while (false);
+    return st;
+  };
+  int st = MP_OK;
+  if (shared_gpu) {
+    for (int t = 0; t < W; ++t) {
+      if (int e = world_barrier(c)) return e;
+      if (t == me) st = measure();
+    }
+    if (int e = world_barrier(c)) return e;
+  } else {
+    st = measure();
+  }
   cudaStreamSynchronize(b.s);
   cudaFree(src);
   cudaFree(b.flush);
