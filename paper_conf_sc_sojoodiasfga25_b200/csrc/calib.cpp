@@ -622,16 +622,16 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
         mp_path_params prm[MP_MAX_PATHS];
         int np = 0;
         paths[np] = mp_path{MP_PATH_DIRECT, -1};
-        prm[np++] = mp_path_params{S.da, S.db, 0, 0, 0, 1, 0, 1};
+        prm[np++] = mp_path_params{S.da, S.db, 0, 0, 0, 1, 0, 1, 0};
         for (int r = 0; r < W; ++r) {
           if (r == s || r == d) continue;
           const LinkMeas &R = lm[static_cast<size_t>(r) * B + j];
           paths[np] = mp_path{MP_PATH_GPU, r};
-          prm[np++] = mp_path_params{S.ra, S.rb, R.ra, R.rb, std::max(R.eps_dev, 1e-8), 1, 0, 1};
+          prm[np++] = mp_path_params{S.ra, S.rb, R.ra, R.rb, std::max(R.eps_dev, 1e-8), 1, 0, 1, 0};
         }
         if (c->host_path) {
           paths[np] = mp_path{MP_PATH_HOST, -1};
-          prm[np++] = mp_path_params{S.h1a, S.h1b, D.h2a, D.h2b, std::max(D.eps_host, 1e-8), 1, 0, 0};
+          prm[np++] = mp_path_params{S.h1a, S.h1b, D.h2a, D.h2b, std::max(D.eps_host, 1e-8), 1, 0, 0, 0};
         }
         if (keep_c && nold == np)
           for (int i = 0; i < np; ++i) prm[i].c = old[i].c;
@@ -993,8 +993,8 @@ extern "C" int mp_calibrate_wake(mp_ctx *c, uint64_t bytes, int reps) {
   const uint64_t per = std::max<uint64_t>(A, (c->slot_bytes - A) / A * A);
   const uint32_t k = static_cast<uint32_t>((bytes + per - 1) / per);
   std::vector<double> wake(W, 0.0);
-  if (const char *e = std::getenv("MPX_RELAY_WAKE_US")) {
-    for (double &w : wake) w = std::max(0.0, std::atof(e) / 1e6);
+  if (const char *env = std::getenv("MPX_RELAY_WAKE_US")) {
+    for (double &w : wake) w = std::max(0.0, std::atof(env) / 1e6);
   } else {
     if (!c->relay_svc) return cfail(c, MP_ERR_STATE, "mp_calibrate_wake: no relay service");
     const auto quiet = std::chrono::nanoseconds(world_relay_linger_ns(c)) + std::chrono::milliseconds(1);
@@ -1253,14 +1253,14 @@ extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int
   mp_path_params prm[MP_MAX_PATHS];
   int np = 0;
   paths[np] = mp_path{MP_PATH_DIRECT, -1};
-  prm[np++] = mp_path_params{fd.alpha, fd.beta, 0, 0, 0, 1, 0, 2};
+  prm[np++] = mp_path_params{fd.alpha, fd.beta, 0, 0, 0, 1, 0, 2, 0};
   for (int r = 0; r < c->n_loop_relays; ++r) {
     paths[np] = mp_path{MP_PATH_GPU, r};
-    prm[np++] = mp_path_params{f1.alpha, f1.beta, f2.alpha, f2.beta, std::max(eps_dev, 1e-8), 1, 0, 4};
+    prm[np++] = mp_path_params{f1.alpha, f1.beta, f2.alpha, f2.beta, std::max(eps_dev, 1e-8), 1, 0, 4, 0};
   }
   if (c->host_path) {
     paths[np] = mp_path{MP_PATH_HOST, -1};
-    prm[np++] = mp_path_params{fh1.alpha, fh1.beta, fh2.alpha, fh2.beta, std::max(eps_host, 1e-8), 1, 0, 2};
+    prm[np++] = mp_path_params{fh1.alpha, fh1.beta, fh2.alpha, fh2.beta, std::max(eps_host, 1e-8), 1, 0, 2, 0};
   }
   mp_port_params port{fd.alpha, 2.0 * fd.beta};
   if (int s = mp_set_model(c, 0, 0, paths, prm, np, &port)) return s;
