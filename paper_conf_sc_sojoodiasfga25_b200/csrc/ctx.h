@@ -131,6 +131,16 @@ struct mp_ctx {
   std::vector<uint8_t *> hseg;              // [world]: mapped host segment of each receiver
   std::vector<uint64_t> send_seq, recv_seq, relay_q, host_q, done_target;
   std::vector<uint64_t> relay_m;            // [world(relay)]: relayed messages sent via each relay
+  // Ring order across streams: ring positions are assigned in call order, so a staged
+  // send (recv with host consumers) on another stream than the previous user of the
+  // same ring waits for it — a later message's CTAs spinning on slots could otherwise
+  // hold the SMs its predecessor needs.  [3·world]: relay ring r (sender side), host
+  // ring to d (sender side, world + d), host ring from s (receiver side, 2·world + s).
+  struct RingOrder {
+    cudaStream_t stream = nullptr;
+    cudaEvent_t done = nullptr;
+  };
+  std::vector<RingOrder> ring_order;
   mpx::CollState *coll = nullptr;           // created by the first collective
   std::vector<uint64_t> eager_send_seq, eager_recv_seq;  // eager protocol (reading C23)
   uint64_t eager_max = 0;                   // messages of 1..eager_max bytes go eager

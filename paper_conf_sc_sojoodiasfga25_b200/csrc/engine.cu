@@ -1129,6 +1129,21 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
       const SendParams::StagedDesc &d = P.sp[i];
       if (d.kind != 1) continue;
       BellEntry *e = d.bell + d.m % kBellRing;
+      // flow control: the entry is reused only once the relay has taken the doorbell
+      // kBellRing messages back (its kernels acknowledge into this rank's control
+      // block); only more than kBellRing relayed messages in flight through one relay
+      // (many streams) ever wait here
+      if (d.m >= kBellRing) {
+        const uint64_t *ack = reinterpret_cast<const uint64_t *>(P.my_ctrl + P.L.bell_ack) + d.relay * 16;
+        const uint64_t need = d.m + 1 - kBellRing, t0 = globaltimer();
+        while (ld_acquire_sys(ack) < need) {
+          if (globaltimer() - t0 > P.timeout_ns) {
+            atomicExch(P.err, DERR_TIMEOUT);
+            break;
+          }
+          __nanosleep(256);
+        }
+      }
       // co-alignment of source and target (mod 16 is the same in every process's
       // mapping: mapped bases are >= 256-B aligned) lets the relay stream its lanes
       const uint64_t region = ld_volatile(&cts->d);
@@ -1351,6 +1366,10 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kern
   __syncthreads();
   uint64_t m = P.m0, q0 = P.q0, k = P.k;
   uint32_t aligned = P.aligned;
+  // doorbell m is taken (the host thread read it for this launch): the sender may reuse
+  // its ring entry kBellRing messages later (flow control in send_gate_kernel)
+  uint64_t *ack = reinterpret_cast<uint64_t *>(P.sender_ctrl + P.L.bell_ack) + P.me * 16;
+  if (blockIdx.x == 0 && threadIdx.x == 0) st_release_sys(ack, m + 1);
   for (;;) {
     if (!relay_message<D>(P, q0, k, aligned, &s_abort, dyn_smem)) break;
     // the sender's next message: CTA 0 looks for its doorbell for up to linger_ns and
@@ -1374,6 +1393,7 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kern
           nq = ld_volatile(&e->q0);
           nk = ld_volatile(&e->k);
           flags = (g >> 32) & 1u;
+          st_release_sys(ack, m + 2);  // doorbell m + 1 taken
         }
       }
       dec[1] = nq;

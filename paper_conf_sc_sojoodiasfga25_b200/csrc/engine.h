@@ -189,6 +189,7 @@ struct CtrlLayout {
   uint64_t eager_cnt = 0;              // [world(sender)][kEagerSlots] u32: CTAs done copying out — on the receiver
   uint64_t relay_dec = 0;              // [world(sender)][kBellRing][4] u64: a relay kernel's next-message decisions
   uint64_t relay_exit = 0;             // [world(sender)] u32, 128-B padded: relay CTAs that have left
+  uint64_t bell_ack = 0;               // [world(relay)] u64, 128-B padded: doorbells the relay has taken — on the sender
   uint64_t total = 0;
 };
 

@@ -96,6 +96,7 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.eager_cnt = take(static_cast<uint64_t>(world) * kEagerSlots * 4);
   L.relay_dec = take(static_cast<uint64_t>(world) * kBellRing * 32);
   L.relay_exit = take(static_cast<uint64_t>(world) * 128);
+  L.bell_ack = take(static_cast<uint64_t>(world) * 128);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
@@ -258,6 +259,7 @@ int world_init(mp_ctx *c) {
   c->recv_seq.assign(W, 0);
   c->relay_q.assign(W, 0);
   c->relay_m.assign(W, 0);
+  c->ring_order.assign(3 * static_cast<size_t>(W), mp_ctx::RingOrder{});
   c->host_q.assign(W, 0);
   c->done_target.assign(W, 0);
   c->eager_send_seq.assign(W, 0);
@@ -423,6 +425,9 @@ int world_finalize(mp_ctx *c) {
   world_stop_relay(c);
   cudaDeviceSynchronize();  // every stream this process enqueued on (not a list of handles
                             // the caller may have destroyed since)
+  for (mp_ctx::RingOrder &o : c->ring_order)
+    if (o.done) cudaEventDestroy(o.done);
+  c->ring_order.clear();
   if (c->allgather) st = barrier(c);
   for (int r = 0; r < static_cast<int>(c->peers.size()); ++r) {
     if (r == c->rank) continue;
@@ -482,6 +487,24 @@ static int eager_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, vo
     return wfail(c, MP_ERR_CUDA, std::string("eager recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   c->launches += 1;
   c->eager_recv_seq[src] += 1;
+  return MP_OK;
+}
+
+// Ring order across streams (ctx.h: ring_order): wait for the ring's previous user when
+// it ran on another stream; after the launch, record this one.
+static int ring_wait(mp_ctx *c, size_t ring, cudaStream_t s) {
+#ifdef MPX_NO_RING_ORDER  // (design experiment: the engine without it)
+  return MP_OK;
+#endif
+  mp_ctx::RingOrder &o = c->ring_order[ring];
+  if (o.done && o.stream != s) CKW(cudaStreamWaitEvent(s, o.done, 0));
+  return MP_OK;
+}
+static int ring_mark(mp_ctx *c, size_t ring, cudaStream_t s) {
+  mp_ctx::RingOrder &o = c->ring_order[ring];
+  if (!o.done) CKW(cudaEventCreateWithFlags(&o.done, cudaEventDisableTiming));
+  CKW(cudaEventRecord(o.done, s));
+  o.stream = s;
   return MP_OK;
 }
 
@@ -552,8 +575,14 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   }
   P.npaths = np;
   P.nblocks = next;
+  const cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  const size_t W = static_cast<size_t>(c->world);
+  for (auto &a : advance)
+    if (int e = ring_wait(c, a.first < 0 ? W + static_cast<size_t>(dst) : static_cast<size_t>(a.first), cs)) return e;
   if (int e = launch_send(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  for (auto &a : advance)
+    if (int e = ring_mark(c, a.first < 0 ? W + static_cast<size_t>(dst) : static_cast<size_t>(a.first), cs)) return e;
   c->launches += 2;  // rendezvous gate + bulk send kernel
   c->send_seq[dst] += 1;
   for (auto &a : advance) {
@@ -616,8 +645,14 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   P.bulk_stages = bulk_stages_for(bytes);
   if (c->host_path) P.host = host_ring(c, src, c->rank);
   P.nblocks = 1 + P.g_host;
+  const size_t ring = 2 * static_cast<size_t>(c->world) + static_cast<size_t>(src);
+  const cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  if (c->host_path)
+    if (int e = ring_wait(c, ring, cs)) return e;
   if (int e = launch_recv(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  if (c->host_path)
+    if (int e = ring_mark(c, ring, cs)) return e;
   c->launches += 1;
   c->recv_seq[src] += 1;
   c->done_target[src] += bytes;

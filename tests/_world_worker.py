@@ -704,6 +704,54 @@ def scenario_wake(rank, world):
     c.close()
 
 
+def scenario_bell_flow(rank, world):
+    """Many relayed messages in flight: rank 0 sends 56 relayed messages to rank 1 and 56
+    to rank 3, every one through relay rank 2 on its own stream (112 streams), receivers
+    posting on 56 streams each, the later messages' streams delayed least.  More doorbells than the relay's
+    ring holds (64: the gates' acknowledgement wait), and send kernels that become
+    resident out of ring order (the cross-stream ring order).  Every message bit-exact."""
+    from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    torch.cuda.set_device(0)
+    n, M = 1 * MiB + 4099, 56
+    gen = torch.Generator(device="cuda").manual_seed(11)
+    src = torch.randint(0, 256, (2 * M, n), dtype=torch.uint8, device="cuda", generator=gen)
+    torch.cuda.synchronize()
+    c = mdist.context_from_dist(device=0, heap_bytes=M * (n + 4096) + 8 * MiB, timeout_s=60.0, calibrate=False)
+    streams = [torch.cuda.Stream() for _ in range(2 * M)]
+    peers = (1, 3)
+    if rank == 0:
+        for i in range(2 * M):
+            d = peers[i % 2]
+            ps = c.paths(0, d)
+            idx = next(j for j, (k, via) in enumerate(ps) if k == mp.MP_PATH_GPU and via == 2)
+            nb = [0] * len(ps)
+            nb[idx] = n
+            ks = [1] + [0] * (len(ps) - 1)
+            ks[idx] = 1
+            c.send(src[i], n, d, tag=i, cfg=c.make_config(nb, ks, 0, d), stream=streams[i])
+        torch.cuda.synchronize()
+    elif rank in peers:
+        bufs = [c.alloc(n) for _ in range(M)]
+        mine = [i for i in range(2 * M) if peers[i % 2] == rank]
+        # posted in order (matching is FIFO per pair), but each stream first sleeps the
+        # longer the earlier its message: the later messages' clear-to-sends arrive first,
+        # so their gates fire (and their send kernels become resident) before the earlier ones'
+        for j in range(M):
+            with torch.cuda.stream(streams[j]):
+                torch.cuda._sleep(40000 * (M - j))
+            c.recv(bufs[j], n, 0, tag=mine[j], stream=streams[j])
+        torch.cuda.synchronize()
+        c.sync()  # sticky device errors (timeout, mismatch) first
+        for j, i in enumerate(mine):
+            assert torch.equal(mp.as_tensor(bufs[j], n), src[i]), f"message {i}"
+        for b in bufs:
+            c.free(b)
+    dist.barrier()
+    c.sync()
+    c.close()
+
+
 def main():
     rank, world, port, scen = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3]), sys.argv[4]
     import faulthandler
@@ -715,7 +763,8 @@ def main():
          "faults": scenario_faults, "register": scenario_register, "coll": scenario_coll,
          "eager": scenario_eager, "devsync": scenario_devsync,
          "bench_plan": scenario_bench_plan, "relay_burst": scenario_relay_burst,
-         "full_size": scenario_full_size, "wake": scenario_wake}[scen](rank, world)
+         "full_size": scenario_full_size, "wake": scenario_wake,
+         "bell_flow": scenario_bell_flow}[scen](rank, world)
         dist.barrier()
         dist.destroy_process_group()
     except BaseException:

@@ -45,8 +45,8 @@ def run_world(world, scenario, timeout, env=None):
         for p in procs:
             if p.poll() is None:
                 p.kill()
-    for r, (p, out) in enumerate(zip(procs, outs)):
-        assert p.returncode == 0, f"rank {r} failed:\n{out[:3000]}\n...\n{out[-3000:]}"
+    bad = [(r, p.returncode, out) for r, (p, out) in enumerate(zip(procs, outs)) if p.returncode != 0]
+    assert not bad, "\n".join(f"rank {r} failed (rc {rc}):\n{out[:2000]}\n...\n{out[-2000:]}" for r, rc, out in bad)
 
 
 @pytest.mark.parametrize("world", [2, 3])
@@ -164,3 +164,14 @@ def test_multirank_relay_wake_calibration():
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     run_world(3, "wake", timeout=400)
+
+
+@pytest.mark.gpu
+def test_multirank_doorbell_flow_control():
+    # 112 relayed messages in flight through one relay (two receivers, 112 streams,
+    # receives posted last-first): doorbell flow control and cross-stream ring order
+    pytest.importorskip("torch")
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    run_world(4, "bell_flow", timeout=500)
