@@ -453,7 +453,9 @@ int mp_deregister(mp_ctx *ctx, int id);
  * given (validated: Σ bytes == n, 1 <= k <= max(1, ⌊b/A⌋), chunk <= slot_bytes,
  * paths available).  Stream-ordered: the send kernel waits on the device for the
  * matching mp_recv.  In single-GPU loopback (dst == rank == 0) the send is
- * recorded and the fused transfer is launched by the matching mp_recv. */
+ * recorded and the fused transfer is launched by the matching mp_recv.  Staged paths
+ * share rings: a send whose relay or host ring was last used by a send on another
+ * stream waits for that send first (ring positions follow call order). */
 int mp_send(mp_ctx *ctx, const void *buf, uint64_t bytes, int dst, int tag,
             const mp_config *cfg, void *stream);
 
