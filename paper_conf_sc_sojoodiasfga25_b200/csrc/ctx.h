@@ -134,8 +134,9 @@ struct mp_ctx {
   // Ring order across streams: ring positions are assigned in call order, so a staged
   // send (recv with host consumers) on another stream than the previous user of the
   // same ring waits for it — a later message's CTAs spinning on slots could otherwise
-  // hold the SMs its predecessor needs.  [3·world]: relay ring r (sender side), host
-  // ring to d (sender side, world + d), host ring from s (receiver side, 2·world + s).
+  // hold the SMs its predecessor needs.  [5·world]: relay ring r (sender side), host
+  // ring to d (sender side, world + d), host ring from s (receiver side, 2·world + s),
+  // eager slots to d (3·world + d) and from s (4·world + s).
   struct RingOrder {
     cudaStream_t stream = nullptr;
     cudaEvent_t done = nullptr;

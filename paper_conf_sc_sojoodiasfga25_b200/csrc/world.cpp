@@ -259,7 +259,7 @@ int world_init(mp_ctx *c) {
   c->recv_seq.assign(W, 0);
   c->relay_q.assign(W, 0);
   c->relay_m.assign(W, 0);
-  c->ring_order.assign(3 * static_cast<size_t>(W), mp_ctx::RingOrder{});
+  c->ring_order.assign(5 * static_cast<size_t>(W), mp_ctx::RingOrder{});
   c->host_q.assign(W, 0);
   c->done_target.assign(W, 0);
   c->eager_send_seq.assign(W, 0);
@@ -468,28 +468,6 @@ static EagerParams eager_params(mp_ctx *c, int sender, int receiver, uint64_t se
   return P;
 }
 
-static int eager_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, void *stream) {
-  EagerParams P = eager_params(c, c->rank, dst, c->eager_send_seq[dst], bytes, tag);
-  P.peer = static_cast<uint32_t>(dst);
-  P.src = static_cast<const uint8_t *>(buf);
-  if (int e = launch_eager_send(P, stream))
-    return wfail(c, MP_ERR_CUDA, std::string("eager send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
-  c->launches += 1;
-  c->eager_send_seq[dst] += 1;
-  return MP_OK;
-}
-
-static int eager_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
-  EagerParams P = eager_params(c, src, c->rank, c->eager_recv_seq[src], bytes, tag);
-  P.peer = static_cast<uint32_t>(src);
-  P.dst = static_cast<uint8_t *>(buf);
-  if (int e = launch_eager_recv(P, stream))
-    return wfail(c, MP_ERR_CUDA, std::string("eager recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
-  c->launches += 1;
-  c->eager_recv_seq[src] += 1;
-  return MP_OK;
-}
-
 // Ring order across streams (ctx.h: ring_order): wait for the ring's previous user when
 // it ran on another stream; after the launch, record this one.
 static int ring_wait(mp_ctx *c, size_t ring, cudaStream_t s) {
@@ -505,6 +483,36 @@ static int ring_mark(mp_ctx *c, size_t ring, cudaStream_t s) {
   if (!o.done) CKW(cudaEventCreateWithFlags(&o.done, cudaEventDisableTiming));
   CKW(cudaEventRecord(o.done, s));
   o.stream = s;
+  return MP_OK;
+}
+
+static int eager_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, void *stream) {
+  EagerParams P = eager_params(c, c->rank, dst, c->eager_send_seq[dst], bytes, tag);
+  P.peer = static_cast<uint32_t>(dst);
+  P.src = static_cast<const uint8_t *>(buf);
+  // the eager slots are a ring too (a send waits for its slot's previous message to be
+  // copied out): same cross-stream order, per destination
+  const size_t ring = 3 * static_cast<size_t>(c->world) + static_cast<size_t>(dst);
+  if (int e = ring_wait(c, ring, static_cast<cudaStream_t>(stream))) return e;
+  if (int e = launch_eager_send(P, stream))
+    return wfail(c, MP_ERR_CUDA, std::string("eager send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  if (int e = ring_mark(c, ring, static_cast<cudaStream_t>(stream))) return e;
+  c->launches += 1;
+  c->eager_send_seq[dst] += 1;
+  return MP_OK;
+}
+
+static int eager_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream) {
+  EagerParams P = eager_params(c, src, c->rank, c->eager_recv_seq[src], bytes, tag);
+  P.peer = static_cast<uint32_t>(src);
+  P.dst = static_cast<uint8_t *>(buf);
+  const size_t ring = 4 * static_cast<size_t>(c->world) + static_cast<size_t>(src);
+  if (int e = ring_wait(c, ring, static_cast<cudaStream_t>(stream))) return e;
+  if (int e = launch_eager_recv(P, stream))
+    return wfail(c, MP_ERR_CUDA, std::string("eager recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  if (int e = ring_mark(c, ring, static_cast<cudaStream_t>(stream))) return e;
+  c->launches += 1;
+  c->eager_recv_seq[src] += 1;
   return MP_OK;
 }
 
