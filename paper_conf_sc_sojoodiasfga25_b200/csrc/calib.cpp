@@ -96,40 +96,29 @@ int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double
 
 // OMB-style timing (reading C21): `W` back-to-back copies of n bytes between the
 // same buffers (no flush — a window of repeated sends), median over
-// `reps` windows; returns seconds per message.  The window is captured once in a CUDA
-// graph and replayed, so it is timed at GPU speed: enqueued from the host, a small
-// message costs 2-3 µs of host submission per call, more than its 1-2 µs on the GPU
-// (DESIGN §6), and the bands would fit the host instead of the link.  (Thread-local
-// capture: the relay service thread keeps launching on its own streams meanwhile.)
+// `reps` windows; returns seconds per message.  Each window is enqueued behind a spin
+// kernel that outlasts the host's enqueue (~3 µs per launch), so its copies run back
+// to back at GPU speed — launched from a stream, as a caller's messages are.  (Round 2
+// first replayed the window from a CUDA graph: also GPU-speed, but a graph launches
+// each kernel ~0.8 µs sooner than a stream does, and the bands then over-predicted
+// stream-launched windows by 16-33 % at 4-16 MiB.)  Enqueued without the spin, a small
+// message would be timed at the host's 2-3 µs per call instead (C27 models
+// that part separately).
 int time_window(Bench &b, void *dst, const void *src, uint64_t n, int reps, int W, double *out, int ctas = 0) {
   mp_ctx *c = b.c;
-  cudaGraph_t g = nullptr;
-  cudaGraphExec_t ge = nullptr;
-  CKC(cudaStreamBeginCapture(b.s, cudaStreamCaptureModeThreadLocal));
-  int st = MP_OK;
-  for (int w = 0; w < W && st == MP_OK; ++w) st = launch_direct_copy(c, dst, src, n, b.s, ctas);
-  const cudaError_t ce = cudaStreamEndCapture(b.s, &g);
-  if (st) {
-    if (g) cudaGraphDestroy(g);
-    return st;
-  }
-  CKC(ce);
-  const cudaError_t ie = cudaGraphInstantiate(&ge, g, 0);
-  cudaGraphDestroy(g);
-  CKC(ie);
   std::vector<double> ts;
-  for (int r = 0; r < reps + 1 && st == MP_OK; ++r) {
-    cudaError_t e = cudaEventRecord(b.e0, b.s);
-    if (e == cudaSuccess) e = cudaGraphLaunch(ge, b.s);
-    if (e == cudaSuccess) e = cudaEventRecord(b.e1, b.s);
-    if (e == cudaSuccess) e = cudaEventSynchronize(b.e1);
+  const uint64_t spin_ns = 50000ull + 6000ull * static_cast<uint64_t>(W);
+  for (int r = 0; r < reps + 1; ++r) {
+    if (launch_spin(spin_ns, b.s) != 0) return cfail(c, MP_ERR_CUDA, "window spin launch");
+    CKC(cudaEventRecord(b.e0, b.s));
+    for (int w = 0; w < W; ++w)
+      if (int st = launch_direct_copy(c, dst, src, n, b.s, ctas)) return st;
+    CKC(cudaEventRecord(b.e1, b.s));
+    CKC(cudaEventSynchronize(b.e1));
     float ms = 0;
-    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, b.e0, b.e1);
-    if (e != cudaSuccess) st = cfail(c, MP_ERR_CUDA, std::string("window graph: ") + cudaGetErrorString(e));
+    CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
     if (r > 0) ts.push_back(ms * 1e-3 / W);  // first window is a warm-up
   }
-  cudaGraphExecDestroy(ge);
-  if (st) return st;
   *out = median(ts);
   return MP_OK;
 }
@@ -472,6 +461,18 @@ int aggregate_ports(mp_ctx *c, uint64_t n, int reps, double *egress, double *ing
   return MP_OK;
 }
 
+// Sizes the band fits sample (C20/C21): powers of two from 4 KiB to 1 GiB, plus 1.5×
+// powers of two from 6 to 96 MiB, where the loopback working set crosses the 126 MB L2
+// and the per-message rate is furthest from a line.
+std::vector<uint64_t> band_sizes() {
+  std::vector<uint64_t> sizes;
+  for (uint64_t s = 4096; s <= (1024ull << 20); s <<= 1) {
+    sizes.push_back(s);
+    if (s >= (4ull << 20) && s <= (64ull << 20)) sizes.push_back(s + s / 2);
+  }
+  return sizes;
+}
+
 // edges = {0}: the plain Step-1 fit (flushed single copies); more edges: one
 // parameter set per size band (reading C20), window-timed (reading C21).
 int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std::vector<double> &edges,
@@ -658,8 +659,7 @@ int calibrate_loop_bands(mp_ctx *c, const std::vector<double> &edges, int reps) 
   mp_path_params base[MP_MAX_PATHS];
   int np = 0;
   if (int s = mp_get_model(c, 0, 0, paths, base, &np, nullptr)) return s;
-  std::vector<uint64_t> sizes;
-  for (uint64_t s = 4096; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
+  const std::vector<uint64_t> sizes = band_sizes();
   const uint64_t big = sizes.back();
   const uint64_t ring_cap = static_cast<uint64_t>(c->slots) * c->slot_bytes;
   Bench b;
@@ -756,12 +756,12 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
       edges.push_back(static_cast<double>(edges_in[j]));
     }
   } else {
-    for (uint64_t e : {0ull, 256ull << 10, 4ull << 20, 16ull << 20, 32ull << 20, 64ull << 20, 128ull << 20}) edges.push_back(static_cast<double>(e));
+    for (uint64_t e : {0ull, 256ull << 10, 4ull << 20, 8ull << 20, 16ull << 20, 32ull << 20, 48ull << 20, 64ull << 20,
+                       128ull << 20})
+      edges.push_back(static_cast<double>(e));
   }
   if (c->world != 1) {
-    std::vector<uint64_t> sizes;
-    for (uint64_t s = 4096; s <= (1024ull << 20); s <<= 1) sizes.push_back(s);
-    if (int s = calibrate_world(c, sizes, reps, edges, true)) return s;
+    if (int s = calibrate_world(c, band_sizes(), reps, edges, true)) return s;
     int32_t derr = 0;
     CKC(cudaMemcpy(&derr, c->d_err, sizeof(derr), cudaMemcpyDeviceToHost));
     if (derr) return cfail(c, MP_ERR_TIMEOUT, "calibration probe timed out");

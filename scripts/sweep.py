@@ -32,16 +32,18 @@ MiB = 1 << 20
 def measure(ctx, dst, src, n, cfg, reps, stream):
     """OMB-style (reading C21): a window of W back-to-back transfers of
     the config, seconds per message = window time / W, median over `reps` windows."""
-    W = 8 if n <= 64 * MiB else 2
+    # windows as Step 1 times its bands (C21): long enough that the events and the first
+    # launch around a window (~2-3 µs) stay a small part of it
+    W = 64 if n <= 4 * MiB else 16 if n <= 64 * MiB else 2
     ts = []
     for r in range(reps + 1):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
-        # a ~100 µs spin kernel first, so that the whole window is enqueued before the
+        # a ~1 ms spin kernel first, so that the whole window is enqueued before the
         # GPU reaches it: the window is then timed at GPU speed, not at the Python
         # loop's (a back-to-back 16 MiB message takes ~4 µs under PDL)
         with torch.cuda.stream(stream):
-            torch.cuda._sleep(200_000)
+            torch.cuda._sleep(2_000_000)
         e0.record(stream)
         for _ in range(W):
             ctx.xfer(dst, src, n, cfg, stream)

@@ -302,21 +302,20 @@ def test_calibrate_bands_installs_bands_and_cuts_small_size_error():
     s = torch.cuda.Stream()
 
     def window_time(n, cfg, w=64, reps=7):
-        # the window is captured in a CUDA graph so that it is GPU-bound (Step 1 times
-        # its band windows the same way, reading C21): enqueued from Python a small
-        # message costs more host time than its ~1-2 µs on the GPU
+        # the window is enqueued behind a ~2 ms spin kernel so that it runs GPU-bound
+        # from a stream (Step 1 times its band windows the same way, reading C21):
+        # enqueued from Python without it, a small message costs more host time than its
+        # ~1-2 µs on the GPU
         assert sum(cfg.as_dict()["bytes"][1:]) == 0, "B200 mode picks direct-only here"
-        g = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(g, stream=s):
-            for _ in range(w):
-                c.xfer(dst, src, n, cfg, torch.cuda.current_stream())
         ts = []
         for _ in range(reps + 1):
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             with torch.cuda.stream(s):
+                torch.cuda._sleep(4_000_000)
                 e0.record(s)
-                g.replay()
+                for _ in range(w):
+                    c.xfer(dst, src, n, cfg, s)
                 e1.record(s)
             e1.synchronize()
             ts.append(e0.elapsed_time(e1) * 1e-3 / w)
