@@ -1009,57 +1009,50 @@ extern "C" int mp_calibrate_wake(mp_ctx *c, uint64_t bytes, int reps) {
     if (int e = world_allgather(c, &no_room, rooms.data(), sizeof(no_room))) return e;
     bool skip = false;
     for (int32_t v : rooms) skip = skip || v;
-    int rc = MP_OK;
+    // rc: a local failure — this rank stops probing but keeps joining every barrier, so
+    // its peers are not stranded; brc: a failed barrier (the bootstrap is gone) — stop.
+    int rc = MP_OK, brc = MP_OK;
     double mine = 0.0;  // this rank's result as the receiver of relay (me − 2) mod W
-    do {
-      if (skip) break;
+    if (!skip) {
       if (cudaMalloc(&src, bytes) != cudaSuccess || cudaMemset(src, 0x3c, bytes) != cudaSuccess ||
-          cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) {
+          cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess)
         rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: buffers");
-        break;
-      }
       for (cudaEvent_t &e : ev)
-        if (cudaEventCreate(&e) != cudaSuccess) rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: events");
-      if (rc) break;
-      for (int r = 0; r < W && !rc; ++r) {
+        if (!rc && cudaEventCreate(&e) != cudaSuccess) rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: events");
+      for (int r = 0; r < W && !brc; ++r) {
         const int s = (r + 1) % W, d = (r + 2) % W;
+        const bool end = me == s || me == d;
         mp_config cfg{};
         mp_path_params prm[MP_MAX_PATHS];
         int np = 0, idx = -1;
-        if ((me == s || me == d) && (rc = mp_get_model(c, s, d, cfg.path, prm, &np, nullptr))) break;
+        if (end && !rc) rc = mp_get_model(c, s, d, cfg.path, prm, &np, nullptr);
         for (int i = 0; i < np; ++i)
           if (cfg.path[i].kind == MP_PATH_GPU && cfg.path[i].via == r) idx = i;
-        if ((me == s || me == d) && idx < 0) {
+        if (end && !rc && idx < 0)
           rc = cfail(c, MP_ERR_TOPOLOGY, "mp_calibrate_wake: pair has no path via relay " + std::to_string(r));
-          break;
-        }
-        if (me == s) {
+        if (me == s && !rc) {
           cfg.npaths = np;
           cfg.bytes[idx] = bytes;
           cfg.chunks[0] = 1;
           cfg.chunks[idx] = k;
         }
         std::vector<double> diffs;
-        for (int i = 0; i < reps && !rc; ++i) {
-          if ((rc = world_barrier(c))) break;
+        for (int i = 0; i < reps && !brc; ++i) {
+          if ((brc = world_barrier(c))) break;
           std::this_thread::sleep_for(quiet);
           if (me == s)
             for (int j = 0; j < 2 && !rc; ++j) rc = mp_send(c, src, bytes, d, -1000 - j, &cfg, st);
-          if (rc) break;
-          if ((rc = world_barrier(c))) break;
-          if (me == d) {
+          if ((brc = world_barrier(c))) break;
+          if (me == d && !rc) {
             cudaEventRecord(ev[0], st);
             rc = mp_recv(c, rbuf, bytes, s, -1000, st);
             cudaEventRecord(ev[1], st);
             if (!rc) rc = mp_recv(c, rbuf, bytes, s, -1001, st);
             cudaEventRecord(ev[2], st);
           }
-          if (rc) break;
-          if (cudaStreamSynchronize(st) != cudaSuccess) {
+          if (end && !rc && cudaStreamSynchronize(st) != cudaSuccess)
             rc = cfail(c, MP_ERR_CUDA, "mp_calibrate_wake: stream");
-            break;
-          }
-          if (me == d) {
+          if (me == d && !rc) {
             float t1 = 0, t2 = 0;
             cudaEventElapsedTime(&t1, ev[0], ev[1]);
             cudaEventElapsedTime(&t2, ev[1], ev[2]);
@@ -1080,13 +1073,14 @@ extern "C" int mp_calibrate_wake(mp_ctx *c, uint64_t bytes, int reps) {
           mine = delta > 1e-6 ? std::max(0.0, T - k * s2 + delta) : 0.0;
         }
       }
-    } while (false);
+    }
     if (st) cudaStreamSynchronize(st);
     for (cudaEvent_t e : ev)
       if (e) cudaEventDestroy(e);
     if (st) cudaStreamDestroy(st);
     if (src) cudaFree(src);
     if (rbuf) mp_free(c, rbuf);
+    if (brc) return brc;
     int32_t ok = rc ? 1 : 0;
     std::vector<int32_t> all_ok(W);
     if (int e = world_allgather(c, &ok, all_ok.data(), sizeof(ok))) return e;
