@@ -599,7 +599,13 @@ int calibrate_world(mp_ctx *c, std::vector<uint64_t> sizes, int reps, const std:
   {  // C14's shared port as aggregates (egress, ingress); heaps are still empty
     double eg = 0.0, in = 0.0;
     const uint64_t n_each = std::min<uint64_t>(cap, 256ull << 20);
-    if (int e = aggregate_ports(c, n_each, std::max(3, reps / 2), &eg, &in)) return e;
+    const int ae = aggregate_ports(c, n_each, std::max(3, reps / 2), &eg, &in);
+    int32_t aok = ae ? 1 : 0;  // agree before the next collective: a local failure must not strand the peers
+    std::vector<int32_t> all_aok(W);
+    if (int s = world_allgather(c, &aok, all_aok.data(), sizeof(aok))) return s;
+    if (ae) return ae;
+    for (int32_t v : all_aok)
+      if (v) return cfail(c, MP_ERR_STATE, "port calibration failed on another rank");
     for (int j = 0; j < B; ++j) {
       m[j].egress_b = eg;
       m[j].ingress_b = in;
