@@ -45,6 +45,9 @@ def run_world(world, scenario, timeout, env=None):
         for p in procs:
             if p.poll() is None:
                 p.kill()
+    if os.environ.get("MPX_TEST_SHOW_OUTPUT") == "1":  # e.g. each rank's compute-sanitizer summary
+        for r, out in enumerate(outs):
+            print(f"--- rank {r} output tail\n{out[-1500:]}")
     bad = [(r, p.returncode, out) for r, (p, out) in enumerate(zip(procs, outs)) if p.returncode != 0]
     assert not bad, "\n".join(f"rank {r} failed (rc {rc}):\n{out[:2000]}\n...\n{out[-2000:]}" for r, rc, out in bad)
 
