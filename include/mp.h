@@ -502,7 +502,7 @@ int mp_calibrate(mp_ctx *ctx, const uint64_t *sizes, int nsizes, int reps);
  * j >= 1 is installed with mp_set_model_band(edges[j]).  ε and, when the pair already
  * has a model, the φ multipliers c are kept (run mp_calibrate first).
  * edges[nedges]: band lower edges in bytes, edges[0] == 0, strictly increasing; NULL
- * = {0, 256 KiB, 4, 8, 16, 32, 48, 64, 128 MiB}; sampled at powers of two from 4 KiB to
+ * = {0, 64 KiB, 256 KiB, 4, 8, 16, 32, 48, 64, 128 MiB}; sampled at powers of two from 4 KiB to
  * 1 GiB plus 6, 12, 24, 48, 96 MiB.  reps: windows per size (median).
  * Collective when world > 1 (same rules as mp_calibrate).
  * Errors: MP_ERR_STATE (model-only), MP_ERR_INVALID (bad edges), MP_ERR_CUDA. */

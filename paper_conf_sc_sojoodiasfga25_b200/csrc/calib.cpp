@@ -107,14 +107,53 @@ int time_copy(Bench &b, void *dst, const void *src, uint64_t n, int reps, double
 int time_window(Bench &b, void *dst, const void *src, uint64_t n, int reps, int W, double *out, int ctas = 0) {
   mp_ctx *c = b.c;
   std::vector<double> ts;
-  const uint64_t spin_ns = 50000ull + 6000ull * static_cast<uint64_t>(W);
-  for (int r = 0; r < reps + 1; ++r) {
+#ifdef MPX_GRAPH_WINDOWS  // (design experiment: the window replayed from a CUDA graph)
+  {
+    cudaGraph_t g = nullptr;
+    cudaGraphExec_t ge = nullptr;
+    CKC(cudaStreamBeginCapture(b.s, cudaStreamCaptureModeThreadLocal));
+    int st = MP_OK;
+    for (int w = 0; w < W && st == MP_OK; ++w) st = launch_direct_copy(c, dst, src, n, b.s, ctas);
+    const cudaError_t ce = cudaStreamEndCapture(b.s, &g);
+    if (st) {
+      if (g) cudaGraphDestroy(g);
+      return st;
+    }
+    CKC(ce);
+    const cudaError_t ie = cudaGraphInstantiate(&ge, g, 0);
+    cudaGraphDestroy(g);
+    CKC(ie);
+    for (int r = 0; r < reps + 1; ++r) {
+      CKC(cudaEventRecord(b.e0, b.s));
+      CKC(cudaGraphLaunch(ge, b.s));
+      CKC(cudaEventRecord(b.e1, b.s));
+      CKC(cudaEventSynchronize(b.e1));
+      float ms = 0;
+      CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
+      if (r > 0) ts.push_back(ms * 1e-3 / W);
+    }
+    cudaGraphExecDestroy(ge);
+    *out = median(ts);
+    return MP_OK;
+  }
+#endif
+  uint64_t spin_ns = 100000ull + 10000ull * static_cast<uint64_t>(W);
+  for (int r = 0, redo = 0; r < reps + 1; ++r) {
     if (launch_spin(spin_ns, b.s) != 0) return cfail(c, MP_ERR_CUDA, "window spin launch");
     CKC(cudaEventRecord(b.e0, b.s));
     for (int w = 0; w < W; ++w)
       if (int st = launch_direct_copy(c, dst, src, n, b.s, ctas)) return st;
     CKC(cudaEventRecord(b.e1, b.s));
+    // the spin must still be running once the whole window is enqueued (else the GPU
+    // waited for the host inside the window): if not, redo with a longer spin
+    const bool covered = cudaEventQuery(b.e0) == cudaErrorNotReady;
     CKC(cudaEventSynchronize(b.e1));
+    if (!covered && redo < 4) {
+      spin_ns *= 2;
+      ++redo;
+      --r;
+      continue;
+    }
     float ms = 0;
     CKC(cudaEventElapsedTime(&ms, b.e0, b.e1));
     if (r > 0) ts.push_back(ms * 1e-3 / W);  // first window is a warm-up
@@ -762,8 +801,8 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
       edges.push_back(static_cast<double>(edges_in[j]));
     }
   } else {
-    for (uint64_t e : {0ull, 256ull << 10, 4ull << 20, 8ull << 20, 16ull << 20, 32ull << 20, 48ull << 20, 64ull << 20,
-                       128ull << 20})
+    for (uint64_t e : {0ull, 64ull << 10, 256ull << 10, 4ull << 20, 8ull << 20, 16ull << 20, 32ull << 20, 48ull << 20,
+                       64ull << 20, 128ull << 20})
       edges.push_back(static_cast<double>(e));
   }
   if (c->world != 1) {
