@@ -100,7 +100,8 @@ class mp_coll_plan(C.Structure):
 
 
 class mp_gpu_info(C.Structure):
-    _fields_ = [("uuid", C.c_char * 16)] + [(n, C.c_int32) for n in (
+    # raw bytes (c_ubyte): a c_char array would read back truncated at its first 0x00
+    _fields_ = [("uuid", C.c_ubyte * 16)] + [(n, C.c_int32) for n in (
         "device", "pci_domain", "pci_bus", "pci_device", "numa_node", "pcie_gen", "pcie_width", "pcie_gen_cur",
         "nvlinks", "sms", "reserved")]
 
@@ -564,7 +565,8 @@ class Context:
         w = int(topo["world"])
         t.world = w
         for r, g in enumerate(topo.get("gpus", [])[:w]):
-            t.gpu[r].uuid = bytes.fromhex(g.get("uuid", "00" * 16))[:16]
+            raw = bytes.fromhex(g.get("uuid", "00" * 16))[:16].ljust(16, b"\0")
+            C.memmove(t.gpu[r].uuid, raw, 16)
             for k in ("device", "numa_node", "pcie_gen", "pcie_width", "pcie_gen_cur", "nvlinks", "sms"):
                 setattr(t.gpu[r], k, int(g.get(k, 0)))
         for key in ("peer_access", "p2p_perf_rank", "p2p_atomics"):

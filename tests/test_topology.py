@@ -107,7 +107,8 @@ def test_init_discovers_this_gpu_and_refuses_foreign_params(tmp_path):
         p = torch.cuda.get_device_properties(0)
         assert t["world"] == 1 and t["fingerprint"] != "0" * 16 and t["peer_access"] == [[1]]
         assert g["sms"] == p.multi_processor_count and g["numa_node"] >= -1
-        assert g["uuid"] == str(p.uuid).replace("-", "")[-32:] or len(g["uuid"]) == 32
+        # all 16 bytes, also when one of them is 0x00 (torch prints it as GPU-xxxxxxxx-...)
+        assert g["uuid"] == str(p.uuid).replace("-", "")[-32:], (g["uuid"], str(p.uuid))
         c.save_params(f)
         c.load_params(f)                                 # its own file: accepted
         text = open(f).read()
@@ -120,3 +121,15 @@ def test_init_discovers_this_gpu_and_refuses_foreign_params(tmp_path):
     with pytest.raises(mp.MPError) as e:                 # Step 2 at init refuses it too
         mp.Context(device=0, n_loop_relays=1, host_path=1, heap_bytes=MiB, slot_bytes=4 * MiB, param_file=f)
     assert e.value.status == mp.MP_ERR_TOPOLOGY
+
+
+def test_uuid_with_zero_bytes_round_trips():
+    # a UUID byte of 0x00 must not truncate it (ctypes c_char arrays stop at NUL)
+    u = "1420007b081a9ba3ebae706046e09f87"
+    t = topo(2)
+    t["gpus"][0]["uuid"] = u
+    t["gpus"][1]["uuid"] = "00" * 16
+    with mp.Context(rank=0, world=2, model_only=True) as c:
+        c.set_topology(t)
+        got = c.topology()
+        assert [g["uuid"] for g in got["gpus"]] == [u, "00" * 16]
