@@ -307,6 +307,17 @@ def workload_config(args, world, d=None):
             "l2": "inputs 1 GiB > 126 MB L2 (no flush)", "parallelism": f"replicas{world}"}
 
 
+def rank_device(local, world):
+    """The GPU of this rank: one per rank.  Ranks whose kernels wait on one another are
+    never separate launches sharing a GPU (B200 profiling guide); the one-GPU stand-in
+    for the multi-rank engine is the emulated world (tests/test_emulated_gpu.py)."""
+    import torch
+    n = torch.cuda.device_count()
+    if n < world:
+        raise SystemExit(f"bench.py --gpus {world}: needs {world} GPUs (one per rank), found {n}")
+    return local
+
+
 def p2p_roles(world):
     """Config 3 on N GPUs (BASELINE.json configs[2]; P:352's 2_GPUs / 3_GPUs setups):
     rank 0 sends one message to rank 1; ranks 2..N-1 are the relay GPUs; the host
@@ -360,8 +371,7 @@ def run_world_p2p(args, world, rank, local):
     from paper_conf_sc_sojoodiasfga25_b200 import mp
 
     dist.init_process_group("gloo")
-    same_gpu = os.environ.get("MPX_BENCH_SAME_GPU") == "1"   # 1-GPU smoke of this path (MPS)
-    dev = 0 if same_gpu else local
+    dev = rank_device(local, world)
     torch.cuda.set_device(dev)
     n = args.size
     roles = p2p_roles(world)
@@ -378,29 +388,28 @@ def run_world_p2p(args, world, rank, local):
     base = {}
 
     # NCCL send/recv on the same pair (context, not the product), before mp_init
-    if not same_gpu:
-        try:
-            g_nccl = dist.new_group(backend="nccl")
-            buf = src if role == "sender" else torch.empty(n, dtype=torch.uint8, device="cuda")
-            nb_steps = max(3, min(args.steps, 20))
-            tb = 0.0
-            for it in range(nb_steps + 2):
-                if it == 2:
-                    torch.cuda.synchronize()
-                    b0 = time.perf_counter()
-                if role == "sender":
-                    dist.send(buf, 1, group=g_nccl)
-                elif role == "receiver":
-                    dist.recv(buf, 0, group=g_nccl)
-            torch.cuda.synchronize()
-            tb = time.perf_counter() - b0 if role in ("sender", "receiver") else 0.0
-            tb = _gather_max(tb)
-            base["nccl_send_recv_GBps"] = n * nb_steps / tb / 1e9
-            dist.destroy_process_group(g_nccl)
-            del buf
-            torch.cuda.synchronize()
-        except Exception as exc:
-            base["nccl_error"] = repr(exc)
+    try:
+        g_nccl = dist.new_group(backend="nccl")
+        buf = src if role == "sender" else torch.empty(n, dtype=torch.uint8, device="cuda")
+        nb_steps = max(3, min(args.steps, 20))
+        tb = 0.0
+        for it in range(nb_steps + 2):
+            if it == 2:
+                torch.cuda.synchronize()
+                b0 = time.perf_counter()
+            if role == "sender":
+                dist.send(buf, 1, group=g_nccl)
+            elif role == "receiver":
+                dist.recv(buf, 0, group=g_nccl)
+        torch.cuda.synchronize()
+        tb = time.perf_counter() - b0 if role in ("sender", "receiver") else 0.0
+        tb = _gather_max(tb)
+        base["nccl_send_recv_GBps"] = n * nb_steps / tb / 1e9
+        dist.destroy_process_group(g_nccl)
+        del buf
+        torch.cuda.synchronize()
+    except Exception as exc:
+        base["nccl_error"] = repr(exc)
 
     ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
                                   timeout_s=60.0, param_file=args.params)
@@ -539,22 +548,14 @@ def run_world_p2p(args, world, rank, local):
             traffic = json.load(open(tp))[f"{world}:{n}"]["rank0:send_kernel"]["nvlink_tx_bytes_per_launch"]
         except Exception:
             traffic = None
-    if not same_gpu:
-        roofline = {"bound": "nvlink+pcie", "achieved": value, "peak": 964.0, "unit": "GB/s",
-                    "frac": value / 964.0, "traffic": traffic,
-                    "peak_source": "nominal summed path roofline of the source GPU: NVLink 5 egress 900 GB/s "
-                                   "+ PCIe Gen5 x16 64 GB/s (north star); measured peer copy 770 GB/s "
-                                   "(B200_PROFILING.md) alongside",
-                    "nvlink_egress_GBps": nvl_gbs, "frac_of_nvlink_nominal": nvl_gbs / 900.0,
-                    "frac_of_measured_peer_copy": nvl_gbs / 770.0, "pcie_GBps": pcie_gbs,
-                    "frac_of_pcie_nominal": pcie_gbs / 64.0, "kernel": "send_kernel + relay_kernel + recv_kernel"}
-    else:  # every rank on one GPU (diagnostic): the shared resource is that GPU's HBM
-        hbm = 2 * n + 2 * sum(b for (k, _), b in zip(paths_, d["bytes"]) if k == 1)
-        peak = measured_peaks()[0]
-        roofline = {"bound": "hbm", "achieved": hbm * per_s / 1e9, "peak": peak, "unit": "GB/s",
-                    "frac": hbm * per_s / 1e9 / peak, "traffic": None,
-                    "peak_source": "MEASURED_PEAKS.json HBM copy (all ranks on one GPU: not an NVLink number)",
-                    "kernel": "send_kernel + relay_kernel + recv_kernel"}
+    roofline = {"bound": "nvlink+pcie", "achieved": value, "peak": 964.0, "unit": "GB/s",
+                "frac": value / 964.0, "traffic": traffic,
+                "peak_source": "nominal summed path roofline of the source GPU: NVLink 5 egress 900 GB/s "
+                               "+ PCIe Gen5 x16 64 GB/s (north star); measured peer copy 770 GB/s "
+                               "(B200_PROFILING.md) alongside",
+                "nvlink_egress_GBps": nvl_gbs, "frac_of_nvlink_nominal": nvl_gbs / 900.0,
+                "frac_of_measured_peer_copy": nvl_gbs / 770.0, "pcie_GBps": pcie_gbs,
+                "frac_of_pcie_nominal": pcie_gbs / 64.0, "kernel": "send_kernel + relay_kernel + recv_kernel"}
     clk_all = [None] * world
     dist.all_gather_object(clk_all, clk.summary())
     pred = n / d["t_pred"] / 1e9 if d["t_pred"] else None
@@ -573,8 +574,7 @@ def run_world_p2p(args, world, rank, local):
         "topology": {"fingerprint": topo["fingerprint"],
                      "gpus": [{k: g[k] for k in ("numa_node", "pcie_gen", "pcie_width", "nvlinks", "sms")}
                               for g in topo["gpus"]],
-                     "peer_access_all": all(all(r) for r in topo["peer_access"]),
-                     "same_gpu_diagnostic": same_gpu},
+                     "peer_access_all": all(all(r) for r in topo["peer_access"])},
     }
     if rank == 0:
         print(json.dumps(line), flush=True)
@@ -600,7 +600,7 @@ def run_world_pairs(args, world, rank, local):
     from paper_conf_sc_sojoodiasfga25_b200 import mp
 
     dist.init_process_group("gloo")
-    dev = 0 if os.environ.get("MPX_BENCH_SAME_GPU") == "1" else local   # 1-GPU smoke of this path
+    dev = rank_device(local, world)
     torch.cuda.set_device(dev)
     n = args.size
     peer = rank + 1 if rank % 2 == 0 else rank - 1
@@ -621,7 +621,7 @@ def run_world_pairs(args, world, rank, local):
     # Baseline (context, not the product): NCCL send/recv between the same pairs, both
     # directions, measured before mp_init so no NCCL kernel runs beside the relay.
     base = {}
-    if os.environ.get("MPX_BENCH_SAME_GPU") != "1" and active:
+    if active:
         try:
             g_nccl = dist.new_group(backend="nccl")
             scratch = torch.empty_like(src)
@@ -751,13 +751,6 @@ def run_world_pairs(args, world, rank, local):
         "roofline": ({"bound": "nvlink", "achieved": achieved, "peak": 770.0, "unit": "GB/s",
                       "frac": achieved / 770.0, "traffic": None, "peak_source":
                       "B200_PROFILING.md measured peer copy, per direction per GPU (nominal 900)",
-                      "kernel": "send_kernel"}
-                     if os.environ.get("MPX_BENCH_SAME_GPU") != "1" else
-                     # every rank on one GPU (diagnostic): the shared resource is that
-                     # GPU's HBM, 2 bytes per payload byte, both directions at once
-                     {"bound": "hbm", "achieved": 2 * achieved * world, "peak": measured_peaks()[0],
-                      "unit": "GB/s", "frac": 2 * achieved * world / measured_peaks()[0],
-                      "traffic": None, "peak_source": "MEASURED_PEAKS.json HBM copy (all ranks on one GPU)",
                       "kernel": "send_kernel"}),
         "per_direction_GBps": per_dir,
         "baselines": base,

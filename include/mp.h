@@ -64,7 +64,8 @@ enum { MP_MODEL_PAPER = 0, MP_MODEL_B200 = 1 };
 /* Init flags. */
 enum {
   MP_INIT_MODEL_ONLY = 1,  /* no CUDA at all: model evaluator + selector only (CPU tests) */
-  MP_INIT_NO_CALIBRATE = 2 /* do not measure α/β at init (use defaults / param file / mp_set_model) */
+  MP_INIT_NO_CALIBRATE = 2, /* do not measure α/β at init (use defaults / param file / mp_set_model) */
+  MP_INIT_EMULATED = 4      /* set by mp_init_emulated only (mp_init rejects it otherwise) */
 };
 
 typedef struct mp_ctx mp_ctx;  /* opaque, library-owned */
@@ -182,6 +183,45 @@ int mp_init(mp_ctx **ctx, const mp_init_args *args);
  * the relay kernels it launched), unmaps and frees everything.  Collective when
  * world > 1.  ctx may be NULL.  Always returns MP_OK or the barrier's failure. */
 int mp_finalize(mp_ctx *ctx);
+
+/* ---------------------------------------------------------------- emulated world
+ *
+ * Every rank of a world as a context of THIS process on ONE GPU, for running the
+ * multi-rank engine where there are fewer GPUs than ranks.  The engine's ranks wait on
+ * one another on the device (the clear-to-send, the relay doorbells and ring flags,
+ * the done counters of Step 5's pipelined chunks), so they must
+ * never be separate launches sharing a GPU: nothing guarantees those launches run at
+ * the same time.  Here every rank's kernels become CTA ranges of ONE cooperative
+ * launch, co-resident by construction.
+ *
+ * mp_init_emulated: args->world (2..MP_MAX_PATHS) contexts, rank r in ctxs[r], all on
+ * args->device, bootstrapped on one thread each through an in-process all-gather (the
+ * same initialisation as a real job; peers' memory is addressed directly instead of
+ * through CUDA IPC).  args->rank, ->allgather, ->allgather_user are ignored; no
+ * calibration (MP_INIT_NO_CALIBRATE is implied: there are no links to time — set the
+ * model with mp_set_model / mp_load_params).  Errors: as mp_init; on any error no
+ * context is returned.
+ * In an emulated world, mp_send / mp_recv (and mp_select, mp_alloc, every model
+ * call) behave as in a real job except that they launch nothing: they record the
+ * kernels' parameter blocks.  mp_register, the collectives and the calibration calls
+ * return MP_ERR_UNSUPPORTED; mp_finalize returns MP_ERR_STATE.
+ *
+ * mp_emu_run: ctxs = the world's n contexts in rank order.  Launches everything they
+ * recorded since the last run as one cooperative grid on `stream` — per send its gate
+ * and send CTAs, per receive its receive CTAs, the eager kernels, and per (relay rank,
+ * sender) the relay kernel that rank's service thread would have launched, which reads
+ * its doorbells on the device — then waits for the stream.  Direct-path CTA groups
+ * are shrunk (same bytes, fewer CTAs) so the grid fits the device's co-resident
+ * capacity.  The recorded work must be one self-contained exchange: every recorded
+ * send matched by a recorded receive.  Errors: MP_ERR_INVALID (not the whole world /
+ * the fixed roles alone exceed one co-resident grid / a relay's doorbells not
+ * consecutive), MP_ERR_CUDA, MP_ERR_TIMEOUT and MP_ERR_MISMATCH (any rank's device
+ * error word; sticky as in a real job).
+ *
+ * mp_finalize_emulated: tears down all n contexts (one thread each) and the world. */
+int mp_init_emulated(mp_ctx **ctxs, const mp_init_args *args);
+int mp_emu_run(mp_ctx **ctxs, int n, void *stream);
+int mp_finalize_emulated(mp_ctx **ctxs, int n);
 
 /* ---------------------------------------------------------------- topology (Step 1) */
 

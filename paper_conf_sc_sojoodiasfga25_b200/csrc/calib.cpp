@@ -792,6 +792,7 @@ int calibrate_loop_bands(mp_ctx *c, const std::vector<double> &edges, int reps) 
 extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedges, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (c->emulated) return cfail(c, MP_ERR_UNSUPPORTED, "calibration: not in an emulated world (no links to time)");
   if (reps <= 0) reps = 5;
   std::vector<double> edges;
   if (edges_in && nedges > 0) {
@@ -833,6 +834,7 @@ extern "C" int mp_calibrate_bands(mp_ctx *c, const uint64_t *edges_in, int nedge
 extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int window, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (c->emulated) return cfail(c, MP_ERR_UNSUPPORTED, "calibration: not in an emulated world (no links to time)");
   if (c->world != 1) return cfail(c, MP_ERR_UNSUPPORTED, "mp_calibrate_window: loopback contexts only");
   if (window <= 0) window = 16;
   if (window < 2) return cfail(c, MP_ERR_INVALID, "window must be >= 2");
@@ -1028,6 +1030,7 @@ extern "C" int mp_calibrate_window(mp_ctx *c, const uint64_t *sizes_in, int nsiz
 extern "C" int mp_calibrate_wake(mp_ctx *c, uint64_t bytes, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (c->emulated) return cfail(c, MP_ERR_UNSUPPORTED, "calibration: not in an emulated world (no links to time)");
   const int W = c->world, me = c->rank;
   if (W < 3) return MP_OK;  // no relay ranks
   if (reps <= 0) reps = 7;
@@ -1206,6 +1209,7 @@ extern "C" int mp_fit_bands(const double *n, const double *t, int m, const doubl
 extern "C" int mp_calibrate(mp_ctx *c, const uint64_t *sizes_in, int nsizes, int reps) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  if (c->emulated) return cfail(c, MP_ERR_UNSUPPORTED, "calibration: not in an emulated world (no links to time)");
   if (reps <= 0) reps = 5;
   if (c->world != 1) {
     std::vector<uint64_t> sizes;

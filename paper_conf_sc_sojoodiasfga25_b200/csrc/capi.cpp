@@ -466,6 +466,11 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
   c->device = a->device;
   c->flags = a->flags;
   c->model_only = (a->flags & MP_INIT_MODEL_ONLY) != 0;
+  c->emulated = (a->flags & MP_INIT_EMULATED) != 0;
+  if (c->emulated && (!mpx::emu_thread() || a->world < 2 || c->model_only)) {  // only through mp_init_emulated
+    delete c;
+    return MP_ERR_INVALID;
+  }
   c->n_loop_relays = a->n_loop_relays < 0 ? 6 : std::min(a->n_loop_relays, MP_MAX_PATHS - 2);
   c->host_path = a->host_path < 0 ? true : a->host_path != 0;
   c->slots = a->slots > 0 ? a->slots : 4;
@@ -537,6 +542,7 @@ int mp_init(mp_ctx **out, const mp_init_args *a) {
 
 int mp_finalize(mp_ctx *c) {
   if (!c) return MP_OK;
+  if (c->emulated && c->emu_world) return MP_ERR_STATE;  // mp_finalize_emulated tears the world down
   if (!c->model_only) {
     cudaSetDevice(c->device);
     coll_release(c);
@@ -546,6 +552,24 @@ int mp_finalize(mp_ctx *c) {
   }
   delete c;
   return MP_OK;
+}
+
+int mp_init_emulated(mp_ctx **ctxs, const mp_init_args *args) {
+  if (!ctxs || !args || args->world < 2 || args->world > MP_MAX_PATHS) return MP_ERR_INVALID;
+  if (args->flags & MP_INIT_MODEL_ONLY) return MP_ERR_INVALID;
+  for (int r = 0; r < args->world; ++r) ctxs[r] = nullptr;
+  return mpx::emu_init_world(ctxs, args);
+}
+
+int mp_finalize_emulated(mp_ctx **ctxs, int n) {
+  if (!ctxs || n < 2 || !ctxs[0] || !ctxs[0]->emulated) return MP_ERR_INVALID;
+  return mpx::emu_finalize_world(ctxs, n);
+}
+
+int mp_emu_run(mp_ctx **ctxs, int n, void *stream) {
+  if (!ctxs || n < 2 || !ctxs[0]) return MP_ERR_INVALID;
+  if (!ctxs[0]->emulated) return fail(ctxs[0], MP_ERR_STATE, "mp_emu_run: not an emulated world");
+  return mpx::emu_run(ctxs, n, stream);
 }
 
 int mp_paths(mp_ctx *c, int src, int dst, mp_path *out, int *npaths) {

@@ -426,6 +426,9 @@ int collective(mp_ctx *c, int coll, int algo, const void *sendbuf, void *recvbuf
                int dtype, void *stream) {
   if (!c) return MP_ERR_INVALID;
   if (c->model_only) return cfail(c, MP_ERR_STATE, "model-only context");
+  // an emulated world runs everything recorded as one grid: a plan's later steps
+  // depend on its earlier ones (and on local kernels in between)
+  if (c->emulated) return cfail(c, MP_ERR_UNSUPPORTED, "collectives: not in an emulated world");
   if (bytes == 0) return MP_OK;
   if (!sendbuf || !recvbuf) return cfail(c, MP_ERR_INVALID, "null buffer");
   mp_coll_plan *P = new (std::nothrow) mp_coll_plan;

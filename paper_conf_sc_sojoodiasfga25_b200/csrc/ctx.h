@@ -69,6 +69,10 @@ struct CacheKeyHash {
 
 }  // namespace mpx
 
+namespace mpx {
+struct EmuWorld;  // world.cpp
+}
+
 struct mp_ctx {
   int rank = 0, world = 1, device = 0, flags = 0;
   bool model_only = true;
@@ -161,6 +165,13 @@ struct mp_ctx {
     int refs = 0;
   };
   std::map<std::pair<int, uint64_t>, IpcMap> ipc_maps;
+  // emulated world (MP_INIT_EMULATED; engine.h EmuTable): the kernels mp_send / mp_recv
+  // would launch, recorded for the next mp_emu_run
+  bool emulated = false;
+  mpx::EmuWorld *emu_world = nullptr;       // shared by the world's contexts (world.cpp)
+  std::vector<mpx::SendParams> emu_send;
+  std::vector<mpx::RecvParams> emu_recv;
+  std::vector<mpx::EagerParams> emu_esend, emu_erecv;
 };
 
 namespace mpx {
@@ -209,6 +220,13 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
                void *stream);
 int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *stream);
 int world_sync(mp_ctx *c);
+// emulated world (world.cpp): bootstrap / teardown of all ranks on one thread each,
+// the one cooperative launch of what they recorded, and whether this thread is one of
+// the bootstrap's rank threads
+int emu_init_world(mp_ctx **ctxs, const mp_init_args *a);
+int emu_finalize_world(mp_ctx **ctxs, int n);
+int emu_run(mp_ctx **ctxs, int n, void *stream);
+bool emu_thread();
 int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id);
 // true when [p, p + n) lies in a receive region (heap or mp_register) of this rank
 bool world_receivable(mp_ctx *c, const void *p, uint64_t n);

@@ -1084,8 +1084,7 @@ struct HostConsumer {
 // lets the bulk send kernel launch only once the clear-to-send has arrived (no bulk
 // CTA is ever resident during the rendezvous); send, receive and eager kernels let
 // their successor launch at once and wait for their predecessor (pdl_enter).
-__global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
-  asm volatile("griddepcontrol.wait;" ::: "memory");
+__device__ void send_gate_body(const SendParams &P) {
   if (threadIdx.x != 0) return;
   MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
   const uint64_t t_start = globaltimer();
@@ -1157,13 +1156,17 @@ __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
       st_release_sys(&e->tag, d.m + 1);
     }
   }
+}
+
+__global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  send_gate_body(P);
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
+// CTA b of the send kernel's grid (the kernel below; one role of emu_kernel).
 template <uint32_t D>
-__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) send_kernel(const __grid_constant__ SendParams P) {
-  extern __shared__ __align__(128) uint8_t dyn_smem[];
-  pdl_enter();
+__device__ void send_body(const SendParams &P, const uint32_t b, uint8_t *dyn_smem) {
   __shared__ int s_abort;
   __shared__ uint64_t s_off, s_region;
   __shared__ uint8_t *s_dst;
@@ -1184,7 +1187,6 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) send_kerne
   __syncthreads();
   if (s_abort) return;
   const uint64_t base = s_off;
-  const uint32_t b = blockIdx.x;
   uint64_t *done = done_at(P.dst_ctrl, P.L, P.me);
   if (b < P.g_direct) {  // A7: direct NVLink stores into the receiver's heap
     if (P.copy_mode == 1)
@@ -1248,15 +1250,21 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) send_kerne
 }
 
 template <uint32_t D>
-__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kernel(const __grid_constant__ RecvParams P) {
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) send_kernel(const __grid_constant__ SendParams P) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
   pdl_enter();
+  send_body<D>(P, blockIdx.x, dyn_smem);
+}
+
+// CTA b of the receive kernel's grid (the kernel below; one role of emu_kernel).
+template <uint32_t D>
+__device__ void recv_body(const RecvParams &P, const uint32_t b, uint8_t *dyn_smem) {
   __shared__ int s_abort;
   __shared__ uint64_t s_k, s_q0, s_hoff, s_hbytes, s_shift, s_align;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
   MsgEntry *hdr = entry_at(P.my_ctrl, P.L.hdr, P.src, P.seq);
-  if (blockIdx.x == 0) {
+  if (b == 0) {
     if (threadIdx.x == 0) {  // post the clear-to-send into the sender's control block
       MsgEntry *cts = entry_at(P.src_ctrl, P.L.cts, P.me, P.seq);
       cts->a = P.region_off;
@@ -1284,7 +1292,7 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kerne
     return;
   }
   // A9 step 3: host-ring consumers, CTA r = lane r of every host slot
-  const uint32_t r = blockIdx.x - 1;
+  const uint32_t r = b - 1;
   if (!wait_word(&hdr->seq1, P.seq + 1, P.timeout_ns, P.err, &s_abort)) return;
   if (threadIdx.x == 0) {
     s_k = ld_volatile(&hdr->c) ? 0 : ld_volatile(&hdr->a);
@@ -1317,6 +1325,13 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kerne
   }
 }
 
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kernel(const __grid_constant__ RecvParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
+  pdl_enter();
+  recv_body<D>(P, blockIdx.x, dyn_smem);
+}
+
 // Relay (A8 step 3): CTA r forwards lane r of chunks [q0, q0 + k) of the sender's ring
 // to the destination its lane header names, counts the bytes into the destination's
 // `done` and returns the lane to the sender — for the launch's first message, then
@@ -1324,9 +1339,8 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kerne
 // linger_ns, so back-to-back relayed messages pay no relaunch.  A relay kernel still
 // ends once its sender goes quiet: nothing outlives the traffic by more than the linger.
 template <uint32_t D>
-__device__ bool relay_message(const RelayParams &P, uint64_t q0, uint64_t k, uint32_t aligned, int *s_abort,
-                              uint8_t *smem) {
-  const uint32_t r = blockIdx.x;
+__device__ bool relay_message(const RelayParams &P, const uint32_t r, uint64_t q0, uint64_t k, uint32_t aligned,
+                              int *s_abort, uint8_t *smem) {
   const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g);
   if (P.copy_mode == 1 && aligned) {  // streamed lane (the sender found source and target co-aligned)
     RelayConsumer R{&P, r, lstride, q0};
@@ -1357,29 +1371,33 @@ __device__ bool relay_message(const RelayParams &P, uint64_t q0, uint64_t k, uin
   return true;
 }
 
+// CTA b of a relay launch; the launch's first message is chunks [q0, q0 + k) of
+// doorbell P.m0 (the relay kernel below: read by the host thread; emu_kernel's relay
+// role: read from the doorbell on the device).
 template <uint32_t D>
-__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kernel(const __grid_constant__ RelayParams P) {
-  extern __shared__ __align__(128) uint8_t dyn_smem[];
+__device__ void relay_body(const RelayParams &P, const uint32_t b, uint64_t q0, uint64_t k, uint32_t aligned,
+                           uint8_t *dyn_smem) {
   __shared__ int s_abort;
   __shared__ uint64_t s_next[4];  // next message: tag, q0, k, flags (bit 0 aligned, bit 1 stop)
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
-  uint64_t m = P.m0, q0 = P.q0, k = P.k;
-  uint32_t aligned = P.aligned;
+  uint64_t m = P.m0;
   // doorbell m is taken (the host thread read it for this launch): the sender may reuse
   // its ring entry kBellRing messages later (flow control in send_gate_kernel)
   uint64_t *ack = reinterpret_cast<uint64_t *>(P.sender_ctrl + P.L.bell_ack) + P.me * 16;
-  if (blockIdx.x == 0 && threadIdx.x == 0) st_release_sys(ack, m + 1);
+  if (b == 0 && threadIdx.x == 0) st_release_sys(ack, m + 1);
   for (;;) {
-    if (!relay_message<D>(P, q0, k, aligned, &s_abort, dyn_smem)) break;
+    if (!relay_message<D>(P, b, q0, k, aligned, &s_abort, dyn_smem)) break;
     // the sender's next message: CTA 0 looks for its doorbell for up to linger_ns and
     // publishes the decision; every CTA follows it
     uint64_t *dec = P.dec + ((m + 1) % kBellRing) * 4;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (b == 0 && threadIdx.x == 0) {
       const BellEntry *e = P.bells + (m + 1) % kBellRing;
       const uint64_t t0 = globaltimer();
       bool found = false;
-      while (P.linger_ns && globaltimer() - t0 < P.linger_ns) {
+      // max_msgs (emu_kernel): the launch serves exactly that many messages
+      const bool more = P.max_msgs == 0 || m + 1 - P.m0 < P.max_msgs;
+      while (more && P.linger_ns && globaltimer() - t0 < P.linger_ns) {
         if (ld_relaxed_sys(&e->tag) == m + 2) {
           found = ld_acquire_sys(&e->tag) == m + 2;
           break;
@@ -1436,16 +1454,20 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kern
   }
 }
 
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) relay_kernel(const __grid_constant__ RelayParams P) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
+  relay_body<D>(P, blockIdx.x, P.q0, P.k, P.aligned, dyn_smem);
+}
+
 
 // Eager protocol (engine.h, reading C23).  Slot = [kEagerHdr header][shift][data]:
 // header words 0/1 = bytes/tag (CTA 0), kEagerShift0 + r = source shift of CTA r's
 // slice, kEagerFlag0 + r = CTA r's sequence flag (seq + 1, released after its slice).
-__global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_constant__ EagerParams P) {
-  pdl_enter();
+__device__ void eager_send_body(const EagerParams &P, const uint32_t r) {
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
-  const uint32_t r = blockIdx.x;
   // the slot is free once the receiver has returned message seq − kEagerSlots
   if (P.seq >= kEagerSlots && !wait_word(P.free_ctr, P.seq + 1 - kEagerSlots, P.timeout_ns, P.err, &s_abort))
     return;
@@ -1466,12 +1488,15 @@ __global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_const
   if (threadIdx.x == 0) st_release_sys(hdr + kEagerFlag0 + r, P.seq + 1);
 }
 
-__global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_constant__ EagerParams P) {
+__global__ void __launch_bounds__(kThreads) eager_send_kernel(const __grid_constant__ EagerParams P) {
   pdl_enter();
+  eager_send_body(P, blockIdx.x);
+}
+
+__device__ void eager_recv_body(const EagerParams &P, const uint32_t r) {
   __shared__ int s_abort;
   if (threadIdx.x == 0) s_abort = 0;
   __syncthreads();
-  const uint32_t r = blockIdx.x;
   const uint64_t *hdr = reinterpret_cast<const uint64_t *>(P.slot);
   // every CTA first checks the sender's size and tag (CTA 0's flag): a receive posted
   // larger than the message would otherwise wait for slices that never come
@@ -1493,6 +1518,11 @@ __global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_const
       red_add_release_sys(P.free_ctr, 1);
     }
   }
+}
+
+__global__ void __launch_bounds__(kThreads) eager_recv_kernel(const __grid_constant__ EagerParams P) {
+  pdl_enter();
+  eager_recv_body(P, blockIdx.x);
 }
 
 // Direct-only messages (the B200-mode pick whenever the shared port is saturated by
@@ -1546,6 +1576,70 @@ __global__ void __launch_bounds__(kThreads) direct_small_kernel(uint8_t *dst, co
 __global__ void __launch_bounds__(kThreads) direct_reg_kernel(const __grid_constant__ DirectArgs A) {
   pdl_enter();
   group_copy<LD_SRC>(A.dst, A.src, A.bytes, blockIdx.x, gridDim.x);
+}
+
+// ------------------------------------------------------------------ emulated world
+//
+// One cooperative grid plays every rank's kernels (engine.h: EmuTable).  The relay
+// role stands in for the relay rank's service thread too: its CTAs read the sender's
+// doorbell for the first message on the device, then run the relay kernel's body,
+// which serves exactly max_msgs messages (the later doorbells through the same
+// next-message decisions as a lingering relay kernel).
+template <uint32_t D>
+__device__ void relay_emu_body(const RelayParams &P, const uint32_t b, uint8_t *smem) {
+  __shared__ uint64_t s_bell[3];
+  __shared__ int s_ok;
+  if (threadIdx.x == 0) {
+    const BellEntry *e = P.bells + P.m0 % kBellRing;
+    const uint64_t t0 = globaltimer();
+    int ok = 1;
+    while (ld_acquire_sys(&e->tag) != P.m0 + 1) {
+      if (*reinterpret_cast<volatile int32_t *>(P.err) != 0) {  // the relay rank already failed
+        ok = 0;
+        break;
+      }
+      if (globaltimer() - t0 > P.timeout_ns) {
+        atomicExch(P.err, DERR_TIMEOUT);
+        ok = 0;
+        break;
+      }
+      __nanosleep(256);
+    }
+    if (ok) {
+      s_bell[0] = ld_volatile(&e->q0);
+      s_bell[1] = ld_volatile(&e->k);
+      s_bell[2] = ld_volatile(&e->g);
+      if (static_cast<uint32_t>(s_bell[2] & 0xffffffffu) != P.g) {  // the role's CTAs are the lanes
+        atomicExch(P.err, DERR_MISMATCH);
+        ok = 0;
+      }
+    }
+    s_ok = ok;
+  }
+  __syncthreads();
+  if (!s_ok) return;
+  relay_body<D>(P, b, s_bell[0], s_bell[1], static_cast<uint32_t>((s_bell[2] >> 32) & 1u), smem);
+}
+
+template <uint32_t D>
+__global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) emu_kernel(const __grid_constant__ EmuTable T) {
+  extern __shared__ __align__(128) uint8_t dyn_smem[];
+  const uint32_t blk = blockIdx.x;
+  for (uint32_t i = 0; i < T.nroles; ++i) {
+    const EmuRole R = T.roles[i];
+    if (blk < R.cta0 || blk >= R.cta0 + R.n) continue;
+    const uint32_t b = blk - R.cta0;
+    switch (R.kind) {
+      case EMU_GATE: send_gate_body(T.send[R.idx]); break;
+      case EMU_SEND: send_body<D>(T.send[R.idx], b, dyn_smem); break;
+      case EMU_RECV: recv_body<D>(T.recv[R.idx], b, dyn_smem); break;
+      case EMU_RELAY: relay_emu_body<D>(T.relay[R.idx], b, dyn_smem); break;
+      case EMU_EAGER_SEND: eager_send_body(T.eager[R.idx], b); break;
+      case EMU_EAGER_RECV: eager_recv_body(T.eager[R.idx], b); break;
+      default: break;
+    }
+    return;
+  }
 }
 
 // Elementwise dst += src (Allreduce, NEXT f3): grid-stride over 16-byte vectors when
@@ -1697,6 +1791,27 @@ int launch_relay(const RelayParams &P, void *stream) {
   else
     relay_kernel<kBulkStages><<<P.g, kThreads, staged_smem<kBulkStages>(), static_cast<cudaStream_t>(stream)>>>(P);
   return static_cast<int>(cudaGetLastError());
+}
+
+int emu_capacity(int *per_sm) {
+  const int smem = static_cast<int>(staged_smem<kBulkStages>());
+  cudaError_t e = cudaFuncSetAttribute(emu_kernel<kBulkStages>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, emu_kernel<kBulkStages>, kThreads, smem);
+  return static_cast<int>(e);
+}
+
+int launch_emu(const EmuTable &T, void *stream) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(T.nblocks);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = staged_smem<kBulkStages>();
+  cfg.stream = static_cast<cudaStream_t>(stream);
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;  // every CTA co-resident, or the launch fails
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return static_cast<int>(cudaLaunchKernelEx(&cfg, emu_kernel<kBulkStages>, T));
 }
 
 int launch_spin(uint64_t ns, void *stream) {

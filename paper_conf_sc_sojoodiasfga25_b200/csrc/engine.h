@@ -255,6 +255,7 @@ struct RelayParams {
   uint64_t q0, k, timeout_ns;
   uint64_t m0;                 // doorbell index of the first message
   uint64_t linger_ns;          // how long CTA 0 waits for the next doorbell (0: one message)
+  uint64_t max_msgs;           // > 0 (emu_kernel): serve exactly this many messages; 0: linger rule
   const BellEntry *bells;      // the sender's doorbell row in this rank's segment (mapped host)
   uint64_t *dec;               // [kBellRing][4] device words: CTA 0's next-message decisions
   uint32_t *exit_cnt;          // device word: CTAs that have left
@@ -279,6 +280,34 @@ struct EagerParams {
   int32_t *err;
   uint32_t pdl;              // 1: launched with programmatic stream serialization (PDL)
 };
+
+// Emulated world (MP_INIT_EMULATED, include/mp.h): every rank is a context of one
+// process on one GPU, and mp_send / mp_recv record their kernels' parameter blocks
+// instead of launching them.  mp_emu_run then launches ONE cooperative grid whose CTA
+// ranges (roles) run those kernels' bodies — the send gate, the send kernel, the
+// receive kernel, the eager kernels and, for every (relay rank, sender) pair, the relay
+// kernel that rank's service thread would have launched (it reads its doorbells on
+// the device instead).  Kernels of different ranks that wait on one another are then
+// co-resident by construction (a cooperative launch), never separate launches sharing
+// a GPU.
+enum EmuKind : uint32_t { EMU_GATE = 0, EMU_SEND, EMU_RECV, EMU_RELAY, EMU_EAGER_SEND, EMU_EAGER_RECV };
+struct EmuRole {
+  uint32_t kind;             // EmuKind
+  uint32_t cta0, n;          // CTA range [cta0, cta0 + n) of the grid
+  uint32_t idx;              // index into the parameter array of its kind
+};
+struct EmuTable {
+  const EmuRole *roles;      // device arrays
+  const SendParams *send;
+  const RecvParams *recv;
+  const RelayParams *relay;
+  const EagerParams *eager;
+  uint32_t nroles, nblocks;
+};
+// Co-resident CTAs per SM of emu_kernel (its grid must not exceed per_sm x SMs).
+int emu_capacity(int *per_sm);
+// Cooperative launch of emu_kernel over T.nblocks CTAs (T's arrays in device memory).
+int launch_emu(const EmuTable &T, void *stream);
 
 int launch_send(const SendParams &P, void *stream);
 int launch_eager_send(const EagerParams &P, void *stream);

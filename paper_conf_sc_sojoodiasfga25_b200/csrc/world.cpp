@@ -17,6 +17,9 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <condition_variable>
+#include <map>
+#include <mutex>
 #include <thread>
 #include <cstdio>
 #include <cstdlib>
@@ -47,6 +50,7 @@ struct RankInfo {
   cudaIpcMemHandle_t ctrl;
   uint64_t jobid;
   uint64_t heap_addr;
+  uint64_t ctrl_addr;  // emulated world: every rank's memory is this process's own
   uint64_t heap_bytes;
   int32_t device;
   int32_t relay_ctas;
@@ -178,8 +182,11 @@ int world_init(mp_ctx *c) {
 
   RankInfo me;
   std::memset(&me, 0, sizeof(me));
-  CKW(cudaIpcGetMemHandle(&me.heap, c->heap.base));
-  CKW(cudaIpcGetMemHandle(&me.ctrl, c->ctrl));
+  if (!c->emulated) {
+    CKW(cudaIpcGetMemHandle(&me.heap, c->heap.base));
+    CKW(cudaIpcGetMemHandle(&me.ctrl, c->ctrl));
+  }
+  me.ctrl_addr = reinterpret_cast<uintptr_t>(c->ctrl);
   me.jobid = std::random_device{}() ^ (static_cast<uint64_t>(std::random_device{}()) << 32) ^
              static_cast<uint64_t>(getpid());
   me.heap_addr = reinterpret_cast<uintptr_t>(c->heap.base);
@@ -209,6 +216,10 @@ int world_init(mp_ctx *c) {
   for (int r = 0; r < W; ++r) {
     if (r == c->rank) {
       c->peers[r] = PeerPtrs{c->heap.base, c->ctrl};
+      continue;
+    }
+    if (c->emulated) {  // one process: a peer's memory is addressed as allocated
+      c->peers[r] = PeerPtrs{reinterpret_cast<uint8_t *>(all[r].heap_addr), reinterpret_cast<uint8_t *>(all[r].ctrl_addr)};
       continue;
     }
     void *h = nullptr, *k = nullptr;
@@ -244,7 +255,15 @@ int world_init(mp_ctx *c) {
   c->hseg_per_src = (static_cast<uint64_t>(c->slots) * c->host_stride + 4095) & ~uint64_t(4095);
   c->hseg_bytes = static_cast<size_t>(bell_bytes(W) + (c->host_path ? c->hseg_per_src * W : 0));
   c->hseg.assign(W, nullptr);
-  if (c->host_path || W >= 3) {
+  if ((c->host_path || W >= 3) && c->emulated) {
+    // one process: every rank registers its own segment once; the others use its address
+    if (int s = map_segment(c, c->rank, true, &c->hseg[c->rank])) return s;
+    shm_unlink(seg_name(c->jobid, c->rank).c_str());
+    const uint64_t mine = reinterpret_cast<uintptr_t>(c->hseg[c->rank]);
+    std::vector<uint64_t> segs(W);
+    if (int s = allgather(c, &mine, segs.data(), sizeof(uint64_t))) return s;
+    for (int r = 0; r < W; ++r) c->hseg[r] = reinterpret_cast<uint8_t *>(segs[r]);
+  } else if (c->host_path || W >= 3) {
     if (int s = map_segment(c, c->rank, true, &c->hseg[c->rank])) return s;
     if (int s = barrier(c)) return s;
     for (int r = 0; r < W; ++r)
@@ -362,7 +381,8 @@ void relay_loop(mp_ctx *c, RelayService *S) {
 
 int world_start_relay(mp_ctx *c) {
   const char *no_relay = std::getenv("MPX_NO_RELAY");  // diagnostics: no relay service
-  if (c->world < 3 || c->relay_svc || (no_relay && no_relay[0] == '1')) return MP_OK;
+  // an emulated world has no relay threads: mp_emu_run's relay roles read the doorbells
+  if (c->world < 3 || c->relay_svc || c->emulated || (no_relay && no_relay[0] == '1')) return MP_OK;
   RelayService *S = new RelayService();
   S->streams.assign(c->world, nullptr);
   S->bells = reinterpret_cast<BellEntry *>(c->hseg[c->rank]);
@@ -429,7 +449,7 @@ int world_finalize(mp_ctx *c) {
     if (o.done) cudaEventDestroy(o.done);
   c->ring_order.clear();
   if (c->allgather) st = barrier(c);
-  for (int r = 0; r < static_cast<int>(c->peers.size()); ++r) {
+  for (int r = 0; r < static_cast<int>(c->peers.size()) && !c->emulated; ++r) {
     if (r == c->rank) continue;
     if (c->peers[r].ctrl) cudaIpcCloseMemHandle(c->peers[r].ctrl);
   }
@@ -437,10 +457,10 @@ int world_finalize(mp_ctx *c) {
   c->ipc_maps.clear();
   c->regions.clear();
   c->peers.clear();
-  for (uint8_t *s : c->hseg)
-    if (s) {
-      cudaHostUnregister(s);
-      munmap(s, c->hseg_bytes);
+  for (size_t r = 0; r < c->hseg.size(); ++r)
+    if (c->hseg[r] && (!c->emulated || static_cast<int>(r) == c->rank)) {  // emulated: own segment only
+      cudaHostUnregister(c->hseg[r]);
+      munmap(c->hseg[r], c->hseg_bytes);
     }
   c->hseg.clear();
   if (c->ctrl) cudaFree(c->ctrl);
@@ -494,7 +514,9 @@ static int eager_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int t
   // copied out): same cross-stream order, per destination
   const size_t ring = 3 * static_cast<size_t>(c->world) + static_cast<size_t>(dst);
   if (int e = ring_wait(c, ring, static_cast<cudaStream_t>(stream))) return e;
-  if (int e = launch_eager_send(P, stream))
+  if (c->emulated) {
+    c->emu_esend.push_back(P);
+  } else if (int e = launch_eager_send(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("eager send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   if (int e = ring_mark(c, ring, static_cast<cudaStream_t>(stream))) return e;
   c->launches += 1;
@@ -508,7 +530,9 @@ static int eager_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, vo
   P.dst = static_cast<uint8_t *>(buf);
   const size_t ring = 4 * static_cast<size_t>(c->world) + static_cast<size_t>(src);
   if (int e = ring_wait(c, ring, static_cast<cudaStream_t>(stream))) return e;
-  if (int e = launch_eager_recv(P, stream))
+  if (c->emulated) {
+    c->emu_erecv.push_back(P);
+  } else if (int e = launch_eager_recv(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("eager recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   if (int e = ring_mark(c, ring, static_cast<cudaStream_t>(stream))) return e;
   c->launches += 1;
@@ -587,7 +611,9 @@ int world_send(mp_ctx *c, const void *buf, uint64_t bytes, int dst, int tag, con
   const size_t W = static_cast<size_t>(c->world);
   for (auto &a : advance)
     if (int e = ring_wait(c, a.first < 0 ? W + static_cast<size_t>(dst) : static_cast<size_t>(a.first), cs)) return e;
-  if (int e = launch_send(P, stream))
+  if (c->emulated) {
+    c->emu_send.push_back(P);
+  } else if (int e = launch_send(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("send launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   for (auto &a : advance)
     if (int e = ring_mark(c, a.first < 0 ? W + static_cast<size_t>(dst) : static_cast<size_t>(a.first), cs)) return e;
@@ -657,7 +683,9 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   const cudaStream_t cs = static_cast<cudaStream_t>(stream);
   if (c->host_path)
     if (int e = ring_wait(c, ring, cs)) return e;
-  if (int e = launch_recv(P, stream))
+  if (c->emulated) {
+    c->emu_recv.push_back(P);
+  } else if (int e = launch_recv(P, stream))
     return wfail(c, MP_ERR_CUDA, std::string("recv launch: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   if (c->host_path)
     if (int e = ring_mark(c, ring, cs)) return e;
@@ -717,6 +745,7 @@ void unmap(mp_ctx *c, int r, uint64_t key) {
 }  // namespace
 
 int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
+  if (c->emulated) return wfail(c, MP_ERR_UNSUPPORTED, "mp_register: not in an emulated world (use mp_alloc)");
   const int W = c->world;
   int rid = -1;
   for (int i = 1; i < static_cast<int>(c->regions.size()); ++i)
@@ -800,6 +829,7 @@ int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
 }
 
 int world_deregister(mp_ctx *c, int id) {
+  if (c->emulated) return wfail(c, MP_ERR_UNSUPPORTED, "mp_deregister: not in an emulated world");
   const int W = c->world;
   if (id <= 0 || id >= static_cast<int>(c->regions.size()) || !c->regions[id].used)
     return wfail(c, MP_ERR_INVALID, "mp_deregister: unknown region id");
@@ -831,6 +861,282 @@ int world_sync(mp_ctx *c) {
   CKW(cudaMemcpy(&e, c->d_err, sizeof(e), cudaMemcpyDeviceToHost));
   if (e == DERR_TIMEOUT) return wfail(c, MP_ERR_TIMEOUT, "a device-side wait timed out");
   if (e == DERR_MISMATCH) return wfail(c, MP_ERR_MISMATCH, "send/recv size or tag mismatch");
+  return MP_OK;
+}
+
+
+// ---------------------------------------------------------------- emulated world
+//
+// MP_INIT_EMULATED (include/mp.h): the ranks of a world are contexts of ONE process on
+// ONE GPU.  mp_init_emulated bootstraps them on one thread each through an in-process
+// all-gather (the same world_init as a real job, with the IPC exchange replaced by
+// the allocations' own addresses); mp_send / mp_recv record their parameter blocks;
+// mp_emu_run launches everything recorded as one cooperative grid (engine.h EmuTable)
+// — the B200 guide's rule for ranks whose kernels wait on one another when there are
+// fewer GPUs than ranks.
+
+struct EmuWorld {
+  int world = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  uint64_t gen = 0;
+  int arrived = 0;
+  bool aborted = false;
+  std::vector<uint8_t> buf, out;
+  std::vector<mp_ctx *> ctxs;
+};
+
+namespace {
+thread_local int t_emu_rank = -1;
+
+// The in-process all-gather: rank t_emu_rank's bytes into slot t_emu_rank; the last
+// arrival publishes the gathered block; a rank whose mp_init failed aborts every
+// pending and later all-gather (no rank waits forever for it).
+int emu_allgather(void *user, const void *in, void *out, uint64_t bytes) {
+  EmuWorld *w = static_cast<EmuWorld *>(user);
+  const int r = t_emu_rank;
+  if (r < 0 || r >= w->world) return -1;
+  std::unique_lock<std::mutex> lk(w->mu);
+  if (w->aborted) return -1;
+  const uint64_t g = w->gen;
+  if (w->arrived == 0) w->buf.assign(bytes * w->world, 0);
+  if (w->buf.size() != bytes * w->world) return -1;
+  std::memcpy(w->buf.data() + bytes * r, in, bytes);
+  if (++w->arrived == w->world) {
+    w->out = w->buf;
+    w->arrived = 0;
+    w->gen += 1;
+    w->cv.notify_all();
+  } else {
+    w->cv.wait(lk, [&] { return w->gen != g || w->aborted; });
+    if (w->gen == g) return -1;  // aborted
+  }
+  std::memcpy(out, w->out.data(), bytes * w->world);
+  return 0;
+}
+
+void emu_abort(EmuWorld *w) {
+  std::lock_guard<std::mutex> lk(w->mu);
+  w->aborted = true;
+  w->cv.notify_all();
+}
+}  // namespace
+
+int emu_init_world(mp_ctx **ctxs, const mp_init_args *a) {
+  const int W = a->world;
+  EmuWorld *w = new EmuWorld();
+  w->world = W;
+  w->ctxs.assign(W, nullptr);
+  std::vector<int> st(W, MP_OK);
+  std::vector<std::thread> th;
+  for (int r = 0; r < W; ++r)
+    th.emplace_back([&, r] {
+      t_emu_rank = r;
+      mp_init_args ar = *a;
+      ar.rank = r;
+      ar.flags = (a->flags | MP_INIT_EMULATED | MP_INIT_NO_CALIBRATE) & ~MP_INIT_MODEL_ONLY;
+      ar.allgather = emu_allgather;
+      ar.allgather_user = w;
+      st[r] = mp_init(&w->ctxs[r], &ar);
+      if (st[r] != MP_OK) emu_abort(w);
+    });
+  for (std::thread &t : th) t.join();
+  int bad = MP_OK;
+  for (int r = 0; r < W; ++r)
+    if (st[r] != MP_OK && bad == MP_OK) bad = st[r];
+  if (bad != MP_OK) {  // ranks that did come up: finalize them without the collective part
+    for (int r = 0; r < W; ++r)
+      if (w->ctxs[r]) {
+        w->ctxs[r]->emu_world = nullptr;
+        w->ctxs[r]->allgather = nullptr;
+        mp_finalize(w->ctxs[r]);
+      }
+    delete w;
+    return bad;
+  }
+  for (int r = 0; r < W; ++r) {
+    w->ctxs[r]->emu_world = w;
+    ctxs[r] = w->ctxs[r];
+  }
+  return MP_OK;
+}
+
+int emu_finalize_world(mp_ctx **ctxs, int n) {
+  EmuWorld *w = ctxs[0]->emu_world;
+  if (!w || n != w->world) return MP_ERR_INVALID;
+  for (int r = 0; r < n; ++r)
+    if (!ctxs[r] || ctxs[r]->emu_world != w || ctxs[r]->rank != r) return MP_ERR_INVALID;
+  std::vector<std::thread> th;
+  for (int r = 0; r < n; ++r)
+    th.emplace_back([=] {
+      t_emu_rank = r;
+      ctxs[r]->emu_world = nullptr;  // mp_finalize's collective part runs on this thread
+      mp_finalize(ctxs[r]);
+    });
+  for (std::thread &t : th) t.join();
+  delete w;
+  return MP_OK;
+}
+
+bool emu_thread() { return t_emu_rank >= 0; }
+
+int emu_run(mp_ctx **ctxs, int n, void *stream) {
+  mp_ctx *c = ctxs[0];
+  EmuWorld *w = c->emu_world;
+  if (!w || n != w->world) return wfail(c, MP_ERR_INVALID, "mp_emu_run: pass every context of one emulated world");
+  for (int r = 0; r < n; ++r)
+    if (!ctxs[r] || ctxs[r]->emu_world != w || ctxs[r]->rank != r)
+      return wfail(c, MP_ERR_INVALID, "mp_emu_run: contexts must be the world's, in rank order");
+  c = w->ctxs[0];
+  CKW(cudaSetDevice(c->device));
+  std::vector<SendParams> send;
+  std::vector<RecvParams> recv;
+  std::vector<EagerParams> eager;
+  std::vector<RelayParams> relay;
+  std::vector<EmuRole> roles;
+  for (int r = 0; r < n; ++r) {
+    mp_ctx *cr = ctxs[r];
+    send.insert(send.end(), cr->emu_send.begin(), cr->emu_send.end());
+    recv.insert(recv.end(), cr->emu_recv.begin(), cr->emu_recv.end());
+  }
+  // relay roles: one per (relay rank, sender), serving that sender's recorded doorbells
+  // m0 .. m0 + count - 1 (what the relay's service thread and its lingering kernels do)
+  std::map<std::pair<uint32_t, uint32_t>, std::vector<std::pair<uint64_t, uint32_t>>> bells;  // -> (m, g)
+  for (const SendParams &P : send)
+    for (uint32_t i = 0; i < P.npaths; ++i)
+      if (P.sp[i].kind == 1) bells[{P.sp[i].relay, P.me}].emplace_back(P.sp[i].m, P.sp[i].g);
+  for (auto &kv : bells) {
+    std::vector<std::pair<uint64_t, uint32_t>> &v = kv.second;
+    std::sort(v.begin(), v.end());
+    for (size_t j = 1; j < v.size(); ++j)
+      if (v[j].first != v[j - 1].first + 1 || v[j].second != v[0].second)
+        return wfail(c, MP_ERR_INVALID, "mp_emu_run: a relay's doorbells must be consecutive with equal lanes");
+    mp_ctx *rc = w->ctxs[kv.first.first];
+    const uint32_t snd = kv.first.second;
+    RelayParams P{};
+    P.me = static_cast<uint32_t>(rc->rank);
+    P.sender = snd;
+    P.g = v[0].second;
+    P.copy_mode = rc->copy_mode;
+    P.stages = shallow_stages();
+    P.timeout_ns = static_cast<uint64_t>(rc->timeout_s * 1e9);
+    P.m0 = v[0].first;
+    P.max_msgs = v.size();
+    P.linger_ns = P.timeout_ns;  // the next doorbell of a recorded message does come
+    P.bells = reinterpret_cast<const BellEntry *>(rc->hseg[rc->rank]) + static_cast<uint64_t>(snd) * kBellRing;
+    P.dec = reinterpret_cast<uint64_t *>(rc->ctrl + rc->L.relay_dec) + static_cast<uint64_t>(snd) * kBellRing * 4;
+    P.exit_cnt = reinterpret_cast<uint32_t *>(rc->ctrl + rc->L.relay_exit + static_cast<uint64_t>(snd) * 128);
+    P.my_ctrl = rc->ctrl;
+    P.sender_ctrl = rc->peers[snd].ctrl;
+    for (int r = 0; r < rc->world; ++r) P.peer[r] = rc->peers[r];
+    P.L = rc->L;
+    P.err = rc->d_err;
+    relay.push_back(P);
+  }
+  for (int r = 0; r < n; ++r) {
+    mp_ctx *cr = ctxs[r];
+    eager.insert(eager.end(), cr->emu_esend.begin(), cr->emu_esend.end());
+  }
+  const size_t n_esend = eager.size();
+  for (int r = 0; r < n; ++r) {
+    mp_ctx *cr = ctxs[r];
+    eager.insert(eager.end(), cr->emu_erecv.begin(), cr->emu_erecv.end());
+  }
+  auto clear = [&] {
+    for (int r = 0; r < n; ++r) {
+      ctxs[r]->emu_send.clear();
+      ctxs[r]->emu_recv.clear();
+      ctxs[r]->emu_esend.clear();
+      ctxs[r]->emu_erecv.clear();
+    }
+  };
+  // Grid: every role co-resident.  Only the direct groups are elastic (any CTA count
+  // moves the same bytes): they share what the fixed roles leave, in proportion to
+  // the CTA counts the real launches would have used.
+  int per_sm = 0;
+  if (int e = emu_capacity(&per_sm)) {
+    clear();
+    return wfail(c, MP_ERR_CUDA, std::string("emu_capacity: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
+  }
+  const uint64_t cap = static_cast<uint64_t>(per_sm) * static_cast<uint64_t>(c->sms);
+  uint64_t fixed = 0, want = 0;
+  for (const SendParams &P : send) {
+    fixed += 1 + (P.nblocks - P.g_direct);
+    want += P.g_direct;
+  }
+  for (const RecvParams &P : recv) fixed += P.nblocks;
+  for (const RelayParams &P : relay) fixed += P.g;
+  for (const EagerParams &P : eager) fixed += P.ctas;
+  if (fixed + send.size() > cap) {
+    clear();
+    return wfail(c, MP_ERR_INVALID, "mp_emu_run: the recorded kernels do not fit one co-resident grid (" +
+                                         std::to_string(fixed + send.size()) + " > " + std::to_string(cap) + " CTAs)");
+  }
+  if (fixed + want > cap)
+    for (SendParams &P : send) {
+      const uint32_t gd = std::max<uint32_t>(1, static_cast<uint32_t>(P.g_direct * (cap - fixed) / want));
+      uint32_t next = gd;
+      for (uint32_t i = 0; i < P.npaths; ++i) {
+        P.sp[i].cta0 = next;
+        next += P.sp[i].g;
+      }
+      P.g_direct = gd;
+      P.nblocks = next;
+    }
+  uint32_t cta = 0;
+  auto add = [&](uint32_t kind, uint32_t cnt, uint32_t idx) {
+    roles.push_back(EmuRole{kind, cta, cnt, idx});
+    cta += cnt;
+  };
+  for (uint32_t i = 0; i < recv.size(); ++i) add(EMU_RECV, recv[i].nblocks, i);
+  for (uint32_t i = 0; i < relay.size(); ++i) add(EMU_RELAY, relay[i].g, i);
+  for (uint32_t i = 0; i < send.size(); ++i) {
+    add(EMU_GATE, 1, i);
+    add(EMU_SEND, send[i].nblocks, i);
+  }
+  for (uint32_t i = 0; i < eager.size(); ++i) add(i < n_esend ? EMU_EAGER_SEND : EMU_EAGER_RECV, eager[i].ctas, i);
+  clear();
+  if (roles.empty()) return MP_OK;
+  // one device block: roles, then the parameter arrays (16-B aligned)
+  auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+  const size_t o_roles = 0, o_send = al(o_roles + roles.size() * sizeof(EmuRole)),
+               o_recv = al(o_send + send.size() * sizeof(SendParams)),
+               o_relay = al(o_recv + recv.size() * sizeof(RecvParams)),
+               o_eager = al(o_relay + relay.size() * sizeof(RelayParams)),
+               o_state = al(o_eager + eager.size() * sizeof(EagerParams)),
+               total = al(o_state + std::max<size_t>(1, relay.size()) * 2 * sizeof(uint64_t));
+  std::vector<uint8_t> h(total, 0);
+  void *d = nullptr;
+  CKW(cudaMalloc(&d, total));
+  uint8_t *db = static_cast<uint8_t *>(d);
+  for (size_t i = 0; i < relay.size(); ++i)
+    relay[i].state = reinterpret_cast<uint64_t *>(db + o_state) + 2 * i;  // the relay's exit record (unread)
+  std::memcpy(h.data() + o_roles, roles.data(), roles.size() * sizeof(EmuRole));
+  if (!send.empty()) std::memcpy(h.data() + o_send, send.data(), send.size() * sizeof(SendParams));
+  if (!recv.empty()) std::memcpy(h.data() + o_recv, recv.data(), recv.size() * sizeof(RecvParams));
+  if (!relay.empty()) std::memcpy(h.data() + o_relay, relay.data(), relay.size() * sizeof(RelayParams));
+  if (!eager.empty()) std::memcpy(h.data() + o_eager, eager.data(), eager.size() * sizeof(EagerParams));
+  EmuTable T{};
+  T.roles = reinterpret_cast<const EmuRole *>(db + o_roles);
+  T.send = reinterpret_cast<const SendParams *>(db + o_send);
+  T.recv = reinterpret_cast<const RecvParams *>(db + o_recv);
+  T.relay = reinterpret_cast<const RelayParams *>(db + o_relay);
+  T.eager = reinterpret_cast<const EagerParams *>(db + o_eager);
+  T.nroles = static_cast<uint32_t>(roles.size());
+  T.nblocks = cta;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(d, h.data(), total, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = static_cast<cudaError_t>(launch_emu(T, stream));
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  cudaFree(d);
+  if (e != cudaSuccess) return wfail(c, MP_ERR_CUDA, std::string("mp_emu_run: ") + cudaGetErrorString(e));
+  for (int r = 0; r < n; ++r) {
+    int32_t de = 0;
+    CKW(cudaMemcpy(&de, ctxs[r]->d_err, sizeof(de), cudaMemcpyDeviceToHost));
+    if (de == DERR_TIMEOUT) return wfail(c, MP_ERR_TIMEOUT, "rank " + std::to_string(r) + ": a device-side wait timed out");
+    if (de == DERR_MISMATCH)
+      return wfail(c, MP_ERR_MISMATCH, "rank " + std::to_string(r) + ": send/recv size or tag mismatch");
+  }
   return MP_OK;
 }
 

@@ -15,7 +15,7 @@ from . import _build
 MP_MAX_PATHS = 16
 MP_PATH_DIRECT, MP_PATH_GPU, MP_PATH_HOST = 0, 1, 2
 MP_MODEL_PAPER, MP_MODEL_B200 = 0, 1
-MP_INIT_MODEL_ONLY, MP_INIT_NO_CALIBRATE = 1, 2
+MP_INIT_MODEL_ONLY, MP_INIT_NO_CALIBRATE, MP_INIT_EMULATED = 1, 2, 4
 MP_OK, MP_ERR_INVALID, MP_ERR_CUDA, MP_ERR_TOPOLOGY, MP_ERR_NOMEM, MP_ERR_STATE = 0, -1, -2, -3, -4, -5
 MP_ERR_UNSUPPORTED, MP_ERR_TIMEOUT, MP_ERR_MISMATCH = -6, -7, -8
 
@@ -197,6 +197,9 @@ def lib():
             "mp_get_host_duplex": (C.c_int, [P, C.c_int, C.POINTER(C.c_double)]),
             "mp_get_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
             "mp_set_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
+            "mp_init_emulated": (C.c_int, [C.POINTER(P), C.POINTER(mp_init_args)]),
+            "mp_emu_run": (C.c_int, [C.POINTER(P), C.c_int, P]),
+            "mp_finalize_emulated": (C.c_int, [C.POINTER(P), C.c_int]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
                                        C.POINTER(C.c_double)]),
@@ -219,7 +222,8 @@ def exported_symbols() -> List[str]:
             "mp_coll_plan_build", "mp_alltoall", "mp_allreduce",
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
             "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_calibrate_wake", "mp_fit_window",
-            "mp_get_topology", "mp_set_topology", "mp_set_submit_time", "mp_get_submit_time"]
+            "mp_get_topology", "mp_set_topology", "mp_set_submit_time", "mp_get_submit_time",
+            "mp_init_emulated", "mp_emu_run", "mp_finalize_emulated"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -321,11 +325,20 @@ class Context:
         self.h = h
         self.world, self.rank = world, rank
 
+    @classmethod
+    def _wrap(cls, h, rank, world):
+        self = cls.__new__(cls)
+        self.h, self.rank, self.world = C.c_void_p(h), rank, world
+        self._emulated = True
+        return self
+
     def _ck(self, st):
         if st != 0:
             raise MPError(st, lib().mp_last_error(self.h).decode())
 
     def close(self):
+        if getattr(self, "_emulated", False):  # EmulatedWorld.close() tears the world down
+            return
         if getattr(self, "h", None):
             lib().mp_finalize(self.h)
             self.h = None
@@ -594,3 +607,41 @@ def as_tensor(ptr: int, n: int):
     """A torch uint8 tensor viewing n bytes of device memory at ptr (e.g. from mp_alloc)."""
     import torch
     return torch.as_tensor(_CudaArray(ptr, n), device="cuda")
+
+
+class EmulatedWorld:
+    """mp_init_emulated / mp_emu_run / mp_finalize_emulated: every rank of a world as a
+    Context of this process on one GPU.  ``ctx[r].send`` / ``ctx[r].recv`` record;
+    ``run()`` launches everything recorded as ONE cooperative grid and waits for it."""
+
+    def __init__(self, world, device=0, host_path=-1, slots=0, relay_ctas=0, heap_bytes=0,
+                 slot_bytes=0, timeout_s=0.0, param_file=None):
+        L = lib()
+        a = mp_init_args()
+        a.rank, a.world, a.device, a.flags = 0, world, device, MP_INIT_NO_CALIBRATE
+        a.n_loop_relays, a.host_path, a.slots, a.relay_ctas = -1, host_path, slots, relay_ctas
+        a.heap_bytes, a.slot_bytes, a.timeout_s = heap_bytes, slot_bytes, timeout_s
+        a.allgather = ALLGATHER()
+        a.param_file = param_file.encode() if param_file else None
+        self._h = (C.c_void_p * world)()
+        st = L.mp_init_emulated(self._h, C.byref(a))
+        if st != 0:
+            raise MPError(st, "mp_init_emulated failed")
+        self.world = world
+        self.ctx = [Context._wrap(self._h[r], r, world) for r in range(world)]
+
+    def run(self, stream=None):
+        st = lib().mp_emu_run(self._h, self.world, _stream(stream))
+        if st != 0:
+            raise MPError(st, lib().mp_last_error(self._h[0]).decode())
+
+    def close(self):
+        if self.ctx:
+            lib().mp_finalize_emulated(self._h, self.world)
+            self.ctx = []
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()

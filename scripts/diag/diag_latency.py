@@ -1,6 +1,6 @@
 #!/usr/bin/env python3
 """osu_latency-style ping-pong on the multi-rank engine (torchrun, 2 ranks; both may
-share one GPU under MPS: scripts/with_mps.sh).  Rank 0 sends n bytes to rank 1 and
+share one GPU under MPS — retired: ranks now get one GPU each).  Rank 0 sends n bytes to rank 1 and
 waits for n bytes back; one-way latency = median round trip / 2 over `iters` (host
 clock around stream-synchronised send/recv, as OSU times blocking MPI calls).
 MPX_EAGER=0 forces the rendezvous protocol.  Prints JSON lines from rank 0."""
@@ -21,7 +21,8 @@ def main():
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     dist.init_process_group("gloo")
     rank = dist.get_rank()
-    dev = 0 if os.environ.get("MPX_BENCH_SAME_GPU") == "1" else int(os.environ.get("LOCAL_RANK", 0))
+    dev = int(os.environ.get("LOCAL_RANK", 0))
+    assert torch.cuda.device_count() > dev, "one GPU per rank"
     torch.cuda.set_device(dev)
     s_tx, s_rx = torch.cuda.Stream(), torch.cuda.Stream()
     big = 1 << 20

@@ -21,7 +21,8 @@ def main():
     from paper_conf_sc_sojoodiasfga25_b200 import mp
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
-    dev = 0 if os.environ.get("MPX_BENCH_SAME_GPU") == "1" else int(os.environ.get("LOCAL_RANK", 0))
+    dev = int(os.environ.get("LOCAL_RANK", 0))
+    assert torch.cuda.device_count() > dev, "one GPU per rank"
     torch.cuda.set_device(dev)
     n = int(os.environ.get("DIAG_BYTES", 64 * MiB))
     K = int(os.environ.get("DIAG_K", "20"))

@@ -14,8 +14,8 @@ Ranks 0 and 1 are the pair; ranks 2.. serve as relay GPUs for the model's config
   ce       the same window as copy-engine peer copies (cudaMemcpyAsync into the
            IPC-mapped receive buffer: what cudaMemcpyPeerAsync does)
   nccl     the same window as NCCL send/recv (measured before mp_init)
-Predicted GB/s (mp_select t_pred) is reported next to the measured one.  All ranks may
-share one GPU (MPX_BENCH_SAME_GPU=1 under MPS: a functional run, not an NVLink number).
+Predicted GB/s (mp_select t_pred) is reported next to the measured one.  One GPU per
+rank (ranks whose kernels wait on one another never share a GPU).
 """
 from __future__ import annotations
 
@@ -48,8 +48,8 @@ def main():
     a = ap.parse_args()
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
-    same_gpu = os.environ.get("MPX_BENCH_SAME_GPU") == "1"
-    dev = 0 if same_gpu else int(os.environ.get("LOCAL_RANK", 0))
+    dev = int(os.environ.get("LOCAL_RANK", 0))
+    assert torch.cuda.device_count() > dev, "one GPU per rank"
     torch.cuda.set_device(dev)
     windows = [int(w) for w in a.windows.split(",")]
     sizes = []
@@ -76,35 +76,34 @@ def main():
         return float(t[0])
 
     # ---- NCCL send/recv windows (before mp_init: no NCCL kernel beside the engine's)
-    if not same_gpu:
-        try:
-            g = dist.new_group(backend="nccl")
-            rb = torch.empty(big, dtype=torch.uint8, device="cuda") if pair else None
-            for n in sizes:
-                skip, it = iters_for(n)
-                for w in windows:
-                    dist.barrier()
-                    if pair:
-                        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                        for i in range(skip + it):
-                            if i == skip:
-                                e0.record()
-                            ops = [dist.P2POp(dist.isend if rank == 0 else dist.irecv,
-                                              src[:n] if rank == 0 else rb[:n], peer, g) for _ in range(w)]
-                            for q in dist.batch_isend_irecv(ops):
-                                q.wait()
-                        e1.record()
-                        torch.cuda.synchronize()
-                        t = e0.elapsed_time(e1) * 1e-3 / it
-                    else:
-                        t = 0.0
-                    t = gmax(t)
-                    emit({"test": "bw", "impl": "nccl", "n": n, "window": w, "GBps": n * w / t / 1e9})
-            dist.destroy_process_group(g)
-            del rb
-            torch.cuda.synchronize()
-        except Exception as exc:  # context, not the product
-            emit({"impl": "nccl", "error": repr(exc)})
+    try:
+        g = dist.new_group(backend="nccl")
+        rb = torch.empty(big, dtype=torch.uint8, device="cuda") if pair else None
+        for n in sizes:
+            skip, it = iters_for(n)
+            for w in windows:
+                dist.barrier()
+                if pair:
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    for i in range(skip + it):
+                        if i == skip:
+                            e0.record()
+                        ops = [dist.P2POp(dist.isend if rank == 0 else dist.irecv,
+                                          src[:n] if rank == 0 else rb[:n], peer, g) for _ in range(w)]
+                        for q in dist.batch_isend_irecv(ops):
+                            q.wait()
+                    e1.record()
+                    torch.cuda.synchronize()
+                    t = e0.elapsed_time(e1) * 1e-3 / it
+                else:
+                    t = 0.0
+                t = gmax(t)
+                emit({"test": "bw", "impl": "nccl", "n": n, "window": w, "GBps": n * w / t / 1e9})
+        dist.destroy_process_group(g)
+        del rb
+        torch.cuda.synchronize()
+    except Exception as exc:  # context, not the product
+        emit({"impl": "nccl", "error": repr(exc)})
 
     ctx = mdist.context_from_dist(device=dev, calibrate=True, heap_bytes=2 * big + 64 * MiB, timeout_s=60.0)
     ctx.set_options(mode=mp.MP_MODEL_B200)

@@ -1,6 +1,6 @@
 #!/bin/bash
 # Round-2 GPU session: tests, bench (both arms), ncu launch list + full captures of the
-# top kernels, multi-rank harness under MPS, per-rank NVLink ncu pass (only on a box
+# top kernels, the emulated multi-rank world, per-rank NVLink ncu pass (only on a box
 # with >= 2 GPUs), loopback sweep.
 # Usage (under gpurun): bash scripts/r02_profile.sh <tag>
 TAG=${1:-r02/prof}
@@ -18,7 +18,8 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"dir
   python bench.py --steps 5 --warmup 3 --no-cpu-baseline --params $OUT/params.txt > $OUT/ncu_direct.log 2>&1
 RELAY_K=32 timeout 600 ncu --set full --clock-control none --import-source on -k regex:xfer_kernel -s 2 -c 1 \
   -o $OUT/relay_full python scripts/relay_one.py > $OUT/ncu_relay.log 2>&1
-STEPS=20 TMO=600 bash scripts/r02_world.sh $TAG/world
+# multi-rank engine on one GPU: the emulated world (one cooperative grid over every rank)
+timeout 900 python -m pytest tests/test_emulated_gpu.py -q -p no:cacheprovider > $OUT/pytest_emulated.log 2>&1
 NG=$(nvidia-smi -L | wc -l)
 if [ "$NG" -ge 2 ]; then  # per-rank NVLink counters need one GPU per rank (ncu serialises a shared device)
   NCU_OUT=$OUT/ncu_world timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node $NG \

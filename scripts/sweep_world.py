@@ -13,8 +13,8 @@ fit a 32 MiB slot are skipped), then a step-1/128 refinement around the best.  E
 config is timed as an OMB window of W back-to-back messages (median of `reps`
 windows, max over the sender's and the receiver's device time); the best of the sweep
 and the B200- and paper-mode picks are re-timed with 3x the repetitions.
-Every rank enumerates the same configs; ranks 2.. only relay.  All ranks may share
-one GPU (MPX_BENCH_SAME_GPU=1 under MPS: a functional run, not an NVLink number).
+Every rank enumerates the same configs; ranks 2.. only relay.  One GPU per rank
+(ranks whose kernels wait on one another never share a GPU).
 """
 from __future__ import annotations
 
@@ -73,8 +73,8 @@ def main():
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
     assert world >= 4, "config 2 needs GPU0, GPU1 and two relays"
-    same_gpu = os.environ.get("MPX_BENCH_SAME_GPU") == "1"
-    dev = 0 if same_gpu else int(os.environ.get("LOCAL_RANK", 0))
+    dev = int(os.environ.get("LOCAL_RANK", 0))
+    assert torch.cuda.device_count() > dev, "one GPU per rank"
     torch.cuda.set_device(dev)
     sizes = [int(s) * MiB for s in a.sizes.split(",")]
     big = max(sizes)
@@ -117,7 +117,7 @@ def main():
         ts.sort()
         return ts[len(ts) // 2]
 
-    report = {"paths": paths, "model": ctx.get_model(0, 1), "topology": ctx.topology(), "same_gpu": same_gpu,
+    report = {"paths": paths, "model": ctx.get_model(0, 1), "topology": ctx.topology(),
               "sizes": {}}
     ks = [1, 2, 4, 8, 16, 32, 64]
     for n in sizes:

@@ -1,4 +1,6 @@
-"""Worker for the multi-rank tests (one process per rank; all ranks may share one GPU).
+"""Worker for the multi-rank tests (one process per rank, one GPU per rank: rank r on
+device r — ranks whose kernels wait on one another never share a GPU; the one-GPU
+stand-in is the emulated world, tests/test_emulated_gpu.py).
 
     python tests/_world_worker.py <rank> <world> <port> <scenario>
 
@@ -20,6 +22,7 @@ import torch  # noqa: E402
 import torch.distributed as dist  # noqa: E402
 
 MiB = 1 << 20
+DEV = int(sys.argv[1]) if len(sys.argv) > 1 and sys.argv[1].isdigit() else 0  # this rank's GPU
 
 
 def scenario_gloo_model(rank, world):
@@ -54,7 +57,7 @@ def scenario_engine(rank, world):
     from oracle import transfer as X
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     # Everything CUDA this process will need is initialised BEFORE mp_init: with
     # (round 1: a persistent relay kernel forbade an idle-device wait later; round 2's
     # relay kernels are bounded — scenario "devsync" — but this order is kept), and driver calls that
@@ -66,7 +69,7 @@ def scenario_engine(rank, world):
     assert int(src_buf[:16].cpu().sum()) >= 0
     torch.cuda.synchronize()
     print(f"rank {rank}: init", flush=True)
-    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=DEV, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0)
     if world >= 3:
         # collective Step 1 after mp_init (the relay service keeps running)
@@ -193,13 +196,13 @@ def scenario_faults(rank, world):
     import synth
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
     src = torch.empty(2 * MiB, dtype=torch.uint8, device="cuda")
     src.copy_(torch.from_numpy(synth.payload(2 * MiB, 0)))
     torch.cuda.synchronize()
     for fault in ("mismatch", "timeout", "eager_mismatch"):
-        c = mdist.context_from_dist(device=0, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+        c = mdist.context_from_dist(device=DEV, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                     timeout_s=3.0)
         nb = 4096 if fault == "eager_mismatch" else 2 * MiB   # 2 MiB: past the eager limit (rendezvous)
         if rank == 0 and fault != "timeout":
@@ -232,13 +235,13 @@ def scenario_register(rank, world):
     from oracle import transfer as X
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
     big = torch.zeros(16 * MiB, dtype=torch.uint8, device="cuda")        # rank 1's targets
     ring = torch.zeros(4 * MiB, dtype=torch.uint8, device="cuda")        # every rank's ring target
     src_buf = torch.empty(8 * MiB, dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=DEV, heap_bytes=16 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0)
     ps = c.paths(0, 1)
     kinds = [k for k, _ in ps]
@@ -316,11 +319,11 @@ def scenario_eager(rank, world):
 
     import synth
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
     src_buf = torch.empty(3 * MiB, dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=DEV, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0)
     sizes = [1, 17, 4095, 16384, 16385, 3 * 16384 + 5, 65537, 300000, MiB - 1, MiB, MiB + 1]
     offs = [(0, 0), (1, 1), (3, 7), (16, 5)]
@@ -368,12 +371,12 @@ def scenario_coll(rank, world):
     from oracle import collectives as OCL
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
     BMAX = 300 * 1024 + 5
     send = torch.zeros(world * BMAX + 64, dtype=torch.uint8, device="cuda")
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=DEV, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0)
     rbuf = c.alloc(world * BMAX + 64)
     rview = mp.as_tensor(rbuf, world * BMAX + 64)
@@ -447,9 +450,9 @@ def scenario_devsync(rank, world):
     from oracle import transfer as X
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
-    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=DEV, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0, calibrate=False)
     # CUDA work created only now, after mp_init: a fresh allocation, a generator kernel
     src_buf = torch.empty(8 * MiB, dtype=torch.uint8, device="cuda")
@@ -541,9 +544,9 @@ def scenario_relay_burst(rank, world):
     from oracle import transfer as X
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
-    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
+    c = mdist.context_from_dist(device=DEV, heap_bytes=64 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4,
                                 timeout_s=60.0, calibrate=False)
     ps = c.paths(0, 1)
     n = 1 * MiB + 4099
@@ -593,13 +596,13 @@ def scenario_full_size(rank, world):
     once; payloads compared whole on the device against the source (O1: dst == src)."""
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     n = (1 << 30) + 4099
     stream = torch.cuda.Stream()
     src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
                         generator=torch.Generator(device="cuda").manual_seed(20251116)) if rank in (0, 1) else None
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=n + 64 * MiB, timeout_s=120.0, calibrate=False)
+    c = mdist.context_from_dist(device=DEV, heap_bytes=n + 64 * MiB, timeout_s=120.0, calibrate=False)
     rbuf = c.alloc(n) if rank == 1 else None
     ps = c.paths(0, 1)
     cfgs = []
@@ -636,13 +639,13 @@ def scenario_wake(rank, world):
     bit-exact and the B200 pick's prediction includes the wake."""
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     stream = torch.cuda.Stream()
     n = 8 * MiB + 4099
     src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
                         generator=torch.Generator(device="cuda").manual_seed(7)) if rank == 0 else None
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=64 * MiB, timeout_s=60.0, calibrate=False)
+    c = mdist.context_from_dist(device=DEV, heap_bytes=64 * MiB, timeout_s=60.0, calibrate=False)
     c.calibrate(sizes=[4 * MiB, 8 * MiB, 16 * MiB], reps=2)   # Step 1, then the wake probe
     wakes = {}
     for s_ in range(world):
@@ -712,12 +715,12 @@ def scenario_bell_flow(rank, world):
     resident out of ring order (the cross-stream ring order).  Every message bit-exact."""
     from paper_conf_sc_sojoodiasfga25_b200 import dist as mdist
     from paper_conf_sc_sojoodiasfga25_b200 import mp
-    torch.cuda.set_device(0)
+    torch.cuda.set_device(DEV)
     n, M = 1 * MiB + 4099, 56
     gen = torch.Generator(device="cuda").manual_seed(11)
     src = torch.randint(0, 256, (2 * M, n), dtype=torch.uint8, device="cuda", generator=gen)
     torch.cuda.synchronize()
-    c = mdist.context_from_dist(device=0, heap_bytes=M * (n + 4096) + 8 * MiB, timeout_s=60.0, calibrate=False)
+    c = mdist.context_from_dist(device=DEV, heap_bytes=M * (n + 4096) + 8 * MiB, timeout_s=60.0, calibrate=False)
     streams = [torch.cuda.Stream() for _ in range(2 * M)]
     peers = (1, 3)
     if rank == 0:

@@ -1,0 +1,220 @@
+"""The multi-rank engine on ONE GPU as an emulated world (include/mp.h: mp_init_emulated,
+mp_emu_run): every rank is a context of this process, and every rank's kernels — the
+send gate and send CTAs, the receive CTAs, the relay kernels a relay rank's service
+thread would launch, the eager kernels — run as CTA ranges of ONE cooperative launch.
+Ranks whose kernels wait on one another are then co-resident by construction, never
+separate launches sharing the GPU (the B200 profiling guide's rule when there are fewer
+GPUs than ranks).  Payloads are checked byte for byte against the oracle's reference
+transfer (oracle/transfer.py: replay of the split)."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import transfer as X
+
+pytestmark = pytest.mark.gpu
+
+MiB = 1 << 20
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    torch.cuda.set_device(0)
+    return torch
+
+
+def world(w, **kw):
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    args = dict(device=0, heap_bytes=96 * MiB, slot_bytes=1 * MiB, slots=2, relay_ctas=4, timeout_s=20.0)
+    args.update(kw)
+    return mp.EmulatedWorld(w, **args)
+
+
+def expected(host, nb, ks, ps):
+    exp = np.zeros(len(host), dtype=np.uint8)
+    if nb is None:
+        exp[:] = host
+    else:
+        X.replay(host, nb, ks, [k for k, _ in ps], 256, exp)
+    return exp
+
+
+def fill(torch, n, seed):
+    host = synth.payload(n, seed)
+    return host, torch.from_numpy(host).cuda()
+
+
+def cases_for(ps, n):
+    """Direct only, one relay alone (k = 5), host alone (k = 4), every path at once."""
+    np_ = len(ps)
+    out = [([n] + [0] * (np_ - 1), [1] + [0] * (np_ - 1))]
+    if np_ > 2:
+        nb, ks = [0] * np_, [1] + [0] * (np_ - 1)
+        nb[1], ks[1] = n, 5
+        out.append((nb, ks))
+    nb, ks = [0] * np_, [1] + [0] * (np_ - 1)
+    nb[-1], ks[-1] = n, 4
+    out.append((nb, ks))
+    nb = [0] + [256 * 1024] * (np_ - 1)
+    nb[0] = n - sum(nb)
+    out.append((nb, [1] + [2] * (np_ - 1)))
+    return out
+
+
+@pytest.mark.parametrize("w", [2, 3, 4])
+def test_emulated_pair_every_path_kind_bit_exact(torch_cuda, w):
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    with world(w) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        assert len(ps) == w  # direct + (w - 2) relays + host
+        n = 3 * MiB + 4099
+        for i, (nb, ks) in enumerate(cases_for(ps, n) + [(None, None)]):
+            host, src = fill(torch, n, i)
+            dst = c1.alloc(n)
+            mp.as_tensor(dst, n).zero_()
+            torch.cuda.synchronize()
+            c0.send(src, n, 1, tag=100 + i, cfg=c0.make_config(nb, ks, 0, 1) if nb else None)
+            c1.recv(dst, n, 0, tag=100 + i)
+            W.run()
+            got = mp.as_tensor(dst, n).cpu().numpy()
+            assert np.array_equal(got, expected(host, nb, ks, ps)), f"world {w} case {i} {nb} {ks}"
+            c1.free(dst)
+        assert c0.launches() > 0
+
+
+def test_emulated_windows_ring_wrap_bidirectional_eager_zero(torch_cuda):
+    """One run holding a window of 4 messages each way between ranks 0 and 1 (every path,
+    k = 2 on 2-slot rings: the relay and host rings wrap twice; the relay role serves
+    four doorbells through the lingering relay's next-message decisions), plus an eager
+    message, a zero-byte message and a message relayed 2 -> 3 through ranks 0 and 1."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    with world(4) as W:
+        c = W.ctx
+        ps = c[0].paths(0, 1)
+        n = 2 * MiB + 77
+        nb = [0] + [256 * 1024] * (len(ps) - 1)
+        nb[0] = n - sum(nb)
+        ks = [1] + [2] * (len(ps) - 1)
+        checks = []
+        for s, d in ((0, 1), (1, 0)):
+            for m in range(4):
+                host, src = fill(torch, n, 10 * s + m)
+                dst = c[d].alloc(n)
+                checks.append((d, dst, n, expected(host, nb, ks, c[s].paths(s, d)), src))
+                c[s].send(src, n, d, tag=m, cfg=c[s].make_config(nb, ks, s, d))
+                c[d].recv(dst, n, s, tag=m)
+        # eager (<= 1 MiB: no rendezvous) and zero-byte messages 2 -> 3
+        host_e, src_e = fill(torch, 300 * 1000 + 5, 99)
+        dst_e = c[3].alloc(len(host_e))
+        c[2].send(src_e, len(host_e), 3, tag=7)
+        c[3].recv(dst_e, len(host_e), 2, tag=7)
+        c[2].send(src_e, 0, 3, tag=8)
+        c[3].recv(dst_e, 0, 2, tag=8)
+        checks.append((3, dst_e, len(host_e), host_e, src_e))
+        # 2 -> 3 through both other ranks as relays, concurrently with the 0 <-> 1 windows
+        ps23 = c[2].paths(2, 3)
+        nb23 = [0] * len(ps23)
+        ks23 = [1] + [0] * (len(ps23) - 1)
+        for i, (k, v) in enumerate(ps23):
+            if k == 1:
+                nb23[i], ks23[i] = MiB, 3
+        n23 = sum(nb23) + 12345
+        nb23[0] = 12345
+        host23, src23 = fill(torch, n23, 123)
+        dst23 = c[3].alloc(n23)
+        c[2].send(src23, n23, 3, tag=9, cfg=c[2].make_config(nb23, ks23, 2, 3))
+        c[3].recv(dst23, n23, 2, tag=9)
+        checks.append((3, dst23, n23, expected(host23, nb23, ks23, ps23), src23))
+        torch.cuda.synchronize()
+        W.run()
+        for j, (d, p, nn, exp, _) in enumerate(checks):
+            assert np.array_equal(mp.as_tensor(p, nn).cpu().numpy(), exp), f"message {j}"
+        # the pairs' sequence state carries over: a second run on the same world
+        host, src = fill(torch, n, 55)
+        dst = c[1].alloc(n)
+        c[0].send(src, n, 1, tag=1, cfg=c[0].make_config(nb, ks, 0, 1))
+        c[1].recv(dst, n, 0, tag=1)
+        W.run()
+        assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, nb, ks, ps))
+
+
+def test_emulated_config3_shape_full_relay_fan(torch_cuda):
+    """BASELINE config 3's shape on one GPU: rank 0 -> rank 1 over direct + 6 relay
+    ranks + the pinned host path (world 8), every path carrying bytes, 64 MiB + 4099 B."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    with world(8, heap_bytes=80 * MiB, slot_bytes=4 * MiB, slots=2) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        assert [k for k, _ in ps] == [0] + [1] * 6 + [2]
+        n = 64 * MiB + 4099
+        nb = [0] + [6 * MiB] * 6 + [2 * MiB]
+        nb[0] = n - sum(nb)
+        ks = [1] + [4] * 6 + [3]
+        host, src = fill(torch, n, 3)
+        dst = c1.alloc(n)
+        c0.send(src, n, 1, tag=3, cfg=c0.make_config(nb, ks, 0, 1))
+        c1.recv(dst, n, 0, tag=3)
+        torch.cuda.synchronize()
+        W.run()
+        assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, nb, ks, ps))
+
+
+def test_emulated_all_pairs_concurrent(torch_cuda):
+    """BASELINE config 5's shape (world 4): every ordered pair sends at once, each over
+    direct + both other ranks as relays + host, in one grid."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    with world(4) as W:
+        c = W.ctx
+        n = 1 * MiB + 2 * 256 * 1024 + 513
+        checks = []
+        for s in range(4):
+            for d in range(4):
+                if s == d:
+                    continue
+                ps = c[s].paths(s, d)
+                nb = [0] + [256 * 1024] * (len(ps) - 1)
+                nb[0] = n - sum(nb)
+                ks = [1] + [2] * (len(ps) - 1)
+                host, src = fill(torch, n, 16 * s + d)
+                dst = c[d].alloc(n)
+                c[s].send(src, n, d, tag=s, cfg=c[s].make_config(nb, ks, s, d))
+                c[d].recv(dst, n, s, tag=s)
+                checks.append((d, dst, expected(host, nb, ks, ps), src))
+        torch.cuda.synchronize()
+        W.run()
+        for j, (d, p, exp, _) in enumerate(checks):
+            assert np.array_equal(mp.as_tensor(p, n).cpu().numpy(), exp), f"pair message {j}"
+
+
+def test_emulated_faults_reported(torch_cuda):
+    """A tag mismatch is MP_ERR_MISMATCH; a send nobody receives is MP_ERR_TIMEOUT —
+    both from the device, neither hangs; the unsupported calls say so."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    with world(3, timeout_s=2.0) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        n = 2 * MiB
+        _, src = fill(torch, n, 1)
+        dst = c1.alloc(n)
+        c0.send(src, n, 1, tag=1)
+        c1.recv(dst, n, 0, tag=2)
+        with pytest.raises(mp.MPError) as e:
+            W.run()
+        assert e.value.status == mp.MP_ERR_MISMATCH
+        with pytest.raises(mp.MPError) as e:
+            c0.calibrate()
+        assert e.value.status == mp.MP_ERR_UNSUPPORTED
+    with world(2, timeout_s=1.0) as W:
+        _, src = fill(torch, 2 * MiB, 1)
+        W.ctx[0].send(src, 2 * MiB, 1, tag=1)
+        with pytest.raises(mp.MPError) as e:
+            W.run()
+        assert e.value.status == mp.MP_ERR_TIMEOUT

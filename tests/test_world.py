@@ -2,8 +2,8 @@
 
 CPU: the bootstrap all-gather and the per-pair model selection are consistent
 across ranks.  GPU: the real multi-rank engine (IPC-mapped heaps, on-demand relay
-kernels, shared pinned host ring) with all ranks on one B200 (same-device CUDA IPC),
-bit-exact against the oracle's reference transfer."""
+kernels, shared pinned host ring), rank r on GPU r,
+bit-exact against the oracle's reference transfer; one GPU per rank (need_gpus)."""
 import os
 import socket
 import subprocess
@@ -52,6 +52,18 @@ def run_world(world, scenario, timeout, env=None):
     assert not bad, "\n".join(f"rank {r} failed (rc {rc}):\n{out[:2000]}\n...\n{out[-2000:]}" for r, rc, out in bad)
 
 
+def need_gpus(world):
+    """A multi-rank GPU test runs with one GPU per rank.  Ranks whose kernels wait on one
+    another are never separate launches sharing a GPU (B200 profiling guide: nothing
+    guarantees they run at the same time; processes spinning on one another raised
+    Xid 109 there).  With fewer GPUs the same engine runs as an emulated world —
+    one cooperative grid over every rank's kernels: tests/test_emulated_gpu.py."""
+    torch = pytest.importorskip("torch")
+    n = torch.cuda.device_count() if torch.cuda.is_available() else 0
+    if n < world:
+        pytest.skip(f"needs {world} GPUs (one per rank), found {n}; one-GPU coverage: test_emulated_gpu.py")
+
+
 @pytest.mark.parametrize("world", [2, 3])
 def test_gloo_bootstrap_and_consistent_selection(world):
     run_world(world, "gloo_model", timeout=240)
@@ -65,41 +77,29 @@ def test_bench_config3_roles_and_plan(world):
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("world", [2, 3])
-def test_multirank_engine_same_gpu(world):
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+def test_multirank_engine(world):
+    need_gpus(world)
     run_world(world, "engine", timeout=400)
 
 
 @pytest.mark.gpu
 def test_multirank_faults_reported_not_hung():
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(2)
     run_world(2, "faults", timeout=300)
 
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("world", [2, 3])
 def test_multirank_registered_buffers(world):
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(world)
     run_world(world, "register", timeout=400)
 
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("world", [2, 3, 4])
 def test_multirank_collectives(world):
-    # NEXT f3: mp_alltoall / mp_allreduce through the multi-rank engine, all ranks on one GPU
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    # NEXT f3: mp_alltoall / mp_allreduce through the multi-rank engine
+    need_gpus(world)
     run_world(world, "coll", timeout=600)
 
 
@@ -107,10 +107,7 @@ def test_multirank_collectives(world):
 @pytest.mark.parametrize("world", [2, 3])
 def test_multirank_eager_protocol(world):
     # reading C23: small messages skip the rendezvous
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(world)
     run_world(world, "eager", timeout=400)
 
 
@@ -118,10 +115,7 @@ def test_multirank_eager_protocol(world):
 def test_multirank_device_sync_with_relays():
     # relay kernels are bounded launches (doorbell thread), so
     # torch.cuda.synchronize() between messages and during a relayed message is safe
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(3)
     run_world(3, "devsync", timeout=400)
 
 
@@ -129,10 +123,7 @@ def test_multirank_device_sync_with_relays():
 def test_multirank_engine_shallow_staged_pipelines():
     # every staged launch at 4 stages (MPX_STAGES=4): the send / recv / relay kernel
     # instances a sender with many relays gets (the default picks 6 when room allows)
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(3)
     run_world(3, "engine", timeout=400, env={"MPX_STAGES": "4"})
 
 
@@ -140,32 +131,23 @@ def test_multirank_engine_shallow_staged_pipelines():
 def test_multirank_relay_burst_doorbell_wrap_and_linger():
     # 160 relayed messages: doorbell / decision rings wrap, lingering relay kernels
     # switch between streamed and per-chunk lanes, relaunch after quiet periods
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(3)
     run_world(3, "relay_burst", timeout=400)
 
 
 @pytest.mark.gpu
 def test_multirank_config3_full_size_bit_exact():
     # BASELINE.json config 3 (1 GiB + 4099 B) through the multi-rank engine in the bench's
-    # launch configuration: B200 pick, paper pick, every path at once; world 3 on one GPU
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    # launch configuration: B200 pick, paper pick, every path at once; world 3
+    need_gpus(3)
     run_world(3, "full_size", timeout=600)
 
 
 @pytest.mark.gpu
 def test_multirank_relay_wake_calibration():
     # reading C28: the collective wake probe after Step 1, the env override, and
-    # relayed messages after it (world 3 on one GPU)
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    # relayed messages after it (world 3)
+    need_gpus(3)
     run_world(3, "wake", timeout=400)
 
 
@@ -173,8 +155,5 @@ def test_multirank_relay_wake_calibration():
 def test_multirank_doorbell_flow_control():
     # 112 relayed messages in flight through one relay (two receivers, 112 streams,
     # receives posted last-first): doorbell flow control and cross-stream ring order
-    pytest.importorskip("torch")
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no GPU")
+    need_gpus(4)
     run_world(4, "bell_flow", timeout=500)
