@@ -218,3 +218,68 @@ def test_emulated_faults_reported(torch_cuda):
         with pytest.raises(mp.MPError) as e:
             W.run()
         assert e.value.status == mp.MP_ERR_TIMEOUT
+
+
+def test_emulated_relay_burst_doorbell_wrap_and_eager_wrap(torch_cuda):
+    """160 relayed messages rank 0 -> rank 1 through relay rank 2 in 20 runs of 8 (the
+    doorbell ring of 64 and the relay's decision ring wrap 2.5 times; each run's relay
+    role serves 8 doorbells), sources alternately co-aligned and misaligned (streamed
+    and per-chunk relay lanes, message by message), plus one eager message per run
+    (the 8 eager slots wrap)."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    with world(3) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        n, M = 1 * MiB + 4099, 8
+        nb = [0] * len(ps)
+        nb[1] = n
+        ks = [1] + [0] * (len(ps) - 1)
+        ks[1] = 3
+        cfg = c0.make_config(nb, ks, 0, 1)
+        src_buf = torch.empty(M * (n + 64), dtype=torch.uint8, device="cuda")
+        bufs = [c1.alloc(n) for _ in range(M)]
+        ne = 40000 + 3
+        ebuf = c1.alloc(ne)
+        for run in range(20):
+            payloads = [synth.payload(n, 1000 + run * M + i) for i in range(M)]
+            for i in range(M):
+                off = i * (n + 64) + (0 if (run + i) % 2 == 0 else 7)
+                v = src_buf[off:off + n]
+                v.copy_(torch.from_numpy(payloads[i]))
+                c0.send(v, n, 1, tag=run * M + i, cfg=cfg)
+                c1.recv(bufs[i], n, 0, tag=run * M + i)
+            he, se = fill(torch, ne, 5000 + run)
+            c0.send(se, ne, 1, tag=-1 - run)
+            c1.recv(ebuf, ne, 0, tag=-1 - run)
+            torch.cuda.synchronize()
+            W.run()
+            for i in range(M):
+                assert np.array_equal(mp.as_tensor(bufs[i], n).cpu().numpy(), expected(payloads[i], nb, ks, ps)), \
+                    f"run {run} message {i}"
+            assert np.array_equal(mp.as_tensor(ebuf, ne).cpu().numpy(), he), f"run {run} eager"
+
+
+def test_emulated_config3_full_size_default_launch_config(torch_cuda):
+    """BASELINE config 3's message size (1 GiB + 4099 B) in the engine's default launch
+    configuration (4 slots of 32 MiB, 16 lanes per stage group, deep staged pipelines):
+    every path at once and direct-only, world 3, compared on the device against the
+    oracle's replay."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    n = (1 << 30) + 4099
+    with mp.EmulatedWorld(3, device=0, heap_bytes=n + 64 * MiB, timeout_s=60.0) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        host = synth.payload(n, 33)
+        src = torch.from_numpy(host).cuda()
+        dst = c1.alloc(n)
+        for nb, ks in (([n - 448 * MiB, 320 * MiB, 128 * MiB], [1, 12, 5]), ([n, 0, 0], [1, 0, 0])):
+            mp.as_tensor(dst, n).zero_()
+            torch.cuda.synchronize()
+            c0.send(src, n, 1, tag=0, cfg=c0.make_config(nb, ks, 0, 1))
+            c1.recv(dst, n, 0, tag=0)
+            W.run()
+            exp = torch.from_numpy(expected(host, nb, ks, ps)).cuda()
+            assert torch.equal(mp.as_tensor(dst, n), exp), (nb, ks)
+            del exp
