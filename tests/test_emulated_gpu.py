@@ -283,3 +283,68 @@ def test_emulated_config3_full_size_default_launch_config(torch_cuda):
             exp = torch.from_numpy(expected(host, nb, ks, ps)).cuda()
             assert torch.equal(mp.as_tensor(dst, n), exp), (nb, ks)
             del exp
+
+
+def _install(ctx, src, dst, tbl, port):
+    ctx.set_model(src, dst, [(t["kind"], t["via"]) for t in tbl],
+                  [{k: (0.0 if k == "beta2" and t["kind"] == 0 else t[k])
+                    for k in ("alpha", "beta", "alpha2", "beta2", "eps", "c", "sigma", "w")} for t in tbl], port)
+
+
+@pytest.mark.parametrize("mode", ["paper", "b200"])
+def test_emulated_config2_model_selected_multipath_split(torch_cuda, mode):
+    """BASELINE config 2 (64 MiB, GPU0 -> GPU1, direct + 2 GPU relays): an NVLink-like
+    parameter table (synth.topology) installed on the sender; the library's pick over
+    direct + both relays (host path masked out) equals the oracle's (bytes, chunks,
+    t_pred within 1e-9), and that multi-path split moves bit-exact through the emulated
+    world's kernels."""
+    torch = torch_cuda
+    from oracle import model as OM
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    n = 64 * MiB
+    port = dict(alpha=1.5e-6, beta=850e9)
+    with world(4, heap_bytes=n + 8 * MiB, slot_bytes=8 * MiB, slots=4) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        o = c0.get_options()
+        o["mode"] = mp.MP_MODEL_PAPER if mode == "paper" else mp.MP_MODEL_B200
+        c0.set_options(**o)
+        ps = c0.paths(0, 1)
+        for seed in (3, 8):
+            tbl = synth.topology(seed, 2, host=True)
+            assert [(t["kind"], t["via"]) for t in tbl] == ps
+            _install(c0, 0, 1, tbl, port)
+            d = c0.select(0, 1, n, 0b0111).as_dict()
+            ref = OM.select(n, [OM.Path(**t) for t in tbl],
+                            OM.Options(mode=o["mode"], stagger=bool(o["stagger"]), align=o["align"],
+                                       c_min=o["c_min"], k_max=o["k_max"], slot_bytes=o["slot_bytes"]),
+                            OM.Port(**port), path_mask=[True, True, True, False])
+            assert d["bytes"] == list(ref.bytes) and d["chunks"] == list(ref.chunks), (d, ref)
+            assert abs(d["t_pred"] - ref.t_pred) <= 1e-9 * ref.t_pred
+            assert sum(d["bytes"][1:3]) > 0, "an NVLink-like table puts bytes on the relays"
+            host, src = fill(torch, n, seed)
+            dst = c1.alloc(n)
+            c0.send(src, n, 1, tag=seed, cfg=c0.make_config(d["bytes"], d["chunks"], 0, 1))
+            c1.recv(dst, n, 0, tag=seed)
+            torch.cuda.synchronize()
+            W.run()
+            assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, d["bytes"], d["chunks"], ps))
+            c1.free(dst)
+
+
+def test_emulated_config1_forced_split(torch_cuda):
+    """BASELINE config 1: 1 MiB GPU0 -> GPU1, direct + 1 relay, 4 chunks, θ = (3/4, 1/4)
+    (SURVEY §8(d)), world 3 (relay rank 2, no host path)."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    n = 1 << 20
+    with world(3, host_path=0) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        assert [k for k, _ in ps] == [0, 1]
+        nb, ks = [3 * n // 4, n // 4], [1, 4]
+        host, src = fill(torch, n, 11)
+        dst = c1.alloc(n)
+        c0.send(src, n, 1, tag=1, cfg=c0.make_config(nb, ks, 0, 1))
+        c1.recv(dst, n, 0, tag=1)
+        W.run()
+        assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, nb, ks, ps))
