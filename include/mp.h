@@ -210,7 +210,8 @@ int mp_finalize(mp_ctx *ctx);
  * recorded since the last run as one cooperative grid on `stream` — per send its gate
  * and send CTAs, per receive its receive CTAs, the eager kernels, and per (relay rank,
  * sender) the relay kernel that rank's service thread would have launched, which reads
- * its doorbells on the device — then waits for the stream.  Direct-path CTA groups
+ * its doorbells on the device — then waits for the stream.  kernel_s (may be NULL):
+ * the grid's device time [s] from CUDA events on `stream`.  Direct-path CTA groups
  * are shrunk (same bytes, fewer CTAs) so the grid fits the device's co-resident
  * capacity.  The recorded work must be one self-contained exchange: every recorded
  * send matched by a recorded receive.  Errors: MP_ERR_INVALID (not the whole world /
@@ -220,7 +221,7 @@ int mp_finalize(mp_ctx *ctx);
  *
  * mp_finalize_emulated: tears down all n contexts (one thread each) and the world. */
 int mp_init_emulated(mp_ctx **ctxs, const mp_init_args *args);
-int mp_emu_run(mp_ctx **ctxs, int n, void *stream);
+int mp_emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s);
 int mp_finalize_emulated(mp_ctx **ctxs, int n);
 
 /* ---------------------------------------------------------------- topology (Step 1) */

@@ -566,10 +566,10 @@ int mp_finalize_emulated(mp_ctx **ctxs, int n) {
   return mpx::emu_finalize_world(ctxs, n);
 }
 
-int mp_emu_run(mp_ctx **ctxs, int n, void *stream) {
+int mp_emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
   if (!ctxs || n < 2 || !ctxs[0]) return MP_ERR_INVALID;
   if (!ctxs[0]->emulated) return fail(ctxs[0], MP_ERR_STATE, "mp_emu_run: not an emulated world");
-  return mpx::emu_run(ctxs, n, stream);
+  return mpx::emu_run(ctxs, n, stream, kernel_s);
 }
 
 int mp_paths(mp_ctx *c, int src, int dst, mp_path *out, int *npaths) {

@@ -225,7 +225,7 @@ int world_sync(mp_ctx *c);
 // the bootstrap's rank threads
 int emu_init_world(mp_ctx **ctxs, const mp_init_args *a);
 int emu_finalize_world(mp_ctx **ctxs, int n);
-int emu_run(mp_ctx **ctxs, int n, void *stream);
+int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s);
 bool emu_thread();
 int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id);
 // true when [p, p + n) lies in a receive region (heap or mp_register) of this rank

@@ -1793,25 +1793,36 @@ int launch_relay(const RelayParams &P, void *stream) {
   return static_cast<int>(cudaGetLastError());
 }
 
-int emu_capacity(int *per_sm) {
-  const int smem = static_cast<int>(staged_smem<kBulkStages>());
-  cudaError_t e = cudaFuncSetAttribute(emu_kernel<kBulkStages>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, emu_kernel<kBulkStages>, kThreads, smem);
+namespace {
+template <uint32_t D>
+cudaError_t emu_occupancy(int *n) {
+  const int smem = static_cast<int>(staged_smem<D>());
+  cudaError_t e = cudaFuncSetAttribute(emu_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(n, emu_kernel<D>, kThreads, smem);
+  return e;
+}
+}  // namespace
+
+int emu_capacity(int *per_sm, int *per_sm_deep) {
+  cudaError_t e = emu_occupancy<kBulkStages>(per_sm);
+  if (e == cudaSuccess) e = emu_occupancy<kDeepStages>(per_sm_deep);
   return static_cast<int>(e);
 }
 
-int launch_emu(const EmuTable &T, void *stream) {
+int launch_emu(const EmuTable &T, uint32_t stages, void *stream) {
+  const bool deep = stages == kDeepStages;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(T.nblocks);
   cfg.blockDim = dim3(kThreads);
-  cfg.dynamicSmemBytes = staged_smem<kBulkStages>();
+  cfg.dynamicSmemBytes = deep ? staged_smem<kDeepStages>() : staged_smem<kBulkStages>();
   cfg.stream = static_cast<cudaStream_t>(stream);
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeCooperative;  // every CTA co-resident, or the launch fails
   at[0].val.cooperative = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return static_cast<int>(cudaLaunchKernelEx(&cfg, emu_kernel<kBulkStages>, T));
+  return static_cast<int>(deep ? cudaLaunchKernelEx(&cfg, emu_kernel<kDeepStages>, T)
+                               : cudaLaunchKernelEx(&cfg, emu_kernel<kBulkStages>, T));
 }
 
 int launch_spin(uint64_t ns, void *stream) {

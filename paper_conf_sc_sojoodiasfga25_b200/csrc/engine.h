@@ -304,10 +304,12 @@ struct EmuTable {
   const EagerParams *eager;
   uint32_t nroles, nblocks;
 };
-// Co-resident CTAs per SM of emu_kernel (its grid must not exceed per_sm x SMs).
-int emu_capacity(int *per_sm);
-// Cooperative launch of emu_kernel over T.nblocks CTAs (T's arrays in device memory).
-int launch_emu(const EmuTable &T, void *stream);
+// Co-resident CTAs per SM of emu_kernel at 4 and at 6 staged-pipeline stages (its grid
+// must not exceed that x SMs).
+int emu_capacity(int *per_sm, int *per_sm_deep);
+// Cooperative launch of emu_kernel over T.nblocks CTAs (T's arrays in device memory);
+// `stages` = shallow_stages() or deep_stages(): the depth of every role's staged pipeline.
+int launch_emu(const EmuTable &T, uint32_t stages, void *stream);
 
 int launch_send(const SendParams &P, void *stream);
 int launch_eager_send(const EagerParams &P, void *stream);

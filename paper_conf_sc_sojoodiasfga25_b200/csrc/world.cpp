@@ -980,7 +980,7 @@ int emu_finalize_world(mp_ctx **ctxs, int n) {
 
 bool emu_thread() { return t_emu_rank >= 0; }
 
-int emu_run(mp_ctx **ctxs, int n, void *stream) {
+int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
   mp_ctx *c = ctxs[0];
   EmuWorld *w = c->emu_world;
   if (!w || n != w->world) return wfail(c, MP_ERR_INVALID, "mp_emu_run: pass every context of one emulated world");
@@ -1018,7 +1018,6 @@ int emu_run(mp_ctx **ctxs, int n, void *stream) {
     P.sender = snd;
     P.g = v[0].second;
     P.copy_mode = rc->copy_mode;
-    P.stages = shallow_stages();
     P.timeout_ns = static_cast<uint64_t>(rc->timeout_s * 1e9);
     P.m0 = v[0].first;
     P.max_msgs = v.size();
@@ -1052,13 +1051,14 @@ int emu_run(mp_ctx **ctxs, int n, void *stream) {
   };
   // Grid: every role co-resident.  Only the direct groups are elastic (any CTA count
   // moves the same bytes): they share what the fixed roles leave, in proportion to
-  // the CTA counts the real launches would have used.
-  int per_sm = 0;
-  if (int e = emu_capacity(&per_sm)) {
+  // the CTA counts the real launches would have used.  Staged pipelines run at the
+  // deep depth when the whole grid fits its occupancy (as the real launches choose per
+  // launch, stages_for), else at 4 stages; MPX_STAGES forces one.
+  int per_sm = 0, per_sm_deep = 0;
+  if (int e = emu_capacity(&per_sm, &per_sm_deep)) {
     clear();
     return wfail(c, MP_ERR_CUDA, std::string("emu_capacity: ") + cudaGetErrorString(static_cast<cudaError_t>(e)));
   }
-  const uint64_t cap = static_cast<uint64_t>(per_sm) * static_cast<uint64_t>(c->sms);
   uint64_t fixed = 0, want = 0;
   for (const SendParams &P : send) {
     fixed += 1 + (P.nblocks - P.g_direct);
@@ -1067,6 +1067,10 @@ int emu_run(mp_ctx **ctxs, int n, void *stream) {
   for (const RecvParams &P : recv) fixed += P.nblocks;
   for (const RelayParams &P : relay) fixed += P.g;
   for (const EagerParams &P : eager) fixed += P.ctas;
+  const uint64_t sms = static_cast<uint64_t>(c->sms);
+  uint32_t stages = fixed + want <= static_cast<uint64_t>(per_sm_deep) * sms ? deep_stages() : shallow_stages();
+  if (c->force_stages) stages = c->force_stages;
+  const uint64_t cap = static_cast<uint64_t>(stages == deep_stages() ? per_sm_deep : per_sm) * sms;
   if (fixed + send.size() > cap) {
     clear();
     return wfail(c, MP_ERR_INVALID, "mp_emu_run: the recorded kernels do not fit one co-resident grid (" +
@@ -1096,6 +1100,7 @@ int emu_run(mp_ctx **ctxs, int n, void *stream) {
   }
   for (uint32_t i = 0; i < eager.size(); ++i) add(i < n_esend ? EMU_EAGER_SEND : EMU_EAGER_RECV, eager[i].ctas, i);
   clear();
+  if (kernel_s) *kernel_s = 0;
   if (roles.empty()) return MP_OK;
   // one device block: roles, then the parameter arrays (16-B aligned)
   auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
@@ -1125,9 +1130,21 @@ int emu_run(mp_ctx **ctxs, int n, void *stream) {
   T.nroles = static_cast<uint32_t>(roles.size());
   T.nblocks = cta;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaEvent_t ev[2] = {nullptr, nullptr};
   cudaError_t e = cudaMemcpyAsync(d, h.data(), total, cudaMemcpyHostToDevice, st);
-  if (e == cudaSuccess) e = static_cast<cudaError_t>(launch_emu(T, stream));
+  if (e == cudaSuccess && kernel_s) e = cudaEventCreate(&ev[0]);
+  if (e == cudaSuccess && kernel_s) e = cudaEventCreate(&ev[1]);
+  if (e == cudaSuccess && kernel_s) e = cudaEventRecord(ev[0], st);
+  if (e == cudaSuccess) e = static_cast<cudaError_t>(launch_emu(T, stages, stream));
+  if (e == cudaSuccess && kernel_s) e = cudaEventRecord(ev[1], st);
   if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e == cudaSuccess && kernel_s) {
+    float ms = 0;
+    e = cudaEventElapsedTime(&ms, ev[0], ev[1]);
+    *kernel_s = ms * 1e-3;
+  }
+  for (cudaEvent_t x : ev)
+    if (x) cudaEventDestroy(x);
   cudaFree(d);
   if (e != cudaSuccess) return wfail(c, MP_ERR_CUDA, std::string("mp_emu_run: ") + cudaGetErrorString(e));
   for (int r = 0; r < n; ++r) {

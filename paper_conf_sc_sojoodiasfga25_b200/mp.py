@@ -198,7 +198,7 @@ def lib():
             "mp_get_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
             "mp_set_topology": (C.c_int, [P, C.POINTER(mp_topology)]),
             "mp_init_emulated": (C.c_int, [C.POINTER(P), C.POINTER(mp_init_args)]),
-            "mp_emu_run": (C.c_int, [C.POINTER(P), C.c_int, P]),
+            "mp_emu_run": (C.c_int, [C.POINTER(P), C.c_int, P, C.POINTER(C.c_double)]),
             "mp_finalize_emulated": (C.c_int, [C.POINTER(P), C.c_int]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
@@ -630,10 +630,14 @@ class EmulatedWorld:
         self.world = world
         self.ctx = [Context._wrap(self._h[r], r, world) for r in range(world)]
 
-    def run(self, stream=None):
-        st = lib().mp_emu_run(self._h, self.world, _stream(stream))
+    def run(self, stream=None) -> float:
+        """Launch what the contexts recorded as one cooperative grid; returns the grid's
+        device time [s] (CUDA events on `stream`)."""
+        t = C.c_double()
+        st = lib().mp_emu_run(self._h, self.world, _stream(stream), C.byref(t))
         if st != 0:
             raise MPError(st, lib().mp_last_error(self._h[0]).decode())
+        return t.value
 
     def close(self):
         if self.ctx:

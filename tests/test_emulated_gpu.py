@@ -348,3 +348,30 @@ def test_emulated_config1_forced_split(torch_cuda):
         c1.recv(dst, n, 0, tag=1)
         W.run()
         assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, nb, ks, ps))
+
+
+@pytest.mark.parametrize("stages", ["4", "6"])
+def test_emulated_both_staged_pipeline_depths(torch_cuda, monkeypatch, stages):
+    """The send / receive / relay bodies at each staged-pipeline depth (MPX_STAGES: the
+    real launches pick one per launch; the emulated grid runs every role at one):
+    every path kind at world 3, co-aligned and misaligned sources."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    monkeypatch.setenv("MPX_STAGES", stages)
+    with world(3, relay_ctas=8, slot_bytes=2 * MiB) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        n = 5 * MiB + 333
+        buf = torch.empty(n + 64, dtype=torch.uint8, device="cuda")
+        for i, (nb, ks) in enumerate(cases_for(ps, n)):
+            for shift in (0, 5):
+                host = synth.payload(n, 40 + i)
+                src = buf[shift:shift + n]
+                src.copy_(torch.from_numpy(host))
+                dst = c1.alloc(n)
+                c0.send(src, n, 1, tag=i, cfg=c0.make_config(nb, ks, 0, 1))
+                c1.recv(dst, n, 0, tag=i)
+                torch.cuda.synchronize()
+                W.run()
+                assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, nb, ks, ps)), (stages, i, shift)
+                c1.free(dst)

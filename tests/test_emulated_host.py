@@ -31,7 +31,7 @@ def test_emulated_bad_arguments():
     assert L.mp_init_emulated(hs, C.byref(a)) == mp.MP_ERR_INVALID
     a.world, a.flags = 2, mp.MP_INIT_MODEL_ONLY
     assert L.mp_init_emulated(hs, C.byref(a)) == mp.MP_ERR_INVALID
-    assert L.mp_emu_run(None, 2, None) == mp.MP_ERR_INVALID
+    assert L.mp_emu_run(None, 2, None, None) == mp.MP_ERR_INVALID
     assert L.mp_finalize_emulated(None, 2) == mp.MP_ERR_INVALID
 
 
