@@ -34,6 +34,7 @@ def main():
     ap.add_argument("--mib", type=int, default=256)
     ap.add_argument("--reps", type=int, default=7)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--case", default=None, help="direct | relay | host | all (default: every case)")
     a = ap.parse_args()
     n = a.mib * MiB
     try:
@@ -59,6 +60,8 @@ def main():
             "all": ([n - 3 * q, 2 * q, q], [1, max(1, 2 * q // (16 * MiB)), max(1, q // (16 * MiB))]),
         }
         for name, (nb, ks) in cases.items():
+            if a.case and name != a.case:
+                continue
             ts = []
             for r in range(a.reps + 1):
                 out.zero_()
