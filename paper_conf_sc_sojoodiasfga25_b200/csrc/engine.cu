@@ -1001,6 +1001,8 @@ struct RelayConsumer {
   uint32_t r;
   uint64_t lstride;
   uint64_t q0;  // the message's first ring sequence
+  uint64_t k;   // the message's chunks
+  uint64_t acc; // bytes of this lane stored so far (counted once, after its last chunk)
   __device__ uint8_t *lane(uint32_t j) const {
     const uint64_t s = (q0 + j) % P->L.slots;
     return P->my_ctrl + P->L.ring_data + (static_cast<uint64_t>(P->sender) * P->L.slots + s) * P->L.stride +
@@ -1030,8 +1032,13 @@ struct RelayConsumer {
     st_release_sys(flags_at(P->sender_ctrl, P->L.relay_free, P->me, P->L.slots, q % P->L.slots) + r,
                    q / P->L.slots + 1);
   }
-  __device__ void stored(uint32_t, const uint64_t *w) {
-    red_add_release_sys(done_at(P->peer[w[0]].ctrl, P->L, P->sender), w[2]);
+  // The receiver only waits for the message's whole byte count (A10), so a lane counts
+  // its bytes once, after its last chunk: one system-scope reduction into the
+  // destination GPU's counter per lane and message instead of one per chunk (the
+  // publisher's other release per chunk, the free flag, is what the sender waits on).
+  __device__ void stored(uint32_t j, const uint64_t *w) {
+    acc += w[2];
+    if (j + 1 == k) red_add_release_sys(done_at(P->peer[w[0]].ctrl, P->L, P->sender), acc);
   }
 };
 
@@ -1276,8 +1283,11 @@ __device__ void recv_body(const RecvParams &P, const uint32_t b, uint8_t *dyn_sm
       // A10: wait until every byte of the message has been counted in
       const uint64_t *done = done_at(P.my_ctrl, P.L, P.src);
       const uint64_t t_start = globaltimer();
-      while (ld_acquire_sys(done) < P.done_target) {
-        if (ld_acquire_sys(&hdr->seq1) == P.seq + 1 && ld_volatile(&hdr->c) == 2) {
+      // polled relaxed, one acquire on success (an acquire load invalidates this SM's
+      // L1 each time; poll_flag)
+      while (ld_relaxed_sys(done) < P.done_target || ld_acquire_sys(done) < P.done_target) {
+        if (ld_relaxed_sys(&hdr->seq1) == P.seq + 1 && ld_acquire_sys(&hdr->seq1) == P.seq + 1 &&
+            ld_volatile(&hdr->c) == 2) {
           atomicExch(P.err, DERR_MISMATCH);
           break;
         }
@@ -1343,7 +1353,7 @@ __device__ bool relay_message(const RelayParams &P, const uint32_t r, uint64_t q
                               int *s_abort, uint8_t *smem) {
   const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g);
   if (P.copy_mode == 1 && aligned) {  // streamed lane (the sender found source and target co-aligned)
-    RelayConsumer R{&P, r, lstride, q0};
+    RelayConsumer R{&P, r, lstride, q0, k, 0};
     lane_stream<LD_RING, D>(R, static_cast<uint32_t>(k), smem);
     return *reinterpret_cast<volatile int32_t *>(P.err) == 0;
   }

@@ -35,6 +35,11 @@ def main():
     ap.add_argument("--reps", type=int, default=7)
     ap.add_argument("--out", default=None)
     ap.add_argument("--case", default=None, help="direct | relay | host | all (default: every case)")
+    ap.add_argument("--slots", type=int, default=0, help="ring slots (default: the library's, 4)")
+    ap.add_argument("--slot-mib", type=int, default=0, help="slot size in MiB (default: the library's, 32)")
+    ap.add_argument("--lanes", type=int, default=16, help="CTAs per stage group (relay_ctas)")
+    ap.add_argument("--chunk-mib", type=int, default=16, help="staged chunk size in MiB")
+    ap.add_argument("--no-host", action="store_true", help="no pinned-host path (direct and relay cases only)")
     a = ap.parse_args()
     n = a.mib * MiB
     try:
@@ -43,25 +48,31 @@ def main():
         peak = None
     torch.cuda.set_device(0)
     rows = []
-    with mp.EmulatedWorld(3, device=0, heap_bytes=n + 64 * MiB, timeout_s=60.0) as W:
+    with mp.EmulatedWorld(3, device=0, heap_bytes=n + 64 * MiB, timeout_s=60.0, slots=a.slots,
+                          slot_bytes=a.slot_mib * MiB, relay_ctas=a.lanes, host_path=0 if a.no_host else -1) as W:
         c0, c1 = W.ctx[0], W.ctx[1]
         ps = c0.paths(0, 1)
-        assert [k for k, _ in ps] == [0, 1, 2]
+        assert [k for k, _ in ps] == ([0, 1] if a.no_host else [0, 1, 2])
         src = torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda",
                             generator=torch.Generator(device="cuda").manual_seed(7))
         dst = c1.alloc(n)
         out = mp.as_tensor(dst, n)
         s = torch.cuda.Stream()
         q = n // 8 // 256 * 256
+        cm = a.chunk_mib
         cases = {
             "direct": ([n, 0, 0], [1, 0, 0]),
-            "relay": ([0, n, 0], [1, max(1, n // (16 * MiB)), 0]),
-            "host": ([0, 0, n], [1, 0, max(1, n // (16 * MiB))]),
-            "all": ([n - 3 * q, 2 * q, q], [1, max(1, 2 * q // (16 * MiB)), max(1, q // (16 * MiB))]),
+            "relay": ([0, n, 0], [1, max(1, n // (cm * MiB)), 0]),
+            "host": ([0, 0, n], [1, 0, max(1, n // (cm * MiB))]),
+            "all": ([n - 3 * q, 2 * q, q], [1, max(1, 2 * q // (cm * MiB)), max(1, q // (cm * MiB))]),
         }
         for name, (nb, ks) in cases.items():
             if a.case and name != a.case:
                 continue
+            if a.no_host:
+                if nb[2]:
+                    continue
+                nb, ks = nb[:2], ks[:2]
             ts = []
             for r in range(a.reps + 1):
                 out.zero_()
@@ -73,10 +84,11 @@ def main():
                 if r:
                     ts.append(t)
             t = statistics.median(ts)
-            hbm = (2 * nb[0] + 4 * nb[1] + 2 * nb[2]) / t / 1e9
+            hbm = (2 * nb[0] + 4 * nb[1] + 2 * sum(nb[2:])) / t / 1e9
             row = {"case": name, "bytes": nb, "chunks": ks, "msg_bytes": n, "s_median": t,
                    "s_min": min(ts), "payload_GBps": n / t / 1e9, "hbm_GBps": hbm,
-                   "hbm_frac": hbm / peak if peak else None, "lanes": 16,
+                   "hbm_frac": hbm / peak if peak else None, "lanes": a.lanes, "slots": a.slots,
+                   "slot_mib": a.slot_mib,
                    "note": "one GPU: every path is an HBM copy; not NVLink evidence"}
             rows.append(row)
             print(json.dumps(row), flush=True)
