@@ -203,8 +203,9 @@ int mp_finalize(mp_ctx *ctx);
  * context is returned.
  * In an emulated world, mp_send / mp_recv (and mp_select, mp_alloc, every model
  * call) behave as in a real job except that they launch nothing: they record the
- * kernels' parameter blocks.  mp_register, the collectives and the calibration calls
- * return MP_ERR_UNSUPPORTED; mp_finalize returns MP_ERR_STATE.
+ * kernels' parameter blocks.  mp_register, mp_alltoall / mp_allreduce (use
+ * mp_emu_alltoall / mp_emu_allreduce) and the calibration calls return
+ * MP_ERR_UNSUPPORTED; mp_finalize returns MP_ERR_STATE.
  *
  * mp_emu_run: ctxs = the world's n contexts in rank order.  Launches everything they
  * recorded since the last run as one cooperative grid on `stream` — per send its gate
@@ -637,6 +638,19 @@ int mp_alltoall(mp_ctx *ctx, const void *sendbuf, void *recvbuf, uint64_t bytes_
  * Errors: MP_ERR_INVALID (dtype, op), as mp_alltoall. */
 int mp_allreduce(mp_ctx *ctx, const void *sendbuf, void *recvbuf, uint64_t count, int dtype, int op,
                  int algo, void *stream);
+
+/* The same two collectives over an emulated world (mp_init_emulated): ctxs = the
+ * world's n contexts in rank order, sendbufs[r] / recvbufs[r] = rank r's buffers (rules
+ * as above).  Every rank's plan runs in lock step on `stream`: every rank's pre copies;
+ * per step, every rank's packing, then its send and receive as ONE cooperative grid
+ * (mp_emu_run), then every rank's unpacking or reduction; every rank's post copies.
+ * Returns once `stream` has finished.  Nothing else may be recorded on the world.
+ * Errors: MP_ERR_INVALID (arguments, dtype, op, plan), MP_ERR_STATE (not an emulated
+ * world), as mp_emu_run. */
+int mp_emu_alltoall(mp_ctx **ctxs, int n, const void *const *sendbufs, void *const *recvbufs,
+                    uint64_t bytes_per_rank, int algo, void *stream);
+int mp_emu_allreduce(mp_ctx **ctxs, int n, const void *const *sendbufs, void *const *recvbufs,
+                     uint64_t count, int dtype, int op, int algo, void *stream);
 
 /* The Hockney fit of Step 1 (reading C12), exposed for parity tests: least squares of
  * T = α + n/β over m samples (n[i] bytes, t[i] seconds, host arrays), each residual

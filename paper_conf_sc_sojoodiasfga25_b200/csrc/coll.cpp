@@ -327,98 +327,208 @@ int local_copy(mp_ctx *c, void *dst, const void *src, uint64_t n, cudaStream_t s
   return launch_direct_copy(c, dst, src, n, s);
 }
 
-int run_plan(mp_ctx *c, const mp_coll_plan &P, const void *sendbuf, void *recvbuf, uint64_t bytes, uint32_t elem,
-             int dtype, void *ustream) {
-  if (!c->coll) c->coll = new (std::nothrow) CollState();
-  if (!c->coll) return MP_ERR_NOMEM;
-  CollState &st = *c->coll;
-  uint64_t maxmsg = 0;
-  for (int j = 0; j < P.nsteps; ++j) maxmsg = std::max(maxmsg, P.step[j].bytes);
-  const uint64_t align = 256;
-  const uint64_t tmp = (P.tmp_bytes + align - 1) / align * align, stg = (maxmsg + align - 1) / align * align;
-  if (int e = ensure(c, st, std::max<uint64_t>(tmp + 2 * stg, 256), 2 + 2 * P.nsteps)) return e;
-  uint8_t *base = static_cast<uint8_t *>(st.scratch);
-  uint8_t *tmpb = base, *stg_s = base + tmp, *stg_r = base + tmp + stg;
-  auto buf = [&](int id) -> uint8_t * {
+// One rank's execution of a plan, in pieces.  The real executor (run_plan) chains
+// them on two internal streams with events; the emulated world's executor
+// (emu_collective) runs every rank's pieces step by step around one cooperative grid
+// per step.
+struct PlanExec {
+  mp_ctx *c = nullptr;
+  const mp_coll_plan *P = nullptr;
+  const void *sendbuf = nullptr;
+  void *recvbuf = nullptr;
+  int dtype = 0;
+  uint8_t *tmpb = nullptr, *stg_s = nullptr, *stg_r = nullptr;
+  const std::vector<mp_config> *cfgs = nullptr;
+  uint64_t seq = 0;
+
+  uint8_t *buf(int id) const {
     return id == MP_BUF_SEND ? const_cast<uint8_t *>(static_cast<const uint8_t *>(sendbuf))
                              : (id == MP_BUF_RECV ? static_cast<uint8_t *>(recvbuf) : tmpb);
-  };
-  const std::vector<mp_config> *cfgs = nullptr;
-  if (c->world > 1 && P.nsteps)
-    if (int e = step_configs(c, st, P, bytes, elem, &cfgs)) return e;
+  }
+  int tag(int j) const { return 0x3C000000 | static_cast<int>((seq & 0xFFFF) << 8) | (j & 0xFF); }
+
+  // scratch [tmp | send staging | recv staging] in the heap, events, per-step configs
+  int setup(uint64_t bytes, uint32_t elem) {
+    if (!c->coll) c->coll = new (std::nothrow) CollState();
+    if (!c->coll) return MP_ERR_NOMEM;
+    CollState &st = *c->coll;
+    uint64_t maxmsg = 0;
+    for (int j = 0; j < P->nsteps; ++j) maxmsg = std::max(maxmsg, P->step[j].bytes);
+    const uint64_t align = 256;
+    const uint64_t tmp = (P->tmp_bytes + align - 1) / align * align, stg = (maxmsg + align - 1) / align * align;
+    if (int e = ensure(c, st, std::max<uint64_t>(tmp + 2 * stg, 256), 2 + 2 * P->nsteps)) return e;
+    uint8_t *base = static_cast<uint8_t *>(st.scratch);
+    tmpb = base;
+    stg_s = base + tmp;
+    stg_r = base + tmp + stg;
+    if (c->world > 1 && P->nsteps)
+      if (int e = step_configs(c, st, *P, bytes, elem, &cfgs)) return e;
+    seq = st.seq++;
+    return MP_OK;
+  }
+  int copies(const mp_coll_copy *k, int n, cudaStream_t s) {
+    for (int i = 0; i < n; ++i)
+      if (int e = local_copy(c, buf(k[i].dst_buf) + k[i].dst_off, buf(k[i].src_buf) + k[i].src_off, k[i].len, s))
+        return e;
+    return MP_OK;
+  }
+  int pre(cudaStream_t s) { return copies(P->pre, P->npre, s); }
+  int post(cudaStream_t s) { return copies(P->post, P->npost, s); }
+  // send side of step j: pack its segments (one segment is sent in place), mp_send
+  int send(int j, cudaStream_t s) {
+    const mp_coll_step &t = P->step[j];
+    const uint8_t *msg = nullptr;
+    if (t.send_nseg == 1) {
+      const mp_coll_seg &g = P->seg[t.send_seg0];
+      msg = buf(g.buf) + g.off;
+    } else {
+      uint64_t o = 0;
+      for (uint32_t k = 0; k < t.send_nseg; ++k) {
+        const mp_coll_seg &g = P->seg[t.send_seg0 + k];
+        if (int e = local_copy(c, stg_s + o, buf(g.buf) + g.off, g.len, s)) return e;
+        o += g.len;
+      }
+      msg = stg_s;
+    }
+    return mp_send(c, msg, t.bytes, t.send_to, tag(j), &(*cfgs)[j], s);
+  }
+  uint64_t recv_bytes(int j) const {
+    const mp_coll_step &t = P->step[j];
+    uint64_t n = 0;
+    for (uint32_t k = 0; k < t.recv_nseg; ++k) n += P->seg[t.recv_seg0 + k].len;
+    return n;
+  }
+  // step j's message lands straight in its target: one receivable segment, no
+  // reduction, and not overlapping what the step still sends (Bruck sends and receives
+  // the same TMP block positions)
+  bool direct_recv(int j) const {
+    const mp_coll_step &t = P->step[j];
+    const mp_coll_seg *g0 = t.recv_nseg ? &P->seg[t.recv_seg0] : nullptr;
+    bool overlap = false;
+    for (uint32_t k = 0; k < t.send_nseg && g0; ++k) {
+      const mp_coll_seg &g = P->seg[t.send_seg0 + k];
+      const uint8_t *a0 = buf(g.buf) + g.off, *b0 = buf(g0->buf) + g0->off;
+      if (a0 < b0 + g0->len && b0 < a0 + g.len) overlap = true;
+    }
+    return t.recv_nseg == 1 && !t.reduce && !overlap &&
+           (g0->buf == MP_BUF_TMP || world_receivable(c, buf(g0->buf) + g0->off, g0->len));
+  }
+  int recv(int j, cudaStream_t s) {
+    const mp_coll_step &t = P->step[j];
+    uint8_t *dst = stg_r;
+    if (direct_recv(j)) {
+      const mp_coll_seg &g0 = P->seg[t.recv_seg0];
+      dst = buf(g0.buf) + g0.off;
+    }
+    return mp_recv(c, dst, recv_bytes(j), t.recv_from, tag(j), s);
+  }
+  // a staged receive of step j: its segments copied (or reduced) out of the staging
+  int unpack(int j, cudaStream_t s) {
+    const mp_coll_step &t = P->step[j];
+    uint64_t o = 0;
+    for (uint32_t k = 0; k < t.recv_nseg; ++k) {
+      const mp_coll_seg &g = P->seg[t.recv_seg0 + k];
+      const int e = t.reduce ? launch_reduce_sum(c, dtype, buf(g.buf) + g.off, stg_r + o, g.len, s)
+                             : local_copy(c, buf(g.buf) + g.off, stg_r + o, g.len, s);
+      if (e) return e;
+      o += g.len;
+    }
+    return MP_OK;
+  }
+};
+
+int run_plan(mp_ctx *c, const mp_coll_plan &P, const void *sendbuf, void *recvbuf, uint64_t bytes, uint32_t elem,
+             int dtype, void *ustream) {
+  PlanExec X;
+  X.c = c;
+  X.P = &P;
+  X.sendbuf = sendbuf;
+  X.recvbuf = recvbuf;
+  X.dtype = dtype;
+  if (int e = X.setup(bytes, elem)) return e;
+  CollState &st = *c->coll;
   cudaStream_t us = static_cast<cudaStream_t>(ustream);
   cudaEvent_t *ev = st.ev.data();
   // fork
   if (cudaEventRecord(ev[0], us) != cudaSuccess || cudaStreamWaitEvent(st.s, ev[0], 0) != cudaSuccess ||
       cudaStreamWaitEvent(st.r, ev[0], 0) != cudaSuccess)
     return cfail(c, MP_ERR_CUDA, "collective fork");
-  for (int i = 0; i < P.npre; ++i) {
-    const mp_coll_copy &k = P.pre[i];
-    if (int e = local_copy(c, buf(k.dst_buf) + k.dst_off, buf(k.src_buf) + k.src_off, k.len, st.s)) return e;
-  }
-  const uint64_t seq = st.seq++;
+  if (int e = X.pre(st.s)) return e;
   cudaEvent_t prev_r = nullptr;
   for (int j = 0; j < P.nsteps; ++j) {
-    const mp_coll_step &s = P.step[j];
-    const int tag = 0x3C000000 | static_cast<int>((seq & 0xFFFF) << 8) | (j & 0xFF);
     cudaEvent_t sent = ev[2 + 2 * j], done_r = ev[3 + 2 * j];
     // send side: after the previous step's receive (its data may be sent now)
     if (prev_r) cudaStreamWaitEvent(st.s, prev_r, 0);
-    const uint8_t *msg = nullptr;
-    if (s.send_nseg == 1) {
-      const mp_coll_seg &g = P.seg[s.send_seg0];
-      msg = buf(g.buf) + g.off;
-    } else {
-      uint64_t o = 0;
-      for (uint32_t k = 0; k < s.send_nseg; ++k) {
-        const mp_coll_seg &g = P.seg[s.send_seg0 + k];
-        if (int e = local_copy(c, stg_s + o, buf(g.buf) + g.off, g.len, st.s)) return e;
-        o += g.len;
-      }
-      msg = stg_s;
-    }
-    if (int e = mp_send(c, msg, s.bytes, s.send_to, tag, &(*cfgs)[j], st.s)) return e;
+    if (int e = X.send(j, st.s)) return e;
     cudaEventRecord(sent, st.s);  // the send kernel has consumed its source
-    // receive side: straight into the target when it is one receivable segment
-    uint64_t rbytes = 0;
-    for (uint32_t k = 0; k < s.recv_nseg; ++k) rbytes += P.seg[s.recv_seg0 + k].len;
-    const mp_coll_seg *g0 = s.recv_nseg ? &P.seg[s.recv_seg0] : nullptr;
-    // a receive straight into the target must not overwrite what this step still sends
-    // (Bruck sends and receives the same TMP block positions)
-    bool overlap = false;
-    for (uint32_t k = 0; k < s.send_nseg && g0; ++k) {
-      const mp_coll_seg &g = P.seg[s.send_seg0 + k];
-      const uint8_t *a0 = buf(g.buf) + g.off, *b0 = buf(g0->buf) + g0->off;
-      if (a0 < b0 + g0->len && b0 < a0 + g.len) overlap = true;
-    }
-    const bool direct = s.recv_nseg == 1 && !s.reduce && !overlap &&
-                        (g0->buf == MP_BUF_TMP || world_receivable(c, buf(g0->buf) + g0->off, g0->len));
     if (prev_r) cudaStreamWaitEvent(st.r, prev_r, 0);
-    if (direct) {
-      if (int e = mp_recv(c, buf(g0->buf) + g0->off, rbytes, s.recv_from, tag, st.r)) return e;
-    } else {
-      if (int e = mp_recv(c, stg_r, rbytes, s.recv_from, tag, st.r)) return e;
+    if (int e = X.recv(j, st.r)) return e;
+    if (!X.direct_recv(j)) {
       cudaStreamWaitEvent(st.r, sent, 0);  // this step's send has read what the unpack overwrites
-      uint64_t o = 0;
-      for (uint32_t k = 0; k < s.recv_nseg; ++k) {
-        const mp_coll_seg &g = P.seg[s.recv_seg0 + k];
-        const int e = s.reduce ? launch_reduce_sum(c, dtype, buf(g.buf) + g.off, stg_r + o, g.len, st.r)
-                               : local_copy(c, buf(g.buf) + g.off, stg_r + o, g.len, st.r);
-        if (e) return e;
-        o += g.len;
-      }
+      if (int e = X.unpack(j, st.r)) return e;
     }
     cudaEventRecord(done_r, st.r);
     prev_r = done_r;
   }
   if (prev_r) cudaStreamWaitEvent(st.s, prev_r, 0);
-  for (int i = 0; i < P.npost; ++i) {
-    const mp_coll_copy &k = P.post[i];
-    if (int e = local_copy(c, buf(k.dst_buf) + k.dst_off, buf(k.src_buf) + k.src_off, k.len, st.s)) return e;
-  }
+  if (int e = X.post(st.s)) return e;
   // join: the receive stream's work is already ordered before the send stream's tail
   cudaEventRecord(ev[1], st.s);
   if (cudaStreamWaitEvent(us, ev[1], 0) != cudaSuccess) return cfail(c, MP_ERR_CUDA, "collective join");
+  return MP_OK;
+}
+
+// The emulated world's executor: every rank's plan in lock step on `stream` — every
+// rank's pre copies; per step, every rank's packing and recorded send / receive, ONE
+// cooperative grid for all of them (mp_emu_run), every rank's unpacking; every rank's
+// post copies.
+int emu_collective(mp_ctx **ctxs, int n, int coll, int algo, const void *const *sendbufs, void *const *recvbufs,
+                   uint64_t bytes, uint32_t elem, int dtype, void *stream) {
+  mp_ctx *c0 = ctxs[0];
+  if (!c0->emu_world) return cfail(c0, MP_ERR_STATE, "not an emulated world");
+  for (int r = 0; r < n; ++r)
+    if (!ctxs[r] || ctxs[r]->rank != r || ctxs[r]->world != n || !sendbufs[r] || !recvbufs[r])
+      return cfail(c0, MP_ERR_INVALID, "emulated collective: every rank's context and buffers, in rank order");
+  if (bytes == 0) return MP_OK;
+  std::vector<mp_coll_plan> plans(static_cast<size_t>(n));
+  std::vector<PlanExec> X(static_cast<size_t>(n));
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  auto discard = [&](int e) {  // nothing recorded may outlive a failed collective
+    cudaStreamSynchronize(s);
+    for (int r = 0; r < n; ++r) {
+      ctxs[r]->emu_send.clear();
+      ctxs[r]->emu_recv.clear();
+      ctxs[r]->emu_esend.clear();
+      ctxs[r]->emu_erecv.clear();
+    }
+    return e;
+  };
+  for (int r = 0; r < n; ++r) {
+    if (int e = mp_coll_plan_build(coll, algo, n, r, bytes, elem, &plans[r]))
+      return cfail(c0, e, "collective plan: invalid algorithm / size for this world");
+    X[r].c = ctxs[r];
+    X[r].P = &plans[r];
+    X[r].sendbuf = sendbufs[r];
+    X[r].recvbuf = recvbufs[r];
+    X[r].dtype = dtype;
+    if (int e = X[r].setup(bytes, elem)) return discard(e);
+    if (plans[r].nsteps != plans[0].nsteps) return discard(cfail(c0, MP_ERR_INVALID, "ranks' plans differ in steps"));
+  }
+  for (int r = 0; r < n; ++r)
+    if (int e = X[r].pre(s)) return discard(e);
+  for (int j = 0; j < plans[0].nsteps; ++j) {
+    for (int r = 0; r < n; ++r) {
+      if (int e = X[r].send(j, s)) return discard(e);
+      if (int e = X[r].recv(j, s)) return discard(e);
+    }
+    if (int e = mp_emu_run(ctxs, n, stream, nullptr)) return discard(e);
+    for (int r = 0; r < n; ++r)
+      if (!X[r].direct_recv(j))
+        if (int e = X[r].unpack(j, s)) return discard(e);
+  }
+  for (int r = 0; r < n; ++r)
+    if (int e = X[r].post(s)) return discard(e);
+  if (cudaStreamSynchronize(s) != cudaSuccess) return cfail(c0, MP_ERR_CUDA, "emulated collective");
   return MP_OK;
 }
 
@@ -471,4 +581,20 @@ extern "C" int mp_allreduce(mp_ctx *c, const void *sendbuf, void *recvbuf, uint6
   if (op != MP_OP_SUM) return cfail(c, MP_ERR_INVALID, "allreduce: unsupported op");
   return collective(c, MP_COLL_ALLREDUCE, algo, sendbuf, recvbuf, count * eb, static_cast<uint32_t>(eb), dtype,
                     stream);
+}
+
+extern "C" int mp_emu_alltoall(mp_ctx **ctxs, int n, const void *const *sendbufs, void *const *recvbufs,
+                               uint64_t bytes_per_rank, int algo, void *stream) {
+  if (!ctxs || n < 2 || !ctxs[0] || !sendbufs || !recvbufs) return MP_ERR_INVALID;
+  return emu_collective(ctxs, n, MP_COLL_ALLTOALL, algo, sendbufs, recvbufs, bytes_per_rank, 1, MP_DT_U8, stream);
+}
+
+extern "C" int mp_emu_allreduce(mp_ctx **ctxs, int n, const void *const *sendbufs, void *const *recvbufs,
+                                uint64_t count, int dtype, int op, int algo, void *stream) {
+  if (!ctxs || n < 2 || !ctxs[0] || !sendbufs || !recvbufs) return MP_ERR_INVALID;
+  const int eb = elem_bytes(dtype);
+  if (eb == 0 || dtype == MP_DT_U8) return cfail(ctxs[0], MP_ERR_INVALID, "allreduce: unsupported dtype");
+  if (op != MP_OP_SUM) return cfail(ctxs[0], MP_ERR_INVALID, "allreduce: unsupported op");
+  return emu_collective(ctxs, n, MP_COLL_ALLREDUCE, algo, sendbufs, recvbufs, count * eb, static_cast<uint32_t>(eb),
+                        dtype, stream);
 }

@@ -200,6 +200,9 @@ def lib():
             "mp_init_emulated": (C.c_int, [C.POINTER(P), C.POINTER(mp_init_args)]),
             "mp_emu_run": (C.c_int, [C.POINTER(P), C.c_int, P, C.POINTER(C.c_double)]),
             "mp_finalize_emulated": (C.c_int, [C.POINTER(P), C.c_int]),
+            "mp_emu_alltoall": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(P), C.POINTER(P), C.c_uint64, C.c_int, P]),
+            "mp_emu_allreduce": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(P), C.POINTER(P), C.c_uint64, C.c_int,
+                                           C.c_int, C.c_int, P]),
             "mp_fit_bands": (C.c_int, [C.POINTER(C.c_double), C.POINTER(C.c_double), C.c_int,
                                        C.POINTER(C.c_double), C.c_int, C.POINTER(C.c_double),
                                        C.POINTER(C.c_double)]),
@@ -223,7 +226,7 @@ def exported_symbols() -> List[str]:
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
             "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_calibrate_wake", "mp_fit_window",
             "mp_get_topology", "mp_set_topology", "mp_set_submit_time", "mp_get_submit_time",
-            "mp_init_emulated", "mp_emu_run", "mp_finalize_emulated"]
+            "mp_init_emulated", "mp_emu_run", "mp_finalize_emulated", "mp_emu_alltoall", "mp_emu_allreduce"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -638,6 +641,24 @@ class EmulatedWorld:
         if st != 0:
             raise MPError(st, lib().mp_last_error(self._h[0]).decode())
         return t.value
+
+    def _bufs(self, xs):
+        assert len(xs) == self.world
+        return (C.c_void_p * self.world)(*[_ptr(x) for x in xs])
+
+    def alltoall(self, sendbufs, recvbufs, bytes_per_rank, algo=MP_ALGO_AUTO, stream=None):
+        """mp_emu_alltoall: every rank's MPI_Alltoall, one cooperative grid per step."""
+        st = lib().mp_emu_alltoall(self._h, self.world, self._bufs(sendbufs), self._bufs(recvbufs), bytes_per_rank,
+                                   algo, _stream(stream))
+        if st != 0:
+            raise MPError(st, lib().mp_last_error(self._h[0]).decode())
+
+    def allreduce(self, sendbufs, recvbufs, count, dtype=MP_DT_F32, algo=MP_ALGO_AUTO, stream=None):
+        """mp_emu_allreduce(MP_OP_SUM): every rank's MPI_Allreduce, one grid per step."""
+        st = lib().mp_emu_allreduce(self._h, self.world, self._bufs(sendbufs), self._bufs(recvbufs), count, dtype,
+                                    MP_OP_SUM, algo, _stream(stream))
+        if st != 0:
+            raise MPError(st, lib().mp_last_error(self._h[0]).decode())
 
     def close(self):
         if self.ctx:

@@ -375,3 +375,71 @@ def test_emulated_both_staged_pipeline_depths(torch_cuda, monkeypatch, stages):
                 W.run()
                 assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), expected(host, nb, ks, ps)), (stages, i, shift)
                 c1.free(dst)
+
+
+@pytest.mark.parametrize("w", [2, 3, 4])
+def test_emulated_collectives_against_mpi_definitions(torch_cuda, w):
+    """NEXT f3 in the emulated world: mp_emu_alltoall (Bruck, pairwise) and
+    mp_emu_allreduce (ring; K-nomial when W is a power of two) — the same plans and
+    per-step multi-path configs as mp_alltoall / mp_allreduce, each step one
+    cooperative grid — against the oracle's MPI definitions: Alltoall and the int32
+    Allreduce exact; fp32 / bf16 sums within the rounding bound of W - 1 reassociated
+    additions; out of place and in place."""
+    torch = torch_cuda
+    from oracle import collectives as OCL
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    BMAX = 300 * 1024 + 5
+    with world(w) as W:
+        sends = [torch.zeros(w * BMAX + 64, dtype=torch.uint8, device="cuda") for _ in range(w)]
+        rbufs = [W.ctx[r].alloc(w * BMAX + 64) for r in range(w)]
+        rviews = [mp.as_tensor(rbufs[r], w * BMAX + 64) for r in range(w)]
+
+        def put(t, arr):
+            t[:arr.nbytes].copy_(torch.from_numpy(arr.view(np.uint8)))
+            torch.cuda.synchronize()
+
+        for algo in (mp.MP_ALGO_BRUCK, mp.MP_ALGO_PAIRWISE):
+            for B in (1000, BMAX):
+                data = [np.random.default_rng(97 * s + B + algo).integers(0, 256, w * B, dtype=np.uint8)
+                        for s in range(w)]
+                for r in range(w):
+                    put(sends[r], data[r])
+                W.alltoall(sends, rviews, B, algo)
+                exp = OCL.alltoall(data, B)
+                for r in range(w):
+                    got = rviews[r][:w * B].cpu().numpy()
+                    assert np.array_equal(got, exp[r]), f"alltoall algo {algo} B {B} rank {r}"
+        algos = [mp.MP_ALGO_RING] + ([mp.MP_ALGO_KNOMIAL] if w & (w - 1) == 0 else [])
+        count = 100003
+        for algo in algos:
+            data = [np.random.default_rng(31 * s + algo).integers(-2 ** 31, 2 ** 31, count, dtype=np.int64)
+                    .astype(np.int32) for s in range(w)]
+            for r in range(w):
+                put(sends[r], data[r])
+            W.allreduce(sends, rviews, count, mp.MP_DT_I32, algo)
+            exp = OCL.allreduce_sum(data).astype(np.int32)
+            for r in range(w):
+                got = rviews[r][:4 * count].cpu().numpy().view(np.int32)
+                assert np.array_equal(got, exp), f"allreduce i32 algo {algo} rank {r}"
+            for dt, eps in ((mp.MP_DT_F32, 2.0 ** -24), (mp.MP_DT_BF16, 2.0 ** -8)):
+                vals, arrs = [], []
+                for r in range(w):
+                    x = np.random.default_rng(53 * r + algo + dt).standard_normal(count).astype(np.float32)
+                    if dt == mp.MP_DT_BF16:  # round to nearest even on the upper 16 bits
+                        u = x.view(np.uint32)
+                        u = ((u + 0x7FFF + ((u >> 16) & 1)) >> 16).astype(np.uint16)
+                        arrs.append(u)
+                        vals.append((u.astype(np.uint32) << 16).view(np.float32))
+                    else:
+                        arrs.append(x)
+                        vals.append(x)
+                    put(rviews[r], arrs[r])
+                W.allreduce(rviews, rviews, count, dt, algo)  # in place
+                exact = OCL.allreduce_sum(vals)
+                bound = (w - 1) * eps * np.sum([np.abs(v.astype(np.float64)) for v in vals], axis=0) * 1.01 + 1e-30
+                for r in range(w):
+                    raw = rviews[r][:arrs[r].nbytes].cpu().numpy()
+                    got = raw.view(np.float32) if dt == mp.MP_DT_F32 else \
+                        (raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32)
+                    err = np.abs(got.astype(np.float64) - exact)
+                    assert (err <= bound).all(), f"allreduce dtype {dt} algo {algo} rank {r}: {np.max(err / bound)}"
