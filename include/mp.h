@@ -203,9 +203,10 @@ int mp_finalize(mp_ctx *ctx);
  * context is returned.
  * In an emulated world, mp_send / mp_recv (and mp_select, mp_alloc, every model
  * call) behave as in a real job except that they launch nothing: they record the
- * kernels' parameter blocks.  mp_register, mp_alltoall / mp_allreduce (use
- * mp_emu_alltoall / mp_emu_allreduce) and the calibration calls return
- * MP_ERR_UNSUPPORTED; mp_finalize returns MP_ERR_STATE.
+ * kernels' parameter blocks.  mp_register / mp_deregister (use mp_emu_register /
+ * mp_emu_deregister), mp_alltoall / mp_allreduce (use mp_emu_alltoall /
+ * mp_emu_allreduce) and the calibration calls return MP_ERR_UNSUPPORTED; mp_finalize
+ * returns MP_ERR_STATE.
  *
  * mp_emu_run: ctxs = the world's n contexts in rank order.  Launches everything they
  * recorded since the last run as one cooperative grid on `stream` — per send its gate
@@ -222,6 +223,12 @@ int mp_finalize(mp_ctx *ctx);
  *
  * mp_finalize_emulated: tears down all n contexts (one thread each) and the world. */
 int mp_init_emulated(mp_ctx **ctxs, const mp_init_args *args);
+/* mp_register / mp_deregister of every rank of an emulated world at once (each rank's
+ * call runs on its own thread: the calls are collective): bufs[r], bytes[r] = rank r's
+ * buffer (NULL / 0: none), its region id returned in ids[r]; rules and errors as
+ * mp_register / mp_deregister (the first failing rank's status). */
+int mp_emu_register(mp_ctx **ctxs, int n, void *const *bufs, const uint64_t *bytes, int *ids);
+int mp_emu_deregister(mp_ctx **ctxs, int n, const int *ids);
 int mp_emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s);
 int mp_finalize_emulated(mp_ctx **ctxs, int n);
 

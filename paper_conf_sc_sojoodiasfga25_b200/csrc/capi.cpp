@@ -566,6 +566,16 @@ int mp_finalize_emulated(mp_ctx **ctxs, int n) {
   return mpx::emu_finalize_world(ctxs, n);
 }
 
+int mp_emu_register(mp_ctx **ctxs, int n, void *const *bufs, const uint64_t *bytes, int *ids) {
+  if (!ctxs || n < 2 || !ctxs[0] || !bufs || !bytes || !ids || !ctxs[0]->emulated) return MP_ERR_INVALID;
+  return mpx::emu_each_rank(ctxs, n, [&](int r) { return mp_register(ctxs[r], bufs[r], bytes[r], &ids[r]); });
+}
+
+int mp_emu_deregister(mp_ctx **ctxs, int n, const int *ids) {
+  if (!ctxs || n < 2 || !ctxs[0] || !ids || !ctxs[0]->emulated) return MP_ERR_INVALID;
+  return mpx::emu_each_rank(ctxs, n, [&](int r) { return mp_deregister(ctxs[r], ids[r]); });
+}
+
 int mp_emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
   if (!ctxs || n < 2 || !ctxs[0]) return MP_ERR_INVALID;
   if (!ctxs[0]->emulated) return fail(ctxs[0], MP_ERR_STATE, "mp_emu_run: not an emulated world");

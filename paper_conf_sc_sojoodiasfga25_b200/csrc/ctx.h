@@ -6,6 +6,7 @@
 
 #include <cstdint>
 #include <deque>
+#include <functional>
 #include <map>
 #include <string>
 #include <unordered_map>
@@ -227,6 +228,8 @@ int emu_init_world(mp_ctx **ctxs, const mp_init_args *a);
 int emu_finalize_world(mp_ctx **ctxs, int n);
 int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s);
 bool emu_thread();
+bool emu_rank_thread(const mp_ctx *c);  // this thread runs c's rank inside emu_each_rank
+int emu_each_rank(mp_ctx **ctxs, int n, const std::function<int(int)> &fn);
 int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id);
 // true when [p, p + n) lies in a receive region (heap or mp_register) of this rank
 bool world_receivable(mp_ctx *c, const void *p, uint64_t n);

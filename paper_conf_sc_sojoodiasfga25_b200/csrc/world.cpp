@@ -18,6 +18,7 @@
 #include <atomic>
 #include <chrono>
 #include <condition_variable>
+#include <functional>
 #include <map>
 #include <mutex>
 #include <thread>
@@ -745,7 +746,8 @@ void unmap(mp_ctx *c, int r, uint64_t key) {
 }  // namespace
 
 int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
-  if (c->emulated) return wfail(c, MP_ERR_UNSUPPORTED, "mp_register: not in an emulated world (use mp_alloc)");
+  if (c->emulated && !emu_rank_thread(c))
+    return wfail(c, MP_ERR_UNSUPPORTED, "mp_register: in an emulated world, through mp_emu_register");
   const int W = c->world;
   int rid = -1;
   for (int i = 1; i < static_cast<int>(c->regions.size()); ++i)
@@ -764,7 +766,7 @@ int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
     } else if (reinterpret_cast<uintptr_t>(buf) + bytes > base + size) {
       me.status = MP_ERR_INVALID;
       c->last_error = "mp_register: buffer runs past its allocation";
-    } else if (cudaIpcGetMemHandle(&me.h, reinterpret_cast<void *>(base)) != cudaSuccess) {
+    } else if (!c->emulated && cudaIpcGetMemHandle(&me.h, reinterpret_cast<void *>(base)) != cudaSuccess) {
       cudaGetLastError();
       me.status = MP_ERR_UNSUPPORTED;
       c->last_error = "mp_register: the allocation cannot be exported with cudaIpc (VMM / expandable segment?)";
@@ -794,6 +796,10 @@ int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
     if (all[r].status != 1) continue;
     if (r == c->rank) {
       row[r] = reinterpret_cast<uintptr_t>(buf);
+      continue;
+    }
+    if (c->emulated) {  // one process: the peer's buffer is addressed as allocated
+      row[r] = all[r].alloc_base + all[r].off;
       continue;
     }
     auto it = c->ipc_maps.find({r, all[r].alloc_base});
@@ -829,7 +835,8 @@ int world_register(mp_ctx *c, void *buf, uint64_t bytes, int *id) {
 }
 
 int world_deregister(mp_ctx *c, int id) {
-  if (c->emulated) return wfail(c, MP_ERR_UNSUPPORTED, "mp_deregister: not in an emulated world");
+  if (c->emulated && !emu_rank_thread(c))
+    return wfail(c, MP_ERR_UNSUPPORTED, "mp_deregister: in an emulated world, through mp_emu_deregister");
   const int W = c->world;
   if (id <= 0 || id >= static_cast<int>(c->regions.size()) || !c->regions[id].used)
     return wfail(c, MP_ERR_INVALID, "mp_deregister: unknown region id");
@@ -979,6 +986,34 @@ int emu_finalize_world(mp_ctx **ctxs, int n) {
 }
 
 bool emu_thread() { return t_emu_rank >= 0; }
+bool emu_rank_thread(const mp_ctx *c) { return t_emu_rank == c->rank; }
+
+// A collective call of every rank of an emulated world, each on its own thread (the
+// in-process all-gather needs all of them at once); the first failure is returned.
+int emu_each_rank(mp_ctx **ctxs, int n, const std::function<int(int)> &fn) {
+  EmuWorld *w = ctxs[0]->emu_world;
+  if (!w || n != w->world) return MP_ERR_INVALID;
+  for (int r = 0; r < n; ++r)
+    if (!ctxs[r] || ctxs[r]->emu_world != w || ctxs[r]->rank != r) return MP_ERR_INVALID;
+  std::vector<int> st(n, MP_OK);
+  std::vector<std::thread> th;
+  for (int r = 0; r < n; ++r)
+    th.emplace_back([&, r] {
+      t_emu_rank = r;
+      cudaSetDevice(ctxs[r]->device);
+      st[r] = fn(r);
+      if (st[r] != MP_OK) emu_abort(w);
+    });
+  for (std::thread &t : th) t.join();
+  {
+    std::lock_guard<std::mutex> lk(w->mu);  // a failed call aborted the all-gathers: reset for later calls
+    w->aborted = false;
+    w->arrived = 0;
+  }
+  for (int r = 0; r < n; ++r)
+    if (st[r] != MP_OK) return st[r];
+  return MP_OK;
+}
 
 int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
   mp_ctx *c = ctxs[0];

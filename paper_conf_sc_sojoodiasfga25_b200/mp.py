@@ -200,6 +200,9 @@ def lib():
             "mp_init_emulated": (C.c_int, [C.POINTER(P), C.POINTER(mp_init_args)]),
             "mp_emu_run": (C.c_int, [C.POINTER(P), C.c_int, P, C.POINTER(C.c_double)]),
             "mp_finalize_emulated": (C.c_int, [C.POINTER(P), C.c_int]),
+            "mp_emu_register": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(P), C.POINTER(C.c_uint64),
+                                          C.POINTER(C.c_int)]),
+            "mp_emu_deregister": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(C.c_int)]),
             "mp_emu_alltoall": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(P), C.POINTER(P), C.c_uint64, C.c_int, P]),
             "mp_emu_allreduce": (C.c_int, [C.POINTER(P), C.c_int, C.POINTER(P), C.POINTER(P), C.c_uint64, C.c_int,
                                            C.c_int, C.c_int, P]),
@@ -226,7 +229,8 @@ def exported_symbols() -> List[str]:
             "mp_set_window_model", "mp_get_window_model", "mp_predict_window", "mp_select_window",
             "mp_set_host_duplex", "mp_get_host_duplex", "mp_calibrate_window", "mp_calibrate_wake", "mp_fit_window",
             "mp_get_topology", "mp_set_topology", "mp_set_submit_time", "mp_get_submit_time",
-            "mp_init_emulated", "mp_emu_run", "mp_finalize_emulated", "mp_emu_alltoall", "mp_emu_allreduce"]
+            "mp_init_emulated", "mp_emu_run", "mp_finalize_emulated", "mp_emu_alltoall", "mp_emu_allreduce",
+            "mp_emu_register", "mp_emu_deregister"]
 
 
 def fit_hockney(n: Sequence[float], t: Sequence[float]):
@@ -645,6 +649,22 @@ class EmulatedWorld:
     def _bufs(self, xs):
         assert len(xs) == self.world
         return (C.c_void_p * self.world)(*[_ptr(x) for x in xs])
+
+    def register(self, tensors):
+        """mp_emu_register: tensors[r] (or None) becomes a receive region of rank r;
+        returns the region ids."""
+        ptrs = (C.c_void_p * self.world)(*[_ptr(t) if t is not None else None for t in tensors])
+        sizes = (C.c_uint64 * self.world)(*[t.numel() * t.element_size() if t is not None else 0 for t in tensors])
+        ids = (C.c_int * self.world)()
+        st = lib().mp_emu_register(self._h, self.world, ptrs, sizes, ids)
+        if st != 0:
+            raise MPError(st, lib().mp_last_error(self._h[0]).decode())
+        return list(ids)
+
+    def deregister(self, ids):
+        st = lib().mp_emu_deregister(self._h, self.world, (C.c_int * self.world)(*ids))
+        if st != 0:
+            raise MPError(st, lib().mp_last_error(self._h[0]).decode())
 
     def alltoall(self, sendbufs, recvbufs, bytes_per_rank, algo=MP_ALGO_AUTO, stream=None):
         """mp_emu_alltoall: every rank's MPI_Alltoall, one cooperative grid per step."""

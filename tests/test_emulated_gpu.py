@@ -443,3 +443,51 @@ def test_emulated_collectives_against_mpi_definitions(torch_cuda, w):
                         (raw.view(np.uint16).astype(np.uint32) << 16).view(np.float32)
                     err = np.abs(got.astype(np.float64) - exact)
                     assert (err <= bound).all(), f"allreduce dtype {dt} algo {algo} rank {r}: {np.max(err / bound)}"
+
+
+def test_emulated_registered_regions(torch_cuda):
+    """mp_register in the emulated world (mp_emu_register): receives into arbitrary torch
+    tensors — two views of one allocation on rank 1, then one tensor per rank in a ring,
+    all ring messages in one grid — over every path at once, bit-exact against the
+    oracle replay, bytes outside the views untouched; a deregistered region is
+    refused; region ids are reused."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    w = 3
+    with world(w, heap_bytes=16 * MiB) as W:
+        c = W.ctx
+        big = torch.zeros(16 * MiB, dtype=torch.uint8, device="cuda")
+        rings = [torch.zeros(4 * MiB, dtype=torch.uint8, device="cuda") for _ in range(w)]
+        va, vb = big[MiB + 256: 9 * MiB], big[10 * MiB: 15 * MiB]
+        ida = W.register([None, va, None])
+        idb = W.register([None, vb, None])
+        idr = W.register(rings)
+        assert len({ida[0], idb[0], idr[0]}) == 3 and ida == [ida[0]] * w
+        ps = c[0].paths(0, 1)
+        na = 3 * MiB + 4099
+        nb = [256 * 1024] * len(ps)
+        nb[0] = na - 256 * 1024 * (len(ps) - 1)
+        ks = [1] + [2] * (len(ps) - 1)
+        for case, (view, n, cb, ck) in enumerate([(va, na, nb, ks), (vb, 5 * MiB, None, None)]):
+            host, src = fill(torch, n, 60 + case)
+            c[0].send(src, n, 1, tag=300 + case, cfg=c[0].make_config(cb, ck, 0, 1) if cb else None)
+            c[1].recv(view[:n], n, 0, tag=300 + case)
+            W.run()
+            assert np.array_equal(view[:n].cpu().numpy(), expected(host, cb, ck, ps)), f"region case {case}"
+        outside = torch.cat([big[:MiB + 256], big[9 * MiB:10 * MiB], big[15 * MiB:]])
+        assert int(outside.count_nonzero()) == 0, "bytes outside the registered views were written"
+        n = 2 * MiB + 333
+        srcs = [fill(torch, n, 70 + r) for r in range(w)]
+        for r in range(w):
+            nxt, prv = (r + 1) % w, (r - 1) % w
+            c[r].recv(rings[r][4096 + 17: 4096 + 17 + n], n, prv, tag=400)
+            c[r].send(srcs[r][1], n, nxt, tag=400)
+        W.run()
+        for r in range(w):
+            assert np.array_equal(rings[r][4096 + 17: 4096 + 17 + n].cpu().numpy(), srcs[(r - 1) % w][0]), f"ring {r}"
+        for ids in (ida, idb, idr):
+            W.deregister(ids)
+        with pytest.raises(mp.MPError):
+            c[1].recv(va[:MiB], MiB, 0, tag=1)
+        assert W.register(rings) == ida  # ids are reused
+        W.deregister(ida)
