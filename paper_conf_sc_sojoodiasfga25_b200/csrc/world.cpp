@@ -1034,6 +1034,22 @@ int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
     send.insert(send.end(), cr->emu_send.begin(), cr->emu_send.end());
     recv.insert(recv.end(), cr->emu_recv.begin(), cr->emu_recv.end());
   }
+  // every recorded receive posts its clear-to-send at once: at most kCtsRing messages
+  // of one ordered pair per run (a real receiver's stream posts them one at a time)
+  {
+    std::map<std::pair<uint32_t, uint32_t>, uint32_t> per_pair;
+    for (const RecvParams &P : recv)
+      if (++per_pair[{P.src, P.me}] > kCtsRing) {
+        for (int r = 0; r < n; ++r) {
+          ctxs[r]->emu_send.clear();
+          ctxs[r]->emu_recv.clear();
+          ctxs[r]->emu_esend.clear();
+          ctxs[r]->emu_erecv.clear();
+        }
+        return wfail(c, MP_ERR_INVALID, "mp_emu_run: more than " + std::to_string(kCtsRing) +
+                                            " rendezvous messages of one pair in one run");
+      }
+  }
   // relay roles: one per (relay rank, sender), serving that sender's recorded doorbells
   // m0 .. m0 + count - 1 (what the relay's service thread and its lingering kernels do)
   std::map<std::pair<uint32_t, uint32_t>, std::vector<std::pair<uint64_t, uint32_t>>> bells;  // -> (m, g)

@@ -491,3 +491,35 @@ def test_emulated_registered_regions(torch_cuda):
             c[1].recv(va[:MiB], MiB, 0, tag=1)
         assert W.register(rings) == ida  # ids are reused
         W.deregister(ida)
+
+
+def test_emulated_doorbell_flow_control_one_grid(torch_cuda, monkeypatch):
+    """72 relayed messages from rank 0 through relay rank 3, all in flight in ONE grid
+    (alternately to ranks 1 and 2: 36 per pair, within the 64 outstanding messages a
+    pair's clear-to-send ring holds; one lane per stage group, 2-slot rings): more than
+    the 64-entry doorbell ring of (sender, relay), so the gates of messages 64.. wait for
+    the relay role to acknowledge doorbells 0.. (flow control) while it serves all 72 in
+    doorbell order; every message bit-exact."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    M = 72
+    monkeypatch.setenv("MPX_EAGER", "0")  # every message takes the rendezvous (and its relay)
+    with world(4, relay_ctas=1, host_path=0, slot_bytes=256 * 1024, slots=2, heap_bytes=64 * MiB) as W:
+        c = W.ctx
+        n = 192 * 1024 + 40
+        checks = []
+        for m in range(M):
+            d = 1 + m % 2
+            ps = c[0].paths(0, d)
+            nb, ks = [0] * len(ps), [1] + [0] * (len(ps) - 1)
+            i = ps.index((1, 3))
+            nb[0], nb[i], ks[i] = 40, n - 40, 1
+            host, src = fill(torch, n, 500 + m)
+            dst = c[d].alloc(n)
+            c[0].send(src, n, d, tag=m, cfg=c[0].make_config(nb, ks, 0, d))
+            c[d].recv(dst, n, 0, tag=m)
+            checks.append((dst, expected(host, nb, ks, ps), src))
+        torch.cuda.synchronize()
+        W.run()
+        for m, (dst, exp, _) in enumerate(checks):
+            assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), exp), m
