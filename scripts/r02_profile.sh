@@ -20,6 +20,7 @@ RELAY_K=32 timeout 600 ncu --set full --clock-control none --import-source on -k
   -o $OUT/relay_full python scripts/relay_one.py > $OUT/ncu_relay.log 2>&1
 # multi-rank engine on one GPU: the emulated world (one cooperative grid over every rank)
 timeout 900 python -m pytest tests/test_emulated_gpu.py -q -p no:cacheprovider > $OUT/pytest_emulated.log 2>&1
+timeout 300 python scripts/emu_perf.py --mib 256 --out $OUT/emu_perf_256.jsonl > $OUT/emu_perf.log 2>&1
 NG=$(nvidia-smi -L | wc -l)
 if [ "$NG" -ge 2 ]; then  # per-rank NVLink counters need one GPU per rank (ncu serialises a shared device)
   NCU_OUT=$OUT/ncu_world timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node $NG \
