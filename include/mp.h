@@ -34,7 +34,8 @@
 extern "C" {
 #endif
 
-#define MP_ABI_VERSION 4  /* 4: mp_path_params.wake (reading C28);
+#define MP_ABI_VERSION 5  /* 5: emulated world (mp_init_emulated, mp_emu_*; MP_INIT_EMULATED);
+                             4: mp_path_params.wake (reading C28);
                              3: topology (mp_get/set_topology), fingerprinted parameter files;
                              2: NEXT f2 calls; mp_model_opts.window (was reserved) */
 #define MP_MAX_PATHS 16

@@ -22,7 +22,7 @@ def test_header_symbols_exported():
     for n in names:
         assert hasattr(L, n), n
     assert sorted(mp.exported_symbols()) == names
-    assert L.mp_abi_version() == 4
+    assert L.mp_abi_version() == 5
 
 
 def test_strerror():
