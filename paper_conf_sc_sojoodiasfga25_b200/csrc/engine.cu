@@ -1631,21 +1631,39 @@ __device__ void relay_emu_body(const RelayParams &P, const uint32_t b, uint8_t *
   relay_body<D>(P, b, s_bell[0], s_bell[1], static_cast<uint32_t>((s_bell[2] >> 32) & 1u), smem);
 }
 
+// A role's parameter block, copied from the table into shared memory before the body
+// runs: the real kernels read theirs from the constant bank (__grid_constant__), and
+// the bodies' acquires invalidate L1, so a block left in global memory would cost an
+// L2 round trip per field access in the pipelines' geometry code.
+constexpr size_t cmax(size_t a, size_t b) { return a > b ? a : b; }
+constexpr size_t kEmuParamBytes =
+    cmax(cmax(sizeof(SendParams), sizeof(RecvParams)), cmax(sizeof(RelayParams), sizeof(EagerParams)));
+
+template <class T>
+__device__ __forceinline__ const T &emu_stage_params(const T *g, uint64_t *sm) {
+  static_assert(sizeof(T) % 8 == 0, "parameter blocks are 8-byte multiples");
+  const uint64_t *src = reinterpret_cast<const uint64_t *>(g);
+  for (uint32_t i = threadIdx.x; i < sizeof(T) / 8; i += blockDim.x) sm[i] = src[i];
+  __syncthreads();
+  return *reinterpret_cast<const T *>(sm);
+}
+
 template <uint32_t D>
 __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) emu_kernel(const __grid_constant__ EmuTable T) {
   extern __shared__ __align__(128) uint8_t dyn_smem[];
+  __shared__ __align__(16) uint64_t s_par[kEmuParamBytes / 8 + 1];
   const uint32_t blk = blockIdx.x;
   for (uint32_t i = 0; i < T.nroles; ++i) {
     const EmuRole R = T.roles[i];
     if (blk < R.cta0 || blk >= R.cta0 + R.n) continue;
     const uint32_t b = blk - R.cta0;
     switch (R.kind) {
-      case EMU_GATE: send_gate_body(T.send[R.idx]); break;
-      case EMU_SEND: send_body<D>(T.send[R.idx], b, dyn_smem); break;
-      case EMU_RECV: recv_body<D>(T.recv[R.idx], b, dyn_smem); break;
-      case EMU_RELAY: relay_emu_body<D>(T.relay[R.idx], b, dyn_smem); break;
-      case EMU_EAGER_SEND: eager_send_body(T.eager[R.idx], b); break;
-      case EMU_EAGER_RECV: eager_recv_body(T.eager[R.idx], b); break;
+      case EMU_GATE: send_gate_body(emu_stage_params(T.send + R.idx, s_par)); break;
+      case EMU_SEND: send_body<D>(emu_stage_params(T.send + R.idx, s_par), b, dyn_smem); break;
+      case EMU_RECV: recv_body<D>(emu_stage_params(T.recv + R.idx, s_par), b, dyn_smem); break;
+      case EMU_RELAY: relay_emu_body<D>(emu_stage_params(T.relay + R.idx, s_par), b, dyn_smem); break;
+      case EMU_EAGER_SEND: eager_send_body(emu_stage_params(T.eager + R.idx, s_par), b); break;
+      case EMU_EAGER_RECV: eager_recv_body(emu_stage_params(T.eager + R.idx, s_par), b); break;
       default: break;
     }
     return;
