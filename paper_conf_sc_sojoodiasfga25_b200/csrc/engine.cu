@@ -36,6 +36,21 @@ __device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
 
 __device__ __forceinline__ void fence_acq_rel_sys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 
+// Polling and publishing under load: an acquire or release at system scope is a
+// MEMBAR.SYS, which measured ~12 µs while the engine's streams are in flight
+// (scripts/diag/lane_trace.py).  Polls are relaxed, with one acquire once the value has
+// arrived; several flags published together share one fence, then relaxed stores
+// (the PTX release pattern: a fence followed by a strong write).
+__device__ __forceinline__ uint64_t ld_relaxed_sys(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ void st_relaxed_sys(uint64_t *p, uint64_t v) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -271,8 +286,11 @@ __device__ __forceinline__ bool wait_flags(const uint64_t *flags, uint32_t n, ui
     const uint64_t t_start = globaltimer();
     int why = 0;
     for (uint32_t it = 0;; ++it) {
-      const bool mine = lane >= n || ld_acquire_sys(flags + lane) >= target;
-      if (__all_sync(0xffffffffu, mine)) break;
+      const bool mine = lane >= n || ld_relaxed_sys(flags + lane) >= target;
+      if (__all_sync(0xffffffffu, mine)) {  // one acquire per flag once all have arrived
+        if (lane < n) (void)ld_acquire_sys(flags + lane);
+        break;
+      }
       if (globaltimer() - t_start > timeout_ns) {
         why = 1;
         break;
@@ -301,7 +319,7 @@ __device__ __forceinline__ bool wait_word(const uint64_t *w, uint64_t target, ui
                                           int32_t *err, int *s_abort) {
   if (threadIdx.x == 0) {
     const uint64_t t_start = globaltimer();
-    for (uint32_t it = 0; ld_acquire_sys(w) < target; ++it) {
+    for (uint32_t it = 0; ld_relaxed_sys(w) < target || ld_acquire_sys(w) < target; ++it) {
       if (globaltimer() - t_start > timeout_ns) {
         atomicExch(err, DERR_TIMEOUT);
         *s_abort = 1;
@@ -439,11 +457,6 @@ __device__ __forceinline__ bool mbar_wait_or_stop(uint32_t bar, uint32_t parity,
   return true;
 }
 
-__device__ __forceinline__ uint64_t ld_relaxed_sys(const uint64_t *p) {
-  uint64_t v;
-  asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
 
 // Block one thread until *f >= target: 1, or -1 on timeout (DERR_TIMEOUT raised) or
 // once the context's error word is set.  Polls relaxed (an acquire load invalidates
@@ -475,6 +488,15 @@ template <int MODE>
 __device__ __forceinline__ void bytes_copy(uint8_t *d, const uint8_t *s, uint64_t n) {
   for (uint64_t i = 0; i < n; ++i) d[i] = ld1<MODE>(s + i);
 }
+
+#ifdef MPX_TRACE  // (design experiment: per-CTA, per-chunk timestamps of the streamed lanes)
+__device__ uint64_t *g_mpx_trace;  // [CTA][128 chunks][4]: ready, loaded, stored, (unused)
+__device__ __forceinline__ void trace(uint32_t j, uint32_t ev) {
+  if (g_mpx_trace && j < 128) g_mpx_trace[(static_cast<uint64_t>(blockIdx.x) * 128 + j) * 4 + ev] = globaltimer();
+}
+#else
+__device__ __forceinline__ void trace(uint32_t, uint32_t) {}
+#endif
 
 // The four roles; a thread returns from here when its role is done (threads other than
 // 0, 32, 64 and 96 at once).
@@ -515,6 +537,7 @@ __device__ void lane_stream_roles(Role &R, uint32_t nchunks, uint8_t *smem) {
         st_release_cta_shared(&s_stop, 1);
         return;
       }
+      trace(j, 0);
       st_release_cta_shared(&s_ready, j + 1);
     }
     return;
@@ -529,8 +552,14 @@ __device__ void lane_stream_roles(Role &R, uint32_t nchunks, uint8_t *smem) {
         __nanosleep(32);
         continue;
       }
-      for (; pl < a; ++pl) R.loaded(pl);
-      for (; ps < b; ++ps) R.stored(ps, s_words[ps % kStreamAhead]);
+      for (; pl < a; ++pl) {
+        trace(pl, 1);
+        R.loaded(pl);
+      }
+      for (; ps < b; ++ps) {
+        trace(ps, 2);
+        R.stored(ps, s_words[ps % kStreamAhead]);
+      }
       st_release_cta_shared(&s_pub, ps);
     }
     return;
@@ -1093,10 +1122,11 @@ struct HostConsumer {
 // their successor launch at once and wait for their predecessor (pdl_enter).
 __device__ void send_gate_body(const SendParams &P) {
   if (threadIdx.x != 0) return;
+  trace(126, 0);
   MsgEntry *cts = entry_at(P.my_ctrl, P.L.cts, P.dst, P.seq);
   const uint64_t t_start = globaltimer();
-  uint64_t seen;
-  while ((seen = ld_acquire_sys(&cts->seq1)) < P.seq + 1) {
+  uint64_t seen = 0;
+  while (ld_relaxed_sys(&cts->seq1) < P.seq + 1 || (seen = ld_acquire_sys(&cts->seq1)) < P.seq + 1) {
     if (globaltimer() - t_start > P.timeout_ns) {
       atomicExch(P.err, DERR_TIMEOUT);
       return;
@@ -1127,42 +1157,52 @@ __device__ void send_gate_body(const SendParams &P) {
   h->e = host_bytes;
   h->f = reinterpret_cast<uintptr_t>(P.src + host_off) & 15u;
   h->g = P.align;
-  st_release_sys(&h->seq1, P.seq + 1);
   if (bad) {
+    st_release_sys(&h->seq1, P.seq + 1);
     atomicExch(P.err, DERR_MISMATCH);
-  } else {
-    for (uint32_t i = 0; i < P.npaths; ++i) {  // doorbells (relay rank's host thread)
-      const SendParams::StagedDesc &d = P.sp[i];
-      if (d.kind != 1) continue;
-      BellEntry *e = d.bell + d.m % kBellRing;
-      // flow control: the entry is reused only once the relay has taken the doorbell
-      // kBellRing messages back (its kernels acknowledge into this rank's control
-      // block); only more than kBellRing relayed messages in flight through one relay
-      // (many streams) ever wait here
-      if (d.m >= kBellRing) {
-        const uint64_t *ack = reinterpret_cast<const uint64_t *>(P.my_ctrl + P.L.bell_ack) + d.relay * 16;
-        const uint64_t need = d.m + 1 - kBellRing, t0 = globaltimer();
-        while (ld_acquire_sys(ack) < need) {
-          if (globaltimer() - t0 > P.timeout_ns) {
-            atomicExch(P.err, DERR_TIMEOUT);
-            break;
-          }
-          __nanosleep(256);
-        }
-      }
-      // co-alignment of source and target (mod 16 is the same in every process's
-      // mapping: mapped bases are >= 256-B aligned) lets the relay stream its lanes
-      const uint64_t region = ld_volatile(&cts->d);
-      const bool aligned = region < kMaxRegions &&
-                           ((reinterpret_cast<uintptr_t>(P.src) ^
-                             (reinterpret_cast<uintptr_t>(region_base(P.my_ctrl, P.L, region, P.dst)) + ld_volatile(&cts->a))) &
-                            15u) == 0;
-      e->q0 = d.q0;
-      e->k = d.k;
-      e->g = d.g | (aligned ? (1ull << 32) : 0ull);
-      st_release_sys(&e->tag, d.m + 1);
-    }
+    return;
   }
+  // doorbells (relay rank's host thread): the fields of every one first, then ONE
+  // system-scope fence for the message header and all of them, then their flags —
+  // a release per flag cost a MEMBAR.SYS each (~12 µs under load), 7 for config 3
+  for (uint32_t i = 0; i < P.npaths; ++i) {
+    const SendParams::StagedDesc &d = P.sp[i];
+    if (d.kind != 1) continue;
+    BellEntry *e = d.bell + d.m % kBellRing;
+    // flow control: the entry is reused only once the relay has taken the doorbell
+    // kBellRing messages back (its kernels acknowledge into this rank's control
+    // block); only more than kBellRing relayed messages in flight through one relay
+    // (many streams) ever wait here
+    if (d.m >= kBellRing) {
+      const uint64_t *ack = reinterpret_cast<const uint64_t *>(P.my_ctrl + P.L.bell_ack) + d.relay * 16;
+      const uint64_t need = d.m + 1 - kBellRing, t0 = globaltimer();
+      while (ld_relaxed_sys(ack) < need || ld_acquire_sys(ack) < need) {
+        if (globaltimer() - t0 > P.timeout_ns) {
+          atomicExch(P.err, DERR_TIMEOUT);
+          break;
+        }
+        __nanosleep(256);
+      }
+    }
+    // co-alignment of source and target (mod 16 is the same in every process's
+    // mapping: mapped bases are >= 256-B aligned) lets the relay stream its lanes
+    const uint64_t region = ld_volatile(&cts->d);
+    const bool aligned = region < kMaxRegions &&
+                         ((reinterpret_cast<uintptr_t>(P.src) ^
+                           (reinterpret_cast<uintptr_t>(region_base(P.my_ctrl, P.L, region, P.dst)) + ld_volatile(&cts->a))) &
+                          15u) == 0;
+    e->q0 = d.q0;
+    e->k = d.k;
+    e->g = d.g | (aligned ? (1ull << 32) : 0ull);
+  }
+  trace(126, 1);
+  fence_acq_rel_sys();
+  st_relaxed_sys(&h->seq1, P.seq + 1);
+  for (uint32_t i = 0; i < P.npaths; ++i) {
+    const SendParams::StagedDesc &d = P.sp[i];
+    if (d.kind == 1) st_relaxed_sys(&(d.bell + d.m % kBellRing)->tag, d.m + 1);
+  }
+  trace(126, 2);
 }
 
 __global__ void send_gate_kernel(const __grid_constant__ SendParams P) {
@@ -1278,8 +1318,10 @@ __device__ void recv_body(const RecvParams &P, const uint32_t b, uint8_t *dyn_sm
       cts->b = P.bytes;
       cts->c = P.tag;
       cts->d = P.region;
+      trace(125, 0);
       fence_acq_rel_sys();
-      st_release_sys(&cts->seq1, P.seq + 1);
+      st_relaxed_sys(&cts->seq1, P.seq + 1);
+      trace(125, 1);
       // A10: wait until every byte of the message has been counted in
       const uint64_t *done = done_at(P.my_ctrl, P.L, P.src);
       const uint64_t t_start = globaltimer();
@@ -1431,7 +1473,7 @@ __device__ void relay_body(const RelayParams &P, const uint32_t b, uint64_t q0, 
     }
     if (threadIdx.x == 0) {
       const uint64_t t0 = globaltimer();
-      while (ld_acquire_sys(dec) != m + 2) {
+      while (ld_relaxed_sys(dec) != m + 2 || ld_acquire_sys(dec) != m + 2) {
         if (globaltimer() - t0 > P.linger_ns + P.timeout_ns) {
           atomicExch(P.err, DERR_TIMEOUT);
           s_abort = 1;
@@ -1599,11 +1641,12 @@ template <uint32_t D>
 __device__ void relay_emu_body(const RelayParams &P, const uint32_t b, uint8_t *smem) {
   __shared__ uint64_t s_bell[3];
   __shared__ int s_ok;
+  if (threadIdx.x == 0) trace(124, 0);
   if (threadIdx.x == 0) {
     const BellEntry *e = P.bells + P.m0 % kBellRing;
     const uint64_t t0 = globaltimer();
     int ok = 1;
-    while (ld_acquire_sys(&e->tag) != P.m0 + 1) {
+    while (ld_relaxed_sys(&e->tag) != P.m0 + 1 || ld_acquire_sys(&e->tag) != P.m0 + 1) {
       if (*reinterpret_cast<volatile int32_t *>(P.err) != 0) {  // the relay rank already failed
         ok = 0;
         break;
@@ -1627,6 +1670,7 @@ __device__ void relay_emu_body(const RelayParams &P, const uint32_t b, uint8_t *
     s_ok = ok;
   }
   __syncthreads();
+  if (threadIdx.x == 0) trace(124, 1);
   if (!s_ok) return;
   relay_body<D>(P, b, s_bell[0], s_bell[1], static_cast<uint32_t>((s_bell[2] >> 32) & 1u), smem);
 }
@@ -1830,6 +1874,14 @@ cudaError_t emu_occupancy(int *n) {
   return e;
 }
 }  // namespace
+
+#ifdef MPX_TRACE
+}  // namespace mpx
+extern "C" int mpx_trace_set(void *p) {
+  return static_cast<int>(cudaMemcpyToSymbol(mpx::g_mpx_trace, &p, sizeof(p)));
+}
+namespace mpx {
+#endif
 
 int emu_capacity(int *per_sm, int *per_sm_deep) {
   cudaError_t e = emu_occupancy<kBulkStages>(per_sm);
