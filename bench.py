@@ -331,14 +331,22 @@ def esel_grid(n, npaths, host_idx):
 
 
 def rank_device(local, world):
-    """The GPU of this rank: one per rank.  Ranks whose kernels wait on one another are
-    never separate launches sharing a GPU (B200 profiling guide); the one-GPU stand-in
-    for the multi-rank engine is the emulated world (tests/test_emulated_gpu.py)."""
+    """The GPU of this rank: one per rank (device LOCAL_RANK, or device 0 when the
+    launcher shows each rank only its own GPU), checked by all-gathering the GPUs'
+    UUIDs.  Ranks whose kernels wait on one another are never separate launches sharing
+    a GPU (B200 profiling guide); the one-GPU stand-in for the multi-rank engine is the
+    emulated world (tests/test_emulated_gpu.py).  Needs the process group."""
     import torch
+    import torch.distributed as dist
     n = torch.cuda.device_count()
-    if n < world:
-        raise SystemExit(f"bench.py --gpus {world}: needs {world} GPUs (one per rank), found {n}")
-    return local
+    dev = local if local < n else 0
+    uuid = str(torch.cuda.get_device_properties(dev).uuid) if n else ""
+    uuids = [None] * world
+    dist.all_gather_object(uuids, uuid)
+    if not n or len(set(uuids)) != world:
+        raise SystemExit(f"bench.py --gpus {world}: needs one GPU per rank; this node gives the ranks "
+                         f"{len(set(u for u in uuids if u))} distinct GPU(s)")
+    return dev
 
 
 def p2p_roles(world):
