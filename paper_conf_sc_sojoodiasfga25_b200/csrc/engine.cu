@@ -1639,15 +1639,40 @@ __global__ void __launch_bounds__(kThreads) direct_reg_kernel(const __grid_const
 // next-message decisions as a lingering relay kernel).
 template <uint32_t D>
 __device__ void relay_emu_body(const RelayParams &P, const uint32_t b, uint8_t *smem) {
+  // CTA 0 alone polls the doorbell in pinned host memory (as the relay rank's one host
+  // thread does) and hands {q0, k, g} to the role's other CTAs through device words:
+  // sixteen CTAs polling host memory at system scope made every MEMBAR.SYS on the GPU
+  // slower (a clear-to-send post 1.6 -> 9.7 µs; scripts/diag/bell_poll.sh)
   __shared__ uint64_t s_bell[3];
   __shared__ int s_ok;
   if (threadIdx.x == 0) trace(124, 0);
   if (threadIdx.x == 0) {
-    const BellEntry *e = P.bells + P.m0 % kBellRing;
     const uint64_t t0 = globaltimer();
     int ok = 1;
-    while (ld_relaxed_sys(&e->tag) != P.m0 + 1 || ld_acquire_sys(&e->tag) != P.m0 + 1) {
-      if (*reinterpret_cast<volatile int32_t *>(P.err) != 0) {  // the relay rank already failed
+    if (b == 0) {
+      const BellEntry *e = P.bells + P.m0 % kBellRing;
+      while (ld_relaxed_sys(&e->tag) != P.m0 + 1 || ld_acquire_sys(&e->tag) != P.m0 + 1) {
+        if (*reinterpret_cast<volatile int32_t *>(P.err) != 0) {  // the relay rank already failed
+          ok = 0;
+          break;
+        }
+        if (globaltimer() - t0 > P.timeout_ns) {
+          atomicExch(P.err, DERR_TIMEOUT);
+          ok = 0;
+          break;
+        }
+        __nanosleep(256);
+      }
+      P.first[1] = ok ? ld_volatile(&e->q0) : 0;
+      P.first[2] = ok ? ld_volatile(&e->k) : 0;
+      P.first[3] = ok ? ld_volatile(&e->g) : 0;
+      asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(P.first), "l"(ok ? P.m0 + 1 : ~0ull) : "memory");
+    }
+    uint64_t tag;
+    for (;;) {
+      asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(tag) : "l"(P.first) : "memory");
+      if (tag == P.m0 + 1) break;
+      if (tag == ~0ull) {  // CTA 0 failed (already reported)
         ok = 0;
         break;
       }
@@ -1656,12 +1681,12 @@ __device__ void relay_emu_body(const RelayParams &P, const uint32_t b, uint8_t *
         ok = 0;
         break;
       }
-      __nanosleep(256);
+      __nanosleep(128);
     }
     if (ok) {
-      s_bell[0] = ld_volatile(&e->q0);
-      s_bell[1] = ld_volatile(&e->k);
-      s_bell[2] = ld_volatile(&e->g);
+      s_bell[0] = ld_volatile(P.first + 1);
+      s_bell[1] = ld_volatile(P.first + 2);
+      s_bell[2] = ld_volatile(P.first + 3);
       if (static_cast<uint32_t>(s_bell[2] & 0xffffffffu) != P.g) {  // the role's CTAs are the lanes
         atomicExch(P.err, DERR_MISMATCH);
         ok = 0;

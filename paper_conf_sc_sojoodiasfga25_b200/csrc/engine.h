@@ -256,6 +256,8 @@ struct RelayParams {
   uint64_t m0;                 // doorbell index of the first message
   uint64_t linger_ns;          // how long CTA 0 waits for the next doorbell (0: one message)
   uint64_t max_msgs;           // > 0 (emu_kernel): serve exactly this many messages; 0: linger rule
+  uint64_t *first;             // emu_kernel: device words {tag, q0, k, g} of the first doorbell,
+                               // read from host memory by CTA 0 alone and handed to the others
   const BellEntry *bells;      // the sender's doorbell row in this rank's segment (mapped host)
   uint64_t *dec;               // [kBellRing][4] device words: CTA 0's next-message decisions
   uint32_t *exit_cnt;          // device word: CTAs that have left

@@ -1160,13 +1160,16 @@ int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
                o_relay = al(o_recv + recv.size() * sizeof(RecvParams)),
                o_eager = al(o_relay + relay.size() * sizeof(RelayParams)),
                o_state = al(o_eager + eager.size() * sizeof(EagerParams)),
-               total = al(o_state + std::max<size_t>(1, relay.size()) * 2 * sizeof(uint64_t));
+               o_first = al(o_state + std::max<size_t>(1, relay.size()) * 2 * sizeof(uint64_t)),
+               total = al(o_first + std::max<size_t>(1, relay.size()) * 4 * sizeof(uint64_t));
   std::vector<uint8_t> h(total, 0);
   void *d = nullptr;
   CKW(cudaMalloc(&d, total));
   uint8_t *db = static_cast<uint8_t *>(d);
-  for (size_t i = 0; i < relay.size(); ++i)
+  for (size_t i = 0; i < relay.size(); ++i) {
     relay[i].state = reinterpret_cast<uint64_t *>(db + o_state) + 2 * i;  // the relay's exit record (unread)
+    relay[i].first = reinterpret_cast<uint64_t *>(db + o_first) + 4 * i;  // zeroed by the upload below
+  }
   std::memcpy(h.data() + o_roles, roles.data(), roles.size() * sizeof(EmuRole));
   if (!send.empty()) std::memcpy(h.data() + o_send, send.data(), send.size() * sizeof(SendParams));
   if (!recv.empty()) std::memcpy(h.data() + o_recv, recv.data(), recv.size() * sizeof(RecvParams));
