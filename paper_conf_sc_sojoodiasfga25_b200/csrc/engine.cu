@@ -474,6 +474,38 @@ __device__ __forceinline__ int poll_flag(const uint64_t *f, uint64_t target, uin
   }
 }
 
+// GPU scope: the loopback engine's device rings are written and read on one GPU, so
+// their flags need only MEMBAR.GPU, not the MEMBAR.SYS that cross-GPU and host-memory
+// handoffs need (µs under load).
+__device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t *p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t *p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// poll_flag at GPU scope (gpu == true) or system scope
+__device__ __forceinline__ int poll_flag_scoped(const uint64_t *f, uint64_t target, uint64_t timeout_ns, int32_t *err,
+                                                bool gpu) {
+  if (!gpu) return poll_flag(f, target, timeout_ns, err);
+  const uint64_t t0 = globaltimer();
+  for (uint32_t it = 0;; ++it) {
+    if (ld_relaxed_gpu(f) >= target && ld_acquire_gpu(f) >= target) return 1;
+    if (globaltimer() - t0 > timeout_ns) {
+      atomicExch(err, DERR_TIMEOUT);
+      return -1;
+    }
+    if ((it & 63u) == 63u && *reinterpret_cast<volatile int32_t *>(err) != 0) return -1;
+    __nanosleep(128);
+  }
+}
+
 __device__ __forceinline__ uint32_t ld_acquire_cta_shared(const uint32_t *p) {
   uint32_t v;
   asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
@@ -767,14 +799,16 @@ struct LoopProducer {
   }
   __device__ int wait(uint32_t j) {
     const uint64_t q = p->q0 + j;
-    return poll_flag(p->freef + (q % p->slots) * kFlagStride + r, q / p->slots, timeout_ns, err);
+    return poll_flag_scoped(p->freef + (q % p->slots) * kFlagStride + r, q / p->slots, timeout_ns, err, !p->host_ring);
   }
   __device__ int fetch(uint32_t, uint64_t *) { return 1; }
   __device__ void before_store(uint32_t) {}
   __device__ void loaded(uint32_t) {}
   __device__ void stored(uint32_t j, const uint64_t *) {
     const uint64_t q = p->q0 + j;
-    st_release_sys(p->full + (q % p->slots) * kFlagStride + r, q / p->slots + 1);
+    uint64_t *f = p->full + (q % p->slots) * kFlagStride + r;
+    if (p->host_ring) st_release_sys(f, q / p->slots + 1);  // data in host memory
+    else st_release_gpu(f, q / p->slots + 1);
   }
 };
 
@@ -792,13 +826,15 @@ struct LoopConsumer {
   }
   __device__ int wait(uint32_t j) {
     const uint64_t q = p->q0 + j;
-    return poll_flag(p->full + (q % p->slots) * kFlagStride + r, q / p->slots + 1, timeout_ns, err);
+    return poll_flag_scoped(p->full + (q % p->slots) * kFlagStride + r, q / p->slots + 1, timeout_ns, err, !p->host_ring);
   }
   __device__ int fetch(uint32_t, uint64_t *) { return 1; }
   __device__ void before_store(uint32_t) {}
   __device__ void loaded(uint32_t j) {
     const uint64_t q = p->q0 + j;
-    st_release_sys(p->freef + (q % p->slots) * kFlagStride + r, q / p->slots + 1);
+    uint64_t *f = p->freef + (q % p->slots) * kFlagStride + r;
+    if (p->host_ring) st_release_sys(f, q / p->slots + 1);
+    else st_release_gpu(f, q / p->slots + 1);
   }
   __device__ void stored(uint32_t, const uint64_t *) {}
 };
