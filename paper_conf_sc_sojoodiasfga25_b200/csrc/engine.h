@@ -190,6 +190,8 @@ struct CtrlLayout {
   uint64_t relay_dec = 0;              // [world(sender)][kBellRing][4] u64: a relay kernel's next-message decisions
   uint64_t relay_exit = 0;             // [world(sender)] u32, 128-B padded: relay CTAs that have left
   uint64_t bell_ack = 0;               // [world(relay)] u64, 128-B padded: doorbells the relay has taken — on the sender
+  uint64_t dcnt = 0;                   // [world(dst)][kCtsRing] u64: direct CTAs of message m done — on the sender
+  uint64_t dfree = 0;                  // [world(dst)][kCtsRing] u64: last message whose direct CTAs were counted + 1
   uint64_t total = 0;
 };
 
