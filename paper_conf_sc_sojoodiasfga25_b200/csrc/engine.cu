@@ -1068,6 +1068,7 @@ struct RelayConsumer {
   uint64_t q0;  // the message's first ring sequence
   uint64_t k;   // the message's chunks
   uint64_t acc; // bytes of this lane stored so far (counted once, after its last chunk)
+  uint64_t m;   // the message's doorbell index on (sender, this relay)
   __device__ uint8_t *lane(uint32_t j) const {
     const uint64_t s = (q0 + j) % P->L.slots;
     return P->my_ctrl + P->L.ring_data + (static_cast<uint64_t>(P->sender) * P->L.slots + s) * P->L.stride +
@@ -1097,13 +1098,28 @@ struct RelayConsumer {
     st_release_sys(flags_at(P->sender_ctrl, P->L.relay_free, P->me, P->L.slots, q % P->L.slots) + r,
                    q / P->L.slots + 1);
   }
-  // The receiver only waits for the message's whole byte count (A10), so a lane counts
-  // its bytes once, after its last chunk: one system-scope reduction into the
-  // destination GPU's counter per lane and message instead of one per chunk (the
-  // publisher's other release per chunk, the free flag, is what the sender waits on).
+  // The receiver only waits for the message's whole byte count (A10).  After its last
+  // chunk a lane adds (its bytes << 8 | 1) into the message's counter slot on this GPU
+  // (GPU-scope acq_rel); the lane that completes the count releases the message's
+  // relayed bytes into the destination's counter — one system-scope release per
+  // relayed message, as the direct group's (§6).  Slot m % kBellRing is reused 64
+  // messages later; a relay's lanes drift at most a message or two apart (the sender's
+  // kernels on one relay ring run in order and wait for its free flags).
   __device__ void stored(uint32_t j, const uint64_t *w) {
     acc += w[2];
-    if (j + 1 == k) red_add_release_sys(done_at(P->peer[w[0]].ctrl, P->L, P->sender), acc);
+    if (j + 1 != k) return;
+    uint64_t *cnt = reinterpret_cast<uint64_t *>(P->my_ctrl + P->L.rcnt) +
+                    static_cast<uint64_t>(P->sender) * kBellRing + m % kBellRing;
+    uint64_t old;
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], %2;"
+                 : "=l"(old)
+                 : "l"(cnt), "l"((acc << 8) | 1u)
+                 : "memory");
+    if ((old & 0xffu) + 1 == P->g) {
+      *reinterpret_cast<volatile uint64_t *>(cnt) = 0;
+      const uint64_t total = (old >> 8) + acc;
+      if (total) red_add_release_sys(done_at(P->peer[w[0]].ctrl, P->L, P->sender), total);
+    }
   }
 };
 
@@ -1460,11 +1476,11 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) recv_kerne
 // linger_ns, so back-to-back relayed messages pay no relaunch.  A relay kernel still
 // ends once its sender goes quiet: nothing outlives the traffic by more than the linger.
 template <uint32_t D>
-__device__ bool relay_message(const RelayParams &P, const uint32_t r, uint64_t q0, uint64_t k, uint32_t aligned,
-                              int *s_abort, uint8_t *smem) {
+__device__ bool relay_message(const RelayParams &P, const uint32_t r, uint64_t m, uint64_t q0, uint64_t k,
+                              uint32_t aligned, int *s_abort, uint8_t *smem) {
   const uint64_t lstride = lane_stride(P.L.slot_bytes, P.g);
   if (P.copy_mode == 1 && aligned) {  // streamed lane (the sender found source and target co-aligned)
-    RelayConsumer R{&P, r, lstride, q0, k, 0};
+    RelayConsumer R{&P, r, lstride, q0, k, 0, m};
     lane_stream<LD_RING, D>(R, static_cast<uint32_t>(k), smem);
     return *reinterpret_cast<volatile int32_t *>(P.err) == 0;
   }
@@ -1508,7 +1524,7 @@ __device__ void relay_body(const RelayParams &P, const uint32_t b, uint64_t q0, 
   uint64_t *ack = reinterpret_cast<uint64_t *>(P.sender_ctrl + P.L.bell_ack) + P.me * 16;
   if (b == 0 && threadIdx.x == 0) st_release_sys(ack, m + 1);
   for (;;) {
-    if (!relay_message<D>(P, b, q0, k, aligned, &s_abort, dyn_smem)) break;
+    if (!relay_message<D>(P, b, m, q0, k, aligned, &s_abort, dyn_smem)) break;
     // the sender's next message: CTA 0 looks for its doorbell for up to linger_ns and
     // publishes the decision; every CTA follows it
     uint64_t *dec = P.dec + ((m + 1) % kBellRing) * 4;

@@ -192,6 +192,8 @@ struct CtrlLayout {
   uint64_t bell_ack = 0;               // [world(relay)] u64, 128-B padded: doorbells the relay has taken — on the sender
   uint64_t dcnt = 0;                   // [world(dst)][kCtsRing] u64: direct CTAs of message m done — on the sender
   uint64_t dfree = 0;                  // [world(dst)][kCtsRing] u64: last message whose direct CTAs were counted + 1
+  uint64_t rcnt = 0;                   // [world(sender)][kBellRing] u64: relay lanes of message m done
+                                       //   (bytes << 8 | lanes) — on the relay
   uint64_t total = 0;
 };
 
