@@ -1302,6 +1302,7 @@ __device__ void send_body(const SendParams &P, const uint32_t b, uint8_t *dyn_sm
   const uint64_t base = s_off;
   uint64_t *done = done_at(P.dst_ctrl, P.L, P.me);
   if (b < P.g_direct) {  // A7: direct NVLink stores into the receiver's heap
+    if (threadIdx.x == 0) trace(120, 0);
     if (P.copy_mode == 1)
       bulk_copy<LD_SRC>(s_dst, P.src, P.direct_bytes, b, P.g_direct, dyn_smem, P.bulk_stages);
     else
@@ -1314,6 +1315,7 @@ __device__ void send_body(const SendParams &P, const uint32_t b, uint8_t *dyn_sm
     // last CTA's RMW acquires before its system-scope release.  The counter slot is
     // reused kCtsRing messages later; the send gate waits for it (dfree).
     __syncthreads();
+    if (threadIdx.x == 0) trace(120, 1);
     if (threadIdx.x == 0) {
       uint64_t *cnt = reinterpret_cast<uint64_t *>(P.my_ctrl + P.L.dcnt) +
                       static_cast<uint64_t>(P.dst) * kCtsRing + P.seq % kCtsRing;
@@ -1321,7 +1323,9 @@ __device__ void send_body(const SendParams &P, const uint32_t b, uint8_t *dyn_sm
       asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(cnt) : "memory");
       if (old + 1 == P.g_direct) {
         *reinterpret_cast<volatile uint64_t *>(cnt) = 0;
+        trace(121, 0);
         if (P.direct_bytes) red_add_release_sys(done, P.direct_bytes);
+        trace(121, 1);
         uint64_t *fr = reinterpret_cast<uint64_t *>(P.my_ctrl + P.L.dfree) +
                        static_cast<uint64_t>(P.dst) * kCtsRing + P.seq % kCtsRing;
         st_release_gpu(fr, P.seq + 1);
@@ -1424,7 +1428,9 @@ __device__ void recv_body(const RecvParams &P, const uint32_t b, uint8_t *dyn_sm
         }
         __nanosleep(128);
       }
+      trace(123, 0);
       fence_acq_rel_sys();
+      trace(123, 1);
     }
     return;
   }
