@@ -1,5 +1,5 @@
 #!/bin/bash
-# Diagnose the multi-rank engine with all ranks on one GPU (under gpurun).
+# Diagnose the multi-rank engine (one GPU per rank: tests/_world_worker.py puts rank r on GPU r).
 # Usage: bash scripts/diag/diag_world.sh <outdir> <world> [MPX_NO_RELAY=0|1]
 OUT=${1:-gpurun_out/diag}; W=${2:-3}; NR=${3:-0}
 mkdir -p $OUT
