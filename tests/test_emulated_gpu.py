@@ -523,3 +523,57 @@ def test_emulated_doorbell_flow_control_one_grid(torch_cuda, monkeypatch):
         W.run()
         for m, (dst, exp, _) in enumerate(checks):
             assert np.array_equal(mp.as_tensor(dst, n).cpu().numpy(), exp), m
+
+
+def test_emulated_random_splits_misaligned_with_canaries(torch_cuda):
+    """Randomised multi-rank parity (seeded): 24 messages rank 0 -> rank 1 at world 4 with
+    random sizes (ragged), random shares over direct / relay 2 / relay 3 / host (any of
+    them possibly empty, shares not multiples of A), random chunk counts up to the slot
+    limit, and source and destination offsets 0-15 B (co-aligned or not: streamed and
+    per-chunk lanes); each payload equal to the oracle replay, 4 KiB canaries on both
+    sides of the destination untouched."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    rng = np.random.default_rng(20251018)
+    CAN = 4096
+    with world(4, slot_bytes=2 * MiB, heap_bytes=64 * MiB) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        ps = c0.paths(0, 1)
+        kinds = [k for k, _ in ps]
+        sbuf = torch.empty(26 * MiB, dtype=torch.uint8, device="cuda")
+        base = c1.alloc(26 * MiB + 2 * CAN + 64)
+        dview = mp.as_tensor(base, 26 * MiB + 2 * CAN + 64)
+        done = 0
+        for case in range(24):
+            n = int(rng.integers(1 * MiB, 24 * MiB))
+            nb = [0] * len(ps)
+            ks = [1] + [0] * (len(ps) - 1)
+            left = n
+            for i in range(1, len(ps)):
+                if rng.random() < 0.75 and left > 1024:
+                    b = int(rng.integers(300, max(301, min(left, 6 * MiB))))
+                    U = b // 256
+                    kmax = max(1, min(U, 12))
+                    k = int(rng.integers(1, kmax + 1))
+                    while 256 * ((U + k - 1) // k) + (b - 256 * U) > 2 * MiB:
+                        k += 1
+                    nb[i], ks[i] = b, k
+                    left -= b
+            nb[0] = left
+            so, do = int(rng.integers(0, 16)), int(rng.integers(0, 16))
+            host = synth.payload(n, 700 + case)
+            src = sbuf[so:so + n]
+            src.copy_(torch.from_numpy(host))
+            dview.fill_(0xA5)
+            dst = base + CAN + do
+            torch.cuda.synchronize()
+            c0.send(src, n, 1, tag=case, cfg=c0.make_config(nb, ks, 0, 1))
+            c1.recv(dst, n, 0, tag=case)
+            W.run()
+            got = dview.cpu().numpy()
+            exp = np.zeros(n, dtype=np.uint8)
+            X.replay(host, nb, ks, kinds, 256, exp)
+            assert np.array_equal(got[CAN + do:CAN + do + n], exp), (case, n, nb, ks, so, do)
+            assert (got[:CAN + do] == 0xA5).all() and (got[CAN + do + n:] == 0xA5).all(), ("canary", case)
+            done += 1
+        assert done == 24
