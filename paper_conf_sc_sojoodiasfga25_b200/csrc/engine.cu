@@ -913,7 +913,15 @@ __global__ void __launch_bounds__(kThreads, D == kBulkStages ? 3 : 2) xfer_kerne
 // Holds a stream for `ns` nanoseconds (calibration of the host submission time, C27).
 __global__ void spin_kernel(uint64_t ns) {
   const uint64_t t0 = globaltimer();
+#ifdef MPX_SPIN_SLEEP  // (design experiment: the sleeping spin of round 2's first sessions)
   while (globaltimer() - t0 < ns) __nanosleep(1000);
+#else
+  // busy: a sleeping warp leaves the GPU idle for the spin's ~1 ms, and the launch-bound
+  // small windows timed right after it then ran slower on some boxes (~1.5 µs per
+  // 64 KiB message against ~1.1 µs behind a busy spin)
+  while (globaltimer() - t0 < ns) {
+  }
+#endif
 }
 
 // Flag ping-pong between block 0 and block 1: ε probe (calibration, C12).
