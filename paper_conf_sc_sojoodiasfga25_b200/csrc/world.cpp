@@ -1027,6 +1027,15 @@ int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
       return wfail(c, MP_ERR_INVALID, "mp_emu_run: contexts must be the world's, in rank order");
   c = w->ctxs[0];
   CKW(cudaSetDevice(c->device));
+  // whatever happens below, the recorded work is consumed by this call
+  auto clear = [&] {
+    for (int r = 0; r < n; ++r) {
+      ctxs[r]->emu_send.clear();
+      ctxs[r]->emu_recv.clear();
+      ctxs[r]->emu_esend.clear();
+      ctxs[r]->emu_erecv.clear();
+    }
+  };
   std::vector<SendParams> send;
   std::vector<RecvParams> recv;
   std::vector<EagerParams> eager;
@@ -1043,12 +1052,7 @@ int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
     std::map<std::pair<uint32_t, uint32_t>, uint32_t> per_pair;
     for (const RecvParams &P : recv)
       if (++per_pair[{P.src, P.me}] > kCtsRing) {
-        for (int r = 0; r < n; ++r) {
-          ctxs[r]->emu_send.clear();
-          ctxs[r]->emu_recv.clear();
-          ctxs[r]->emu_esend.clear();
-          ctxs[r]->emu_erecv.clear();
-        }
+        clear();
         return wfail(c, MP_ERR_INVALID, "mp_emu_run: more than " + std::to_string(kCtsRing) +
                                             " rendezvous messages of one pair in one run");
       }
@@ -1063,8 +1067,10 @@ int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
     std::vector<std::pair<uint64_t, uint32_t>> &v = kv.second;
     std::sort(v.begin(), v.end());
     for (size_t j = 1; j < v.size(); ++j)
-      if (v[j].first != v[j - 1].first + 1 || v[j].second != v[0].second)
+      if (v[j].first != v[j - 1].first + 1 || v[j].second != v[0].second) {
+        clear();
         return wfail(c, MP_ERR_INVALID, "mp_emu_run: a relay's doorbells must be consecutive with equal lanes");
+      }
     mp_ctx *rc = w->ctxs[kv.first.first];
     const uint32_t snd = kv.first.second;
     RelayParams P{};
@@ -1095,14 +1101,6 @@ int emu_run(mp_ctx **ctxs, int n, void *stream, double *kernel_s) {
     mp_ctx *cr = ctxs[r];
     eager.insert(eager.end(), cr->emu_erecv.begin(), cr->emu_erecv.end());
   }
-  auto clear = [&] {
-    for (int r = 0; r < n; ++r) {
-      ctxs[r]->emu_send.clear();
-      ctxs[r]->emu_recv.clear();
-      ctxs[r]->emu_esend.clear();
-      ctxs[r]->emu_erecv.clear();
-    }
-  };
   // Grid: every role co-resident.  Only the direct groups are elastic (any CTA count
   // moves the same bytes): they share what the fixed roles leave, in proportion to
   // the CTA counts the real launches would have used.  Staged pipelines run at the
