@@ -182,7 +182,9 @@ int mp_init(mp_ctx **ctx, const mp_init_args *args);
 /* Destroy a context (the end of the Step 5 engine's lifetime): waits for
  * outstanding work on this device (cudaDeviceSynchronize), stops the relay service (waits for
  * the relay kernels it launched), unmaps and frees everything.  Collective when
- * world > 1.  ctx may be NULL.  Always returns MP_OK or the barrier's failure. */
+ * world > 1.  ctx may be NULL.  Returns MP_OK or the barrier's failure; MP_ERR_STATE
+ * (and does nothing) for a context of an emulated world: mp_finalize_emulated tears
+ * those down. */
 int mp_finalize(mp_ctx *ctx);
 
 /* ---------------------------------------------------------------- emulated world
