@@ -220,7 +220,9 @@ int mp_finalize(mp_ctx *ctx);
  * are shrunk (same bytes, fewer CTAs) so the grid fits the device's co-resident
  * capacity.  The recorded work must be one self-contained exchange: every recorded
  * send matched by a recorded receive, at most 64 rendezvous messages per ordered pair
- * (every receive posts its clear-to-send at once).  Errors: MP_ERR_INVALID (not the whole world /
+ * (every receive posts its clear-to-send at once; mp_recv refuses a 65th with
+ * MP_ERR_INVALID before recording it).  A refused run drops what was recorded and
+ * leaves the pairs' sequence state inconsistent: create a new world.  Errors: MP_ERR_INVALID (not the whole world /
  * the fixed roles alone exceed one co-resident grid / a relay's doorbells not
  * consecutive), MP_ERR_CUDA, MP_ERR_TIMEOUT and MP_ERR_MISMATCH (any rank's device
  * error word; sticky as in a real job).

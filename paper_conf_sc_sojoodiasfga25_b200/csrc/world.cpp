@@ -655,6 +655,13 @@ int world_recv(mp_ctx *c, void *buf, uint64_t bytes, int src, int tag, void *str
   if (region < 0)
     return wfail(c, MP_ERR_INVALID, "mp_recv buffer must come from mp_alloc or mp_register when world > 1");
   if (bytes > 0 && bytes <= c->eager_max) return eager_recv(c, buf, bytes, src, tag, stream);
+  if (c->emulated) {  // every recorded receive posts its clear-to-send at once (mp_emu_run)
+    uint32_t pending = 0;
+    for (const RecvParams &R : c->emu_recv) pending += R.src == static_cast<uint32_t>(src) ? 1u : 0u;
+    if (pending >= kCtsRing)
+      return wfail(c, MP_ERR_INVALID, "mp_recv: at most " + std::to_string(kCtsRing) +
+                                          " rendezvous messages of one pair per mp_emu_run");
+  }
   RecvParams P{};
   P.me = static_cast<uint32_t>(c->rank);
   P.src = static_cast<uint32_t>(src);

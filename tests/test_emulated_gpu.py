@@ -577,3 +577,27 @@ def test_emulated_random_splits_misaligned_with_canaries(torch_cuda):
             assert (got[:CAN + do] == 0xA5).all() and (got[CAN + do + n:] == 0xA5).all(), ("canary", case)
             done += 1
         assert done == 24
+
+
+def test_emulated_limits_refused(torch_cuda, monkeypatch):
+    """The emulated world's own rule fails loudly, before any state changes: a 65th
+    rendezvous receive of one pair recorded for the same run (every receive posts its
+    clear-to-send at once) is MP_ERR_INVALID, and the 64 recorded messages still go
+    through; mp_finalize on one of its contexts is MP_ERR_STATE."""
+    torch = torch_cuda
+    from paper_conf_sc_sojoodiasfga25_b200 import mp
+    monkeypatch.setenv("MPX_EAGER", "0")
+    with world(2, host_path=0) as W:
+        c0, c1 = W.ctx[0], W.ctx[1]
+        host, src = fill(torch, 8192, 1)
+        dst = c1.alloc(65 * 8192)
+        for m in range(64):
+            c1.recv(dst + m * 8192, 8192, 0, tag=m)
+            c0.send(src, 8192, 1, tag=m)
+        with pytest.raises(mp.MPError) as e:
+            c1.recv(dst + 64 * 8192, 8192, 0, tag=64)
+        assert e.value.status == mp.MP_ERR_INVALID
+        W.run()
+        got = mp.as_tensor(dst, 64 * 8192).cpu().numpy().reshape(64, 8192)
+        assert all(np.array_equal(g, host) for g in got)
+        assert mp.lib().mp_finalize(c0.h) == mp.MP_ERR_STATE
