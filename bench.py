@@ -922,7 +922,7 @@ def main():
     s_up, s_dn = torch.cuda.Stream(), torch.cuda.Stream()
     # enough steps that the pipeline's fill (the first H2D and the last D2H, which
     # overlap nothing) is a small part of the timed region
-    e2e_steps = max(3, min(24, args.steps // 4))
+    e2e_steps = max(3, min(48, args.steps // 4))
     torch.cuda.synchronize()
     ev = lambda: torch.cuda.Event()  # noqa: E731
     up_done, x_done, dn_done = [ev(), ev()], [ev(), ev()], [ev(), ev()]
