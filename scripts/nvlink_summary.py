@@ -26,7 +26,8 @@ def main():
     for p in sorted(glob.glob(os.path.join(d, "ncu_rank*.csv"))):
         rank = int(os.path.basename(p)[8:-4])
         for r in rows(p):
-            k = r["Kernel Name"].split("(")[0].split("::")[-1]
+            # "void mpx::<unnamed>::send_kernel<6>(mpx::SendParams)" -> "send_kernel"
+            k = r["Kernel Name"].split("(")[0].split("::")[-1].split("<")[0]
             try:
                 v = float(r["Metric Value"].replace(",", ""))
             except ValueError:
