@@ -527,6 +527,17 @@ def scenario_bench_plan(rank, world):
     assert w["paths"] == f"direct+{world - 2}relay+host" and w["selected"] == bench.split_label(d)
     assert w["parallelism"] == f"p2p-1pair+{world - 2}relays"
     c.close()
+    # one GPU per rank, checked across the ranks by GPU UUID: with fewer GPUs than ranks
+    # (none on the CPU box) every rank refuses, none proceeds alone
+    n_gpu = torch.cuda.device_count() if torch.cuda.is_available() else 0
+    if n_gpu >= world:
+        assert bench.rank_device(rank, world) == rank
+    else:
+        try:
+            bench.rank_device(rank, world)
+            raise AssertionError("rank_device accepted fewer GPUs than ranks")
+        except SystemExit as e:
+            assert "one GPU per rank" in str(e)
 
 
 def scenario_relay_burst(rank, world):
