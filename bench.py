@@ -442,8 +442,9 @@ def run_world_p2p(args, world, rank, local):
     except Exception as exc:
         base["nccl_error"] = repr(exc)
 
-    ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
-                                  timeout_s=60.0, param_file=args.params)
+    # Step 2: a parameter file of this topology replaces Step 1's calibration
+    ctx = mdist.context_from_dist(device=dev, calibrate=not (args.no_calibrate or args.params),
+                                  heap_bytes=n + 64 * MiB, timeout_s=60.0, param_file=args.params)
     if args.save_params and rank == 0:
         ctx.save_params(args.save_params)
     _, cfg = p2p_plan(ctx, world, n, args.mode)
@@ -673,8 +674,8 @@ def run_world_pairs(args, world, rank, local):
         except Exception as exc:
             base["nccl_error"] = repr(exc)
 
-    ctx = mdist.context_from_dist(device=dev, calibrate=not args.no_calibrate, heap_bytes=n + 64 * MiB,
-                                  timeout_s=60.0)
+    ctx = mdist.context_from_dist(device=dev, calibrate=not (args.no_calibrate or args.params),
+                                  heap_bytes=n + 64 * MiB, timeout_s=60.0, param_file=args.params)
     ctx.set_options(mode=mp.MP_MODEL_B200 if args.mode == "b200" else mp.MP_MODEL_PAPER)
     # the communication pattern is known ahead of time: select jointly for all
     # concurrent flows (NEXT f1, mp_select_flows) — every rank computes the same configs
