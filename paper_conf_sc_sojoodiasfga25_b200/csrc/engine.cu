@@ -1111,13 +1111,17 @@ struct RelayConsumer {
   // (GPU-scope acq_rel); the lane that completes the count releases the message's
   // relayed bytes into the destination's counter — one system-scope release per
   // relayed message, as the direct group's (§6).  Slot m % kBellRing is reused 64
-  // messages later; a relay's lanes drift at most a message or two apart (the sender's
-  // kernels on one relay ring run in order and wait for its free flags).
+  // messages later: a lane first waits until message m - 64 has been counted (rfree; a
+  // relay's lanes drift at most a message or two apart, so this never waits in
+  // practice: the sender's kernels on one relay ring run in order and wait for its
+  // free flags).
   __device__ void stored(uint32_t j, const uint64_t *w) {
     acc += w[2];
     if (j + 1 != k) return;
-    uint64_t *cnt = reinterpret_cast<uint64_t *>(P->my_ctrl + P->L.rcnt) +
-                    static_cast<uint64_t>(P->sender) * kBellRing + m % kBellRing;
+    const uint64_t slot = static_cast<uint64_t>(P->sender) * kBellRing + m % kBellRing;
+    uint64_t *cnt = reinterpret_cast<uint64_t *>(P->my_ctrl + P->L.rcnt) + slot;
+    uint64_t *fr = reinterpret_cast<uint64_t *>(P->my_ctrl + P->L.rfree) + slot;
+    if (m >= kBellRing && poll_flag_scoped(fr, m + 1 - kBellRing, P->timeout_ns, P->err, true) < 0) return;
     uint64_t old;
     asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], %2;"
                  : "=l"(old)
@@ -1127,6 +1131,7 @@ struct RelayConsumer {
       *reinterpret_cast<volatile uint64_t *>(cnt) = 0;
       const uint64_t total = (old >> 8) + acc;
       if (total) red_add_release_sys(done_at(P->peer[w[0]].ctrl, P->L, P->sender), total);
+      st_release_gpu(fr, m + 1);
     }
   }
 };
@@ -1518,6 +1523,20 @@ __device__ bool relay_message(const RelayParams &P, const uint32_t r, uint64_t m
     uint64_t *fr = flags_at(P.sender_ctrl, P.L.relay_free, P.me, P.L.slots, s) + r;
     publish(done_at(P.peer[dst].ctrl, P.L, P.sender), len, fr, u + 1);
     __syncthreads();
+  }
+  // the per-chunk path counted its bytes chunk by chunk; the message still takes its
+  // turn in the lanes' counter slot so that the streamed messages after it see it done
+  if (threadIdx.x == 0) {
+    const uint64_t slot = static_cast<uint64_t>(P.sender) * kBellRing + m % kBellRing;
+    uint64_t *cnt = reinterpret_cast<uint64_t *>(P.my_ctrl + P.L.rcnt) + slot;
+    uint64_t *rf = reinterpret_cast<uint64_t *>(P.my_ctrl + P.L.rfree) + slot;
+    if (m >= kBellRing && poll_flag_scoped(rf, m + 1 - kBellRing, P.timeout_ns, P.err, true) < 0) return false;
+    uint64_t old;
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(cnt) : "memory");
+    if ((old & 0xffu) + 1 == P.g) {
+      *reinterpret_cast<volatile uint64_t *>(cnt) = 0;
+      st_release_gpu(rf, m + 1);
+    }
   }
   return true;
 }

@@ -194,6 +194,7 @@ struct CtrlLayout {
   uint64_t dfree = 0;                  // [world(dst)][kCtsRing] u64: last message whose direct CTAs were counted + 1
   uint64_t rcnt = 0;                   // [world(sender)][kBellRing] u64: relay lanes of message m done
                                        //   (bytes << 8 | lanes) — on the relay
+  uint64_t rfree = 0;                  // [world(sender)][kBellRing] u64: last relayed message counted + 1
   uint64_t total = 0;
 };
 

@@ -105,6 +105,7 @@ CtrlLayout layout(uint32_t world, uint32_t slots, uint64_t slot_bytes) {
   L.dcnt = take(static_cast<uint64_t>(world) * kCtsRing * 8);
   L.dfree = take(static_cast<uint64_t>(world) * kCtsRing * 8);
   L.rcnt = take(static_cast<uint64_t>(world) * kBellRing * 8);
+  L.rfree = take(static_cast<uint64_t>(world) * kBellRing * 8);
   L.ring_data = take(world >= 3 ? static_cast<uint64_t>(world) * slots * L.stride : 0);
   L.total = off;
   return L;
